@@ -1,0 +1,187 @@
+/*
+ * pagoda.h — C ABI of the B200-native Pagoda runtime (host side).
+ *
+ * Pagoda (Yeh, Sabne, Sakdhnagool, Eigenmann, Rogers; PPoPP'17; cited P:<line> of
+ * /root/reference/PAPER.md) virtualises GPU SMs for narrow tasks (< 500 threads,
+ * P:18-20): a persistent MasterKernel pulls tasks that CPU
+ * threads spawn into a TaskTable, allocates executor warps, shared
+ * memory and named barriers to them at warp granularity (Alg. 1/2 P:738-880,
+ * §5), runs their bodies and signals completion.
+ *
+ * Calls follow Table 1: taskSpawn / wait / check / waitAll on the
+ * host.  The bare paper names would collide with POSIX wait(2), so the C ABI
+ * prefixes them with `pagoda_`.
+ *
+ * Conventions for every function below
+ *   - thread-safe: any number of host threads may spawn / wait concurrently;
+ *   - errors are negative errno values, never exceptions; 0 (or a valid id) on success;
+ *   - pointers named `args` are HOST pointers, copied before the call returns;
+ *     device pointers carried INSIDE args are caller-owned and must stay valid
+ *     until wait/check reports the task done;
+ *   - the context owns every pinned-host and device buffer it allocated.
+ */
+#ifndef PAGODA_H
+#define PAGODA_H
+#include <stddef.h>
+#include <stdint.h>
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct pagoda_ctx pagoda_ctx;   /* opaque: rings, MasterKernel stream, counters */
+typedef int64_t pagoda_task_t;          /* >= 0: task id; < 0: -errno */
+
+/* ---- limits fixed by the design ---------------- */
+#define PAGODA_ARGS_MAX      40   /* bytes of inline task arguments per TaskTable entry */
+#define PAGODA_GRANULE       512  /* shared-memory allocation granule */
+#define PAGODA_MAX_EXEC_WARPS 31  /* executor warps per MTB: warp 0 schedules */
+#define PAGODA_BAR_IDS       15   /* named barriers 1..15 per MTB; 0 is the MTB's own */
+
+/* config flags */
+#define PAGODA_TRACE         0x1u /* record the per-MTB scheduler ledger (tests; slows scheduling) */
+
+typedef struct {
+    int      device;        /* CUDA device ordinal (default 0) */
+    int      mtbs_per_sm;   /* MasterKernel thread blocks (MTBs) per SM: 1 or 2 (default 2) */
+    int      num_sms;       /* SMs to occupy, 0 = all (148 on B200) */
+    uint32_t ring_entries;  /* TaskTable ring entries, host and device, power of 2 (default 65536) */
+    uint32_t comp_entries;  /* completion window, power of 2 >= ring_entries (default 1<<20) */
+    uint32_t arena_bytes;   /* shared-memory arena per MTB, multiple of 512 (default 96 KiB at 2 MTB/SM) */
+    uint32_t exec_warps;    /* executor warps per MTB, 1..31 (default 31; fewer = debug config) */
+    uint32_t flags;         /* PAGODA_TRACE */
+    uint32_t trace_events;  /* ledger capacity per MTB when PAGODA_TRACE (default 8192) */
+    double   watchdog_s;    /* wait/waitAll/shutdown give up with -ETIMEDOUT after this many
+                               seconds without progress (default 60; <= 0 disables) */
+} pagoda_config;
+
+/* Fill *cfg with the defaults above. */
+void pagoda_config_default(pagoda_config* cfg);
+
+/* Start Pagoda on cfg->device: allocate the pinned TaskTable ring, doorbell and
+ * completion window, the device ring, and launch the persistent MasterKernel
+ * (cooperative launch: all MTBs co-resident).  cfg NULL = defaults.
+ * While the MasterKernel runs it holds every warp of the SMs it occupies, so
+ * other kernels on that device wait until pagoda_shutdown (copies still run).
+ * Returns 0 and *out, or -ENODEV (no such device / not sm_100), -ENOMEM, -EINVAL
+ * (bad config), -EIO (launch failed). */
+int pagoda_init(const pagoda_config* cfg, pagoda_ctx** out);
+
+/* waitAll, then stop the MasterKernel, free everything and *out is invalid.
+ * Returns 0, -EIO (device fault seen), -ETIMEDOUT (watchdog; resources leaked). */
+int pagoda_shutdown(pagoda_ctx* ctx);
+
+/* taskSpawn (Table 1, §3): spawn one task of n_threadblocks
+ * thread blocks of `threads` threads (rounded up to whole warps), each block
+ * with `shmem_bytes` of shared memory (getSMPtr) and, if sync_flag, a named
+ * barrier (syncBlock).  func_id selects a compiled-in task body
+ * (pagoda_tasks.h); args/args_bytes (<= 40) are copied into the entry.
+ * Non-blocking: returns once the entry is published (it blocks, with back-off,
+ * only while the TaskTable ring or completion window is full, as the paper's
+ * CPU does when no entry is free).
+ * Returns the task id (>= 0, strictly increasing per context) or
+ *   -EINVAL  threads < 1, n_threadblocks < 1, ceil(threads/32)*n_tb > executor
+ *            warps per MTB (all warps of a task live in one MTB),
+ *            n_tb * round_up(shmem, 512) > arena, sync with > 15 multi-warp TBs,
+ *            unknown func_id, args_bytes > 40 or args NULL with args_bytes > 0;
+ *   -ESHUTDOWN after pagoda_shutdown began;  -EIO after a device fault. */
+pagoda_task_t pagoda_taskSpawn(pagoda_ctx* ctx, int threads, int n_threadblocks, int shmem_bytes,
+                               int sync_flag, int func_id, const void* args, size_t args_bytes);
+
+/* wait (Table 1): block until task `id` is done.  After it returns 0
+ * the task's device writes are visible to later host copies and to every task
+ * spawned afterwards.  Returns 0, -EINVAL (id never issued), -EIO, -ETIMEDOUT. */
+int pagoda_wait(pagoda_ctx* ctx, pagoda_task_t id);
+
+/* check (Table 1): non-blocking; 1 if done, 0 if pending, < 0 error. */
+int pagoda_check(pagoda_ctx* ctx, pagoda_task_t id);
+
+/* waitAll (Table 1): block until every task whose id was issued before
+ * the call is done.  Returns 0, -EIO, -ETIMEDOUT. */
+int pagoda_waitAll(pagoda_ctx* ctx);
+
+/* Convenience for C and Python callers: spawn n tasks of one shape, task i's
+ * args at args_base + i*args_stride (args_bytes each); each is a separate
+ * pagoda_taskSpawn.  ids_out (nullable) receives the ids.  Returns the number
+ * spawned (n) or the first error (tasks before it stay spawned). */
+int64_t pagoda_taskSpawnMany(pagoda_ctx* ctx, int n, int threads, int n_threadblocks, int shmem_bytes,
+                             int sync_flag, int func_id, const void* args_base, size_t args_stride,
+                             size_t args_bytes, pagoda_task_t* ids_out);
+
+/* Same with a per-task shape: shapes[i] = {threads, n_threadblocks, shmem_bytes,
+ * sync_flag, func_id} (5 int32 per task). */
+int64_t pagoda_taskSpawnShapes(pagoda_ctx* ctx, int n, const int32_t* shapes, const void* args_base,
+                               size_t args_stride, size_t args_bytes, pagoda_task_t* ids_out);
+
+/* Runtime facts and counters. */
+typedef struct {
+    int      device, sm_count, n_mtb, mtbs_per_sm, exec_warps, arena_bytes, regs_per_thread;
+    uint32_t ring_entries, comp_entries;
+    int64_t  spawned;       /* ids issued */
+    int64_t  completed_low; /* every id below this is known done */
+    uint32_t device_error;  /* 0 or a PAGODA_DEVERR_* code */
+    int      running;       /* MasterKernel still resident */
+} pagoda_info;
+int pagoda_get_info(pagoda_ctx* ctx, pagoda_info* out);
+
+#define PAGODA_DEVERR_SYNC_WITHOUT_FLAG 1u  /* syncBlock() in a multi-warp TB spawned with sync=0 */
+#define PAGODA_DEVERR_BAD_FUNC          2u  /* entry with unknown func_id reached an executor */
+
+/* Ledger (PAGODA_TRACE): copy up to cap 32-byte events of MTB `mtb` into dst
+ * (host memory), after pagoda_shutdown's drain or while idle.  Layout: see
+ * DESIGN.md "Trace ledger".  Returns the number of events recorded (may be > cap
+ * if the buffer overflowed: then only cap were kept) or -EINVAL. */
+int64_t pagoda_trace_read(pagoda_ctx* ctx, int mtb, void* dst, size_t cap);
+
+/* Executor intervals (PAGODA_TRACE): per executor warp a list of
+ * {u64 task_id; u32 tb; u16 mtb; u16 warp; u64 t_start_ns; u64 t_end_ns} (32 B).
+ * Copies up to cap records of (mtb, warp) into dst; returns the count. */
+int64_t pagoda_trace_read_exec(pagoda_ctx* ctx, int mtb, int warp, void* dst, size_t cap);
+
+/* Host-side preparation of the 3DES task's device tables:
+ * writes PAGODA_TDES_TABLE_BYTES bytes to dst (HOST memory) for the EDE3 key
+ * K1|K2|K3 (24 bytes, FIPS 46-3 byte order).  Copy them to device memory and
+ * pass the device pointer in pagoda_tdes_args.tables.  Returns 0. */
+#define PAGODA_TDES_TABLE_BYTES (2048 + 384 + 16384 + 16384)
+int pagoda_tdes_tables(const uint8_t key24[24], void* dst);
+
+/* Naive baseline (the paper's CUDA-HyperQ): launch
+ * each task as its own kernel <<<n_tb, threads, shmem>>> of the same body on
+ * streams[i % n_streams] (n_streams <= 32), from the calling thread, then
+ * synchronise.  shapes/args as in pagoda_taskSpawnShapes (args are the same
+ * device-pointer blocks).  Returns 0 or -EIO.  If elapsed_ns is non-NULL it
+ * receives first-launch -> all-done host time. */
+int pagoda_naive_run(int device, int n, const int32_t* shapes, const void* args_base, size_t args_stride,
+                     size_t args_bytes, int n_streams, int64_t* elapsed_ns);
+
+/* ---- multi-GPU pool: one context per GPU, least-loaded picker */
+typedef struct pagoda_pool pagoda_pool;
+/* Start one context per device in devices[0..n_dev) with cfg (device field ignored). */
+int pagoda_pool_init(int n_dev, const int* devices, const pagoda_config* cfg, pagoda_pool** out);
+/* Index of the device with the fewest in-flight warps (spawned, not yet seen
+ * completed); ties go to the lowest index.  warps_hint is added to the chosen
+ * device's in-flight count (the caller then spawns there). */
+int pagoda_pool_pick(pagoda_pool* pool, int warps_hint);
+pagoda_ctx* pagoda_pool_ctx(pagoda_pool* pool, int index);
+int pagoda_pool_size(pagoda_pool* pool);
+/* Spawn on the least-loaded context; *index_out (nullable) gets the chosen index.
+ * args_per_dev[i] (args_bytes each) are the args to use if device i is chosen. */
+pagoda_task_t pagoda_pool_spawn(pagoda_pool* pool, int threads, int n_threadblocks, int shmem_bytes,
+                                int sync_flag, int func_id, const void* const* args_per_dev,
+                                size_t args_bytes, int* index_out);
+int pagoda_pool_waitAll(pagoda_pool* pool);
+int pagoda_pool_shutdown(pagoda_pool* pool);
+
+/* In-flight warps of one context: warps of spawned tasks minus those of the
+ * tasks below its completion watermark (the pool's load measure). */
+int64_t pagoda_inflight_warps(pagoda_ctx* ctx);
+/* The picker rule alone (host-only, testable without a GPU): index of the
+ * smallest of loads[0..n), ties to the lowest index; -EINVAL if n < 1. */
+int pagoda_pick_least_loaded(const int64_t* loads, int n);
+
+/* Library version string. */
+const char* pagoda_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

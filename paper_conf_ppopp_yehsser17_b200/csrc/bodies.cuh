@@ -1,0 +1,399 @@
+/*
+ * bodies.cuh — the task bodies, written once as __device__ subroutines over an
+ * Env (pagoda_device.cuh) and instantiated twice: inside the MasterKernel
+ * (TaskEnv) and as the naive one-launch-per-task baseline (NativeEnv).
+ *
+ * What each body computes is DESIGN.md "Task bodies" (the paper gives the
+ * benchmark names and sizes only: Tables 3-4).  fp32 bodies use
+ * explicitly rounded intrinsics (__fmul_rn / __fadd_rn / __fmaf_rn) so that
+ * nvcc cannot contract or reorder: the operation order is the definition's.
+ *
+ * Work partition: thread getTid() of a task with T = n_tb * warps_tb * 32
+ * threads (idle padding lanes included) takes output items getTid(), +T, ...
+ * Bodies with two dependent passes (FB, CONV) keep each thread block
+ * self-contained: a TB computes the intermediate values its own outputs need,
+ * into its own shared memory or scratch region, and only syncBlock()s itself.
+ */
+#ifndef PAGODA_BODIES_CUH
+#define PAGODA_BODIES_CUH
+#include <stdint.h>
+
+#include "pagoda_device.cuh"
+#include "pagoda_tasks.h"
+
+namespace pagoda {
+
+template <class Env>
+__device__ __forceinline__ int total_threads(const Env& e)
+{
+    return e.getNumBlocks() * e.getBlockWarps() * 32;
+}
+template <class Env>
+__device__ __forceinline__ int tb_threads(const Env& e)
+{
+    return e.getBlockWarps() * 32;
+}
+
+/* ------------------------------------------------------------- test bodies */
+template <class Env>
+__device__ void body_mark(const Env& e, const pagoda_mark_args& a)
+{
+    if (e.getBlockTid() < e.getBlockDim()) {
+        a.out[a.base + (uint32_t)e.getTid()] = a.tag;
+        atomicAdd(a.cnt, 1u);
+    }
+}
+
+template <class Env>
+__device__ void body_tid(const Env& e, const pagoda_tid_args& a)
+{
+    if (e.getBlockTid() < e.getBlockDim())
+        a.out[a.base + (uint32_t)e.getTid()] = ((uint32_t)e.getBlockIdx() << 16) | (uint32_t)e.getBlockTid();
+}
+
+/* P phases of: write my word, syncBlock, read the word of the thread 32 lanes
+ * further on (another warp of the same TB), syncBlock.  Scratch: shared memory
+ * if granted, else args.scratch[tb * threads_tb_rounded + ...]. */
+template <class Env>
+__device__ void body_bar(const Env& e, const pagoda_bar_args& a)
+{
+    const int n = tb_threads(e), bt = e.getBlockTid();
+    volatile uint32_t* buf = (e.getSMBytes() >= (uint32_t)n * 4u)
+                                 ? reinterpret_cast<volatile uint32_t*>(e.getSMPtr())
+                                 : reinterpret_cast<volatile uint32_t*>(a.scratch) + e.getBlockIdx() * n;
+    uint32_t errs = 0;
+    for (uint32_t p = 0; p < a.phases; p++) {
+        buf[bt] = p * 1000003u + (uint32_t)bt;
+        e.syncBlock();
+        int nb = (bt + 32) % n;
+        if (buf[nb] != p * 1000003u + (uint32_t)nb) errs++;
+        e.syncBlock();
+    }
+    if (errs) atomicAdd(a.err, errs);
+}
+
+/* Fill the TB's shared memory, hold it, then verify nobody else wrote it. */
+template <class Env>
+__device__ void body_smem(const Env& e, const pagoda_smem_args& a)
+{
+    uint32_t* p = reinterpret_cast<uint32_t*>(e.getSMPtr());
+    const uint32_t words = min(a.bytes, e.getSMBytes()) / 4u;
+    const uint32_t key = a.seed * 2654435761u + (uint32_t)e.getBlockIdx() * 40503u;
+    const int n = tb_threads(e);
+    uint32_t errs = 0;
+    if (e.getBlockTid() == 0 && ((uintptr_t)p & 31u) != 0) errs++;   /* getSMPtr is 32-byte aligned */
+    for (uint32_t i = e.getBlockTid(); i < words; i += n) p[i] = key ^ (i * 0x9E3779B9u);
+    if (a.spin_ns) {
+        uint64_t t0 = globaltimer_ns();
+        while (globaltimer_ns() - t0 < a.spin_ns) { }
+    }
+    e.syncBlock();
+    for (uint32_t i = e.getBlockTid(); i < words; i += n) errs += (p[i] != (key ^ (i * 0x9E3779B9u)));
+    if (errs) atomicAdd(a.err, errs);
+}
+
+template <class Env>
+__device__ void body_spin(const Env&, const pagoda_spin_args& a)
+{
+    uint64_t t0 = globaltimer_ns();
+    while (globaltimer_ns() - t0 < a.ns) { }
+}
+
+template <class Env>
+__device__ void body_gate(const Env&, const pagoda_gate_args& a)
+{
+    if (lane_id() == 0) {
+        while (*a.flag == 0) __nanosleep(1000);
+    }
+    __syncwarp();
+}
+
+/* ------------------------------------------------------------- MB
+ * Table 3; strict '>' escape test, count includes
+ * the escaping step, multiply-then-add never fused. */
+template <class Env>
+__device__ void body_mb(const Env& e, const pagoda_mb_args& a)
+{
+    const int T = total_threads(e);
+    for (int p = e.getTid(); p < 4096; p += T) {
+        const int gx = 64 * a.tx + (p & 63), gy = 64 * a.ty + (p >> 6);
+        const float cr = __fadd_rn(a.x0, __fmul_rn((float)gx, a.dx));
+        const float ci = __fadd_rn(a.y0, __fmul_rn((float)gy, a.dx));
+        float zr = 0.0f, zi = 0.0f;
+        int n = 0;
+        while (n < a.maxit) {
+            const float zr2 = __fmul_rn(zr, zr);
+            const float zi2 = __fmul_rn(zi, zi);
+            if (__fadd_rn(zr2, zi2) > 4.0f) break;
+            const float t = __fadd_rn(zr, zr);
+            zi = __fadd_rn(__fmul_rn(t, zi), ci);
+            zr = __fadd_rn(__fsub_rn(zr2, zi2), cr);
+            n++;
+        }
+        a.out[p] = (uint16_t)n;
+    }
+}
+
+/* ------------------------------------------------------------- 3DES
+ * TDEA EDE3, ECB (NIST [5]).  tables =
+ * pagoda_tdes_tables(): SP[8][64] u32 (S-box j then P, for the 6-bit input of
+ * box j), 48 round keys as 8 six-bit chunks each (execution order
+ * K1[0..15], K2[15..0], K3[0..15]), IP and FP byte tables [8][256] u64.
+ * Since FP then IP cancel between the three DES stages, a block is
+ * IP, 48 rounds with a half-swap after every 16, FP. */
+constexpr uint32_t kTdesStageBytes = 2048 + 384;
+constexpr uint32_t kTdesIpOff = 2432, kTdesFpOff = 2432 + 16384;
+
+__device__ __forceinline__ uint64_t tdes_perm(const uint64_t* tab, uint64_t x)
+{
+    uint64_t r = 0;
+#pragma unroll
+    for (int b = 0; b < 8; b++) r |= __ldg(&tab[b * 256 + (int)((x >> (56 - 8 * b)) & 0xFF)]);
+    return r;
+}
+
+template <class Env>
+__device__ void body_tdes(const Env& e, const pagoda_tdes_args& a)
+{
+    const uint32_t* sp = a.tables;
+    const uint8_t* keys = reinterpret_cast<const uint8_t*>(a.tables + 512);
+    if (e.getSMBytes() >= kTdesStageBytes && e.canSync()) {   /* stage SP boxes + round keys into the TB's shmem */
+        uint32_t* s = reinterpret_cast<uint32_t*>(e.getSMPtr());
+        if (e.getBlockTid() < 32) e.stage(s, a.tables, kTdesStageBytes);
+        e.syncBlock();
+        sp = s;
+        keys = reinterpret_cast<const uint8_t*>(s + 512);
+    }
+    const uint64_t* ipt = reinterpret_cast<const uint64_t*>(reinterpret_cast<const char*>(a.tables) + kTdesIpOff);
+    const uint64_t* fpt = reinterpret_cast<const uint64_t*>(reinterpret_cast<const char*>(a.tables) + kTdesFpOff);
+    const int T = total_threads(e);
+    for (uint32_t blk = (uint32_t)e.getTid(); blk < a.nblk; blk += (uint32_t)T) {
+        uint64_t x = a.in[blk];
+        /* bytes are the block in FIPS (big-endian) order */
+        x = ((uint64_t)__byte_perm((uint32_t)x, 0, 0x0123) << 32) | __byte_perm((uint32_t)(x >> 32), 0, 0x0123);
+        x = tdes_perm(ipt, x);
+        uint32_t l = (uint32_t)(x >> 32), r = (uint32_t)x;
+#pragma unroll 1
+        for (int st = 0; st < 3; st++) {
+#pragma unroll 2
+            for (int rd = 0; rd < 16; rd++) {
+                const uint32_t* kr = reinterpret_cast<const uint32_t*>(keys + (st * 16 + rd) * 8);
+                const uint32_t k0 = kr[0], k1 = kr[1];
+                uint32_t f = 0;
+#pragma unroll
+                for (int j = 0; j < 8; j++) {
+                    const uint32_t kj = ((j < 4 ? k0 : k1) >> (8 * (j & 3))) & 63u;
+                    const uint32_t six = (__funnelshift_l(r, r, 4 * j + 5) & 63u) ^ kj;
+                    f |= sp[j * 64 + six];
+                }
+                const uint32_t t = l ^ f;
+                l = r;
+                r = t;
+            }
+            const uint32_t t = l;   /* undo the last half-swap: stage output (R16, L16) */
+            l = r;
+            r = t;
+        }
+        x = tdes_perm(fpt, ((uint64_t)l << 32) | r);
+        x = ((uint64_t)__byte_perm((uint32_t)x, 0, 0x0123) << 32) | __byte_perm((uint32_t)(x >> 32), 0, 0x0123);
+        a.out[blk] = x;
+    }
+}
+
+/* ------------------------------------------------------------- MM
+ * CUDA SDK MatrixMul [22] (Table 3); 32x32x32 fp32; C[i][j] is the
+ * fma chain over k ascending from 0.  A and B are staged into the TB's shmem
+ * with TMA bulk copies when 8 KiB were granted and the TB can synchronise. */
+template <class Env>
+__device__ void body_mm(const Env& e, const pagoda_mm_args& a)
+{
+    const float* A = a.A;
+    const float* B = a.B;
+    if (e.getSMBytes() >= 8192 && e.canSync()) {
+        float* s = reinterpret_cast<float*>(e.getSMPtr());
+        const int w = e.getBlockTid() >> 5;
+        if (e.getBlockWarps() >= 2) {
+            if (w == 0) e.stage(s, A, 4096);
+            else if (w == 1) e.stage(s + 1024, B, 4096);
+        } else {
+            e.stage(s, A, 4096);
+            e.stage(s + 1024, B, 4096);
+        }
+        e.syncBlock();
+        A = s;
+        B = s + 1024;
+    }
+    const int T = total_threads(e);
+    for (int idx = e.getTid(); idx < 1024; idx += T) {
+        const int i = idx >> 5, j = idx & 31;
+        float acc = 0.0f;
+#pragma unroll 8
+        for (int k = 0; k < 32; k++) acc = __fmaf_rn(A[i * 32 + k], B[k * 32 + j], acc);
+        a.C[idx] = acc;
+    }
+}
+
+/* ------------------------------------------------------------- FB
+ * Fig. 1c: VH = H (*) r, VD[m] = VH[8m],
+ * VU = up-sample of VD, y = F (*) VU; causal, fma chains k ascending.
+ * Only VH[8m] is ever used, and the zero terms of VU add exactly +0, so
+ * y[j] = sum over k = j mod 8, j mod 8 + 8, ... <= min(31, j) of F[k] VD[(j-k)/8]. */
+template <class Env>
+__device__ void body_fb(const Env& e, const pagoda_fb_args& a)
+{
+    float* vd = (e.getSMBytes() >= 1024) ? reinterpret_cast<float*>(e.getSMPtr())
+                                         : a.scratch + 256 * e.getBlockIdx();
+    const int n = tb_threads(e), bt = e.getBlockTid();
+    for (int m = bt; m < 256; m += n) {
+        float acc = 0.0f;
+        const int kmax = min(31, 8 * m);
+        for (int k = 0; k <= kmax; k++) acc = __fmaf_rn(a.H[k], a.r[8 * m - k], acc);
+        vd[m] = acc;
+    }
+    e.syncBlock();
+    const int T = total_threads(e);
+    for (int j = e.getTid(); j < 2048; j += T) {
+        float acc = 0.0f;
+        const int kmax = min(31, j);
+        for (int k = j & 7; k <= kmax; k += 8) acc = __fmaf_rn(a.F[k], vd[(j - k) >> 3], acc);
+        a.y[j] = acc;
+    }
+}
+
+/* ------------------------------------------------------------- BF
+ * Table 3: v[c][t] = sum_k h[c][k] x[c][t-k]
+ * (16 taps), y[b][t] = sum_c w[b][c] v[c][t], out = |y|^2.  No barrier:
+ * each thread computes the v values its own t needs. */
+__device__ __forceinline__ void cmac(float& re, float& im, float ar, float ai, float br, float bi)
+{
+    re = __fmaf_rn(ar, br, re);
+    re = __fmaf_rn(-ai, bi, re);
+    im = __fmaf_rn(ar, bi, im);
+    im = __fmaf_rn(ai, br, im);
+}
+
+template <class Env>
+__device__ void body_bf(const Env& e, const pagoda_bf_args& a)
+{
+    const int T = total_threads(e);
+    const float2* x = reinterpret_cast<const float2*>(a.x);
+    const float2* h = reinterpret_cast<const float2*>(a.h);
+    const float2* w = reinterpret_cast<const float2*>(a.w);
+    for (int t = e.getTid(); t < 512; t += T) {
+        float vr[4], vi[4];
+#pragma unroll
+        for (int c = 0; c < 4; c++) {
+            float re = 0.0f, im = 0.0f;
+            const int kmax = min(15, t);
+            for (int k = 0; k <= kmax; k++) {
+                const float2 hk = h[c * 16 + k], xv = x[c * 512 + t - k];
+                cmac(re, im, hk.x, hk.y, xv.x, xv.y);
+            }
+            vr[c] = re;
+            vi[c] = im;
+        }
+#pragma unroll
+        for (int b = 0; b < 4; b++) {
+            float re = 0.0f, im = 0.0f;
+#pragma unroll
+            for (int c = 0; c < 4; c++) {
+                const float2 wb = w[b * 4 + c];
+                cmac(re, im, wb.x, wb.y, vr[c], vi[c]);
+            }
+            a.out[b * 512 + t] = __fmaf_rn(re, re, __fmul_rn(im, im));
+        }
+    }
+}
+
+/* ------------------------------------------------------------- CONV
+ * CUDA SDK convolutionSeparable [19], DESIGN.md "CONV":
+ * tmp[y][x] = sum_{d=-8..8} img[y][x+d] krow[8-d], out[y][x] = sum_d
+ * tmp[y+d][x] kcol[8-d], zero outside, d ascending.  TB j produces output rows
+ * [r0, r1) and first computes the tmp rows [r0-8, r1+8) they need into
+ * scratch + 16384*j (same row indexing as the full image). */
+template <class Env>
+__device__ void body_conv(const Env& e, const pagoda_conv_args& a)
+{
+    const int nb = e.getNumBlocks(), j = e.getBlockIdx();
+    const int r0 = (128 * j) / nb, r1 = (128 * (j + 1)) / nb;
+    const int t0 = max(0, r0 - 8), t1 = min(128, r1 + 8);
+    float* tmp = a.scratch + 16384 * j;
+    const int n = tb_threads(e), bt = e.getBlockTid();
+    for (int idx = t0 * 128 + bt; idx < t1 * 128; idx += n) {
+        const int y = idx >> 7, x = idx & 127;
+        float acc = 0.0f;
+        for (int d = -8; d <= 8; d++)
+            if (x + d >= 0 && x + d < 128) acc = __fmaf_rn(a.img[y * 128 + x + d], a.krow[8 - d], acc);
+        tmp[idx] = acc;
+    }
+    e.syncBlock();
+    for (int idx = r0 * 128 + bt; idx < r1 * 128; idx += n) {
+        const int y = idx >> 7, x = idx & 127;
+        float acc = 0.0f;
+        for (int d = -8; d <= 8; d++)
+            if (y + d >= 0 && y + d < 128) acc = __fmaf_rn(tmp[(y + d) * 128 + x], a.kcol[8 - d], acc);
+        a.out[idx] = acc;
+    }
+}
+
+/* ------------------------------------------------------------- DCT
+ * CUDA SDK DCT8x8 [21]: per 8x8 block
+ * T[u][y] = sum_x C[u][x] X[x][y], Y[u][v] = sum_y T[u][y] C[v][y].
+ * Work item (block, u): one thread computes T[u][*] and Y[u][*]. */
+template <class Env>
+__device__ void body_dct(const Env& e, const pagoda_dct_args& a)
+{
+    const int T = total_threads(e);
+    for (int item = e.getTid(); item < 256 * 8; item += T) {
+        const int blk = item >> 3, u = item & 7;
+        const int by = blk >> 4, bx = blk & 15;
+        const float* X = a.img + (by * 8) * 128 + bx * 8;
+        float Tu[8];
+#pragma unroll
+        for (int y = 0; y < 8; y++) {
+            float acc = 0.0f;
+#pragma unroll
+            for (int x = 0; x < 8; x++) acc = __fmaf_rn(a.coef[u * 8 + x], X[x * 128 + y], acc);
+            Tu[y] = acc;
+        }
+        float* Y = a.out + (by * 8 + u) * 128 + bx * 8;
+#pragma unroll
+        for (int v = 0; v < 8; v++) {
+            float acc = 0.0f;
+#pragma unroll
+            for (int y = 0; y < 8; y++) acc = __fmaf_rn(Tu[y], a.coef[v * 8 + y], acc);
+            Y[v] = acc;
+        }
+    }
+}
+
+/* ------------------------------------------------------------- dispatch */
+template <class Env>
+__device__ __forceinline__ bool run_body(int func_id, const Env& e, const void* args)
+{
+    switch (func_id) {
+    case PAGODA_NOP: return true;
+    case PAGODA_MARK: body_mark(e, *static_cast<const pagoda_mark_args*>(args)); return true;
+    case PAGODA_TID: body_tid(e, *static_cast<const pagoda_tid_args*>(args)); return true;
+    case PAGODA_BAR: body_bar(e, *static_cast<const pagoda_bar_args*>(args)); return true;
+    case PAGODA_SMEM: body_smem(e, *static_cast<const pagoda_smem_args*>(args)); return true;
+    case PAGODA_SPIN: body_spin(e, *static_cast<const pagoda_spin_args*>(args)); return true;
+    case PAGODA_GATE: body_gate(e, *static_cast<const pagoda_gate_args*>(args)); return true;
+    case PAGODA_MB: body_mb(e, *static_cast<const pagoda_mb_args*>(args)); return true;
+    case PAGODA_TDES: body_tdes(e, *static_cast<const pagoda_tdes_args*>(args)); return true;
+    case PAGODA_MM: body_mm(e, *static_cast<const pagoda_mm_args*>(args)); return true;
+    case PAGODA_FB: body_fb(e, *static_cast<const pagoda_fb_args*>(args)); return true;
+    case PAGODA_BF: body_bf(e, *static_cast<const pagoda_bf_args*>(args)); return true;
+    case PAGODA_CONV: body_conv(e, *static_cast<const pagoda_conv_args*>(args)); return true;
+    case PAGODA_DCT: body_dct(e, *static_cast<const pagoda_dct_args*>(args)); return true;
+    default: return false;
+    }
+}
+
+__host__ __device__ inline bool known_func(int f)
+{
+    return (f >= PAGODA_NOP && f <= PAGODA_GATE) || (f >= PAGODA_MB && f <= PAGODA_DCT);
+}
+
+} // namespace pagoda
+#endif

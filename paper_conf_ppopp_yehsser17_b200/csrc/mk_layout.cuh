@@ -1,0 +1,122 @@
+/*
+ * mk_layout.cuh — data layout shared by the host runtime (runtime.cu) and the
+ * MasterKernel (master_kernel.cu).  DESIGN.md "Data layout" draws it.
+ *
+ * TaskTable entry (#TBs, #threads/TB, kernel, shmem/TB, sync flag,
+ * inputs, ready, sched).  The ready/sched handshake is replaced by
+ * doorbell ordering: an entry is visible to the GPU iff its index < the
+ * published count, and its completion lives in the completion window.
+ */
+#ifndef PAGODA_MK_LAYOUT_CUH
+#define PAGODA_MK_LAYOUT_CUH
+#include <stdint.h>
+
+#include "pagoda.h"
+#include "pagoda_device.cuh"
+
+namespace pagoda {
+
+struct __align__(64) TaskEntry {
+    uint64_t id;
+    uint16_t func_id;
+    uint16_t threads_tb;   /* requested threads per TB */
+    uint8_t  warps_tb;     /* ceil(threads/32) */
+    uint8_t  n_tb;
+    uint8_t  gran_tb;      /* ceil(shmem/512) granules per TB */
+    uint8_t  flags;        /* bit0 = sync */
+    uint32_t shmem_bytes;  /* requested bytes per TB */
+    uint32_t reserved;
+    uint8_t  args[PAGODA_ARGS_MAX];
+};
+static_assert(sizeof(TaskEntry) == 64, "TaskEntry is 64 bytes");
+
+/* pinned, mapped host memory: written by one side, read by the other over PCIe */
+struct HostCtl {
+    alignas(64) volatile uint64_t published;  /* host -> GPU doorbell: entries [0, published) written */
+    volatile uint32_t terminate;              /* host -> GPU: drain and exit */
+    alignas(64) volatile uint64_t consumed;   /* GPU -> host: entries copied to the device ring */
+    alignas(64) volatile uint32_t error;      /* GPU -> host: device error word (PAGODA_DEVERR_*) */
+    volatile uint32_t ingest_alive;
+    alignas(64) volatile uint64_t pad[8];
+};
+
+/* device memory, L2-resident: the device ring's counters */
+struct DevCtl {
+    alignas(128) uint64_t tail;    /* entries published into the device ring (ingest warp) */
+    alignas(128) uint64_t head;    /* entries claimed by schedulers (CAS) */
+    alignas(128) uint32_t stop;    /* set by ingest after terminate: schedulers drain and exit */
+    alignas(128) uint32_t error;   /* device error word (executors atomicOr) */
+    alignas(128) uint32_t exited;  /* MTBs that exited */
+};
+
+struct LedgerEvent {   /* 32 B; identical field order to the oracle's checker input */
+    uint32_t seq;
+    uint16_t mtb;
+    uint8_t  kind;     /* 1 ALLOC, 2 FREE_WARPS, 3 FREE_TB */
+    uint8_t  bar_id;
+    uint64_t task_id;
+    uint32_t warp_mask;
+    uint16_t tb;
+    uint16_t gran_off;
+    uint16_t gran_len;
+    uint16_t pad;
+    uint32_t pad2;
+};
+static_assert(sizeof(LedgerEvent) == 32, "LedgerEvent is 32 bytes");
+
+struct ExecRecord {    /* 32 B */
+    uint64_t task_id;
+    uint32_t tb;
+    uint16_t mtb;
+    uint16_t warp;
+    uint64_t t_start;
+    uint64_t t_end;
+};
+static_assert(sizeof(ExecRecord) == 32, "ExecRecord is 32 bytes");
+
+struct MkParams {
+    const TaskEntry* hring;   /* pinned host ring (mapped) */
+    HostCtl*         hctl;    /* pinned host control (mapped) */
+    int64_t*         comp;    /* pinned completion window (mapped) */
+    TaskEntry*       dring;   /* device ring */
+    DevCtl*          dctl;
+    uint32_t ring_mask;
+    uint32_t comp_mask;
+    int      exec_warps;      /* executor warps per MTB (warps 1..exec_warps) */
+    int      arena_granules;
+    int      n_mtb;
+    uint32_t trace_cap;       /* 0 = tracing off */
+    LedgerEvent* trace;       /* [n_mtb][trace_cap] */
+    uint32_t*    trace_count; /* [n_mtb] */
+    ExecRecord*  exec_trace;  /* [n_mtb][32][trace_cap] */
+    uint32_t*    exec_count;  /* [n_mtb][32] */
+};
+
+constexpr int kIngestWarp = 31;          /* warp 31 of MTB 0 feeds the device ring */
+constexpr int kMaxGranules = 1024;       /* lane-distributed bitmap: 32 lanes x 32 bits */
+
+/* Per-MTB control block at the start of dynamic shared memory (P:456-458:
+ * "the remaining shared memory ... stores scheduling data structures"). */
+struct MtbShared {
+    uint64_t  exec_bar[32];          /*    0: per-warp dispatch mbarriers (replaces the exec flag) */
+    uint64_t  stage_bar[32];         /*  256: per-warp TMA staging mbarriers */
+    WarpSlot  wt[32];                /*  512: WarpTable (Table 2) */
+    TaskEntry tasks[32];             /* 1536: task slots (entries claimed by this MTB) */
+    uint32_t  task_warps_left[32];   /* 3584: doneCtr (Alg. 1 L16, L41) */
+    uint32_t  tb_warps_left[32];     /* 3712: per-TB counter (lastWarpInBlock, Alg. 1 L35) */
+    uint16_t  tb_goff[32];           /* 3840 */
+    uint16_t  tb_glen[32];           /* 3904 */
+    uint8_t   tb_bar[32];            /* 3968 */
+    uint8_t   pend[32];              /* 4000: FIFO of claimed, not yet placed task slots */
+    uint32_t  mb_warps;              /* 4032: mailbox: warps that finished (atomicOr by executors) */
+    uint32_t  mb_tbs;                /*       mailbox: TB records whose last warp finished */
+    uint32_t  mb_tasks;              /*       mailbox: task slots whose last warp finished */
+    uint32_t  pad_;
+    uint64_t  tb_task[32];           /* 4048: task id of each TB record (ledger) */
+    uint16_t  tb_idx[32];            /* 4304: TB index j of each TB record (ledger) */
+};
+static_assert(offsetof(MtbShared, wt) == kWarpTableOffset, "WarpTable offset");
+static_assert(sizeof(MtbShared) <= kArenaOffset, "control block fits below the arena");
+
+} // namespace pagoda
+#endif

@@ -1,0 +1,494 @@
+/*
+ * runtime.cu — host side of the C ABI in include/pagoda.h.
+ *
+ * Spawn path (P:500-539 re-designed):
+ *   id = next_id++                       (the TaskTable index, also the task id)
+ *   wait until ring slot id mod R is free (GPU-posted `consumed` > id - R)
+ *   wait until completion slot id mod C is free (task id - C done)
+ *   write the 64-byte entry into the pinned host ring
+ *   in-order commit: wait for published == id, then published = id + 1
+ * The doorbell store is the only thing the GPU polls; no CUDA call per spawn.
+ *
+ * Completion (replaces the lazy aggregate copy-back + timeout):
+ * the task's last warp writes comp[id mod C] = id into pinned memory; a slot
+ * holds the newest finished occupant, and occupant id + C is only spawned after
+ * id is done, so "comp[id mod C] >= id" <=> id done.
+ */
+#include <cuda_runtime.h>
+#include <errno.h>
+#include <stdint.h>
+#include <stdio.h>
+#include <stdlib.h>
+#include <string.h>
+#include <time.h>
+#include <immintrin.h>
+
+#include <algorithm>
+#include <atomic>
+#include <chrono>
+#include <mutex>
+#include <thread>
+#include <vector>
+
+#include "bodies.cuh"
+#include "mk_layout.cuh"
+#include "pagoda.h"
+
+namespace pagoda {
+cudaError_t launch_master(int mtbs_per_sm, int n_mtb, size_t smem_bytes, cudaStream_t stream, MkParams* params,
+                          int* regs_out);
+}
+using namespace pagoda;
+
+static const uint32_t kIngestGranules = 32;   /* MTB 0 lends 16 KiB of its arena to the ingest warp */
+
+struct pagoda_ctx {
+    pagoda_config cfg;
+    int device = 0, sm_count = 0, n_mtb = 0, regs = 0;
+    int max_task_warps = 31;          /* largest warps*n_tb some MTB can host */
+    uint32_t max_task_granules = 0;   /* largest n_tb*granules some MTB can host */
+    uint32_t R = 0, C = 0;
+    cudaStream_t stream = nullptr;
+    /* pinned, mapped */
+    HostCtl* hctl = nullptr;
+    TaskEntry* hring = nullptr;
+    volatile int64_t* comp = nullptr;
+    /* device */
+    TaskEntry* dring = nullptr;
+    DevCtl* dctl = nullptr;
+    LedgerEvent* trace = nullptr;
+    uint32_t* trace_count = nullptr;
+    ExecRecord* exec_trace = nullptr;
+    uint32_t* exec_count = nullptr;
+    /* host state */
+    std::atomic<uint64_t> next_id{0};
+    std::atomic<uint64_t> published{0};     /* host mirror of hctl->published */
+    std::atomic<uint64_t> consumed_cache{0};
+    std::atomic<uint64_t> low{0};           /* every id < low is done */
+    std::mutex low_mtx;
+    std::atomic<int> shutting{0};
+    std::atomic<int> faulted{0};
+    std::vector<int64_t> warps_prefix;      /* warps_prefix[id mod C] = sum of warps of tasks <= id */
+    std::atomic<int64_t> warps_spawned{0};
+};
+
+/* ------------------------------------------------------------------ helpers */
+static inline uint64_t now_ns()
+{
+    timespec ts;
+    clock_gettime(CLOCK_MONOTONIC, &ts);
+    return (uint64_t)ts.tv_sec * 1000000000ull + (uint64_t)ts.tv_nsec;
+}
+
+/* Spin with pause / yield back-off; every ~1 ms check device faults and the
+ * watchdog.  pred() returns true when done. */
+template <class Pred>
+static int spin_until(pagoda_ctx* c, Pred pred)
+{
+    if (pred()) return 0;
+    const uint64_t t0 = now_ns();
+    uint64_t last_check = t0;
+    uint64_t spins = 0;
+    for (;;) {
+        if (pred()) return 0;
+        if (++spins < 4096) {
+            _mm_pause();
+            continue;
+        }
+        if ((spins & 63) == 0) std::this_thread::yield();
+        else _mm_pause();
+        const uint64_t t = now_ns();
+        if (t - last_check > 1000000ull) {
+            last_check = t;
+            if (c->hctl->error) return -EIO;
+            if (!c->shutting.load(std::memory_order_relaxed) || true) {
+                cudaError_t q = cudaStreamQuery(c->stream);
+                if (q != cudaErrorNotReady) {   /* MasterKernel gone (fault or exited) */
+                    if (pred()) return 0;
+                    c->faulted.store(1);
+                    return -EIO;
+                }
+            }
+            if (c->cfg.watchdog_s > 0 && (double)(t - t0) * 1e-9 > c->cfg.watchdog_s) return -ETIMEDOUT;
+        }
+    }
+}
+
+static void advance_low(pagoda_ctx* c, uint64_t limit)
+{
+    std::unique_lock<std::mutex> lk(c->low_mtx, std::try_to_lock);
+    if (!lk.owns_lock()) return;
+    uint64_t l = c->low.load(std::memory_order_relaxed);
+    const uint64_t mask = c->C - 1;
+    while (l < limit && c->comp[l & mask] >= (int64_t)l) l++;
+    c->low.store(l, std::memory_order_release);
+}
+
+extern "C" {
+
+void pagoda_config_default(pagoda_config* cfg)
+{
+    if (!cfg) return;
+    memset(cfg, 0, sizeof *cfg);
+    cfg->device = 0;
+    cfg->mtbs_per_sm = 2;
+    cfg->num_sms = 0;
+    cfg->ring_entries = 1u << 16;
+    cfg->comp_entries = 1u << 20;
+    cfg->arena_bytes = 96 * 1024;
+    cfg->exec_warps = 31;
+    cfg->flags = 0;
+    cfg->trace_events = 8192;
+    cfg->watchdog_s = 60.0;
+}
+
+static bool pow2(uint32_t x) { return x && !(x & (x - 1)); }
+
+static void free_ctx(pagoda_ctx* c)
+{
+    if (!c) return;
+    if (c->hctl) cudaFreeHost(c->hctl);
+    if (c->hring) cudaFreeHost(c->hring);
+    if (c->comp) cudaFreeHost((void*)c->comp);
+    if (c->dring) cudaFree(c->dring);
+    if (c->dctl) cudaFree(c->dctl);
+    if (c->trace) cudaFree(c->trace);
+    if (c->trace_count) cudaFree(c->trace_count);
+    if (c->exec_trace) cudaFree(c->exec_trace);
+    if (c->exec_count) cudaFree(c->exec_count);
+    if (c->stream) cudaStreamDestroy(c->stream);
+    delete c;
+}
+
+int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
+{
+    if (!out) return -EINVAL;
+    *out = nullptr;
+    pagoda_config cfg;
+    if (cfg_in) cfg = *cfg_in;
+    else pagoda_config_default(&cfg);
+    if (cfg.mtbs_per_sm != 1 && cfg.mtbs_per_sm != 2) return -EINVAL;
+    if (!pow2(cfg.ring_entries) || !pow2(cfg.comp_entries) || cfg.comp_entries < cfg.ring_entries) return -EINVAL;
+    if (cfg.exec_warps < 1 || cfg.exec_warps > 31) return -EINVAL;
+    if (cfg.arena_bytes % PAGODA_GRANULE || cfg.arena_bytes / PAGODA_GRANULE > (uint32_t)kMaxGranules ||
+        cfg.arena_bytes < kIngestGranules * PAGODA_GRANULE)
+        return -EINVAL;
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || cfg.device < 0 || cfg.device >= ndev) {
+        cudaGetLastError();
+        return -ENODEV;
+    }
+    if (cudaSetDevice(cfg.device) != cudaSuccess) return -ENODEV;
+    cudaDeviceProp prop;
+    if (cudaGetDeviceProperties(&prop, cfg.device) != cudaSuccess) return -ENODEV;
+    if (prop.major != 10) return -ENODEV;   /* built for sm_100a only */
+    const size_t smem = kArenaOffset + cfg.arena_bytes;
+    if (smem * (size_t)cfg.mtbs_per_sm + 1024 * (size_t)cfg.mtbs_per_sm > (size_t)prop.sharedMemPerMultiprocessor ||
+        smem > (size_t)prop.sharedMemPerBlockOptin)
+        return -EINVAL;
+    if (cfg.num_sms < 0 || cfg.num_sms > prop.multiProcessorCount) return -EINVAL;
+
+    pagoda_ctx* c = new (std::nothrow) pagoda_ctx;
+    if (!c) return -ENOMEM;
+    c->cfg = cfg;
+    c->device = cfg.device;
+    c->sm_count = prop.multiProcessorCount;
+    const int nsm = cfg.num_sms ? cfg.num_sms : prop.multiProcessorCount;
+    c->n_mtb = nsm * cfg.mtbs_per_sm;
+    c->R = cfg.ring_entries;
+    c->C = cfg.comp_entries;
+    const uint32_t arena_g = cfg.arena_bytes / PAGODA_GRANULE;
+    if (c->n_mtb == 1) {   /* MTB 0 alone: it also hosts the ingest warp and its staging */
+        c->max_task_warps = cfg.exec_warps == 31 ? 30 : (int)cfg.exec_warps;
+        c->max_task_granules = arena_g - kIngestGranules;
+    } else {
+        c->max_task_warps = (int)cfg.exec_warps;
+        c->max_task_granules = arena_g;
+    }
+    c->warps_prefix.assign(c->C, 0);
+
+    int rc = -ENOMEM;
+    if (cudaHostAlloc((void**)&c->hctl, sizeof(HostCtl), cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess)
+        goto fail;
+    memset((void*)c->hctl, 0, sizeof(HostCtl));
+    if (cudaHostAlloc((void**)&c->hring, (size_t)c->R * sizeof(TaskEntry), cudaHostAllocMapped | cudaHostAllocPortable) !=
+        cudaSuccess)
+        goto fail;
+    memset(c->hring, 0, (size_t)c->R * sizeof(TaskEntry));
+    if (cudaHostAlloc((void**)&c->comp, (size_t)c->C * sizeof(int64_t), cudaHostAllocMapped | cudaHostAllocPortable) !=
+        cudaSuccess)
+        goto fail;
+    for (uint32_t i = 0; i < c->C; i++) c->comp[i] = -1;
+    if (cudaMalloc(&c->dring, (size_t)c->R * sizeof(TaskEntry)) != cudaSuccess) goto fail;
+    if (cudaMalloc(&c->dctl, sizeof(DevCtl)) != cudaSuccess) goto fail;
+    if (cudaMemset(c->dctl, 0, sizeof(DevCtl)) != cudaSuccess) goto fail;
+    if (cfg.flags & PAGODA_TRACE) {
+        const size_t cap = cfg.trace_events ? cfg.trace_events : 8192;
+        c->cfg.trace_events = (uint32_t)cap;
+        if (cudaMalloc(&c->trace, (size_t)c->n_mtb * cap * sizeof(LedgerEvent)) != cudaSuccess) goto fail;
+        if (cudaMalloc(&c->trace_count, (size_t)c->n_mtb * sizeof(uint32_t)) != cudaSuccess) goto fail;
+        if (cudaMalloc(&c->exec_trace, (size_t)c->n_mtb * 32 * cap * sizeof(ExecRecord)) != cudaSuccess) goto fail;
+        if (cudaMalloc(&c->exec_count, (size_t)c->n_mtb * 32 * sizeof(uint32_t)) != cudaSuccess) goto fail;
+        cudaMemset(c->trace_count, 0, (size_t)c->n_mtb * sizeof(uint32_t));
+        cudaMemset(c->exec_count, 0, (size_t)c->n_mtb * 32 * sizeof(uint32_t));
+    }
+    if (cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking) != cudaSuccess) goto fail;
+    if (cudaDeviceSynchronize() != cudaSuccess) goto fail;
+    {
+        MkParams p;
+        memset(&p, 0, sizeof p);
+        void* dptr = nullptr;
+        cudaHostGetDevicePointer(&dptr, (void*)c->hring, 0);
+        p.hring = (const TaskEntry*)dptr;
+        cudaHostGetDevicePointer(&dptr, (void*)c->hctl, 0);
+        p.hctl = (HostCtl*)dptr;
+        cudaHostGetDevicePointer(&dptr, (void*)c->comp, 0);
+        p.comp = (int64_t*)dptr;
+        p.dring = c->dring;
+        p.dctl = c->dctl;
+        p.ring_mask = c->R - 1;
+        p.comp_mask = c->C - 1;
+        p.exec_warps = (int)cfg.exec_warps;
+        p.arena_granules = (int)arena_g;
+        p.n_mtb = c->n_mtb;
+        if (cfg.flags & PAGODA_TRACE) {
+            p.trace_cap = c->cfg.trace_events;
+            p.trace = c->trace;
+            p.trace_count = c->trace_count;
+            p.exec_trace = c->exec_trace;
+            p.exec_count = c->exec_count;
+        }
+        cudaError_t e = launch_master(cfg.mtbs_per_sm, c->n_mtb, smem, c->stream, &p, &c->regs);
+        if (e != cudaSuccess) {
+            fprintf(stderr, "pagoda_init: MasterKernel launch failed: %s\n", cudaGetErrorString(e));
+            cudaGetLastError();
+            rc = -EIO;
+            goto fail;
+        }
+    }
+    *out = c;
+    return 0;
+fail:
+    cudaGetLastError();
+    free_ctx(c);
+    return rc;
+}
+
+pagoda_task_t pagoda_taskSpawn(pagoda_ctx* c, int threads, int n_tb, int shmem_bytes, int sync_flag, int func_id,
+                               const void* args, size_t args_bytes)
+{
+    if (!c) return -EINVAL;
+    if (c->shutting.load(std::memory_order_acquire)) return -ESHUTDOWN;
+    if (c->faulted.load(std::memory_order_relaxed)) return -EIO;
+    if (threads < 1 || threads > 1024 || n_tb < 1 || shmem_bytes < 0) return -EINVAL;
+    const int wtb = (threads + 31) / 32;
+    if ((long)wtb * n_tb > c->max_task_warps) return -EINVAL;
+    const uint32_t gtb = ((uint32_t)shmem_bytes + PAGODA_GRANULE - 1) / PAGODA_GRANULE;
+    if ((uint64_t)gtb * (uint64_t)n_tb > c->max_task_granules) return -EINVAL;
+    if (sync_flag && wtb > 1 && n_tb > PAGODA_BAR_IDS) return -EINVAL;
+    if (!known_func(func_id)) return -EINVAL;
+    if (args_bytes > PAGODA_ARGS_MAX || (args_bytes > 0 && !args)) return -EINVAL;
+
+    const uint64_t id = c->next_id.fetch_add(1, std::memory_order_acq_rel);
+    /* 1. ring slot free: the ingest warp has copied entry id - R */
+    if (id >= c->R && c->consumed_cache.load(std::memory_order_acquire) <= id - c->R) {
+        int rc = spin_until(c, [&] {
+            const uint64_t v = c->hctl->consumed;
+            uint64_t cur = c->consumed_cache.load(std::memory_order_relaxed);
+            while (v > cur && !c->consumed_cache.compare_exchange_weak(cur, v)) { }
+            return v > id - c->R;
+        });
+        if (rc) return rc;
+    }
+    /* 2. completion slot free: task id - C is done */
+    if (id >= c->C && c->low.load(std::memory_order_acquire) <= id - c->C) {
+        int rc = spin_until(c, [&] {
+            advance_low(c, id - c->C + 1);
+            return c->low.load(std::memory_order_acquire) > id - c->C;
+        });
+        if (rc) return rc;
+    }
+    /* 3. the entry */
+    TaskEntry e;
+    memset(&e, 0, sizeof e);
+    e.id = id;
+    e.func_id = (uint16_t)func_id;
+    e.threads_tb = (uint16_t)threads;
+    e.warps_tb = (uint8_t)wtb;
+    e.n_tb = (uint8_t)n_tb;
+    e.gran_tb = (uint8_t)gtb;
+    e.flags = sync_flag ? 1 : 0;
+    e.shmem_bytes = (uint32_t)shmem_bytes;
+    if (args_bytes) memcpy(e.args, args, args_bytes);
+    {
+        const __m128i* s = reinterpret_cast<const __m128i*>(&e);
+        __m128i* d = reinterpret_cast<__m128i*>(&c->hring[id & (c->R - 1)]);
+        _mm_store_si128(d + 0, _mm_load_si128(s + 0));
+        _mm_store_si128(d + 1, _mm_load_si128(s + 1));
+        _mm_store_si128(d + 2, _mm_load_si128(s + 2));
+        _mm_store_si128(d + 3, _mm_load_si128(s + 3));
+    }
+    const int64_t w = (int64_t)wtb * n_tb;
+    /* 4. in-order commit of the doorbell (x86 stores are ordered; the fence is for the compiler) */
+    if (c->published.load(std::memory_order_acquire) != id) {
+        int rc = spin_until(c, [&] { return c->published.load(std::memory_order_acquire) == id; });
+        if (rc) return rc;
+    }
+    c->warps_prefix[id & (c->C - 1)] = c->warps_spawned.fetch_add(w, std::memory_order_relaxed) + w;
+    std::atomic_thread_fence(std::memory_order_release);
+    c->hctl->published = id + 1;
+    c->published.store(id + 1, std::memory_order_release);
+    return (pagoda_task_t)id;
+}
+
+int64_t pagoda_taskSpawnMany(pagoda_ctx* c, int n, int threads, int n_tb, int shmem_bytes, int sync_flag, int func_id,
+                             const void* args_base, size_t args_stride, size_t args_bytes, pagoda_task_t* ids_out)
+{
+    const char* a = static_cast<const char*>(args_base);
+    for (int i = 0; i < n; i++) {
+        pagoda_task_t id = pagoda_taskSpawn(c, threads, n_tb, shmem_bytes, sync_flag, func_id,
+                                            a ? a + (size_t)i * args_stride : nullptr, args_bytes);
+        if (id < 0) return id;
+        if (ids_out) ids_out[i] = id;
+    }
+    return n;
+}
+
+int64_t pagoda_taskSpawnShapes(pagoda_ctx* c, int n, const int32_t* shapes, const void* args_base, size_t args_stride,
+                               size_t args_bytes, pagoda_task_t* ids_out)
+{
+    const char* a = static_cast<const char*>(args_base);
+    for (int i = 0; i < n; i++) {
+        const int32_t* s = shapes + 5 * (size_t)i;
+        pagoda_task_t id =
+            pagoda_taskSpawn(c, s[0], s[1], s[2], s[3], s[4], a ? a + (size_t)i * args_stride : nullptr, args_bytes);
+        if (id < 0) return id;
+        if (ids_out) ids_out[i] = id;
+    }
+    return n;
+}
+
+int pagoda_check(pagoda_ctx* c, pagoda_task_t id)
+{
+    if (!c) return -EINVAL;
+    if (id < 0 || (uint64_t)id >= c->next_id.load(std::memory_order_acquire)) return -EINVAL;
+    if ((uint64_t)id < c->low.load(std::memory_order_acquire)) return 1;
+    if (c->comp[(uint64_t)id & (c->C - 1)] >= id) return 1;
+    if (c->hctl->error) return -EIO;
+    return 0;
+}
+
+int pagoda_wait(pagoda_ctx* c, pagoda_task_t id)
+{
+    if (!c) return -EINVAL;
+    if (id < 0 || (uint64_t)id >= c->next_id.load(std::memory_order_acquire)) return -EINVAL;
+    if ((uint64_t)id < c->low.load(std::memory_order_acquire)) return 0;
+    volatile int64_t* slot = &c->comp[(uint64_t)id & (c->C - 1)];
+    int rc = spin_until(c, [&] { return *slot >= id; });
+    std::atomic_thread_fence(std::memory_order_acquire);
+    return rc;
+}
+
+int pagoda_waitAll(pagoda_ctx* c)
+{
+    if (!c) return -EINVAL;
+    const uint64_t n = c->next_id.load(std::memory_order_acquire);
+    int rc = spin_until(c, [&] {
+        advance_low(c, n);
+        return c->low.load(std::memory_order_acquire) >= n;
+    });
+    std::atomic_thread_fence(std::memory_order_acquire);
+    return rc;
+}
+
+int pagoda_shutdown(pagoda_ctx* c)
+{
+    if (!c) return -EINVAL;
+    int rc = 0;
+    if (!c->faulted.load()) rc = pagoda_waitAll(c);
+    c->shutting.store(1, std::memory_order_release);
+    c->hctl->terminate = 1;
+    /* the MasterKernel drains and exits: wait for the stream (bounded) */
+    const uint64_t t0 = now_ns();
+    cudaError_t q;
+    while ((q = cudaStreamQuery(c->stream)) == cudaErrorNotReady) {
+        std::this_thread::sleep_for(std::chrono::microseconds(50));
+        if (c->cfg.watchdog_s > 0 && (double)(now_ns() - t0) * 1e-9 > c->cfg.watchdog_s) {
+            fprintf(stderr, "pagoda_shutdown: MasterKernel did not exit (watchdog)\n");
+            return -ETIMEDOUT;   /* leak: freeing live buffers would fault the kernel */
+        }
+    }
+    if (q != cudaSuccess) {
+        fprintf(stderr, "pagoda_shutdown: MasterKernel error: %s\n", cudaGetErrorString(q));
+        rc = -EIO;
+    }
+    if (c->hctl->error && rc == 0) rc = -EIO;
+    cudaSetDevice(c->device);
+    free_ctx(c);
+    return rc;
+}
+
+int pagoda_get_info(pagoda_ctx* c, pagoda_info* o)
+{
+    if (!c || !o) return -EINVAL;
+    memset(o, 0, sizeof *o);
+    o->device = c->device;
+    o->sm_count = c->sm_count;
+    o->n_mtb = c->n_mtb;
+    o->mtbs_per_sm = c->cfg.mtbs_per_sm;
+    o->exec_warps = (int)c->cfg.exec_warps;
+    o->arena_bytes = (int)c->cfg.arena_bytes;
+    o->regs_per_thread = c->regs;
+    o->ring_entries = c->R;
+    o->comp_entries = c->C;
+    o->spawned = (int64_t)c->next_id.load();
+    advance_low(c, c->next_id.load());
+    o->completed_low = (int64_t)c->low.load();
+    o->device_error = c->hctl->error;
+    o->running = cudaStreamQuery(c->stream) == cudaErrorNotReady;
+    return 0;
+}
+
+int64_t pagoda_trace_read(pagoda_ctx* c, int mtb, void* dst, size_t cap)
+{
+    if (!c || !c->trace || mtb < 0 || mtb >= c->n_mtb) return -EINVAL;
+    uint32_t n = 0;
+    if (cudaMemcpy(&n, c->trace_count + mtb, 4, cudaMemcpyDeviceToHost) != cudaSuccess) return -EIO;
+    const size_t k = std::min<size_t>({(size_t)n, cap, (size_t)c->cfg.trace_events});
+    if (k && dst &&
+        cudaMemcpy(dst, c->trace + (size_t)mtb * c->cfg.trace_events, k * sizeof(LedgerEvent), cudaMemcpyDeviceToHost) !=
+            cudaSuccess)
+        return -EIO;
+    return n;
+}
+
+int64_t pagoda_trace_read_exec(pagoda_ctx* c, int mtb, int warp, void* dst, size_t cap)
+{
+    if (!c || !c->exec_trace || mtb < 0 || mtb >= c->n_mtb || warp < 0 || warp > 31) return -EINVAL;
+    uint32_t n = 0;
+    const size_t idx = (size_t)mtb * 32 + (size_t)warp;
+    if (cudaMemcpy(&n, c->exec_count + idx, 4, cudaMemcpyDeviceToHost) != cudaSuccess) return -EIO;
+    const size_t k = std::min<size_t>({(size_t)n, cap, (size_t)c->cfg.trace_events});
+    if (k && dst &&
+        cudaMemcpy(dst, c->exec_trace + idx * c->cfg.trace_events, k * sizeof(ExecRecord), cudaMemcpyDeviceToHost) !=
+            cudaSuccess)
+        return -EIO;
+    return n;
+}
+
+/* in-flight warps of a context = warps spawned - warps of the tasks below the
+ * low watermark (tasks completed out of order above it still count) */
+int64_t pagoda_inflight_warps(pagoda_ctx* c)
+{
+    if (!c) return -EINVAL;
+    const uint64_t n = c->next_id.load(std::memory_order_acquire);
+    advance_low(c, n);
+    const uint64_t l = c->low.load(std::memory_order_acquire);
+    const int64_t spawned = c->warps_spawned.load(std::memory_order_acquire);
+    const int64_t done = l ? c->warps_prefix[(l - 1) & (c->C - 1)] : 0;
+    return spawned - done;
+}
+
+const char* pagoda_version(void) { return "pagoda-b200 0.1 (sm_100a)"; }
+
+} /* extern "C" */

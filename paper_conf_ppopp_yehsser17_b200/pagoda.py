@@ -1,0 +1,253 @@
+"""Thin ctypes binding of libpagoda.so (include/pagoda.h) — argument marshalling
+only; every step of the hot path runs in the library's C++/CUDA code.
+
+There is no fallback: if libpagoda.so is missing this module raises on use.
+PyTorch (if used by the caller) only provides device memory; pass
+tensor.data_ptr() values inside the args records.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import errno
+import os
+
+import numpy as np
+
+PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(PKG, "libpagoda.so")
+
+TRACE = 0x1
+
+
+class pagoda_config(C.Structure):
+    _fields_ = [("device", C.c_int), ("mtbs_per_sm", C.c_int), ("num_sms", C.c_int),
+                ("ring_entries", C.c_uint32), ("comp_entries", C.c_uint32), ("arena_bytes", C.c_uint32),
+                ("exec_warps", C.c_uint32), ("flags", C.c_uint32), ("trace_events", C.c_uint32),
+                ("watchdog_s", C.c_double)]
+
+
+class pagoda_info(C.Structure):
+    _fields_ = [("device", C.c_int), ("sm_count", C.c_int), ("n_mtb", C.c_int), ("mtbs_per_sm", C.c_int),
+                ("exec_warps", C.c_int), ("arena_bytes", C.c_int), ("regs_per_thread", C.c_int),
+                ("ring_entries", C.c_uint32), ("comp_entries", C.c_uint32), ("spawned", C.c_int64),
+                ("completed_low", C.c_int64), ("device_error", C.c_uint32), ("running", C.c_int)]
+
+
+LEDGER_DTYPE = np.dtype([("seq", "<u4"), ("mtb", "<u2"), ("kind", "u1"), ("bar_id", "u1"),
+                         ("task_id", "<u8"), ("warp_mask", "<u4"), ("tb", "<u2"), ("gran_off", "<u2"),
+                         ("gran_len", "<u2"), ("pad", "<u2"), ("pad2", "<u4")])
+EXEC_DTYPE = np.dtype([("task_id", "<u8"), ("tb", "<u4"), ("mtb", "<u2"), ("warp", "<u2"),
+                       ("t_start", "<u8"), ("t_end", "<u8")])
+
+# names declared in include/pagoda.h (the ABI test checks the library exports them)
+_lib = None
+
+
+def lib() -> C.CDLL:
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise RuntimeError(f"{LIB_PATH} is not built: run paper_conf_ppopp_yehsser17_b200.build.build() "
+                               "(there is no CPU fallback)")
+        L = C.CDLL(LIB_PATH)
+        P, I, I64, SZ, U32 = C.c_void_p, C.c_int, C.c_int64, C.c_size_t, C.c_uint32
+        L.pagoda_config_default.argtypes = [C.POINTER(pagoda_config)]
+        L.pagoda_init.argtypes = [C.POINTER(pagoda_config), C.POINTER(P)]
+        L.pagoda_shutdown.argtypes = [P]
+        L.pagoda_taskSpawn.argtypes = [P, I, I, I, I, I, P, SZ]
+        L.pagoda_taskSpawn.restype = I64
+        L.pagoda_wait.argtypes = [P, I64]
+        L.pagoda_check.argtypes = [P, I64]
+        L.pagoda_waitAll.argtypes = [P]
+        L.pagoda_taskSpawnMany.argtypes = [P, I, I, I, I, I, I, P, SZ, SZ, P]
+        L.pagoda_taskSpawnMany.restype = I64
+        L.pagoda_taskSpawnShapes.argtypes = [P, I, P, P, SZ, SZ, P]
+        L.pagoda_taskSpawnShapes.restype = I64
+        L.pagoda_get_info.argtypes = [P, C.POINTER(pagoda_info)]
+        L.pagoda_trace_read.argtypes = [P, I, P, SZ]
+        L.pagoda_trace_read.restype = I64
+        L.pagoda_trace_read_exec.argtypes = [P, I, I, P, SZ]
+        L.pagoda_trace_read_exec.restype = I64
+        L.pagoda_tdes_tables.argtypes = [P, P]
+        L.pagoda_naive_run.argtypes = [I, I, P, P, SZ, SZ, I, C.POINTER(I64)]
+        L.pagoda_pool_init.argtypes = [I, P, C.POINTER(pagoda_config), C.POINTER(P)]
+        L.pagoda_pool_pick.argtypes = [P, I]
+        L.pagoda_pool_ctx.argtypes = [P, I]
+        L.pagoda_pool_ctx.restype = P
+        L.pagoda_pool_size.argtypes = [P]
+        L.pagoda_pool_spawn.argtypes = [P, I, I, I, I, I, P, SZ, C.POINTER(I)]
+        L.pagoda_pool_spawn.restype = I64
+        L.pagoda_pool_waitAll.argtypes = [P]
+        L.pagoda_pool_shutdown.argtypes = [P]
+        L.pagoda_inflight_warps.argtypes = [P]
+        L.pagoda_inflight_warps.restype = I64
+        L.pagoda_pick_least_loaded.argtypes = [P, I]
+        L.pagoda_version.restype = C.c_char_p
+        _lib = L
+    return _lib
+
+
+class PagodaError(OSError):
+    pass
+
+
+def _check(rc: int, what: str) -> int:
+    if rc < 0:
+        raise PagodaError(-rc, f"{what}: {os.strerror(-rc)}")
+    return rc
+
+
+def _ptr(a):
+    if a is None:
+        return None
+    if isinstance(a, np.ndarray):
+        assert a.flags["C_CONTIGUOUS"]
+        return a.ctypes.data_as(C.c_void_p)
+    return a
+
+
+def default_config(**kw) -> pagoda_config:
+    cfg = pagoda_config()
+    lib().pagoda_config_default(C.byref(cfg))
+    for k, v in kw.items():
+        setattr(cfg, k, v)
+    return cfg
+
+
+class Pagoda:
+    """One Pagoda context (one MasterKernel on one GPU).  Method names follow
+    the paper's Table 1."""
+
+    def __init__(self, **config):
+        self.cfg = default_config(**config)
+        self.h = C.c_void_p()
+        _check(lib().pagoda_init(C.byref(self.cfg), C.byref(self.h)), "pagoda_init")
+        self._alive = True
+
+    # --- Table 1 -----------------------------------------------------------
+    def taskSpawn(self, threads: int, n_tb: int, shmem: int, sync: bool, func_id: int, args=None) -> int:
+        """Returns the task id (>= 0) or a negative errno (no exception, as the C ABI)."""
+        if args is None:
+            return lib().pagoda_taskSpawn(self.h, threads, n_tb, shmem, int(sync), func_id, None, 0)
+        b = args.tobytes() if isinstance(args, np.ndarray) else bytes(args)
+        return lib().pagoda_taskSpawn(self.h, threads, n_tb, shmem, int(sync), func_id, b, len(b))
+
+    def wait(self, task_id: int) -> int:
+        return lib().pagoda_wait(self.h, task_id)
+
+    def check(self, task_id: int) -> int:
+        return lib().pagoda_check(self.h, task_id)
+
+    def waitAll(self) -> int:
+        return lib().pagoda_waitAll(self.h)
+
+    # --- batch conveniences (each task is still one taskSpawn in C) --------
+    def spawn_many(self, n, threads, n_tb, shmem, sync, func_id, args: np.ndarray | None, ids=False):
+        out = np.empty(n, np.int64) if ids else None
+        stride = args.dtype.itemsize if args is not None else 0
+        rc = lib().pagoda_taskSpawnMany(self.h, n, threads, n_tb, shmem, int(sync), func_id, _ptr(args),
+                                        stride, stride, _ptr(out))
+        _check(rc, "pagoda_taskSpawnMany")
+        return out
+
+    def spawn_shapes(self, shapes: np.ndarray, args: np.ndarray, ids=False):
+        """shapes: int32 [n,5] = threads, n_tb, shmem, sync, func_id; args: uint8 [n,40]."""
+        shapes = np.ascontiguousarray(shapes, np.int32)
+        args = np.ascontiguousarray(args, np.uint8)
+        n = len(shapes)
+        out = np.empty(n, np.int64) if ids else None
+        rc = lib().pagoda_taskSpawnShapes(self.h, n, _ptr(shapes), _ptr(args), args.shape[1], args.shape[1],
+                                          _ptr(out))
+        _check(rc, "pagoda_taskSpawnShapes")
+        return out
+
+    def info(self) -> pagoda_info:
+        i = pagoda_info()
+        _check(lib().pagoda_get_info(self.h, C.byref(i)), "pagoda_get_info")
+        return i
+
+    def inflight_warps(self) -> int:
+        return lib().pagoda_inflight_warps(self.h)
+
+    def trace(self, mtb: int) -> np.ndarray:
+        n = _check(lib().pagoda_trace_read(self.h, mtb, None, 0), "pagoda_trace_read")
+        buf = np.zeros(min(n, self.cfg.trace_events), LEDGER_DTYPE)
+        _check(lib().pagoda_trace_read(self.h, mtb, _ptr(buf), len(buf)), "pagoda_trace_read")
+        if n > len(buf):
+            raise PagodaError(errno.ENOSPC, f"trace overflow on MTB {mtb}: {n} events")
+        return buf
+
+    def exec_trace(self, mtb: int, warp: int) -> np.ndarray:
+        n = _check(lib().pagoda_trace_read_exec(self.h, mtb, warp, None, 0), "pagoda_trace_read_exec")
+        buf = np.zeros(min(n, self.cfg.trace_events), EXEC_DTYPE)
+        _check(lib().pagoda_trace_read_exec(self.h, mtb, warp, _ptr(buf), len(buf)), "pagoda_trace_read_exec")
+        return buf
+
+    def shutdown(self) -> int:
+        if not self._alive:
+            return 0
+        self._alive = False
+        return lib().pagoda_shutdown(self.h)
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.shutdown()
+
+
+# --------------------------------------------------------------------- misc
+def tdes_tables(key24: bytes) -> np.ndarray:
+    out = np.zeros(2048 + 384 + 16384 + 16384, np.uint8)
+    k = np.frombuffer(key24, np.uint8).copy()
+    _check(lib().pagoda_tdes_tables(_ptr(k), _ptr(out)), "pagoda_tdes_tables")
+    return out
+
+
+def naive_run(device: int, shapes: np.ndarray, args: np.ndarray, n_streams: int = 32) -> int:
+    """One kernel launch per task; returns elapsed host ns (launch of the first
+    task -> all done)."""
+    shapes = np.ascontiguousarray(shapes, np.int32)
+    args = np.ascontiguousarray(args, np.uint8)
+    ns = C.c_int64(0)
+    _check(lib().pagoda_naive_run(device, len(shapes), _ptr(shapes), _ptr(args), args.shape[1], args.shape[1],
+                                  n_streams, C.byref(ns)), "pagoda_naive_run")
+    return ns.value
+
+
+def pick_least_loaded(loads) -> int:
+    a = np.ascontiguousarray(loads, np.int64)
+    return lib().pagoda_pick_least_loaded(_ptr(a), len(a))
+
+
+def version() -> str:
+    return lib().pagoda_version().decode()
+
+
+class Pool:
+    """One context per GPU plus the least-loaded picker."""
+
+    def __init__(self, devices, **config):
+        self.cfg = default_config(**config)
+        self.devices = list(devices)
+        d = np.array(self.devices, np.int32)
+        self.h = C.c_void_p()
+        _check(lib().pagoda_pool_init(len(d), _ptr(d), C.byref(self.cfg), C.byref(self.h)), "pagoda_pool_init")
+
+    def pick(self, warps_hint: int) -> int:
+        return lib().pagoda_pool_pick(self.h, warps_hint)
+
+    def spawn(self, threads, n_tb, shmem, sync, func_id, args_per_dev):
+        bufs = [C.create_string_buffer(bytes(a), len(bytes(a))) for a in args_per_dev]
+        arr = (C.c_void_p * len(bufs))(*[C.cast(b, C.c_void_p) for b in bufs])
+        idx = C.c_int(-1)
+        nbytes = len(bytes(args_per_dev[0]))
+        tid = lib().pagoda_pool_spawn(self.h, threads, n_tb, shmem, int(sync), func_id, arr, nbytes,
+                                      C.byref(idx))
+        return tid, idx.value
+
+    def waitAll(self) -> int:
+        return lib().pagoda_pool_waitAll(self.h)
+
+    def shutdown(self) -> int:
+        return lib().pagoda_pool_shutdown(self.h)

@@ -1,0 +1,159 @@
+"""Parity: the CUDA path (through the C-ABI) against the oracle, element by
+element, on the same seeded inputs.
+
+Bar (BASELINE.json north star): bit-exact for integer tasks (Mandelbrot counts,
+3DES ciphertext); fp32 tasks within rel = |g-o| / max(|o|, 1e-6 max|o|) <= 1e-5
+elementwise.  The fp32 bodies fix their operation order on both sides, so they
+are also expected to be bit-exact, and that is asserted too.
+
+Sizes: the oracle-sized cases span several tiles / MTBs and ragged shapes; the
+BASELINE.json full sizes run in the launch configuration bench.py times and are
+checked on sampled tasks the oracle computes one by one (plus, for 3DES, every
+packet against an independent library implementation).
+"""
+import numpy as np
+import pytest
+
+import oracle
+from paper_conf_ppopp_yehsser17_b200 import inputs as I
+from paper_conf_ppopp_yehsser17_b200 import workloads as W
+from paper_conf_ppopp_yehsser17_b200.pagoda import Pagoda, naive_run
+
+pytestmark = pytest.mark.gpu
+
+TOL = 1e-5
+
+
+def fp32_close(g, o):
+    g = np.asarray(g, np.float64)
+    o = np.asarray(o, np.float64)
+    den = np.maximum(np.abs(o), 1e-6 * np.abs(o).max())
+    rel = np.abs(g - o) / den
+    return rel.max()
+
+
+def run(w, **cfg):
+    with Pagoda(**cfg) as p:
+        p.spawn_shapes(w.shapes, w.args)
+        assert p.waitAll() == 0
+        assert p.info().device_error == 0
+    return w.outputs()
+
+
+# ---------------------------------------------------------------- MB (config 1)
+def test_mandelbrot_config1_bit_exact():
+    w = W.mandelbrot(1024)
+    out = run(w)["out"]
+    for k in range(1024):
+        ref = oracle.mandelbrot_tile(int(w.host["tx"][k]), int(w.host["ty"][k]))
+        assert np.array_equal(out[k], ref), k
+    assert int(out.astype(np.int64).sum()) == 199370695
+
+
+@pytest.mark.parametrize("threads", [32, 100, 992])
+def test_mandelbrot_other_thread_counts(threads):
+    w = W.mandelbrot(96, threads=threads)
+    out = run(w)["out"]
+    for k in range(0, 96, 7):
+        assert np.array_equal(out[k], oracle.mandelbrot_tile(int(w.host["tx"][k]), int(w.host["ty"][k])))
+
+
+# ---------------------------------------------------------------- 3DES (config 2)
+def _tdes_ref(packet):
+    return oracle.tdes_ecb(packet, I.TDES_KEYS)
+
+
+@pytest.mark.parametrize("shmem,threads", [(2560, 128), (0, 128), (2560, 96), (2560, 32)])
+def test_tdes_small_bit_exact(shmem, threads):
+    w = W.tdes(48, shmem=shmem, threads=threads)
+    out = run(w)["out"]
+    for k in range(48):
+        assert np.array_equal(out[k], _tdes_ref(w.host["packets"][k])), k
+    assert out[0, :24].tobytes().hex() == "a826fd8ce53b855fcce21c8112256fe668d5c05dd9b6b900"
+
+
+def test_tdes_config2_full_size():
+    from cryptography.hazmat.decrepit.ciphers.algorithms import TripleDES
+    from cryptography.hazmat.primitives.ciphers import Cipher, modes
+    w = W.tdes(32768)
+    out = run(w)["out"]
+    pk = w.host["packets"]
+    enc = Cipher(TripleDES(I.TDES_KEYS), modes.ECB()).encryptor()
+    ref_all = np.frombuffer(enc.update(pk.tobytes()) + enc.finalize(), np.uint8).reshape(pk.shape)
+    assert np.array_equal(out, ref_all)                    # every packet, independent library
+    rng = np.random.default_rng(2)
+    for k in list(rng.choice(32768, 24, replace=False)) + [0, 32767]:
+        assert np.array_equal(out[k], _tdes_ref(pk[k])), k  # sampled, the oracle
+
+
+# ---------------------------------------------------------------- MM (config 3)
+def _mm_check(w, out, ks):
+    for k in ks:
+        ref = oracle.mm32(w.host["A"][k], w.host["B"][k])
+        assert fp32_close(out[k], ref) <= TOL
+        assert np.array_equal(out[k], ref), k
+
+
+@pytest.mark.parametrize("shmem,threads", [(8192, 256), (0, 256), (8192, 64), (8192, 32), (4096, 1000 // 4)])
+def test_mm_small(shmem, threads):
+    w = W.matmul(300, shmem=shmem, threads=threads)
+    _mm_check(w, run(w)["C"], range(300))
+
+
+def test_mm_config3_full_size():
+    w = W.matmul(65536)
+    out = run(w)["C"]
+    rng = np.random.default_rng(3)
+    _mm_check(w, out, list(rng.choice(65536, 256, replace=False)) + [0, 65535])
+
+
+# ---------------------------------------------------------------- mix (config 4)
+def _mix_check(w, out, frac=1.0, seed=0):
+    rng = np.random.default_rng(seed)
+
+    def pick(n):
+        return range(n) if frac >= 1 else rng.choice(n, max(1, int(n * frac)), replace=False)
+
+    r, H, F = w.host["fb"]
+    for k in pick(len(r)):
+        ref = oracle.filterbank(r[k], H[k], F[k])
+        assert fp32_close(out["fb"][k], ref) <= TOL and np.array_equal(out["fb"][k], ref), ("fb", k)
+    x, h, ww = w.host["bf"]
+    for k in pick(len(x)):
+        ref = oracle.beamformer(x[k], h[k], ww[k])
+        assert fp32_close(out["bf"][k], ref) <= TOL and np.array_equal(out["bf"][k], ref), ("bf", k)
+    img, kr, kc = w.host["conv"]
+    for k in pick(len(img)):
+        ref = oracle.conv(img[k], kr[k], kc[k])
+        assert fp32_close(out["conv"][k], ref) <= TOL and np.array_equal(out["conv"][k], ref), ("conv", k)
+    im, coef = w.host["dct"]
+    for k in pick(len(im)):
+        ref = oracle.dct(im[k], coef)
+        assert fp32_close(out["dct"][k], ref) <= TOL and np.array_equal(out["dct"][k], ref), ("dct", k)
+
+
+def test_mix_small_all_shapes():
+    w = W.mix(160)     # threads 32..512, shmem 0..48 KiB, ragged per task
+    _mix_check(w, run(w))
+
+
+def test_mix_config4_full_size_sampled():
+    w = W.mix(32768)
+    _mix_check(w, run(w), frac=0.004, seed=4)
+
+
+# ---------------------------------------------------------------- the naive baseline runs the same bodies
+def test_naive_baseline_parity():
+    w = W.mandelbrot(64)
+    naive_run(0, w.shapes, w.args, 32)
+    out = w.outputs()["out"]
+    for k in range(0, 64, 5):
+        assert np.array_equal(out[k], oracle.mandelbrot_tile(int(w.host["tx"][k]), int(w.host["ty"][k])))
+    w = W.mix(40)
+    naive_run(0, w.shapes, w.args, 32)
+    _mix_check(w, w.outputs())
+    w = W.tdes(16)
+    naive_run(0, w.shapes, w.args, 32)
+    out = w.outputs()["out"]
+    for k in range(16):
+        assert np.array_equal(out[k], _tdes_ref(w.host["packets"][k]))

@@ -1,0 +1,238 @@
+"""Runtime semantics on the GPU through the C-ABI (Table 1):
+spawn/wait/check/waitAll contract, exactly-once completion, getTid, syncBlock,
+getSMPtr, liveness, validation, multiple producers, and the scheduler ledger
+replayed by the oracle-side checker."""
+import errno
+import threading
+import time
+
+import numpy as np
+import pytest
+
+from gpu_util import Dev, ptr
+from paper_conf_ppopp_yehsser17_b200 import tasks as T
+from paper_conf_ppopp_yehsser17_b200.pagoda import Pagoda, TRACE
+
+pytestmark = pytest.mark.gpu
+
+
+def test_init_info_shutdown():
+    with Pagoda() as p:
+        i = p.info()
+        assert i.sm_count == 148 and i.n_mtb == 296 and i.running == 1
+        assert i.regs_per_thread <= 32
+        assert p.waitAll() == 0
+    # 1 MTB per SM variant (64 registers per thread)
+    with Pagoda(mtbs_per_sm=1, arena_bytes=200 * 1024) as p:
+        assert p.info().n_mtb == 148
+        ids = p.spawn_many(1000, 128, 1, 0, False, T.NOP, None, ids=True)
+        assert p.waitAll() == 0 and all(p.check(int(i)) == 1 for i in ids[::97])
+
+
+def test_nop_many_shapes_exactly_once():
+    shapes = [(32, 1, 0, 0), (128, 1, 0, 0), (256, 1, 8192, 1), (100, 3, 600, 1), (992, 1, 0, 1), (64, 15, 0, 1),
+              (32, 31, 512, 1)]
+    with Pagoda() as p:
+        ids = []
+        for k in range(3000):
+            th, nb, sh, sy = shapes[k % len(shapes)]
+            ids.append(p.taskSpawn(th, nb, sh, sy, T.NOP))
+        assert ids == list(range(3000))
+        assert p.waitAll() == 0
+        assert all(p.check(i) == 1 for i in ids)
+        assert p.wait(1234) == 0
+        assert p.info().completed_low == 3000
+
+
+def test_lone_task_liveness():
+    """A single task with nothing spawned after it must still run (the paper
+    needs a last-task flush for this)."""
+    with Pagoda() as p:
+        time.sleep(0.05)
+        t0 = time.perf_counter()
+        tid = p.taskSpawn(128, 1, 0, False, T.NOP)
+        assert p.wait(tid) == 0
+        assert time.perf_counter() - t0 < 0.5
+
+
+def test_mark_counts_and_tid_bijection():
+    n = 400
+    shapes = [(32, 1), (96, 2), (128, 1), (100, 3), (256, 1), (40, 7), (512, 1), (992, 1)]
+    dev = Dev()
+    cap = 992 * n
+    out = dev.zeros(cap * 4)
+    cnt = dev.zeros(n * 4)
+    tids = dev.zeros(cap * 4)
+    base = np.zeros(n, np.int64)
+    b = 0
+    for k in range(n):
+        th, nb = shapes[k % len(shapes)]
+        base[k] = b
+        b += ((th + 31) // 32) * 32 * nb
+    assert b <= cap
+    with Pagoda() as p:
+        for k in range(n):
+            th, nb = shapes[k % len(shapes)]
+            a = T.records(T.MARK, 1)
+            a["out"], a["cnt"], a["base"], a["tag"] = ptr(out), ptr(cnt) + 4 * k, base[k], k + 1
+            assert p.taskSpawn(th, nb, 0, False, T.MARK, a) == 2 * k
+            t = T.records(T.TID, 1)
+            t["out"], t["base"] = ptr(tids), base[k]
+            assert p.taskSpawn(th, nb, 0, False, T.TID, t) == 2 * k + 1
+        assert p.waitAll() == 0
+    o = Dev.get(out, np.uint32)
+    c = Dev.get(cnt, np.uint32)
+    tv = Dev.get(tids, np.uint32)
+    for k in range(n):
+        th, nb = shapes[k % len(shapes)]
+        w = (th + 31) // 32
+        assert c[k] == th * nb                     # every live thread ran exactly once
+        seg = o[base[k]: base[k] + 32 * w * nb].reshape(nb, 32 * w)
+        assert (seg[:, :th] == k + 1).all() and (seg[:, th:] == 0).all()
+        ts = tv[base[k]: base[k] + 32 * w * nb].reshape(nb, 32 * w)
+        for j in range(nb):                        # getTid = (j*w + warp)*32 + lane
+            assert (ts[j, :th] == (j << 16) + np.arange(th)).all()
+
+
+def test_barrier_and_smem_isolation_under_sharing():
+    """BAR tasks (multi-phase syncBlock across warps) and SMEM tasks (fill,
+    hold, verify) share MTBs with each other and with NOP traffic: zero
+    errors means barrier IDs scope only their TB and granules never overlap."""
+    dev = Dev()
+    err = dev.zeros(8)
+    scratch = dev.zeros(4 * 992 * 15)
+    with Pagoda() as p:
+        for k in range(3000):
+            kind = k % 3
+            if kind == 0:
+                a = T.records(T.BAR, 1)
+                a["err"], a["scratch"], a["phases"] = ptr(err), ptr(scratch) + 0, 8
+                th = [64, 128, 256, 512][k % 4]
+                # shared-memory scratch (granted) so tasks do not share the global scratch
+                assert p.taskSpawn(th, 1, th * 4, True, T.BAR, a) >= 0
+            elif kind == 1:
+                a = T.records(T.SMEM, 1)
+                a["err"], a["bytes"], a["spin_ns"], a["seed"] = ptr(err) + 4, [512, 3000, 8192, 20000][k % 4], 2000, k
+                assert p.taskSpawn([32, 64, 128][k % 3], 1, int(a["bytes"][0]), True, T.SMEM, a) >= 0
+            else:
+                assert p.taskSpawn(32 * (1 + k % 8), 1, 0, False, T.NOP) >= 0
+        assert p.waitAll() == 0
+    e = Dev.get(err, np.uint32)
+    assert e[0] == 0, "barrier errors"
+    assert e[1] == 0, "shared-memory corruption / misalignment"
+
+
+def test_check_gate_semantics():
+    import torch
+    flag = torch.zeros(16, dtype=torch.int32).pin_memory()
+    with Pagoda() as p:
+        a = T.records(T.GATE, 1)
+        a["flag"] = flag.data_ptr()
+        tid = p.taskSpawn(32, 1, 0, False, T.GATE, a)
+        after = p.taskSpawn(64, 1, 0, False, T.NOP)
+        time.sleep(0.05)
+        assert p.check(tid) == 0                  # still gated
+        assert p.wait(after) == 0                 # others flow past a blocked task
+        flag[0] = 1
+        assert p.wait(tid) == 0 and p.check(tid) == 1
+        assert p.check(tid + 100) == -errno.EINVAL
+        assert p.wait(-1) == -errno.EINVAL
+
+
+def test_validation_and_shutdown_errors():
+    p = Pagoda()
+    E = -errno.EINVAL
+    assert p.taskSpawn(0, 1, 0, 0, T.NOP) == E
+    assert p.taskSpawn(993, 1, 0, 0, T.NOP) == E
+    assert p.taskSpawn(128, 8, 0, 0, T.NOP) == E
+    assert p.taskSpawn(32, 1, 96 * 1024 + 1, 0, T.NOP) == E
+    assert p.taskSpawn(128, 1, 0, 0, 99) == E
+    assert p.taskSpawn(128, 1, 0, 0, T.NOP, b"\0" * 41) == E
+    assert p.taskSpawn(992, 1, 96 * 1024, 1, T.NOP) >= 0   # a whole MTB
+    assert p.taskSpawn(32, 31, 0, 1, T.NOP) >= 0
+    assert p.shutdown() == 0
+
+
+def test_multi_producer_ids_unique():
+    n_thr, per = 4, 4000
+    got = [[] for _ in range(n_thr)]
+    with Pagoda() as p:
+        def prod(i):
+            for _ in range(per):
+                got[i].append(p.taskSpawn(64, 1, 0, False, T.NOP))
+        th = [threading.Thread(target=prod, args=(i,)) for i in range(n_thr)]
+        [t.start() for t in th]
+        [t.join() for t in th]
+        assert p.waitAll() == 0
+        for g in got:
+            assert all(b > a for a, b in zip(g, g[1:]))          # increasing per producer
+        allids = sorted(sum(got, []))
+        assert allids == list(range(n_thr * per))              # unique across producers
+
+
+def test_ring_wraparound_and_completion_window():
+    """More tasks than ring entries and completion slots: slots are reused only
+    after their previous occupant is consumed / done."""
+    with Pagoda(ring_entries=256, comp_entries=512) as p:
+        ids = p.spawn_many(20000, 64, 1, 0, False, T.NOP, None, ids=True)
+        assert p.waitAll() == 0
+        assert ids[-1] == 19999 and p.check(19999) == 1 and p.check(5) == 1
+
+
+def test_chain_visibility():
+    """Task k reads task k-1's output after a host wait (memory visibility
+    across tasks)."""
+    dev = Dev()
+    # MM with B = I copies A exactly; chain A_k = C_{k-1}, each spawned after wait(k-1)
+    eye = np.eye(32, dtype=np.float32)
+    A0 = np.arange(1024, dtype=np.float32).reshape(32, 32) / 7
+    Ibuf = dev.put(eye)
+    mats = [dev.put(A0)] + [dev.zeros(4096) for _ in range(30)]
+    with Pagoda() as p:
+        for k in range(1, 31):
+            a = T.records(T.MM, 1)
+            a["A"], a["B"], a["C"] = ptr(mats[k - 1]), ptr(Ibuf), ptr(mats[k])
+            tid = p.taskSpawn(256, 1, 8192, True, T.MM, a)
+            assert p.wait(tid) == 0
+    assert np.array_equal(Dev.get(mats[30], np.float32, (32, 32)), A0)
+
+
+def test_ledger_invariants_debug_config():
+    """Trace mode on a small grid with few executor warps and a small arena:
+    the oracle-side checker replays every MTB's allocator events (no double
+    assignment of warps / granules / barrier IDs, frees match allocs, every
+    TB allocated once on one MTB, everything freed)."""
+    import oracle
+    rng = np.random.default_rng(5)
+    alphabet = [(32, 1, 0, 0), (64, 1, 0, 1), (128, 1, 0, 1), (32, 1, 512, 0), (64, 1, 2048, 1), (128, 1, 4096, 1),
+                (32, 3, 1024, 1), (96, 2, 0, 1)]
+    dev = Dev()
+    err = dev.zeros(8)
+    n = 1500
+    with Pagoda(num_sms=2, mtbs_per_sm=1, exec_warps=8, arena_bytes=16 * 1024 + 16384, flags=TRACE,
+                trace_events=16384) as p:
+        info = p.info()
+        meta = []
+        for k in range(n):
+            th, nb, sh, sy = alphabet[rng.integers(len(alphabet))]
+            a = T.records(T.SMEM, 1)
+            a["err"], a["bytes"], a["spin_ns"], a["seed"] = ptr(err), sh, int(rng.integers(0, 3000)), k
+            tid = p.taskSpawn(th, nb, sh, sy, T.SMEM if sh else T.NOP, a if sh else None)
+            assert tid == k
+            meta.append((tid, ((th + 31) // 32) * nb, nb))
+        assert p.waitAll() == 0
+        time.sleep(0.05)      # let schedulers fold the last frees into the ledger
+        evs = np.concatenate([p.trace(m) for m in range(info.n_mtb)])
+        ex = [p.exec_trace(m, w) for m in range(info.n_mtb) for w in range(32)]
+    assert Dev.get(err, np.uint32)[0] == 0
+    tasks = np.array(meta, oracle.TASK_DTYPE)
+    granules = (16 * 1024 + 16384) // 512
+    # MTB 0 lends 32 granules to the ingest warp: checking against the full arena is the weaker bound
+    ok, msg = oracle.ledger_check(evs.view(oracle.LEDGER_DTYPE), info.n_mtb, 8, granules, 15, tasks)
+    assert ok, msg
+    # a warp never runs two tasks at once
+    for e in ex:
+        if len(e) > 1:
+            s = np.sort(e, order="t_start")
+            assert (s["t_start"][1:] >= s["t_end"][:-1]).all()
+    assert sum(len(e) for e in ex) == sum(m[1] for m in meta)
