@@ -39,6 +39,7 @@ typedef int64_t pagoda_task_t;          /* >= 0: task id; < 0: -errno */
 
 /* config flags */
 #define PAGODA_TRACE         0x1u /* record the per-MTB scheduler ledger (tests; slows scheduling) */
+#define PAGODA_NO_START      0x2u /* pagoda_init allocates but does not launch; call pagoda_start(_drain) */
 
 typedef struct {
     int      device;        /* CUDA device ordinal (default 0) */
@@ -111,6 +112,36 @@ int64_t pagoda_taskSpawnMany(pagoda_ctx* ctx, int n, int threads, int n_threadbl
  * sync_flag, func_id} (5 int32 per task). */
 int64_t pagoda_taskSpawnShapes(pagoda_ctx* ctx, int n, const int32_t* shapes, const void* args_base,
                                size_t args_stride, size_t args_bytes, pagoda_task_t* ids_out);
+
+/* ---- MasterKernel sessions ------------------------------------------------
+ * pagoda_init starts a session.  pagoda_stop waits for every issued task,
+ * asks the MasterKernel to drain and exit, and waits for it (the ring, the
+ * completion window and the ids carry over); pagoda_start launches a new
+ * session.  While stopped, other kernels can use the GPU; spawns are accepted
+ * and run at the next start; wait/waitAll on unfinished tasks return -EAGAIN.
+ * Returns 0, -EALREADY (stop: not running), -EBUSY (start: running), -EIO,
+ * -ETIMEDOUT. */
+int pagoda_stop(pagoda_ctx* ctx);
+int pagoda_start(pagoda_ctx* ctx);
+/* Start a self-terminating session: it runs every task already spawned (while
+ * stopped; at most ring_entries of them) and exits without a host signal.
+ * For tools that serialise kernel launches (Nsight Compute).  Follow with
+ * pagoda_stop to collect it. */
+int pagoda_start_drain(pagoda_ctx* ctx);
+/* Device time of the last finished session: CUDA events recorded on the
+ * MasterKernel's stream just before its launch and just after it (so the
+ * second completes when the kernel exits).  -EBUSY while a session runs. */
+int pagoda_session_ms(pagoda_ctx* ctx, float* ms);
+
+/* ---- measurement helpers (CLOCK_MONOTONIC ns) -------------------------------
+ * Spawn n tasks as pagoda_taskSpawnShapes does, recording spawn_ns[i] just
+ * before task i's spawn call, while a poller thread records done_ns[i] when
+ * check() first reports it done.  Returns n or the first error. */
+int64_t pagoda_run_timed(pagoda_ctx* ctx, int n, const int32_t* shapes, const void* args_base,
+                         size_t args_stride, size_t args_bytes, int64_t* spawn_ns, int64_t* done_ns);
+/* Closed loop, one task in flight: lat_ns[i] = spawn -> wait() return of task i. */
+int pagoda_latency_loop(pagoda_ctx* ctx, int n, int threads, int n_threadblocks, int shmem_bytes,
+                        int sync_flag, int func_id, const void* args, size_t args_bytes, int64_t* lat_ns);
 
 /* Runtime facts and counters. */
 typedef struct {

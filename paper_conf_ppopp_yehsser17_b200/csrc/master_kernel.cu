@@ -8,7 +8,7 @@
  * into the device ring.
  *
  *   host ring --(ingest: LDGSTS over PCIe -> smem -> L2 device ring)--> device ring
- *   device ring --(scheduler: speculative copy + CAS claim)--> MTB task slots
+ *   device ring --(scheduler: fetch-add tickets, per-cell sequence numbers)--> MTB task slots
  *   task slot --(place: warps / granules / barrier from bitmaps)--> WarpTable + mbarrier arrive
  *   executor warp --(body)--> mailboxes (deferred free) + completion record (D->H)
  *
@@ -92,15 +92,6 @@ __device__ __forceinline__ void st_relaxed_sys(volatile uint64_t* p, uint64_t v)
 __device__ __forceinline__ void st_relaxed_sys32(volatile uint32_t* p, uint32_t v)
 {
     asm volatile("st.relaxed.sys.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
-}
-__device__ __forceinline__ bool cas_acq_rel_gpu(uint64_t* p, uint64_t expect, uint64_t desired)
-{
-    uint64_t old;
-    asm volatile("atom.acq_rel.gpu.global.cas.b64 %0, [%1], %2, %3;"
-                 : "=l"(old)
-                 : "l"(p), "l"(expect), "l"(desired)
-                 : "memory");
-    return old == expect;
 }
 __device__ __forceinline__ void cp_async16(void* smem, const void* gmem)
 {
@@ -215,42 +206,54 @@ __device__ void executor(MtbShared& S, char* arena, const MkParams& p, int mtb, 
  * Replaces the paper's one-cudaMemcpy-per-spawn with ready-field pipelining
  * (P:516-539): the host publishes a doorbell after writing entries; this warp
  * acquires it over PCIe, pulls the entries with asynchronous 16-byte copies
- * (many in flight, no registers held) into shared memory, writes them to the
- * device ring and releases the device tail. */
+ * (many in flight, no registers held) into shared memory and publishes them
+ * into the device ring, a bounded MPMC queue with one sequence word per cell:
+ * the producer may fill the cell of position t once seq == t (its previous
+ * occupant was consumed), then releases seq = t + 1. */
 constexpr int kIngestBatch = 256;                       /* entries per round (16 KiB staging) */
 constexpr uint32_t kIngestStageBytes = kIngestBatch * 64;
 
 __device__ void ingest(const MkParams& p, char* stage_buf)
 {
     const uint32_t lane = threadIdx.x & 31u;
-    const uint64_t R = (uint64_t)p.ring_mask + 1;
-    uint64_t copied = 0;
+    uint64_t copied = *(volatile uint64_t*)&p.dctl->tail;   /* resumes after a stop/start */
     uint32_t last_err = 0;
     int idle = 0;
     for (;;) {
-        uint64_t pub = 0, head = 0;
+        uint64_t pub = 0;
         uint32_t term = 0, err = 0;
         if (lane == 0) {
             pub = ld_acquire_sys(&p.hctl->published);
             term = ld_relaxed_sys32(&p.hctl->terminate);
-            head = ld_acquire_gpu(&p.dctl->head);
             err = *(volatile uint32_t*)&p.dctl->error;
             if (err != last_err) st_relaxed_sys32(&p.hctl->error, err);
         }
         pub = __shfl_sync(0xffffffffu, pub, 0);
         term = __shfl_sync(0xffffffffu, term, 0);
-        head = __shfl_sync(0xffffffffu, head, 0);
         last_err = __shfl_sync(0xffffffffu, err, 0);
+        if (term == kStopAbort) {   /* host watchdog: abandon the queue, let idle MTBs exit */
+            if (lane == 0) st_release_gpu32(&p.dctl->stop, kStopAbort);
+            return;
+        }
         if (pub > copied) {
-            uint64_t n = pub - copied;
-            const uint64_t space = R - (copied - head);
-            if (n > space) n = space;
-            if (n > (uint64_t)kIngestBatch) n = kIngestBatch;
+            uint32_t n = (uint32_t)min(pub - copied, (uint64_t)kIngestBatch);
+            /* free cells: the longest prefix whose previous occupant was consumed */
+            uint32_t ready = n;
+            for (uint32_t base = 0; base < n; base += 32u) {
+                const uint64_t t = copied + base + lane;
+                const bool ok = base + lane >= n || ld_acquire_gpu(&p.dseq[t & p.ring_mask]) == t;
+                const uint32_t bad = __ballot_sync(0xffffffffu, !ok);
+                if (bad) {
+                    ready = base + (uint32_t)__ffs(bad) - 1u;
+                    break;
+                }
+            }
+            n = ready;
             if (n == 0) {              /* device ring full: wait for the schedulers */
-                __nanosleep(200);
+                __nanosleep(128);
                 continue;
             }
-            const uint32_t chunks = (uint32_t)n * 4u;
+            const uint32_t chunks = n * 4u;
             for (uint32_t c = lane; c < chunks; c += 32u) {
                 const uint64_t e = (copied + (c >> 2)) & p.ring_mask;
                 cp_async16(stage_buf + c * 16u, reinterpret_cast<const int4*>(p.hring + e) + (c & 3u));
@@ -262,10 +265,15 @@ __device__ void ingest(const MkParams& p, char* stage_buf)
                 const int4 v = *reinterpret_cast<const int4*>(stage_buf + c * 16u);
                 __stcg(reinterpret_cast<int4*>(p.dring + e) + (c & 3u), v);
             }
+            __syncwarp();   /* every lane's entry stores precede each cell's release */
+            for (uint32_t i = lane; i < n; i += 32u) {
+                const uint64_t t = copied + i;
+                st_release_gpu(&p.dseq[t & p.ring_mask], t + 1);
+            }
             __syncwarp();
             copied += n;
             if (lane == 0) {
-                st_release_gpu(&p.dctl->tail, copied);   /* entries before the tail are complete */
+                st_release_gpu(&p.dctl->tail, copied);     /* hint for schedulers: work exists */
                 st_relaxed_sys(&p.hctl->consumed, copied); /* host may now reuse those ring slots */
             }
             idle = 0;
@@ -281,13 +289,16 @@ __device__ void ingest(const MkParams& p, char* stage_buf)
 /* ------------------------------------------------------------------ scheduler
  * Alg. 1 L1-28 + Alg. 2, re-designed: one warp per MTB owns the
  * MTB's free masks (warps, TB records, task slots, barrier IDs: one word each;
- * granules: a 1024-bit lane-distributed bitmap).  It claims entries from the
- * device ring only while it has free resources, in ring order, so tasks flow
- * to whichever MTB frees resources first. */
+ * granules: a 1024-bit lane-distributed bitmap).  It takes TICKETS (ring
+ * positions) with one fetch-add on the device head, as many as its free warps
+ * fit at the last task size seen, so no claim ever fails or retries; a ticket
+ * is loaded into a task slot once its cell is published, and placed in FIFO
+ * order as soon as the MTB has the resources. */
 struct Sched {
     uint32_t free_w, free_task, free_tbs, free_bar, exec_mask;
     uint32_t fg;         /* this lane's 32 granule bits */
-    uint32_t ph, pt;     /* pending FIFO of claimed, unplaced task slots */
+    uint32_t ph, pl, pt; /* FIFO: [ph,pl) loaded task slots, [pl,pt) tickets not yet loaded */
+    uint32_t est_w;      /* warps of the last loaded task (0 = none yet) */
     uint32_t seq;        /* ledger clock */
 };
 
@@ -368,13 +379,21 @@ __device__ bool sched_place(MtbShared& S, Sched& st, const MkParams& p, int mtb,
     return true;
 }
 
-/* Claim up to 32 entries at the device ring head that fit the free resources.
- * Entries are copied into free task slots BEFORE the CAS that claims them:
- * until the CAS succeeds no scheduler owns them, so the ingest warp cannot
- * have recycled their ring slots (it only reuses slots below the head). */
+/* Take tickets: as many tasks as the free warps fit at the last task size
+ * (one ticket when the size is unknown), never more than the ring holds. */
 __device__ int sched_claim(MtbShared& S, Sched& st, const MkParams& p)
 {
     const uint32_t lane = threadIdx.x & 31u;
+    const uint32_t queued = st.pt - st.ph;
+    const uint32_t cap = 32u - queued;
+    uint32_t want;
+    if (st.est_w == 0) want = queued == 0 ? 1u : 0u;
+    else {
+        want = (uint32_t)__popc(st.free_w) / st.est_w;
+        want = want > queued ? want - queued : 0u;
+    }
+    want = min(want, cap);
+    if (want == 0) return 0;
     uint64_t head = 0, tail = 0;
     if (lane == 0) {
         head = ld_relaxed_gpu(&p.dctl->head);
@@ -383,51 +402,53 @@ __device__ int sched_claim(MtbShared& S, Sched& st, const MkParams& p)
     head = __shfl_sync(0xffffffffu, head, 0);
     tail = __shfl_sync(0xffffffffu, tail, 0);
     if (head >= tail) return 0;
-    uint32_t n = (uint32_t)min((uint64_t)32, tail - head);
-    n = min(n, (uint32_t)__popc(st.free_task));
-    n = min(n, 32u - (st.pt - st.ph));
-    if (n == 0) return 0;
-    /* speculative copy: 4 x 16 B per entry, L2 only (the slot may hold an older lap in L1) */
-    for (uint32_t c = lane; c < n * 4u; c += 32u) {
-        const uint32_t i = c >> 2;
-        const TaskEntry* src = p.dring + ((head + i) & p.ring_mask);
-        const int4 v = __ldcg(reinterpret_cast<const int4*>(src) + (c & 3u));
-        reinterpret_cast<int4*>(&S.tasks[nth_set_bit(st.free_task, i)])[c & 3u] = v;
-    }
-    __syncwarp();
-    /* needs of entry `lane`; inclusive prefix sums over the lanes */
-    uint32_t nw = 0, nt = 0, nb = 0, ng = 0, my_slot = 0;
-    if (lane < n) {
-        my_slot = nth_set_bit(st.free_task, lane);
-        const TaskEntry& e = S.tasks[my_slot];
-        nw = (uint32_t)e.warps_tb * e.n_tb;
-        nt = e.n_tb;
-        nb = ((e.flags & 1u) && e.warps_tb > 1) ? e.n_tb : 0;
-        ng = (uint32_t)e.gran_tb * e.n_tb;
-    }
-#pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-        const uint32_t a = __shfl_up_sync(0xffffffffu, nw, d), b = __shfl_up_sync(0xffffffffu, nt, d);
-        const uint32_t c = __shfl_up_sync(0xffffffffu, nb, d), g = __shfl_up_sync(0xffffffffu, ng, d);
-        if (lane >= (uint32_t)d) { nw += a; nt += b; nb += c; ng += g; }
-    }
-    const uint32_t free_g = __reduce_add_sync(0xffffffffu, (uint32_t)__popc(st.fg));
-    const bool fit = lane < n && nw <= (uint32_t)__popc(st.free_w) && nt <= (uint32_t)__popc(st.free_tbs) &&
-                     nb <= (uint32_t)__popc(st.free_bar) && ng <= free_g;
-    const uint32_t fb = __ballot_sync(0xffffffffu, fit);
-    const uint32_t k = (fb == 0xffffffffu) ? 32u : (uint32_t)(__ffs(~fb) - 1);
-    if (k == 0) return 0;
-    bool ok = false;
-    if (lane == 0) ok = cas_acq_rel_gpu(&p.dctl->head, head, head + k);
-    ok = __shfl_sync(0xffffffffu, (int)ok, 0) != 0;
-    if (!ok) return -1;
-    if (lane < k) S.pend[(st.pt + lane) & 31u] = (uint8_t)my_slot;
-    uint32_t used = 0;
-    for (uint32_t i = 0; i < k; i++) used |= 1u << nth_set_bit(st.free_task, i);
-    st.free_task &= ~used;
+    const uint32_t k = (uint32_t)min((uint64_t)want, tail - head);
+    unsigned long long t0 = 0;
+    if (lane == 0) t0 = atomicAdd(reinterpret_cast<unsigned long long*>(&p.dctl->head), (unsigned long long)k);
+    t0 = __shfl_sync(0xffffffffu, t0, 0);
+    if (lane < k) S.pend_ticket[(st.pt + lane) & 31u] = t0 + lane;
     st.pt += k;
     __syncwarp();
     return (int)k;
+}
+
+/* Load the published tickets at the front of the FIFO into free task slots,
+ * then hand their cells back to the producer (seq = t + R). */
+__device__ int sched_load(MtbShared& S, Sched& st, const MkParams& p)
+{
+    const uint32_t lane = threadIdx.x & 31u;
+    const uint32_t n = min(st.pt - st.pl, (uint32_t)__popc(st.free_task));
+    if (n == 0) return 0;
+    uint64_t t = 0;
+    bool ready = false;
+    if (lane < n) {
+        t = S.pend_ticket[(st.pl + lane) & 31u];
+        ready = ld_acquire_gpu(&p.dseq[t & p.ring_mask]) == t + 1;
+    }
+    const uint32_t nr = __ballot_sync(0xffffffffu, !ready);
+    const uint32_t r = nr ? (uint32_t)__ffs(nr) - 1u : 32u;   /* leading published tickets */
+    if (r == 0) return 0;
+    for (uint32_t c = lane; c < r * 4u; c += 32u) {
+        const uint32_t i = c >> 2;
+        const uint64_t ti = S.pend_ticket[(st.pl + i) & 31u];
+        const int4 v = __ldcg(reinterpret_cast<const int4*>(p.dring + (ti & p.ring_mask)) + (c & 3u));
+        reinterpret_cast<int4*>(&S.tasks[nth_set_bit(st.free_task, i)])[c & 3u] = v;
+    }
+    __syncwarp();   /* all copies (loads) precede the release of each cell */
+    uint32_t used = 0;
+    if (lane < r) {
+        const uint32_t slot = nth_set_bit(st.free_task, lane);
+        S.pend[(st.pl + lane) & 31u] = (uint8_t)slot;
+        st_release_gpu(&p.dseq[t & p.ring_mask], t + (uint64_t)p.ring_mask + 1);
+        used = 1u << slot;
+    }
+    used = __reduce_or_sync(0xffffffffu, used);
+    st.free_task &= ~used;
+    st.pl += r;
+    __syncwarp();
+    const TaskEntry& last = S.tasks[S.pend[(st.pl - 1) & 31u]];
+    st.est_w = (uint32_t)last.warps_tb * last.n_tb;
+    return (int)r;
 }
 
 __device__ void scheduler(MtbShared& S, const MkParams& p, int mtb, int arena_granules)
@@ -442,7 +463,8 @@ __device__ void scheduler(MtbShared& S, const MkParams& p, int mtb, int arena_gr
     st.free_tbs = 0xffffffffu;
     st.free_bar = 0xfffeu;        /* named barriers 1..15; 0 belongs to the MTB */
     st.fg = bm_range_bits(0, (uint32_t)arena_granules, lane);
-    st.ph = st.pt = 0;
+    st.ph = st.pl = st.pt = 0;
+    st.est_w = 0;
     st.seq = 0;
     uint32_t backoff = 0;
     for (;;) {
@@ -479,33 +501,33 @@ __device__ void scheduler(MtbShared& S, const MkParams& p, int mtb, int arena_gr
             st.free_w |= mw;
             st.free_task |= mk;
         }
-        /* ---- place claimed tasks in FIFO order (Alg. 1 L14-28) */
-        while (st.ph != st.pt) {
+        /* ---- load published tickets, place loaded tasks in FIFO order (Alg. 1 L14-28) */
+        if (st.pl != st.pt && sched_load(S, st, p) > 0) progress = true;
+        while (st.ph != st.pl) {
             if (!sched_place(S, st, p, mtb, S.pend[st.ph & 31u])) break;
             st.ph++;
             progress = true;
         }
-        /* ---- claim more while resources are free */
-        if (st.ph == st.pt && st.free_w && st.free_task) {
-            const int k = sched_claim(S, st, p);
-            if (k != 0) progress = true;   /* k < 0: lost a CAS race; retry at once */
-        }
+        /* ---- take more tickets while resources are free.  MTB 0 (one warp short: it hosts the
+         * ingest warp) does not take blind tickets unless it is the only MTB (validation then
+         * caps every task to its capacity), so no ticket can land where it never fits. */
+        if (st.free_w && (mtb != 0 || p.n_mtb == 1) && sched_claim(S, st, p) > 0) progress = true;
         if (progress) {
             backoff = 0;
             continue;
         }
-        /* ---- idle */
-        if (st.free_w == st.exec_mask && st.ph == st.pt) {
+        /* ---- idle: exit once stopped, drained, and holding no ticket that can still be published */
+        {
             uint32_t stop = 0;
             if (lane == 0) stop = ld_acquire_gpu32(&p.dctl->stop);
             stop = __shfl_sync(0xffffffffu, stop, 0);
-            if (stop) {
-                uint64_t head = 0, tail = 0;
-                if (lane == 0) {
-                    head = ld_relaxed_gpu(&p.dctl->head);
-                    tail = ld_acquire_gpu(&p.dctl->tail);
-                }
-                if (__shfl_sync(0xffffffffu, (int)(head >= tail), 0)) break;
+            if (stop == kStopAbort && st.free_w == st.exec_mask) break;   /* host watchdog gave up */
+            if (stop && st.free_w == st.exec_mask && st.ph == st.pl) {
+                uint64_t tail = 0;
+                if (lane == 0) tail = ld_acquire_gpu(&p.dctl->tail);
+                tail = __shfl_sync(0xffffffffu, tail, 0);
+                /* after stop the tail is final: tickets at or past it are void */
+                if (st.pl == st.pt || S.pend_ticket[st.pl & 31u] >= tail) break;
             }
         }
         backoff = backoff ? min(backoff * 2u, 1024u) : 32u;

@@ -42,8 +42,8 @@ struct HostCtl {
 
 /* device memory, L2-resident: the device ring's counters */
 struct DevCtl {
-    alignas(128) uint64_t tail;    /* entries published into the device ring (ingest warp) */
-    alignas(128) uint64_t head;    /* entries claimed by schedulers (CAS) */
+    alignas(128) uint64_t tail;    /* entries published into the device ring (ingest warp; a hint) */
+    alignas(128) uint64_t head;    /* tickets handed out to schedulers (fetch-add) */
     alignas(128) uint32_t stop;    /* set by ingest after terminate: schedulers drain and exit */
     alignas(128) uint32_t error;   /* device error word (executors atomicOr) */
     alignas(128) uint32_t exited;  /* MTBs that exited */
@@ -79,6 +79,8 @@ struct MkParams {
     HostCtl*         hctl;    /* pinned host control (mapped) */
     int64_t*         comp;    /* pinned completion window (mapped) */
     TaskEntry*       dring;   /* device ring */
+    uint64_t*        dseq;    /* per-cell sequence numbers (bounded MPMC queue): cell of position t holds
+                                 t (free for the producer), t+1 (entry t published), t+R (entry t consumed) */
     DevCtl*          dctl;
     uint32_t ring_mask;
     uint32_t comp_mask;
@@ -93,6 +95,7 @@ struct MkParams {
 };
 
 constexpr int kIngestWarp = 31;          /* warp 31 of MTB 0 feeds the device ring */
+constexpr uint32_t kStopAbort = 2;       /* HostCtl.terminate / DevCtl.stop value: abandon work and exit */
 constexpr int kMaxGranules = 1024;       /* lane-distributed bitmap: 32 lanes x 32 bits */
 
 /* Per-MTB control block at the start of dynamic shared memory (P:456-458:
@@ -114,6 +117,7 @@ struct MtbShared {
     uint32_t  pad_;
     uint64_t  tb_task[32];           /* 4048: task id of each TB record (ledger) */
     uint16_t  tb_idx[32];            /* 4304: TB index j of each TB record (ledger) */
+    uint64_t  pend_ticket[32];       /* 4368: claimed ring positions, FIFO (pend[] holds their slots once loaded) */
 };
 static_assert(offsetof(MtbShared, wt) == kWarpTableOffset, "WarpTable offset");
 static_assert(sizeof(MtbShared) <= kArenaOffset, "control block fits below the arena");

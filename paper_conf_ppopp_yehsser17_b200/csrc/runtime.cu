@@ -55,6 +55,7 @@ struct pagoda_ctx {
     volatile int64_t* comp = nullptr;
     /* device */
     TaskEntry* dring = nullptr;
+    uint64_t* dseq = nullptr;
     DevCtl* dctl = nullptr;
     LedgerEvent* trace = nullptr;
     uint32_t* trace_count = nullptr;
@@ -70,6 +71,13 @@ struct pagoda_ctx {
     std::atomic<int> faulted{0};
     std::vector<int64_t> warps_prefix;      /* warps_prefix[id mod C] = sum of warps of tasks <= id */
     std::atomic<int64_t> warps_spawned{0};
+    /* MasterKernel session */
+    MkParams params;
+    size_t smem = 0;
+    cudaEvent_t ev_start = nullptr, ev_stop = nullptr;
+    std::atomic<int> running{0};
+    std::mutex session_mtx;
+    int sessions = 0;
 };
 
 /* ------------------------------------------------------------------ helpers */
@@ -101,13 +109,12 @@ static int spin_until(pagoda_ctx* c, Pred pred)
         if (t - last_check > 1000000ull) {
             last_check = t;
             if (c->hctl->error) return -EIO;
-            if (!c->shutting.load(std::memory_order_relaxed) || true) {
-                cudaError_t q = cudaStreamQuery(c->stream);
-                if (q != cudaErrorNotReady) {   /* MasterKernel gone (fault or exited) */
-                    if (pred()) return 0;
-                    c->faulted.store(1);
-                    return -EIO;
-                }
+            if (!c->running.load(std::memory_order_acquire)) return pred() ? 0 : -EAGAIN;   /* stopped */
+            cudaError_t q = cudaStreamQuery(c->stream);
+            if (q != cudaErrorNotReady) {   /* MasterKernel gone while it should run: fault */
+                if (pred()) return 0;
+                c->faulted.store(1);
+                return -EIO;
             }
             if (c->cfg.watchdog_s > 0 && (double)(t - t0) * 1e-9 > c->cfg.watchdog_s) return -ETIMEDOUT;
         }
@@ -144,6 +151,72 @@ void pagoda_config_default(pagoda_config* cfg)
 
 static bool pow2(uint32_t x) { return x && !(x & (x - 1)); }
 
+/* Launch one MasterKernel session on the context's stream, bracketed by CUDA
+ * events recorded before and after the launch (ev_stop completes at kernel exit). */
+static int start_kernel(pagoda_ctx* c)
+{
+    cudaSetDevice(c->device);
+    if (c->trace_count) {
+        cudaMemsetAsync(c->trace_count, 0, (size_t)c->n_mtb * sizeof(uint32_t), c->stream);
+        cudaMemsetAsync(c->exec_count, 0, (size_t)c->n_mtb * 32 * sizeof(uint32_t), c->stream);
+    }
+    cudaEventRecord(c->ev_start, c->stream);
+    cudaError_t e = launch_master(c->cfg.mtbs_per_sm, c->n_mtb, c->smem, c->stream, &c->params, &c->regs);
+    if (e != cudaSuccess) {
+        fprintf(stderr, "pagoda: MasterKernel launch failed: %s\n", cudaGetErrorString(e));
+        cudaGetLastError();
+        return -EIO;
+    }
+    cudaEventRecord(c->ev_stop, c->stream);   /* completes when the session's kernel exits */
+    c->running.store(1, std::memory_order_release);
+    c->sessions++;
+    return 0;
+}
+
+/* Ask the running session to drain and exit; wait (bounded) for it. */
+static int stop_kernel(pagoda_ctx* c, bool abort_now = false)
+{
+    c->hctl->terminate = abort_now ? kStopAbort : 1;
+    const uint64_t t0 = now_ns();
+    cudaError_t q;
+    bool aborted = abort_now;
+    while ((q = cudaStreamQuery(c->stream)) == cudaErrorNotReady) {
+        std::this_thread::sleep_for(std::chrono::microseconds(20));
+        const double waited = (double)(now_ns() - t0) * 1e-9;
+        if (!aborted && c->cfg.watchdog_s > 0 && waited > c->cfg.watchdog_s) {
+            /* abandon the queue: idle MTBs exit, tasks still running are waited for a while */
+            fprintf(stderr, "pagoda: MasterKernel did not drain (watchdog): aborting the session\n");
+            c->hctl->terminate = kStopAbort;
+            aborted = true;
+        }
+        if (aborted && waited > c->cfg.watchdog_s + 10.0) {
+            fprintf(stderr, "pagoda: MasterKernel did not exit after abort\n");
+            return -ETIMEDOUT;   /* still resident: buffers must not be freed */
+        }
+    }
+    c->running.store(0, std::memory_order_release);
+    if (aborted) {
+        c->faulted.store(1);
+        return -ETIMEDOUT;
+    }
+    if (q != cudaSuccess) {
+        fprintf(stderr, "pagoda: MasterKernel error: %s\n", cudaGetErrorString(q));
+        c->faulted.store(1);
+        return -EIO;
+    }
+    /* reset the session flags for the next start; ring positions carry over,
+     * except tickets handed out past the final tail, which are void: head = tail */
+    c->hctl->terminate = 0;
+    const uint32_t zero = 0;
+    uint64_t tail = 0;
+    cudaMemcpy(&tail, &c->dctl->tail, 8, cudaMemcpyDeviceToHost);
+    cudaMemcpy(&c->dctl->head, &tail, 8, cudaMemcpyHostToDevice);
+    cudaMemcpy(&c->dctl->stop, &zero, 4, cudaMemcpyHostToDevice);
+    cudaMemcpy(&c->dctl->exited, &zero, 4, cudaMemcpyHostToDevice);
+    if (cudaStreamSynchronize(c->stream) != cudaSuccess) return -EIO;
+    return c->hctl->error ? -EIO : 0;
+}
+
 static void free_ctx(pagoda_ctx* c)
 {
     if (!c) return;
@@ -151,6 +224,7 @@ static void free_ctx(pagoda_ctx* c)
     if (c->hring) cudaFreeHost(c->hring);
     if (c->comp) cudaFreeHost((void*)c->comp);
     if (c->dring) cudaFree(c->dring);
+    if (c->dseq) cudaFree(c->dseq);
     if (c->dctl) cudaFree(c->dctl);
     if (c->trace) cudaFree(c->trace);
     if (c->trace_count) cudaFree(c->trace_count);
@@ -220,6 +294,13 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
         goto fail;
     for (uint32_t i = 0; i < c->C; i++) c->comp[i] = -1;
     if (cudaMalloc(&c->dring, (size_t)c->R * sizeof(TaskEntry)) != cudaSuccess) goto fail;
+    if (cudaMalloc(&c->dseq, (size_t)c->R * sizeof(uint64_t)) != cudaSuccess) goto fail;
+    {   /* cell i starts free for position i */
+        std::vector<uint64_t> seq(c->R);
+        for (uint32_t i = 0; i < c->R; i++) seq[i] = i;
+        if (cudaMemcpy(c->dseq, seq.data(), seq.size() * sizeof(uint64_t), cudaMemcpyHostToDevice) != cudaSuccess)
+            goto fail;
+    }
     if (cudaMalloc(&c->dctl, sizeof(DevCtl)) != cudaSuccess) goto fail;
     if (cudaMemset(c->dctl, 0, sizeof(DevCtl)) != cudaSuccess) goto fail;
     if (cfg.flags & PAGODA_TRACE) {
@@ -233,9 +314,10 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
         cudaMemset(c->exec_count, 0, (size_t)c->n_mtb * 32 * sizeof(uint32_t));
     }
     if (cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking) != cudaSuccess) goto fail;
+    if (cudaEventCreate(&c->ev_start) != cudaSuccess || cudaEventCreate(&c->ev_stop) != cudaSuccess) goto fail;
     if (cudaDeviceSynchronize() != cudaSuccess) goto fail;
     {
-        MkParams p;
+        MkParams& p = c->params;
         memset(&p, 0, sizeof p);
         void* dptr = nullptr;
         cudaHostGetDevicePointer(&dptr, (void*)c->hring, 0);
@@ -245,6 +327,7 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
         cudaHostGetDevicePointer(&dptr, (void*)c->comp, 0);
         p.comp = (int64_t*)dptr;
         p.dring = c->dring;
+        p.dseq = c->dseq;
         p.dctl = c->dctl;
         p.ring_mask = c->R - 1;
         p.comp_mask = c->C - 1;
@@ -258,13 +341,9 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
             p.exec_trace = c->exec_trace;
             p.exec_count = c->exec_count;
         }
-        cudaError_t e = launch_master(cfg.mtbs_per_sm, c->n_mtb, smem, c->stream, &p, &c->regs);
-        if (e != cudaSuccess) {
-            fprintf(stderr, "pagoda_init: MasterKernel launch failed: %s\n", cudaGetErrorString(e));
-            cudaGetLastError();
-            rc = -EIO;
-            goto fail;
-        }
+        c->smem = smem;
+        rc = (cfg.flags & PAGODA_NO_START) ? 0 : start_kernel(c);
+        if (rc) goto fail;
     }
     *out = c;
     return 0;
@@ -401,29 +480,61 @@ int pagoda_waitAll(pagoda_ctx* c)
     return rc;
 }
 
+int pagoda_stop(pagoda_ctx* c)
+{
+    if (!c) return -EINVAL;
+    std::lock_guard<std::mutex> lk(c->session_mtx);
+    if (!c->running.load()) return -EALREADY;
+    int rc = c->faulted.load() ? -EIO : pagoda_waitAll(c);
+    int r2 = stop_kernel(c);
+    return rc ? rc : r2;
+}
+
+int pagoda_start(pagoda_ctx* c)
+{
+    if (!c) return -EINVAL;
+    std::lock_guard<std::mutex> lk(c->session_mtx);
+    if (c->shutting.load() || c->faulted.load()) return -EIO;
+    if (c->running.load()) return -EBUSY;
+    return start_kernel(c);
+}
+
+int pagoda_start_drain(pagoda_ctx* c)
+{
+    if (!c) return -EINVAL;
+    std::lock_guard<std::mutex> lk(c->session_mtx);
+    if (c->shutting.load() || c->faulted.load()) return -EIO;
+    if (c->running.load()) return -EBUSY;
+    c->hctl->terminate = 1;   /* the session exits once everything already published is done */
+    return start_kernel(c);
+}
+
+int pagoda_session_ms(pagoda_ctx* c, float* ms)
+{
+    if (!c || !ms) return -EINVAL;
+    if (c->running.load() || c->sessions == 0) return -EBUSY;
+    return cudaEventElapsedTime(ms, c->ev_start, c->ev_stop) == cudaSuccess ? 0 : -EIO;
+}
+
 int pagoda_shutdown(pagoda_ctx* c)
 {
     if (!c) return -EINVAL;
     int rc = 0;
-    if (!c->faulted.load()) rc = pagoda_waitAll(c);
-    c->shutting.store(1, std::memory_order_release);
-    c->hctl->terminate = 1;
-    /* the MasterKernel drains and exits: wait for the stream (bounded) */
-    const uint64_t t0 = now_ns();
-    cudaError_t q;
-    while ((q = cudaStreamQuery(c->stream)) == cudaErrorNotReady) {
-        std::this_thread::sleep_for(std::chrono::microseconds(50));
-        if (c->cfg.watchdog_s > 0 && (double)(now_ns() - t0) * 1e-9 > c->cfg.watchdog_s) {
-            fprintf(stderr, "pagoda_shutdown: MasterKernel did not exit (watchdog)\n");
-            return -ETIMEDOUT;   /* leak: freeing live buffers would fault the kernel */
+    {
+        std::lock_guard<std::mutex> lk(c->session_mtx);
+        if (c->running.load()) {
+            if (!c->faulted.load()) rc = pagoda_waitAll(c);
+            c->shutting.store(1, std::memory_order_release);
+            const int r2 = stop_kernel(c, rc != 0 || c->faulted.load());
+            if (c->running.load()) return r2;   /* still resident: freeing live buffers would fault it */
+            if (!rc) rc = r2;
         }
-    }
-    if (q != cudaSuccess) {
-        fprintf(stderr, "pagoda_shutdown: MasterKernel error: %s\n", cudaGetErrorString(q));
-        rc = -EIO;
+        c->shutting.store(1, std::memory_order_release);
     }
     if (c->hctl->error && rc == 0) rc = -EIO;
     cudaSetDevice(c->device);
+    if (c->ev_start) cudaEventDestroy(c->ev_start);
+    if (c->ev_stop) cudaEventDestroy(c->ev_stop);
     free_ctx(c);
     return rc;
 }

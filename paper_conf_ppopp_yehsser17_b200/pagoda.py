@@ -17,6 +17,7 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(PKG, "libpagoda.so")
 
 TRACE = 0x1
+NO_START = 0x2
 
 
 class pagoda_config(C.Structure):
@@ -83,6 +84,13 @@ def lib() -> C.CDLL:
         L.pagoda_inflight_warps.restype = I64
         L.pagoda_pick_least_loaded.argtypes = [P, I]
         L.pagoda_version.restype = C.c_char_p
+        L.pagoda_stop.argtypes = [P]
+        L.pagoda_start.argtypes = [P]
+        L.pagoda_start_drain.argtypes = [P]
+        L.pagoda_session_ms.argtypes = [P, C.POINTER(C.c_float)]
+        L.pagoda_run_timed.argtypes = [P, I, P, P, SZ, SZ, P, P]
+        L.pagoda_run_timed.restype = I64
+        L.pagoda_latency_loop.argtypes = [P, I, I, I, I, I, I, P, SZ, P]
         _lib = L
     return _lib
 
@@ -160,6 +168,39 @@ class Pagoda:
                                           _ptr(out))
         _check(rc, "pagoda_taskSpawnShapes")
         return out
+
+    # --- sessions ------------------------------------------------------------
+    def stop(self) -> int:
+        return lib().pagoda_stop(self.h)
+
+    def start(self) -> int:
+        return lib().pagoda_start(self.h)
+
+    def start_drain(self) -> int:
+        return lib().pagoda_start_drain(self.h)
+
+    def session_ms(self) -> float:
+        ms = C.c_float(0)
+        _check(lib().pagoda_session_ms(self.h, C.byref(ms)), "pagoda_session_ms")
+        return ms.value
+
+    # --- measurement ---------------------------------------------------------
+    def run_timed(self, shapes: np.ndarray, args: np.ndarray):
+        """Spawn all; returns (spawn_ns, done_ns) int64 arrays (CLOCK_MONOTONIC)."""
+        shapes = np.ascontiguousarray(shapes, np.int32)
+        args = np.ascontiguousarray(args, np.uint8)
+        n = len(shapes)
+        sp, dn = np.zeros(n, np.int64), np.zeros(n, np.int64)
+        _check(lib().pagoda_run_timed(self.h, n, _ptr(shapes), _ptr(args), args.shape[1], args.shape[1],
+                                      _ptr(sp), _ptr(dn)), "pagoda_run_timed")
+        return sp, dn
+
+    def latency_loop(self, n, threads, n_tb, shmem, sync, func_id, args=None) -> np.ndarray:
+        lat = np.zeros(n, np.int64)
+        b = (args.tobytes() if isinstance(args, np.ndarray) else bytes(args)) if args is not None else None
+        _check(lib().pagoda_latency_loop(self.h, n, threads, n_tb, shmem, int(sync), func_id, b,
+                                         len(b) if b else 0, _ptr(lat)), "pagoda_latency_loop")
+        return lat
 
     def info(self) -> pagoda_info:
         i = pagoda_info()

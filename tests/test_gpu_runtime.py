@@ -236,3 +236,34 @@ def test_ledger_invariants_debug_config():
             s = np.sort(e, order="t_start")
             assert (s["t_start"][1:] >= s["t_end"][:-1]).all()
     assert sum(len(e) for e in ex) == sum(m[1] for m in meta)
+
+
+def test_sessions_stop_start_and_drain():
+    """pagoda_stop / pagoda_start keep ring positions and ids; a drain session
+    runs everything spawned while stopped and exits by itself; every task still
+    completes exactly once (MARK counters)."""
+    from paper_conf_ppopp_yehsser17_b200.pagoda import NO_START
+    dev = Dev()
+    n = 6000
+    cnt = dev.zeros(4 * n)
+    out = dev.zeros(4 * 64 * n)
+    a = T.records(T.MARK, n)
+    a["out"], a["cnt"] = ptr(out), ptr(cnt) + 4 * np.arange(n)
+    a["base"], a["tag"] = 64 * np.arange(n), np.arange(n) + 1
+    with Pagoda(flags=NO_START) as p:
+        ids = p.spawn_many(2000, 64, 1, 0, False, T.MARK, a[:2000], ids=True)   # while stopped
+        assert p.check(int(ids[-1])) == 0
+        assert p.start_drain() == 0
+        assert p.stop() == 0
+        assert p.check(int(ids[-1])) == 1 and p.session_ms() > 0
+        for s in range(2):
+            assert p.start() == 0
+            lo = 2000 + 2000 * s
+            ids = p.spawn_many(2000, 64, 1, 0, False, T.MARK, a[lo:lo + 2000], ids=True)
+            assert p.stop() == 0
+            assert all(p.check(int(i)) == 1 for i in ids[::97])
+        assert p.start() == 0
+    c = Dev.get(cnt, np.uint32)
+    assert (c == 64).all()
+    o = Dev.get(out, np.uint32).reshape(n, 64)
+    assert (o == (np.arange(n) + 1)[:, None]).all()
