@@ -58,6 +58,9 @@ def parse():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--quick", action="store_true", help="skip everything but the timed steps (for ncu)")
+    ap.add_argument("--mtbs", type=int, default=0, help="MTBs per SM (default: the workload preset)")
+    ap.add_argument("--arena-kb", type=int, default=0, help="task arena per MTB in KiB (default: preset)")
+    ap.add_argument("--no-resident", action="store_true", help="3DES: stage SP tables per task instead")
     ap.add_argument("--prespawn", action="store_true",
                     help="spawn a step's tasks before launching a self-draining session (ncu-compatible)")
     return ap.parse_args()
@@ -217,10 +220,10 @@ def workload_config(name):
     }[name]
 
 
-def make_workload(name):
+def make_workload(name, resident=False):
     from paper_conf_ppopp_yehsser17_b200 import workloads as W
-    if name == "tdes":
-        return W.tdes(32768)
+    if name == "tdes":   # with resident SP tables a task only stages its 384 B of round keys
+        return W.tdes(32768, shmem=512 if resident else 2560)
     if name == "mb":
         return W.mandelbrot(1024)
     if name == "mm":
@@ -228,6 +231,28 @@ def make_workload(name):
     if name == "mix":
         return W.mix(32768)
     return W.nop(200000)
+
+
+# per-workload context presets
+PRESETS = {
+    "tdes": {"mtbs_per_sm": 2, "arena_bytes": 40 * 1024, "resident": True},
+    "mb": {"mtbs_per_sm": 2, "arena_bytes": 96 * 1024, "resident": False},
+    "mm": {"mtbs_per_sm": 2, "arena_bytes": 96 * 1024, "resident": False},
+    "mix": {"mtbs_per_sm": 2, "arena_bytes": 96 * 1024, "resident": False},
+    "nop": {"mtbs_per_sm": 2, "arena_bytes": 96 * 1024, "resident": False},
+}
+
+
+def use_resident(a):
+    return PRESETS[a.workload]["resident"] and not a.no_resident
+
+
+def ctx_config(a, PG):
+    pr = PRESETS[a.workload]
+    cfg = {"flags": PG.NO_START | (PG.RESIDENT_TDES if use_resident(a) else 0),
+           "mtbs_per_sm": a.mtbs or pr["mtbs_per_sm"],
+           "arena_bytes": (a.arena_kb * 1024) if a.arena_kb else pr["arena_bytes"]}
+    return cfg
 
 
 # ----------------------------------------------------------------- main GPU leg
@@ -245,7 +270,7 @@ def main():
     torch.cuda.set_device(d.local)
     dev = d.local
     peaks = measured_peaks()
-    w = make_workload(a.workload)
+    w = make_workload(a.workload, use_resident(a))
     n = w.n
     out = {}
 
@@ -259,7 +284,7 @@ def main():
                         "how": "one <<<n_tb, threads, shmem>>> launch per task, same bodies, 32 streams, "
                                "CUDA_DEVICE_MAX_CONNECTIONS=32, first launch -> cudaDeviceSynchronize"}
 
-    p = PG.Pagoda(device=dev, flags=PG.NO_START)
+    p = PG.Pagoda(device=dev, **ctx_config(a, PG))
 
     def step():
         if a.prespawn:
@@ -343,7 +368,11 @@ def main():
             "dtype": DTYPE[a.workload],
             "data": "synthetic (seeded splitmix64 inputs, SURVEY §8(c) recipe)",
             "config": workload_config(a.workload) | {"parallelism": f"{d.world} GPU(s), one MasterKernel each",
-                                                      "mtbs": info.n_mtb, "regs_per_thread": info.regs_per_thread},
+                                                      "mtbs": info.n_mtb, "regs_per_thread": info.regs_per_thread,
+                                                      "context": {k: v for k, v in ctx_config(a, PG).items()
+                                                                  if k != "flags"} | {
+                                                          "resident_tdes_tables": use_resident(a)},
+                                                      "task_shmem_bytes": int(w.shapes[0][2])},
             "gpu_launches": a.steps, "device_ms_per_step": dev_avg_ms, "clocks": clk}
     if lat:
         line["p50_spawn_to_done_us"] = lat["loaded_us"]["p50"]

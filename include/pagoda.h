@@ -40,6 +40,8 @@ typedef int64_t pagoda_task_t;          /* >= 0: task id; < 0: -errno */
 /* config flags */
 #define PAGODA_TRACE         0x1u /* record the per-MTB scheduler ledger (tests; slows scheduling) */
 #define PAGODA_NO_START      0x2u /* pagoda_init allocates but does not launch; call pagoda_start(_drain) */
+#define PAGODA_RESIDENT_TDES 0x4u /* keep 64 KiB of lane-replicated 3DES S-box tables resident in every MTB
+                                     (conflict-free lookups; the arena starts after them) */
 
 typedef struct {
     int      device;        /* CUDA device ordinal (default 0) */
@@ -156,6 +158,7 @@ int pagoda_get_info(pagoda_ctx* ctx, pagoda_info* out);
 
 #define PAGODA_DEVERR_SYNC_WITHOUT_FLAG 1u  /* syncBlock() in a multi-warp TB spawned with sync=0 */
 #define PAGODA_DEVERR_BAD_FUNC          2u  /* entry with unknown func_id reached an executor */
+#define PAGODA_DEVERR_LAYOUT            4u  /* resident tables did not fit the shared-memory layout (fell back) */
 
 /* Ledger (PAGODA_TRACE): copy up to cap 32-byte events of MTB `mtb` into dst
  * (host memory), after pagoda_shutdown's drain or while idle.  Layout: see

@@ -27,7 +27,7 @@ namespace pagoda {
 /* One WarpTable slot (Table 2), 32 bytes, written by the scheduler
  * warp before it releases the executor warp (Alg. 2 L9-14 P:846-851). */
 struct WarpSlot {
-    uint32_t smem_off;    /* byte offset of this TB's shared memory in the MTB arena (SMindex) */
+    uint32_t smem_off;    /* byte offset of this TB's shared memory from the MTB's shared-memory base (SMindex) */
     uint32_t smem_bytes;  /* granted bytes (request rounded up to 512) */
     uint16_t tb;          /* thread-block index j within the task */
     uint16_t threads_tb;  /* requested threads per TB */
@@ -45,9 +45,12 @@ static_assert(sizeof(WarpSlot) == 32, "WarpSlot is 32 bytes");
 enum : uint8_t { SLOT_TERMINATE = 0xFF };
 
 /* Byte offsets inside the MTB's dynamic shared memory (the control block is
- * laid out in csrc/mk_layout.cuh, which static_asserts both). */
+ * laid out in csrc/mk_layout.cuh, which static_asserts them).  The task arena
+ * follows the control block, or the resident tables when a context has them. */
 constexpr uint32_t kWarpTableOffset = 512;
-constexpr uint32_t kArenaOffset = 5120;   /* 1 KiB aligned */
+constexpr uint32_t kControlBytes = 5120;            /* arena offset without resident tables */
+constexpr uint32_t kResidentOffset = 8192;          /* 8 KiB aligned: lane bits OR into addresses */
+constexpr uint32_t kResidentTdesBytes = 8 * 64 * 32 * 4;   /* 3DES SP tables, one copy per lane */
 
 __device__ __forceinline__ uint32_t lane_id() { return threadIdx.x & 31u; }
 
@@ -71,10 +74,11 @@ __device__ __forceinline__ uint32_t smem_u32(const void* p)
 /* ---------------------------------------------------------------- TaskEnv */
 struct TaskEnv {
     WarpSlot s;
-    char*     arena;        /* MTB arena base */
+    char*     smem_base;    /* MTB dynamic shared memory base */
     uint64_t* stage_bar;    /* this warp's staging mbarrier */
     uint32_t* stage_phase;  /* its parity (register of the executor loop) */
     uint32_t* dev_error;    /* device error word */
+    uint32_t  resident;     /* shared-window address of the MTB-resident 3DES tables, 0 if none */
 
     __device__ __forceinline__ int getTid() const
     {
@@ -85,8 +89,10 @@ struct TaskEnv {
     __device__ __forceinline__ int getBlockDim() const { return s.threads_tb; }
     __device__ __forceinline__ int getBlockWarps() const { return s.warps_tb; }
     __device__ __forceinline__ int getNumBlocks() const { return s.n_tb; }
-    __device__ __forceinline__ char* getSMPtr() const { return arena + s.smem_off; }
+    __device__ __forceinline__ char* getSMPtr() const { return smem_base + s.smem_off; }
     __device__ __forceinline__ uint32_t getSMBytes() const { return s.smem_bytes; }
+    /* MTB-resident, lane-replicated 3DES SP tables (context flag PAGODA_RESIDENT_TDES) */
+    __device__ __forceinline__ uint32_t getResidentTdes() const { return resident; }
     /* true if syncBlock() is legal: a 1-warp TB, or a TB spawned with sync=1 */
     __device__ __forceinline__ bool canSync() const { return s.warps_tb == 1 || s.bar_id != 0; }
     __device__ __forceinline__ void syncBlock() const
@@ -145,6 +151,7 @@ struct NativeEnv {
         return native_smem;
     }
     __device__ __forceinline__ uint32_t getSMBytes() const { return smem_bytes; }
+    __device__ __forceinline__ uint32_t getResidentTdes() const { return 0; }
     __device__ __forceinline__ bool canSync() const { return true; }
     __device__ __forceinline__ void syncBlock() const { __syncthreads(); }
     __device__ __forceinline__ void stage(void* smem_dst, const void* gsrc, uint32_t bytes) const
@@ -183,7 +190,7 @@ __device__ __forceinline__ void syncBlock()
 __device__ __forceinline__ char* getSMPtr()
 {
     extern __shared__ __align__(1024) unsigned char pagoda_mk_smem[];
-    return reinterpret_cast<char*>(pagoda_mk_smem) + pagoda::kArenaOffset + pagoda_my_slot().smem_off;
+    return reinterpret_cast<char*>(pagoda_mk_smem) + pagoda_my_slot().smem_off;
 }
 
 #endif

@@ -137,10 +137,17 @@ __device__ void body_mb(const Env& e, const pagoda_mb_args& a)
 /* ------------------------------------------------------------- 3DES
  * TDEA EDE3, ECB (NIST [5]).  tables =
  * pagoda_tdes_tables(): SP[8][64] u32 (S-box j then P, for the 6-bit input of
- * box j), 48 round keys as 8 six-bit chunks each (execution order
+ * box j), 48 round keys as a (kx, ky) u32 pair each (execution order
  * K1[0..15], K2[15..0], K3[0..15]), IP and FP byte tables [8][256] u64.
  * Since FP then IP cancel between the three DES stages, a block is
- * IP, 48 rounds with a half-swap after every 16, FP. */
+ * IP, 48 rounds with a half-swap after every 16, FP.
+ *
+ * Round function without the E table: the 6-bit input of S-box j is
+ * rotl(R, 4j+5) & 63 ^ k_j, so x = rotl(R,5) ^ kx holds the inputs of boxes
+ * 0,6,4,2 in bytes 0..3 and y = rotl(R,1) ^ ky those of boxes 7,5,3,1 (kx, ky
+ * pack the key chunks the same way).  The 8 S-box outputs after P are disjoint,
+ * so f = XOR of 8 table words.  Three table placements: MTB-resident with one
+ * copy per lane (conflict-free), staged in the TB's shared memory, or global. */
 constexpr uint32_t kTdesStageBytes = 2048 + 384;
 constexpr uint32_t kTdesIpOff = 2432, kTdesFpOff = 2432 + 16384;
 
@@ -152,20 +159,50 @@ __device__ __forceinline__ uint64_t tdes_perm(const uint64_t* tab, uint64_t x)
     return r;
 }
 
-template <class Env>
-__device__ void body_tdes(const Env& e, const pagoda_tdes_args& a)
+template <int kOff>
+__device__ __forceinline__ uint32_t lds_at(uint32_t addr)
 {
-    const uint32_t* sp = a.tables;
-    const uint8_t* keys = reinterpret_cast<const uint8_t*>(a.tables + 512);
-    if (e.getSMBytes() >= kTdesStageBytes && e.canSync()) {   /* stage SP boxes + round keys into the TB's shmem */
-        uint32_t* s = reinterpret_cast<uint32_t*>(e.getSMPtr());
-        if (e.getBlockTid() < 32) e.stage(s, a.tables, kTdesStageBytes);
-        e.syncBlock();
-        sp = s;
-        keys = reinterpret_cast<const uint8_t*>(s + 512);
+    uint32_t v;
+    asm("ld.shared.u32 %0, [%1+%2];" : "=r"(v) : "r"(addr), "n"(kOff));
+    return v;
+}
+
+enum { kTdesResident = 0, kTdesShared = 1, kTdesGlobal = 2 };
+
+/* f(R) for table placement kMode.  resident: entry (j,v) at rl + 8192 j + 128 v
+ * with rl = base | lane*4 (base 8 KiB aligned); shared: at sb + 256 j + 4 v
+ * (sb 256-byte aligned); global: sp[64 j + v]. */
+template <int kMode>
+__device__ __forceinline__ uint32_t tdes_f(uint32_t r, uint32_t kx, uint32_t ky, uint32_t tb, const uint32_t* sp)
+{
+    const uint32_t x = __funnelshift_l(r, r, 5) ^ kx;
+    const uint32_t y = __funnelshift_l(r, r, 1) ^ ky;
+    if (kMode == kTdesResident) {
+        const uint32_t m = 63u << 7;
+        return lds_at<0 * 8192>(tb | ((x << 7) & m)) ^ lds_at<6 * 8192>(tb | ((x >> 1) & m)) ^
+               lds_at<4 * 8192>(tb | ((x >> 9) & m)) ^ lds_at<2 * 8192>(tb | ((x >> 17) & m)) ^
+               lds_at<7 * 8192>(tb | ((y << 7) & m)) ^ lds_at<5 * 8192>(tb | ((y >> 1) & m)) ^
+               lds_at<3 * 8192>(tb | ((y >> 9) & m)) ^ lds_at<1 * 8192>(tb | ((y >> 17) & m));
+    } else if (kMode == kTdesShared) {
+        const uint32_t m = 63u << 2;
+        return lds_at<0 * 256>(tb | ((x << 2) & m)) ^ lds_at<6 * 256>(tb | ((x >> 6) & m)) ^
+               lds_at<4 * 256>(tb | ((x >> 14) & m)) ^ lds_at<2 * 256>(tb | ((x >> 22) & m)) ^
+               lds_at<7 * 256>(tb | ((y << 2) & m)) ^ lds_at<5 * 256>(tb | ((y >> 6) & m)) ^
+               lds_at<3 * 256>(tb | ((y >> 14) & m)) ^ lds_at<1 * 256>(tb | ((y >> 22) & m));
+    } else {
+        return __ldg(sp + 0 * 64 + (x & 63)) ^ __ldg(sp + 6 * 64 + ((x >> 8) & 63)) ^
+               __ldg(sp + 4 * 64 + ((x >> 16) & 63)) ^ __ldg(sp + 2 * 64 + ((x >> 24) & 63)) ^
+               __ldg(sp + 7 * 64 + (y & 63)) ^ __ldg(sp + 5 * 64 + ((y >> 8) & 63)) ^
+               __ldg(sp + 3 * 64 + ((y >> 16) & 63)) ^ __ldg(sp + 1 * 64 + ((y >> 24) & 63));
     }
+}
+
+template <int kMode, class Env>
+__device__ __forceinline__ void tdes_blocks(const Env& e, const pagoda_tdes_args& a, uint32_t tb, uint32_t kb)
+{
     const uint64_t* ipt = reinterpret_cast<const uint64_t*>(reinterpret_cast<const char*>(a.tables) + kTdesIpOff);
     const uint64_t* fpt = reinterpret_cast<const uint64_t*>(reinterpret_cast<const char*>(a.tables) + kTdesFpOff);
+    const uint2* gkeys = reinterpret_cast<const uint2*>(a.tables + 512);
     const int T = total_threads(e);
     for (uint32_t blk = (uint32_t)e.getTid(); blk < a.nblk; blk += (uint32_t)T) {
         uint64_t x = a.in[blk];
@@ -175,18 +212,12 @@ __device__ void body_tdes(const Env& e, const pagoda_tdes_args& a)
         uint32_t l = (uint32_t)(x >> 32), r = (uint32_t)x;
 #pragma unroll 1
         for (int st = 0; st < 3; st++) {
-#pragma unroll 2
+#pragma unroll 4
             for (int rd = 0; rd < 16; rd++) {
-                const uint32_t* kr = reinterpret_cast<const uint32_t*>(keys + (st * 16 + rd) * 8);
-                const uint32_t k0 = kr[0], k1 = kr[1];
-                uint32_t f = 0;
-#pragma unroll
-                for (int j = 0; j < 8; j++) {
-                    const uint32_t kj = ((j < 4 ? k0 : k1) >> (8 * (j & 3))) & 63u;
-                    const uint32_t six = (__funnelshift_l(r, r, 4 * j + 5) & 63u) ^ kj;
-                    f |= sp[j * 64 + six];
-                }
-                const uint32_t t = l ^ f;
+                uint2 k;
+                if (kb) asm("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(k.x), "=r"(k.y) : "r"(kb + (st * 16 + rd) * 8));
+                else k = __ldg(gkeys + st * 16 + rd);
+                const uint32_t t = l ^ tdes_f<kMode>(r, k.x, k.y, tb, a.tables);
                 l = r;
                 r = t;
             }
@@ -198,6 +229,23 @@ __device__ void body_tdes(const Env& e, const pagoda_tdes_args& a)
         x = ((uint64_t)__byte_perm((uint32_t)x, 0, 0x0123) << 32) | __byte_perm((uint32_t)(x >> 32), 0, 0x0123);
         a.out[blk] = x;
     }
+}
+
+template <class Env>
+__device__ void body_tdes(const Env& e, const pagoda_tdes_args& a)
+{
+    const uint32_t res = e.getResidentTdes();
+    const uint32_t need = res ? 384u : kTdesStageBytes;
+    uint32_t sb = 0;
+    if (e.getSMBytes() >= need && e.canSync()) {   /* stage round keys (and SP boxes) into the TB's shmem */
+        char* s = e.getSMPtr();
+        if (e.getBlockTid() < 32) e.stage(s, res ? reinterpret_cast<const char*>(a.tables) + 2048 : (const char*)a.tables, need);
+        e.syncBlock();
+        sb = smem_u32(s);
+    }
+    if (res) tdes_blocks<kTdesResident>(e, a, res | (lane_id() << 2), sb);
+    else if (sb) tdes_blocks<kTdesShared>(e, a, sb, sb + 2048);
+    else tdes_blocks<kTdesGlobal>(e, a, 0, 0);
 }
 
 /* ------------------------------------------------------------- MM

@@ -77,6 +77,16 @@ __device__ __forceinline__ void st_release_gpu(uint64_t* p, uint64_t v)
 {
     asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
+__device__ __forceinline__ void st_relaxed_gpu32(uint32_t* p, uint32_t v)
+{
+    asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ uint32_t ld_relaxed_gpu32(const uint32_t* p)
+{
+    uint32_t v;
+    asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
 __device__ __forceinline__ void st_release_gpu32(uint32_t* p, uint32_t v)
 {
     asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
@@ -160,7 +170,7 @@ __device__ __forceinline__ void trace_ev(const MkParams& p, int mtb, uint32_t& s
  * deferred release: the last warp of a TB returns its shmem granules and
  * barrier ID through the scheduler's mailbox (markSMForDealloc), the last warp
  * of the task posts its completion record, every warp returns itself. */
-__device__ void executor(MtbShared& S, char* arena, const MkParams& p, int mtb, int w)
+__device__ void executor(MtbShared& S, char* smem_base, const MkParams& p, int mtb, int w, uint32_t resident)
 {
     const uint32_t lane = threadIdx.x & 31u;
     uint32_t phase = 0, stage_phase = 0;
@@ -172,7 +182,8 @@ __device__ void executor(MtbShared& S, char* arena, const MkParams& p, int mtb, 
         const TaskEntry& t = S.tasks[s.task];
         uint64_t t0 = 0;
         if (p.trace_cap) t0 = globaltimer_ns();
-        TaskEnv env{s, arena, &S.stage_bar[w], &stage_phase, &p.dctl->error};
+        TaskEnv env{s, smem_base, &S.stage_bar[w], &stage_phase, &p.dctl->error,
+                    resident};
         if (!run_body(t.func_id, env, t.args) && lane == 0) atomicOr(&p.dctl->error, PAGODA_DEVERR_BAD_FUNC);
         __syncwarp();
         if (lane == 0) {
@@ -210,8 +221,7 @@ __device__ void executor(MtbShared& S, char* arena, const MkParams& p, int mtb, 
  * into the device ring, a bounded MPMC queue with one sequence word per cell:
  * the producer may fill the cell of position t once seq == t (its previous
  * occupant was consumed), then releases seq = t + 1. */
-constexpr int kIngestBatch = 256;                       /* entries per round (16 KiB staging) */
-constexpr uint32_t kIngestStageBytes = kIngestBatch * 64;
+/* kIngestBatch, kIngestStageBytes: mk_layout.cuh */
 
 __device__ void ingest(const MkParams& p, char* stage_buf)
 {
@@ -237,17 +247,23 @@ __device__ void ingest(const MkParams& p, char* stage_buf)
         }
         if (pub > copied) {
             uint32_t n = (uint32_t)min(pub - copied, (uint64_t)kIngestBatch);
-            /* free cells: the longest prefix whose previous occupant was consumed */
-            uint32_t ready = n;
-            for (uint32_t base = 0; base < n; base += 32u) {
-                const uint64_t t = copied + base + lane;
-                const bool ok = base + lane >= n || ld_acquire_gpu(&p.dseq[t & p.ring_mask]) == t;
-                const uint32_t bad = __ballot_sync(0xffffffffu, !ok);
-                if (bad) {
-                    ready = base + (uint32_t)__ffs(bad) - 1u;
-                    break;
-                }
+            /* free cells: the longest prefix whose previous occupant was consumed.  All the
+             * sequence loads are issued before any is used (one L2 round trip), then one
+             * fence gives them acquire semantics. */
+            constexpr int kSeqPerLane = kIngestBatch / 32;
+            uint32_t sv[kSeqPerLane];
+#pragma unroll
+            for (int i = 0; i < kSeqPerLane; i++) {
+                const uint64_t t = copied + (uint64_t)i * 32u + lane;
+                sv[i] = (uint32_t)i * 32u + lane < n ? ld_relaxed_gpu32(&p.dseq[t & p.ring_mask]) : (uint32_t)t;
             }
+            uint32_t ready = n;
+#pragma unroll
+            for (int i = 0; i < kSeqPerLane; i++) {
+                const uint32_t bad = __ballot_sync(0xffffffffu, sv[i] != (uint32_t)(copied + (uint64_t)i * 32u + lane));
+                if (bad && ready == n) ready = min(n, (uint32_t)i * 32u + (uint32_t)__ffs(bad) - 1u);
+            }
+            __threadfence();
             n = ready;
             if (n == 0) {              /* device ring full: wait for the schedulers */
                 __nanosleep(128);
@@ -265,10 +281,11 @@ __device__ void ingest(const MkParams& p, char* stage_buf)
                 const int4 v = *reinterpret_cast<const int4*>(stage_buf + c * 16u);
                 __stcg(reinterpret_cast<int4*>(p.dring + e) + (c & 3u), v);
             }
-            __syncwarp();   /* every lane's entry stores precede each cell's release */
+            __syncwarp();      /* every lane's entry stores precede ... */
+            __threadfence();   /* ... one warp-wide fence, so each lane's relaxed seq store releases them */
             for (uint32_t i = lane; i < n; i += 32u) {
                 const uint64_t t = copied + i;
-                st_release_gpu(&p.dseq[t & p.ring_mask], t + 1);
+                st_relaxed_gpu32(&p.dseq[t & p.ring_mask], (uint32_t)(t + 1));
             }
             __syncwarp();
             copied += n;
@@ -358,7 +375,7 @@ __device__ bool sched_place(MtbShared& S, Sched& st, const MkParams& p, int mtb,
         trace_ev(p, mtb, st.seq, 1, id, (uint16_t)j, m, (uint16_t)off, (uint16_t)gtb, (uint8_t)bar);
         if ((m >> lane) & 1u) {   /* Alg. 2 L9-12: lane l fills warp l's WarpTable slot */
             WarpSlot ws;
-            ws.smem_off = off * PAGODA_GRANULE;
+            ws.smem_off = p.arena_offset + off * PAGODA_GRANULE;
             ws.smem_bytes = gtb * PAGODA_GRANULE;
             ws.tb = (uint16_t)j;
             ws.threads_tb = threads;
@@ -423,7 +440,7 @@ __device__ int sched_load(MtbShared& S, Sched& st, const MkParams& p)
     bool ready = false;
     if (lane < n) {
         t = S.pend_ticket[(st.pl + lane) & 31u];
-        ready = ld_acquire_gpu(&p.dseq[t & p.ring_mask]) == t + 1;
+        ready = ld_acquire_gpu32(&p.dseq[t & p.ring_mask]) == (uint32_t)(t + 1);
     }
     const uint32_t nr = __ballot_sync(0xffffffffu, !ready);
     const uint32_t r = nr ? (uint32_t)__ffs(nr) - 1u : 32u;   /* leading published tickets */
@@ -439,7 +456,7 @@ __device__ int sched_load(MtbShared& S, Sched& st, const MkParams& p)
     if (lane < r) {
         const uint32_t slot = nth_set_bit(st.free_task, lane);
         S.pend[(st.pl + lane) & 31u] = (uint8_t)slot;
-        st_release_gpu(&p.dseq[t & p.ring_mask], t + (uint64_t)p.ring_mask + 1);
+        st_release_gpu32(&p.dseq[t & p.ring_mask], (uint32_t)(t + (uint64_t)p.ring_mask + 1));
         used = 1u << slot;
     }
     used = __reduce_or_sync(0xffffffffu, used);
@@ -547,13 +564,30 @@ __global__ void __launch_bounds__(1024, kMinBlocks) master_kernel(MkParams p)
 {
     extern __shared__ __align__(1024) unsigned char pagoda_mk_smem[];
     MtbShared& S = *reinterpret_cast<MtbShared*>(pagoda_mk_smem);
-    char* arena = reinterpret_cast<char*>(pagoda_mk_smem) + kArenaOffset;
+    char* smem_base = reinterpret_cast<char*>(pagoda_mk_smem);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, mtb = blockIdx.x;
     int arena_granules = p.arena_granules;
     char* ingest_stage = nullptr;
     if (mtb == 0) {   /* MTB 0 lends the top of its arena to the ingest warp */
         arena_granules -= (int)(kIngestStageBytes / PAGODA_GRANULE);
-        ingest_stage = arena + (size_t)arena_granules * PAGODA_GRANULE;
+        ingest_stage = smem_base + p.arena_offset + (size_t)arena_granules * PAGODA_GRANULE;
+    }
+    uint32_t resident = 0;   /* shared-window address of the resident tables */
+    if (p.resident_tdes_src) {
+        /* task-class resident tables (key-independent 3DES S-box/P tables), one copy per
+         * lane: word (j*64 + v)*32 + lane holds SP[j][v], so any 32 lookups are conflict-free.
+         * The region's WINDOW address must be 8 KiB aligned (lookups OR lane and index bits
+         * into it); the dynamic segment itself starts after the CTA's reserved shared memory. */
+        const uint32_t base = smem_u32(smem_base);
+        resident = (base + kControlBytes + 8191u) & ~8191u;
+        if (resident - base + kResidentTdesBytes <= p.arena_offset) {
+            uint32_t* dst = reinterpret_cast<uint32_t*>(smem_base + (resident - base));
+            for (uint32_t i = threadIdx.x; i < kResidentTdesBytes / 4; i += blockDim.x)
+                dst[i] = __ldg(p.resident_tdes_src + (i >> 5));
+        } else {
+            resident = 0;   /* layout does not fit: bodies fall back to per-task tables */
+            if (threadIdx.x == 0) atomicOr(&p.dctl->error, PAGODA_DEVERR_LAYOUT);
+        }
     }
     if (warp == 0) {
         mbar_init(&S.exec_bar[lane], 1);
@@ -566,7 +600,7 @@ __global__ void __launch_bounds__(1024, kMinBlocks) master_kernel(MkParams p)
     __syncthreads();
     if (warp == 0) scheduler(S, p, mtb, arena_granules);
     else if (mtb == 0 && warp == kIngestWarp) ingest(p, ingest_stage);
-    else if (warp <= p.exec_warps) executor(S, arena, p, mtb, warp);
+    else if (warp <= p.exec_warps) executor(S, smem_base, p, mtb, warp, resident);
 }
 
 template __global__ void master_kernel<1>(MkParams);

@@ -79,13 +79,16 @@ struct MkParams {
     HostCtl*         hctl;    /* pinned host control (mapped) */
     int64_t*         comp;    /* pinned completion window (mapped) */
     TaskEntry*       dring;   /* device ring */
-    uint64_t*        dseq;    /* per-cell sequence numbers (bounded MPMC queue): cell of position t holds
+    uint32_t*        dseq;    /* per-cell sequence numbers mod 2^32 (bounded MPMC queue): cell of position t holds
                                  t (free for the producer), t+1 (entry t published), t+R (entry t consumed) */
     DevCtl*          dctl;
     uint32_t ring_mask;
     uint32_t comp_mask;
     int      exec_warps;      /* executor warps per MTB (warps 1..exec_warps) */
     int      arena_granules;
+    uint32_t arena_offset;    /* byte offset of the task arena in dynamic shared memory */
+    const uint32_t* resident_tdes_src;   /* 2 KiB SP table in device memory, replicated per lane
+                                            at kResidentOffset when non-null */
     int      n_mtb;
     uint32_t trace_cap;       /* 0 = tracing off */
     LedgerEvent* trace;       /* [n_mtb][trace_cap] */
@@ -95,6 +98,8 @@ struct MkParams {
 };
 
 constexpr int kIngestWarp = 31;          /* warp 31 of MTB 0 feeds the device ring */
+constexpr int kIngestBatch = 512;        /* entries per ingest round */
+constexpr uint32_t kIngestStageBytes = kIngestBatch * 64;   /* its staging, lent by MTB 0 from the top of its arena */
 constexpr uint32_t kStopAbort = 2;       /* HostCtl.terminate / DevCtl.stop value: abandon work and exit */
 constexpr int kMaxGranules = 1024;       /* lane-distributed bitmap: 32 lanes x 32 bits */
 
@@ -120,7 +125,7 @@ struct MtbShared {
     uint64_t  pend_ticket[32];       /* 4368: claimed ring positions, FIFO (pend[] holds their slots once loaded) */
 };
 static_assert(offsetof(MtbShared, wt) == kWarpTableOffset, "WarpTable offset");
-static_assert(sizeof(MtbShared) <= kArenaOffset, "control block fits below the arena");
+static_assert(sizeof(MtbShared) <= kControlBytes && kControlBytes <= kResidentOffset, "control block fits");
 
 } // namespace pagoda
 #endif

@@ -40,7 +40,7 @@ cudaError_t launch_master(int mtbs_per_sm, int n_mtb, size_t smem_bytes, cudaStr
 }
 using namespace pagoda;
 
-static const uint32_t kIngestGranules = 32;   /* MTB 0 lends 16 KiB of its arena to the ingest warp */
+static const uint32_t kIngestGranules = kIngestStageBytes / PAGODA_GRANULE;   /* MTB 0 lends them to the ingest warp */
 
 struct pagoda_ctx {
     pagoda_config cfg;
@@ -55,7 +55,8 @@ struct pagoda_ctx {
     volatile int64_t* comp = nullptr;
     /* device */
     TaskEntry* dring = nullptr;
-    uint64_t* dseq = nullptr;
+    uint32_t* resident_src = nullptr;
+    uint32_t* dseq = nullptr;
     DevCtl* dctl = nullptr;
     LedgerEvent* trace = nullptr;
     uint32_t* trace_count = nullptr;
@@ -225,6 +226,7 @@ static void free_ctx(pagoda_ctx* c)
     if (c->comp) cudaFreeHost((void*)c->comp);
     if (c->dring) cudaFree(c->dring);
     if (c->dseq) cudaFree(c->dseq);
+    if (c->resident_src) cudaFree(c->resident_src);
     if (c->dctl) cudaFree(c->dctl);
     if (c->trace) cudaFree(c->trace);
     if (c->trace_count) cudaFree(c->trace_count);
@@ -256,7 +258,8 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
     cudaDeviceProp prop;
     if (cudaGetDeviceProperties(&prop, cfg.device) != cudaSuccess) return -ENODEV;
     if (prop.major != 10) return -ENODEV;   /* built for sm_100a only */
-    const size_t smem = kArenaOffset + cfg.arena_bytes;
+    const uint32_t arena_offset = (cfg.flags & PAGODA_RESIDENT_TDES) ? kResidentOffset + kResidentTdesBytes : kControlBytes;
+    const size_t smem = arena_offset + cfg.arena_bytes;
     if (smem * (size_t)cfg.mtbs_per_sm + 1024 * (size_t)cfg.mtbs_per_sm > (size_t)prop.sharedMemPerMultiprocessor ||
         smem > (size_t)prop.sharedMemPerBlockOptin)
         return -EINVAL;
@@ -294,11 +297,11 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
         goto fail;
     for (uint32_t i = 0; i < c->C; i++) c->comp[i] = -1;
     if (cudaMalloc(&c->dring, (size_t)c->R * sizeof(TaskEntry)) != cudaSuccess) goto fail;
-    if (cudaMalloc(&c->dseq, (size_t)c->R * sizeof(uint64_t)) != cudaSuccess) goto fail;
+    if (cudaMalloc(&c->dseq, (size_t)c->R * sizeof(uint32_t)) != cudaSuccess) goto fail;
     {   /* cell i starts free for position i */
-        std::vector<uint64_t> seq(c->R);
+        std::vector<uint32_t> seq(c->R);
         for (uint32_t i = 0; i < c->R; i++) seq[i] = i;
-        if (cudaMemcpy(c->dseq, seq.data(), seq.size() * sizeof(uint64_t), cudaMemcpyHostToDevice) != cudaSuccess)
+        if (cudaMemcpy(c->dseq, seq.data(), seq.size() * sizeof(uint32_t), cudaMemcpyHostToDevice) != cudaSuccess)
             goto fail;
     }
     if (cudaMalloc(&c->dctl, sizeof(DevCtl)) != cudaSuccess) goto fail;
@@ -333,6 +336,14 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
         p.comp_mask = c->C - 1;
         p.exec_warps = (int)cfg.exec_warps;
         p.arena_granules = (int)arena_g;
+        p.arena_offset = arena_offset;
+        if (cfg.flags & PAGODA_RESIDENT_TDES) {   /* the key-independent SP table, replicated by each MTB */
+            std::vector<uint8_t> tab(PAGODA_TDES_TABLE_BYTES);
+            const uint8_t zero_key[24] = {0};
+            pagoda_tdes_tables(zero_key, tab.data());
+            if (cudaMalloc(&c->resident_src, 2048) != cudaSuccess || cudaMemcpy(c->resident_src, tab.data(), 2048, cudaMemcpyHostToDevice) != cudaSuccess) goto fail;
+            p.resident_tdes_src = c->resident_src;
+        }
         p.n_mtb = c->n_mtb;
         if (cfg.flags & PAGODA_TRACE) {
             p.trace_cap = c->cfg.trace_events;

@@ -8,8 +8,9 @@
  * Output layout (bytes):
  *   [0, 2048)        SP[8][64] u32: P(S_j(six) placed in nibble j) for the 6-bit
  *                    input six = b1..b6 of box j (b1 = most significant)
- *   [2048, 2432)     48 round keys x 8 chunks (u8, 6 bits each), execution order
- *                    K1 rounds 1..16, K2 rounds 16..1 (decrypt), K3 rounds 1..16
+ *   [2048, 2432)     48 round keys as (kx, ky) u32 pairs, execution order
+ *                    K1 rounds 1..16, K2 rounds 16..1 (decrypt), K3 rounds 1..16;
+ *                    kx bytes 0..3 = the key chunks of S-boxes 0,6,4,2, ky of 7,5,3,1
  *   [2432, 18816)    IPT[8][256] u64: IP of byte b (b = 0 most significant) alone
  *   [18816, 35200)   FPT[8][256] u64: IP^-1 likewise
  */
@@ -98,14 +99,17 @@ extern "C" int pagoda_tdes_tables(const uint8_t key24[24], void* dst)
             const uint64_t nib = (uint64_t)kS[j][row * 16 + col] << (28 - 4 * j);
             sp[j * 64 + six] = (uint32_t)bits_permute(nib, kPerm, 32, 32);
         }
-    uint8_t* rk = out + 2048;
+    uint32_t* rk = reinterpret_cast<uint32_t*>(out + 2048);
     uint64_t k1[16], k2[16], k3[16];
     subkeys(key24, k1);
     subkeys(key24 + 8, k2);
     subkeys(key24 + 16, k3);
     for (int r = 0; r < 48; r++) {
         const uint64_t k = r < 16 ? k1[r] : (r < 32 ? k2[31 - r] : k3[r - 32]);
-        for (int j = 0; j < 8; j++) rk[r * 8 + j] = (uint8_t)((k >> (42 - 6 * j)) & 63u);
+        uint32_t c[8];   /* c[j] = the 6 key bits that meet S-box j's input */
+        for (int j = 0; j < 8; j++) c[j] = (uint32_t)((k >> (42 - 6 * j)) & 63u);
+        rk[2 * r + 0] = c[0] | (c[6] << 8) | (c[4] << 16) | (c[2] << 24);   /* kx: boxes 0,6,4,2 */
+        rk[2 * r + 1] = c[7] | (c[5] << 8) | (c[3] << 16) | (c[1] << 24);   /* ky: boxes 7,5,3,1 */
     }
     int fp[64];   /* IP^-1: IP maps input bit kIP[k] to output bit k+1 */
     for (int k = 0; k < 64; k++) fp[kIP[k] - 1] = k + 1;

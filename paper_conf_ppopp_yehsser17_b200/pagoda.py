@@ -18,6 +18,7 @@ LIB_PATH = os.path.join(PKG, "libpagoda.so")
 
 TRACE = 0x1
 NO_START = 0x2
+RESIDENT_TDES = 0x4
 
 
 class pagoda_config(C.Structure):

@@ -80,7 +80,7 @@ def _des_with_product_tables(tab: np.ndarray, block: int) -> int:
     """Run the GPU body's round structure on the CPU with the product's tables
     (same index arithmetic as body_tdes in csrc/bodies.cuh)."""
     sp = tab[:2048].view(np.uint32).reshape(8, 64)
-    keys = tab[2048:2432].reshape(48, 8)
+    keys = tab[2048:2432].view(np.uint32).reshape(48, 2)
     ipt = tab[2432:2432 + 16384].view(np.uint64).reshape(8, 256)
     fpt = tab[2432 + 16384:].view(np.uint64).reshape(8, 256)
 
@@ -98,10 +98,12 @@ def _des_with_product_tables(tab: np.ndarray, block: int) -> int:
     l, r = x >> 32, x & 0xFFFFFFFF
     for st in range(3):
         for rd in range(16):
+            kx, ky = (int(v) for v in keys[st * 16 + rd])
+            x = rotl(r, 5) ^ kx          # bytes 0..3: inputs of S-boxes 0, 6, 4, 2
+            y = rotl(r, 1) ^ ky          # bytes 0..3: inputs of S-boxes 7, 5, 3, 1
             f = 0
-            for j in range(8):
-                six = (rotl(r, 4 * j + 5) & 63) ^ int(keys[st * 16 + rd, j])
-                f |= int(sp[j, six])
+            for b, (jx, jy) in enumerate(zip((0, 6, 4, 2), (7, 5, 3, 1))):
+                f ^= int(sp[jx, (x >> 8 * b) & 63]) ^ int(sp[jy, (y >> 8 * b) & 63])
             l, r = r, l ^ f
         l, r = r, l
     return perm(fpt, (l << 32) | r)

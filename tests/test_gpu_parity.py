@@ -17,7 +17,7 @@ import pytest
 import oracle
 from paper_conf_ppopp_yehsser17_b200 import inputs as I
 from paper_conf_ppopp_yehsser17_b200 import workloads as W
-from paper_conf_ppopp_yehsser17_b200.pagoda import Pagoda, naive_run
+from paper_conf_ppopp_yehsser17_b200.pagoda import RESIDENT_TDES, Pagoda, naive_run
 
 pytestmark = pytest.mark.gpu
 
@@ -63,20 +63,24 @@ def _tdes_ref(packet):
     return oracle.tdes_ecb(packet, I.TDES_KEYS)
 
 
-@pytest.mark.parametrize("shmem,threads", [(2560, 128), (0, 128), (2560, 96), (2560, 32)])
-def test_tdes_small_bit_exact(shmem, threads):
+@pytest.mark.parametrize("shmem,threads,resident", [(2560, 128, 0), (0, 128, 0), (2560, 96, 0), (2560, 32, 0),
+                                                   (512, 128, 1), (0, 128, 1), (512, 32, 1), (2560, 256, 1)])
+def test_tdes_small_bit_exact(shmem, threads, resident):
     w = W.tdes(48, shmem=shmem, threads=threads)
-    out = run(w)["out"]
+    cfg = {"flags": RESIDENT_TDES, "arena_bytes": 40 * 1024} if resident else {}
+    out = run(w, **cfg)["out"]
     for k in range(48):
         assert np.array_equal(out[k], _tdes_ref(w.host["packets"][k])), k
     assert out[0, :24].tobytes().hex() == "a826fd8ce53b855fcce21c8112256fe668d5c05dd9b6b900"
 
 
-def test_tdes_config2_full_size():
+@pytest.mark.parametrize("cfg", [{}, {"flags": RESIDENT_TDES, "arena_bytes": 40 * 1024},
+                                 {"flags": RESIDENT_TDES, "mtbs_per_sm": 1, "arena_bytes": 128 * 1024}])
+def test_tdes_config2_full_size(cfg):
     from cryptography.hazmat.decrepit.ciphers.algorithms import TripleDES
     from cryptography.hazmat.primitives.ciphers import Cipher, modes
-    w = W.tdes(32768)
-    out = run(w)["out"]
+    w = W.tdes(32768, shmem=512 if cfg else 2560)
+    out = run(w, **cfg)["out"]
     pk = w.host["packets"]
     enc = Cipher(TripleDES(I.TDES_KEYS), modes.ECB()).encryptor()
     ref_all = np.frombuffer(enc.update(pk.tobytes()) + enc.finalize(), np.uint8).reshape(pk.shape)
