@@ -197,7 +197,17 @@ __device__ __forceinline__ uint32_t tdes_f(uint32_t r, uint32_t kx, uint32_t ky,
     }
 }
 
-template <int kMode, class Env>
+/* round key i of the current stage: from the TB's shared memory (kKeysShared) or global */
+template <bool kKeysShared, int kI>
+__device__ __forceinline__ uint2 tdes_key(uint32_t kb, const uint2* gk)
+{
+    uint2 k;
+    if (kKeysShared) asm("ld.shared.v2.u32 {%0, %1}, [%2+%3];" : "=r"(k.x), "=r"(k.y) : "r"(kb), "n"(kI * 8));
+    else k = __ldg(gk + kI);
+    return k;
+}
+
+template <int kMode, bool kKeysShared, class Env>
 __device__ __forceinline__ void tdes_blocks(const Env& e, const pagoda_tdes_args& a, uint32_t tb, uint32_t kb)
 {
     const uint64_t* ipt = reinterpret_cast<const uint64_t*>(reinterpret_cast<const char*>(a.tables) + kTdesIpOff);
@@ -212,15 +222,20 @@ __device__ __forceinline__ void tdes_blocks(const Env& e, const pagoda_tdes_args
         uint32_t l = (uint32_t)(x >> 32), r = (uint32_t)x;
 #pragma unroll 1
         for (int st = 0; st < 3; st++) {
-#pragma unroll 4
-            for (int rd = 0; rd < 16; rd++) {
-                uint2 k;
-                if (kb) asm("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(k.x), "=r"(k.y) : "r"(kb + (st * 16 + rd) * 8));
-                else k = __ldg(gkeys + st * 16 + rd);
-                const uint32_t t = l ^ tdes_f<kMode>(r, k.x, k.y, tb, a.tables);
-                l = r;
-                r = t;
+            const uint32_t kst = kb + st * 128;    /* 16 rounds x 8 bytes per stage */
+            const uint2* gst = gkeys + st * 16;
+#define PAGODA_TDES_ROUND(I)                                                         \
+            {                                                                        \
+                const uint2 k = tdes_key<kKeysShared, I>(kst, gst);                  \
+                const uint32_t t = l ^ tdes_f<kMode>(r, k.x, k.y, tb, a.tables);     \
+                l = r;                                                               \
+                r = t;                                                               \
             }
+            PAGODA_TDES_ROUND(0) PAGODA_TDES_ROUND(1) PAGODA_TDES_ROUND(2) PAGODA_TDES_ROUND(3)
+            PAGODA_TDES_ROUND(4) PAGODA_TDES_ROUND(5) PAGODA_TDES_ROUND(6) PAGODA_TDES_ROUND(7)
+            PAGODA_TDES_ROUND(8) PAGODA_TDES_ROUND(9) PAGODA_TDES_ROUND(10) PAGODA_TDES_ROUND(11)
+            PAGODA_TDES_ROUND(12) PAGODA_TDES_ROUND(13) PAGODA_TDES_ROUND(14) PAGODA_TDES_ROUND(15)
+#undef PAGODA_TDES_ROUND
             const uint32_t t = l;   /* undo the last half-swap: stage output (R16, L16) */
             l = r;
             r = t;
@@ -243,9 +258,10 @@ __device__ void body_tdes(const Env& e, const pagoda_tdes_args& a)
         e.syncBlock();
         sb = smem_u32(s);
     }
-    if (res) tdes_blocks<kTdesResident>(e, a, res | (lane_id() << 2), sb);
-    else if (sb) tdes_blocks<kTdesShared>(e, a, sb, sb + 2048);
-    else tdes_blocks<kTdesGlobal>(e, a, 0, 0);
+    if (res && sb) tdes_blocks<kTdesResident, true>(e, a, res | (lane_id() << 2), sb);
+    else if (res) tdes_blocks<kTdesResident, false>(e, a, res | (lane_id() << 2), 0);
+    else if (sb) tdes_blocks<kTdesShared, true>(e, a, sb, sb + 2048);
+    else tdes_blocks<kTdesGlobal, false>(e, a, 0, 0);
 }
 
 /* ------------------------------------------------------------- MM

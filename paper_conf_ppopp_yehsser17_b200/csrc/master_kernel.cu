@@ -405,8 +405,8 @@ __device__ int sched_claim(MtbShared& S, Sched& st, const MkParams& p)
     const uint32_t cap = 32u - queued;
     uint32_t want;
     if (st.est_w == 0) want = queued == 0 ? 1u : 0u;
-    else {
-        want = (uint32_t)__popc(st.free_w) / st.est_w;
+    else {   /* what fits now, plus one task of lookahead so the next is loaded when warps free */
+        want = (uint32_t)__popc(st.free_w) / st.est_w + 1u;
         want = want > queued ? want - queued : 0u;
     }
     want = min(want, cap);
@@ -419,7 +419,11 @@ __device__ int sched_claim(MtbShared& S, Sched& st, const MkParams& p)
     head = __shfl_sync(0xffffffffu, head, 0);
     tail = __shfl_sync(0xffffffffu, tail, 0);
     if (head >= tail) return 0;
-    const uint32_t k = (uint32_t)min((uint64_t)want, tail - head);
+    /* a backlog smaller than what every MTB could take is handed out one ticket at a time,
+     * so consecutive (often similar-cost) tasks spread over MTBs instead of piling up */
+    const uint64_t backlog = tail - head;
+    if (backlog < (uint64_t)p.n_mtb * 8u) want = 1;
+    const uint32_t k = (uint32_t)min((uint64_t)want, backlog);
     unsigned long long t0 = 0;
     if (lane == 0) t0 = atomicAdd(reinterpret_cast<unsigned long long*>(&p.dctl->head), (unsigned long long)k);
     t0 = __shfl_sync(0xffffffffu, t0, 0);
@@ -528,7 +532,7 @@ __device__ void scheduler(MtbShared& S, const MkParams& p, int mtb, int arena_gr
         /* ---- take more tickets while resources are free.  MTB 0 (one warp short: it hosts the
          * ingest warp) does not take blind tickets unless it is the only MTB (validation then
          * caps every task to its capacity), so no ticket can land where it never fits. */
-        if (st.free_w && (mtb != 0 || p.n_mtb == 1) && sched_claim(S, st, p) > 0) progress = true;
+        if ((mtb != 0 || p.n_mtb == 1) && sched_claim(S, st, p) > 0) progress = true;
         if (progress) {
             backoff = 0;
             continue;
@@ -547,7 +551,9 @@ __device__ void scheduler(MtbShared& S, const MkParams& p, int mtb, int arena_gr
                 if (st.pl == st.pt || S.pend_ticket[st.pl & 31u] >= tail) break;
             }
         }
-        backoff = backoff ? min(backoff * 2u, 1024u) : 32u;
+        /* with work queued only shared-memory mailboxes are polled: stay responsive;
+         * otherwise the ring is polled in L2: back off */
+        backoff = (st.ph != st.pt) ? 32u : (backoff ? min(backoff * 2u, 1024u) : 32u);
         __nanosleep(backoff);
     }
     /* drain: release every executor warp with a terminate slot */

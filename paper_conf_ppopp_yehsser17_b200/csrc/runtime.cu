@@ -41,6 +41,7 @@ cudaError_t launch_master(int mtbs_per_sm, int n_mtb, size_t smem_bytes, cudaStr
 using namespace pagoda;
 
 static const uint32_t kIngestGranules = kIngestStageBytes / PAGODA_GRANULE;   /* MTB 0 lends them to the ingest warp */
+static const int kSpawnChunk = 64;   /* batched spawns publish the doorbell once per chunk */
 
 struct pagoda_ctx {
     pagoda_config cfg;
@@ -244,7 +245,9 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
     if (cfg_in) cfg = *cfg_in;
     else pagoda_config_default(&cfg);
     if (cfg.mtbs_per_sm != 1 && cfg.mtbs_per_sm != 2) return -EINVAL;
-    if (!pow2(cfg.ring_entries) || !pow2(cfg.comp_entries) || cfg.comp_entries < cfg.ring_entries) return -EINVAL;
+    if (!pow2(cfg.ring_entries) || !pow2(cfg.comp_entries) || cfg.comp_entries < cfg.ring_entries ||
+        cfg.ring_entries < 2 * kSpawnChunk)
+        return -EINVAL;
     if (cfg.exec_warps < 1 || cfg.exec_warps > 31) return -EINVAL;
     if (cfg.arena_bytes % PAGODA_GRANULE || cfg.arena_bytes / PAGODA_GRANULE > (uint32_t)kMaxGranules ||
         cfg.arena_bytes < kIngestGranules * PAGODA_GRANULE)
@@ -431,31 +434,109 @@ pagoda_task_t pagoda_taskSpawn(pagoda_ctx* c, int threads, int n_tb, int shmem_b
     return (pagoda_task_t)id;
 }
 
+/* Batched spawn: the same entries taskSpawn would write, but ids are reserved
+ * a chunk at a time and the doorbell is published once per chunk (the GPU
+ * sees the chunk's tasks together, the host does one atomic and one doorbell
+ * store per chunk instead of per task).  Every task is validated first. */
+} /* extern "C" */
+
+template <class ShapeOf>
+static int64_t spawn_batch(pagoda_ctx* c, int n, ShapeOf shape_of, const void* args_base, size_t args_stride,
+                           size_t args_bytes, pagoda_task_t* ids_out)
+{
+    if (!c || n < 0) return -EINVAL;
+    if (c->shutting.load(std::memory_order_acquire)) return -ESHUTDOWN;
+    if (c->faulted.load(std::memory_order_relaxed)) return -EIO;
+    if (args_bytes > PAGODA_ARGS_MAX || (args_bytes > 0 && !args_base)) return -EINVAL;
+    for (int i = 0; i < n; i++) {
+        const int32_t* s = shape_of(i);
+        const int threads = s[0], n_tb = s[1], shmem = s[2], sync = s[3], func = s[4];
+        if (threads < 1 || threads > 1024 || n_tb < 1 || shmem < 0) return -EINVAL;
+        const int wtb = (threads + 31) / 32;
+        if ((long)wtb * n_tb > c->max_task_warps) return -EINVAL;
+        const uint32_t gtb = ((uint32_t)shmem + PAGODA_GRANULE - 1) / PAGODA_GRANULE;
+        if ((uint64_t)gtb * (uint64_t)n_tb > c->max_task_granules) return -EINVAL;
+        if (sync && wtb > 1 && n_tb > PAGODA_BAR_IDS) return -EINVAL;
+        if (!known_func(func)) return -EINVAL;
+    }
+    const char* a = static_cast<const char*>(args_base);
+    for (int base = 0; base < n; base += kSpawnChunk) {
+        const int m = std::min(kSpawnChunk, n - base);
+        const uint64_t id0 = c->next_id.fetch_add((uint64_t)m, std::memory_order_acq_rel);
+        const uint64_t last = id0 + (uint64_t)m - 1;
+        if (last >= c->R && c->consumed_cache.load(std::memory_order_acquire) <= last - c->R) {
+            int rc = spin_until(c, [&] {
+                const uint64_t v = c->hctl->consumed;
+                uint64_t cur = c->consumed_cache.load(std::memory_order_relaxed);
+                while (v > cur && !c->consumed_cache.compare_exchange_weak(cur, v)) { }
+                return v > last - c->R;
+            });
+            if (rc) return rc;
+        }
+        if (last >= c->C && c->low.load(std::memory_order_acquire) <= last - c->C) {
+            int rc = spin_until(c, [&] {
+                advance_low(c, last - c->C + 1);
+                return c->low.load(std::memory_order_acquire) > last - c->C;
+            });
+            if (rc) return rc;
+        }
+        int64_t w_chunk[kSpawnChunk];
+        for (int i = 0; i < m; i++) {
+            const int32_t* s = shape_of(base + i);
+            const uint64_t id = id0 + (uint64_t)i;
+            TaskEntry e;
+            memset(&e, 0, sizeof e);
+            const int wtb = (s[0] + 31) / 32;
+            e.id = id;
+            e.func_id = (uint16_t)s[4];
+            e.threads_tb = (uint16_t)s[0];
+            e.warps_tb = (uint8_t)wtb;
+            e.n_tb = (uint8_t)s[1];
+            e.gran_tb = (uint8_t)(((uint32_t)s[2] + PAGODA_GRANULE - 1) / PAGODA_GRANULE);
+            e.flags = s[3] ? 1 : 0;
+            e.shmem_bytes = (uint32_t)s[2];
+            if (args_bytes) memcpy(e.args, a + (size_t)(base + i) * args_stride, args_bytes);
+            const __m128i* src = reinterpret_cast<const __m128i*>(&e);
+            __m128i* d = reinterpret_cast<__m128i*>(&c->hring[id & (c->R - 1)]);
+            _mm_store_si128(d + 0, _mm_load_si128(src + 0));
+            _mm_store_si128(d + 1, _mm_load_si128(src + 1));
+            _mm_store_si128(d + 2, _mm_load_si128(src + 2));
+            _mm_store_si128(d + 3, _mm_load_si128(src + 3));
+            w_chunk[i] = (int64_t)wtb * s[1];
+            if (ids_out) ids_out[base + i] = (pagoda_task_t)id;
+        }
+        if (c->published.load(std::memory_order_acquire) != id0) {
+            int rc = spin_until(c, [&] { return c->published.load(std::memory_order_acquire) == id0; });
+            if (rc) return rc;
+        }
+        int64_t ws = c->warps_spawned.load(std::memory_order_relaxed);
+        for (int i = 0; i < m; i++) {
+            ws += w_chunk[i];
+            c->warps_prefix[(id0 + (uint64_t)i) & (c->C - 1)] = ws;
+        }
+        c->warps_spawned.store(ws, std::memory_order_relaxed);
+        std::atomic_thread_fence(std::memory_order_release);
+        c->hctl->published = last + 1;
+        c->published.store(last + 1, std::memory_order_release);
+    }
+    return n;
+}
+
+extern "C" {
+
 int64_t pagoda_taskSpawnMany(pagoda_ctx* c, int n, int threads, int n_tb, int shmem_bytes, int sync_flag, int func_id,
                              const void* args_base, size_t args_stride, size_t args_bytes, pagoda_task_t* ids_out)
 {
-    const char* a = static_cast<const char*>(args_base);
-    for (int i = 0; i < n; i++) {
-        pagoda_task_t id = pagoda_taskSpawn(c, threads, n_tb, shmem_bytes, sync_flag, func_id,
-                                            a ? a + (size_t)i * args_stride : nullptr, args_bytes);
-        if (id < 0) return id;
-        if (ids_out) ids_out[i] = id;
-    }
-    return n;
+    const int32_t shape[5] = {threads, n_tb, shmem_bytes, sync_flag, func_id};
+    return spawn_batch(c, n, [&](int) { return shape; }, args_base, args_stride, args_bytes, ids_out);
 }
 
 int64_t pagoda_taskSpawnShapes(pagoda_ctx* c, int n, const int32_t* shapes, const void* args_base, size_t args_stride,
                                size_t args_bytes, pagoda_task_t* ids_out)
 {
-    const char* a = static_cast<const char*>(args_base);
-    for (int i = 0; i < n; i++) {
-        const int32_t* s = shapes + 5 * (size_t)i;
-        pagoda_task_t id =
-            pagoda_taskSpawn(c, s[0], s[1], s[2], s[3], s[4], a ? a + (size_t)i * args_stride : nullptr, args_bytes);
-        if (id < 0) return id;
-        if (ids_out) ids_out[i] = id;
-    }
-    return n;
+    if (!shapes && n > 0) return -EINVAL;
+    return spawn_batch(c, n, [&](int i) { return shapes + 5 * (size_t)i; }, args_base, args_stride, args_bytes,
+                       ids_out);
 }
 
 int pagoda_check(pagoda_ctx* c, pagoda_task_t id)
