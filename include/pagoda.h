@@ -102,6 +102,11 @@ int pagoda_check(pagoda_ctx* ctx, pagoda_task_t id);
  * the call is done.  Returns 0, -EIO, -ETIMEDOUT. */
 int pagoda_waitAll(pagoda_ctx* ctx);
 
+/* Block until every task with id < end is done (ids issued later are not
+ * waited for).  For callers that pipeline copies per spawn batch.  Returns 0,
+ * -EINVAL, -EIO, -ETIMEDOUT, -EAGAIN (session stopped). */
+int pagoda_waitBelow(pagoda_ctx* ctx, pagoda_task_t end);
+
 /* Convenience for C and Python callers: spawn n tasks of one shape, task i's
  * args at args_base + i*args_stride (args_bytes each); each is a separate
  * pagoda_taskSpawn.  ids_out (nullable) receives the ids.  Returns the number

@@ -308,11 +308,23 @@ __device__ void body_fb(const Env& e, const pagoda_fb_args& a)
     float* vd = (e.getSMBytes() >= 1024) ? reinterpret_cast<float*>(e.getSMPtr())
                                          : a.scratch + 256 * e.getBlockIdx();
     const int n = tb_threads(e), bt = e.getBlockTid();
-    for (int m = bt; m < 256; m += n) {
-        float acc = 0.0f;
-        const int kmax = min(31, 8 * m);
-        for (int k = 0; k <= kmax; k++) acc = __fmaf_rn(a.H[k], a.r[8 * m - k], acc);
-        vd[m] = acc;
+    /* four VD chains per thread advance together (ILP); r outside [0, 2048) reads as 0, and an
+     * fma with a zero factor leaves the (never -0) accumulator unchanged: identical to skipping */
+    for (int m0 = bt; m0 < 256; m0 += 4 * n) {
+        float acc[4] = {0.0f, 0.0f, 0.0f, 0.0f};
+#pragma unroll 8
+        for (int k = 0; k < 32; k++) {
+            const float hk = a.H[k];
+#pragma unroll
+            for (int i = 0; i < 4; i++) {
+                const int idx = 8 * (m0 + i * n) - k;
+                const float rv = (m0 + i * n < 256 && idx >= 0) ? a.r[idx] : 0.0f;
+                acc[i] = __fmaf_rn(hk, rv, acc[i]);
+            }
+        }
+#pragma unroll
+        for (int i = 0; i < 4; i++)
+            if (m0 + i * n < 256) vd[m0 + i * n] = acc[i];
     }
     e.syncBlock();
     const int T = total_threads(e);
@@ -344,17 +356,17 @@ __device__ void body_bf(const Env& e, const pagoda_bf_args& a)
     const float2* h = reinterpret_cast<const float2*>(a.h);
     const float2* w = reinterpret_cast<const float2*>(a.w);
     for (int t = e.getTid(); t < 512; t += T) {
-        float vr[4], vi[4];
+        /* all 16 taps of all 4 channels unrolled: 8 independent fma chains; x before the
+         * start of the signal reads as 0 (exact: see FB) */
+        float vr[4] = {0.0f, 0.0f, 0.0f, 0.0f}, vi[4] = {0.0f, 0.0f, 0.0f, 0.0f};
 #pragma unroll
-        for (int c = 0; c < 4; c++) {
-            float re = 0.0f, im = 0.0f;
-            const int kmax = min(15, t);
-            for (int k = 0; k <= kmax; k++) {
-                const float2 hk = h[c * 16 + k], xv = x[c * 512 + t - k];
-                cmac(re, im, hk.x, hk.y, xv.x, xv.y);
+        for (int k = 0; k < 16; k++) {
+#pragma unroll
+            for (int c = 0; c < 4; c++) {
+                const float2 hk = h[c * 16 + k];
+                const float2 xv = (t - k >= 0) ? x[c * 512 + t - k] : make_float2(0.0f, 0.0f);
+                cmac(vr[c], vi[c], hk.x, hk.y, xv.x, xv.y);
             }
-            vr[c] = re;
-            vi[c] = im;
         }
 #pragma unroll
         for (int b = 0; b < 4; b++) {
@@ -383,20 +395,53 @@ __device__ void body_conv(const Env& e, const pagoda_conv_args& a)
     const int t0 = max(0, r0 - 8), t1 = min(128, r1 + 8);
     float* tmp = a.scratch + 16384 * j;
     const int n = tb_threads(e), bt = e.getBlockTid();
-    for (int idx = t0 * 128 + bt; idx < t1 * 128; idx += n) {
-        const int y = idx >> 7, x = idx & 127;
-        float acc = 0.0f;
-        for (int d = -8; d <= 8; d++)
-            if (x + d >= 0 && x + d < 128) acc = __fmaf_rn(a.img[y * 128 + x + d], a.krow[8 - d], acc);
-        tmp[idx] = acc;
+    /* Each thread produces 4 neighbouring outputs with a sliding register window: per tap one
+     * new input load, one kernel load and 4 independent fma chains.  Samples outside the image
+     * read as 0, which is exact (an fma with a zero factor leaves the accumulator unchanged). */
+    for (int item = bt; item < (t1 - t0) * 32; item += n) {           /* row pass */
+        const int y = t0 + (item >> 5), x0 = (item & 31) * 4;
+        const float* row = a.img + y * 128;
+        auto in = [&](int xx) { return (xx >= 0 && xx < 128) ? row[xx] : 0.0f; };
+        float w0 = in(x0 - 8), w1 = in(x0 - 7), w2 = in(x0 - 6), w3 = in(x0 - 5);
+        float c0 = 0.0f, c1 = 0.0f, c2 = 0.0f, c3 = 0.0f;
+#pragma unroll
+        for (int d = -8; d <= 8; d++) {
+            const float k = a.krow[8 - d];
+            c0 = __fmaf_rn(w0, k, c0);
+            c1 = __fmaf_rn(w1, k, c1);
+            c2 = __fmaf_rn(w2, k, c2);
+            c3 = __fmaf_rn(w3, k, c3);
+            w0 = w1;
+            w1 = w2;
+            w2 = w3;
+            if (d < 8) w3 = in(x0 + 4 + d);
+        }
+        *reinterpret_cast<float4*>(tmp + y * 128 + x0) = make_float4(c0, c1, c2, c3);
     }
     e.syncBlock();
-    for (int idx = r0 * 128 + bt; idx < r1 * 128; idx += n) {
-        const int y = idx >> 7, x = idx & 127;
-        float acc = 0.0f;
-        for (int d = -8; d <= 8; d++)
-            if (y + d >= 0 && y + d < 128) acc = __fmaf_rn(tmp[(y + d) * 128 + x], a.kcol[8 - d], acc);
-        a.out[idx] = acc;
+    const int groups = (r1 - r0 + 3) / 4;
+    for (int item = bt; item < groups * 128; item += n) {             /* column pass */
+        const int x = item & 127, y0 = r0 + (item >> 7) * 4;
+        auto tv = [&](int yy) { return (yy >= 0 && yy < 128) ? tmp[yy * 128 + x] : 0.0f; };
+        float w0 = tv(y0 - 8), w1 = tv(y0 - 7), w2 = tv(y0 - 6), w3 = tv(y0 - 5);
+        float c0 = 0.0f, c1 = 0.0f, c2 = 0.0f, c3 = 0.0f;
+#pragma unroll
+        for (int d = -8; d <= 8; d++) {
+            const float k = a.kcol[8 - d];
+            c0 = __fmaf_rn(w0, k, c0);
+            c1 = __fmaf_rn(w1, k, c1);
+            c2 = __fmaf_rn(w2, k, c2);
+            c3 = __fmaf_rn(w3, k, c3);
+            w0 = w1;
+            w1 = w2;
+            w2 = w3;
+            if (d < 8) w3 = tv(y0 + 4 + d);
+        }
+        float* o = a.out + y0 * 128 + x;
+        if (y0 + 0 < r1) o[0] = c0;       /* rows of another TB's band (or past the image) are */
+        if (y0 + 1 < r1) o[128] = c1;     /* computed from values this TB never wrote: dropped */
+        if (y0 + 2 < r1) o[256] = c2;
+        if (y0 + 3 < r1) o[384] = c3;
     }
 }
 
@@ -412,22 +457,42 @@ __device__ void body_dct(const Env& e, const pagoda_dct_args& a)
         const int blk = item >> 3, u = item & 7;
         const int by = blk >> 4, bx = blk & 15;
         const float* X = a.img + (by * 8) * 128 + bx * 8;
-        float Tu[8];
+        /* row x of the block arrives as two float4; the 8 chains T[u][*] advance together
+         * (each still accumulates over x ascending) */
+        float Tu[8] = {0.0f, 0.0f, 0.0f, 0.0f, 0.0f, 0.0f, 0.0f, 0.0f};
 #pragma unroll
-        for (int y = 0; y < 8; y++) {
-            float acc = 0.0f;
-#pragma unroll
-            for (int x = 0; x < 8; x++) acc = __fmaf_rn(a.coef[u * 8 + x], X[x * 128 + y], acc);
-            Tu[y] = acc;
+        for (int x = 0; x < 8; x++) {
+            const float cu = a.coef[u * 8 + x];
+            const float4 lo = *reinterpret_cast<const float4*>(X + x * 128);
+            const float4 hi = *reinterpret_cast<const float4*>(X + x * 128 + 4);
+            Tu[0] = __fmaf_rn(cu, lo.x, Tu[0]);
+            Tu[1] = __fmaf_rn(cu, lo.y, Tu[1]);
+            Tu[2] = __fmaf_rn(cu, lo.z, Tu[2]);
+            Tu[3] = __fmaf_rn(cu, lo.w, Tu[3]);
+            Tu[4] = __fmaf_rn(cu, hi.x, Tu[4]);
+            Tu[5] = __fmaf_rn(cu, hi.y, Tu[5]);
+            Tu[6] = __fmaf_rn(cu, hi.z, Tu[6]);
+            Tu[7] = __fmaf_rn(cu, hi.w, Tu[7]);
         }
-        float* Y = a.out + (by * 8 + u) * 128 + bx * 8;
+        float Yv[8];
 #pragma unroll
         for (int v = 0; v < 8; v++) {
+            const float4 clo = *reinterpret_cast<const float4*>(a.coef + v * 8);
+            const float4 chi = *reinterpret_cast<const float4*>(a.coef + v * 8 + 4);
             float acc = 0.0f;
-#pragma unroll
-            for (int y = 0; y < 8; y++) acc = __fmaf_rn(Tu[y], a.coef[v * 8 + y], acc);
-            Y[v] = acc;
+            acc = __fmaf_rn(Tu[0], clo.x, acc);
+            acc = __fmaf_rn(Tu[1], clo.y, acc);
+            acc = __fmaf_rn(Tu[2], clo.z, acc);
+            acc = __fmaf_rn(Tu[3], clo.w, acc);
+            acc = __fmaf_rn(Tu[4], chi.x, acc);
+            acc = __fmaf_rn(Tu[5], chi.y, acc);
+            acc = __fmaf_rn(Tu[6], chi.z, acc);
+            acc = __fmaf_rn(Tu[7], chi.w, acc);
+            Yv[v] = acc;
         }
+        float* Y = a.out + (by * 8 + u) * 128 + bx * 8;
+        *reinterpret_cast<float4*>(Y) = make_float4(Yv[0], Yv[1], Yv[2], Yv[3]);
+        *reinterpret_cast<float4*>(Y + 4) = make_float4(Yv[4], Yv[5], Yv[6], Yv[7]);
     }
 }
 

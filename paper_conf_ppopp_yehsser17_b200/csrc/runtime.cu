@@ -560,6 +560,18 @@ int pagoda_wait(pagoda_ctx* c, pagoda_task_t id)
     return rc;
 }
 
+int pagoda_waitBelow(pagoda_ctx* c, pagoda_task_t end)
+{
+    if (!c || end < 0) return -EINVAL;
+    const uint64_t n = std::min<uint64_t>((uint64_t)end, c->next_id.load(std::memory_order_acquire));
+    int rc = spin_until(c, [&] {
+        advance_low(c, n);
+        return c->low.load(std::memory_order_acquire) >= n;
+    });
+    std::atomic_thread_fence(std::memory_order_acquire);
+    return rc;
+}
+
 int pagoda_waitAll(pagoda_ctx* c)
 {
     if (!c) return -EINVAL;

@@ -61,6 +61,7 @@ def lib() -> C.CDLL:
         L.pagoda_wait.argtypes = [P, I64]
         L.pagoda_check.argtypes = [P, I64]
         L.pagoda_waitAll.argtypes = [P]
+        L.pagoda_waitBelow.argtypes = [P, I64]
         L.pagoda_taskSpawnMany.argtypes = [P, I, I, I, I, I, I, P, SZ, SZ, P]
         L.pagoda_taskSpawnMany.restype = I64
         L.pagoda_taskSpawnShapes.argtypes = [P, I, P, P, SZ, SZ, P]
@@ -149,6 +150,9 @@ class Pagoda:
 
     def waitAll(self) -> int:
         return lib().pagoda_waitAll(self.h)
+
+    def waitBelow(self, end: int) -> int:
+        return lib().pagoda_waitBelow(self.h, end)
 
     # --- batch conveniences (each task is still one taskSpawn in C) --------
     def spawn_many(self, n, threads, n_tb, shmem, sync, func_id, args: np.ndarray | None, ids=False):
