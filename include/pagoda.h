@@ -34,7 +34,8 @@ typedef int64_t pagoda_task_t;          /* >= 0: task id; < 0: -errno */
 /* ---- limits fixed by the design ---------------- */
 #define PAGODA_ARGS_MAX      40   /* bytes of inline task arguments per TaskTable entry */
 #define PAGODA_GRANULE       512  /* shared-memory allocation granule */
-#define PAGODA_MAX_EXEC_WARPS 31  /* executor warps per MTB: warp 0 schedules */
+#define PAGODA_MAX_EXEC_WARPS 32  /* worker warps per MTB: every warp executes; the paper's dedicated
+                                     scheduler warp is a token passed between them */
 #define PAGODA_BAR_IDS       15   /* named barriers 1..15 per MTB; 0 is the MTB's own */
 
 /* config flags */
@@ -50,7 +51,7 @@ typedef struct {
     uint32_t ring_entries;  /* TaskTable ring entries, host and device, power of 2 (default 65536) */
     uint32_t comp_entries;  /* completion window, power of 2 >= ring_entries (default 1<<20) */
     uint32_t arena_bytes;   /* shared-memory arena per MTB, multiple of 512 (default 96 KiB at 2 MTB/SM) */
-    uint32_t exec_warps;    /* executor warps per MTB, 1..31 (default 31; fewer = debug config) */
+    uint32_t exec_warps;    /* worker warps per MTB, 1..32 (default 32; fewer = debug config) */
     uint32_t flags;         /* PAGODA_TRACE */
     uint32_t trace_events;  /* ledger capacity per MTB when PAGODA_TRACE (default 8192) */
     double   watchdog_s;    /* wait/waitAll/shutdown give up with -ETIMEDOUT after this many
@@ -82,8 +83,8 @@ int pagoda_shutdown(pagoda_ctx* ctx);
  * only while the TaskTable ring or completion window is full, as the paper's
  * CPU does when no entry is free).
  * Returns the task id (>= 0, strictly increasing per context) or
- *   -EINVAL  threads < 1, n_threadblocks < 1, ceil(threads/32)*n_tb > executor
- *            warps per MTB (all warps of a task live in one MTB),
+ *   -EINVAL  threads < 1 or > 1024, n_threadblocks < 1, ceil(threads/32)*n_tb > worker
+ *            warps per MTB (32; all warps of a task live in one MTB),
  *            n_tb * round_up(shmem, 512) > arena, sync with > 15 multi-warp TBs,
  *            unknown func_id, args_bytes > 40 or args NULL with args_bytes > 0;
  *   -ESHUTDOWN after pagoda_shutdown began;  -EIO after a device fault. */

@@ -42,7 +42,7 @@ struct WarpSlot {
 };
 static_assert(sizeof(WarpSlot) == 32, "WarpSlot is 32 bytes");
 
-enum : uint8_t { SLOT_TERMINATE = 0xFF };
+enum : uint8_t { SLOT_TERMINATE = 0xFF, SLOT_SCHED = 0xFE /* take over the scheduler token */ };
 
 /* Byte offsets inside the MTB's dynamic shared memory (the control block is
  * laid out in csrc/mk_layout.cuh, which static_asserts them).  The task arena

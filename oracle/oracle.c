@@ -498,8 +498,8 @@ int orc_ledger_check(const orc_ledger_event* ev_in, size_t n_ev, int n_mtb, int 
     memcpy(ev, ev_in, n_ev * sizeof *ev);
     qsort(ev, n_ev, sizeof *ev, ev_cmp);
 
-    uint32_t valid_w = 0;
-    for (int w = 1; w <= exec_warps; w++) valid_w |= 1u << w;
+    uint32_t valid_w = 0;   /* worker warps 0..exec_warps-1 (every warp executes) */
+    for (int w = 0; w < exec_warps && w < 32; w++) valid_w |= 1u << w;
 
     for (size_t i = 0; i < n_ev; i++) {
         const orc_ledger_event* e = &ev[i];

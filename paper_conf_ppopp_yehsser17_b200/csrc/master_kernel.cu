@@ -2,10 +2,11 @@
  * master_kernel.cu — the persistent MasterKernel (Fig. 1b).
  *
  * Grid: one cooperative launch of n_mtb = num_sms * mtbs_per_sm thread blocks
- * ("MTBs") of 1024 threads.  In every MTB warp 0 is the scheduler
- * and warps 1..31 are executors.  Warp 31 of MTB 0 is instead the
- * ingest warp that moves published TaskTable entries from the pinned host ring
- * into the device ring.
+ * ("MTBs") of 1024 threads.  The paper makes warp 0 of every MTB its
+ * scheduler and warps 1..31 executors; here every warp executes and
+ * the scheduler is a token the warps pass around (self-scheduling, see below).
+ * Warp 31 of MTB 0 is instead the ingest warp that moves published TaskTable
+ * entries from the pinned host ring into the device ring.
  *
  *   host ring --(ingest: LDGSTS over PCIe -> smem -> L2 device ring)--> device ring
  *   device ring --(scheduler: fetch-add tickets, per-cell sequence numbers)--> MTB task slots
@@ -165,52 +166,46 @@ __device__ __forceinline__ void trace_ev(const MkParams& p, int mtb, uint32_t& s
     seq++;
 }
 
-/* ------------------------------------------------------------------ executor
- * Alg. 1 L29-43: wait for dispatch, run the body, then the
- * deferred release: the last warp of a TB returns its shmem granules and
- * barrier ID through the scheduler's mailbox (markSMForDealloc), the last warp
- * of the task posts its completion record, every warp returns itself. */
-__device__ void executor(MtbShared& S, char* smem_base, const MkParams& p, int mtb, int w, uint32_t resident)
+/* ------------------------------------------------------------------ task execution
+ * Alg. 1 L29-43: run the body, then the deferred release: the last
+ * warp of a TB returns its shmem granules and barrier ID through the mailbox
+ * (markSMForDealloc), the last warp of the task posts its completion record,
+ * every warp returns itself. */
+__device__ __forceinline__ void run_task(MtbShared& S, char* smem_base, const MkParams& p, int mtb, int w,
+                                         uint32_t resident, uint32_t& stage_phase, const WarpSlot& s)
 {
     const uint32_t lane = threadIdx.x & 31u;
-    uint32_t phase = 0, stage_phase = 0;
-    for (;;) {
-        mbar_wait(&S.exec_bar[w], phase);
-        phase ^= 1u;
-        const WarpSlot s = S.wt[w];
-        if (s.task == SLOT_TERMINATE) return;
-        const TaskEntry& t = S.tasks[s.task];
-        uint64_t t0 = 0;
-        if (p.trace_cap) t0 = globaltimer_ns();
-        TaskEnv env{s, smem_base, &S.stage_bar[w], &stage_phase, &p.dctl->error,
-                    resident};
-        if (!run_body(t.func_id, env, t.args) && lane == 0) atomicOr(&p.dctl->error, PAGODA_DEVERR_BAD_FUNC);
-        __syncwarp();
-        if (lane == 0) {
-            /* this warp's global writes -> visible GPU-wide before anyone learns the warp is done */
-            __threadfence();
-            if (p.trace_cap) {
-                uint32_t* cnt = &p.exec_count[mtb * 32 + w];
-                const uint32_t i = *cnt;
-                if (i < p.trace_cap) {
-                    ExecRecord r{s.task_id, s.tb, (uint16_t)mtb, (uint16_t)w, t0, globaltimer_ns()};
-                    p.exec_trace[((size_t)mtb * 32 + w) * p.trace_cap + i] = r;
-                }
-                *cnt = i + 1;
+    const TaskEntry& t = S.tasks[s.task];
+    uint64_t t0 = 0;
+    if (p.trace_cap) t0 = globaltimer_ns();
+    TaskEnv env{s, smem_base, &S.stage_bar[w], &stage_phase, &p.dctl->error, resident};
+    if (!run_body(t.func_id, env, t.args) && lane == 0) atomicOr(&p.dctl->error, PAGODA_DEVERR_BAD_FUNC);
+    __syncwarp();
+    if (lane == 0) {
+        /* this warp's global writes -> visible GPU-wide before anyone learns the warp is done */
+        __threadfence();
+        if (p.trace_cap) {
+            uint32_t* cnt = &p.exec_count[mtb * 32 + w];
+            const uint32_t i = *cnt;
+            if (i < p.trace_cap) {
+                ExecRecord r{s.task_id, s.tb, (uint16_t)mtb, (uint16_t)w, t0, globaltimer_ns()};
+                p.exec_trace[((size_t)mtb * 32 + w) * p.trace_cap + i] = r;
             }
-            if (atomicSub(&S.tb_warps_left[s.tbslot], 1u) == 1u) atomicOr(&S.mb_tbs, 1u << s.tbslot);
-            if (atomicSub(&S.task_warps_left[s.task], 1u) == 1u) {
-                /* last warp of the task (Alg. 1 L41-42): the task's writes, ordered before the
-                 * counter decrements of all its warps, become visible system-wide before the
-                 * completion record the host polls (a posted PCIe write, no handshake). */
-                st_release_sys(&p.comp[s.task_id & p.comp_mask], (int64_t)s.task_id);
-                atomicOr(&S.mb_tasks, 1u << s.task);
-            }
-            __threadfence_block();   /* TB / task frees are visible before the warp frees itself */
-            atomicOr(&S.mb_warps, 1u << w);
+            *cnt = i + 1;
         }
-        __syncwarp();
+        if (atomicSub(&S.tb_warps_left[s.tbslot], 1u) == 1u) atomicOr(&S.mb_tbs, 1u << s.tbslot);
+        if (atomicSub(&S.task_warps_left[s.task], 1u) == 1u) {
+            /* last warp of the task (Alg. 1 L41-42): the task's writes, ordered before the
+             * counter decrements of all its warps, become visible system-wide before the
+             * completion record the host polls (a posted PCIe write, no handshake). */
+            st_release_sys(&p.comp[s.task_id & p.comp_mask], (int64_t)s.task_id);
+            atomicOr(&S.mb_tasks, 1u << s.task);
+        }
+        __threadfence_block();   /* TB / task frees are visible before the warp frees itself */
+        atomicOr(&S.mb_warps, 1u << w);
+        __threadfence_block();   /* ... and the warp's free bit before its attempt at the token */
     }
+    __syncwarp();
 }
 
 /* ------------------------------------------------------------------ ingest
@@ -472,96 +467,217 @@ __device__ int sched_load(MtbShared& S, Sched& st, const MkParams& p)
     return (int)r;
 }
 
-__device__ void scheduler(MtbShared& S, const MkParams& p, int mtb, int arena_granules)
+/* ------------------------------------------------------------------ self-scheduling
+ * The paper dedicates warp 0 of every MTB to scheduling.  Here the
+ * scheduler is a TOKEN in shared memory instead: the warp holding it runs
+ * scheduling rounds; a warp that finishes a task posts its frees and tries to
+ * take the token; a holder that dispatches a task to itself hands the token to
+ * another free warp (or releases it when none is free).  Invariant: either some
+ * warp holds the token, or every worker is running a task (and the next one to
+ * finish takes it).  So every warp of the MTB executes tasks: eight 4-warp tasks
+ * per MTB instead of seven (SURVEY App. A "v2: self-scheduling"). */
+__device__ __forceinline__ void sst_save(MtbShared& S, const Sched& st)
 {
     const uint32_t lane = threadIdx.x & 31u;
-    Sched st;
-    st.exec_mask = 0;
-    for (int w = 1; w <= p.exec_warps && w < 32; w++)
-        if (!(mtb == 0 && w == kIngestWarp)) st.exec_mask |= 1u << w;
-    st.free_w = st.exec_mask;
-    st.free_task = 0xffffffffu;
-    st.free_tbs = 0xffffffffu;
-    st.free_bar = 0xfffeu;        /* named barriers 1..15; 0 belongs to the MTB */
-    st.fg = bm_range_bits(0, (uint32_t)arena_granules, lane);
-    st.ph = st.pl = st.pt = 0;
-    st.est_w = 0;
-    st.seq = 0;
-    uint32_t backoff = 0;
+    S.sst_fg[lane] = st.fg;
+    if (lane == 0) {
+        S.sst_free_w = st.free_w;
+        S.sst_free_task = st.free_task;
+        S.sst_free_tbs = st.free_tbs;
+        S.sst_free_bar = st.free_bar;
+        S.sst_ph = st.ph;
+        S.sst_pl = st.pl;
+        S.sst_pt = st.pt;
+        S.sst_est_w = st.est_w;
+        S.sst_seq = st.seq;
+    }
+    __syncwarp();
+}
+
+__device__ __forceinline__ void sst_load(MtbShared& S, Sched& st, uint32_t exec_mask)
+{
+    __syncwarp();
+    st.fg = S.sst_fg[threadIdx.x & 31u];
+    st.free_w = S.sst_free_w;
+    st.free_task = S.sst_free_task;
+    st.free_tbs = S.sst_free_tbs;
+    st.free_bar = S.sst_free_bar;
+    st.ph = S.sst_ph;
+    st.pl = S.sst_pl;
+    st.pt = S.sst_pt;
+    st.est_w = S.sst_est_w;
+    st.seq = S.sst_seq;
+    st.exec_mask = exec_mask;
+}
+
+__device__ __forceinline__ bool token_try(MtbShared& S)
+{
+    uint32_t got = 0;
+    if ((threadIdx.x & 31u) == 0) {
+        got = atomicCAS(&S.token, 0u, 1u) == 0u;
+        __threadfence_block();
+    }
+    return __shfl_sync(0xffffffffu, got, 0) != 0;
+}
+
+__device__ __forceinline__ void token_release(MtbShared& S)
+{
+    __syncwarp();
+    if ((threadIdx.x & 31u) == 0) {
+        __threadfence_block();
+        atomicExch(&S.token, 0u);
+        __threadfence_block();
+    }
+    __syncwarp();
+}
+
+/* fold the mailboxes into the holder's state (deallocMarkedSM, Alg. 1 L22) */
+__device__ bool sched_fold(MtbShared& S, Sched& st, const MkParams& p, int mtb)
+{
+    const uint32_t lane = threadIdx.x & 31u;
+    uint32_t mw = 0, mt = 0, mk = 0;
+    if (lane == 0) {
+        if (*(volatile uint32_t*)&S.mb_warps) mw = atomicExch(&S.mb_warps, 0u);
+        __threadfence_block();
+        if (*(volatile uint32_t*)&S.mb_tbs) mt = atomicExch(&S.mb_tbs, 0u);
+        if (*(volatile uint32_t*)&S.mb_tasks) mk = atomicExch(&S.mb_tasks, 0u);
+    }
+    mw = __shfl_sync(0xffffffffu, mw, 0);
+    mt = __shfl_sync(0xffffffffu, mt, 0);
+    mk = __shfl_sync(0xffffffffu, mk, 0);
+    if (!(mw | mt | mk)) return false;
+    for (uint32_t b = mt; b; b &= b - 1u) {
+        const uint32_t tbs = __ffs(b) - 1;
+        const uint32_t goff = S.tb_goff[tbs], glen = S.tb_glen[tbs], bar = S.tb_bar[tbs];
+        if (glen) st.fg |= bm_range_bits(goff, glen, lane);
+        if (bar) st.free_bar |= 1u << bar;
+        st.free_tbs |= 1u << tbs;
+        if (p.trace_cap)
+            trace_ev(p, mtb, st.seq, 3, S.tb_task[tbs], S.tb_idx[tbs], 0, (uint16_t)goff, (uint16_t)glen, (uint8_t)bar);
+    }
+    if (p.trace_cap) {
+        for (uint32_t b = mw; b; b &= b - 1u) {
+            const uint32_t w = __ffs(b) - 1;
+            trace_ev(p, mtb, st.seq, 2, S.wt[w].task_id, S.wt[w].tb, 1u << w, 0, 0, 0);
+        }
+    }
+    st.free_w |= mw;
+    st.free_task |= mk;
+    return true;
+}
+
+/* One scheduling round: fold, load published tickets, place in FIFO order
+ * (Alg. 1 L14-28), take more tickets.  Sets exit when the session is over. */
+__device__ bool sched_round(MtbShared& S, Sched& st, const MkParams& p, int mtb, bool& exit)
+{
+    const uint32_t lane = threadIdx.x & 31u;
+    bool progress = sched_fold(S, st, p, mtb);
+    if (st.pl != st.pt && sched_load(S, st, p) > 0) progress = true;
+    while (st.ph != st.pl) {
+        if (!sched_place(S, st, p, mtb, S.pend[st.ph & 31u])) break;
+        st.ph++;
+        progress = true;
+    }
+    /* MTB 0 (one warp short: it hosts the ingest warp) takes no blind tickets unless it is the
+     * only MTB (validation then caps every task to its capacity), so no ticket lands where it
+     * can never fit */
+    if ((mtb != 0 || p.n_mtb == 1) && sched_claim(S, st, p) > 0) progress = true;
+    exit = false;
+    if (!progress && st.free_w == st.exec_mask && st.ph == st.pl) {
+        uint32_t stop = 0;
+        if (lane == 0) stop = ld_acquire_gpu32(&p.dctl->stop);
+        stop = __shfl_sync(0xffffffffu, stop, 0);
+        if (stop == kStopAbort) exit = true;   /* host watchdog gave up */
+        else if (stop) {
+            uint64_t tail = 0;
+            if (lane == 0) tail = ld_acquire_gpu(&p.dctl->tail);
+            tail = __shfl_sync(0xffffffffu, tail, 0);
+            /* after stop the tail is final: tickets at or past it are void */
+            exit = st.pl == st.pt || S.pend_ticket[st.pl & 31u] >= tail;
+        }
+    }
+    return progress;
+}
+
+/* The holder w has dispatched a task to itself: pass the token to another free
+ * warp (it wakes with a SCHED slot), else release it — re-checking the mailbox
+ * afterwards so a warp that freed itself meanwhile, and failed to take the
+ * token, is not left without a scheduler. */
+__device__ void sched_handoff(MtbShared& S, Sched& st, const MkParams& p, int mtb)
+{
+    const uint32_t lane = threadIdx.x & 31u;
     for (;;) {
-        bool progress = false;
-        /* ---- fold the mailboxes (deallocMarkedSM, Alg. 1 L22) */
-        uint32_t mw = 0, mt = 0, mk = 0;
-        if (lane == 0) {
-            if (*(volatile uint32_t*)&S.mb_warps) mw = atomicExch(&S.mb_warps, 0u);
-            __threadfence_block();
-            if (*(volatile uint32_t*)&S.mb_tbs) mt = atomicExch(&S.mb_tbs, 0u);
-            if (*(volatile uint32_t*)&S.mb_tasks) mk = atomicExch(&S.mb_tasks, 0u);
-        }
-        mw = __shfl_sync(0xffffffffu, mw, 0);
-        mt = __shfl_sync(0xffffffffu, mt, 0);
-        mk = __shfl_sync(0xffffffffu, mk, 0);
-        if (mw | mt | mk) {
-            progress = true;
-            for (uint32_t b = mt; b; b &= b - 1u) {
-                const uint32_t tbs = __ffs(b) - 1;
-                const uint32_t goff = S.tb_goff[tbs], glen = S.tb_glen[tbs], bar = S.tb_bar[tbs];
-                if (glen) st.fg |= bm_range_bits(goff, glen, lane);
-                if (bar) st.free_bar |= 1u << bar;
-                st.free_tbs |= 1u << tbs;
-                if (p.trace_cap)
-                    trace_ev(p, mtb, st.seq, 3, S.tb_task[tbs], S.tb_idx[tbs], 0, (uint16_t)goff, (uint16_t)glen,
-                             (uint8_t)bar);
+        sched_fold(S, st, p, mtb);
+        if (st.free_w) {
+            const uint32_t h = __ffs(st.free_w) - 1;
+            sst_save(S, st);
+            if (lane == h) {
+                S.wt[h].task = SLOT_SCHED;
+                mbar_arrive(&S.exec_bar[h]);   /* release: the saved state is visible to h */
             }
-            if (p.trace_cap) {
-                for (uint32_t b = mw; b; b &= b - 1u) {
-                    const uint32_t w = __ffs(b) - 1;
-                    trace_ev(p, mtb, st.seq, 2, S.wt[w].task_id, S.wt[w].tb, 1u << w, 0, 0, 0);
+            __syncwarp();
+            return;
+        }
+        sst_save(S, st);
+        token_release(S);
+        uint32_t pending = 0;
+        if (lane == 0) pending = *(volatile uint32_t*)&S.mb_warps;
+        pending = __shfl_sync(0xffffffffu, pending, 0);
+        if (!pending || !token_try(S)) return;
+        sst_load(S, st, st.exec_mask);
+    }
+}
+
+/* Every worker warp runs this loop (warps 0..exec_warps-1; MTB 0's warp 31 ingests). */
+__device__ void worker(MtbShared& S, char* smem_base, const MkParams& p, int mtb, int w, uint32_t resident,
+                       uint32_t exec_mask, bool holder)
+{
+    const uint32_t lane = threadIdx.x & 31u;
+    uint32_t phase = 0, stage_phase = 0, backoff = 0;
+    Sched st;
+    if (holder) sst_load(S, st, exec_mask);
+    for (;;) {
+        if (holder) {
+            bool exit = false;
+            const bool progress = sched_round(S, st, p, mtb, exit);
+            if (exit) {   /* drain: release every other worker with a terminate slot */
+                if (((exec_mask & ~(1u << w)) >> lane) & 1u) {
+                    S.wt[lane].task = SLOT_TERMINATE;
+                    mbar_arrive(&S.exec_bar[lane]);
                 }
+                if (lane == 0) atomicAdd(&p.dctl->exited, 1u);
+                return;
             }
-            st.free_w |= mw;
-            st.free_task |= mk;
+            if ((st.free_w >> w) & 1u) {   /* still free: keep scheduling */
+                if (progress) backoff = 0;
+                else {
+                    /* with work queued only shared-memory mailboxes are polled: stay responsive;
+                     * otherwise the ring is polled in L2: back off */
+                    backoff = (st.ph != st.pt) ? 32u : (backoff ? min(backoff * 2u, 1024u) : 32u);
+                    __nanosleep(backoff);
+                }
+                continue;
+            }
+            sched_handoff(S, st, p, mtb);   /* dispatched (by itself or before it took the token) */
+            holder = false;
         }
-        /* ---- load published tickets, place loaded tasks in FIFO order (Alg. 1 L14-28) */
-        if (st.pl != st.pt && sched_load(S, st, p) > 0) progress = true;
-        while (st.ph != st.pl) {
-            if (!sched_place(S, st, p, mtb, S.pend[st.ph & 31u])) break;
-            st.ph++;
-            progress = true;
-        }
-        /* ---- take more tickets while resources are free.  MTB 0 (one warp short: it hosts the
-         * ingest warp) does not take blind tickets unless it is the only MTB (validation then
-         * caps every task to its capacity), so no ticket can land where it never fits. */
-        if ((mtb != 0 || p.n_mtb == 1) && sched_claim(S, st, p) > 0) progress = true;
-        if (progress) {
+        mbar_wait(&S.exec_bar[w], phase);
+        phase ^= 1u;
+        const WarpSlot s = S.wt[w];
+        if (s.task == SLOT_TERMINATE) return;
+        if (s.task == SLOT_SCHED) {
+            holder = true;
             backoff = 0;
+            sst_load(S, st, exec_mask);
             continue;
         }
-        /* ---- idle: exit once stopped, drained, and holding no ticket that can still be published */
-        {
-            uint32_t stop = 0;
-            if (lane == 0) stop = ld_acquire_gpu32(&p.dctl->stop);
-            stop = __shfl_sync(0xffffffffu, stop, 0);
-            if (stop == kStopAbort && st.free_w == st.exec_mask) break;   /* host watchdog gave up */
-            if (stop && st.free_w == st.exec_mask && st.ph == st.pl) {
-                uint64_t tail = 0;
-                if (lane == 0) tail = ld_acquire_gpu(&p.dctl->tail);
-                tail = __shfl_sync(0xffffffffu, tail, 0);
-                /* after stop the tail is final: tickets at or past it are void */
-                if (st.pl == st.pt || S.pend_ticket[st.pl & 31u] >= tail) break;
-            }
+        run_task(S, smem_base, p, mtb, w, resident, stage_phase, s);
+        if (token_try(S)) {
+            holder = true;
+            backoff = 0;
+            sst_load(S, st, exec_mask);
         }
-        /* with work queued only shared-memory mailboxes are polled: stay responsive;
-         * otherwise the ring is polled in L2: back off */
-        backoff = (st.ph != st.pt) ? 32u : (backoff ? min(backoff * 2u, 1024u) : 32u);
-        __nanosleep(backoff);
     }
-    /* drain: release every executor warp with a terminate slot */
-    if ((st.exec_mask >> lane) & 1u) {
-        S.wt[lane].task = SLOT_TERMINATE;
-        mbar_arrive(&S.exec_bar[lane]);
-    }
-    if (lane == 0) atomicAdd(&p.dctl->exited, 1u);
 }
 
 /* ------------------------------------------------------------------ the kernel */
@@ -595,18 +711,31 @@ __global__ void __launch_bounds__(1024, kMinBlocks) master_kernel(MkParams p)
             if (threadIdx.x == 0) atomicOr(&p.dctl->error, PAGODA_DEVERR_LAYOUT);
         }
     }
+    /* worker warps 0..exec_warps-1 (MTB 0: minus the ingest warp) */
+    uint32_t exec_mask = p.exec_warps >= 32 ? 0xffffffffu : ((1u << p.exec_warps) - 1u);
+    if (mtb == 0) exec_mask &= ~(1u << kIngestWarp);
+    const int first = __ffs(exec_mask) - 1;
     if (warp == 0) {
         mbar_init(&S.exec_bar[lane], 1);
         mbar_init(&S.stage_bar[lane], 1);
+        /* initial scheduler state, owned by the first worker (it starts with the token) */
+        S.sst_fg[lane] = bm_range_bits(0, (uint32_t)arena_granules, lane);
         if (lane == 0) {
             S.mb_warps = S.mb_tbs = S.mb_tasks = 0;
+            S.sst_free_w = exec_mask;
+            S.sst_free_task = 0xffffffffu;
+            S.sst_free_tbs = 0xffffffffu;
+            S.sst_free_bar = 0xfffeu;   /* named barriers 1..15; 0 belongs to the MTB */
+            S.sst_ph = S.sst_pl = S.sst_pt = 0;
+            S.sst_est_w = 0;
+            S.sst_seq = 0;
+            S.token = 1;
             asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         }
     }
     __syncthreads();
-    if (warp == 0) scheduler(S, p, mtb, arena_granules);
-    else if (mtb == 0 && warp == kIngestWarp) ingest(p, ingest_stage);
-    else if (warp <= p.exec_warps) executor(S, smem_base, p, mtb, warp, resident);
+    if (mtb == 0 && warp == kIngestWarp) ingest(p, ingest_stage);
+    else if ((exec_mask >> warp) & 1u) worker(S, smem_base, p, mtb, warp, resident, exec_mask, warp == first);
 }
 
 template __global__ void master_kernel<1>(MkParams);

@@ -123,6 +123,11 @@ struct MtbShared {
     uint64_t  tb_task[32];           /* 4048: task id of each TB record (ledger) */
     uint16_t  tb_idx[32];            /* 4304: TB index j of each TB record (ledger) */
     uint64_t  pend_ticket[32];       /* 4368: claimed ring positions, FIFO (pend[] holds their slots once loaded) */
+    /* scheduler state while parked between token holders (self-scheduling) */
+    uint32_t  sst_fg[32];            /* 4624: granule bitmap, word l = granules [32l, 32l+32) */
+    uint32_t  sst_free_w, sst_free_task, sst_free_tbs, sst_free_bar;
+    uint32_t  sst_ph, sst_pl, sst_pt, sst_est_w, sst_seq;
+    uint32_t  token;                 /* 1 while some warp holds the scheduler token */
 };
 static_assert(offsetof(MtbShared, wt) == kWarpTableOffset, "WarpTable offset");
 static_assert(sizeof(MtbShared) <= kControlBytes && kControlBytes <= kResidentOffset, "control block fits");

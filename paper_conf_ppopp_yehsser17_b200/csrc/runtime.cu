@@ -145,7 +145,7 @@ void pagoda_config_default(pagoda_config* cfg)
     cfg->ring_entries = 1u << 16;
     cfg->comp_entries = 1u << 20;
     cfg->arena_bytes = 96 * 1024;
-    cfg->exec_warps = 31;
+    cfg->exec_warps = 32;
     cfg->flags = 0;
     cfg->trace_events = 8192;
     cfg->watchdog_s = 60.0;
@@ -248,7 +248,7 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
     if (!pow2(cfg.ring_entries) || !pow2(cfg.comp_entries) || cfg.comp_entries < cfg.ring_entries ||
         cfg.ring_entries < 2 * kSpawnChunk)
         return -EINVAL;
-    if (cfg.exec_warps < 1 || cfg.exec_warps > 31) return -EINVAL;
+    if (cfg.exec_warps < 1 || cfg.exec_warps > 32) return -EINVAL;
     if (cfg.arena_bytes % PAGODA_GRANULE || cfg.arena_bytes / PAGODA_GRANULE > (uint32_t)kMaxGranules ||
         cfg.arena_bytes < kIngestGranules * PAGODA_GRANULE)
         return -EINVAL;
@@ -279,7 +279,7 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
     c->C = cfg.comp_entries;
     const uint32_t arena_g = cfg.arena_bytes / PAGODA_GRANULE;
     if (c->n_mtb == 1) {   /* MTB 0 alone: it also hosts the ingest warp and its staging */
-        c->max_task_warps = cfg.exec_warps == 31 ? 30 : (int)cfg.exec_warps;
+        c->max_task_warps = cfg.exec_warps == 32 ? 31 : (int)cfg.exec_warps;
         c->max_task_granules = arena_g - kIngestGranules;
     } else {
         c->max_task_warps = (int)cfg.exec_warps;

@@ -48,7 +48,7 @@ def test_no_oracle_in_product():
 def test_config_default(L):
     c = PG.default_config()
     assert (c.mtbs_per_sm, c.ring_entries, c.comp_entries, c.arena_bytes, c.exec_warps) == (2, 65536, 1 << 20,
-                                                                                          96 * 1024, 31)
+                                                                                          96 * 1024, 32)
 
 
 def test_init_without_gpu_fails_loudly(L):

@@ -31,7 +31,7 @@ def test_init_info_shutdown():
 
 def test_nop_many_shapes_exactly_once():
     shapes = [(32, 1, 0, 0), (128, 1, 0, 0), (256, 1, 8192, 1), (100, 3, 600, 1), (992, 1, 0, 1), (64, 15, 0, 1),
-              (32, 31, 512, 1)]
+              (32, 31, 512, 1), (1024, 1, 0, 1), (32, 32, 0, 0)]
     with Pagoda() as p:
         ids = []
         for k in range(3000):
@@ -143,13 +143,14 @@ def test_validation_and_shutdown_errors():
     p = Pagoda()
     E = -errno.EINVAL
     assert p.taskSpawn(0, 1, 0, 0, T.NOP) == E
-    assert p.taskSpawn(993, 1, 0, 0, T.NOP) == E
-    assert p.taskSpawn(128, 8, 0, 0, T.NOP) == E
+    assert p.taskSpawn(1025, 1, 0, 0, T.NOP) == E          # > 1024 threads
+    assert p.taskSpawn(128, 9, 0, 0, T.NOP) == E           # 36 warps > 32 per MTB
     assert p.taskSpawn(32, 1, 96 * 1024 + 1, 0, T.NOP) == E
     assert p.taskSpawn(128, 1, 0, 0, 99) == E
     assert p.taskSpawn(128, 1, 0, 0, T.NOP, b"\0" * 41) == E
-    assert p.taskSpawn(992, 1, 96 * 1024, 1, T.NOP) >= 0   # a whole MTB
-    assert p.taskSpawn(32, 31, 0, 1, T.NOP) >= 0
+    assert p.taskSpawn(1024, 1, 96 * 1024, 1, T.NOP) >= 0  # a whole MTB: all 32 warps (self-scheduling)
+    assert p.taskSpawn(128, 8, 0, 1, T.NOP) >= 0
+    assert p.taskSpawn(32, 32, 0, 1, T.NOP) >= 0
     assert p.shutdown() == 0
 
 

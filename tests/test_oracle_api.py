@@ -74,7 +74,7 @@ def tasks(*rows):
     return np.array(list(rows), O.TASK_DTYPE)
 
 
-def check(events, ts, n_mtb=2, exec_warps=31, gran=192, bars=15):
+def check(events, ts, n_mtb=2, exec_warps=31, gran=192, bars=15):   # workers = warps 0..30
     return O.ledger_check(np.array(events, O.LEDGER_DTYPE), n_mtb, exec_warps, gran, bars, ts)
 
 
@@ -95,7 +95,7 @@ def test_ledger_accepts_valid_trace(orc):
     ([ev(0, 0, 1, 1, 0, 0b10, 0, 4), ev(1, 0, 1, 2, 0, 0b100, 3, 2)], "granule 3 double"),
     ([ev(0, 0, 1, 1, 0, 0b10, 0, 0, 3), ev(1, 0, 1, 2, 0, 0b100, 0, 0, 3)], "barrier id 3"),
     ([ev(0, 0, 1, 1, 0, 0b10, 190, 4)], "exceed arena"),
-    ([ev(0, 0, 1, 1, 0, 1 << 0)], "bad warp mask"),
+    ([ev(0, 0, 1, 1, 0, 1 << 31)], "bad warp mask"),   # warp 31 > exec_warps - 1 = 30
     ([ev(0, 0, 1, 1, 0, 0b10), ev(1, 0, 2, 1, 0, 0b110)], "not live"),
     ([ev(0, 0, 1, 1, 0, 0b10, 0, 2), ev(1, 0, 2, 1, 0, 0b10), ev(2, 0, 3, 1, 0, 0, 0, 1)], "differ"),
     ([ev(0, 0, 1, 1, 0, 0b10)], "never freed"),
