@@ -151,6 +151,18 @@ int64_t pagoda_run_timed(pagoda_ctx* ctx, int n, const int32_t* shapes, const vo
 int pagoda_latency_loop(pagoda_ctx* ctx, int n, int threads, int n_threadblocks, int shmem_bytes,
                         int sync_flag, int func_id, const void* args, size_t args_bytes, int64_t* lat_ns);
 
+/* Runtime counters accumulated on the device since the context was created
+ * (read while stopped or running; ns are %globaltimer nanoseconds). */
+enum {
+    PAGODA_CTR_INGEST_BATCHES = 0, PAGODA_CTR_INGEST_ENTRIES, PAGODA_CTR_INGEST_NS_DOORBELL,
+    PAGODA_CTR_INGEST_NS_COPY, PAGODA_CTR_INGEST_NS_PUBLISH, PAGODA_CTR_INGEST_RING_FULL,
+    PAGODA_CTR_SCHED_ROUNDS, PAGODA_CTR_SCHED_PROGRESS, PAGODA_CTR_TICKETS, PAGODA_CTR_CLAIM_EMPTY,
+    PAGODA_CTR_LOAD_NOT_READY, PAGODA_CTR_PLACED, PAGODA_CTR_PLACE_NOFIT, PAGODA_CTR_HANDOFFS,
+    PAGODA_CTR_COUNT = 16
+};
+/* Copy min(n, PAGODA_CTR_COUNT) counters into out[]; returns the number copied or < 0. */
+int pagoda_read_counters(pagoda_ctx* ctx, uint64_t* out, int n);
+
 /* Runtime facts and counters. */
 typedef struct {
     int      device, sm_count, n_mtb, mtbs_per_sm, exec_warps, arena_bytes, regs_per_thread;

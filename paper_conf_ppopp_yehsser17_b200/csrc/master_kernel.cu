@@ -78,6 +78,10 @@ __device__ __forceinline__ void st_release_gpu(uint64_t* p, uint64_t v)
 {
     asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
+__device__ __forceinline__ void st_relaxed_gpu(uint64_t* p, uint64_t v)
+{
+    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
 __device__ __forceinline__ void st_relaxed_gpu32(uint32_t* p, uint32_t v)
 {
     asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
@@ -149,6 +153,13 @@ __device__ __forceinline__ uint32_t bm_range_bits(uint32_t off, uint32_t g, uint
     return (n == 32u ? 0xffffffffu : ((1u << n) - 1u)) << (lo - lane * 32u);
 }
 
+/* scheduler counters: holder-private shared-memory words, added to DevCtl.ctr at exit */
+enum { kScRounds = 0, kScProgress, kScTickets, kScClaimEmpty, kScLoadNotReady, kScPlaced, kScNoFit, kScHandoffs };
+__device__ __forceinline__ void sc_add(MtbShared& S, int i, uint32_t v)
+{
+    if ((threadIdx.x & 31u) == 0) S.sctr[i] += v;
+}
+
 /* ------------------------------------------------------------------ trace */
 __device__ __forceinline__ void trace_ev(const MkParams& p, int mtb, uint32_t& seq, uint8_t kind, uint64_t task_id,
                                          uint16_t tb, uint32_t mask, uint16_t goff, uint16_t glen, uint8_t bar)
@@ -216,85 +227,156 @@ __device__ __forceinline__ void run_task(MtbShared& S, char* smem_base, const Mk
  * into the device ring, a bounded MPMC queue with one sequence word per cell:
  * the producer may fill the cell of position t once seq == t (its previous
  * occupant was consumed), then releases seq = t + 1. */
-/* kIngestBatch, kIngestStageBytes: mk_layout.cuh */
+/* stage sizes: ingest_stage_entries() in mk_layout.cuh */
 
-__device__ void ingest(const MkParams& p, char* stage_buf)
+__device__ __forceinline__ void tma_load_1d(void* smem_dst, const void* gsrc, uint32_t bytes, uint64_t* bar)
+{
+    asm volatile("cp.async.bulk.shared::cta.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                     smem_u32(smem_dst)),
+                 "l"(gsrc), "r"(bytes), "r"(smem_u32(bar))
+                 : "memory");
+}
+__device__ __forceinline__ void tma_store_1d(void* gdst, const void* smem_src, uint32_t bytes)
+{
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(gdst), "r"(smem_u32(smem_src)),
+                 "r"(bytes)
+                 : "memory");
+}
+
+/* The ingest warp, a two-stage TMA pipeline: while stage s's batch (up to 256
+ * entries = 16 KiB) is pulled from the pinned host ring by one bulk copy over
+ * PCIe, the other stage's batch is bulk-stored into the device ring and its
+ * cells are published.  A batch may wrap the ring end: then it is two copies. */
+__device__ __forceinline__ void fence_acq_rel_gpu()
+{
+    asm volatile("fence.acq_rel.gpu;" ::: "memory");
+}
+
+__device__ void ingest(const MkParams& p, char* stage_buf, uint64_t* bars)
 {
     const uint32_t lane = threadIdx.x & 31u;
-    uint64_t copied = *(volatile uint64_t*)&p.dctl->tail;   /* resumes after a stop/start */
-    uint32_t last_err = 0;
+    const uint32_t kIngestStageEntries = p.ingest_stage_entries;
+    const uint64_t R = (uint64_t)p.ring_mask + 1;
+    uint64_t copied = *(volatile uint64_t*)&p.dctl->tail;   /* published into the device ring (resumes) */
+    uint64_t fetched = copied;                               /* loaded (or loading) into a stage */
+    uint64_t pub = copied;                                   /* last doorbell value seen */
+    uint64_t st_start[2] = {0, 0};
+    uint32_t st_n[2] = {0, 0};
+    uint32_t phase = 0;      /* bit s = parity of stage s's mbarrier */
+    uint32_t os = 0, ns = 0, inflight = 0, term = 0, last_err = 0;
     int idle = 0;
+    unsigned long long c_batches = 0, c_entries = 0, c_ns_db = 0, c_ns_copy = 0, c_ns_pub = 0, c_full = 0;
     for (;;) {
-        uint64_t pub = 0;
-        uint32_t term = 0, err = 0;
-        if (lane == 0) {
-            pub = ld_acquire_sys(&p.hctl->published);
-            term = ld_relaxed_sys32(&p.hctl->terminate);
-            err = *(volatile uint32_t*)&p.dctl->error;
-            if (err != last_err) st_relaxed_sys32(&p.hctl->error, err);
+        /* ---- doorbell: only when everything seen so far is fetched */
+        if (fetched >= pub) {
+            const uint64_t t0 = globaltimer_ns();
+            uint32_t err = 0;
+            if (lane == 0) {
+                pub = ld_acquire_sys(&p.hctl->published);
+                term = ld_relaxed_sys32(&p.hctl->terminate);
+                err = *(volatile uint32_t*)&p.dctl->error;
+                if (err != last_err) st_relaxed_sys32(&p.hctl->error, err);
+            }
+            pub = __shfl_sync(0xffffffffu, pub, 0);
+            term = __shfl_sync(0xffffffffu, term, 0);
+            last_err = __shfl_sync(0xffffffffu, err, 0);
+            c_ns_db += globaltimer_ns() - t0;
+            if (term == kStopAbort) {   /* host watchdog: abandon the queue, let idle MTBs exit */
+                if (lane == 0) st_release_gpu32(&p.dctl->stop, kStopAbort);
+                break;
+            }
         }
-        pub = __shfl_sync(0xffffffffu, pub, 0);
-        term = __shfl_sync(0xffffffffu, term, 0);
-        last_err = __shfl_sync(0xffffffffu, err, 0);
-        if (term == kStopAbort) {   /* host watchdog: abandon the queue, let idle MTBs exit */
-            if (lane == 0) st_release_gpu32(&p.dctl->stop, kStopAbort);
-            return;
+        /* ---- fill free stages (the doorbell acquire orders these async-proxy reads) */
+        while (inflight < 2 && fetched < pub) {
+            const uint32_t n = (uint32_t)min(pub - fetched, (uint64_t)kIngestStageEntries);
+            if (lane == 0) {
+                asm volatile("fence.proxy.async.global;" ::: "memory");
+                char* dst = stage_buf + ns * (kIngestStageEntries * 64u);
+                const uint32_t e0 = (uint32_t)(fetched & p.ring_mask);
+                const uint32_t n1 = min(n, (uint32_t)(R - e0));
+                asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(&bars[ns])),
+                             "r"(n * 64u)
+                             : "memory");
+                tma_load_1d(dst, p.hring + e0, n1 * 64u, &bars[ns]);
+                if (n1 < n) tma_load_1d(dst + n1 * 64u, p.hring, (n - n1) * 64u, &bars[ns]);
+            }
+            st_start[ns] = fetched;
+            st_n[ns] = n;
+            fetched += n;
+            ns ^= 1u;
+            inflight++;
+            idle = 0;
         }
-        if (pub > copied) {
-            uint32_t n = (uint32_t)min(pub - copied, (uint64_t)kIngestBatch);
-            /* free cells: the longest prefix whose previous occupant was consumed.  All the
-             * sequence loads are issued before any is used (one L2 round trip), then one
-             * fence gives them acquire semantics. */
-            constexpr int kSeqPerLane = kIngestBatch / 32;
-            uint32_t sv[kSeqPerLane];
+        if (inflight) {
+            /* ---- complete the oldest stage */
+            const uint64_t t1 = globaltimer_ns();
+            mbar_wait(&bars[os], (phase >> os) & 1u);
+            phase ^= 1u << os;
+            const uint64_t s = st_start[os];
+            const uint32_t n = st_n[os];
+            const uint64_t t2 = globaltimer_ns();
+            c_ns_copy += t2 - t1;
+            /* the device cells must be free: seq == position (their previous occupants loaded) */
+            for (uint32_t base = 0; base < n;) {   /* 256 cells per round trip (8 loads per lane) */
+                uint32_t sv[8];
 #pragma unroll
-            for (int i = 0; i < kSeqPerLane; i++) {
-                const uint64_t t = copied + (uint64_t)i * 32u + lane;
-                sv[i] = (uint32_t)i * 32u + lane < n ? ld_relaxed_gpu32(&p.dseq[t & p.ring_mask]) : (uint32_t)t;
-            }
-            uint32_t ready = n;
+                for (int i = 0; i < 8; i++) {
+                    const uint32_t k = base + (uint32_t)i * 32u + lane;
+                    sv[i] = k < n ? ld_relaxed_gpu32(&p.dseq[(s + k) & p.ring_mask]) : (uint32_t)(s + k);
+                }
+                uint32_t bad = 0;
 #pragma unroll
-            for (int i = 0; i < kSeqPerLane; i++) {
-                const uint32_t bad = __ballot_sync(0xffffffffu, sv[i] != (uint32_t)(copied + (uint64_t)i * 32u + lane));
-                if (bad && ready == n) ready = min(n, (uint32_t)i * 32u + (uint32_t)__ffs(bad) - 1u);
+                for (int i = 0; i < 8; i++)
+                    bad |= __ballot_sync(0xffffffffu, sv[i] != (uint32_t)(s + base + (uint32_t)i * 32u + lane));
+                if (bad) {   /* device ring full: wait for the schedulers */
+                    c_full++;
+                    __nanosleep(128);
+                    continue;
+                }
+                base += 256u;
             }
-            __threadfence();
-            n = ready;
-            if (n == 0) {              /* device ring full: wait for the schedulers */
-                __nanosleep(128);
-                continue;
+            fence_acq_rel_gpu();   /* acquire: the cells' previous readers are done with them */
+            if (lane == 0) {
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                const char* src = stage_buf + os * (kIngestStageEntries * 64u);
+                const uint32_t e0 = (uint32_t)(s & p.ring_mask);
+                const uint32_t n1 = min(n, (uint32_t)(R - e0));
+                tma_store_1d(p.dring + e0, src, n1 * 64u);
+                if (n1 < n) tma_store_1d(p.dring, src + n1 * 64u, (n - n1) * 64u);
+                asm volatile("cp.async.bulk.commit_group;\n\tcp.async.bulk.wait_group 0;" ::: "memory");
+                asm volatile("fence.proxy.async.global;" ::: "memory");
             }
-            const uint32_t chunks = n * 4u;
-            for (uint32_t c = lane; c < chunks; c += 32u) {
-                const uint64_t e = (copied + (c >> 2)) & p.ring_mask;
-                cp_async16(stage_buf + c * 16u, reinterpret_cast<const int4*>(p.hring + e) + (c & 3u));
-            }
-            cp_async_wait_all();
             __syncwarp();
-            for (uint32_t c = lane; c < chunks; c += 32u) {
-                const uint64_t e = (copied + (c >> 2)) & p.ring_mask;
-                const int4 v = *reinterpret_cast<const int4*>(stage_buf + c * 16u);
-                __stcg(reinterpret_cast<int4*>(p.dring + e) + (c & 3u), v);
-            }
-            __syncwarp();      /* every lane's entry stores precede ... */
-            __threadfence();   /* ... one warp-wide fence, so each lane's relaxed seq store releases them */
+            fence_acq_rel_gpu();   /* the entry writes precede every lane's relaxed cell release */
             for (uint32_t i = lane; i < n; i += 32u) {
-                const uint64_t t = copied + i;
+                const uint64_t t = s + i;
                 st_relaxed_gpu32(&p.dseq[t & p.ring_mask], (uint32_t)(t + 1));
             }
             __syncwarp();
-            copied += n;
+            copied = s + n;
             if (lane == 0) {
-                st_release_gpu(&p.dctl->tail, copied);     /* hint for schedulers: work exists */
+                st_relaxed_gpu(&p.dctl->tail, copied);     /* hint for schedulers: work exists */
                 st_relaxed_sys(&p.hctl->consumed, copied); /* host may now reuse those ring slots */
             }
-            idle = 0;
+            c_ns_pub += globaltimer_ns() - t2;
+            c_batches++;
+            c_entries += n;
+            inflight--;
+            os ^= 1u;
         } else if (term) {
             if (lane == 0) st_release_gpu32(&p.dctl->stop, 1u);
-            return;
+            break;
         } else if (++idle > 64) {
             __nanosleep(256);
         }
+    }
+    if (lane == 0) {
+        atomicAdd(&p.dctl->ctr[PAGODA_CTR_INGEST_BATCHES], c_batches);
+        atomicAdd(&p.dctl->ctr[PAGODA_CTR_INGEST_ENTRIES], c_entries);
+        atomicAdd(&p.dctl->ctr[PAGODA_CTR_INGEST_NS_DOORBELL], c_ns_db);
+        atomicAdd(&p.dctl->ctr[PAGODA_CTR_INGEST_NS_COPY], c_ns_copy);
+        atomicAdd(&p.dctl->ctr[PAGODA_CTR_INGEST_NS_PUBLISH], c_ns_pub);
+        atomicAdd(&p.dctl->ctr[PAGODA_CTR_INGEST_RING_FULL], c_full);
     }
 }
 
@@ -312,6 +394,7 @@ struct Sched {
     uint32_t ph, pl, pt; /* FIFO: [ph,pl) loaded task slots, [pl,pt) tickets not yet loaded */
     uint32_t est_w;      /* warps of the last loaded task (0 = none yet) */
     uint32_t seq;        /* ledger clock */
+    uint32_t holder_bit; /* the warp holding the scheduler token (this warp) */
 };
 
 __device__ __forceinline__ uint32_t nth_set_bit(uint32_t mask, uint32_t n)
@@ -343,9 +426,11 @@ __device__ bool sched_place(MtbShared& S, Sched& st, const MkParams& p, int mtb,
     for (uint32_t j = 0; j < ntb; j++) {
         const uint32_t tbs = __ffs(st.free_tbs) - 1;
         st.free_tbs &= ~(1u << tbs);
-        uint32_t m = 0, fw = st.free_w;
+        /* lowest free warps, the token holder last: it keeps scheduling unless it is needed */
+        uint32_t m = 0, fw = st.free_w & ~st.holder_bit;
         for (uint32_t i = 0; i < wtb; i++) {
-            m |= fw & (0u - fw);   /* lowest free warp */
+            if (!fw) fw = st.free_w & st.holder_bit;
+            m |= fw & (0u - fw);
             fw &= fw - 1u;
         }
         st.free_w &= ~m;
@@ -413,7 +498,10 @@ __device__ int sched_claim(MtbShared& S, Sched& st, const MkParams& p)
     }
     head = __shfl_sync(0xffffffffu, head, 0);
     tail = __shfl_sync(0xffffffffu, tail, 0);
-    if (head >= tail) return 0;
+    if (head >= tail) {
+        sc_add(S, kScClaimEmpty, 1);
+        return 0;
+    }
     /* a backlog smaller than what every MTB could take is handed out one ticket at a time,
      * so consecutive (often similar-cost) tasks spread over MTBs instead of piling up */
     const uint64_t backlog = tail - head;
@@ -423,6 +511,7 @@ __device__ int sched_claim(MtbShared& S, Sched& st, const MkParams& p)
     if (lane == 0) t0 = atomicAdd(reinterpret_cast<unsigned long long*>(&p.dctl->head), (unsigned long long)k);
     t0 = __shfl_sync(0xffffffffu, t0, 0);
     if (lane < k) S.pend_ticket[(st.pt + lane) & 31u] = t0 + lane;
+    sc_add(S, kScTickets, k);
     st.pt += k;
     __syncwarp();
     return (int)k;
@@ -443,7 +532,10 @@ __device__ int sched_load(MtbShared& S, Sched& st, const MkParams& p)
     }
     const uint32_t nr = __ballot_sync(0xffffffffu, !ready);
     const uint32_t r = nr ? (uint32_t)__ffs(nr) - 1u : 32u;   /* leading published tickets */
-    if (r == 0) return 0;
+    if (r == 0) {
+        sc_add(S, kScLoadNotReady, 1);
+        return 0;
+    }
     for (uint32_t c = lane; c < r * 4u; c += 32u) {
         const uint32_t i = c >> 2;
         const uint64_t ti = S.pend_ticket[(st.pl + i) & 31u];
@@ -508,6 +600,7 @@ __device__ __forceinline__ void sst_load(MtbShared& S, Sched& st, uint32_t exec_
     st.est_w = S.sst_est_w;
     st.seq = S.sst_seq;
     st.exec_mask = exec_mask;
+    st.holder_bit = 1u << (threadIdx.x >> 5);
 }
 
 __device__ __forceinline__ bool token_try(MtbShared& S)
@@ -574,7 +667,11 @@ __device__ bool sched_round(MtbShared& S, Sched& st, const MkParams& p, int mtb,
     bool progress = sched_fold(S, st, p, mtb);
     if (st.pl != st.pt && sched_load(S, st, p) > 0) progress = true;
     while (st.ph != st.pl) {
-        if (!sched_place(S, st, p, mtb, S.pend[st.ph & 31u])) break;
+        if (!sched_place(S, st, p, mtb, S.pend[st.ph & 31u])) {
+            sc_add(S, kScNoFit, 1);
+            break;
+        }
+        sc_add(S, kScPlaced, 1);
         st.ph++;
         progress = true;
     }
@@ -583,6 +680,8 @@ __device__ bool sched_round(MtbShared& S, Sched& st, const MkParams& p, int mtb,
      * can never fit */
     if ((mtb != 0 || p.n_mtb == 1) && sched_claim(S, st, p) > 0) progress = true;
     exit = false;
+    sc_add(S, kScRounds, 1);
+    if (progress) sc_add(S, kScProgress, 1);
     if (!progress && st.free_w == st.exec_mask && st.ph == st.pl) {
         uint32_t stop = 0;
         if (lane == 0) stop = ld_acquire_gpu32(&p.dctl->stop);
@@ -611,6 +710,7 @@ __device__ void sched_handoff(MtbShared& S, Sched& st, const MkParams& p, int mt
         if (st.free_w) {
             const uint32_t h = __ffs(st.free_w) - 1;
             sst_save(S, st);
+            sc_add(S, kScHandoffs, 1);
             if (lane == h) {
                 S.wt[h].task = SLOT_SCHED;
                 mbar_arrive(&S.exec_bar[h]);   /* release: the saved state is visible to h */
@@ -645,7 +745,11 @@ __device__ void worker(MtbShared& S, char* smem_base, const MkParams& p, int mtb
                     S.wt[lane].task = SLOT_TERMINATE;
                     mbar_arrive(&S.exec_bar[lane]);
                 }
-                if (lane == 0) atomicAdd(&p.dctl->exited, 1u);
+                if (lane == 0) {
+                    atomicAdd(&p.dctl->exited, 1u);
+                    for (int i = 0; i < 8; i++)
+                        atomicAdd(&p.dctl->ctr[PAGODA_CTR_SCHED_ROUNDS + i], (unsigned long long)S.sctr[i]);
+                }
                 return;
             }
             if ((st.free_w >> w) & 1u) {   /* still free: keep scheduling */
@@ -691,7 +795,7 @@ __global__ void __launch_bounds__(1024, kMinBlocks) master_kernel(MkParams p)
     int arena_granules = p.arena_granules;
     char* ingest_stage = nullptr;
     if (mtb == 0) {   /* MTB 0 lends the top of its arena to the ingest warp */
-        arena_granules -= (int)(kIngestStageBytes / PAGODA_GRANULE);
+        arena_granules -= (int)(2u * p.ingest_stage_entries * 64u / PAGODA_GRANULE);
         ingest_stage = smem_base + p.arena_offset + (size_t)arena_granules * PAGODA_GRANULE;
     }
     uint32_t resident = 0;   /* shared-window address of the resident tables */
@@ -718,6 +822,7 @@ __global__ void __launch_bounds__(1024, kMinBlocks) master_kernel(MkParams p)
     if (warp == 0) {
         mbar_init(&S.exec_bar[lane], 1);
         mbar_init(&S.stage_bar[lane], 1);
+        if (lane < 2) mbar_init(&S.ingest_bar[lane], 1);
         /* initial scheduler state, owned by the first worker (it starts with the token) */
         S.sst_fg[lane] = bm_range_bits(0, (uint32_t)arena_granules, lane);
         if (lane == 0) {
@@ -730,11 +835,12 @@ __global__ void __launch_bounds__(1024, kMinBlocks) master_kernel(MkParams p)
             S.sst_est_w = 0;
             S.sst_seq = 0;
             S.token = 1;
+            for (int i = 0; i < 8; i++) S.sctr[i] = 0;
             asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         }
     }
     __syncthreads();
-    if (mtb == 0 && warp == kIngestWarp) ingest(p, ingest_stage);
+    if (mtb == 0 && warp == kIngestWarp) ingest(p, ingest_stage, S.ingest_bar);
     else if ((exec_mask >> warp) & 1u) worker(S, smem_base, p, mtb, warp, resident, exec_mask, warp == first);
 }
 

@@ -40,6 +40,9 @@ struct HostCtl {
     alignas(64) volatile uint64_t pad[8];
 };
 
+/* runtime counters, summed over the session (index = PAGODA_CTR_* in pagoda.h) */
+constexpr int kNumCounters = 16;
+
 /* device memory, L2-resident: the device ring's counters */
 struct DevCtl {
     alignas(128) uint64_t tail;    /* entries published into the device ring (ingest warp; a hint) */
@@ -47,6 +50,7 @@ struct DevCtl {
     alignas(128) uint32_t stop;    /* set by ingest after terminate: schedulers drain and exit */
     alignas(128) uint32_t error;   /* device error word (executors atomicOr) */
     alignas(128) uint32_t exited;  /* MTBs that exited */
+    alignas(128) unsigned long long ctr[kNumCounters];   /* runtime counters (pagoda_read_counters) */
 };
 
 struct LedgerEvent {   /* 32 B; identical field order to the oracle's checker input */
@@ -87,6 +91,7 @@ struct MkParams {
     int      exec_warps;      /* executor warps per MTB (warps 1..exec_warps) */
     int      arena_granules;
     uint32_t arena_offset;    /* byte offset of the task arena in dynamic shared memory */
+    uint32_t ingest_stage_entries;   /* entries per ingest stage (2 stages, multiple of 32) */
     const uint32_t* resident_tdes_src;   /* 2 KiB SP table in device memory, replicated per lane
                                             at kResidentOffset when non-null */
     int      n_mtb;
@@ -98,8 +103,15 @@ struct MkParams {
 };
 
 constexpr int kIngestWarp = 31;          /* warp 31 of MTB 0 feeds the device ring */
-constexpr int kIngestBatch = 512;        /* entries per ingest round */
-constexpr uint32_t kIngestStageBytes = kIngestBatch * 64;   /* its staging, lent by MTB 0 from the top of its arena */
+/* ingest staging: 2 stages of MkParams::ingest_stage_entries entries (64 B each), lent by MTB 0
+ * from the top of its arena; the host sizes them (ingest_stage_entries()) */
+constexpr uint32_t kIngestMaxStageEntries = 1024;
+__host__ __device__ inline uint32_t ingest_stage_entries(uint32_t arena_bytes, int n_mtb)
+{
+    if (n_mtb == 1) return 128;   /* MTB 0 also runs tasks: keep most of its arena */
+    uint32_t e = arena_bytes / (2u * 64u) / 32u * 32u;
+    return e > kIngestMaxStageEntries ? kIngestMaxStageEntries : e;
+}
 constexpr uint32_t kStopAbort = 2;       /* HostCtl.terminate / DevCtl.stop value: abandon work and exit */
 constexpr int kMaxGranules = 1024;       /* lane-distributed bitmap: 32 lanes x 32 bits */
 
@@ -128,6 +140,8 @@ struct MtbShared {
     uint32_t  sst_free_w, sst_free_task, sst_free_tbs, sst_free_bar;
     uint32_t  sst_ph, sst_pl, sst_pt, sst_est_w, sst_seq;
     uint32_t  token;                 /* 1 while some warp holds the scheduler token */
+    uint32_t  sctr[8];               /* scheduler counters (holder-only), flushed at exit */
+    uint64_t  ingest_bar[2];         /* MTB 0: the ingest warp's two TMA stage mbarriers */
 };
 static_assert(offsetof(MtbShared, wt) == kWarpTableOffset, "WarpTable offset");
 static_assert(sizeof(MtbShared) <= kControlBytes && kControlBytes <= kResidentOffset, "control block fits");

@@ -40,7 +40,6 @@ cudaError_t launch_master(int mtbs_per_sm, int n_mtb, size_t smem_bytes, cudaStr
 }
 using namespace pagoda;
 
-static const uint32_t kIngestGranules = kIngestStageBytes / PAGODA_GRANULE;   /* MTB 0 lends them to the ingest warp */
 static const int kSpawnChunk = 64;   /* batched spawns publish the doorbell once per chunk */
 
 struct pagoda_ctx {
@@ -250,7 +249,7 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
         return -EINVAL;
     if (cfg.exec_warps < 1 || cfg.exec_warps > 32) return -EINVAL;
     if (cfg.arena_bytes % PAGODA_GRANULE || cfg.arena_bytes / PAGODA_GRANULE > (uint32_t)kMaxGranules ||
-        cfg.arena_bytes < kIngestGranules * PAGODA_GRANULE)
+        cfg.arena_bytes < 2u * 128u * 64u + 8u * PAGODA_GRANULE)   /* ingest staging + room for tasks */
         return -EINVAL;
     int ndev = 0;
     if (cudaGetDeviceCount(&ndev) != cudaSuccess || cfg.device < 0 || cfg.device >= ndev) {
@@ -280,7 +279,7 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
     const uint32_t arena_g = cfg.arena_bytes / PAGODA_GRANULE;
     if (c->n_mtb == 1) {   /* MTB 0 alone: it also hosts the ingest warp and its staging */
         c->max_task_warps = cfg.exec_warps == 32 ? 31 : (int)cfg.exec_warps;
-        c->max_task_granules = arena_g - kIngestGranules;
+        c->max_task_granules = arena_g - 2u * ingest_stage_entries(cfg.arena_bytes, 1) * 64u / PAGODA_GRANULE;
     } else {
         c->max_task_warps = (int)cfg.exec_warps;
         c->max_task_granules = arena_g;
@@ -340,6 +339,7 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
         p.exec_warps = (int)cfg.exec_warps;
         p.arena_granules = (int)arena_g;
         p.arena_offset = arena_offset;
+        p.ingest_stage_entries = ingest_stage_entries(cfg.arena_bytes, c->n_mtb);
         if (cfg.flags & PAGODA_RESIDENT_TDES) {   /* the key-independent SP table, replicated by each MTB */
             std::vector<uint8_t> tab(PAGODA_TDES_TABLE_BYTES);
             const uint8_t zero_key[24] = {0};
@@ -702,6 +702,14 @@ int64_t pagoda_inflight_warps(pagoda_ctx* c)
     const int64_t spawned = c->warps_spawned.load(std::memory_order_acquire);
     const int64_t done = l ? c->warps_prefix[(l - 1) & (c->C - 1)] : 0;
     return spawned - done;
+}
+
+int pagoda_read_counters(pagoda_ctx* c, uint64_t* out, int n)
+{
+    if (!c || !out || n < 0) return -EINVAL;
+    const int k = std::min(n, kNumCounters);
+    if (cudaMemcpy(out, c->dctl->ctr, (size_t)k * 8, cudaMemcpyDeviceToHost) != cudaSuccess) return -EIO;
+    return k;
 }
 
 const char* pagoda_version(void) { return "pagoda-b200 0.1 (sm_100a)"; }

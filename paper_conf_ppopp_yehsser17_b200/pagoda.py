@@ -93,6 +93,7 @@ def lib() -> C.CDLL:
         L.pagoda_run_timed.argtypes = [P, I, P, P, SZ, SZ, P, P]
         L.pagoda_run_timed.restype = I64
         L.pagoda_latency_loop.argtypes = [P, I, I, I, I, I, I, P, SZ, P]
+        L.pagoda_read_counters.argtypes = [P, P, I]
         _lib = L
     return _lib
 
@@ -211,6 +212,15 @@ class Pagoda:
         i = pagoda_info()
         _check(lib().pagoda_get_info(self.h, C.byref(i)), "pagoda_get_info")
         return i
+
+    COUNTERS = ("ingest_batches", "ingest_entries", "ingest_ns_doorbell", "ingest_ns_copy", "ingest_ns_publish",
+                "ingest_ring_full", "sched_rounds", "sched_progress", "tickets", "claim_empty", "load_not_ready",
+                "placed", "place_nofit", "handoffs")
+
+    def counters(self) -> dict:
+        out = np.zeros(16, np.uint64)
+        _check(lib().pagoda_read_counters(self.h, _ptr(out), 16), "pagoda_read_counters")
+        return {k: int(out[i]) for i, k in enumerate(self.COUNTERS)}
 
     def inflight_warps(self) -> int:
         return lib().pagoda_inflight_warps(self.h)
