@@ -185,7 +185,7 @@ int pagoda_get_info(pagoda_ctx* ctx, pagoda_info* out);
 int64_t pagoda_trace_read(pagoda_ctx* ctx, int mtb, void* dst, size_t cap);
 
 /* Executor intervals (PAGODA_TRACE): per executor warp a list of
- * {u64 task_id; u32 tb; u16 mtb; u16 warp; u64 t_start_ns; u64 t_end_ns} (32 B).
+ * {u64 task_id; u16 tb; u16 smid; u16 mtb; u16 warp; u64 t_start_ns; u64 t_end_ns} (32 B).
  * Copies up to cap records of (mtb, warp) into dst; returns the count. */
 int64_t pagoda_trace_read_exec(pagoda_ctx* ctx, int mtb, int warp, void* dst, size_t cap);
 

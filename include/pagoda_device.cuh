@@ -89,7 +89,11 @@ struct TaskEnv {
     __device__ __forceinline__ int getBlockDim() const { return s.threads_tb; }
     __device__ __forceinline__ int getBlockWarps() const { return s.warps_tb; }
     __device__ __forceinline__ int getNumBlocks() const { return s.n_tb; }
-    __device__ __forceinline__ char* getSMPtr() const { return smem_base + s.smem_off; }
+    __device__ __forceinline__ char* getSMPtr() const
+    {   /* derived from the __shared__ symbol itself, so nvcc emits LDS/STS, not generic LD/ST */
+        extern __shared__ __align__(1024) unsigned char pagoda_mk_smem[];
+        return reinterpret_cast<char*>(pagoda_mk_smem) + s.smem_off;
+    }
     __device__ __forceinline__ uint32_t getSMBytes() const { return s.smem_bytes; }
     /* MTB-resident, lane-replicated 3DES SP tables (context flag PAGODA_RESIDENT_TDES) */
     __device__ __forceinline__ uint32_t getResidentTdes() const { return resident; }

@@ -115,20 +115,45 @@ template <class Env>
 __device__ void body_mb(const Env& e, const pagoda_mb_args& a)
 {
     const int T = total_threads(e);
+    const int maxit = a.maxit;
     for (int p = e.getTid(); p < 4096; p += T) {
         const int gx = 64 * a.tx + (p & 63), gy = 64 * a.ty + (p >> 6);
         const float cr = __fadd_rn(a.x0, __fmul_rn((float)gx, a.dx));
         const float ci = __fadd_rn(a.y0, __fmul_rn((float)gy, a.dx));
         float zr = 0.0f, zi = 0.0f;
         int n = 0;
-        while (n < a.maxit) {
-            const float zr2 = __fmul_rn(zr, zr);
-            const float zi2 = __fmul_rn(zi, zi);
-            if (__fadd_rn(zr2, zi2) > 4.0f) break;
-            const float t = __fadd_rn(zr, zr);
-            zi = __fadd_rn(__fmul_rn(t, zi), ci);
-            zr = __fadd_rn(__fsub_rn(zr2, zi2), cr);
-            n++;
+        /* Four iterations per branch: each step tests |z|^2 > 4 on its own z and
+         * updates z unconditionally; the count advances to the first escaping step
+         * (steps after it only touch values that are discarded).  A branch per
+         * iteration costs more than the iteration itself on the critical path. */
+        for (;;) {
+            if (n + 4 > maxit) {   /* remainder: one iteration at a time */
+                while (n < maxit) {
+                    const float zr2 = __fmul_rn(zr, zr);
+                    const float zi2 = __fmul_rn(zi, zi);
+                    if (__fadd_rn(zr2, zi2) > 4.0f) break;
+                    const float t = __fadd_rn(zr, zr);
+                    zi = __fadd_rn(__fmul_rn(t, zi), ci);
+                    zr = __fadd_rn(__fsub_rn(zr2, zi2), cr);
+                    n++;
+                }
+                break;
+            }
+            bool esc[4];
+#pragma unroll
+            for (int s = 0; s < 4; s++) {
+                const float zr2 = __fmul_rn(zr, zr);
+                const float zi2 = __fmul_rn(zi, zi);
+                esc[s] = __fadd_rn(zr2, zi2) > 4.0f;
+                const float t = __fadd_rn(zr, zr);
+                zi = __fadd_rn(__fmul_rn(t, zi), ci);
+                zr = __fadd_rn(__fsub_rn(zr2, zi2), cr);
+            }
+            if (esc[0] | esc[1] | esc[2] | esc[3]) {
+                n += esc[0] ? 0 : esc[1] ? 1 : esc[2] ? 2 : 3;
+                break;
+            }
+            n += 4;
         }
         a.out[p] = (uint16_t)n;
     }

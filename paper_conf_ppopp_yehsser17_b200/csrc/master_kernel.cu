@@ -193,13 +193,16 @@ __device__ __forceinline__ void run_task(MtbShared& S, char* smem_base, const Mk
     if (!run_body(t.func_id, env, t.args) && lane == 0) atomicOr(&p.dctl->error, PAGODA_DEVERR_BAD_FUNC);
     __syncwarp();
     if (lane == 0) {
-        /* this warp's global writes -> visible GPU-wide before anyone learns the warp is done */
-        __threadfence();
+        /* this warp's global writes -> visible GPU-wide before anyone learns the warp is done
+         * (release; the last warp's st.release.sys then publishes them system-wide) */
+        asm volatile("fence.acq_rel.gpu;" ::: "memory");
         if (p.trace_cap) {
             uint32_t* cnt = &p.exec_count[mtb * 32 + w];
             const uint32_t i = *cnt;
             if (i < p.trace_cap) {
-                ExecRecord r{s.task_id, s.tb, (uint16_t)mtb, (uint16_t)w, t0, globaltimer_ns()};
+                uint32_t smid;
+                asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+                ExecRecord r{s.task_id, s.tb, (uint16_t)smid, (uint16_t)mtb, (uint16_t)w, t0, globaltimer_ns()};
                 p.exec_trace[((size_t)mtb * 32 + w) * p.trace_cap + i] = r;
             }
             *cnt = i + 1;
@@ -477,7 +480,9 @@ __device__ bool sched_place(MtbShared& S, Sched& st, const MkParams& p, int mtb,
 }
 
 /* Take tickets: as many tasks as the free warps fit at the last task size
- * (one ticket when the size is unknown), never more than the ring holds. */
+ * (one ticket when the size is unknown), never more than the ring holds; one
+ * at a time while the backlog is smaller than what all MTBs could take, so
+ * consecutive (often similar-cost) tasks spread over MTBs. */
 __device__ int sched_claim(MtbShared& S, Sched& st, const MkParams& p)
 {
     const uint32_t lane = threadIdx.x & 31u;
@@ -502,8 +507,6 @@ __device__ int sched_claim(MtbShared& S, Sched& st, const MkParams& p)
         sc_add(S, kScClaimEmpty, 1);
         return 0;
     }
-    /* a backlog smaller than what every MTB could take is handed out one ticket at a time,
-     * so consecutive (often similar-cost) tasks spread over MTBs instead of piling up */
     const uint64_t backlog = tail - head;
     if (backlog < (uint64_t)p.n_mtb * 8u) want = 1;
     const uint32_t k = (uint32_t)min((uint64_t)want, backlog);

@@ -70,7 +70,8 @@ static_assert(sizeof(LedgerEvent) == 32, "LedgerEvent is 32 bytes");
 
 struct ExecRecord {    /* 32 B */
     uint64_t task_id;
-    uint32_t tb;
+    uint16_t tb;
+    uint16_t smid;     /* %smid: the SM the MTB runs on */
     uint16_t mtb;
     uint16_t warp;
     uint64_t t_start;

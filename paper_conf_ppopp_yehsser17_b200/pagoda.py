@@ -38,7 +38,7 @@ class pagoda_info(C.Structure):
 LEDGER_DTYPE = np.dtype([("seq", "<u4"), ("mtb", "<u2"), ("kind", "u1"), ("bar_id", "u1"),
                          ("task_id", "<u8"), ("warp_mask", "<u4"), ("tb", "<u2"), ("gran_off", "<u2"),
                          ("gran_len", "<u2"), ("pad", "<u2"), ("pad2", "<u4")])
-EXEC_DTYPE = np.dtype([("task_id", "<u8"), ("tb", "<u4"), ("mtb", "<u2"), ("warp", "<u2"),
+EXEC_DTYPE = np.dtype([("task_id", "<u8"), ("tb", "<u2"), ("smid", "<u2"), ("mtb", "<u2"), ("warp", "<u2"),
                        ("t_start", "<u8"), ("t_end", "<u8")])
 
 # names declared in include/pagoda.h (the ABI test checks the library exports them)
