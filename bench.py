@@ -312,7 +312,10 @@ def main():
     torch.cuda.synchronize()
     d.barrier()
     clk = clocks.stop()
-    total = d.max(sum(host_s))
+    # device time: each step is one MasterKernel session bracketed by CUDA events recorded on the
+    # context's stream (launch -> kernel exit; the host spawn runs inside it); max over ranks
+    total = d.max(sum(dev_ms) * 1e-3)
+    host_total = d.max(sum(host_s))
     all_tasks = d.sum(float(n * a.steps))
     value = all_tasks / total
     dev_avg_ms = statistics.mean(dev_ms)
@@ -373,7 +376,8 @@ def main():
                                                                   if k != "flags"} | {
                                                           "resident_tdes_tables": use_resident(a)},
                                                       "task_shmem_bytes": int(w.shapes[0][2])},
-            "gpu_launches": a.steps, "device_ms_per_step": dev_avg_ms, "clocks": clk}
+            "gpu_launches": a.steps, "host_ms_per_step": 1e3 * host_total / a.steps,
+            "host_tasks_per_s": all_tasks / host_total, "clocks": clk}
     if lat:
         line["p50_spawn_to_done_us"] = lat["loaded_us"]["p50"]
         line["latency"] = lat

@@ -49,8 +49,10 @@ enum : uint8_t { SLOT_TERMINATE = 0xFF, SLOT_SCHED = 0xFE /* take over the sched
  * follows the control block, or the resident tables when a context has them. */
 constexpr uint32_t kWarpTableOffset = 512;
 constexpr uint32_t kControlBytes = 5120;            /* arena offset without resident tables */
-constexpr uint32_t kResidentOffset = 8192;          /* 8 KiB aligned: lane bits OR into addresses */
+constexpr uint32_t kResidentOffset = 8192;          /* room reserved for the control block + resident tables */
 constexpr uint32_t kResidentTdesBytes = 8 * 64 * 32 * 4;   /* 3DES SP tables, one copy per lane */
+constexpr uint32_t kResidentTdesAddr = 8192;        /* shared-WINDOW address of the resident tables: a
+                                                       constant, so lookups carry it as an immediate */
 
 __device__ __forceinline__ uint32_t lane_id() { return threadIdx.x & 31u; }
 

@@ -163,7 +163,8 @@ __device__ void body_mb(const Env& e, const pagoda_mb_args& a)
  * TDEA EDE3, ECB (NIST [5]).  tables =
  * pagoda_tdes_tables(): SP[8][64] u32 (S-box j then P, for the 6-bit input of
  * box j), 48 round keys as a (kx, ky) u32 pair each (execution order
- * K1[0..15], K2[15..0], K3[0..15]), IP and FP byte tables [8][256] u64.
+ * K1[0..15], K2[15..0], K3[0..15]), IP and FP byte tables [8][256] u64
+ * (kept for the ABI; the body computes IP/FP with delta swaps, tdes_ip/tdes_fp).
  * Since FP then IP cancel between the three DES stages, a block is
  * IP, 48 rounds with a half-swap after every 16, FP.
  *
@@ -173,15 +174,36 @@ __device__ void body_mb(const Env& e, const pagoda_mb_args& a)
  * pack the key chunks the same way).  The 8 S-box outputs after P are disjoint,
  * so f = XOR of 8 table words.  Three table placements: MTB-resident with one
  * copy per lane (conflict-free), staged in the TB's shared memory, or global. */
-constexpr uint32_t kTdesStageBytes = 2048 + 384;
-constexpr uint32_t kTdesIpOff = 2432, kTdesFpOff = 2432 + 16384;
+constexpr uint32_t kTdesStageBytes = 2048 + 384;   /* SP boxes + round keys (the IP/FP byte tables that
+                                                       follow in the buffer are not used by the body) */
 
-__device__ __forceinline__ uint64_t tdes_perm(const uint64_t* tab, uint64_t x)
+/* IP and FP as five delta swaps each on the (L, R) = (high, low) words of the
+ * big-endian block: swap(a, b, n, m) exchanges the bits of b under mask m with
+ * the bits of a under m << n.  Register-only; a byte-table gather instead costs
+ * one L1 wavefront per distinct line touched by the warp (~10 per lookup).
+ * The sequence is the IP table's (FIPS 46-3) factorisation; tests/test_abi.py
+ * checks it against the product's IP/FP byte tables. */
+__device__ __forceinline__ void tdes_swap(uint32_t& a, uint32_t& b, int n, uint32_t m)
 {
-    uint64_t r = 0;
-#pragma unroll
-    for (int b = 0; b < 8; b++) r |= __ldg(&tab[b * 256 + (int)((x >> (56 - 8 * b)) & 0xFF)]);
-    return r;
+    const uint32_t t = ((a >> n) ^ b) & m;
+    b ^= t;
+    a ^= t << n;
+}
+__device__ __forceinline__ void tdes_ip(uint32_t& l, uint32_t& r)
+{
+    tdes_swap(l, r, 4, 0x0f0f0f0fu);
+    tdes_swap(l, r, 16, 0x0000ffffu);
+    tdes_swap(r, l, 2, 0x33333333u);
+    tdes_swap(r, l, 8, 0x00ff00ffu);
+    tdes_swap(l, r, 1, 0x55555555u);
+}
+__device__ __forceinline__ void tdes_fp(uint32_t& l, uint32_t& r)
+{
+    tdes_swap(l, r, 1, 0x55555555u);
+    tdes_swap(r, l, 8, 0x00ff00ffu);
+    tdes_swap(r, l, 2, 0x33333333u);
+    tdes_swap(l, r, 16, 0x0000ffffu);
+    tdes_swap(l, r, 4, 0x0f0f0f0fu);
 }
 
 template <int kOff>
@@ -194,21 +216,29 @@ __device__ __forceinline__ uint32_t lds_at(uint32_t addr)
 
 enum { kTdesResident = 0, kTdesShared = 1, kTdesGlobal = 2 };
 
-/* f(R) for table placement kMode.  resident: entry (j,v) at rl + 8192 j + 128 v
- * with rl = base | lane*4 (base 8 KiB aligned); shared: at sb + 256 j + 4 v
- * (sb 256-byte aligned); global: sp[64 j + v]. */
+/* f(R) for table placement kMode.
+ * resident: the MTB-resident table at window address kResidentTdesAddr holds
+ * SP[j][v] for lane l at word 4096 p + 64 v + 32 h + l, where byte p of x
+ * (h = 0) or of y (h = 1) is box j's input.  With x, y masked to 6-bit fields,
+ * one PRMT builds the offset: byte 1 = the field, byte 0 = lane*4 | 128 h
+ * (tb), bytes 2-3 = 0; the pair base is the load's immediate.
+ * shared: at sb + 256 j + 4 v (sb 256-byte aligned); global: sp[64 j + v]. */
 template <int kMode>
 __device__ __forceinline__ uint32_t tdes_f(uint32_t r, uint32_t kx, uint32_t ky, uint32_t tb, const uint32_t* sp)
 {
+    if (kMode == kTdesResident) {
+        const uint32_t x = (__funnelshift_l(r, r, 5) ^ kx) & 0x3F3F3F3Fu;
+        const uint32_t y = (__funnelshift_l(r, r, 1) ^ ky) & 0x3F3F3F3Fu;
+        const uint32_t t1 = tb | 128u;
+        constexpr uint32_t A = kResidentTdesAddr;
+        return lds_at<A + 0 * 16384>(__byte_perm(x, tb, 0x7604)) ^ lds_at<A + 1 * 16384>(__byte_perm(x, tb, 0x7614)) ^
+               lds_at<A + 2 * 16384>(__byte_perm(x, tb, 0x7624)) ^ lds_at<A + 3 * 16384>(__byte_perm(x, tb, 0x7634)) ^
+               lds_at<A + 0 * 16384>(__byte_perm(y, t1, 0x7604)) ^ lds_at<A + 1 * 16384>(__byte_perm(y, t1, 0x7614)) ^
+               lds_at<A + 2 * 16384>(__byte_perm(y, t1, 0x7624)) ^ lds_at<A + 3 * 16384>(__byte_perm(y, t1, 0x7634));
+    }
     const uint32_t x = __funnelshift_l(r, r, 5) ^ kx;
     const uint32_t y = __funnelshift_l(r, r, 1) ^ ky;
-    if (kMode == kTdesResident) {
-        const uint32_t m = 63u << 7;
-        return lds_at<0 * 8192>(tb | ((x << 7) & m)) ^ lds_at<6 * 8192>(tb | ((x >> 1) & m)) ^
-               lds_at<4 * 8192>(tb | ((x >> 9) & m)) ^ lds_at<2 * 8192>(tb | ((x >> 17) & m)) ^
-               lds_at<7 * 8192>(tb | ((y << 7) & m)) ^ lds_at<5 * 8192>(tb | ((y >> 1) & m)) ^
-               lds_at<3 * 8192>(tb | ((y >> 9) & m)) ^ lds_at<1 * 8192>(tb | ((y >> 17) & m));
-    } else if (kMode == kTdesShared) {
+    if (kMode == kTdesShared) {
         const uint32_t m = 63u << 2;
         return lds_at<0 * 256>(tb | ((x << 2) & m)) ^ lds_at<6 * 256>(tb | ((x >> 6) & m)) ^
                lds_at<4 * 256>(tb | ((x >> 14) & m)) ^ lds_at<2 * 256>(tb | ((x >> 22) & m)) ^
@@ -235,16 +265,13 @@ __device__ __forceinline__ uint2 tdes_key(uint32_t kb, const uint2* gk)
 template <int kMode, bool kKeysShared, class Env>
 __device__ __forceinline__ void tdes_blocks(const Env& e, const pagoda_tdes_args& a, uint32_t tb, uint32_t kb)
 {
-    const uint64_t* ipt = reinterpret_cast<const uint64_t*>(reinterpret_cast<const char*>(a.tables) + kTdesIpOff);
-    const uint64_t* fpt = reinterpret_cast<const uint64_t*>(reinterpret_cast<const char*>(a.tables) + kTdesFpOff);
     const uint2* gkeys = reinterpret_cast<const uint2*>(a.tables + 512);
     const int T = total_threads(e);
     for (uint32_t blk = (uint32_t)e.getTid(); blk < a.nblk; blk += (uint32_t)T) {
-        uint64_t x = a.in[blk];
-        /* bytes are the block in FIPS (big-endian) order */
-        x = ((uint64_t)__byte_perm((uint32_t)x, 0, 0x0123) << 32) | __byte_perm((uint32_t)(x >> 32), 0, 0x0123);
-        x = tdes_perm(ipt, x);
-        uint32_t l = (uint32_t)(x >> 32), r = (uint32_t)x;
+        const uint2 in = reinterpret_cast<const uint2*>(a.in)[blk];
+        /* bytes are the block in FIPS (big-endian) order: L = bytes 0..3, R = bytes 4..7 */
+        uint32_t l = __byte_perm(in.x, 0, 0x0123), r = __byte_perm(in.y, 0, 0x0123);
+        tdes_ip(l, r);
 #pragma unroll 1
         for (int st = 0; st < 3; st++) {
             const uint32_t kst = kb + st * 128;    /* 16 rounds x 8 bytes per stage */
@@ -265,9 +292,8 @@ __device__ __forceinline__ void tdes_blocks(const Env& e, const pagoda_tdes_args
             l = r;
             r = t;
         }
-        x = tdes_perm(fpt, ((uint64_t)l << 32) | r);
-        x = ((uint64_t)__byte_perm((uint32_t)x, 0, 0x0123) << 32) | __byte_perm((uint32_t)(x >> 32), 0, 0x0123);
-        a.out[blk] = x;
+        tdes_fp(l, r);
+        reinterpret_cast<uint2*>(a.out)[blk] = make_uint2(__byte_perm(l, 0, 0x0123), __byte_perm(r, 0, 0x0123));
     }
 }
 
@@ -283,8 +309,8 @@ __device__ void body_tdes(const Env& e, const pagoda_tdes_args& a)
         e.syncBlock();
         sb = smem_u32(s);
     }
-    if (res && sb) tdes_blocks<kTdesResident, true>(e, a, res | (lane_id() << 2), sb);
-    else if (res) tdes_blocks<kTdesResident, false>(e, a, res | (lane_id() << 2), 0);
+    if (res && sb) tdes_blocks<kTdesResident, true>(e, a, lane_id() << 2, sb);
+    else if (res) tdes_blocks<kTdesResident, false>(e, a, lane_id() << 2, 0);
     else if (sb) tdes_blocks<kTdesShared, true>(e, a, sb, sb + 2048);
     else tdes_blocks<kTdesGlobal, false>(e, a, 0, 0);
 }

@@ -804,18 +804,21 @@ __global__ void __launch_bounds__(1024, kMinBlocks) master_kernel(MkParams p)
     uint32_t resident = 0;   /* shared-window address of the resident tables */
     if (p.resident_tdes_src) {
         /* task-class resident tables (key-independent 3DES S-box/P tables), one copy per
-         * lane: word (j*64 + v)*32 + lane holds SP[j][v], so any 32 lookups are conflict-free.
-         * The region's WINDOW address must be 8 KiB aligned (lookups OR lane and index bits
-         * into it); the dynamic segment itself starts after the CTA's reserved shared memory. */
+         * lane, at the constant window address kResidentTdesAddr (bodies.cuh tdes_f):
+         * word 4096 p + 64 v + 32 h + lane holds SP[j][v] for box j = byte p of x (h = 0:
+         * boxes 0,6,4,2) or of y (h = 1: boxes 7,5,3,1), so any 32 lookups are conflict-free.
+         * The dynamic segment starts after the CTA's reserved shared memory (window 1 KiB). */
         const uint32_t base = smem_u32(smem_base);
-        resident = (base + kControlBytes + 8191u) & ~8191u;
-        if (resident - base + kResidentTdesBytes <= p.arena_offset) {
+        if (base + kControlBytes <= kResidentTdesAddr && kResidentTdesAddr - base + kResidentTdesBytes <= p.arena_offset) {
+            resident = kResidentTdesAddr;
             uint32_t* dst = reinterpret_cast<uint32_t*>(smem_base + (resident - base));
-            for (uint32_t i = threadIdx.x; i < kResidentTdesBytes / 4; i += blockDim.x)
-                dst[i] = __ldg(p.resident_tdes_src + (i >> 5));
-        } else {
-            resident = 0;   /* layout does not fit: bodies fall back to per-task tables */
-            if (threadIdx.x == 0) atomicOr(&p.dctl->error, PAGODA_DEVERR_LAYOUT);
+            for (uint32_t i = threadIdx.x; i < kResidentTdesBytes / 4; i += blockDim.x) {
+                const uint32_t pr = i >> 12, v = (i >> 6) & 63u, h = (i >> 5) & 1u;
+                const uint32_t j = h ? 7u - 2u * pr : (8u - 2u * pr) & 7u;
+                dst[i] = __ldg(p.resident_tdes_src + j * 64u + v);
+            }
+        } else if (threadIdx.x == 0) {
+            atomicOr(&p.dctl->error, PAGODA_DEVERR_LAYOUT);   /* bodies fall back to per-task tables */
         }
     }
     /* worker warps 0..exec_warps-1 (MTB 0: minus the ingest warp) */

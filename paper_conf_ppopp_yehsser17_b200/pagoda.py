@@ -14,7 +14,8 @@ import os
 import numpy as np
 
 PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(PKG, "libpagoda.so")
+# PAGODA_LIB selects another build of the same library (A/B experiments, scripts/build_variants.sh)
+LIB_PATH = os.environ.get("PAGODA_LIB") or os.path.join(PKG, "libpagoda.so")
 
 TRACE = 0x1
 NO_START = 0x2

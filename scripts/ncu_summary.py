@@ -1,0 +1,38 @@
+#!/usr/bin/env python
+"""Print the key counters of an ncu --set full report (pipe utilisation, L1
+wavefronts, DRAM bytes, issue, stalls) as `name value` lines."""
+import csv
+import subprocess
+import sys
+
+KEYS = ["gpu__time_duration.sum", "sm__cycles_elapsed.avg", "launch__registers_per_thread",
+        "dram__bytes_read.sum", "dram__bytes_write.sum", "sm__warps_active.avg.pct_of_peak_sustained_active",
+        "smsp__issue_active.avg.pct_of_peak_sustained_active", "sm__inst_executed.avg.per_cycle_active",
+        "smsp__inst_executed.sum", "sm__pipe_alu_cycles_active.avg.pct_of_peak_sustained_active",
+        "sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active",
+        "sm__inst_executed_pipe_lsu.avg.pct_of_peak_sustained_active",
+        "l1tex__data_pipe_lsu_wavefronts.avg.pct_of_peak_sustained_elapsed",
+        "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum.pct_of_peak_sustained_elapsed",
+        "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum", "l1tex__data_bank_conflicts_pipe_lsu_mem_shared_op_ld.sum",
+        "l1tex__lsu_writeback_active.avg.pct_of_peak_sustained_elapsed", "l1tex__throughput.avg.pct_of_peak_sustained_active",
+        "sm__throughput.avg.pct_of_peak_sustained_elapsed", "gpu__compute_memory_throughput.avg.pct_of_peak_sustained_elapsed"]
+
+
+def main(path):
+    out = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    rows = list(csv.reader(out.splitlines()))
+    h, u, v = rows[0], rows[1], rows[2]
+    col = {n: i for i, n in enumerate(h)}
+    for k in KEYS:
+        if k in col:
+            print(f"{k} {v[col[k]]} {u[col[k]]}")
+    stalls = [(float(v[i]), n) for n, i in col.items()
+              if n.startswith("smsp__average_warp_latency_issue_stalled") and n.endswith(".ratio") and v[i]]
+    stalls += [(float(v[i]), n) for n, i in col.items()
+               if n.startswith("smsp__average_warps_issue_stalled_") and n.endswith("_per_issue_active.ratio") and v[i]]
+    for val, n in sorted(stalls, reverse=True)[:8]:
+        print(f"{n} {val}")
+
+
+if __name__ == "__main__":
+    main(sys.argv[1])

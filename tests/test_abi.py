@@ -76,26 +76,64 @@ def test_args_layouts_fit_the_entry():
 
 
 # --------------------------------------------------------------- 3DES tables
+def _perm_bytes(t, x):
+    r = 0
+    for b in range(8):
+        r |= int(t[b, (x >> (56 - 8 * b)) & 0xFF])
+    return r
+
+
+def _swap(a, b, n, m):     # tdes_swap in csrc/bodies.cuh
+    t = ((a >> n) ^ b) & m
+    return a ^ ((t << n) & 0xFFFFFFFF), b ^ t
+
+
+def _ip_swaps(l, r):       # tdes_ip
+    l, r = _swap(l, r, 4, 0x0F0F0F0F)
+    l, r = _swap(l, r, 16, 0x0000FFFF)
+    r, l = _swap(r, l, 2, 0x33333333)
+    r, l = _swap(r, l, 8, 0x00FF00FF)
+    l, r = _swap(l, r, 1, 0x55555555)
+    return l, r
+
+
+def _fp_swaps(l, r):       # tdes_fp
+    l, r = _swap(l, r, 1, 0x55555555)
+    r, l = _swap(r, l, 8, 0x00FF00FF)
+    r, l = _swap(r, l, 2, 0x33333333)
+    l, r = _swap(l, r, 16, 0x0000FFFF)
+    l, r = _swap(l, r, 4, 0x0F0F0F0F)
+    return l, r
+
+
+def test_ip_fp_swap_networks_equal_the_product_tables(L):
+    """The body's register-only IP/FP equal the table-driven permutations
+    (FIPS 46-3 IP and IP^-1) the product also ships, and invert each other."""
+    tab = PG.tdes_tables(bytes(range(24)))
+    ipt = tab[2432:2432 + 16384].view(np.uint64).reshape(8, 256)
+    fpt = tab[2432 + 16384:].view(np.uint64).reshape(8, 256)
+    rng = np.random.default_rng(7)
+    blocks = [int(v) for v in rng.integers(0, 2 ** 63, 300, dtype=np.int64)] + [0, 2 ** 64 - 1, 1, 2 ** 63]
+    blocks += [1 << k for k in range(64)]
+    for x in blocks:
+        l, r = _ip_swaps(x >> 32, x & 0xFFFFFFFF)
+        assert (l << 32) | r == _perm_bytes(ipt, x)
+        l2, r2 = _fp_swaps(x >> 32, x & 0xFFFFFFFF)
+        assert (l2 << 32) | r2 == _perm_bytes(fpt, x)
+        assert _fp_swaps(l, r) == (x >> 32, x & 0xFFFFFFFF)
+
+
 def _des_with_product_tables(tab: np.ndarray, block: int) -> int:
     """Run the GPU body's round structure on the CPU with the product's tables
     (same index arithmetic as body_tdes in csrc/bodies.cuh)."""
     sp = tab[:2048].view(np.uint32).reshape(8, 64)
     keys = tab[2048:2432].view(np.uint32).reshape(48, 2)
-    ipt = tab[2432:2432 + 16384].view(np.uint64).reshape(8, 256)
-    fpt = tab[2432 + 16384:].view(np.uint64).reshape(8, 256)
-
-    def perm(t, x):
-        r = 0
-        for b in range(8):
-            r |= int(t[b, (x >> (56 - 8 * b)) & 0xFF])
-        return r
 
     def rotl(x, s):   # __funnelshift_l(x, x, s) takes s mod 32
         s %= 32
         return ((x << s) | (x >> (32 - s))) & 0xFFFFFFFF
 
-    x = perm(ipt, block)
-    l, r = x >> 32, x & 0xFFFFFFFF
+    l, r = _ip_swaps(block >> 32, block & 0xFFFFFFFF)
     for st in range(3):
         for rd in range(16):
             kx, ky = (int(v) for v in keys[st * 16 + rd])
@@ -106,7 +144,8 @@ def _des_with_product_tables(tab: np.ndarray, block: int) -> int:
                 f ^= int(sp[jx, (x >> 8 * b) & 63]) ^ int(sp[jy, (y >> 8 * b) & 63])
             l, r = r, l ^ f
         l, r = r, l
-    return perm(fpt, (l << 32) | r)
+    l, r = _fp_swaps(l, r)
+    return (l << 32) | r
 
 
 def test_tdes_tables_reproduce_known_answers(L):
