@@ -358,7 +358,7 @@ def main():
     cpu = None
     if not a.no_cpu and not a.quick and d.rank == 0 and d.world == 1:
         threads = os.cpu_count() or 1
-        ns = {"tdes": 4096, "mb": 1024, "mm": 65536, "mix": 4096, "nop": 4096}[a.workload]
+        ns = {"tdes": 16384, "mb": 1024, "mm": 65536, "mix": 4096, "nop": 16384}[a.workload]
         rate, dt, what = oracle_rate(a.workload if a.workload != "nop" else "tdes", ns, threads)
         cpu = {"value": rate, "unit": "tasks/s", "cores": threads, "kind": "oracle",
                "sample": f"{what}, {dt:.1f} s wall on {threads} threads"}
@@ -420,24 +420,55 @@ def roofline(workload, n, dev_ms, clk, peaks):
 
 def e2e_run(p, w, steps, torch):
     """Host-resident inputs (pinned) -> H2D -> spawn -> wait -> D2H, per step,
-    chunked so copies of chunk i+1 overlap the tasks of chunk i."""
-    if w.name == "tdes":
-        din, dout = w._keep[0], w._keep[1]
-        per_in = per_out = 4096
-        host_in = torch.from_numpy(w.host["packets"].reshape(-1).copy()).pin_memory()
-    elif w.name == "mm":
-        din = None
+    chunked so that the H2D copy of chunk i+1, the tasks of chunk i and the D2H
+    copy of chunk i-1 overlap (PCIe is full duplex).  A second host thread
+    drains: it waits for each chunk's last task (pagoda_waitBelow releases the
+    GIL) and queues that chunk's D2H copy."""
+    import queue
+    import threading
+    if w.name != "tdes":
         return None
-    else:
-        return None
+    din, dout = w._keep[0], w._keep[1]
+    per_in = per_out = 4096
+    host_in = torch.from_numpy(w.host["packets"].reshape(-1).copy()).pin_memory()
     host_out = torch.empty(w.n * per_out, dtype=torch.uint8).pin_memory()
     chunks = 16
     bounds = np.linspace(0, w.n, chunks + 1).astype(int)
     s_in, s_out = torch.cuda.Stream(), torch.cuda.Stream()
+    dev = torch.cuda.current_device()
+
+    tl = {"h2d": [], "spawned": [], "done": [], "d2h": []}   # last step's timeline (us from t0)
+
+    def drain(q, done, t0):
+        torch.cuda.set_device(dev)
+        evs = []
+        while True:
+            item = q.get()
+            if item is None:
+                break
+            c, end = item
+            assert p.waitBelow(end) == 0
+            tl["done"].append((time.perf_counter_ns() - t0) / 1e3)
+            lo, hi = bounds[c], bounds[c + 1]
+            with torch.cuda.stream(s_out):
+                host_out[lo * per_out:hi * per_out].copy_(dout[lo * per_out:hi * per_out], non_blocking=True)
+                e = torch.cuda.Event()
+                e.record(s_out)
+            evs.append(e)
+        for e in evs:
+            e.synchronize()
+            tl["d2h"].append((time.perf_counter_ns() - t0) / 1e3)
+        done.set()
+
     times = []
     assert p.start() == 0
     for it in range(steps + 1):
+        for v in tl.values():
+            v.clear()
+        q, done = queue.SimpleQueue(), threading.Event()
         t0 = time.perf_counter_ns()
+        th = threading.Thread(target=drain, args=(q, done, t0), daemon=True)
+        th.start()
         evs = []
         for c in range(chunks):            # every H2D copy queued at once on the copy stream
             lo, hi = bounds[c], bounds[c + 1]
@@ -446,25 +477,26 @@ def e2e_run(p, w, steps, torch):
                 e = torch.cuda.Event()
                 e.record(s_in)
             evs.append(e)
-        ends = []
         for c in range(chunks):            # a chunk's tasks are spawned as soon as its bytes landed
             lo, hi = bounds[c], bounds[c + 1]
             evs[c].synchronize()
+            tl["h2d"].append((time.perf_counter_ns() - t0) / 1e3)
             ids = p.spawn_shapes(w.shapes[lo:hi], w.args[lo:hi], ids=True)
-            ends.append(int(ids[-1]) + 1)
-        for c in range(chunks):            # D2H of chunk c once every task of it is done
-            lo, hi = bounds[c], bounds[c + 1]
-            assert p.waitBelow(ends[c]) == 0
-            with torch.cuda.stream(s_out):
-                host_out[lo * per_out:hi * per_out].copy_(dout[lo * per_out:hi * per_out], non_blocking=True)
-        s_out.synchronize()
+            tl["spawned"].append((time.perf_counter_ns() - t0) / 1e3)
+            q.put((c, int(ids[-1]) + 1))
+        q.put(None)
+        th.join()
+        assert done.is_set()
         if it > 0:
             times.append((time.perf_counter_ns() - t0) * 1e-9)
     assert p.stop() == 0
+    assert torch.equal(host_out, dout[: w.n * per_out].cpu()), "e2e: host copy differs from device output"
     tot = sum(times)
     return {"value": w.n * steps / tot, "unit": "tasks/s", "h2d_bytes_per_step": w.n * per_in,
             "d2h_bytes_per_step": w.n * per_out, "ms_per_step": 1e3 * tot / steps,
-            "how": "pinned host packets -> H2D (16 chunks, copy stream) -> taskSpawn per task -> waitBelow -> D2H per chunk"}
+            "how": "pinned host packets -> H2D (16 chunks, copy stream) -> taskSpawn per task; a drain thread "
+                   "waitBelow()s each chunk and queues its D2H on a second copy stream (both directions overlap)",
+            "timeline_us": {k: [round(x, 1) for x in v] for k, v in tl.items()}}
 
 
 if __name__ == "__main__":

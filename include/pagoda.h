@@ -158,6 +158,8 @@ enum {
     PAGODA_CTR_INGEST_NS_COPY, PAGODA_CTR_INGEST_NS_PUBLISH, PAGODA_CTR_INGEST_RING_FULL,
     PAGODA_CTR_SCHED_ROUNDS, PAGODA_CTR_SCHED_PROGRESS, PAGODA_CTR_TICKETS, PAGODA_CTR_CLAIM_EMPTY,
     PAGODA_CTR_LOAD_NOT_READY, PAGODA_CTR_PLACED, PAGODA_CTR_PLACE_NOFIT, PAGODA_CTR_HANDOFFS,
+    PAGODA_CTR_INGEST_NS_FENCE,   /* ns of the ingest publish phase spent in its fences */
+    PAGODA_CTR_INGEST_NS_STORE,   /* ns spent in the bulk store into the device ring */
     PAGODA_CTR_COUNT = 16
 };
 /* Copy min(n, PAGODA_CTR_COUNT) counters into out[]; returns the number copied or < 0. */

@@ -252,13 +252,17 @@ __device__ __forceinline__ uint32_t tdes_f(uint32_t r, uint32_t kx, uint32_t ky,
     }
 }
 
-/* round key i of the current stage: from the TB's shared memory (kKeysShared) or global */
+/* round keys i, i+1 of the current stage: from the TB's shared memory (kKeysShared) or global */
 template <bool kKeysShared, int kI>
-__device__ __forceinline__ uint2 tdes_key(uint32_t kb, const uint2* gk)
+__device__ __forceinline__ uint4 tdes_key2(uint32_t kb, const uint2* gk)
 {
-    uint2 k;
-    if (kKeysShared) asm("ld.shared.v2.u32 {%0, %1}, [%2+%3];" : "=r"(k.x), "=r"(k.y) : "r"(kb), "n"(kI * 8));
-    else k = __ldg(gk + kI);
+    uint4 k;
+    if (kKeysShared) {
+        asm("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4+%5];" : "=r"(k.x), "=r"(k.y), "=r"(k.z), "=r"(k.w) : "r"(kb), "n"(kI * 8));
+    } else {
+        const uint2 a = __ldg(gk + kI), b = __ldg(gk + kI + 1);
+        k = make_uint4(a.x, a.y, b.x, b.y);
+    }
     return k;
 }
 
@@ -276,18 +280,20 @@ __device__ __forceinline__ void tdes_blocks(const Env& e, const pagoda_tdes_args
         for (int st = 0; st < 3; st++) {
             const uint32_t kst = kb + st * 128;    /* 16 rounds x 8 bytes per stage */
             const uint2* gst = gkeys + st * 16;
-#define PAGODA_TDES_ROUND(I)                                                         \
+/* two rounds per key load: one 16-byte shared load (one wavefront) for keys I, I+1 */
+#define PAGODA_TDES_ROUND2(I)                                                        \
             {                                                                        \
-                const uint2 k = tdes_key<kKeysShared, I>(kst, gst);                  \
-                const uint32_t t = l ^ tdes_f<kMode>(r, k.x, k.y, tb, a.tables);     \
+                const uint4 k = tdes_key2<kKeysShared, I>(kst, gst);                 \
+                uint32_t t = l ^ tdes_f<kMode>(r, k.x, k.y, tb, a.tables);           \
+                l = r;                                                               \
+                r = t;                                                               \
+                t = l ^ tdes_f<kMode>(r, k.z, k.w, tb, a.tables);                    \
                 l = r;                                                               \
                 r = t;                                                               \
             }
-            PAGODA_TDES_ROUND(0) PAGODA_TDES_ROUND(1) PAGODA_TDES_ROUND(2) PAGODA_TDES_ROUND(3)
-            PAGODA_TDES_ROUND(4) PAGODA_TDES_ROUND(5) PAGODA_TDES_ROUND(6) PAGODA_TDES_ROUND(7)
-            PAGODA_TDES_ROUND(8) PAGODA_TDES_ROUND(9) PAGODA_TDES_ROUND(10) PAGODA_TDES_ROUND(11)
-            PAGODA_TDES_ROUND(12) PAGODA_TDES_ROUND(13) PAGODA_TDES_ROUND(14) PAGODA_TDES_ROUND(15)
-#undef PAGODA_TDES_ROUND
+            PAGODA_TDES_ROUND2(0) PAGODA_TDES_ROUND2(2) PAGODA_TDES_ROUND2(4) PAGODA_TDES_ROUND2(6)
+            PAGODA_TDES_ROUND2(8) PAGODA_TDES_ROUND2(10) PAGODA_TDES_ROUND2(12) PAGODA_TDES_ROUND2(14)
+#undef PAGODA_TDES_ROUND2
             const uint32_t t = l;   /* undo the last half-swap: stage output (R16, L16) */
             l = r;
             r = t;

@@ -44,6 +44,20 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity)
             : "memory");
     }
 }
+__device__ __forceinline__ void fence_acq_rel_gpu()
+{
+    asm volatile("fence.acq_rel.gpu;" ::: "memory");
+}
+__device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity, uint32_t hint_ns)
+{
+    uint32_t done;
+    asm volatile(
+        "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3; selp.u32 %0, 1, 0, p; }"
+        : "=r"(done)
+        : "r"(smem_u32(bar)), "r"(parity), "r"(hint_ns)
+        : "memory");
+    return done != 0;
+}
 __device__ __forceinline__ uint64_t ld_acquire_gpu(const uint64_t* p)
 {
     uint64_t v;
@@ -177,6 +191,116 @@ __device__ __forceinline__ void trace_ev(const MkParams& p, int mtb, uint32_t& s
     seq++;
 }
 
+/* ------------------------------------------------------------------ completion records
+ * A fence waits for every memory operation in flight on its SM, any warp's,
+ * including posted PCIe writes to pinned host memory, which crawl while copy
+ * engines keep the link busy (scripts/micro/membar_probe.cu; DESIGN.md
+ * "PCIe isolation").  So SMs that run tasks never touch host memory: the last
+ * warp of a task marks its slot in comp_pending; whichever warp holds the
+ * MTB's poster flag releases the tasks' writes with one GPU-scope fence and
+ * appends their ids to the device completion queue (one fetch-add per batch);
+ * MTB 0's forwarder moves them to the host's completion window.  With a single
+ * MTB there is no such split: the record goes to the host directly behind a
+ * system-scope fence.  The task slot is returned (mb_tasks) only after its id
+ * was read, so the id stays valid until then. */
+__device__ __noinline__ void post_completions(MtbShared& S, const MkParams& p)
+{
+    const uint32_t lane = threadIdx.x & 31u;
+    for (;;) {
+        uint32_t got = 0;
+        if (lane == 0) got = atomicExch(&S.poster, 1u) == 0u;
+        if (!__shfl_sync(0xffffffffu, got, 0)) return;   /* the holder will see our bit */
+        for (;;) {
+            uint32_t m = 0;
+            if (lane == 0) m = atomicExch(&S.comp_pending, 0u);
+            m = __shfl_sync(0xffffffffu, m, 0);
+            if (!m) break;
+            const bool mine = (m >> lane) & 1u;
+            const uint64_t id = mine ? S.tasks[lane].id : 0;
+            if (p.n_mtb == 1) {
+                asm volatile("fence.acq_rel.sys;" ::: "memory");
+                if (mine) st_relaxed_sys(reinterpret_cast<volatile uint64_t*>(&p.comp[id & p.comp_mask]), id);
+            } else {
+                fence_acq_rel_gpu();   /* release: the tasks' writes (fenced by each of their warps) */
+                unsigned long long base = 0;
+                if (lane == 0) base = atomicAdd(reinterpret_cast<unsigned long long*>(&p.dctl->dq_tail),
+                                                (unsigned long long)__popc(m));
+                base = __shfl_sync(0xffffffffu, base, 0);
+                if (mine) {
+                    const uint64_t slot = base + (uint64_t)__popc(m & ((1u << lane) - 1u));
+                    uint64_t* q = &p.dq[slot & p.dq_mask];
+                    while (*(volatile uint64_t*)q != 0) __nanosleep(64);   /* previous lap not forwarded yet */
+                    st_relaxed_gpu(q, id + 1);
+                }
+            }
+            __syncwarp();
+            if (lane == 0) {
+                __threadfence_block();
+                atomicOr(&S.mb_tasks, m);   /* the scheduler may now reuse those task slots */
+            }
+        }
+        uint32_t again = 0;
+        if (lane == 0) {
+            atomicExch(&S.poster, 0u);
+            __threadfence_block();   /* release the flag, then re-check: a bit set meanwhile by a */
+            again = *(volatile uint32_t*)&S.comp_pending != 0u;   /* warp that found the flag taken */
+        }
+        if (!__shfl_sync(0xffffffffu, again, 0)) return;
+    }
+}
+
+/* MTB 0's forwarder (n_mtb > 1): the completion queue in order -> the host's
+ * completion window.  Per sweep: find the run of filled records (up to 1024),
+ * one system-scope fence (cumulative: orders the task writes the posters
+ * released), then post the records and clear their queue slots.  Exits once
+ * every MTB exited and the queue is drained. */
+__device__ void comp_forwarder(MtbShared& S, const MkParams& p)
+{
+    const uint32_t lane = threadIdx.x & 31u;
+    uint64_t c = *(volatile uint64_t*)&p.dctl->dq_head;
+    uint32_t idle = 0;
+    for (;;) {
+        uint32_t n = 0;   /* the run of filled records at c, c+1, ... (8 loads per lane in flight) */
+        bool gap = false;
+        for (int trip = 0; trip < 4 && !gap; trip++) {
+            uint64_t v[8];
+#pragma unroll
+            for (int i = 0; i < 8; i++) v[i] = *(volatile uint64_t*)&p.dq[(c + n + (uint32_t)i * 32u + lane) & p.dq_mask];
+#pragma unroll
+            for (int i = 0; i < 8; i++) {
+                const uint32_t full = __ballot_sync(0xffffffffu, v[i] != 0);
+                if (!gap) {
+                    if (full == 0xffffffffu) n += 32u;
+                    else {
+                        n += (uint32_t)__ffs(~full) - 1u;
+                        gap = true;
+                    }
+                }
+            }
+        }
+        if (n == 0) {
+            uint32_t done = 0;
+            if (lane == 0) done = *(volatile uint32_t*)&p.dctl->exited >= (uint32_t)p.n_mtb &&
+                                  *(volatile uint64_t*)&p.dctl->dq_tail == c;
+            if (__shfl_sync(0xffffffffu, done, 0)) break;
+            __nanosleep(idle < 16 ? 64 : 512);
+            idle++;
+            continue;
+        }
+        idle = 0;
+        asm volatile("fence.acq_rel.sys;" ::: "memory");
+        for (uint32_t i = lane; i < n; i += 32u) {
+            uint64_t* q = &p.dq[(c + i) & p.dq_mask];
+            const uint64_t id = *(volatile uint64_t*)q - 1;
+            st_relaxed_sys(reinterpret_cast<volatile uint64_t*>(&p.comp[id & p.comp_mask]), id);
+            st_relaxed_gpu(q, 0);
+        }
+        __syncwarp();
+        c += n;
+    }
+    if (lane == 0) *(volatile uint64_t*)&p.dctl->dq_head = c;
+}
+
 /* ------------------------------------------------------------------ task execution
  * Alg. 1 L29-43: run the body, then the deferred release: the last
  * warp of a TB returns its shmem granules and barrier ID through the mailbox
@@ -192,9 +316,10 @@ __device__ __forceinline__ void run_task(MtbShared& S, char* smem_base, const Mk
     TaskEnv env{s, smem_base, &S.stage_bar[w], &stage_phase, &p.dctl->error, resident};
     if (!run_body(t.func_id, env, t.args) && lane == 0) atomicOr(&p.dctl->error, PAGODA_DEVERR_BAD_FUNC);
     __syncwarp();
+    uint32_t last = 0;
     if (lane == 0) {
         /* this warp's global writes -> visible GPU-wide before anyone learns the warp is done
-         * (release; the last warp's st.release.sys then publishes them system-wide) */
+         * (release; the completion poster's system-scope fence then publishes them to the host) */
         asm volatile("fence.acq_rel.gpu;" ::: "memory");
         if (p.trace_cap) {
             uint32_t* cnt = &p.exec_count[mtb * 32 + w];
@@ -209,17 +334,46 @@ __device__ __forceinline__ void run_task(MtbShared& S, char* smem_base, const Mk
         }
         if (atomicSub(&S.tb_warps_left[s.tbslot], 1u) == 1u) atomicOr(&S.mb_tbs, 1u << s.tbslot);
         if (atomicSub(&S.task_warps_left[s.task], 1u) == 1u) {
-            /* last warp of the task (Alg. 1 L41-42): the task's writes, ordered before the
-             * counter decrements of all its warps, become visible system-wide before the
-             * completion record the host polls (a posted PCIe write, no handshake). */
-            st_release_sys(&p.comp[s.task_id & p.comp_mask], (int64_t)s.task_id);
-            atomicOr(&S.mb_tasks, 1u << s.task);
+            /* last warp of the task (Alg. 1 L41-42): its completion record is pending */
+            atomicOr(&S.comp_pending, 1u << s.task);
+            __threadfence_block();   /* pending bit before the poster-flag attempt */
+            last = 1;
         }
+    }
+    if (__shfl_sync(0xffffffffu, last, 0)) post_completions(S, p);
+    if (lane == 0) {
         __threadfence_block();   /* TB / task frees are visible before the warp frees itself */
         atomicOr(&S.mb_warps, 1u << w);
         __threadfence_block();   /* ... and the warp's free bit before its attempt at the token */
     }
     __syncwarp();
+}
+
+/* MTB 0's host poster (n_mtb > 1): the ingest warp's host-visible stores
+ * (consumed count, device error word) are made here, so that the ingest warp's
+ * own fences never wait for a posted PCIe write.  Exits after every MTB did. */
+__device__ void host_poster(MtbShared& S, const MkParams& p)
+{
+    const uint32_t lane = threadIdx.x & 31u;
+    if (lane != 0) return;
+    uint64_t last = ~0ull;
+    uint32_t last_err = 0;
+    for (;;) {
+        const uint32_t done = *(volatile uint32_t*)&S.ingest_done;
+        const uint32_t exited = *(volatile uint32_t*)&p.dctl->exited;
+        const uint64_t c = *(volatile uint64_t*)&S.ingest_copied;
+        const uint32_t err = *(volatile uint32_t*)&p.dctl->error;
+        if (c != last) {
+            st_relaxed_sys(&p.hctl->consumed, c);
+            last = c;
+        }
+        if (err != last_err) {
+            st_relaxed_sys32(&p.hctl->error, err);
+            last_err = err;
+        }
+        if (done && exited >= (uint32_t)p.n_mtb) break;
+        __nanosleep(256);
+    }
 }
 
 /* ------------------------------------------------------------------ ingest
@@ -246,63 +400,139 @@ __device__ __forceinline__ void tma_store_1d(void* gdst, const void* smem_src, u
                  : "memory");
 }
 
-/* The ingest warp, a two-stage TMA pipeline: while stage s's batch (up to 256
- * entries = 16 KiB) is pulled from the pinned host ring by one bulk copy over
- * PCIe, the other stage's batch is bulk-stored into the device ring and its
- * cells are published.  A batch may wrap the ring end: then it is two copies. */
-__device__ __forceinline__ void fence_acq_rel_gpu()
-{
-    asm volatile("fence.acq_rel.gpu;" ::: "memory");
-}
+struct IngestCtr {
+    unsigned long long batches = 0, entries = 0, ns_db = 0, ns_copy = 0, ns_pub = 0, full = 0, ns_fence = 0,
+                       ns_store = 0;
+};
 
-__device__ void ingest(const MkParams& p, char* stage_buf, uint64_t* bars)
+/* Publish one staged batch [s, s+n) into the device ring: wait until its cells
+ * are free (seq == position: previous occupants loaded), acquire, bulk-store
+ * the entries, order them before the cells' release (seq = position + 1). */
+__device__ __forceinline__ bool ingest_publish(const MkParams& p, const char* src, uint64_t s, uint32_t n,
+                                               IngestCtr& c)
 {
     const uint32_t lane = threadIdx.x & 31u;
-    const uint32_t kIngestStageEntries = p.ingest_stage_entries;
     const uint64_t R = (uint64_t)p.ring_mask + 1;
+    for (uint32_t base = 0; base < n;) {   /* 256 cells per round trip (8 loads per lane) */
+        uint32_t sv[8];
+#pragma unroll
+        for (int i = 0; i < 8; i++) {
+            const uint32_t k = base + (uint32_t)i * 32u + lane;
+            /* acquire (LDG.STRONG + L1 invalidate, no MEMBAR): the cell's previous reader is done */
+            sv[i] = k < n ? ld_acquire_gpu32(&p.dseq[(s + k) & p.ring_mask]) : (uint32_t)(s + k);
+        }
+        uint32_t bad = 0;
+#pragma unroll
+        for (int i = 0; i < 8; i++) bad |= __ballot_sync(0xffffffffu, sv[i] != (uint32_t)(s + base + (uint32_t)i * 32u + lane));
+        if (bad) {   /* device ring full: wait for the schedulers */
+            c.full++;
+            if (*(volatile uint32_t*)&p.dctl->stop == kStopAbort) return false;
+            __nanosleep(128);
+            continue;
+        }
+        base += 256u;
+    }
+    const uint64_t t3 = globaltimer_ns();
+    __syncwarp();          /* every lane's acquire precedes lane 0's bulk store */
+    const uint64_t t4 = globaltimer_ns();
+    if (lane == 0) {
+        asm volatile("fence.proxy.async.global;" ::: "memory");   /* generic acquire -> async-proxy writes */
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        const uint32_t e0 = (uint32_t)(s & p.ring_mask);
+        const uint32_t n1 = min(n, (uint32_t)(R - e0));
+        tma_store_1d(p.dring + e0, src, n1 * 64u);
+        if (n1 < n) tma_store_1d(p.dring, src + n1 * 64u, (n - n1) * 64u);
+        asm volatile("cp.async.bulk.commit_group;\n\tcp.async.bulk.wait_group 0;" ::: "memory");
+        asm volatile("fence.proxy.async.global;" ::: "memory");
+    }
+    __syncwarp();
+    const uint64_t t5 = globaltimer_ns();
+    fence_acq_rel_gpu();   /* the entry writes precede every lane's relaxed cell release */
+    const uint64_t t6 = globaltimer_ns();
+    c.ns_fence += (t4 - t3) + (t6 - t5);
+    c.ns_store += t5 - t4;
+    for (uint32_t i = lane; i < n; i += 32u) {
+        const uint64_t t = s + i;
+        st_relaxed_gpu32(&p.dseq[t & p.ring_mask], (uint32_t)(t + 1));
+    }
+    __syncwarp();
+    if (lane == 0) st_relaxed_gpu(&p.dctl->tail, s + n);   /* hint for schedulers: work exists */
+    c.batches++;
+    c.entries += n;
+    return true;
+}
+
+/* doorbell: lane 0 reads the host's published count and terminate word */
+__device__ __forceinline__ void ingest_doorbell(const MkParams& p, uint64_t& pub, uint32_t& term, uint32_t& last_err,
+                                                bool post_err, IngestCtr& c)
+{
+    const uint32_t lane = threadIdx.x & 31u;
+    const uint64_t t0 = globaltimer_ns();
+    uint32_t err = 0;
+    if (lane == 0) {
+        pub = ld_acquire_sys(&p.hctl->published);
+        term = ld_relaxed_sys32(&p.hctl->terminate);
+        err = *(volatile uint32_t*)&p.dctl->error;
+        if (post_err && err != last_err) st_relaxed_sys32(&p.hctl->error, err);
+    }
+    pub = __shfl_sync(0xffffffffu, pub, 0);
+    term = __shfl_sync(0xffffffffu, term, 0);
+    last_err = __shfl_sync(0xffffffffu, err, 0);
+    c.ns_db += globaltimer_ns() - t0;
+}
+
+/* issue the bulk copy of host ring entries [f, f+n) into a stage (lane 0) */
+__device__ __forceinline__ void ingest_load(const MkParams& p, char* dst, uint64_t f, uint32_t n, uint64_t* bar)
+{
+    if ((threadIdx.x & 31u) != 0) return;
+    const uint64_t R = (uint64_t)p.ring_mask + 1;
+    asm volatile("fence.proxy.async.global;" ::: "memory");   /* the doorbell acquire orders these reads */
+    const uint32_t e0 = (uint32_t)(f & p.ring_mask);
+    const uint32_t n1 = min(n, (uint32_t)(R - e0));
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(n * 64u) : "memory");
+    tma_load_1d(dst, p.hring + e0, n1 * 64u, bar);
+    if (n1 < n) tma_load_1d(dst + n1 * 64u, p.hring, (n - n1) * 64u, bar);
+}
+
+__device__ void ingest_flush(const MkParams& p, const IngestCtr& c)
+{
+    if ((threadIdx.x & 31u) != 0) return;
+    if (c.batches) atomicAdd(&p.dctl->ctr[PAGODA_CTR_INGEST_BATCHES], c.batches);
+    if (c.entries) atomicAdd(&p.dctl->ctr[PAGODA_CTR_INGEST_ENTRIES], c.entries);
+    if (c.ns_db) atomicAdd(&p.dctl->ctr[PAGODA_CTR_INGEST_NS_DOORBELL], c.ns_db);
+    if (c.ns_copy) atomicAdd(&p.dctl->ctr[PAGODA_CTR_INGEST_NS_COPY], c.ns_copy);
+    if (c.ns_pub) atomicAdd(&p.dctl->ctr[PAGODA_CTR_INGEST_NS_PUBLISH], c.ns_pub);
+    if (c.full) atomicAdd(&p.dctl->ctr[PAGODA_CTR_INGEST_RING_FULL], c.full);
+    if (c.ns_fence) atomicAdd(&p.dctl->ctr[PAGODA_CTR_INGEST_NS_FENCE], c.ns_fence);
+    if (c.ns_store) atomicAdd(&p.dctl->ctr[PAGODA_CTR_INGEST_NS_STORE], c.ns_store);
+}
+
+/* Single-warp ingest (a context of one MTB, where MTB 0 also runs tasks): a
+ * two-stage TMA pipeline, stage s pulled from the host ring while the other
+ * is published; host-visible stores (consumed, error) made inline. */
+__device__ void ingest(MtbShared& S, const MkParams& p, char* stage_buf, uint64_t* bars)
+{
+    const uint32_t lane = threadIdx.x & 31u;
+    const uint32_t SE = p.ingest_stage_entries;
     uint64_t copied = *(volatile uint64_t*)&p.dctl->tail;   /* published into the device ring (resumes) */
     uint64_t fetched = copied;                               /* loaded (or loading) into a stage */
     uint64_t pub = copied;                                   /* last doorbell value seen */
     uint64_t st_start[2] = {0, 0};
     uint32_t st_n[2] = {0, 0};
-    uint32_t phase = 0;      /* bit s = parity of stage s's mbarrier */
-    uint32_t os = 0, ns = 0, inflight = 0, term = 0, last_err = 0;
+    uint32_t phase = 0, os = 0, ns = 0, inflight = 0, term = 0, last_err = 0;
     int idle = 0;
-    unsigned long long c_batches = 0, c_entries = 0, c_ns_db = 0, c_ns_copy = 0, c_ns_pub = 0, c_full = 0;
+    IngestCtr c;
     for (;;) {
-        /* ---- doorbell: only when everything seen so far is fetched */
         if (fetched >= pub) {
-            const uint64_t t0 = globaltimer_ns();
-            uint32_t err = 0;
-            if (lane == 0) {
-                pub = ld_acquire_sys(&p.hctl->published);
-                term = ld_relaxed_sys32(&p.hctl->terminate);
-                err = *(volatile uint32_t*)&p.dctl->error;
-                if (err != last_err) st_relaxed_sys32(&p.hctl->error, err);
-            }
-            pub = __shfl_sync(0xffffffffu, pub, 0);
-            term = __shfl_sync(0xffffffffu, term, 0);
-            last_err = __shfl_sync(0xffffffffu, err, 0);
-            c_ns_db += globaltimer_ns() - t0;
+            ingest_doorbell(p, pub, term, last_err, true, c);
             if (term == kStopAbort) {   /* host watchdog: abandon the queue, let idle MTBs exit */
                 if (lane == 0) st_release_gpu32(&p.dctl->stop, kStopAbort);
                 break;
             }
         }
-        /* ---- fill free stages (the doorbell acquire orders these async-proxy reads) */
         while (inflight < 2 && fetched < pub) {
-            const uint32_t n = (uint32_t)min(pub - fetched, (uint64_t)kIngestStageEntries);
-            if (lane == 0) {
-                asm volatile("fence.proxy.async.global;" ::: "memory");
-                char* dst = stage_buf + ns * (kIngestStageEntries * 64u);
-                const uint32_t e0 = (uint32_t)(fetched & p.ring_mask);
-                const uint32_t n1 = min(n, (uint32_t)(R - e0));
-                asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(&bars[ns])),
-                             "r"(n * 64u)
-                             : "memory");
-                tma_load_1d(dst, p.hring + e0, n1 * 64u, &bars[ns]);
-                if (n1 < n) tma_load_1d(dst + n1 * 64u, p.hring, (n - n1) * 64u, &bars[ns]);
-            }
+            const uint32_t n = (uint32_t)min(pub - fetched, (uint64_t)SE);
+            ingest_load(p, stage_buf + ns * (SE * 64u), fetched, n, &bars[ns]);
             st_start[ns] = fetched;
             st_n[ns] = n;
             fetched += n;
@@ -311,59 +541,15 @@ __device__ void ingest(const MkParams& p, char* stage_buf, uint64_t* bars)
             idle = 0;
         }
         if (inflight) {
-            /* ---- complete the oldest stage */
             const uint64_t t1 = globaltimer_ns();
             mbar_wait(&bars[os], (phase >> os) & 1u);
             phase ^= 1u << os;
-            const uint64_t s = st_start[os];
-            const uint32_t n = st_n[os];
             const uint64_t t2 = globaltimer_ns();
-            c_ns_copy += t2 - t1;
-            /* the device cells must be free: seq == position (their previous occupants loaded) */
-            for (uint32_t base = 0; base < n;) {   /* 256 cells per round trip (8 loads per lane) */
-                uint32_t sv[8];
-#pragma unroll
-                for (int i = 0; i < 8; i++) {
-                    const uint32_t k = base + (uint32_t)i * 32u + lane;
-                    sv[i] = k < n ? ld_relaxed_gpu32(&p.dseq[(s + k) & p.ring_mask]) : (uint32_t)(s + k);
-                }
-                uint32_t bad = 0;
-#pragma unroll
-                for (int i = 0; i < 8; i++)
-                    bad |= __ballot_sync(0xffffffffu, sv[i] != (uint32_t)(s + base + (uint32_t)i * 32u + lane));
-                if (bad) {   /* device ring full: wait for the schedulers */
-                    c_full++;
-                    __nanosleep(128);
-                    continue;
-                }
-                base += 256u;
-            }
-            fence_acq_rel_gpu();   /* acquire: the cells' previous readers are done with them */
-            if (lane == 0) {
-                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-                const char* src = stage_buf + os * (kIngestStageEntries * 64u);
-                const uint32_t e0 = (uint32_t)(s & p.ring_mask);
-                const uint32_t n1 = min(n, (uint32_t)(R - e0));
-                tma_store_1d(p.dring + e0, src, n1 * 64u);
-                if (n1 < n) tma_store_1d(p.dring, src + n1 * 64u, (n - n1) * 64u);
-                asm volatile("cp.async.bulk.commit_group;\n\tcp.async.bulk.wait_group 0;" ::: "memory");
-                asm volatile("fence.proxy.async.global;" ::: "memory");
-            }
-            __syncwarp();
-            fence_acq_rel_gpu();   /* the entry writes precede every lane's relaxed cell release */
-            for (uint32_t i = lane; i < n; i += 32u) {
-                const uint64_t t = s + i;
-                st_relaxed_gpu32(&p.dseq[t & p.ring_mask], (uint32_t)(t + 1));
-            }
-            __syncwarp();
-            copied = s + n;
-            if (lane == 0) {
-                st_relaxed_gpu(&p.dctl->tail, copied);     /* hint for schedulers: work exists */
-                st_relaxed_sys(&p.hctl->consumed, copied); /* host may now reuse those ring slots */
-            }
-            c_ns_pub += globaltimer_ns() - t2;
-            c_batches++;
-            c_entries += n;
+            c.ns_copy += t2 - t1;
+            if (!ingest_publish(p, stage_buf + os * (SE * 64u), st_start[os], st_n[os], c)) break;
+            copied = st_start[os] + st_n[os];
+            if (lane == 0) st_relaxed_sys(&p.hctl->consumed, copied);   /* host may reuse those ring slots */
+            c.ns_pub += globaltimer_ns() - t2;
             inflight--;
             os ^= 1u;
         } else if (term) {
@@ -374,13 +560,106 @@ __device__ void ingest(const MkParams& p, char* stage_buf, uint64_t* bars)
         }
     }
     if (lane == 0) {
-        atomicAdd(&p.dctl->ctr[PAGODA_CTR_INGEST_BATCHES], c_batches);
-        atomicAdd(&p.dctl->ctr[PAGODA_CTR_INGEST_ENTRIES], c_entries);
-        atomicAdd(&p.dctl->ctr[PAGODA_CTR_INGEST_NS_DOORBELL], c_ns_db);
-        atomicAdd(&p.dctl->ctr[PAGODA_CTR_INGEST_NS_COPY], c_ns_copy);
-        atomicAdd(&p.dctl->ctr[PAGODA_CTR_INGEST_NS_PUBLISH], c_ns_pub);
-        atomicAdd(&p.dctl->ctr[PAGODA_CTR_INGEST_RING_FULL], c_full);
+        *(volatile uint64_t*)&S.ingest_copied = copied;
+        __threadfence_block();
+        *(volatile uint32_t*)&S.ingest_done = 1u;
     }
+    ingest_flush(p, c);
+}
+
+/* Two-warp ingest (n_mtb > 1).  A fence waits for ALL of its warp's outstanding
+ * memory operations, including a bulk read of the host ring still crossing a
+ * busy PCIe link; so the warp that fences (the publisher) is not the warp that
+ * reads host memory (the loader).  They hand the two stages back and forth
+ * through mbarriers: full[s] (bulk copy landed; an arrival without bytes and
+ * n = ~0 ends the stream) and empty[s] (the publisher is done with the stage). */
+__device__ void ingest_loader(MtbShared& S, const MkParams& p, char* stage_buf)
+{
+    const uint32_t lane = threadIdx.x & 31u;
+    const uint32_t SE = p.ingest_stage_entries;
+    uint64_t fetched = *(volatile uint64_t*)&p.dctl->tail;
+    uint64_t pub = fetched;
+    uint32_t term = 0, last_err = 0, ns = 0;
+    uint32_t uses[2] = {0, 0};
+    int idle = 0;
+    IngestCtr c;
+    for (;;) {
+        if (fetched >= pub) {
+            ingest_doorbell(p, pub, term, last_err, false, c);
+            if (term == kStopAbort) {   /* host watchdog: the publisher sees stop and leaves too */
+                if (lane == 0) st_release_gpu32(&p.dctl->stop, kStopAbort);
+                break;
+            }
+        }
+        const bool end = term && fetched >= pub;
+        if (fetched < pub || end) {
+            if (uses[ns]) mbar_wait(&S.ingest_empty[ns], (uses[ns] - 1u) & 1u);   /* stage free again */
+            uses[ns]++;
+            if (end) {
+                if (lane == 0) {
+                    S.ing_n[ns] = ~0u;
+                    mbar_arrive(&S.ingest_bar[ns]);
+                }
+                break;
+            }
+            const uint32_t n = (uint32_t)min(pub - fetched, (uint64_t)SE);
+            if (lane == 0) {
+                S.ing_start[ns] = fetched;
+                S.ing_n[ns] = n;
+            }
+            ingest_load(p, stage_buf + ns * (SE * 64u), fetched, n, &S.ingest_bar[ns]);
+            fetched += n;
+            ns ^= 1u;
+            idle = 0;
+        } else if (++idle > 64) {
+            __nanosleep(256);
+        }
+    }
+    ingest_flush(p, c);
+}
+
+__device__ void ingest_publisher(MtbShared& S, const MkParams& p, char* stage_buf)
+{
+    const uint32_t lane = threadIdx.x & 31u;
+    const uint32_t SE = p.ingest_stage_entries;
+    uint32_t os = 0;
+    uint32_t uses[2] = {0, 0};
+    uint64_t copied = *(volatile uint64_t*)&p.dctl->tail;
+    bool aborted = false;
+    IngestCtr c;
+    for (;;) {
+        const uint64_t t1 = globaltimer_ns();
+        while (!mbar_try_wait(&S.ingest_bar[os], uses[os] & 1u, 20000u)) {
+            if (*(volatile uint32_t*)&p.dctl->stop == kStopAbort) {
+                aborted = true;
+                break;
+            }
+        }
+        if (aborted) break;
+        uses[os]++;
+        const uint64_t t2 = globaltimer_ns();
+        const uint32_t n = *(volatile uint32_t*)&S.ing_n[os];
+        if (n == ~0u) break;
+        c.ns_copy += t2 - t1;
+        const uint64_t s = *(volatile uint64_t*)&S.ing_start[os];
+        if (!ingest_publish(p, stage_buf + os * (SE * 64u), s, n, c)) {
+            aborted = true;
+            break;
+        }
+        copied = s + n;
+        if (lane == 0) {
+            *(volatile uint64_t*)&S.ingest_copied = copied;   /* for the host poster */
+            mbar_arrive(&S.ingest_empty[os]);
+        }
+        c.ns_pub += globaltimer_ns() - t2;
+        os ^= 1u;
+    }
+    if (lane == 0) {
+        if (!aborted) st_release_gpu32(&p.dctl->stop, 1u);   /* everything published: drain and exit */
+        __threadfence_block();
+        *(volatile uint32_t*)&S.ingest_done = 1u;
+    }
+    ingest_flush(p, c);
 }
 
 /* ------------------------------------------------------------------ scheduler
@@ -678,10 +957,9 @@ __device__ bool sched_round(MtbShared& S, Sched& st, const MkParams& p, int mtb,
         st.ph++;
         progress = true;
     }
-    /* MTB 0 (one warp short: it hosts the ingest warp) takes no blind tickets unless it is the
-     * only MTB (validation then caps every task to its capacity), so no ticket lands where it
-     * can never fit */
-    if ((mtb != 0 || p.n_mtb == 1) && sched_claim(S, st, p) > 0) progress = true;
+    /* MTB 0 (the I/O MTB: ingest, host stores) and the MTB sharing its SM take no tickets
+     * unless MTB 0 is the only MTB (validation then caps every task to its capacity) */
+    if (!S.no_tickets && sched_claim(S, st, p) > 0) progress = true;
     exit = false;
     sc_add(S, kScRounds, 1);
     if (progress) sc_add(S, kScProgress, 1);
@@ -797,12 +1075,29 @@ __global__ void __launch_bounds__(1024, kMinBlocks) master_kernel(MkParams p)
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, mtb = blockIdx.x;
     int arena_granules = p.arena_granules;
     char* ingest_stage = nullptr;
-    if (mtb == 0) {   /* MTB 0 lends the top of its arena to the ingest warp */
+    const bool io = mtb == 0 && p.n_mtb > 1;   /* the I/O MTB: runs no tasks */
+    if (io) {
+        ingest_stage = smem_base + p.stage_offset;   /* everything after the control block */
+        arena_granules = 0;
+    } else if (mtb == 0) {   /* MTB 0 alone: it lends the top of its arena to the ingest warp */
         arena_granules -= (int)(2u * p.ingest_stage_entries * 64u / PAGODA_GRANULE);
         ingest_stage = smem_base + p.arena_offset + (size_t)arena_granules * PAGODA_GRANULE;
     }
+    /* PCIe isolation: MTB 0 announces its SM; an MTB on the same SM runs no tasks either */
+    uint32_t no_tickets = io ? 1u : 0u;
+    if (p.n_mtb > 1 && threadIdx.x == 0) {
+        uint32_t smid;
+        asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+        if (mtb == 0) {
+            st_release_gpu32(&p.dctl->io_smid, smid);
+        } else {   /* co-resident with MTB 0 by the cooperative launch: it writes at once */
+            uint32_t io_sm;
+            while ((io_sm = ld_acquire_gpu32(&p.dctl->io_smid)) == kIoSmidNone) __nanosleep(32);
+            if (io_sm == smid && p.io_sm_exclusive) no_tickets = 1u;
+        }
+    }
     uint32_t resident = 0;   /* shared-window address of the resident tables */
-    if (p.resident_tdes_src) {
+    if (p.resident_tdes_src && !io) {
         /* task-class resident tables (key-independent 3DES S-box/P tables), one copy per
          * lane, at the constant window address kResidentTdesAddr (bodies.cuh tdes_f):
          * word 4096 p + 64 v + 32 h + lane holds SP[j][v] for box j = byte p of x (h = 0:
@@ -824,11 +1119,16 @@ __global__ void __launch_bounds__(1024, kMinBlocks) master_kernel(MkParams p)
     /* worker warps 0..exec_warps-1 (MTB 0: minus the ingest warp) */
     uint32_t exec_mask = p.exec_warps >= 32 ? 0xffffffffu : ((1u << p.exec_warps) - 1u);
     if (mtb == 0) exec_mask &= ~(1u << kIngestWarp);
+    if (io)   /* the I/O roles: loader (31), host poster (30), publisher (29), forwarder (28) */
+        exec_mask &= ~((1u << kHostPosterWarp) | (1u << kIngestPublisherWarp) | (1u << kForwarderWarp));
     const int first = __ffs(exec_mask) - 1;
     if (warp == 0) {
         mbar_init(&S.exec_bar[lane], 1);
         mbar_init(&S.stage_bar[lane], 1);
-        if (lane < 2) mbar_init(&S.ingest_bar[lane], 1);
+        if (lane < 2) {
+            mbar_init(&S.ingest_bar[lane], 1);
+            mbar_init(&S.ingest_empty[lane], 1);
+        }
         /* initial scheduler state, owned by the first worker (it starts with the token) */
         S.sst_fg[lane] = bm_range_bits(0, (uint32_t)arena_granules, lane);
         if (lane == 0) {
@@ -841,12 +1141,23 @@ __global__ void __launch_bounds__(1024, kMinBlocks) master_kernel(MkParams p)
             S.sst_est_w = 0;
             S.sst_seq = 0;
             S.token = 1;
+            S.comp_pending = 0;
+            S.no_tickets = no_tickets;
+            S.poster = 0;
+            /* where ingest resumes: the host poster must never post a smaller consumed count
+             * (a spawn blocked on a ring slot would wait for it forever) */
+            S.ingest_copied = *(volatile uint64_t*)&p.dctl->tail;
+            S.ingest_done = 0;
             for (int i = 0; i < 8; i++) S.sctr[i] = 0;
             asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         }
     }
     __syncthreads();
-    if (mtb == 0 && warp == kIngestWarp) ingest(p, ingest_stage, S.ingest_bar);
+    if (mtb == 0 && p.n_mtb == 1 && warp == kIngestWarp) ingest(S, p, ingest_stage, S.ingest_bar);
+    else if (mtb == 0 && warp == kIngestWarp) ingest_loader(S, p, ingest_stage);
+    else if (mtb == 0 && warp == kIngestPublisherWarp) ingest_publisher(S, p, ingest_stage);
+    else if (mtb == 0 && warp == kHostPosterWarp) host_poster(S, p);
+    else if (mtb == 0 && warp == kForwarderWarp) comp_forwarder(S, p);
     else if ((exec_mask >> warp) & 1u) worker(S, smem_base, p, mtb, warp, resident, exec_mask, warp == first);
 }
 

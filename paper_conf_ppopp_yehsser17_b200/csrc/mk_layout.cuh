@@ -51,7 +51,11 @@ struct DevCtl {
     alignas(128) uint32_t error;   /* device error word (executors atomicOr) */
     alignas(128) uint32_t exited;  /* MTBs that exited */
     alignas(128) unsigned long long ctr[kNumCounters];   /* runtime counters (pagoda_read_counters) */
+    alignas(128) uint64_t dq_tail; /* completion queue: records reserved by task posters (fetch-add) */
+    alignas(128) uint64_t dq_head; /* completion queue: records forwarded to the host (forwarder; resumes) */
+    alignas(128) uint32_t io_smid; /* the SM of MTB 0 (kIoSmidNone until MTB 0 starts) */
 };
+constexpr uint32_t kIoSmidNone = 0xFFFFFFFFu;
 
 struct LedgerEvent {   /* 32 B; identical field order to the oracle's checker input */
     uint32_t seq;
@@ -96,6 +100,10 @@ struct MkParams {
     const uint32_t* resident_tdes_src;   /* 2 KiB SP table in device memory, replicated per lane
                                             at kResidentOffset when non-null */
     int      n_mtb;
+    uint64_t*        dq;      /* device completion queue (n_mtb > 1): id + 1 per record, 0 = empty */
+    uint32_t dq_mask;
+    uint32_t stage_offset;    /* n_mtb > 1: MTB 0's ingest stages start at this dynamic-smem offset */
+    uint32_t io_sm_exclusive; /* the MTB sharing MTB 0's SM runs no tasks (several SMs) */
     uint32_t trace_cap;       /* 0 = tracing off */
     LedgerEvent* trace;       /* [n_mtb][trace_cap] */
     uint32_t*    trace_count; /* [n_mtb] */
@@ -104,13 +112,20 @@ struct MkParams {
 };
 
 constexpr int kIngestWarp = 31;          /* warp 31 of MTB 0 feeds the device ring */
-/* ingest staging: 2 stages of MkParams::ingest_stage_entries entries (64 B each), lent by MTB 0
- * from the top of its arena; the host sizes them (ingest_stage_entries()) */
+constexpr int kHostPosterWarp = 30;      /* warp 30 of MTB 0 (when n_mtb > 1): host-visible ingest stores */
+constexpr int kIngestPublisherWarp = 29; /* warp 29 of MTB 0 (when n_mtb > 1): publishes staged batches;
+                                            warp 31 then only loads them from the host ring */
+constexpr int kForwarderWarp = 28;       /* warp 28 of MTB 0 (when n_mtb > 1): completion records -> host */
+constexpr uint32_t kDqEntries = 1u << 16;  /* device completion queue */
+/* ingest staging: 2 stages of MkParams::ingest_stage_entries entries (64 B each).  One MTB: lent
+ * from the top of MTB 0's arena (128 entries).  Several: MTB 0 runs no tasks and gives its whole
+ * shared memory after the control block (stage_offset) to them. */
 constexpr uint32_t kIngestMaxStageEntries = 1024;
-__host__ __device__ inline uint32_t ingest_stage_entries(uint32_t arena_bytes, int n_mtb)
+constexpr uint32_t kStageOffset = 6144;   /* > kControlBytes, 1 KiB aligned */
+__host__ __device__ inline uint32_t ingest_stage_entries(uint32_t smem_bytes, int n_mtb)
 {
     if (n_mtb == 1) return 128;   /* MTB 0 also runs tasks: keep most of its arena */
-    uint32_t e = arena_bytes / (2u * 64u) / 32u * 32u;
+    uint32_t e = (smem_bytes - kStageOffset) / (2u * 64u) / 32u * 32u;
     return e > kIngestMaxStageEntries ? kIngestMaxStageEntries : e;
 }
 constexpr uint32_t kStopAbort = 2;       /* HostCtl.terminate / DevCtl.stop value: abandon work and exit */
@@ -143,6 +158,14 @@ struct MtbShared {
     uint32_t  token;                 /* 1 while some warp holds the scheduler token */
     uint32_t  sctr[8];               /* scheduler counters (holder-only), flushed at exit */
     uint64_t  ingest_bar[2];         /* MTB 0: the ingest warp's two TMA stage mbarriers */
+    uint64_t  ingest_empty[2];       /* MTB 0: stage s free again (publisher -> loader) */
+    uint64_t  ing_start[2];          /* MTB 0: first ring position of the batch in stage s */
+    uint32_t  ing_n[2];              /* MTB 0: entries in stage s (~0: end of stream) */
+    uint64_t  ingest_copied;         /* MTB 0: entries published into the device ring (for the host poster) */
+    uint32_t  ingest_done;           /* MTB 0: the ingest warp has exited */
+    uint32_t  comp_pending;          /* task slots finished, completion record not yet posted */
+    uint32_t  no_tickets;            /* this MTB runs no tasks (MTB 0 and the MTB sharing its SM) */
+    uint32_t  poster;                /* 1 while some warp posts completion records */
 };
 static_assert(offsetof(MtbShared, wt) == kWarpTableOffset, "WarpTable offset");
 static_assert(sizeof(MtbShared) <= kControlBytes && kControlBytes <= kResidentOffset, "control block fits");

@@ -57,6 +57,7 @@ struct pagoda_ctx {
     TaskEntry* dring = nullptr;
     uint32_t* resident_src = nullptr;
     uint32_t* dseq = nullptr;
+    uint64_t* dq = nullptr;                 /* device completion queue (n_mtb > 1) */
     DevCtl* dctl = nullptr;
     LedgerEvent* trace = nullptr;
     uint32_t* trace_count = nullptr;
@@ -209,11 +210,16 @@ static int stop_kernel(pagoda_ctx* c, bool abort_now = false)
      * except tickets handed out past the final tail, which are void: head = tail */
     c->hctl->terminate = 0;
     const uint32_t zero = 0;
+    uint32_t derr = 0;   /* the device error word, whether or not the kernel posted it before exiting */
+    cudaMemcpy(&derr, &c->dctl->error, 4, cudaMemcpyDeviceToHost);
+    if (derr) c->hctl->error |= derr;
     uint64_t tail = 0;
     cudaMemcpy(&tail, &c->dctl->tail, 8, cudaMemcpyDeviceToHost);
     cudaMemcpy(&c->dctl->head, &tail, 8, cudaMemcpyHostToDevice);
     cudaMemcpy(&c->dctl->stop, &zero, 4, cudaMemcpyHostToDevice);
     cudaMemcpy(&c->dctl->exited, &zero, 4, cudaMemcpyHostToDevice);
+    const uint32_t none = kIoSmidNone;   /* MTB 0 announces its SM again next session */
+    cudaMemcpy(&c->dctl->io_smid, &none, 4, cudaMemcpyHostToDevice);
     if (cudaStreamSynchronize(c->stream) != cudaSuccess) return -EIO;
     return c->hctl->error ? -EIO : 0;
 }
@@ -226,6 +232,7 @@ static void free_ctx(pagoda_ctx* c)
     if (c->comp) cudaFreeHost((void*)c->comp);
     if (c->dring) cudaFree(c->dring);
     if (c->dseq) cudaFree(c->dseq);
+    if (c->dq) cudaFree(c->dq);
     if (c->resident_src) cudaFree(c->resident_src);
     if (c->dctl) cudaFree(c->dctl);
     if (c->trace) cudaFree(c->trace);
@@ -308,6 +315,9 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
     }
     if (cudaMalloc(&c->dctl, sizeof(DevCtl)) != cudaSuccess) goto fail;
     if (cudaMemset(c->dctl, 0, sizeof(DevCtl)) != cudaSuccess) goto fail;
+    if (cudaMemset(&c->dctl->io_smid, 0xFF, sizeof(uint32_t)) != cudaSuccess) goto fail;
+    if (cudaMalloc(&c->dq, (size_t)kDqEntries * sizeof(uint64_t)) != cudaSuccess) goto fail;
+    if (cudaMemset(c->dq, 0, (size_t)kDqEntries * sizeof(uint64_t)) != cudaSuccess) goto fail;
     if (cfg.flags & PAGODA_TRACE) {
         const size_t cap = cfg.trace_events ? cfg.trace_events : 8192;
         c->cfg.trace_events = (uint32_t)cap;
@@ -339,7 +349,11 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
         p.exec_warps = (int)cfg.exec_warps;
         p.arena_granules = (int)arena_g;
         p.arena_offset = arena_offset;
-        p.ingest_stage_entries = ingest_stage_entries(cfg.arena_bytes, c->n_mtb);
+        p.ingest_stage_entries = ingest_stage_entries(c->n_mtb == 1 ? cfg.arena_bytes : (uint32_t)smem, c->n_mtb);
+        p.stage_offset = kStageOffset;
+        p.io_sm_exclusive = nsm > 1 ? 1u : 0u;   /* one SM: its other MTB must run the tasks */
+        p.dq = c->dq;
+        p.dq_mask = kDqEntries - 1;
         if (cfg.flags & PAGODA_RESIDENT_TDES) {   /* the key-independent SP table, replicated by each MTB */
             std::vector<uint8_t> tab(PAGODA_TDES_TABLE_BYTES);
             const uint8_t zero_key[24] = {0};

@@ -216,7 +216,7 @@ class Pagoda:
 
     COUNTERS = ("ingest_batches", "ingest_entries", "ingest_ns_doorbell", "ingest_ns_copy", "ingest_ns_publish",
                 "ingest_ring_full", "sched_rounds", "sched_progress", "tickets", "claim_empty", "load_not_ready",
-                "placed", "place_nofit", "handoffs")
+                "placed", "place_nofit", "handoffs", "ingest_ns_fence", "ingest_ns_store")
 
     def counters(self) -> dict:
         out = np.zeros(16, np.uint64)

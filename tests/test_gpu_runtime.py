@@ -268,3 +268,17 @@ def test_sessions_stop_start_and_drain():
     assert (c == 64).all()
     o = Dev.get(out, np.uint32).reshape(n, 64)
     assert (o == (np.arange(n) + 1)[:, None]).all()
+
+
+@pytest.mark.gpu
+def test_session_starting_exactly_at_the_ring_wrap():
+    """Each session spawns exactly R tasks, so every new session's first spawn
+    needs ring slot 0 of the previous lap: the host must see the consumed count
+    of the previous session (a reset of it would block the spawn forever)."""
+    R = 4096
+    from paper_conf_ppopp_yehsser17_b200.pagoda import NO_START
+    with Pagoda(ring_entries=R, flags=NO_START, watchdog_s=20.0) as p:
+        for _ in range(4):
+            assert p.start() == 0
+            p.spawn_many(R, 128, 1, 0, False, T.NOP, None)
+            assert p.stop() == 0
