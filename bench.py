@@ -432,7 +432,7 @@ def e2e_run(p, w, steps, torch):
     per_in = per_out = 4096
     host_in = torch.from_numpy(w.host["packets"].reshape(-1).copy()).pin_memory()
     host_out = torch.empty(w.n * per_out, dtype=torch.uint8).pin_memory()
-    chunks = 16
+    chunks, ahead = 32, 4
     bounds = np.linspace(0, w.n, chunks + 1).astype(int)
     s_in, s_out = torch.cuda.Stream(), torch.cuda.Stream()
     dev = torch.cuda.current_device()
@@ -470,15 +470,21 @@ def e2e_run(p, w, steps, torch):
         th = threading.Thread(target=drain, args=(q, done, t0), daemon=True)
         th.start()
         evs = []
-        for c in range(chunks):            # every H2D copy queued at once on the copy stream
+
+        def issue(c):                      # H2D copy of chunk c on the copy stream
             lo, hi = bounds[c], bounds[c + 1]
             with torch.cuda.stream(s_in):
                 din[lo * per_in:hi * per_in].copy_(host_in[lo * per_in:hi * per_in], non_blocking=True)
                 e = torch.cuda.Event()
                 e.record(s_in)
             evs.append(e)
-        for c in range(chunks):            # a chunk's tasks are spawned as soon as its bytes landed
-            lo, hi = bounds[c], bounds[c + 1]
+
+        for c in range(min(ahead, chunks)):
+            issue(c)
+        for c in range(chunks):            # a chunk's tasks are spawned as soon as its bytes landed;
+            lo, hi = bounds[c], bounds[c + 1]   # copies stay `ahead` chunks in front
+            if c + ahead < chunks:
+                issue(c + ahead)
             evs[c].synchronize()
             tl["h2d"].append((time.perf_counter_ns() - t0) / 1e3)
             ids = p.spawn_shapes(w.shapes[lo:hi], w.args[lo:hi], ids=True)
@@ -494,7 +500,7 @@ def e2e_run(p, w, steps, torch):
     tot = sum(times)
     return {"value": w.n * steps / tot, "unit": "tasks/s", "h2d_bytes_per_step": w.n * per_in,
             "d2h_bytes_per_step": w.n * per_out, "ms_per_step": 1e3 * tot / steps,
-            "how": "pinned host packets -> H2D (16 chunks, copy stream) -> taskSpawn per task; a drain thread "
+            "how": "pinned host packets -> H2D (32 chunks, copy stream, 4 ahead) -> taskSpawn per task; a drain thread "
                    "waitBelow()s each chunk and queues its D2H on a second copy stream (both directions overlap)",
             "timeline_us": {k: [round(x, 1) for x in v] for k, v in tl.items()}}
 

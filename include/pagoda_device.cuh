@@ -73,40 +73,48 @@ __device__ __forceinline__ uint32_t smem_u32(const void* p)
     return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
 
-/* ---------------------------------------------------------------- TaskEnv */
+/* ---------------------------------------------------------------- TaskEnv
+ * Everything a body asks for is read from the executor warp's WarpTable slot in
+ * shared memory when asked (no register holds it across the body). */
+constexpr uint32_t kStageBarOffset = 256;     /* per-warp TMA staging mbarriers (MtbShared.stage_bar) */
+constexpr uint32_t kStagePhaseOffset = 4900;  /* their parities, one u32 per warp (MtbShared.stage_ph) */
+
 struct TaskEnv {
-    WarpSlot s;
-    char*     smem_base;    /* MTB dynamic shared memory base */
-    uint64_t* stage_bar;    /* this warp's staging mbarrier */
-    uint32_t* stage_phase;  /* its parity (register of the executor loop) */
     uint32_t* dev_error;    /* device error word */
     uint32_t  resident;     /* shared-window address of the MTB-resident 3DES tables, 0 if none */
 
+    static __device__ __forceinline__ unsigned char* mk_smem()
+    {   /* the __shared__ symbol itself, so nvcc emits LDS/STS, not generic LD/ST */
+        extern __shared__ __align__(1024) unsigned char pagoda_mk_smem[];
+        return pagoda_mk_smem;
+    }
+    __device__ __forceinline__ const WarpSlot& s() const
+    {
+        return *reinterpret_cast<const WarpSlot*>(mk_smem() + kWarpTableOffset + (threadIdx.x >> 5) * sizeof(WarpSlot));
+    }
     __device__ __forceinline__ int getTid() const
     {
-        return ((int)s.tb * (int)s.warps_tb + (int)s.warp_in_tb) * 32 + (int)lane_id();
+        const WarpSlot& w = s();
+        return ((int)w.tb * (int)w.warps_tb + (int)w.warp_in_tb) * 32 + (int)lane_id();
     }
-    __device__ __forceinline__ int getBlockIdx() const { return s.tb; }
-    __device__ __forceinline__ int getBlockTid() const { return (int)s.warp_in_tb * 32 + (int)lane_id(); }
-    __device__ __forceinline__ int getBlockDim() const { return s.threads_tb; }
-    __device__ __forceinline__ int getBlockWarps() const { return s.warps_tb; }
-    __device__ __forceinline__ int getNumBlocks() const { return s.n_tb; }
-    __device__ __forceinline__ char* getSMPtr() const
-    {   /* derived from the __shared__ symbol itself, so nvcc emits LDS/STS, not generic LD/ST */
-        extern __shared__ __align__(1024) unsigned char pagoda_mk_smem[];
-        return reinterpret_cast<char*>(pagoda_mk_smem) + s.smem_off;
-    }
-    __device__ __forceinline__ uint32_t getSMBytes() const { return s.smem_bytes; }
+    __device__ __forceinline__ int getBlockIdx() const { return s().tb; }
+    __device__ __forceinline__ int getBlockTid() const { return (int)s().warp_in_tb * 32 + (int)lane_id(); }
+    __device__ __forceinline__ int getBlockDim() const { return s().threads_tb; }
+    __device__ __forceinline__ int getBlockWarps() const { return s().warps_tb; }
+    __device__ __forceinline__ int getNumBlocks() const { return s().n_tb; }
+    __device__ __forceinline__ char* getSMPtr() const { return reinterpret_cast<char*>(mk_smem()) + s().smem_off; }
+    __device__ __forceinline__ uint32_t getSMBytes() const { return s().smem_bytes; }
     /* MTB-resident, lane-replicated 3DES SP tables (context flag PAGODA_RESIDENT_TDES) */
     __device__ __forceinline__ uint32_t getResidentTdes() const { return resident; }
     /* true if syncBlock() is legal: a 1-warp TB, or a TB spawned with sync=1 */
-    __device__ __forceinline__ bool canSync() const { return s.warps_tb == 1 || s.bar_id != 0; }
+    __device__ __forceinline__ bool canSync() const { return s().warps_tb == 1 || s().bar_id != 0; }
     __device__ __forceinline__ void syncBlock() const
     {
-        if (s.warps_tb == 1) {
+        const uint32_t wtb = s().warps_tb, bar = s().bar_id;
+        if (wtb == 1) {
             __syncwarp();
-        } else if (s.bar_id != 0) {
-            named_bar_sync(s.bar_id, 32u * s.warps_tb);
+        } else if (bar != 0) {
+            named_bar_sync(bar, 32u * wtb);
         } else {
             /* spawned with sync=0: contract violation */
             atomicOr(dev_error, 1u);
@@ -120,7 +128,9 @@ struct TaskEnv {
     __device__ __forceinline__ void stage(void* smem_dst, const void* gsrc, uint32_t bytes) const
     {
         if (bytes == 0) return;
-        uint32_t bar = smem_u32(stage_bar);
+        const uint32_t warp = threadIdx.x >> 5;
+        const uint32_t bar = smem_u32(mk_smem() + kStageBarOffset + warp * 8u);
+        uint32_t* stage_phase = reinterpret_cast<uint32_t*>(mk_smem() + kStagePhaseOffset + warp * 4u);
         if (lane_id() == 0) {
             asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
             asm volatile(

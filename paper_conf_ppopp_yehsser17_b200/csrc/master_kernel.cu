@@ -203,7 +203,7 @@ __device__ __forceinline__ void trace_ev(const MkParams& p, int mtb, uint32_t& s
  * MTB there is no such split: the record goes to the host directly behind a
  * system-scope fence.  The task slot is returned (mb_tasks) only after its id
  * was read, so the id stays valid until then. */
-__device__ __noinline__ void post_completions(MtbShared& S, const MkParams& p)
+__device__ __forceinline__ void post_completions(MtbShared& S, const MkParams& p)
 {
     const uint32_t lane = threadIdx.x & 31u;
     for (;;) {
@@ -307,13 +307,14 @@ __device__ void comp_forwarder(MtbShared& S, const MkParams& p)
  * (markSMForDealloc), the last warp of the task posts its completion record,
  * every warp returns itself. */
 __device__ __forceinline__ void run_task(MtbShared& S, char* smem_base, const MkParams& p, int mtb, int w,
-                                         uint32_t resident, uint32_t& stage_phase, const WarpSlot& s)
+                                         uint32_t resident)
 {
     const uint32_t lane = threadIdx.x & 31u;
+    const WarpSlot& s = S.wt[w];   /* read from shared memory when needed */
     const TaskEntry& t = S.tasks[s.task];
     uint64_t t0 = 0;
     if (p.trace_cap) t0 = globaltimer_ns();
-    TaskEnv env{s, smem_base, &S.stage_bar[w], &stage_phase, &p.dctl->error, resident};
+    TaskEnv env{&p.dctl->error, resident};
     if (!run_body(t.func_id, env, t.args) && lane == 0) atomicOr(&p.dctl->error, PAGODA_DEVERR_BAD_FUNC);
     __syncwarp();
     uint32_t last = 0;
@@ -1009,59 +1010,66 @@ __device__ void sched_handoff(MtbShared& S, Sched& st, const MkParams& p, int mt
     }
 }
 
+/* One holder phase: the warp owns the scheduler token and runs rounds until it
+ * dispatched itself (hands the token on) or the session ends (returns true).
+ * The scheduler state lives only here (loaded from / saved to shared memory),
+ * so no register holds it while the warp runs task bodies. */
+__device__ __noinline__ bool holder_phase(MtbShared& S, const MkParams& p, int mtb, int w, uint32_t exec_mask)
+{
+    const uint32_t lane = threadIdx.x & 31u;
+    Sched st;
+    sst_load(S, st, exec_mask);
+    uint32_t backoff = 0;
+    for (;;) {
+        bool exit = false;
+        const bool progress = sched_round(S, st, p, mtb, exit);
+        if (exit) {   /* drain: release every other worker with a terminate slot */
+            if (((exec_mask & ~(1u << w)) >> lane) & 1u) {
+                S.wt[lane].task = SLOT_TERMINATE;
+                mbar_arrive(&S.exec_bar[lane]);
+            }
+            if (lane == 0) {
+                atomicAdd(&p.dctl->exited, 1u);
+                for (int i = 0; i < 8; i++)
+                    atomicAdd(&p.dctl->ctr[PAGODA_CTR_SCHED_ROUNDS + i], (unsigned long long)S.sctr[i]);
+            }
+            return true;
+        }
+        if ((st.free_w >> w) & 1u) {   /* still free: keep scheduling */
+            if (progress) backoff = 0;
+            else {
+                /* with work queued only shared-memory mailboxes are polled: stay responsive;
+                 * otherwise the ring is polled in L2: back off */
+                backoff = (st.ph != st.pt) ? 32u : (backoff ? min(backoff * 2u, 1024u) : 32u);
+                __nanosleep(backoff);
+            }
+            continue;
+        }
+        sched_handoff(S, st, p, mtb);   /* dispatched (by itself or before it took the token) */
+        return false;
+    }
+}
+
 /* Every worker warp runs this loop (warps 0..exec_warps-1; MTB 0's warp 31 ingests). */
 __device__ void worker(MtbShared& S, char* smem_base, const MkParams& p, int mtb, int w, uint32_t resident,
                        uint32_t exec_mask, bool holder)
 {
-    const uint32_t lane = threadIdx.x & 31u;
-    uint32_t phase = 0, stage_phase = 0, backoff = 0;
-    Sched st;
-    if (holder) sst_load(S, st, exec_mask);
+    uint32_t phase = 0;
     for (;;) {
         if (holder) {
-            bool exit = false;
-            const bool progress = sched_round(S, st, p, mtb, exit);
-            if (exit) {   /* drain: release every other worker with a terminate slot */
-                if (((exec_mask & ~(1u << w)) >> lane) & 1u) {
-                    S.wt[lane].task = SLOT_TERMINATE;
-                    mbar_arrive(&S.exec_bar[lane]);
-                }
-                if (lane == 0) {
-                    atomicAdd(&p.dctl->exited, 1u);
-                    for (int i = 0; i < 8; i++)
-                        atomicAdd(&p.dctl->ctr[PAGODA_CTR_SCHED_ROUNDS + i], (unsigned long long)S.sctr[i]);
-                }
-                return;
-            }
-            if ((st.free_w >> w) & 1u) {   /* still free: keep scheduling */
-                if (progress) backoff = 0;
-                else {
-                    /* with work queued only shared-memory mailboxes are polled: stay responsive;
-                     * otherwise the ring is polled in L2: back off */
-                    backoff = (st.ph != st.pt) ? 32u : (backoff ? min(backoff * 2u, 1024u) : 32u);
-                    __nanosleep(backoff);
-                }
-                continue;
-            }
-            sched_handoff(S, st, p, mtb);   /* dispatched (by itself or before it took the token) */
+            if (holder_phase(S, p, mtb, w, exec_mask)) return;
             holder = false;
         }
         mbar_wait(&S.exec_bar[w], phase);
         phase ^= 1u;
-        const WarpSlot s = S.wt[w];
-        if (s.task == SLOT_TERMINATE) return;
-        if (s.task == SLOT_SCHED) {
+        const uint8_t task = *(volatile uint8_t*)&S.wt[w].task;
+        if (task == SLOT_TERMINATE) return;
+        if (task == SLOT_SCHED) {
             holder = true;
-            backoff = 0;
-            sst_load(S, st, exec_mask);
             continue;
         }
-        run_task(S, smem_base, p, mtb, w, resident, stage_phase, s);
-        if (token_try(S)) {
-            holder = true;
-            backoff = 0;
-            sst_load(S, st, exec_mask);
-        }
+        run_task(S, smem_base, p, mtb, w, resident);
+        holder = token_try(S);
     }
 }
 
@@ -1125,6 +1133,7 @@ __global__ void __launch_bounds__(1024, kMinBlocks) master_kernel(MkParams p)
     if (warp == 0) {
         mbar_init(&S.exec_bar[lane], 1);
         mbar_init(&S.stage_bar[lane], 1);
+        S.stage_ph[lane] = 0;
         if (lane < 2) {
             mbar_init(&S.ingest_bar[lane], 1);
             mbar_init(&S.ingest_empty[lane], 1);

@@ -165,9 +165,12 @@ struct MtbShared {
     uint32_t  ingest_done;           /* MTB 0: the ingest warp has exited */
     uint32_t  comp_pending;          /* task slots finished, completion record not yet posted */
     uint32_t  no_tickets;            /* this MTB runs no tasks (MTB 0 and the MTB sharing its SM) */
+    uint32_t  stage_ph[32];          /* parity of each warp's staging mbarrier (TaskEnv::stage) */
     uint32_t  poster;                /* 1 while some warp posts completion records */
 };
 static_assert(offsetof(MtbShared, wt) == kWarpTableOffset, "WarpTable offset");
+static_assert(offsetof(MtbShared, stage_bar) == kStageBarOffset, "staging mbarriers offset");
+static_assert(offsetof(MtbShared, stage_ph) == kStagePhaseOffset, "staging parities offset");
 static_assert(sizeof(MtbShared) <= kControlBytes && kControlBytes <= kResidentOffset, "control block fits");
 
 } // namespace pagoda
