@@ -2,7 +2,7 @@
 """bench.py — narrow tasks/s and p50 spawn-to-done latency of the B200 Pagoda
 hot path (BASELINE.json "metric"), one JSON line on rank 0.
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload tdes|mb|mm|mix|nop]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload tdes|mb|mm|mix|nop|c5|mpe|tdes_var]
     python bench.py --impl reference ...     # the oracle on the host cores (base contract's reference arm)
     torchrun --nproc-per-node N bench.py --gpus N   # one process per GPU
 
@@ -44,7 +44,26 @@ BASE = json.load(open(os.path.join(ROOT, "BASELINE.json")))
 # algorithmic work per task
 TDES_LOOKUPS_PER_TASK = 512 * 48 * 8          # S-box table lookups (LDS) per 4 KiB packet
 LDS_LANES_PER_SM_CLK = 32                     # one 128 B shared-memory wavefront per SM per clock
-DTYPE = {"tdes": "u32", "mb": "f32", "mm": "f32", "mix": "f32", "nop": "none"}   # arithmetic type of the path
+DTYPE = {"tdes": "u32", "mb": "f32", "mm": "f32", "mix": "f32", "nop": "none", "c5": "f32+u32", "mpe": "f32+u32",
+         "tdes_var": "u32", "mm_tc": "tf32x3"}   # arithmetic type of the path
+WORKLOADS = ("tdes", "mb", "mm", "mix", "nop", "c5", "mpe", "tdes_var", "mm_tc")
+STRONG = ("c5",)   # total work fixed as N grows; the others: each rank runs the whole config
+
+# Algorithmic work per task by body:
+#   fma  = fp32 lane-ops on the FMA pipe (an FFMA, FMUL or FADD each count 1),
+#   lds  = S-box table lookups (shared-memory lanes), hbm = bytes in + out.
+# MB: 8 ops per iteration x 194,698 iterations, the config-1 tile average (configs 5 and MPE cycle
+# uniformly through config 1's 1024 tiles).  3DES: per 8-byte block 48 rounds x 8 lookups.
+DEMAND = {
+    "mb": {"fma": 8 * 199370695 / 1024, "hbm": 8192},
+    "mm": {"fma": 32768, "hbm": 12288},
+    "mm_tc": {"hbm": 12288},
+    "fb": {"fma": 130080, "hbm": 16640},
+    "bf": {"fma": 166912, "hbm": 25216},
+    "conv": {"fma": 557056, "hbm": 131208},
+    "dct": {"fma": 262144, "hbm": 131328},
+}
+TDES_LOOKUPS_PER_BLOCK = 48 * 8
 
 
 def parse():
@@ -53,7 +72,7 @@ def parse():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="pagoda", choices=["pagoda", "reference"])
-    ap.add_argument("--workload", default="tdes", choices=["tdes", "mb", "mm", "mix", "nop"])
+    ap.add_argument("--workload", default="tdes", choices=list(WORKLOADS))
     ap.add_argument("--no-naive", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
@@ -150,32 +169,88 @@ class Clocks:
 
 
 # ----------------------------------------------------------------- CPU oracle leg
+def oracle_tasks(workload: str, n_sample: int):
+    """The first n_sample tasks of the workload as oracle calls (host inputs
+    from inputs.py, the same seeded recipe the GPU workload uses)."""
+    import oracle
+    from paper_conf_ppopp_yehsser17_b200 import inputs as I
+    oracle.lib()
+
+    def body(kind, pool_host, j):
+        if kind == "mb":
+            return lambda: oracle.mandelbrot_tile(int(j % 1024) % 32, int(j % 1024) // 32)
+        if kind == "tdes":
+            flat, off = pool_host
+            return lambda: oracle.tdes_ecb(flat[off[j]:off[j + 1]], I.TDES_KEYS)
+        if kind == "mm":
+            A, B = pool_host
+            return lambda: oracle.mm32(A[j], B[j])
+        if kind == "fb":
+            r, H, F = pool_host
+            return lambda: oracle.filterbank(r[j], H[j], F[j])
+        if kind == "bf":
+            x, h, w = pool_host
+            return lambda: oracle.beamformer(x[j], h[j], w[j])
+        if kind == "conv":
+            img, kr, kc = pool_host
+            return lambda: oracle.conv(img[j], kr[j], kc[j])
+        im, coef = pool_host
+        return lambda: oracle.dct(im[j], coef)
+
+    def pool(kind, size, var=False):
+        if kind == "mb":
+            return None
+        if kind == "tdes":
+            return I.tdes_var_packets(I.tdes_var_sizes(size) if var else np.full(size, 4096, np.int64))
+        if kind == "mm":
+            return I.mm_inputs(size)
+        if kind == "fb":
+            return I.fb_inputs(size)
+        if kind == "bf":
+            return I.bf_inputs(size)
+        if kind == "conv":
+            return I.conv_inputs(size)
+        return I.dct_inputs(size), I.dct_coef()
+
+    if workload == "mm_tc":
+        A, B = I.mm_inputs(n_sample)
+        return [(lambda k=k: oracle.mm32_exact(A[k], B[k])) for k in range(n_sample)], \
+            f"{n_sample} 32x32x32 MM tasks (fp64-accumulated definition)"
+    if workload in ("tdes", "mb", "mm", "tdes_var"):
+        kind = "tdes" if workload == "tdes_var" else workload
+        ph = pool(kind, n_sample, var=workload == "tdes_var")
+        what = {"tdes": f"{n_sample} of the 32768 3DES packets (4 KiB, EDE3 ECB)",
+                "mb": f"{n_sample} Mandelbrot tiles of config 1", "mm": f"{n_sample} 32x32x32 fp32 MM tasks",
+                "tdes_var": f"{n_sample} of the irregular (2-64 KiB) 3DES packets"}[workload]
+        return [body(kind, ph, k) for k in range(n_sample)], what
+    if workload == "mix":
+        kinds = I.mix_schedule(n_sample)[0]
+        names = I.MIX_KINDS
+    elif workload == "mpe":
+        kinds = I.mpe_schedule(32768)[:n_sample]
+        names = I.MPE_KINDS
+    else:   # c5 (and nop: a mixed sample stands in)
+        kinds = I.c5_schedule(n_sample)[0]
+        names = I.C5_KINDS
+    pools = {k: pool(k, n_sample, var=workload == "mpe") for k in names}
+    rank = np.zeros(n_sample, np.int64)
+    for ki in range(len(names)):
+        i = np.nonzero(kinds == ki)[0]
+        rank[i] = np.arange(len(i))
+    # config 4 / MPE: each task its own input (the i-th of its kind); config 5: pool entry i mod 4096
+    idx = np.arange(n_sample) if workload in ("c5", "nop") else rank
+    what = f"the first {n_sample} tasks of {workload} ({', '.join(names)})"
+    return [body(names[kinds[k]], pools[names[kinds[k]]], int(idx[k])) for k in range(n_sample)], what
+
+
 def oracle_rate(workload: str, n_sample: int, threads: int):
     """The oracle as it stands, on `threads` host threads over n_sample tasks of
     the workload: returns (tasks/s, seconds, sample description)."""
     import concurrent.futures as cf
-
-    import oracle
-    from paper_conf_ppopp_yehsser17_b200 import inputs as I
-    oracle.lib()
-    if workload == "tdes":
-        pk = I.tdes_packets(n_sample)
-        def one(k): oracle.tdes_ecb(pk[k], I.TDES_KEYS)
-        what = f"{n_sample} of the 32768 3DES packets (4 KiB, EDE3 ECB)"
-    elif workload == "mb":
-        def one(k): oracle.mandelbrot_tile(k % 32, (k // 32) % 32)
-        what = f"{n_sample} Mandelbrot tiles of config 1"
-    elif workload == "mm":
-        A, B = I.mm_inputs(n_sample)
-        def one(k): oracle.mm32(A[k], B[k])
-        what = f"{n_sample} 32x32x32 fp32 MM tasks"
-    else:
-        r, H, F = I.fb_inputs(n_sample)
-        def one(k): oracle.filterbank(r[k], H[k], F[k])
-        what = f"{n_sample} FB tasks (mix proxy)"
+    calls, what = oracle_tasks(workload, n_sample)
     t0 = time.perf_counter()
     with cf.ThreadPoolExecutor(max_workers=threads) as ex:
-        list(ex.map(one, range(n_sample)))
+        list(ex.map(lambda f: f(), calls))
     dt = time.perf_counter() - t0
     return n_sample / dt, dt, what
 
@@ -185,7 +260,7 @@ def run_reference(a, d: Dist):
     if d.rank != 0:
         return
     threads = os.cpu_count() or 1
-    n_sample = {"tdes": 2048, "mb": 512, "mm": 20000, "mix": 2048, "nop": 2048}[a.workload]
+    n_sample = REF_SAMPLE[a.workload]
     wl = "tdes" if a.workload == "nop" else a.workload
     for _ in range(a.warmup):
         oracle_rate(wl, max(64, n_sample // 8), threads)
@@ -196,7 +271,8 @@ def run_reference(a, d: Dist):
     tot = sum(times)
     v = n_sample * a.steps / tot
     line = {"metric": BASE["metric"], "value": v, "unit": "tasks/s", "n_gpus": a.gpus, "steps": a.steps,
-            "warmup": a.warmup, "ms_per_step": 1e3 * tot / a.steps, "higher_is_better": True, "scaling": "weak",
+            "warmup": a.warmup, "ms_per_step": 1e3 * tot / a.steps, "higher_is_better": True,
+            "scaling": "strong" if wl in STRONG else "weak",
             "vs_baseline": None, "dtype": DTYPE[wl], "data": "synthetic",
             "impl": "reference",
             "config": workload_config(wl) | {"step_sample_tasks": n_sample},
@@ -217,11 +293,35 @@ def workload_config(name):
         "mix": {"workload": "configs[3]: FB/BF/CONV/DCT mix, 32768 tasks, 32-512 threads, 0-48 KiB shmem",
                 "n_tasks": 32768},
         "nop": {"workload": "NOP 128-thread tasks (runtime ceiling)", "n_tasks": 200000, "threads": 128},
+        "c5": {"workload": "configs[4]: 1M mixed tasks over the 7 bodies (MB, 3DES, MM as configs 1-3; FB/BF/CONV/DCT "
+                           "as config 4), per-kind pools of 4096 inputs replicated per GPU, strong scaling",
+               "n_tasks": 1000000, "l2": "outputs 32 GB > L2"},
+        "mpe": {"workload": "NEXT-1 MPE: MB + irregular 3DES (2-64 KiB) + FB + MM, 8192 tasks each",
+                "n_tasks": 32768},
+        "mm_tc": {"workload": "NEXT-4: configs[2] on the tensor cores (3xTF32 mma.sync), 65536 tasks x 256 threads",
+                  "n_tasks": 65536, "threads": 256, "l2": "inputs+outputs 768 MiB > L2"},
+        "tdes_var": {"workload": "NEXT-1 irregular 3DES: 32768 packets log-uniform 2-64 KiB, 128 threads each",
+                     "n_tasks": 32768, "l2": "inputs+outputs 1.2 GB > L2"},
     }[name]
 
 
-def make_workload(name, resident=False):
+REF_SAMPLE = {"tdes": 2048, "mb": 512, "mm": 20000, "mix": 2048, "nop": 2048, "c5": 2048, "mpe": 1024,
+              "tdes_var": 512, "mm_tc": 20000}   # --impl reference: tasks per step
+CPU_SAMPLE = {"tdes": 16384, "mb": 1024, "mm": 65536, "mix": 4096, "nop": 16384, "c5": 4096, "mpe": 4096,
+              "tdes_var": 4096, "mm_tc": 65536}  # cpu_baseline sample
+
+
+def make_workload(name, resident=False, d=None):
     from paper_conf_ppopp_yehsser17_b200 import workloads as W
+    if name == "c5":
+        return W.c5(1_000_000, resident=resident, shard=(d.rank, d.world) if d else (0, 1))
+    if name == "mpe":
+        return W.mpe(32768, resident=resident)
+    if name == "tdes_var":
+        return W.tdes_var(32768, resident=resident)
+    if name == "mm_tc":
+        from paper_conf_ppopp_yehsser17_b200 import tasks as T
+        return W.matmul(65536, func=T.MM_TC)
     if name == "tdes":   # with resident SP tables a task only stages its 384 B of round keys
         return W.tdes(32768, shmem=512 if resident else 2560)
     if name == "mb":
@@ -240,6 +340,10 @@ PRESETS = {
     "mm": {"mtbs_per_sm": 2, "arena_bytes": 96 * 1024, "resident": False},
     "mix": {"mtbs_per_sm": 1, "arena_bytes": 200 * 1024, "resident": False},
     "nop": {"mtbs_per_sm": 2, "arena_bytes": 96 * 1024, "resident": False},
+    "c5": {"mtbs_per_sm": 1, "arena_bytes": 144 * 1024, "resident": True},
+    "mpe": {"mtbs_per_sm": 2, "arena_bytes": 40 * 1024, "resident": True},
+    "tdes_var": {"mtbs_per_sm": 2, "arena_bytes": 40 * 1024, "resident": True},
+    "mm_tc": {"mtbs_per_sm": 2, "arena_bytes": 96 * 1024, "resident": False},
 }
 
 
@@ -270,7 +374,7 @@ def main():
     torch.cuda.set_device(d.local)
     dev = d.local
     peaks = measured_peaks()
-    w = make_workload(a.workload, use_resident(a))
+    w = make_workload(a.workload, use_resident(a), d)
     n = w.n
     out = {}
 
@@ -283,6 +387,17 @@ def main():
         out["naive"] = {"tasks_per_s": n / statistics.median(reps), "streams": 32,
                         "how": "one <<<n_tb, threads, shmem>>> launch per task, same bodies, 32 streams, "
                                "CUDA_DEVICE_MAX_CONNECTIONS=32, first launch -> cudaDeviceSynchronize"}
+
+    # --- static fusion (NEXT-2): every task in ONE launch, 256 threads per task
+    if not a.no_naive and not a.quick and w.name != "nop":
+        PG.fused_run(dev, w.shapes[: min(n, 2048)], w.args[: min(n, 2048)], 256)   # warm-up
+        reps = [PG.fused_run(dev, w.shapes, w.args, 256) for _ in range(3)]
+        host_ns = statistics.median(r[0] for r in reps)
+        out["static_fusion"] = {"tasks_per_s": n / (host_ns * 1e-9),
+                                "kernel_tasks_per_s": n / (statistics.median(r[1] for r in reps) * 1e-3),
+                                "threads_per_task": 256,
+                                "how": "one launch of n blocks x 256 threads, block i runs task i's body (task table "
+                                       "H2D inside the timed region); kernel_ only: CUDA events around the kernel"}
 
     p = PG.Pagoda(device=dev, **ctx_config(a, PG))
 
@@ -346,6 +461,15 @@ def main():
             p.spawn_shapes(w.shapes, w.args)
         assert p.waitAll() == 0
         out["persistent_tasks_per_s"] = 3 * n / ((time.perf_counter_ns() - t0) * 1e-9)
+        # Pagoda-Batching (NEXT-2): no spawn until the previous batch has finished;
+        # batch = what the GPU runs at once at 4 warps per task (8 per MTB)
+        batch = info.n_mtb * 8
+        t0 = time.perf_counter_ns()
+        for lo in range(0, n, batch):
+            p.spawn_shapes(w.shapes[lo:lo + batch], w.args[lo:lo + batch])
+            assert p.waitAll() == 0
+        out["batching"] = {"tasks_per_s": n / ((time.perf_counter_ns() - t0) * 1e-9), "batch": batch,
+                           "how": "spawn a batch, waitAll, spawn the next (GeMTC-style, P:1347-1352), same session"}
         assert p.stop() == 0
 
     # --- e2e: the same metric through the C-ABI with HOST buffers (copies inside the timed region)
@@ -358,15 +482,15 @@ def main():
     cpu = None
     if not a.no_cpu and not a.quick and d.rank == 0 and d.world == 1:
         threads = os.cpu_count() or 1
-        ns = {"tdes": 16384, "mb": 1024, "mm": 65536, "mix": 4096, "nop": 16384}[a.workload]
-        rate, dt, what = oracle_rate(a.workload if a.workload != "nop" else "tdes", ns, threads)
+        rate, dt, what = oracle_rate(a.workload if a.workload != "nop" else "tdes", CPU_SAMPLE[a.workload], threads)
         cpu = {"value": rate, "unit": "tasks/s", "cores": threads, "kind": "oracle",
                "sample": f"{what}, {dt:.1f} s wall on {threads} threads"}
 
     if d.rank != 0:
         return
     line = {"metric": BASE["metric"], "value": value, "unit": "tasks/s", "n_gpus": d.world, "steps": a.steps,
-            "warmup": a.warmup, "ms_per_step": 1e3 * total / a.steps, "higher_is_better": True, "scaling": "weak",
+            "warmup": a.warmup, "ms_per_step": 1e3 * total / a.steps, "higher_is_better": True,
+            "scaling": "strong" if a.workload in STRONG else "weak",
             "vs_baseline": None,
             "dtype": DTYPE[a.workload],
             "data": "synthetic (seeded splitmix64 inputs, SURVEY §8(c) recipe)",
@@ -384,7 +508,7 @@ def main():
     line.update(out)
     if "naive" in out:
         line["speedup_vs_naive"] = (value / d.world) / out["naive"]["tasks_per_s"]
-    line["roofline"] = roofline(a.workload, n, dev_avg_ms, clk, peaks)
+    line["roofline"] = roofline(a.workload, n, dev_avg_ms, clk, peaks, w)
     line["cpu_baseline"] = cpu
     if e2e:
         line["e2e"] = e2e
@@ -393,29 +517,49 @@ def main():
     print(json.dumps(line), flush=True)
 
 
-def roofline(workload, n, dev_ms, clk, peaks):
+def work_totals(w):
+    """Algorithmic work of one step of workload w, summed over its tasks by
+    body (DEMAND; 3DES from each task's block count)."""
+    from paper_conf_ppopp_yehsser17_b200 import tasks as T
+    tot = {"fma": 0.0, "lds": 0.0, "hbm": 0.0}
+    func = w.shapes[:, 4]
+    for fid, name in T.NAMES.items():
+        m = func == fid
+        cnt = int(m.sum())
+        if cnt == 0:
+            continue
+        if name == "tdes":
+            nblk = w.args[m][:, 24:28].copy().view(np.uint32).astype(np.float64).sum()
+            tot["lds"] += nblk * TDES_LOOKUPS_PER_BLOCK
+            tot["hbm"] += nblk * 16
+        elif name in DEMAND:
+            for r, v in DEMAND[name].items():
+                tot[r] += cnt * v
+    return tot
+
+
+def roofline(workload, n, dev_ms, clk, peaks, w):
+    """The resource with the largest roofline time bounds the step; achieved =
+    its algorithmic units / the device time of one step."""
     sm_mhz = peaks.get("sm_max_mhz", 1965.0)
-    if workload == "tdes":
-        peak = 148 * LDS_LANES_PER_SM_CLK * sm_mhz * 1e6 / 1e9          # G lookups/s
-        achieved = n * TDES_LOOKUPS_PER_TASK / (dev_ms * 1e-3) / 1e9
-        return {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "G S-box lookups/s (LDS lanes)",
-                "frac": achieved / peak, "traffic": None,
-                "per_unit": f"{TDES_LOOKUPS_PER_TASK} lookups/task; peak = 148 SM x 32 LDS lanes/clk x "
-                            f"{sm_mhz:.0f} MHz (MEASURED_PEAKS sm_max_mhz)"}
-    if workload in ("mm", "mix"):
-        per = {"mm": 12288, "mix": None}[workload]
-        hbm = peaks.get("hbm_gbs", 6549.4)
-        if per is None:
-            return {"bound": "hbm", "achieved": None, "peak": hbm, "unit": "GB/s", "frac": None, "traffic": None}
-        achieved = n * per / (dev_ms * 1e-3) / 1e9
-        return {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s", "frac": achieved / hbm,
-                "traffic": None, "per_unit": f"{per} B/task (A, B in, C out)"}
-    if workload == "mb":
-        peak = 148 * 128 * sm_mhz * 1e6 / 1e12
-        achieved = 199370695 * 8 / (dev_ms * 1e-3) / 1e12
-        return {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "T fp32 lane-op/s", "frac": achieved / peak,
-                "traffic": None, "per_unit": "8 fp32 ops per iteration, 199,370,695 iterations"}
-    return {"bound": "alu", "achieved": None, "peak": None, "unit": None, "frac": None, "traffic": None}
+    tot = work_totals(w)
+    peak = {"fma": 148 * 128 * sm_mhz * 1e6, "lds": 148 * LDS_LANES_PER_SM_CLK * sm_mhz * 1e6,
+            "hbm": peaks.get("hbm_gbs", 6544.0) * 1e9}
+    t_roof = {r: tot[r] / peak[r] for r in tot}
+    r = max(t_roof, key=t_roof.get)
+    if tot[r] == 0:
+        return {"bound": "alu", "achieved": None, "peak": None, "unit": None, "frac": None, "traffic": None,
+                "per_unit": "NOP tasks: no algorithmic work (runtime ceiling)"}
+    scale, unit, bound = {"fma": (1e12, "T fp32 lane-op/s", "alu"), "lds": (1e9, "G S-box lookups/s (LDS lanes)", "alu"),
+                          "hbm": (1e9, "GB/s", "hbm")}[r]
+    achieved = tot[r] / (dev_ms * 1e-3) / scale
+    pk = peak[r] / scale
+    return {"bound": bound, "resource": r, "achieved": achieved, "peak": pk, "unit": unit, "frac": achieved / pk,
+            "traffic": None, "roofline_us": {k: v * 1e6 for k, v in t_roof.items()},
+            "per_unit": {"tdes": f"{TDES_LOOKUPS_PER_BLOCK} lookups and 16 B per 8-byte block",
+                         **{k: v for k, v in DEMAND.items()}},
+            "peak_from": f"fma: 148 SM x 128 lanes x {sm_mhz:.0f} MHz; lds: 148 x 32 lanes x {sm_mhz:.0f} MHz; "
+                         f"hbm: MEASURED_PEAKS hbm_gbs"}
 
 
 def e2e_run(p, w, steps, torch):

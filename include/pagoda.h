@@ -207,6 +207,18 @@ int pagoda_tdes_tables(const uint8_t key24[24], void* dst);
 int pagoda_naive_run(int device, int n, const int32_t* shapes, const void* args_base, size_t args_stride,
                      size_t args_bytes, int n_streams, int64_t* elapsed_ns);
 
+/* Static-fusion baseline (NEXT-2; "static task fusion combines
+ * multiple tasks into a monolithic large task"): ONE kernel launch of n thread
+ * blocks of threads_per_task threads (multiple of 32, the paper uses 256);
+ * block i runs task i's body with its shared-memory request (the launch
+ * reserves the largest).  Every task must have n_threadblocks == 1.  The task
+ * table (func id, shmem, args) is copied to the device inside the timed
+ * region.  elapsed_ns (nullable): host time from that copy to completion;
+ * kernel_ms (nullable): CUDA-event time of the kernel alone.
+ * Returns 0, -EINVAL, -ENOMEM, -EIO. */
+int pagoda_fused_run(int device, int n, const int32_t* shapes, const void* args_base, size_t args_stride,
+                     size_t args_bytes, int threads_per_task, int64_t* elapsed_ns, float* kernel_ms);
+
 /* ---- multi-GPU pool: one context per GPU, least-loaded picker */
 typedef struct pagoda_pool pagoda_pool;
 /* Start one context per device in devices[0..n_dev) with cfg (device field ignored). */

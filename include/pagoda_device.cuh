@@ -182,6 +182,35 @@ struct NativeEnv {
     uint32_t smem_bytes;
 };
 
+/* ---------------------------------------------------------------- FusedEnv
+ * For the static-fusion baseline: all tasks fused into one
+ * monolithic kernel, one thread block of a fixed size per (single-TB) task. */
+struct FusedEnv {
+    __device__ __forceinline__ int getTid() const { return (int)threadIdx.x; }
+    __device__ __forceinline__ int getBlockIdx() const { return 0; }
+    __device__ __forceinline__ int getBlockTid() const { return (int)threadIdx.x; }
+    __device__ __forceinline__ int getBlockDim() const { return (int)blockDim.x; }
+    __device__ __forceinline__ int getBlockWarps() const { return (int)(blockDim.x >> 5); }
+    __device__ __forceinline__ int getNumBlocks() const { return 1; }
+    __device__ __forceinline__ char* getSMPtr() const
+    {
+        extern __shared__ __align__(1024) char native_smem[];
+        return native_smem;
+    }
+    __device__ __forceinline__ uint32_t getSMBytes() const { return smem_bytes; }
+    __device__ __forceinline__ uint32_t getResidentTdes() const { return 0; }
+    __device__ __forceinline__ bool canSync() const { return true; }
+    __device__ __forceinline__ void syncBlock() const { __syncthreads(); }
+    __device__ __forceinline__ void stage(void* smem_dst, const void* gsrc, uint32_t bytes) const
+    {
+        const int4* s = reinterpret_cast<const int4*>(gsrc);
+        int4* d = reinterpret_cast<int4*>(smem_dst);
+        for (uint32_t i = lane_id(); i < bytes / 16u; i += 32u) d[i] = s[i];
+        __syncwarp();
+    }
+    uint32_t smem_bytes;
+};
+
 } // namespace pagoda
 
 /* ---------------------------------------------------------------- paper API

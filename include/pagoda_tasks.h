@@ -30,7 +30,9 @@ enum pagoda_func_id {
     PAGODA_FB   = 19,  /* FilterBank, one channel of 2048 */
     PAGODA_BF   = 20,  /* BeamFormer, 4 ch x 512 complex */
     PAGODA_CONV = 21,  /* separable 17-tap convolution, 128x128 */
-    PAGODA_DCT  = 22   /* 8x8 DCT-II over 128x128 */
+    PAGODA_DCT  = 22,  /* 8x8 DCT-II over 128x128 */
+    /* variants */
+    PAGODA_MM_TC = 23  /* the MM task on the tensor cores: 3xTF32 mma.sync (args: pagoda_mm_args) */
 };
 
 typedef struct { uint32_t* out; uint32_t* cnt; uint32_t base; uint32_t tag; } pagoda_mark_args;

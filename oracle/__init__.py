@@ -26,7 +26,7 @@ LIB = os.path.join(HERE, "liboracle.so")
 CFLAGS = ["-O2", "-std=c11", "-Wall", "-ffp-contract=off", "-fno-fast-math", "-fPIC", "-shared"]
 
 # func ids — the oracle's own numbering (oracle.h)
-NOP, MARK, TID, MB, TDES, MM, FB, BF, CONV, DCT = 0, 1, 2, 16, 17, 18, 19, 20, 21, 22
+NOP, MARK, TID, MB, TDES, MM, FB, BF, CONV, DCT, MM_TC = 0, 1, 2, 16, 17, 18, 19, 20, 21, 22, 23
 
 _lock = threading.Lock()
 _lib = None
@@ -56,6 +56,7 @@ def lib():
             L.orc_des_block.restype = C.c_uint64
             L.orc_tdes_ecb.argtypes = [P, P, SZ, P, I]
             L.orc_mm32.argtypes = [P, P, P]
+            L.orc_mm32_f64.argtypes = [P, P, P]
             L.orc_filterbank.argtypes = [P, P, P, P]
             L.orc_beamformer.argtypes = [P, P, P, P]
             L.orc_conv.argtypes = [P, P, P, P]
@@ -111,6 +112,14 @@ def mm32(A, B) -> np.ndarray:
     A = np.ascontiguousarray(A, np.float32); B = np.ascontiguousarray(B, np.float32)
     Cm = np.zeros((32, 32), np.float32)
     lib().orc_mm32(_p(A), _p(B), _p(Cm))
+    return Cm
+
+
+def mm32_exact(A, B) -> np.ndarray:
+    """C = A B accumulated in fp64, rounded once (the tensor-core MM variant's definition)."""
+    A = np.ascontiguousarray(A, np.float32); B = np.ascontiguousarray(B, np.float32)
+    Cm = np.zeros((32, 32), np.float32)
+    lib().orc_mm32_f64(_p(A), _p(B), _p(Cm))
     return Cm
 
 

@@ -191,6 +191,20 @@ void orc_mm32(const float* A, const float* B, float* C)
         }
 }
 
+/* MM on the tensor cores: the same product C = A B,
+ * whose summation order the hardware picks; the definition is the exact
+ * product, here accumulated in fp64 (each fp32 x fp32 product is exact in
+ * fp64) and rounded once to fp32.  Parity: |g - o| <= 1e-5 sum_k |a_ik b_kj|. */
+void orc_mm32_f64(const float* A, const float* B, float* C)
+{
+    for (int i = 0; i < 32; i++)
+        for (int j = 0; j < 32; j++) {
+            double acc = 0.0;
+            for (int k = 0; k < 32; k++) acc += (double)A[i * 32 + k] * (double)B[k * 32 + j];
+            C[i * 32 + j] = (float)acc;
+        }
+}
+
 /* ======================================================================
  * FB — FilterBank, Fig. 1c made precise (§8(c) FB): one channel,
  * N_sim=2048, N_col=32, N_samp=8.  Causal convolution (guard read as >= 0),
@@ -330,7 +344,7 @@ static int known_func(int f)
 {
     switch (f) {
     case ORC_NOP: case ORC_MARK: case ORC_TID: case ORC_MB: case ORC_TDES: case ORC_MM:
-    case ORC_FB: case ORC_BF: case ORC_CONV: case ORC_DCT: return 1;
+    case ORC_FB: case ORC_BF: case ORC_CONV: case ORC_DCT: case ORC_MM_TC: return 1;
     default: return 0;
     }
 }
@@ -343,7 +357,7 @@ static size_t args_size(int f)
     case ORC_TID: return sizeof(orc_tid_args);
     case ORC_MB: return sizeof(orc_mb_args);
     case ORC_TDES: return sizeof(orc_tdes_args);
-    case ORC_MM: return sizeof(orc_mm_args);
+    case ORC_MM: case ORC_MM_TC: return sizeof(orc_mm_args);
     case ORC_FB: return sizeof(orc_fb_args);
     case ORC_BF: return sizeof(orc_bf_args);
     case ORC_CONV: return sizeof(orc_conv_args);
@@ -401,6 +415,11 @@ int64_t orc_taskSpawn(orc_ctx* c, int threads, int n_tb, int shmem_bytes, int sy
     case ORC_MM: {
         const orc_mm_args* a = (const orc_mm_args*)args;
         orc_mm32(a->A, a->B, a->C);
+        break;
+    }
+    case ORC_MM_TC: {
+        const orc_mm_args* a = (const orc_mm_args*)args;
+        orc_mm32_f64(a->A, a->B, a->C);
         break;
     }
     case ORC_FB: {

@@ -29,7 +29,7 @@ extern "C" {
 enum {
     ORC_NOP = 0, ORC_MARK = 1, ORC_TID = 2,
     ORC_MB = 16, ORC_TDES = 17, ORC_MM = 18, ORC_FB = 19, ORC_BF = 20,
-    ORC_CONV = 21, ORC_DCT = 22
+    ORC_CONV = 21, ORC_DCT = 22, ORC_MM_TC = 23
 };
 
 /* ---- per-body argument blocks (host pointers; each <= 40 bytes) */
@@ -49,6 +49,7 @@ void orc_des_key_schedule(const uint8_t key8[8], uint64_t subkeys[16]);
 uint64_t orc_des_block(uint64_t block, const uint64_t subkeys[16], int decrypt);
 void orc_tdes_ecb(const uint8_t* in, uint8_t* out, size_t nbytes, const uint8_t key24[24], int decrypt);
 void orc_mm32(const float* A, const float* B, float* C);
+void orc_mm32_f64(const float* A, const float* B, float* C);   /* exact product, one rounding (NEXT-4) */
 void orc_filterbank(const float* r, const float* H, const float* F, float* y);
 void orc_beamformer(const float* x, const float* h, const float* w, float* out);
 void orc_conv(const float* img, const float* krow, const float* kcol, float* out);

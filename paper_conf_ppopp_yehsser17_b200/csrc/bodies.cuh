@@ -354,6 +354,74 @@ __device__ void body_mm(const Env& e, const pagoda_mm_args& a)
     }
 }
 
+/* ------------------------------------------------------------- MM, tensor cores
+ * NEXT-4: the same C = A B (32x32x32 fp32) on the tensor cores
+ * as 3xTF32: x = hi + lo with hi = tf32(x) and lo = tf32(x - hi), and
+ * C += lo_A hi_B + hi_A lo_B + hi_A hi_B (the small terms first; lo_A lo_B is
+ * below fp32 resolution), with mma.sync.m16n8k8 (fp32 accumulate).  A task is
+ * 2 x 4 tiles of 16x8; warp w of the task takes tiles w, w + W, ...  The
+ * products are summed in the tensor core's order, not the fma chain's, so
+ * parity is |g - o| <= 1e-5 sum_k |a_ik b_kj|.
+ * tcgen05 needs M >= 64 and a TMEM allocation per CTA: a 32x32 task is below
+ * both. */
+__device__ __forceinline__ void tf32_split(float x, uint32_t& hi, uint32_t& lo)
+{
+    asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(hi) : "f"(x));
+    const float r = __fsub_rn(x, __uint_as_float(hi));
+    asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(lo) : "f"(r));
+}
+
+__device__ __forceinline__ void mma_tf32(float (&c)[4], const uint32_t (&a)[4], uint32_t b0, uint32_t b1)
+{
+    asm volatile(
+        "mma.sync.aligned.m16n8k8.row.col.f32.tf32.tf32.f32 {%0, %1, %2, %3}, {%4, %5, %6, %7}, {%8, %9}, "
+        "{%0, %1, %2, %3};"
+        : "+f"(c[0]), "+f"(c[1]), "+f"(c[2]), "+f"(c[3])
+        : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b0), "r"(b1));
+}
+
+template <class Env>
+__device__ void body_mm_tc(const Env& e, const pagoda_mm_args& a)
+{
+    const float* A = a.A;
+    const float* B = a.B;
+    if (e.getSMBytes() >= 8192 && e.canSync()) {   /* stage A, B with TMA bulk copies, as body_mm */
+        float* s = reinterpret_cast<float*>(e.getSMPtr());
+        const int w = e.getBlockTid() >> 5;
+        if (e.getBlockWarps() >= 2) {
+            if (w == 0) e.stage(s, A, 4096);
+            else if (w == 1) e.stage(s + 1024, B, 4096);
+        } else {
+            e.stage(s, A, 4096);
+            e.stage(s + 1024, B, 4096);
+        }
+        e.syncBlock();
+        A = s;
+        B = s + 1024;
+    }
+    const int lane = (int)lane_id(), g = lane >> 2, t = lane & 3;
+    const int nw = total_threads(e) >> 5;
+    for (int tile = e.getTid() >> 5; tile < 8; tile += nw) {
+        const int m0 = (tile >> 2) * 16, n0 = (tile & 3) * 8;
+        float c[4] = {0.0f, 0.0f, 0.0f, 0.0f};
+#pragma unroll 1
+        for (int k0 = 0; k0 < 32; k0 += 8) {
+            uint32_t ah[4], al[4], bh0, bl0, bh1, bl1;
+            tf32_split(A[(m0 + g) * 32 + k0 + t], ah[0], al[0]);
+            tf32_split(A[(m0 + g + 8) * 32 + k0 + t], ah[1], al[1]);
+            tf32_split(A[(m0 + g) * 32 + k0 + t + 4], ah[2], al[2]);
+            tf32_split(A[(m0 + g + 8) * 32 + k0 + t + 4], ah[3], al[3]);
+            tf32_split(B[(k0 + t) * 32 + n0 + g], bh0, bl0);
+            tf32_split(B[(k0 + t + 4) * 32 + n0 + g], bh1, bl1);
+            mma_tf32(c, al, bh0, bh1);
+            mma_tf32(c, ah, bl0, bl1);
+            mma_tf32(c, ah, bh0, bh1);
+        }
+        *reinterpret_cast<float2*>(a.C + (m0 + g) * 32 + n0 + 2 * t) = make_float2(c[0], c[1]);
+        *reinterpret_cast<float2*>(a.C + (m0 + g + 8) * 32 + n0 + 2 * t) = make_float2(c[2], c[3]);
+    }
+}
+
 /* ------------------------------------------------------------- FB
  * Fig. 1c: VH = H (*) r, VD[m] = VH[8m],
  * VU = up-sample of VD, y = F (*) VU; causal, fma chains k ascending.
@@ -572,13 +640,14 @@ __device__ __forceinline__ bool run_body(int func_id, const Env& e, const void* 
     case PAGODA_BF: body_bf(e, *static_cast<const pagoda_bf_args*>(args)); return true;
     case PAGODA_CONV: body_conv(e, *static_cast<const pagoda_conv_args*>(args)); return true;
     case PAGODA_DCT: body_dct(e, *static_cast<const pagoda_dct_args*>(args)); return true;
+    case PAGODA_MM_TC: body_mm_tc(e, *static_cast<const pagoda_mm_args*>(args)); return true;
     default: return false;
     }
 }
 
 __host__ __device__ inline bool known_func(int f)
 {
-    return (f >= PAGODA_NOP && f <= PAGODA_GATE) || (f >= PAGODA_MB && f <= PAGODA_DCT);
+    return (f >= PAGODA_NOP && f <= PAGODA_GATE) || (f >= PAGODA_MB && f <= PAGODA_MM_TC);
 }
 
 } // namespace pagoda

@@ -171,3 +171,72 @@ def mix_schedule(n_tasks: int, seed: int = SEED ^ TAG["mix"]):
     thr = np.array(MIX_THREADS)[(z[:, 1] % np.uint64(len(MIX_THREADS))).astype(np.int64)]
     shm = np.array(MIX_SHMEM_KB)[(z[:, 2] % np.uint64(len(MIX_SHMEM_KB))).astype(np.int64)] * 1024
     return kinds.astype(np.int32), thr.astype(np.int32), shm.astype(np.int32)
+
+
+# ---------------------------------------------------------------- NEXT-1: irregular 3DES packets
+TDES_VAR_MIN, TDES_VAR_MAX = 2048, 65536   # NetBench packet sizes 2K-64K (Table 3)
+
+
+def tdes_var_sizes(n_tasks: int, first: int = 0) -> np.ndarray:
+    """Packet bytes per task, log-uniform in [2 KiB, 64 KiB], whole 8-byte
+    blocks: blocks = floor(256 * 32^u), u = the task's draw mapped to [0, 1)."""
+    z = splitmix64(np.arange(first, first + n_tasks), 1, SEED ^ TAG["tdes"] ^ 0x5A5A)[:, 0]
+    u = (z >> np.uint64(11)).astype(np.float64) * 2.0 ** -53
+    blocks = np.floor((TDES_VAR_MIN // 8) * (TDES_VAR_MAX / TDES_VAR_MIN) ** u).astype(np.int64)
+    return (np.clip(blocks, TDES_VAR_MIN // 8, TDES_VAR_MAX // 8) * 8).astype(np.int64)
+
+
+def splitmix64_ragged(task_of: np.ndarray, k_of: np.ndarray, seed: int) -> np.ndarray:
+    """Output number k_of[e] (0-based) of the stream of task task_of[e], per
+    element (the same numbers splitmix64() gives, for ragged per-task counts)."""
+    t = np.asarray(task_of, np.uint64)
+    k = np.asarray(k_of, np.uint64) + np.uint64(1)
+    with np.errstate(over="ignore"):
+        z = (np.uint64(seed) ^ (t * _TASK_MUL)) + k * _GOLDEN
+        z = (z ^ (z >> np.uint64(30))) * _M1
+        z = (z ^ (z >> np.uint64(27))) * _M2
+        z = z ^ (z >> np.uint64(31))
+    return z
+
+
+def tdes_var_packets(sizes: np.ndarray, first: int = 0):
+    """Flat uint8 payload of the irregular 3DES workload and the byte offset of
+    every packet: packet k is the first sizes[k] bytes of task (first+k)'s
+    3DES stream (so equal-size packets equal tdes_packets()' bytes); packet 0
+    of task 0 starts with the SP 800-67 plaintext."""
+    sizes = np.asarray(sizes, np.int64)
+    off = np.zeros(len(sizes) + 1, np.int64)
+    np.cumsum(sizes, out=off[1:])
+    nblk = sizes // 8
+    task = np.repeat(np.arange(first, first + len(sizes), dtype=np.int64), nblk)
+    k = np.arange(int(nblk.sum()), dtype=np.int64) - np.repeat(off[:-1] // 8, nblk)
+    z = splitmix64_ragged(task, k, SEED ^ TAG["tdes"])
+    flat = z.astype("<u8").view(np.uint8).copy()
+    if first == 0 and len(sizes) > 0:
+        flat[:24] = np.frombuffer(TDES_KAT_PLAIN, dtype=np.uint8)
+    return flat, off
+
+
+# ---------------------------------------------------------------- NEXT-1: MPE, config 5
+MPE_KINDS = ("mb", "tdes", "fb", "mm")     # P:1111-1123: 8K tasks of each, 32K in total
+C5_KINDS = ("mb", "tdes", "mm", "fb", "bf", "conv", "dct")
+
+
+def mpe_schedule(n_tasks: int, seed: int = SEED ^ TAG["mix"] ^ 0x3E3E) -> np.ndarray:
+    """Kind index (into MPE_KINDS) per task: n/4 of each in a seeded order."""
+    z = splitmix64(np.arange(n_tasks), 1, seed)[:, 0]
+    kinds = np.arange(n_tasks) % len(MPE_KINDS)
+    return kinds[np.argsort(z, kind="stable")].astype(np.int32)
+
+
+def c5_schedule(n_tasks: int, seed: int = SEED ^ TAG["mix"] ^ 0xC5C5):
+    """Config 5: kind of task i = a seeded uniform draw over
+    the 7 bodies (C5_KINDS); threads / shmem requests for FB, BF, CONV, DCT as
+    in config 4 (uniform in MIX_THREADS / MIX_SHMEM_KB).  Returns (kind[n],
+    threads[n], shmem[n]); the threads / shmem of MB, 3DES, MM are their
+    configs' fixed shapes and are filled in by the workload."""
+    z = splitmix64(np.arange(n_tasks), 3, seed)
+    kinds = (z[:, 0] % np.uint64(len(C5_KINDS))).astype(np.int32)
+    thr = np.array(MIX_THREADS)[(z[:, 1] % np.uint64(len(MIX_THREADS))).astype(np.int64)]
+    shm = np.array(MIX_SHMEM_KB)[(z[:, 2] % np.uint64(len(MIX_SHMEM_KB))).astype(np.int64)] * 1024
+    return kinds, thr.astype(np.int32), shm.astype(np.int32)

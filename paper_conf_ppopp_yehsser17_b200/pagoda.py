@@ -74,6 +74,7 @@ def lib() -> C.CDLL:
         L.pagoda_trace_read_exec.restype = I64
         L.pagoda_tdes_tables.argtypes = [P, P]
         L.pagoda_naive_run.argtypes = [I, I, P, P, SZ, SZ, I, C.POINTER(I64)]
+        L.pagoda_fused_run.argtypes = [I, I, P, P, SZ, SZ, I, C.POINTER(I64), C.POINTER(C.c_float)]
         L.pagoda_pool_init.argtypes = [I, P, C.POINTER(pagoda_config), C.POINTER(P)]
         L.pagoda_pool_pick.argtypes = [P, I]
         L.pagoda_pool_ctx.argtypes = [P, I]
@@ -270,6 +271,17 @@ def naive_run(device: int, shapes: np.ndarray, args: np.ndarray, n_streams: int 
     _check(lib().pagoda_naive_run(device, len(shapes), _ptr(shapes), _ptr(args), args.shape[1], args.shape[1],
                                   n_streams, C.byref(ns)), "pagoda_naive_run")
     return ns.value
+
+
+def fused_run(device: int, shapes: np.ndarray, args: np.ndarray, threads_per_task: int = 256):
+    """Static fusion: all tasks in one kernel launch; returns (elapsed host ns
+    incl. the task-table copy, kernel-only ms)."""
+    shapes = np.ascontiguousarray(shapes, np.int32)
+    args = np.ascontiguousarray(args, np.uint8)
+    ns, ms = C.c_int64(0), C.c_float(0)
+    _check(lib().pagoda_fused_run(device, len(shapes), _ptr(shapes), _ptr(args), args.shape[1], args.shape[1],
+                                  threads_per_task, C.byref(ns), C.byref(ms)), "pagoda_fused_run")
+    return ns.value, ms.value
 
 
 def pick_least_loaded(loads) -> int:

@@ -111,6 +111,34 @@ def test_mm_config3_full_size():
     _mm_check(w, out, list(rng.choice(65536, 256, replace=False)) + [0, 65535])
 
 
+# ---------------------------------------------------------------- MM on the tensor cores (NEXT-4, 3xTF32)
+def _mm_tc_check(w, out, ks):
+    for k in ks:
+        a, b = w.host["A"][k].astype(np.float64), w.host["B"][k].astype(np.float64)
+        ref = oracle.mm32_exact(w.host["A"][k], w.host["B"][k]).astype(np.float64)
+        bound = TOL * (np.abs(a) @ np.abs(b))      # normwise: the summation order is the hardware's
+        assert (np.abs(out[k].astype(np.float64) - ref) <= bound).all(), k
+
+
+@pytest.mark.parametrize("shmem,threads", [(8192, 256), (0, 256), (8192, 64), (8192, 32), (0, 96)])
+def test_mm_tc_small(shmem, threads):
+    from paper_conf_ppopp_yehsser17_b200 import tasks as T
+    w = W.matmul(300, shmem=shmem, threads=threads, func=T.MM_TC)
+    _mm_tc_check(w, run(w)["C"], range(300))
+
+
+def test_mm_tc_integer_exact_and_full_size():
+    from paper_conf_ppopp_yehsser17_b200 import tasks as T
+    w = W.matmul(64, func=T.MM_TC, integer=True)    # integer inputs: every partial sum exact in fp32
+    out = run(w)["C"]
+    for k in range(64):
+        assert np.array_equal(out[k], oracle.mm32_exact(w.host["A"][k], w.host["B"][k])), k
+    w = W.matmul(65536, func=T.MM_TC)
+    out = run(w)["C"]
+    rng = np.random.default_rng(5)
+    _mm_tc_check(w, out, list(rng.choice(65536, 256, replace=False)) + [0, 65535])
+
+
 # ---------------------------------------------------------------- mix (config 4)
 def _mix_check(w, out, frac=1.0, seed=0):
     rng = np.random.default_rng(seed)
@@ -161,3 +189,24 @@ def test_naive_baseline_parity():
     out = w.outputs()["out"]
     for k in range(16):
         assert np.array_equal(out[k], _tdes_ref(w.host["packets"][k]))
+
+
+# ---------------------------------------------------------------- static fusion (NEXT-2) runs the same bodies
+def test_static_fusion_parity():
+    from paper_conf_ppopp_yehsser17_b200.pagoda import PagodaError, fused_run
+    w = W.mix(120)
+    ns, ms = fused_run(0, w.shapes, w.args, 256)
+    assert ns > 0 and ms > 0
+    _mix_check(w, w.outputs())
+    w = W.tdes(40)
+    fused_run(0, w.shapes, w.args, 64)
+    out = w.outputs()["out"]
+    for k in range(40):
+        assert np.array_equal(out[k], _tdes_ref(w.host["packets"][k]))
+    w = W.matmul(50)
+    fused_run(0, w.shapes, w.args, 256)
+    _mm_check(w, w.outputs()["C"], range(50))
+    bad = w.shapes.copy()
+    bad[3, 1] = 2   # multi-block tasks cannot be fused one block per task
+    with pytest.raises(PagodaError):
+        fused_run(0, bad, w.args, 256)

@@ -147,6 +147,26 @@ def test_mm_within_error_bound(orc):
     assert not np.allclose(orc.mm32(A[0], B[0]), (A[0].astype(np.float64) @ B[0].T), atol=1e-3)
 
 
+def test_mm_exact_variant(orc):
+    """mm32_exact (NEXT-4's definition): integer inputs exact; random inputs
+    equal the exactly rounded product (exact rational sum via fractions,
+    rounded once to fp32; 32 products of 24-bit values fit a double
+    exactly, their sum may not); a transposed operand is caught."""
+    from fractions import Fraction
+    A, B = inputs.mm_inputs(3, integer=True)
+    for i in range(3):
+        ref = A[i].astype(np.int64) @ B[i].astype(np.int64)
+        assert np.array_equal(orc.mm32_exact(A[i], B[i]).astype(np.int64), ref)
+    A, B = inputs.mm_inputs(2)
+    got = orc.mm32_exact(A[0], B[0])
+    for i, j in [(0, 0), (3, 17), (31, 31), (12, 5), (20, 30)]:
+        exact = sum(Fraction(float(A[0][i, k])) * Fraction(float(B[0][k, j])) for k in range(32))
+        near = np.float32(float(exact))            # exact -> double -> fp32: one ulp of slack for double rounding
+        assert abs(float(got[i, j]) - float(exact)) <= abs(float(near) - float(exact)) + 1e-12, (i, j)
+    assert np.array_equal(orc.mm32_exact(A[1], np.eye(32, dtype=np.float32)), A[1])
+    assert not np.allclose(got, A[0].astype(np.float64) @ B[0].T, atol=1e-3)
+
+
 # ------------------------------------------------------------------ FB
 def _fb_fp64(r, H, F):
     r, H, F = (np.asarray(v, np.float64) for v in (r, H, F))
@@ -297,3 +317,40 @@ def test_occupancy_paper_examples(orc):
     # one 256-thread task on 24 SMMs = 0.52 %, 32 HyperQ tasks = 16.67 %
     assert round(orc.occupancy_pct(8, 24), 2) == 0.52
     assert round(orc.occupancy_pct(8 * 32, 24), 2) == 16.67
+
+
+# ---------------------------------------------------------------- NEXT-1 / config 5 input recipes (host logic)
+def test_tdes_var_sizes_log_uniform():
+    from paper_conf_ppopp_yehsser17_b200 import inputs as I
+    s = I.tdes_var_sizes(32768)
+    assert s.min() >= 2048 and s.max() <= 65536 and np.all(s % 8 == 0)
+    # log-uniform: log2(size/2048) is uniform on [0, 5): each octave holds ~1/5 of the packets
+    oct_ = np.floor(np.log2(s / 2048)).astype(int)
+    frac = np.bincount(oct_, minlength=5)[:5] / len(s)
+    assert np.all(np.abs(frac - 0.2) < 0.02), frac
+    assert abs(s.mean() - (65536 - 2048) / np.log(32)) / s.mean() < 0.03   # E[size] of log-uniform
+
+
+def test_tdes_var_packets_are_the_tdes_streams():
+    """Equal sizes reproduce tdes_packets(); a ragged packet is the prefix of
+    its task's stream; the oracle encrypts it like the library does."""
+    from paper_conf_ppopp_yehsser17_b200 import inputs as I
+    flat, off = I.tdes_var_packets(np.array([4096, 2048, 16], np.int64))
+    full = I.tdes_packets(3, 4096)
+    assert np.array_equal(flat[off[0]:off[1]], full[0])
+    assert np.array_equal(flat[off[1]:off[2]], full[1, :2048])
+    assert np.array_equal(flat[off[2]:off[3]], full[2, :16])
+
+
+def test_schedules_mpe_and_c5():
+    from paper_conf_ppopp_yehsser17_b200 import inputs as I
+    k = I.mpe_schedule(32768)
+    assert np.array_equal(np.bincount(k), [8192] * 4)           # 8K of each (P:1121-1123)
+    assert not np.array_equal(k[:8], np.arange(8) % 4)          # shuffled
+    kinds, thr, shm = I.c5_schedule(1_000_000)
+    c = np.bincount(kinds, minlength=7)
+    assert np.all(np.abs(c / 1e6 - 1 / 7) < 0.002), c           # seeded uniform draw over 7 bodies
+    assert set(np.unique(thr)) == set(I.MIX_THREADS)
+    assert set(np.unique(shm // 1024)) == set(I.MIX_SHMEM_KB)
+    k2 = I.c5_schedule(1000)[0]
+    assert np.array_equal(k2, kinds[:1000])                     # prefix-stable: shards agree with the whole
