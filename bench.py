@@ -399,6 +399,10 @@ def main():
                                 "how": "one launch of n blocks x 256 threads, block i runs task i's body (task table "
                                        "H2D inside the timed region); kernel_ only: CUDA events around the kernel"}
 
+    pp = None
+    if not a.quick:   # PCIe round-trip floor of any spawn -> done handshake
+        pp = PG.pingpong(dev, 2000) / 1e3
+
     p = PG.Pagoda(device=dev, **ctx_config(a, PG))
 
     def step():
@@ -447,6 +451,8 @@ def main():
         assert p.start() == 0
         iso = p.latency_loop(2000, 128, 1, 0, False, 0) / 1e3
         lat["isolated_nop128_us"] = {"p50": float(np.percentile(iso, 50)), "p99": float(np.percentile(iso, 99))}
+        lat["pingpong_floor_us"] = {"p50": float(np.percentile(pp, 50)), "p99": float(np.percentile(pp, 99))}
+        lat["isolated_nop128_over_floor"] = lat["isolated_nop128_us"]["p50"] / lat["pingpong_floor_us"]["p50"]
         s0 = w.shapes[0]
         iso2 = p.latency_loop(300, int(s0[0]), int(s0[1]), int(s0[2]), bool(s0[3]), int(s0[4]), w.args[0]) / 1e3
         lat["isolated_task_us"] = {"p50": float(np.percentile(iso2, 50)), "p99": float(np.percentile(iso2, 99))}

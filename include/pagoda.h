@@ -151,6 +151,13 @@ int64_t pagoda_run_timed(pagoda_ctx* ctx, int n, const int32_t* shapes, const vo
 int pagoda_latency_loop(pagoda_ctx* ctx, int n, int threads, int n_threadblocks, int shmem_bytes,
                         int sync_flag, int func_id, const void* args, size_t args_bytes, int64_t* lat_ns);
 
+/* PCIe round-trip floor: one GPU warp echoes a pinned-host
+ * counter n times (host writes i, the GPU polls with ld.acquire.sys and writes
+ * back i, the host polls); rtt_ns[i] = host write -> echo seen.  Must run
+ * while no MasterKernel holds the device.  Returns 0, -EINVAL, -ENODEV,
+ * -ENOMEM, -EIO, -ETIMEDOUT. */
+int pagoda_pingpong(int device, int n, int64_t* rtt_ns);
+
 /* Runtime counters accumulated on the device since the context was created
  * (read while stopped or running; ns are %globaltimer nanoseconds). */
 enum {

@@ -2,8 +2,10 @@
  * measure.cu — measurement helpers over the public API (pagoda.h
  * "Measurement"): a timed spawn run that records per-task spawn and done
  * times (the metric's p50 spawn-to-done latency under load), and the isolated
- * closed-loop latency of one task at a time.  Host clock: CLOCK_MONOTONIC.
+ * closed-loop latency of one task at a time, and the PCIe ping-pong that
+ * floors both (SURVEY §8(d) "Latency").  Host clock: CLOCK_MONOTONIC.
  */
+#include <cuda_runtime.h>
 #include <errno.h>
 #include <stdint.h>
 #include <string.h>
@@ -78,4 +80,58 @@ extern "C" int pagoda_latency_loop(pagoda_ctx* c, int n, int threads, int n_tb, 
         lat_ns[i] = mono_ns() - t0;
     }
     return 0;
+}
+
+/* ------------------------------------------------------------------ ping-pong floor
+ * One persistent warp echoes a pinned-host counter: the host writes ping = i,
+ * the GPU (ld.acquire.sys poll) answers pong = i, the host polls pong.  A
+ * round trip is the least any spawn -> done handshake over PCIe can cost. */
+__global__ void pingpong_kernel(volatile int64_t* ping, volatile int64_t* pong, int n)
+{
+    if (threadIdx.x != 0) return;
+    for (int64_t i = 1; i <= n; i++) {
+        int64_t v;
+        do {
+            asm volatile("ld.acquire.sys.global.s64 %0, [%1];" : "=l"(v) : "l"(ping) : "memory");
+        } while (v != i && v >= 0);
+        if (v < 0) return;   /* the host gave up */
+        asm volatile("st.release.sys.global.s64 [%0], %1;" ::"l"(pong), "l"(i) : "memory");
+    }
+}
+
+extern "C" int pagoda_pingpong(int device, int n, int64_t* rtt_ns)
+{
+    if (n < 1 || !rtt_ns) return -EINVAL;
+    if (cudaSetDevice(device) != cudaSuccess) return -ENODEV;
+    int64_t* h = nullptr;
+    if (cudaHostAlloc(&h, 256, cudaHostAllocMapped) != cudaSuccess) return -ENOMEM;
+    volatile int64_t* ping = h;
+    volatile int64_t* pong = h + 8;   /* separate 64 B lines */
+    *ping = 0;
+    *pong = 0;
+    int64_t *dping = nullptr, *dpong = nullptr;
+    cudaHostGetDevicePointer((void**)&dping, h, 0);
+    dpong = dping + 8;
+    cudaStream_t st;
+    cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking);
+    pingpong_kernel<<<1, 32, 0, st>>>(dping, dpong, n);
+    int rc = cudaGetLastError() == cudaSuccess ? 0 : -EIO;
+    for (int i = 1; i <= n && !rc; i++) {
+        const int64_t t0 = mono_ns();
+        __atomic_store_n(ping, (int64_t)i, __ATOMIC_RELEASE);
+        int64_t spins = 0;
+        while (__atomic_load_n(pong, __ATOMIC_ACQUIRE) != i) {
+            if (++spins > 200000000ll) {
+                rc = -ETIMEDOUT;
+                __atomic_store_n(ping, (int64_t)-1, __ATOMIC_RELEASE);   /* release the kernel */
+                break;
+            }
+            _mm_pause();
+        }
+        rtt_ns[i - 1] = mono_ns() - t0;
+    }
+    if (cudaStreamSynchronize(st) != cudaSuccess && !rc) rc = -EIO;
+    cudaStreamDestroy(st);
+    cudaFreeHost(h);
+    return rc;
 }

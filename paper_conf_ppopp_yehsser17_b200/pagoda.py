@@ -74,6 +74,7 @@ def lib() -> C.CDLL:
         L.pagoda_trace_read_exec.restype = I64
         L.pagoda_tdes_tables.argtypes = [P, P]
         L.pagoda_naive_run.argtypes = [I, I, P, P, SZ, SZ, I, C.POINTER(I64)]
+        L.pagoda_pingpong.argtypes = [I, I, P]
         L.pagoda_fused_run.argtypes = [I, I, P, P, SZ, SZ, I, C.POINTER(I64), C.POINTER(C.c_float)]
         L.pagoda_pool_init.argtypes = [I, P, C.POINTER(pagoda_config), C.POINTER(P)]
         L.pagoda_pool_pick.argtypes = [P, I]
@@ -282,6 +283,13 @@ def fused_run(device: int, shapes: np.ndarray, args: np.ndarray, threads_per_tas
     _check(lib().pagoda_fused_run(device, len(shapes), _ptr(shapes), _ptr(args), args.shape[1], args.shape[1],
                                   threads_per_task, C.byref(ns), C.byref(ms)), "pagoda_fused_run")
     return ns.value, ms.value
+
+
+def pingpong(device: int, n: int = 2000) -> np.ndarray:
+    """PCIe round-trip floor: n host -> GPU -> host echoes (ns each)."""
+    out = np.zeros(n, np.int64)
+    _check(lib().pagoda_pingpong(device, n, _ptr(out)), "pagoda_pingpong")
+    return out
 
 
 def pick_least_loaded(loads) -> int:

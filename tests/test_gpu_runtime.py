@@ -282,3 +282,14 @@ def test_session_starting_exactly_at_the_ring_wrap():
             assert p.start() == 0
             p.spawn_many(R, 128, 1, 0, False, T.NOP, None)
             assert p.stop() == 0
+
+
+def test_pingpong_floor():
+    """The PCIe round-trip floor: every echo returns, in
+    microseconds, and an isolated NOP task costs at least one round trip."""
+    from paper_conf_ppopp_yehsser17_b200.pagoda import pingpong
+    rtt = pingpong(0, 500)
+    assert (rtt > 0).all() and np.median(rtt) < 50_000
+    with Pagoda() as p:
+        lat = p.latency_loop(200, 128, 1, 0, False, T.NOP)
+    assert np.median(lat) >= 0.9 * np.median(rtt)
