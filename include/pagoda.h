@@ -82,10 +82,15 @@ int pagoda_shutdown(pagoda_ctx* ctx);
  * Non-blocking: returns once the entry is published (it blocks, with back-off,
  * only while the TaskTable ring or completion window is full, as the paper's
  * CPU does when no entry is free).
+ * A task whose thread blocks all fit one MTB (warps, shared memory, 15
+ * barrier IDs) runs inside one MTB.  A larger task (e.g. the
+ * "64K threads" of Fig. 8) is spread TB by TB over k MTB-sized
+ * TaskTable entries; it consumes k ids (the returned one is the first; ids
+ * stay strictly increasing but skip k - 1) and completes when its last TB does.
  * Returns the task id (>= 0, strictly increasing per context) or
- *   -EINVAL  threads < 1 or > 1024, n_threadblocks < 1, ceil(threads/32)*n_tb > worker
- *            warps per MTB (32; all warps of a task live in one MTB),
- *            n_tb * round_up(shmem, 512) > arena, sync with > 15 multi-warp TBs,
+ *   -EINVAL  threads < 1 or > 1024, n_threadblocks < 1 or (spread) > 65535,
+ *            ceil(threads/32) > worker warps per MTB (32), round_up(shmem, 512)
+ *            > arena (one TB must fit an MTB), k > ring_entries / 4,
  *            unknown func_id, args_bytes > 40 or args NULL with args_bytes > 0;
  *   -ESHUTDOWN after pagoda_shutdown began;  -EIO after a device fault. */
 pagoda_task_t pagoda_taskSpawn(pagoda_ctx* ctx, int threads, int n_threadblocks, int shmem_bytes,

@@ -37,7 +37,7 @@ struct WarpSlot {
     uint8_t  n_tb;        /* TBs in the task */
     uint8_t  bar_id;      /* named barrier (barId), 0 = none */
     uint8_t  tbslot;      /* per-MTB TB record */
-    uint16_t pad0;
+    uint16_t n_tb_all;    /* TBs of the whole task (> n_tb when it is spread over several MTBs) */
     uint64_t task_id;     /* host-visible id (for tracing) */
 };
 static_assert(sizeof(WarpSlot) == 32, "WarpSlot is 32 bytes");
@@ -48,7 +48,7 @@ enum : uint8_t { SLOT_TERMINATE = 0xFF, SLOT_SCHED = 0xFE /* take over the sched
  * laid out in csrc/mk_layout.cuh, which static_asserts them).  The task arena
  * follows the control block, or the resident tables when a context has them. */
 constexpr uint32_t kWarpTableOffset = 512;
-constexpr uint32_t kControlBytes = 5120;            /* arena offset without resident tables */
+constexpr uint32_t kControlBytes = 6144;            /* arena offset without resident tables */
 constexpr uint32_t kResidentOffset = 8192;          /* room reserved for the control block + resident tables */
 constexpr uint32_t kResidentTdesBytes = 8 * 64 * 32 * 4;   /* 3DES SP tables, one copy per lane */
 constexpr uint32_t kResidentTdesAddr = 8192;        /* shared-WINDOW address of the resident tables: a
@@ -77,7 +77,7 @@ __device__ __forceinline__ uint32_t smem_u32(const void* p)
  * Everything a body asks for is read from the executor warp's WarpTable slot in
  * shared memory when asked (no register holds it across the body). */
 constexpr uint32_t kStageBarOffset = 256;     /* per-warp TMA staging mbarriers (MtbShared.stage_bar) */
-constexpr uint32_t kStagePhaseOffset = 4900;  /* their parities, one u32 per warp (MtbShared.stage_ph) */
+constexpr uint32_t kStagePhaseOffset = 4824;  /* their parities, one u32 per warp (MtbShared.stage_ph) */
 
 struct TaskEnv {
     uint32_t* dev_error;    /* device error word */
@@ -101,7 +101,7 @@ struct TaskEnv {
     __device__ __forceinline__ int getBlockTid() const { return (int)s().warp_in_tb * 32 + (int)lane_id(); }
     __device__ __forceinline__ int getBlockDim() const { return s().threads_tb; }
     __device__ __forceinline__ int getBlockWarps() const { return s().warps_tb; }
-    __device__ __forceinline__ int getNumBlocks() const { return s().n_tb; }
+    __device__ __forceinline__ int getNumBlocks() const { return s().n_tb_all; }
     __device__ __forceinline__ char* getSMPtr() const { return reinterpret_cast<char*>(mk_smem()) + s().smem_off; }
     __device__ __forceinline__ uint32_t getSMBytes() const { return s().smem_bytes; }
     /* MTB-resident, lane-replicated 3DES SP tables (context flag PAGODA_RESIDENT_TDES) */

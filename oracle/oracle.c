@@ -328,10 +328,11 @@ struct orc_ctx {
 #define ORC_ARGS_MAX 40
 #define ORC_GRANULE 512   /* §5.1: the smallest allocation is 512 B */
 #define ORC_BAR_IDS 15    /* 16 named barriers, ID 0 kept for the MTB itself */
+#define ORC_MAX_SPREAD 16384   /* MTB entries of one task: a quarter of the default 65536-entry ring */
 
 int orc_init(int exec_warps_per_mtb, int arena_bytes, orc_ctx** out)
 {
-    if (!out || exec_warps_per_mtb < 1 || exec_warps_per_mtb > 31 || arena_bytes < 0) return -EINVAL;
+    if (!out || exec_warps_per_mtb < 1 || exec_warps_per_mtb > 32 || arena_bytes < 0) return -EINVAL;
     orc_ctx* c = (orc_ctx*)calloc(1, sizeof *c);
     if (!c) return -ENOMEM;
     c->exec_warps = exec_warps_per_mtb;
@@ -371,17 +372,27 @@ int64_t orc_taskSpawn(orc_ctx* c, int threads, int n_tb, int shmem_bytes, int sy
 {
     if (!c) return -EINVAL;
     if (c->shut) return -ESHUTDOWN;
-    if (threads < 1 || n_tb < 1 || shmem_bytes < 0) return -EINVAL;
+    if (threads < 1 || threads > 1024 || n_tb < 1 || shmem_bytes < 0) return -EINVAL;
+    /* Every thread block must fit one MTB.  The paper keeps all warps of a task in one MTB
+     * yet runs "64K threads" per task (Fig. 8); read: a task whose
+     * TBs do not fit one MTB is spread, TB by TB, over k = ceil(n_tb / cap) MTB entries, cap =
+     * the TBs one MTB hosts (warps, shared memory, 15 barrier IDs when it syncs), and it
+     * consumes k task ids, the first being its id (DESIGN.md "Readings" 6). */
     int warps_tb = (threads + 31) / 32;
-    if ((long)warps_tb * n_tb > c->exec_warps) return -EINVAL;
+    if (warps_tb > c->exec_warps) return -EINVAL;
     long gran_tb = (shmem_bytes + ORC_GRANULE - 1) / ORC_GRANULE;
-    if (gran_tb * n_tb * ORC_GRANULE > c->arena_bytes) return -EINVAL;
-    if (sync_flag && warps_tb > 1 && n_tb > ORC_BAR_IDS) return -EINVAL;
+    if (gran_tb * ORC_GRANULE > c->arena_bytes) return -EINVAL;
+    long cap = c->exec_warps / warps_tb;
+    if (gran_tb && c->arena_bytes / (gran_tb * ORC_GRANULE) < cap) cap = c->arena_bytes / (gran_tb * ORC_GRANULE);
+    if (sync_flag && warps_tb > 1 && cap > ORC_BAR_IDS) cap = ORC_BAR_IDS;
+    const long k = (n_tb + cap - 1) / cap;
+    if (k > 1 && (n_tb > 65535 || k > ORC_MAX_SPREAD)) return -EINVAL;
     if (!known_func(func_id)) return -EINVAL;
     if (args_bytes > ORC_ARGS_MAX || (args_bytes > 0 && !args)) return -EINVAL;
     if (args_bytes < args_size(func_id)) return -EINVAL;
 
-    int64_t id = c->next_id++;
+    int64_t id = c->next_id;
+    c->next_id += k;
     long total_threads_rounded = (long)warps_tb * 32 * n_tb;
     switch (func_id) {
     case ORC_NOP: break;

@@ -223,34 +223,14 @@ enum { kTdesResident = 0, kTdesShared = 1, kTdesGlobal = 2 };
  * one PRMT builds the offset: byte 1 = the field, byte 0 = lane*4 | 128 h
  * (tb), bytes 2-3 = 0; the pair base is the load's immediate.
  * shared: at sb + 256 j + 4 v (sb 256-byte aligned); global: sp[64 j + v]. */
-#ifndef PAGODA_TDES_VARIANT
-#define PAGODA_TDES_VARIANT 0
-#endif
-__device__ __forceinline__ uint32_t imad1(uint32_t a, uint32_t one, uint32_t c)
-{   /* a * one + c with `one` opaque to ptxas, so it stays an IMAD (FMA pipe) */
-    uint32_t d;
-    asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(one), "r"(c));
-    return d;
-}
-
 template <int kMode>
-__device__ __forceinline__ uint32_t tdes_f(uint32_t r, uint32_t kx, uint32_t ky, uint32_t tb, const uint32_t* sp,
-                                           uint32_t one = 1)
+__device__ __forceinline__ uint32_t tdes_f(uint32_t r, uint32_t kx, uint32_t ky, uint32_t tb, const uint32_t* sp)
 {
     if (kMode == kTdesResident) {
         const uint32_t x = (__funnelshift_l(r, r, 5) ^ kx) & 0x3F3F3F3Fu;
         const uint32_t y = (__funnelshift_l(r, r, 1) ^ ky) & 0x3F3F3F3Fu;
         const uint32_t t1 = tb | 128u;
         constexpr uint32_t A = kResidentTdesAddr;
-#if PAGODA_TDES_VARIANT == 1
-        /* the 8 words have disjoint bits: XOR = ADD, summed by IMADs on the idle FMA pipe */
-        const uint32_t w0 = lds_at<A + 0 * 16384>(__byte_perm(x, tb, 0x7604)), w1 = lds_at<A + 1 * 16384>(__byte_perm(x, tb, 0x7614));
-        const uint32_t w2 = lds_at<A + 2 * 16384>(__byte_perm(x, tb, 0x7624)), w3 = lds_at<A + 3 * 16384>(__byte_perm(x, tb, 0x7634));
-        const uint32_t w4 = lds_at<A + 0 * 16384>(__byte_perm(y, t1, 0x7604)), w5 = lds_at<A + 1 * 16384>(__byte_perm(y, t1, 0x7614));
-        const uint32_t w6 = lds_at<A + 2 * 16384>(__byte_perm(y, t1, 0x7624)), w7 = lds_at<A + 3 * 16384>(__byte_perm(y, t1, 0x7634));
-        return imad1(imad1(imad1(w0, one, w1), one, imad1(w2, one, w3)), one,
-                     imad1(imad1(w4, one, w5), one, imad1(w6, one, w7)));
-#endif
         return lds_at<A + 0 * 16384>(__byte_perm(x, tb, 0x7604)) ^ lds_at<A + 1 * 16384>(__byte_perm(x, tb, 0x7614)) ^
                lds_at<A + 2 * 16384>(__byte_perm(x, tb, 0x7624)) ^ lds_at<A + 3 * 16384>(__byte_perm(x, tb, 0x7634)) ^
                lds_at<A + 0 * 16384>(__byte_perm(y, t1, 0x7604)) ^ lds_at<A + 1 * 16384>(__byte_perm(y, t1, 0x7614)) ^
@@ -291,7 +271,6 @@ __device__ __forceinline__ void tdes_blocks(const Env& e, const pagoda_tdes_args
 {
     const uint2* gkeys = reinterpret_cast<const uint2*>(a.tables + 512);
     const int T = total_threads(e);
-    const uint32_t one = (uint32_t)__popc(__activemask()) >> 5;   /* 1 (warps are converged here) */
     for (uint32_t blk = (uint32_t)e.getTid(); blk < a.nblk; blk += (uint32_t)T) {
         const uint2 in = reinterpret_cast<const uint2*>(a.in)[blk];
         /* bytes are the block in FIPS (big-endian) order: L = bytes 0..3, R = bytes 4..7 */
@@ -305,10 +284,10 @@ __device__ __forceinline__ void tdes_blocks(const Env& e, const pagoda_tdes_args
 #define PAGODA_TDES_ROUND2(I)                                                        \
             {                                                                        \
                 const uint4 k = tdes_key2<kKeysShared, I>(kst, gst);                 \
-                uint32_t t = l ^ tdes_f<kMode>(r, k.x, k.y, tb, a.tables, one);      \
+                uint32_t t = l ^ tdes_f<kMode>(r, k.x, k.y, tb, a.tables);           \
                 l = r;                                                               \
                 r = t;                                                               \
-                t = l ^ tdes_f<kMode>(r, k.z, k.w, tb, a.tables, one);               \
+                t = l ^ tdes_f<kMode>(r, k.z, k.w, tb, a.tables);                    \
                 l = r;                                                               \
                 r = t;                                                               \
             }

@@ -20,6 +20,9 @@
 
 #include "bodies.cuh"
 #include "mk_layout.cuh"
+#ifndef PAGODA_TDES_VARIANT
+#define PAGODA_TDES_VARIANT 0
+#endif
 
 namespace pagoda {
 
@@ -80,6 +83,12 @@ __device__ __forceinline__ uint64_t ld_acquire_sys(const volatile uint64_t* p)
 {
     uint64_t v;
     asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ uint32_t ld_acquire_sys32(const volatile uint32_t* p)
+{
+    uint32_t v;
+    asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
     return v;
 }
 __device__ __forceinline__ uint32_t ld_relaxed_sys32(const volatile uint32_t* p)
@@ -215,19 +224,34 @@ __device__ __forceinline__ void post_completions(MtbShared& S, const MkParams& p
             if (lane == 0) m = atomicExch(&S.comp_pending, 0u);
             m = __shfl_sync(0xffffffffu, m, 0);
             if (!m) break;
-            const bool mine = (m >> lane) & 1u;
-            const uint64_t id = mine ? S.tasks[lane].id : 0;
+            const bool done = (m >> lane) & 1u;
+            const uint64_t id = done ? S.tasks[lane].id : 0;
+            bool mine = done;
+            if (__any_sync(0xffffffffu, done && (S.tasks[lane].flags & kEntryGroup))) {
+                /* entries of a spread task: count its finished TBs; the entry completing the last posts
+                 * the task (release of this entry's writes before the count, acquire of the others' after) */
+                fence_acq_rel_gpu();
+                if (done && (S.tasks[lane].flags & kEntryGroup)) {
+                    const TaskEntry& te = S.tasks[lane];
+                    uint32_t* g = &p.grp[id & p.comp_mask];
+                    const uint32_t ntb_all = te.reserved >> 16;
+                    mine = atomicAdd(g, (uint32_t)te.n_tb) + te.n_tb == ntb_all;
+                    if (mine) atomicExch(g, 0u);   /* every other entry of the task has added */
+                }
+                fence_acq_rel_gpu();
+            }
             if (p.n_mtb == 1) {
                 asm volatile("fence.acq_rel.sys;" ::: "memory");
                 if (mine) st_relaxed_sys(reinterpret_cast<volatile uint64_t*>(&p.comp[id & p.comp_mask]), id);
             } else {
                 fence_acq_rel_gpu();   /* release: the tasks' writes (fenced by each of their warps) */
+                const uint32_t pm = __ballot_sync(0xffffffffu, mine);
                 unsigned long long base = 0;
-                if (lane == 0) base = atomicAdd(reinterpret_cast<unsigned long long*>(&p.dctl->dq_tail),
-                                                (unsigned long long)__popc(m));
+                if (lane == 0 && pm) base = atomicAdd(reinterpret_cast<unsigned long long*>(&p.dctl->dq_tail),
+                                                      (unsigned long long)__popc(pm));
                 base = __shfl_sync(0xffffffffu, base, 0);
                 if (mine) {
-                    const uint64_t slot = base + (uint64_t)__popc(m & ((1u << lane) - 1u));
+                    const uint64_t slot = base + (uint64_t)__popc(pm & ((1u << lane) - 1u));
                     uint64_t* q = &p.dq[slot & p.dq_mask];
                     while (*(volatile uint64_t*)q != 0) __nanosleep(64);   /* previous lap not forwarded yet */
                     st_relaxed_gpu(q, id + 1);
@@ -321,7 +345,13 @@ __device__ __forceinline__ void run_task(MtbShared& S, char* smem_base, const Mk
     if (lane == 0) {
         /* this warp's global writes -> visible GPU-wide before anyone learns the warp is done
          * (release; the completion poster's system-scope fence then publishes them to the host) */
+#if PAGODA_TDES_VARIANT == 2
+        /* CTA-scope release: the completion poster (same MTB) acquires it through the shared-memory
+         * counters below and its GPU-scope fence then releases every warp's writes (cumulativity) */
+        asm volatile("fence.acq_rel.cta;" ::: "memory");
+#else
         asm volatile("fence.acq_rel.gpu;" ::: "memory");
+#endif
         if (p.trace_cap) {
             uint32_t* cnt = &p.exec_count[mtb * 32 + w];
             const uint32_t i = *cnt;
@@ -457,7 +487,8 @@ __device__ __forceinline__ bool ingest_publish(const MkParams& p, const char* sr
         st_relaxed_gpu32(&p.dseq[t & p.ring_mask], (uint32_t)(t + 1));
     }
     __syncwarp();
-    if (lane == 0) st_relaxed_gpu(&p.dctl->tail, s + n);   /* hint for schedulers: work exists */
+    /* hint for schedulers that work exists (publishers finish out of order: the max) */
+    if (lane == 0) atomicMax(reinterpret_cast<unsigned long long*>(&p.dctl->tail), (unsigned long long)(s + n));
     c.batches++;
     c.entries += n;
     return true;
@@ -473,6 +504,10 @@ __device__ __forceinline__ void ingest_doorbell(const MkParams& p, uint64_t& pub
     if (lane == 0) {
         pub = ld_acquire_sys(&p.hctl->published);
         term = ld_relaxed_sys32(&p.hctl->terminate);
+        if (term) {   /* the host publishes every entry of the session before it sets terminate: */
+            term = ld_acquire_sys32(&p.hctl->terminate);   /* re-read the count after an acquire of it */
+            pub = ld_acquire_sys(&p.hctl->published);       /* (so this count is final) */
+        }
         err = *(volatile uint32_t*)&p.dctl->error;
         if (post_err && err != last_err) st_relaxed_sys32(&p.hctl->error, err);
     }
@@ -568,49 +603,54 @@ __device__ void ingest(MtbShared& S, const MkParams& p, char* stage_buf, uint64_
     ingest_flush(p, c);
 }
 
-/* Two-warp ingest (n_mtb > 1).  A fence waits for ALL of its warp's outstanding
+/* Multi-warp ingest (n_mtb > 1).  A fence waits for ALL of its warp's outstanding
  * memory operations, including a bulk read of the host ring still crossing a
- * busy PCIe link; so the warp that fences (the publisher) is not the warp that
- * reads host memory (the loader).  They hand the two stages back and forth
- * through mbarriers: full[s] (bulk copy landed; an arrival without bytes and
- * n = ~0 ends the stream) and empty[s] (the publisher is done with the stage). */
+ * busy PCIe link; so the warps that fence (the publishers) are not the warp
+ * that reads host memory (the loader).  The loader fills kIngestStages stages
+ * in ring order; stage k goes to buffer k mod kIngestStages and publisher
+ * k mod kIngestPublishers, so each publisher owns every P-th stage, double-
+ * buffered, and the publishers' per-batch latencies overlap.  Handshakes per
+ * buffer: full[b] (bulk copy landed; an arrival without bytes and n = ~0 ends
+ * a publisher's stream) and empty[b] (its publisher is done with it).
+ * Publishers finish out of order; the contiguous published prefix (what the
+ * host may reuse) advances over per-stage completion records. */
 __device__ void ingest_loader(MtbShared& S, const MkParams& p, char* stage_buf)
 {
     const uint32_t lane = threadIdx.x & 31u;
     const uint32_t SE = p.ingest_stage_entries;
     uint64_t fetched = *(volatile uint64_t*)&p.dctl->tail;
     uint64_t pub = fetched;
-    uint32_t term = 0, last_err = 0, ns = 0;
-    uint32_t uses[2] = {0, 0};
+    uint32_t term = 0, last_err = 0, k = 0, ends = 0;
     int idle = 0;
     IngestCtr c;
     for (;;) {
         if (fetched >= pub) {
             ingest_doorbell(p, pub, term, last_err, false, c);
-            if (term == kStopAbort) {   /* host watchdog: the publisher sees stop and leaves too */
+            if (term == kStopAbort) {   /* host watchdog: the publishers see stop and leave too */
                 if (lane == 0) st_release_gpu32(&p.dctl->stop, kStopAbort);
                 break;
             }
         }
         const bool end = term && fetched >= pub;
         if (fetched < pub || end) {
-            if (uses[ns]) mbar_wait(&S.ingest_empty[ns], (uses[ns] - 1u) & 1u);   /* stage free again */
-            uses[ns]++;
-            if (end) {
+            const uint32_t b = k % kIngestStages;
+            if (k >= kIngestStages) mbar_wait(&S.ingest_empty[b], (k / kIngestStages - 1u) & 1u);   /* free again */
+            k++;
+            if (end) {   /* one end marker per publisher, in its next stage */
                 if (lane == 0) {
-                    S.ing_n[ns] = ~0u;
-                    mbar_arrive(&S.ingest_bar[ns]);
+                    S.ing_n[b] = ~0u;
+                    mbar_arrive(&S.ingest_bar[b]);
                 }
-                break;
+                if (++ends == kIngestPublishers) break;
+                continue;
             }
             const uint32_t n = (uint32_t)min(pub - fetched, (uint64_t)SE);
             if (lane == 0) {
-                S.ing_start[ns] = fetched;
-                S.ing_n[ns] = n;
+                S.ing_start[b] = fetched;
+                S.ing_n[b] = n;
             }
-            ingest_load(p, stage_buf + ns * (SE * 64u), fetched, n, &S.ingest_bar[ns]);
+            ingest_load(p, stage_buf + b * (SE * 64u), fetched, n, &S.ingest_bar[b]);
             fetched += n;
-            ns ^= 1u;
             idle = 0;
         } else if (++idle > 64) {
             __nanosleep(256);
@@ -619,46 +659,76 @@ __device__ void ingest_loader(MtbShared& S, const MkParams& p, char* stage_buf)
     ingest_flush(p, c);
 }
 
-__device__ void ingest_publisher(MtbShared& S, const MkParams& p, char* stage_buf)
+/* stage k was published (end position e): record it, then advance the
+ * contiguous prefix as far as the records reach (one publisher at a time) */
+__device__ __forceinline__ void ingest_finish(MtbShared& S, uint32_t k, uint64_t e)
+{
+    if ((threadIdx.x & 31u) != 0) return;
+    const uint32_t slot = k % kIngestFinSlots;
+    *(volatile uint64_t*)&S.ing_fin_end[slot] = e;
+    __threadfence_block();
+    *(volatile uint32_t*)&S.ing_fin[slot] = k + 1u;
+    __threadfence_block();
+    for (;;) {
+        if (atomicCAS(&S.ing_lock, 0u, 1u) != 0u) return;   /* the holder re-checks after releasing */
+        __threadfence_block();
+        uint32_t q = *(volatile uint32_t*)&S.ing_prefix_k;
+        uint64_t end = 0;
+        bool moved = false;
+        while (*(volatile uint32_t*)&S.ing_fin[q % kIngestFinSlots] == q + 1u) {
+            end = *(volatile uint64_t*)&S.ing_fin_end[q % kIngestFinSlots];
+            q++;
+            moved = true;
+        }
+        if (moved) {
+            *(volatile uint64_t*)&S.ingest_copied = end;   /* for the host poster */
+            *(volatile uint32_t*)&S.ing_prefix_k = q;
+        }
+        __threadfence_block();
+        atomicExch(&S.ing_lock, 0u);
+        __threadfence_block();
+        /* a record written while the lock was held may have been missed: look again */
+        if (*(volatile uint32_t*)&S.ing_fin[q % kIngestFinSlots] != q + 1u) return;
+    }
+}
+
+__device__ __noinline__ void ingest_publisher(MtbShared& S, const MkParams& p, char* stage_buf, uint32_t me)
 {
     const uint32_t lane = threadIdx.x & 31u;
     const uint32_t SE = p.ingest_stage_entries;
-    uint32_t os = 0;
-    uint32_t uses[2] = {0, 0};
-    uint64_t copied = *(volatile uint64_t*)&p.dctl->tail;
     bool aborted = false;
     IngestCtr c;
-    for (;;) {
+    for (uint32_t k = me;; k += kIngestPublishers) {   /* my stages: me, me + P, ... */
+        const uint32_t b = k % kIngestStages;
         const uint64_t t1 = globaltimer_ns();
-        while (!mbar_try_wait(&S.ingest_bar[os], uses[os] & 1u, 20000u)) {
+        while (!mbar_try_wait(&S.ingest_bar[b], (k / kIngestStages) & 1u, 20000u)) {
             if (*(volatile uint32_t*)&p.dctl->stop == kStopAbort) {
                 aborted = true;
                 break;
             }
         }
         if (aborted) break;
-        uses[os]++;
         const uint64_t t2 = globaltimer_ns();
-        const uint32_t n = *(volatile uint32_t*)&S.ing_n[os];
+        const uint32_t n = *(volatile uint32_t*)&S.ing_n[b];
         if (n == ~0u) break;
         c.ns_copy += t2 - t1;
-        const uint64_t s = *(volatile uint64_t*)&S.ing_start[os];
-        if (!ingest_publish(p, stage_buf + os * (SE * 64u), s, n, c)) {
+        const uint64_t s = *(volatile uint64_t*)&S.ing_start[b];
+        if (!ingest_publish(p, stage_buf + b * (SE * 64u), s, n, c)) {
             aborted = true;
             break;
         }
-        copied = s + n;
-        if (lane == 0) {
-            *(volatile uint64_t*)&S.ingest_copied = copied;   /* for the host poster */
-            mbar_arrive(&S.ingest_empty[os]);
-        }
+        ingest_finish(S, k, s + n);
+        if (lane == 0) mbar_arrive(&S.ingest_empty[b]);
         c.ns_pub += globaltimer_ns() - t2;
-        os ^= 1u;
     }
     if (lane == 0) {
-        if (!aborted) st_release_gpu32(&p.dctl->stop, 1u);   /* everything published: drain and exit */
-        __threadfence_block();
-        *(volatile uint32_t*)&S.ingest_done = 1u;
+        /* the last publisher out: every stage was published (each saw its end marker after its
+         * data stages), so the device ring's tail is final: drain and exit */
+        if (atomicAdd(&S.ing_pubs_done, 1u) + 1u == kIngestPublishers) {
+            if (!aborted && *(volatile uint32_t*)&p.dctl->stop != kStopAbort) st_release_gpu32(&p.dctl->stop, 1u);
+            __threadfence_block();
+            *(volatile uint32_t*)&S.ingest_done = 1u;
+        }
     }
     ingest_flush(p, c);
 }
@@ -704,6 +774,9 @@ __device__ bool sched_place(MtbShared& S, Sched& st, const MkParams& p, int mtb,
     }
     const uint64_t id = e.id;
     const uint16_t threads = e.threads_tb;
+    /* a spread task's entry covers its TBs [tb0, tb0 + ntb) of ntb_all */
+    const bool group = e.flags & kEntryGroup;
+    const uint32_t tb0 = group ? (e.reserved & 0xFFFFu) : 0u, ntb_all = group ? (e.reserved >> 16) : ntb;
     if (lane == 0) S.task_warps_left[slot] = wtb * ntb;
     uint32_t all = 0;
     for (uint32_t j = 0; j < ntb; j++) {
@@ -733,14 +806,14 @@ __device__ bool sched_place(MtbShared& S, Sched& st, const MkParams& p, int mtb,
             S.tb_glen[tbs] = (uint16_t)gtb;
             S.tb_bar[tbs] = (uint8_t)bar;
             S.tb_task[tbs] = id;
-            S.tb_idx[tbs] = (uint16_t)j;
+            S.tb_idx[tbs] = (uint16_t)(tb0 + j);
         }
-        trace_ev(p, mtb, st.seq, 1, id, (uint16_t)j, m, (uint16_t)off, (uint16_t)gtb, (uint8_t)bar);
+        trace_ev(p, mtb, st.seq, 1, id, (uint16_t)(tb0 + j), m, (uint16_t)off, (uint16_t)gtb, (uint8_t)bar);
         if ((m >> lane) & 1u) {   /* Alg. 2 L9-12: lane l fills warp l's WarpTable slot */
             WarpSlot ws;
             ws.smem_off = p.arena_offset + off * PAGODA_GRANULE;
             ws.smem_bytes = gtb * PAGODA_GRANULE;
-            ws.tb = (uint16_t)j;
+            ws.tb = (uint16_t)(tb0 + j);
             ws.threads_tb = threads;
             ws.task = (uint8_t)slot;
             ws.warp_in_tb = (uint8_t)__popc(m & ((1u << lane) - 1u));
@@ -748,7 +821,7 @@ __device__ bool sched_place(MtbShared& S, Sched& st, const MkParams& p, int mtb,
             ws.n_tb = (uint8_t)ntb;
             ws.bar_id = (uint8_t)bar;
             ws.tbslot = (uint8_t)tbs;
-            ws.pad0 = 0;
+            ws.n_tb_all = (uint16_t)ntb_all;
             ws.task_id = id;
             S.wt[lane] = ws;
         }
@@ -1127,17 +1200,21 @@ __global__ void __launch_bounds__(1024, kMinBlocks) master_kernel(MkParams p)
     /* worker warps 0..exec_warps-1 (MTB 0: minus the ingest warp) */
     uint32_t exec_mask = p.exec_warps >= 32 ? 0xffffffffu : ((1u << p.exec_warps) - 1u);
     if (mtb == 0) exec_mask &= ~(1u << kIngestWarp);
-    if (io)   /* the I/O roles: loader (31), host poster (30), publisher (29), forwarder (28) */
-        exec_mask &= ~((1u << kHostPosterWarp) | (1u << kIngestPublisherWarp) | (1u << kForwarderWarp));
+    if (io)   /* the I/O roles: loader (31), host poster (30), forwarder (28), publishers (29, 27, ...) */
+    {
+        exec_mask &= ~((1u << kHostPosterWarp) | (1u << kForwarderWarp));
+        for (uint32_t i = 0; i < kIngestPublishers; i++) exec_mask &= ~(1u << ingest_publisher_warp(i));
+    }
     const int first = __ffs(exec_mask) - 1;
     if (warp == 0) {
         mbar_init(&S.exec_bar[lane], 1);
         mbar_init(&S.stage_bar[lane], 1);
         S.stage_ph[lane] = 0;
-        if (lane < 2) {
+        if (lane < kIngestStages) {
             mbar_init(&S.ingest_bar[lane], 1);
             mbar_init(&S.ingest_empty[lane], 1);
         }
+        for (uint32_t i = lane; i < kIngestFinSlots; i += 32u) S.ing_fin[i] = 0;
         /* initial scheduler state, owned by the first worker (it starts with the token) */
         S.sst_fg[lane] = bm_range_bits(0, (uint32_t)arena_granules, lane);
         if (lane == 0) {
@@ -1157,6 +1234,9 @@ __global__ void __launch_bounds__(1024, kMinBlocks) master_kernel(MkParams p)
              * (a spawn blocked on a ring slot would wait for it forever) */
             S.ingest_copied = *(volatile uint64_t*)&p.dctl->tail;
             S.ingest_done = 0;
+            S.ing_prefix_k = 0;
+            S.ing_lock = 0;
+            S.ing_pubs_done = 0;
             for (int i = 0; i < 8; i++) S.sctr[i] = 0;
             asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         }
@@ -1164,7 +1244,8 @@ __global__ void __launch_bounds__(1024, kMinBlocks) master_kernel(MkParams p)
     __syncthreads();
     if (mtb == 0 && p.n_mtb == 1 && warp == kIngestWarp) ingest(S, p, ingest_stage, S.ingest_bar);
     else if (mtb == 0 && warp == kIngestWarp) ingest_loader(S, p, ingest_stage);
-    else if (mtb == 0 && warp == kIngestPublisherWarp) ingest_publisher(S, p, ingest_stage);
+    else if (io && ingest_publisher_index(warp) < kIngestPublishers)
+        ingest_publisher(S, p, ingest_stage, ingest_publisher_index(warp));
     else if (mtb == 0 && warp == kHostPosterWarp) host_poster(S, p);
     else if (mtb == 0 && warp == kForwarderWarp) comp_forwarder(S, p);
     else if ((exec_mask >> warp) & 1u) worker(S, smem_base, p, mtb, warp, resident, exec_mask, warp == first);

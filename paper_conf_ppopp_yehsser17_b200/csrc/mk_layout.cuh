@@ -23,12 +23,13 @@ struct __align__(64) TaskEntry {
     uint8_t  warps_tb;     /* ceil(threads/32) */
     uint8_t  n_tb;
     uint8_t  gran_tb;      /* ceil(shmem/512) granules per TB */
-    uint8_t  flags;        /* bit0 = sync */
+    uint8_t  flags;        /* bit0 = sync, bit1 = one entry of a task spread over several MTBs (kEntryGroup) */
     uint32_t shmem_bytes;  /* requested bytes per TB */
-    uint32_t reserved;
+    uint32_t reserved;     /* group entries: first TB (bits 0-15) | the task's TB count (bits 16-31) */
     uint8_t  args[PAGODA_ARGS_MAX];
 };
 static_assert(sizeof(TaskEntry) == 64, "TaskEntry is 64 bytes");
+constexpr uint8_t kEntrySync = 1, kEntryGroup = 2;
 
 /* pinned, mapped host memory: written by one side, read by the other over PCIe */
 struct HostCtl {
@@ -101,6 +102,7 @@ struct MkParams {
                                             at kResidentOffset when non-null */
     int      n_mtb;
     uint64_t*        dq;      /* device completion queue (n_mtb > 1): id + 1 per record, 0 = empty */
+    uint32_t*        grp;     /* [comp_mask + 1] TBs finished per spread task (group), by id; 0 between uses */
     uint32_t dq_mask;
     uint32_t stage_offset;    /* n_mtb > 1: MTB 0's ingest stages start at this dynamic-smem offset */
     uint32_t io_sm_exclusive; /* the MTB sharing MTB 0's SM runs no tasks (several SMs) */
@@ -113,19 +115,32 @@ struct MkParams {
 
 constexpr int kIngestWarp = 31;          /* warp 31 of MTB 0 feeds the device ring */
 constexpr int kHostPosterWarp = 30;      /* warp 30 of MTB 0 (when n_mtb > 1): host-visible ingest stores */
-constexpr int kIngestPublisherWarp = 29; /* warp 29 of MTB 0 (when n_mtb > 1): publishes staged batches;
-                                            warp 31 then only loads them from the host ring */
 constexpr int kForwarderWarp = 28;       /* warp 28 of MTB 0 (when n_mtb > 1): completion records -> host */
+/* n_mtb > 1: kIngestPublishers publisher warps (29, 27, 26, ...) publish the loader's stages
+ * round-robin, each double-buffered (kIngestStages = 2 x publishers), so their per-batch
+ * latencies (cell checks, the bulk store, the release fence) overlap */
+#ifndef PAGODA_INGEST_PUBLISHERS
+#define PAGODA_INGEST_PUBLISHERS 2
+#endif
+constexpr uint32_t kIngestPublishers = PAGODA_INGEST_PUBLISHERS;
+constexpr uint32_t kIngestStages = 2u * kIngestPublishers;
+constexpr uint32_t kIngestFinSlots = 64;   /* >= kIngestStages: per-stage completion records */
+static_assert(kIngestPublishers >= 1 && kIngestPublishers <= 4, "publisher warps 29, 27, 26, 25");
+__host__ __device__ constexpr int ingest_publisher_warp(uint32_t i) { return i == 0 ? 29 : 28 - (int)i; }
+__host__ __device__ constexpr uint32_t ingest_publisher_index(int warp)   /* kIngestPublishers+ if none */
+{
+    return warp == 29 ? 0u : (warp >= 25 && warp <= 27) ? (uint32_t)(28 - warp) : 99u;
+}
 constexpr uint32_t kDqEntries = 1u << 16;  /* device completion queue */
 /* ingest staging: 2 stages of MkParams::ingest_stage_entries entries (64 B each).  One MTB: lent
  * from the top of MTB 0's arena (128 entries).  Several: MTB 0 runs no tasks and gives its whole
  * shared memory after the control block (stage_offset) to them. */
 constexpr uint32_t kIngestMaxStageEntries = 1024;
-constexpr uint32_t kStageOffset = 6144;   /* > kControlBytes, 1 KiB aligned */
+constexpr uint32_t kStageOffset = 7168;   /* > kControlBytes, 1 KiB aligned */
 __host__ __device__ inline uint32_t ingest_stage_entries(uint32_t smem_bytes, int n_mtb)
 {
     if (n_mtb == 1) return 128;   /* MTB 0 also runs tasks: keep most of its arena */
-    uint32_t e = (smem_bytes - kStageOffset) / (2u * 64u) / 32u * 32u;
+    uint32_t e = (smem_bytes - kStageOffset) / (kIngestStages * 64u) / 32u * 32u;
     return e > kIngestMaxStageEntries ? kIngestMaxStageEntries : e;
 }
 constexpr uint32_t kStopAbort = 2;       /* HostCtl.terminate / DevCtl.stop value: abandon work and exit */
@@ -157,16 +172,22 @@ struct MtbShared {
     uint32_t  sst_ph, sst_pl, sst_pt, sst_est_w, sst_seq;
     uint32_t  token;                 /* 1 while some warp holds the scheduler token */
     uint32_t  sctr[8];               /* scheduler counters (holder-only), flushed at exit */
-    uint64_t  ingest_bar[2];         /* MTB 0: the ingest warp's two TMA stage mbarriers */
-    uint64_t  ingest_empty[2];       /* MTB 0: stage s free again (publisher -> loader) */
-    uint64_t  ing_start[2];          /* MTB 0: first ring position of the batch in stage s */
-    uint32_t  ing_n[2];              /* MTB 0: entries in stage s (~0: end of stream) */
-    uint64_t  ingest_copied;         /* MTB 0: entries published into the device ring (for the host poster) */
-    uint32_t  ingest_done;           /* MTB 0: the ingest warp has exited */
-    uint32_t  comp_pending;          /* task slots finished, completion record not yet posted */
-    uint32_t  no_tickets;            /* this MTB runs no tasks (MTB 0 and the MTB sharing its SM) */
     uint32_t  stage_ph[32];          /* parity of each warp's staging mbarrier (TaskEnv::stage) */
     uint32_t  poster;                /* 1 while some warp posts completion records */
+    uint32_t  ingest_done;           /* MTB 0: the ingest warps have exited */
+    uint64_t  ingest_copied;         /* MTB 0: entries published into the device ring, a prefix (host poster) */
+    /* MTB 0 ingest, the rest of its control block */
+    uint64_t  ingest_bar[kIngestStages];    /* stage s loaded (TMA complete_tx; n = ~0 without bytes: end) */
+    uint64_t  ingest_empty[kIngestStages];  /* stage s free again (publisher -> loader) */
+    uint64_t  ing_start[kIngestStages];     /* first ring position of the batch in stage s */
+    uint32_t  ing_n[kIngestStages];         /* entries in stage s (~0: end of stream) */
+    uint64_t  ing_fin_end[kIngestFinSlots]; /* stage k published: its end position ... */
+    uint32_t  ing_fin[kIngestFinSlots];     /* ... and k + 1, in slot k mod kIngestFinSlots */
+    uint32_t  ing_prefix_k;                 /* stages [0, k) all published (ingest_copied is their end) */
+    uint32_t  ing_lock;                     /* serialises prefix advances */
+    uint32_t  ing_pubs_done;                /* publishers that saw their end marker */
+    uint32_t  comp_pending;          /* task slots finished, completion record not yet posted */
+    uint32_t  no_tickets;            /* this MTB runs no tasks (MTB 0 and the MTB sharing its SM) */
 };
 static_assert(offsetof(MtbShared, wt) == kWarpTableOffset, "WarpTable offset");
 static_assert(offsetof(MtbShared, stage_bar) == kStageBarOffset, "staging mbarriers offset");

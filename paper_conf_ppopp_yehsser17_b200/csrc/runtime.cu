@@ -58,6 +58,7 @@ struct pagoda_ctx {
     uint32_t* resident_src = nullptr;
     uint32_t* dseq = nullptr;
     uint64_t* dq = nullptr;                 /* device completion queue (n_mtb > 1) */
+    uint32_t* grp = nullptr;                /* per-id TB counters of spread tasks */
     DevCtl* dctl = nullptr;
     LedgerEvent* trace = nullptr;
     uint32_t* trace_count = nullptr;
@@ -132,6 +133,89 @@ static void advance_low(pagoda_ctx* c, uint64_t limit)
     while (l < limit && c->comp[l & mask] >= (int64_t)l) l++;
     c->low.store(l, std::memory_order_release);
 }
+
+/* ------------------------------------------------------------------ task shapes
+ * A task whose thread blocks do not fit one MTB (all warps of a task in one
+ * MTB, vs "64K threads" per task in Fig. 8) is spread
+ * over k consecutive TaskTable entries ("a group"), each a run of at most
+ * `cap` of its TBs that one MTB can host; it consumes k ids, the first is the
+ * task's id, and the MasterKernel posts it when the last TB finished
+ * (DESIGN.md "Readings" 6).  Sub-entries: flags bit 1, reserved = first TB
+ * (low 16 bits) | the task's TB count (high 16 bits). */
+struct Split {
+    int wtb = 0, cap = 0, k = 0;
+    uint32_t gtb = 0;
+};
+
+static int shape_check(const pagoda_ctx* c, const int32_t* s, Split& o)
+{
+    const int threads = s[0], n_tb = s[1], shmem = s[2], sync = s[3], func = s[4];
+    if (threads < 1 || threads > 1024 || n_tb < 1 || shmem < 0) return -EINVAL;
+    if (!known_func(func)) return -EINVAL;
+    o.wtb = (threads + 31) / 32;
+    o.gtb = ((uint32_t)shmem + PAGODA_GRANULE - 1) / PAGODA_GRANULE;
+    if (o.wtb > c->max_task_warps || o.gtb > c->max_task_granules) return -EINVAL;   /* one TB must fit an MTB */
+    if (o.wtb * n_tb <= c->max_task_warps && o.gtb * (uint32_t)n_tb <= c->max_task_granules &&
+        !(sync && o.wtb > 1 && n_tb > PAGODA_BAR_IDS)) {   /* fits one MTB (the common case: no divisions) */
+        o.cap = n_tb;
+        o.k = 1;
+        return 0;
+    }
+    int cap = c->max_task_warps / o.wtb;
+    if (o.gtb) cap = std::min<int>(cap, (int)(c->max_task_granules / o.gtb));
+    if (sync && o.wtb > 1) cap = std::min(cap, PAGODA_BAR_IDS);
+    o.cap = cap;
+    o.k = (n_tb + cap - 1) / cap;
+    if (o.k > 1 && (n_tb > 65535 || (uint32_t)o.k > c->R / 4)) return -EINVAL;
+    return 0;
+}
+
+/* consecutive tasks mostly share a shape: validate a shape once */
+struct ShapeMemo {
+    int32_t last[5] = {-1, -1, -1, -1, -1};
+    Split sp;
+    int rc = 0;
+    int check(const pagoda_ctx* c, const int32_t* s, Split& out)
+    {
+        if (s[0] != last[0] || s[1] != last[1] || s[2] != last[2] || s[3] != last[3] || s[4] != last[4]) {
+            rc = shape_check(c, s, sp);
+            memcpy(last, s, sizeof last);
+        }
+        out = sp;
+        return rc;
+    }
+};
+
+/* write entry j of a task (id0 = the task's id) into the host ring slot id0 + j */
+static inline void write_entry(pagoda_ctx* c, uint64_t id0, int j, const int32_t* s, const Split& sp, const void* args,
+                               size_t args_bytes)
+{
+    TaskEntry e;
+    memset(&e, 0, sizeof e);
+    const int tb0 = j * sp.cap;
+    e.id = id0;
+    e.func_id = (uint16_t)s[4];
+    e.threads_tb = (uint16_t)s[0];
+    e.warps_tb = (uint8_t)sp.wtb;
+    e.n_tb = (uint8_t)std::min(sp.cap, s[1] - tb0);
+    e.gran_tb = (uint8_t)sp.gtb;
+    e.flags = (s[3] ? 1 : 0) | (sp.k > 1 ? kEntryGroup : 0);
+    e.shmem_bytes = (uint32_t)s[2];
+    e.reserved = sp.k > 1 ? ((uint32_t)tb0 | ((uint32_t)s[1] << 16)) : 0u;
+    if (args_bytes) memcpy(e.args, args, args_bytes);
+    const __m128i* src = reinterpret_cast<const __m128i*>(&e);
+    __m128i* d = reinterpret_cast<__m128i*>(&c->hring[(id0 + (uint64_t)j) & (c->R - 1)]);
+    _mm_store_si128(d + 0, _mm_load_si128(src + 0));
+    _mm_store_si128(d + 1, _mm_load_si128(src + 1));
+    _mm_store_si128(d + 2, _mm_load_si128(src + 2));
+    _mm_store_si128(d + 3, _mm_load_si128(src + 3));
+    if (j > 0) c->comp[(id0 + (uint64_t)j) & (c->C - 1)] = (int64_t)(id0 + (uint64_t)j);   /* internal ids: only
+        the first is ever handed out, and the watermark passes them once it passed the first */
+}
+
+template <class ShapeOf>
+static int64_t spawn_batch(pagoda_ctx* c, int n, ShapeOf shape_of, const void* args_base, size_t args_stride,
+                           size_t args_bytes, pagoda_task_t* ids_out);
 
 extern "C" {
 
@@ -233,6 +317,7 @@ static void free_ctx(pagoda_ctx* c)
     if (c->dring) cudaFree(c->dring);
     if (c->dseq) cudaFree(c->dseq);
     if (c->dq) cudaFree(c->dq);
+    if (c->grp) cudaFree(c->grp);
     if (c->resident_src) cudaFree(c->resident_src);
     if (c->dctl) cudaFree(c->dctl);
     if (c->trace) cudaFree(c->trace);
@@ -317,6 +402,8 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
     if (cudaMemset(c->dctl, 0, sizeof(DevCtl)) != cudaSuccess) goto fail;
     if (cudaMemset(&c->dctl->io_smid, 0xFF, sizeof(uint32_t)) != cudaSuccess) goto fail;
     if (cudaMalloc(&c->dq, (size_t)kDqEntries * sizeof(uint64_t)) != cudaSuccess) goto fail;
+    if (cudaMalloc(&c->grp, (size_t)c->C * sizeof(uint32_t)) != cudaSuccess) goto fail;
+    if (cudaMemset(c->grp, 0, (size_t)c->C * sizeof(uint32_t)) != cudaSuccess) goto fail;
     if (cudaMemset(c->dq, 0, (size_t)kDqEntries * sizeof(uint64_t)) != cudaSuccess) goto fail;
     if (cfg.flags & PAGODA_TRACE) {
         const size_t cap = cfg.trace_events ? cfg.trace_events : 8192;
@@ -353,6 +440,7 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
         p.stage_offset = kStageOffset;
         p.io_sm_exclusive = nsm > 1 ? 1u : 0u;   /* one SM: its other MTB must run the tasks */
         p.dq = c->dq;
+        p.grp = c->grp;
         p.dq_mask = kDqEntries - 1;
         if (cfg.flags & PAGODA_RESIDENT_TDES) {   /* the key-independent SP table, replicated by each MTB */
             std::vector<uint8_t> tab(PAGODA_TDES_TABLE_BYTES);
@@ -387,14 +475,17 @@ pagoda_task_t pagoda_taskSpawn(pagoda_ctx* c, int threads, int n_tb, int shmem_b
     if (!c) return -EINVAL;
     if (c->shutting.load(std::memory_order_acquire)) return -ESHUTDOWN;
     if (c->faulted.load(std::memory_order_relaxed)) return -EIO;
-    if (threads < 1 || threads > 1024 || n_tb < 1 || shmem_bytes < 0) return -EINVAL;
-    const int wtb = (threads + 31) / 32;
-    if ((long)wtb * n_tb > c->max_task_warps) return -EINVAL;
-    const uint32_t gtb = ((uint32_t)shmem_bytes + PAGODA_GRANULE - 1) / PAGODA_GRANULE;
-    if ((uint64_t)gtb * (uint64_t)n_tb > c->max_task_granules) return -EINVAL;
-    if (sync_flag && wtb > 1 && n_tb > PAGODA_BAR_IDS) return -EINVAL;
-    if (!known_func(func_id)) return -EINVAL;
+    const int32_t shape[5] = {threads, n_tb, shmem_bytes, sync_flag, func_id};
+    Split sp;
+    if (int rc = shape_check(c, shape, sp)) return rc;
     if (args_bytes > PAGODA_ARGS_MAX || (args_bytes > 0 && !args)) return -EINVAL;
+    if (sp.k > 1) {   /* spread over several MTB entries: the batched path writes the group */
+        pagoda_task_t id = -1;
+        const int64_t rc = spawn_batch(c, 1, [&](int) { return shape; }, args, args_bytes, args_bytes, &id);
+        return rc < 0 ? (pagoda_task_t)rc : id;
+    }
+    const int wtb = sp.wtb;
+    const uint32_t gtb = sp.gtb;
 
     const uint64_t id = c->next_id.fetch_add(1, std::memory_order_acq_rel);
     /* 1. ring slot free: the ingest warp has copied entry id - R */
@@ -416,25 +507,8 @@ pagoda_task_t pagoda_taskSpawn(pagoda_ctx* c, int threads, int n_tb, int shmem_b
         if (rc) return rc;
     }
     /* 3. the entry */
-    TaskEntry e;
-    memset(&e, 0, sizeof e);
-    e.id = id;
-    e.func_id = (uint16_t)func_id;
-    e.threads_tb = (uint16_t)threads;
-    e.warps_tb = (uint8_t)wtb;
-    e.n_tb = (uint8_t)n_tb;
-    e.gran_tb = (uint8_t)gtb;
-    e.flags = sync_flag ? 1 : 0;
-    e.shmem_bytes = (uint32_t)shmem_bytes;
-    if (args_bytes) memcpy(e.args, args, args_bytes);
-    {
-        const __m128i* s = reinterpret_cast<const __m128i*>(&e);
-        __m128i* d = reinterpret_cast<__m128i*>(&c->hring[id & (c->R - 1)]);
-        _mm_store_si128(d + 0, _mm_load_si128(s + 0));
-        _mm_store_si128(d + 1, _mm_load_si128(s + 1));
-        _mm_store_si128(d + 2, _mm_load_si128(s + 2));
-        _mm_store_si128(d + 3, _mm_load_si128(s + 3));
-    }
+    write_entry(c, id, 0, shape, sp, args, args_bytes);
+    (void)gtb;
     const int64_t w = (int64_t)wtb * n_tb;
     /* 4. in-order commit of the doorbell (x86 stores are ordered; the fence is for the compiler) */
     if (c->published.load(std::memory_order_acquire) != id) {
@@ -462,22 +536,25 @@ static int64_t spawn_batch(pagoda_ctx* c, int n, ShapeOf shape_of, const void* a
     if (c->shutting.load(std::memory_order_acquire)) return -ESHUTDOWN;
     if (c->faulted.load(std::memory_order_relaxed)) return -EIO;
     if (args_bytes > PAGODA_ARGS_MAX || (args_bytes > 0 && !args_base)) return -EINVAL;
+    ShapeMemo memo;
     for (int i = 0; i < n; i++) {
-        const int32_t* s = shape_of(i);
-        const int threads = s[0], n_tb = s[1], shmem = s[2], sync = s[3], func = s[4];
-        if (threads < 1 || threads > 1024 || n_tb < 1 || shmem < 0) return -EINVAL;
-        const int wtb = (threads + 31) / 32;
-        if ((long)wtb * n_tb > c->max_task_warps) return -EINVAL;
-        const uint32_t gtb = ((uint32_t)shmem + PAGODA_GRANULE - 1) / PAGODA_GRANULE;
-        if ((uint64_t)gtb * (uint64_t)n_tb > c->max_task_granules) return -EINVAL;
-        if (sync && wtb > 1 && n_tb > PAGODA_BAR_IDS) return -EINVAL;
-        if (!known_func(func)) return -EINVAL;
+        Split sp;
+        if (int rc = memo.check(c, shape_of(i), sp)) return rc;
     }
     const char* a = static_cast<const char*>(args_base);
-    for (int base = 0; base < n; base += kSpawnChunk) {
-        const int m = std::min(kSpawnChunk, n - base);
-        const uint64_t id0 = c->next_id.fetch_add((uint64_t)m, std::memory_order_acq_rel);
-        const uint64_t last = id0 + (uint64_t)m - 1;
+    for (int base = 0; base < n;) {
+        /* a chunk: up to kSpawnChunk tasks, each one or more entries (ids) */
+        Split sps[kSpawnChunk];
+        int m = 0;
+        uint64_t K = 0;
+        while (base + m < n && m < kSpawnChunk) {
+            memo.check(c, shape_of(base + m), sps[m]);
+            if (m > 0 && K + (uint64_t)sps[m].k > (uint64_t)(c->R / 4)) break;
+            K += (uint64_t)sps[m].k;
+            m++;
+        }
+        const uint64_t id0 = c->next_id.fetch_add(K, std::memory_order_acq_rel);
+        const uint64_t last = id0 + K - 1;
         if (last >= c->R && c->consumed_cache.load(std::memory_order_acquire) <= last - c->R) {
             int rc = spin_until(c, [&] {
                 const uint64_t v = c->hctl->consumed;
@@ -494,44 +571,31 @@ static int64_t spawn_batch(pagoda_ctx* c, int n, ShapeOf shape_of, const void* a
             });
             if (rc) return rc;
         }
-        int64_t w_chunk[kSpawnChunk];
+        uint64_t id = id0;
         for (int i = 0; i < m; i++) {
             const int32_t* s = shape_of(base + i);
-            const uint64_t id = id0 + (uint64_t)i;
-            TaskEntry e;
-            memset(&e, 0, sizeof e);
-            const int wtb = (s[0] + 31) / 32;
-            e.id = id;
-            e.func_id = (uint16_t)s[4];
-            e.threads_tb = (uint16_t)s[0];
-            e.warps_tb = (uint8_t)wtb;
-            e.n_tb = (uint8_t)s[1];
-            e.gran_tb = (uint8_t)(((uint32_t)s[2] + PAGODA_GRANULE - 1) / PAGODA_GRANULE);
-            e.flags = s[3] ? 1 : 0;
-            e.shmem_bytes = (uint32_t)s[2];
-            if (args_bytes) memcpy(e.args, a + (size_t)(base + i) * args_stride, args_bytes);
-            const __m128i* src = reinterpret_cast<const __m128i*>(&e);
-            __m128i* d = reinterpret_cast<__m128i*>(&c->hring[id & (c->R - 1)]);
-            _mm_store_si128(d + 0, _mm_load_si128(src + 0));
-            _mm_store_si128(d + 1, _mm_load_si128(src + 1));
-            _mm_store_si128(d + 2, _mm_load_si128(src + 2));
-            _mm_store_si128(d + 3, _mm_load_si128(src + 3));
-            w_chunk[i] = (int64_t)wtb * s[1];
+            for (int j = 0; j < sps[i].k; j++)
+                write_entry(c, id, j, s, sps[i], args_bytes ? a + (size_t)(base + i) * args_stride : nullptr,
+                            args_bytes);
             if (ids_out) ids_out[base + i] = (pagoda_task_t)id;
+            id += (uint64_t)sps[i].k;
         }
         if (c->published.load(std::memory_order_acquire) != id0) {
             int rc = spin_until(c, [&] { return c->published.load(std::memory_order_acquire) == id0; });
             if (rc) return rc;
         }
         int64_t ws = c->warps_spawned.load(std::memory_order_relaxed);
-        for (int i = 0; i < m; i++) {
-            ws += w_chunk[i];
-            c->warps_prefix[(id0 + (uint64_t)i) & (c->C - 1)] = ws;
+        id = id0;
+        for (int i = 0; i < m; i++) {   /* a task's warps count at its first id, its other ids add none */
+            const int32_t* s = shape_of(base + i);
+            ws += (int64_t)sps[i].wtb * s[1];
+            for (int j = 0; j < sps[i].k; j++) c->warps_prefix[(id++) & (c->C - 1)] = ws;
         }
         c->warps_spawned.store(ws, std::memory_order_relaxed);
         std::atomic_thread_fence(std::memory_order_release);
         c->hctl->published = last + 1;
         c->published.store(last + 1, std::memory_order_release);
+        base += m;
     }
     return n;
 }
@@ -603,8 +667,24 @@ int pagoda_stop(pagoda_ctx* c)
     if (!c) return -EINVAL;
     std::lock_guard<std::mutex> lk(c->session_mtx);
     if (!c->running.load()) return -EALREADY;
-    int rc = c->faulted.load() ? -EIO : pagoda_waitAll(c);
-    int r2 = stop_kernel(c);
+    if (c->faulted.load()) {
+        const int r2 = stop_kernel(c);
+        return r2 ? r2 : -EIO;
+    }
+    /* Every task issued before the call is published, then terminate: the MasterKernel drains
+     * everything published and exits (the ingest reads terminate before the published count),
+     * so the stop does not wait for the host to observe the last completion first. */
+    const uint64_t n = c->next_id.load(std::memory_order_acquire);
+    int rc = spin_until(c, [&] { return c->published.load(std::memory_order_acquire) >= n; });
+    const int r2 = stop_kernel(c);
+    if (!rc && !r2) {   /* the session drained: every id below n has its completion record */
+        rc = spin_until(c, [&] {
+            advance_low(c, n);
+            return c->low.load(std::memory_order_acquire) >= n;
+        });
+        if (rc == -EAGAIN) rc = -EIO;   /* published before terminate, yet not completed */
+        std::atomic_thread_fence(std::memory_order_acquire);
+    }
     return rc ? rc : r2;
 }
 

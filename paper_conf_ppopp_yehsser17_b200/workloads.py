@@ -285,7 +285,7 @@ class PooledWorkload(Workload):
         raise NotImplementedError("pooled workloads are read per task: task_output(k)")
 
 
-def pooled(name, pool: InputPool, kinds, in_idx, threads, shmem, device="cuda", resident=False, fill=None):
+def pooled(name, pool: InputPool, kinds, in_idx, threads, shmem, device="cuda", resident=False, fill=None, n_tb=1):
     """kinds[i] indexes pool.kinds; in_idx[i] the pool entry; threads / shmem
     are used for FB, BF, CONV, DCT (MB, 3DES, MM take their configs' shapes).
     fill: byte value the output buffer is initialised with (None: left as
@@ -295,20 +295,20 @@ def pooled(name, pool: InputPool, kinds, in_idx, threads, shmem, device="cuda", 
     kinds = np.asarray(kinds, np.int32)
     in_idx = np.asarray(in_idx, np.int64)
     shapes = np.zeros((n, 5), np.int32)
-    shapes[:, 0], shapes[:, 1], shapes[:, 2] = threads, 1, shmem
+    shapes[:, 0], shapes[:, 1], shapes[:, 2] = threads, n_tb, shmem
     out_len = np.zeros(n, np.int64)
     scr_len = np.zeros(n, np.int64)
     for ki, k in enumerate(pool.kinds):
         i = np.nonzero(kinds == ki)[0]
         out_len[i] = pool.out_bytes(k, in_idx[i])
-        scr_len[i] = SCRATCH_BYTES.get(k, 0)
+        scr_len[i] = SCRATCH_BYTES.get(k, 0) * n_tb   # FB / CONV: one scratch region per TB
         shapes[i, 3], shapes[i, 4] = SYNC[k], KIND_FUNC[k]
         if k == "mb":
-            shapes[i, 0], shapes[i, 2] = 128, 0
+            shapes[i, 0], shapes[i, 1], shapes[i, 2] = 128, 1, 0
         elif k == "tdes":
-            shapes[i, 0], shapes[i, 2] = 128, (512 if resident else 2560)
+            shapes[i, 0], shapes[i, 1], shapes[i, 2] = 128, 1, (512 if resident else 2560)
         elif k == "mm":
-            shapes[i, 0], shapes[i, 2] = 256, 8192
+            shapes[i, 0], shapes[i, 1], shapes[i, 2] = 256, 1, 8192
     span = (out_len + scr_len + _ALIGN - 1) // _ALIGN * _ALIGN
     base = np.zeros(n + 1, np.int64)
     np.cumsum(span, out=base[1:])
@@ -378,3 +378,11 @@ def tdes_var(n_tasks=32768, device="cuda", resident=False, fill=None):
     Table 3), one task of 128 threads each."""
     pool = InputPool(("tdes",), n_tasks, device, var_tdes=True)
     return pooled("tdes_var", pool, np.zeros(n_tasks, np.int32), np.arange(n_tasks), 128, 0, device, resident, fill)
+
+
+def conv_only(n_tasks, device="cuda", threads=256, shmem=0, fill=None, n_tb=1):
+    """CONV tasks alone (each its own 128x128 input), for the large-task sweep;
+    n_tb thread blocks per task (a task larger than an MTB is spread)."""
+    pool = InputPool(("conv",), n_tasks, device)
+    return pooled("conv", pool, np.zeros(n_tasks, np.int32), np.arange(n_tasks), threads, shmem, device, fill=fill,
+                  n_tb=n_tb)

@@ -3,6 +3,8 @@
   tasks   : #tasks in {32 .. 32768} of 3DES (4 KiB, 128 threads)   (Fig. 6)
   threads : threads per task in {32 .. 1024}, 32768 3DES tasks      (Fig. 7)
             and 8192 MB tiles (MB repeats config 1's 1024 tiles)
+  large   : 4096 CONV tasks (128x128) of 128 .. 16384 threads; above 1024 the task is
+            several 1024-thread TBs spread over MTBs (Fig. 8's large tasks)
 
 Each point: Pagoda (one session: start -> spawn all -> stop; CUDA-event
 device time and host time), the naive one-launch-per-task baseline and the
@@ -47,6 +49,8 @@ def time_naive(w):
 
 
 def time_fused(w):
+    if (w.shapes[:, 1] != 1).any():
+        return None   # static fusion runs one thread block per task
     PG.fused_run(0, w.shapes[:256], w.args[:256], 256)
     r = [PG.fused_run(0, w.shapes, w.args, 256) for _ in range(3)]
     return w.n / (statistics.median(x[0] for x in r) * 1e-9)
@@ -57,7 +61,7 @@ def point(sweep, label, w, **cfg):
     out = {"sweep": sweep, **label, "n_tasks": w.n, "pagoda_tasks_per_s": dev, "pagoda_host_tasks_per_s": host,
            "naive_tasks_per_s": time_naive(w), "fused_tasks_per_s": time_fused(w)}
     out["speedup_vs_naive"] = dev / out["naive_tasks_per_s"]
-    out["speedup_vs_fused"] = dev / out["fused_tasks_per_s"]
+    out["speedup_vs_fused"] = dev / out["fused_tasks_per_s"] if out["fused_tasks_per_s"] else None
     print(json.dumps(out), flush=True)
 
 
@@ -72,6 +76,9 @@ def main():
         point("threads", {"body": "tdes", "threads": th}, w, **res)
         w = W.mandelbrot(8192, threads=th)
         point("threads", {"body": "mb", "threads": th}, w)
+    for th in (128, 512, 1024, 4096, 16384):       # Fig. 8: large tasks, spread over MTBs above 1024
+        w = W.conv_only(4096, threads=min(th, 1024), n_tb=max(1, th // 1024))
+        point("large", {"body": "conv", "threads": th, "tbs": max(1, th // 1024)}, w)
 
 
 if __name__ == "__main__":

@@ -144,8 +144,8 @@ def test_validation_and_shutdown_errors():
     E = -errno.EINVAL
     assert p.taskSpawn(0, 1, 0, 0, T.NOP) == E
     assert p.taskSpawn(1025, 1, 0, 0, T.NOP) == E          # > 1024 threads
-    assert p.taskSpawn(128, 9, 0, 0, T.NOP) == E           # 36 warps > 32 per MTB
-    assert p.taskSpawn(32, 1, 96 * 1024 + 1, 0, T.NOP) == E
+    assert p.taskSpawn(32, 1, 96 * 1024 + 1, 0, T.NOP) == E   # one TB larger than an MTB's arena
+    assert p.taskSpawn(32, 65536, 0, 0, T.NOP) == E         # > 65535 TBs
     assert p.taskSpawn(128, 1, 0, 0, 99) == E
     assert p.taskSpawn(128, 1, 0, 0, T.NOP, b"\0" * 41) == E
     assert p.taskSpawn(1024, 1, 96 * 1024, 1, T.NOP) >= 0  # a whole MTB: all 32 warps (self-scheduling)
@@ -293,3 +293,72 @@ def test_pingpong_floor():
     with Pagoda() as p:
         lat = p.latency_loop(200, 128, 1, 0, False, T.NOP)
     assert np.median(lat) >= 0.9 * np.median(rtt)
+
+
+# ---------------------------------------------------------------- tasks spread over several MTBs (NEXT-3)
+def test_spread_tasks_ids_and_exactly_once():
+    """Tasks larger than one MTB (Fig. 8's large tasks): MARK and
+    TID over k MTB entries run every thread once, the task completes once, and
+    it consumes k ids; the oracle-side rule gives the same ids."""
+    import oracle as O
+    dev = Dev()
+    cases = [(128, 64, 0, 1), (32, 2048, 0, 0), (1024, 5, 0, 1), (100, 40, 600, 1), (64, 17, 48 * 1024, 1)]
+    cap = sum(th * nb for th, nb, _, _ in cases)
+    out = dev.zeros(4 * 4 * (32 * 2048 + 4096))
+    cnt = dev.zeros(4 * len(cases))
+    tid_out = dev.zeros(4 * 32 * 2048)
+    orc = O.Ctx(exec_warps=32)
+    with Pagoda() as p:
+        ids, base = [], 0
+        for i, (th, nb, sh, sy) in enumerate(cases):
+            args = np.array([(ptr(out) + 4 * base, ptr(cnt) + 4 * i, 0, 1000 + i)], T.ARGS[T.MARK])
+            ids.append(p.taskSpawn(th, nb, sh, sy, T.MARK, args))
+            assert orc.spawn(th, nb, sh, sy, O.NOP, None) == ids[-1]   # same id rule
+            base += ((th + 31) // 32) * 32 * nb
+        targs = np.array([(ptr(tid_out), 0, 0)], T.ARGS[T.TID])
+        tid_id = p.taskSpawn(32, 2048, 0, 0, T.TID, targs)
+        nop = p.taskSpawn(32, 1, 0, 0, T.NOP)
+        assert ids[0] == 0 and ids[1] == 8 and tid_id > ids[-1] and nop > tid_id
+        assert p.waitAll() == 0 and p.info().device_error == 0
+        assert all(p.check(i) == 1 for i in ids + [tid_id, nop])
+    c = Dev.get(cnt, np.uint32)
+    o = Dev.get(out, np.uint32)
+    base = 0
+    for i, (th, nb, _, _) in enumerate(cases):
+        assert c[i] == th * nb, (i, c[i])
+        span = ((th + 31) // 32) * 32
+        seg = o[base: base + span * nb].reshape(nb, span)
+        assert (seg[:, :th] == 1000 + i).all() and (seg[:, th:] == 0).all(), i
+        base += span * nb
+    t = Dev.get(tid_out, np.uint32)
+    assert np.array_equal(t >> 16, np.arange(32 * 2048) // 32)           # getBlockIdx: global TB index
+    assert np.array_equal(t & 0xFFFF, np.arange(32 * 2048) % 32)         # getBlockTid
+
+
+def test_spread_task_parity_and_sync():
+    """Bodies over spread tasks: a Mandelbrot tile with 4096 threads (16 TBs of
+    256 = 2 MTB entries), 3DES with 32 TBs, and BAR phases (syncBlock per TB)
+    over 40 syncing TBs."""
+    import oracle as O
+    from paper_conf_ppopp_yehsser17_b200 import inputs as I
+    from paper_conf_ppopp_yehsser17_b200 import workloads as W
+    mb = W.mandelbrot(8, threads=256)
+    mb.shapes[:, 1] = 16
+    td = W.tdes(6, shmem=2560)
+    td.shapes[:, 1] = 32
+    dev = Dev()
+    err = dev.zeros(4)
+    scratch = dev.zeros(4 * 1024 * 40)
+    bargs = np.array([(ptr(err), ptr(scratch), 5, 0)], T.ARGS[T.BAR])
+    with Pagoda() as p:
+        p.spawn_shapes(mb.shapes, mb.args)
+        p.spawn_shapes(td.shapes, td.args)
+        p.taskSpawn(128, 40, 0, 1, T.BAR, bargs)
+        assert p.waitAll() == 0 and p.info().device_error == 0
+    out = mb.outputs()["out"]
+    for k in range(8):
+        assert np.array_equal(out[k], O.mandelbrot_tile(int(mb.host["tx"][k]), int(mb.host["ty"][k])))
+    out = td.outputs()["out"]
+    for k in range(6):
+        assert np.array_equal(out[k], O.tdes_ecb(td.host["packets"][k], I.TDES_KEYS))
+    assert Dev.get(err, np.uint32)[0] == 0

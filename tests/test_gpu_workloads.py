@@ -127,3 +127,14 @@ def test_c5_shards_partition_the_tasks():
         assert np.array_equal(p.kinds, full.kinds[p.first:p.first + p.n])
         assert np.array_equal(p.in_idx, full.in_idx[p.first:p.first + p.n])
         assert np.array_equal(p.shapes, full.shapes[p.first:p.first + p.n])
+
+
+# ---------------------------------------------------------------- large tasks spread over MTBs (NEXT-3)
+@pytest.mark.parametrize("threads,n_tb,shmem", [(1024, 16, 0), (512, 8, 48 * 1024), (256, 3, 4096)])
+def test_conv_large_tasks(threads, n_tb, shmem):
+    """CONV with up to 16384 threads per task (16 TBs spread over MTBs; each TB
+    computes the row pass its own outputs need, Fig. 8's large tasks)."""
+    w = W.conv_only(12, threads=threads, shmem=shmem, fill=0xAB, n_tb=n_tb)
+    assert (w.shapes[:, 1] == n_tb).all()
+    run(w)
+    assert check_tasks(w, range(12)) == {"conv"}

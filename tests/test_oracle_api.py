@@ -22,15 +22,18 @@ def test_spawn_ids_monotone_and_semantics(orc):
 @pytest.mark.parametrize("threads,ntb,shmem,sync,func,nargs,ok", [
     (0, 1, 0, 0, O.NOP, 0, False),          # threads < 1
     (992, 1, 0, 0, O.NOP, 0, True),         # 31 warps: one whole MTB
-    (993, 1, 0, 0, O.NOP, 0, False),        # 32 warps > 31 executor warps
-    (128, 8, 0, 0, O.NOP, 0, False),        # 4 warps x 8 TBs = 32 > 31
+    (993, 1, 0, 0, O.NOP, 0, False),        # one TB of 32 warps > 31 executor warps
+    (1025, 1, 0, 0, O.NOP, 0, False),       # > 1024 threads per TB
+    (128, 8, 0, 0, O.NOP, 0, True),         # 4 warps x 8 TBs = 32 > 31: spread over 2 MTBs
     (128, 7, 0, 1, O.NOP, 0, True),
     (32, 1, 96 * 1024, 0, O.NOP, 0, True),  # whole arena
-    (32, 1, 96 * 1024 + 1, 0, O.NOP, 0, False),
-    (32, 2, 48 * 1024 + 1, 0, O.NOP, 0, False),  # 2 x 97 granules > 192
+    (32, 1, 96 * 1024 + 1, 0, O.NOP, 0, False),   # one TB larger than an MTB's arena
+    (32, 2, 48 * 1024 + 1, 0, O.NOP, 0, True),    # 2 x 97 granules > 192: spread
     (32, 31, 0, 1, O.NOP, 0, True),         # 1-warp TBs need no barrier ID
     (64, 15, 0, 1, O.NOP, 0, True),         # 15 barrier IDs (16 minus ID 0)
-    (64, 16, 0, 1, O.NOP, 0, False),        # needs 32 warps anyway
+    (64, 16, 0, 1, O.NOP, 0, True),         # 16 syncing TBs: spread (15 + 1)
+    (32, 65536, 0, 0, O.NOP, 0, False),     # > 65535 TBs
+    (1024, 1, 0, 0, O.NOP, 0, False),       # 32 warps > the 31 executor warps of this context
     (128, 1, 0, 0, 99, 0, False),           # unknown func
     (128, 1, 0, 0, O.NOP, 41, False),       # args > 40 B
     (128, 1, -1, 0, O.NOP, 0, False),
@@ -42,6 +45,24 @@ def test_validation_table(orc, threads, ntb, shmem, sync, func, nargs, ok):
     assert (rc >= 0) == ok, rc
     if not ok:
         assert rc == -errno.EINVAL
+
+
+def test_spread_task_ids(orc):
+    """A task larger than one MTB consumes k = ceil(n_tb / cap) ids (its id is
+    the first), and runs every TB: MARK over 64 TBs of 4 warps (cap 7 per MTB
+    of 31 warps -> 10 entries)."""
+    ctx = O.Ctx()
+    out = np.zeros(64 * 128, np.uint32)
+    cnt = np.zeros(1, np.uint32)
+    a = ctx.spawn(128, 1, 0, 0, O.NOP, None)
+    args = struct.pack("<QQII", out.ctypes.data, cnt.ctypes.data, 0, 5)
+    b = ctx.spawn(128, 64, 0, 1, O.MARK, args)
+    c = ctx.spawn(128, 1, 0, 0, O.NOP, None)
+    assert (a, b, c) == (0, 1, 1 + 10)
+    assert (out == 5).all() and cnt[0] == 64 * 128
+    assert ctx.wait(b) == 0 and ctx.check(b + 3) == 1 and ctx.waitAll() == 0
+    ctx32 = O.Ctx(exec_warps=32)
+    assert ctx32.spawn(1024, 3, 0, 1, O.NOP, None) == 0 and ctx32.spawn(32, 1, 0, 0, O.NOP, None) == 3
 
 
 def test_mark_and_tid_bodies(orc):
