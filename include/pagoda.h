@@ -172,7 +172,10 @@ enum {
     PAGODA_CTR_LOAD_NOT_READY, PAGODA_CTR_PLACED, PAGODA_CTR_PLACE_NOFIT, PAGODA_CTR_HANDOFFS,
     PAGODA_CTR_INGEST_NS_FENCE,   /* ns of the ingest publish phase spent in its fences */
     PAGODA_CTR_INGEST_NS_STORE,   /* ns spent in the bulk store into the device ring */
-    PAGODA_CTR_COUNT = 16
+    /* profiling builds only (-DPAGODA_PROFILE=1), else 0: scheduler-holder and executor time split */
+    PAGODA_CTR_SCHED_NS_FOLD, PAGODA_CTR_SCHED_NS_LOAD, PAGODA_CTR_SCHED_NS_PLACE, PAGODA_CTR_SCHED_NS_CLAIM,
+    PAGODA_CTR_SCHED_NS_SLEEP, PAGODA_CTR_EXEC_NS_BODY, PAGODA_CTR_EXEC_NS_FENCE, PAGODA_CTR_EXEC_NS_POST,
+    PAGODA_CTR_COUNT = 24
 };
 /* Copy min(n, PAGODA_CTR_COUNT) counters into out[]; returns the number copied or < 0. */
 int pagoda_read_counters(pagoda_ctx* ctx, uint64_t* out, int n);

@@ -20,8 +20,15 @@
 
 #include "bodies.cuh"
 #include "mk_layout.cuh"
-#ifndef PAGODA_TDES_VARIANT
-#define PAGODA_TDES_VARIANT 0
+/* A/B switches (scripts/build_variants.sh) */
+#ifndef PAGODA_CTA_FENCE
+#define PAGODA_CTA_FENCE 0    /* executors release with a CTA-scope fence (the poster's GPU fence covers them) */
+#endif
+#ifndef PAGODA_CLAIM_FIRST
+#define PAGODA_CLAIM_FIRST 0  /* a scheduling round claims before it loads: fresh tickets load in the same round */
+#endif
+#ifndef PAGODA_CLAIM_SMALL
+#define PAGODA_CLAIM_SMALL 1  /* tickets per claim while the backlog is below what all MTBs could take */
 #endif
 
 namespace pagoda {
@@ -183,6 +190,20 @@ __device__ __forceinline__ void sc_add(MtbShared& S, int i, uint32_t v)
     if ((threadIdx.x & 31u) == 0) S.sctr[i] += v;
 }
 
+/* profiling builds: ns per scheduler phase (holder-private) and per executor step */
+#ifndef PAGODA_PROFILE
+#define PAGODA_PROFILE 0
+#endif
+enum { kPfFold = 0, kPfLoad, kPfPlace, kPfClaim, kPfSleep, kPfBody, kPfFence, kPfPost };
+__device__ __forceinline__ uint64_t pf_now() { return PAGODA_PROFILE ? globaltimer_ns() : 0; }
+__device__ __forceinline__ void pf_add(MtbShared& S, int i, uint64_t t0, bool shared_atomic)
+{
+    if (!PAGODA_PROFILE || (threadIdx.x & 31u) != 0) return;
+    const unsigned long long d = globaltimer_ns() - t0;
+    if (shared_atomic) atomicAdd(&S.sprof[i], d);
+    else S.sprof[i] += d;
+}
+
 /* ------------------------------------------------------------------ trace */
 __device__ __forceinline__ void trace_ev(const MkParams& p, int mtb, uint32_t& seq, uint8_t kind, uint64_t task_id,
                                          uint16_t tb, uint32_t mask, uint16_t goff, uint16_t glen, uint8_t bar)
@@ -339,13 +360,16 @@ __device__ __forceinline__ void run_task(MtbShared& S, char* smem_base, const Mk
     uint64_t t0 = 0;
     if (p.trace_cap) t0 = globaltimer_ns();
     TaskEnv env{&p.dctl->error, resident};
+    uint64_t tp = pf_now();
     if (!run_body(t.func_id, env, t.args) && lane == 0) atomicOr(&p.dctl->error, PAGODA_DEVERR_BAD_FUNC);
     __syncwarp();
+    pf_add(S, kPfBody, tp, true);
+    tp = pf_now();
     uint32_t last = 0;
     if (lane == 0) {
         /* this warp's global writes -> visible GPU-wide before anyone learns the warp is done
          * (release; the completion poster's system-scope fence then publishes them to the host) */
-#if PAGODA_TDES_VARIANT == 2
+#if PAGODA_CTA_FENCE
         /* CTA-scope release: the completion poster (same MTB) acquires it through the shared-memory
          * counters below and its GPU-scope fence then releases every warp's writes (cumulativity) */
         asm volatile("fence.acq_rel.cta;" ::: "memory");
@@ -371,7 +395,10 @@ __device__ __forceinline__ void run_task(MtbShared& S, char* smem_base, const Mk
             last = 1;
         }
     }
+    pf_add(S, kPfFence, tp, true);
+    tp = pf_now();
     if (__shfl_sync(0xffffffffu, last, 0)) post_completions(S, p);
+    pf_add(S, kPfPost, tp, true);
     if (lane == 0) {
         __threadfence_block();   /* TB / task frees are visible before the warp frees itself */
         atomicOr(&S.mb_warps, 1u << w);
@@ -861,7 +888,7 @@ __device__ int sched_claim(MtbShared& S, Sched& st, const MkParams& p)
         return 0;
     }
     const uint64_t backlog = tail - head;
-    if (backlog < (uint64_t)p.n_mtb * 8u) want = 1;
+    if (backlog < (uint64_t)p.n_mtb * 8u) want = min(want, (uint32_t)PAGODA_CLAIM_SMALL);
     const uint32_t k = (uint32_t)min((uint64_t)want, backlog);
     unsigned long long t0 = 0;
     if (lane == 0) t0 = atomicAdd(reinterpret_cast<unsigned long long*>(&p.dctl->head), (unsigned long long)k);
@@ -1020,8 +1047,18 @@ __device__ bool sched_fold(MtbShared& S, Sched& st, const MkParams& p, int mtb)
 __device__ bool sched_round(MtbShared& S, Sched& st, const MkParams& p, int mtb, bool& exit)
 {
     const uint32_t lane = threadIdx.x & 31u;
+    uint64_t t0 = pf_now();
     bool progress = sched_fold(S, st, p, mtb);
+    pf_add(S, kPfFold, t0, true);
+    if (PAGODA_CLAIM_FIRST) {
+        t0 = pf_now();
+        if (!S.no_tickets && sched_claim(S, st, p) > 0) progress = true;
+        pf_add(S, kPfClaim, t0, true);
+    }
+    t0 = pf_now();
     if (st.pl != st.pt && sched_load(S, st, p) > 0) progress = true;
+    pf_add(S, kPfLoad, t0, true);
+    t0 = pf_now();
     while (st.ph != st.pl) {
         if (!sched_place(S, st, p, mtb, S.pend[st.ph & 31u])) {
             sc_add(S, kScNoFit, 1);
@@ -1031,9 +1068,14 @@ __device__ bool sched_round(MtbShared& S, Sched& st, const MkParams& p, int mtb,
         st.ph++;
         progress = true;
     }
+    pf_add(S, kPfPlace, t0, true);
     /* MTB 0 (the I/O MTB: ingest, host stores) and the MTB sharing its SM take no tickets
      * unless MTB 0 is the only MTB (validation then caps every task to its capacity) */
-    if (!S.no_tickets && sched_claim(S, st, p) > 0) progress = true;
+    if (!PAGODA_CLAIM_FIRST) {
+        t0 = pf_now();
+        if (!S.no_tickets && sched_claim(S, st, p) > 0) progress = true;
+        pf_add(S, kPfClaim, t0, true);
+    }
     exit = false;
     sc_add(S, kScRounds, 1);
     if (progress) sc_add(S, kScProgress, 1);
@@ -1105,6 +1147,8 @@ __device__ __noinline__ bool holder_phase(MtbShared& S, const MkParams& p, int m
                 atomicAdd(&p.dctl->exited, 1u);
                 for (int i = 0; i < 8; i++)
                     atomicAdd(&p.dctl->ctr[PAGODA_CTR_SCHED_ROUNDS + i], (unsigned long long)S.sctr[i]);
+                if (PAGODA_PROFILE)   /* (executors still finishing their last task may add a little after) */
+                    for (int i = 0; i < 8; i++) atomicAdd(&p.dctl->ctr[PAGODA_CTR_SCHED_NS_FOLD + i], S.sprof[i]);
             }
             return true;
         }
@@ -1114,7 +1158,9 @@ __device__ __noinline__ bool holder_phase(MtbShared& S, const MkParams& p, int m
                 /* with work queued only shared-memory mailboxes are polled: stay responsive;
                  * otherwise the ring is polled in L2: back off */
                 backoff = (st.ph != st.pt) ? 32u : (backoff ? min(backoff * 2u, 1024u) : 32u);
+                const uint64_t t0 = pf_now();
                 __nanosleep(backoff);
+                pf_add(S, kPfSleep, t0, true);
             }
             continue;
         }
@@ -1238,6 +1284,7 @@ __global__ void __launch_bounds__(1024, kMinBlocks) master_kernel(MkParams p)
             S.ing_lock = 0;
             S.ing_pubs_done = 0;
             for (int i = 0; i < 8; i++) S.sctr[i] = 0;
+            for (int i = 0; i < 8; i++) S.sprof[i] = 0;
             asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         }
     }

@@ -42,7 +42,7 @@ struct HostCtl {
 };
 
 /* runtime counters, summed over the session (index = PAGODA_CTR_* in pagoda.h) */
-constexpr int kNumCounters = 16;
+constexpr int kNumCounters = 24;
 
 /* device memory, L2-resident: the device ring's counters */
 struct DevCtl {
@@ -188,6 +188,7 @@ struct MtbShared {
     uint32_t  ing_pubs_done;                /* publishers that saw their end marker */
     uint32_t  comp_pending;          /* task slots finished, completion record not yet posted */
     uint32_t  no_tickets;            /* this MTB runs no tasks (MTB 0 and the MTB sharing its SM) */
+    unsigned long long sprof[8];     /* PAGODA_PROFILE: ns per phase (PAGODA_CTR_SCHED_NS_FOLD + i) */
 };
 static_assert(offsetof(MtbShared, wt) == kWarpTableOffset, "WarpTable offset");
 static_assert(offsetof(MtbShared, stage_bar) == kStageBarOffset, "staging mbarriers offset");

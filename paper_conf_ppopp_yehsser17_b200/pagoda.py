@@ -218,11 +218,13 @@ class Pagoda:
 
     COUNTERS = ("ingest_batches", "ingest_entries", "ingest_ns_doorbell", "ingest_ns_copy", "ingest_ns_publish",
                 "ingest_ring_full", "sched_rounds", "sched_progress", "tickets", "claim_empty", "load_not_ready",
-                "placed", "place_nofit", "handoffs", "ingest_ns_fence", "ingest_ns_store")
+                "placed", "place_nofit", "handoffs", "ingest_ns_fence", "ingest_ns_store",
+                "sched_ns_fold", "sched_ns_load", "sched_ns_place", "sched_ns_claim", "sched_ns_sleep",
+                "exec_ns_body", "exec_ns_fence", "exec_ns_post")
 
     def counters(self) -> dict:
-        out = np.zeros(16, np.uint64)
-        _check(lib().pagoda_read_counters(self.h, _ptr(out), 16), "pagoda_read_counters")
+        out = np.zeros(len(self.COUNTERS), np.uint64)
+        _check(lib().pagoda_read_counters(self.h, _ptr(out), len(out)), "pagoda_read_counters")
         return {k: int(out[i]) for i, k in enumerate(self.COUNTERS)}
 
     def inflight_warps(self) -> int:

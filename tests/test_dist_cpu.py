@@ -61,3 +61,36 @@ def test_reference_arm_two_ranks():
     assert len(lines) == 1
     d = json.loads(lines[0])
     assert d["impl"] == "reference" and d["value"] > 0 and d["cpu_baseline"]["kind"] == "oracle"
+
+
+def _c5_worker(rank, world, port, q):
+    """Config 5's strong-scaling shard on each rank (host side: CPU buffers stand in
+    for device memory), and the whole-job task count bench.py reports."""
+    os.environ.update({"RANK": str(rank), "LOCAL_RANK": str(rank), "WORLD_SIZE": str(world),
+                       "MASTER_ADDR": "127.0.0.1", "MASTER_PORT": str(port)})
+    sys.path.insert(0, ROOT)
+    import bench
+    from paper_conf_ppopp_yehsser17_b200 import workloads as W
+    d = bench.Dist()
+    w = W.c5(10000, device="cpu", pool_size=64, shard=(d.rank, d.world))
+    total = d.sum(float(w.n))
+    q.put((rank, w.first, w.n, total, int(w.shapes[0, 4])))
+    import torch.distributed as dist
+    dist.destroy_process_group()
+
+
+def test_c5_strong_scaling_shards_two_ranks():
+    world, port = 2, _free_port()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_c5_worker, args=(r, world, port, q)) for r in range(world)]
+    [p.start() for p in procs]
+    [p.join(timeout=300) for p in procs]
+    assert all(p.exitcode == 0 for p in procs)
+    res = sorted(q.get(timeout=5) for _ in range(world))
+    assert [(r[1], r[2]) for r in res] == [(0, 5000), (5000, 5000)]   # disjoint, covering, contiguous
+    assert all(r[3] == 10000.0 for r in res)                          # the whole job's tasks on every rank
+    from paper_conf_ppopp_yehsser17_b200 import inputs as I
+    from paper_conf_ppopp_yehsser17_b200 import workloads as W
+    kinds = I.c5_schedule(10000)[0]
+    assert res[1][4] == W.KIND_FUNC[I.C5_KINDS[kinds[5000]]]          # rank 1 starts at global task 5000
