@@ -560,8 +560,16 @@ def roofline(workload, n, dev_ms, clk, peaks, w):
                           "hbm": (1e9, "GB/s", "hbm")}[r]
     achieved = tot[r] / (dev_ms * 1e-3) / scale
     pk = peak[r] / scale
+    traffic = None
+    try:   # DRAM bytes per launch of this workload's MasterKernel from a committed ncu --set full capture
+        tr = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json"))).get(workload)
+        if tr:
+            traffic = {"dram_bytes_per_launch": tr["dram_bytes_per_launch"],
+                       "algorithmic_hbm_bytes": tot["hbm"], "source": tr["source"]}
+    except (OSError, ValueError, KeyError):
+        pass
     return {"bound": bound, "resource": r, "achieved": achieved, "peak": pk, "unit": unit, "frac": achieved / pk,
-            "traffic": None, "roofline_us": {k: v * 1e6 for k, v in t_roof.items()},
+            "traffic": traffic, "roofline_us": {k: v * 1e6 for k, v in t_roof.items()},
             "per_unit": {"tdes": f"{TDES_LOOKUPS_PER_BLOCK} lookups and 16 B per 8-byte block",
                          **{k: v for k, v in DEMAND.items()}},
             "peak_from": f"fma: 148 SM x 128 lanes x {sm_mhz:.0f} MHz; lds: 148 x 32 lanes x {sm_mhz:.0f} MHz; "

@@ -303,6 +303,62 @@ __device__ __forceinline__ void tdes_blocks(const Env& e, const pagoda_tdes_args
     }
 }
 
+#ifndef PAGODA_TDES_PAIR
+#define PAGODA_TDES_PAIR 0
+#endif
+struct FirstBlockOnly {   /* makes tdes_blocks process block 0 of its args only */
+    __device__ __forceinline__ int getTid() const { return 0; }
+    __device__ __forceinline__ int getNumBlocks() const { return 1; }
+    __device__ __forceinline__ int getBlockWarps() const { return 1; }
+};
+/* Two blocks per loop trip (blocks b and b + T of this thread): one round-key load serves both,
+ * halving the key wavefronts, and the two rounds are independent chains.  Resident tables,
+ * keys in the TB's shared memory. */
+template <class Env>
+__device__ __forceinline__ void tdes_blocks_pair(const Env& e, const pagoda_tdes_args& a, uint32_t tb, uint32_t kb)
+{
+    const uint32_t T = (uint32_t)total_threads(e);
+    uint32_t blk = (uint32_t)e.getTid();
+    for (; blk + T < a.nblk; blk += 2u * T) {
+        const uint2 in0 = reinterpret_cast<const uint2*>(a.in)[blk];
+        const uint2 in1 = reinterpret_cast<const uint2*>(a.in)[blk + T];
+        uint32_t l0 = __byte_perm(in0.x, 0, 0x0123), r0 = __byte_perm(in0.y, 0, 0x0123);
+        uint32_t l1 = __byte_perm(in1.x, 0, 0x0123), r1 = __byte_perm(in1.y, 0, 0x0123);
+        tdes_ip(l0, r0);
+        tdes_ip(l1, r1);
+#pragma unroll 1
+        for (int st = 0; st < 3; st++) {
+            const uint32_t kst = kb + st * 128;
+#define PAGODA_TDES_ROUND2P(I)                                                                   \
+            {                                                                                    \
+                const uint4 k = tdes_key2<true, I>(kst, nullptr);                                \
+                uint32_t t0 = l0 ^ tdes_f<kTdesResident>(r0, k.x, k.y, tb, nullptr);             \
+                uint32_t t1 = l1 ^ tdes_f<kTdesResident>(r1, k.x, k.y, tb, nullptr);             \
+                l0 = r0; r0 = t0; l1 = r1; r1 = t1;                                              \
+                t0 = l0 ^ tdes_f<kTdesResident>(r0, k.z, k.w, tb, nullptr);                      \
+                t1 = l1 ^ tdes_f<kTdesResident>(r1, k.z, k.w, tb, nullptr);                      \
+                l0 = r0; r0 = t0; l1 = r1; r1 = t1;                                              \
+            }
+            PAGODA_TDES_ROUND2P(0) PAGODA_TDES_ROUND2P(2) PAGODA_TDES_ROUND2P(4) PAGODA_TDES_ROUND2P(6)
+            PAGODA_TDES_ROUND2P(8) PAGODA_TDES_ROUND2P(10) PAGODA_TDES_ROUND2P(12) PAGODA_TDES_ROUND2P(14)
+#undef PAGODA_TDES_ROUND2P
+            uint32_t t = l0; l0 = r0; r0 = t;
+            t = l1; l1 = r1; r1 = t;
+        }
+        tdes_fp(l0, r0);
+        tdes_fp(l1, r1);
+        reinterpret_cast<uint2*>(a.out)[blk] = make_uint2(__byte_perm(l0, 0, 0x0123), __byte_perm(r0, 0, 0x0123));
+        reinterpret_cast<uint2*>(a.out)[blk + T] = make_uint2(__byte_perm(l1, 0, 0x0123), __byte_perm(r1, 0, 0x0123));
+    }
+    if (blk < a.nblk) {   /* an odd block left: the single-block loop from it */
+        pagoda_tdes_args rest = a;
+        rest.in += blk;
+        rest.out += blk;
+        rest.nblk = 1;
+        tdes_blocks<kTdesResident, true>(FirstBlockOnly{}, rest, tb, kb);
+    }
+}
+
 template <class Env>
 __device__ void body_tdes(const Env& e, const pagoda_tdes_args& a)
 {
@@ -315,7 +371,8 @@ __device__ void body_tdes(const Env& e, const pagoda_tdes_args& a)
         e.syncBlock();
         sb = smem_u32(s);
     }
-    if (res && sb) tdes_blocks<kTdesResident, true>(e, a, lane_id() << 2, sb);
+    if (PAGODA_TDES_PAIR && res && sb) tdes_blocks_pair(e, a, lane_id() << 2, sb);
+    else if (res && sb) tdes_blocks<kTdesResident, true>(e, a, lane_id() << 2, sb);
     else if (res) tdes_blocks<kTdesResident, false>(e, a, lane_id() << 2, 0);
     else if (sb) tdes_blocks<kTdesShared, true>(e, a, sb, sb + 2048);
     else tdes_blocks<kTdesGlobal, false>(e, a, 0, 0);
