@@ -80,6 +80,7 @@ def parse():
     ap.add_argument("--mtbs", type=int, default=0, help="MTBs per SM (default: the workload preset)")
     ap.add_argument("--arena-kb", type=int, default=0, help="task arena per MTB in KiB (default: preset)")
     ap.add_argument("--no-resident", action="store_true", help="3DES: stage SP tables per task instead")
+    ap.add_argument("--no-const-keys", action="store_true", help="3DES: stage round keys per task instead")
     ap.add_argument("--prespawn", action="store_true",
                     help="spawn a step's tasks before launching a self-draining session (ncu-compatible)")
     return ap.parse_args()
@@ -404,6 +405,8 @@ def main():
         pp = PG.pingpong(dev, 2000) / 1e3
 
     p = PG.Pagoda(device=dev, **ctx_config(a, PG))
+    if use_resident(a) and w.tdes_tables and not a.no_const_keys:
+        p.tdes_register(w.tdes_tables)   # resident round keys (constant bank) for the resident SP tables
 
     def step():
         if a.prespawn:
@@ -504,7 +507,9 @@ def main():
                                                       "mtbs": info.n_mtb, "regs_per_thread": info.regs_per_thread,
                                                       "context": {k: v for k, v in ctx_config(a, PG).items()
                                                                   if k != "flags"} | {
-                                                          "resident_tdes_tables": use_resident(a)},
+                                                          "resident_tdes_tables": use_resident(a),
+                                                          "resident_tdes_keys": bool(use_resident(a) and w.tdes_tables
+                                                                                     and not a.no_const_keys)},
                                                       "task_shmem_bytes": int(w.shapes[0][2])},
             "gpu_launches": a.steps, "host_ms_per_step": 1e3 * host_total / a.steps,
             "host_tasks_per_s": all_tasks / host_total, "clocks": clk}

@@ -213,6 +213,15 @@ int64_t pagoda_trace_read_exec(pagoda_ctx* ctx, int mtb, int warp, void* dst, si
 #define PAGODA_TDES_TABLE_BYTES (2048 + 384 + 16384 + 16384)
 int pagoda_tdes_tables(const uint8_t key24[24], void* dst);
 
+/* Register a 3DES key schedule as resident task-class data (with
+ * PAGODA_RESIDENT_TDES): 3DES tasks whose `tables` pointer equals dev_tables
+ * (device memory written by pagoda_tdes_tables) take their 48 round keys from
+ * the MasterKernel's constant bank instead of staging them through shared
+ * memory.  One schedule per device and process; NULL unregisters.  Call while
+ * the context is stopped (NO_START or after pagoda_stop): -EBUSY otherwise.
+ * Returns 0, -EINVAL (unreadable pointer), -EBUSY, -EIO. */
+int pagoda_tdes_register(pagoda_ctx* ctx, const void* dev_tables);
+
 /* Naive baseline (the paper's CUDA-HyperQ): launch
  * each task as its own kernel <<<n_tb, threads, shmem>>> of the same body on
  * streams[i % n_streams] (n_streams <= 32), from the calling thread, then

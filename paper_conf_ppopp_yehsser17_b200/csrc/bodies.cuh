@@ -252,13 +252,26 @@ __device__ __forceinline__ uint32_t tdes_f(uint32_t r, uint32_t kx, uint32_t ky,
     }
 }
 
-/* round keys i, i+1 of the current stage: from the TB's shared memory (kKeysShared) or global */
-template <bool kKeysShared, int kI>
-__device__ __forceinline__ uint4 tdes_key2(uint32_t kb, const uint2* gk)
+/* A registered key schedule (pagoda_tdes_register): the 48 round keys in this
+ * module's constant bank, used by tasks whose tables pointer is the registered
+ * one, so the round keys come from the constant cache and not the shared-
+ * memory pipe the S-box lookups saturate.  Zero (never matching) in the
+ * baselines' translation units. */
+static __constant__ uint2 c_tdes_keys[48];
+static __constant__ unsigned long long c_tdes_tables;
+
+enum { kKeysGlobal = 0, kKeysShared = 1, kKeysConst = 2 };
+/* round keys i, i+1 of stage st: from the TB's shared memory (kb = its stage base), global
+ * (gk = the stage's keys) or the constant bank */
+template <int kKeys, int kI>
+__device__ __forceinline__ uint4 tdes_key2(uint32_t kb, const uint2* gk, int st)
 {
     uint4 k;
-    if (kKeysShared) {
+    if (kKeys == kKeysShared) {
         asm("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4+%5];" : "=r"(k.x), "=r"(k.y), "=r"(k.z), "=r"(k.w) : "r"(kb), "n"(kI * 8));
+    } else if (kKeys == kKeysConst) {
+        const uint2 a = c_tdes_keys[st * 16 + kI], b = c_tdes_keys[st * 16 + kI + 1];
+        k = make_uint4(a.x, a.y, b.x, b.y);
     } else {
         const uint2 a = __ldg(gk + kI), b = __ldg(gk + kI + 1);
         k = make_uint4(a.x, a.y, b.x, b.y);
@@ -266,7 +279,7 @@ __device__ __forceinline__ uint4 tdes_key2(uint32_t kb, const uint2* gk)
     return k;
 }
 
-template <int kMode, bool kKeysShared, class Env>
+template <int kMode, int kKeys, class Env>
 __device__ __forceinline__ void tdes_blocks(const Env& e, const pagoda_tdes_args& a, uint32_t tb, uint32_t kb)
 {
     const uint2* gkeys = reinterpret_cast<const uint2*>(a.tables + 512);
@@ -283,7 +296,7 @@ __device__ __forceinline__ void tdes_blocks(const Env& e, const pagoda_tdes_args
 /* two rounds per key load: one 16-byte shared load (one wavefront) for keys I, I+1 */
 #define PAGODA_TDES_ROUND2(I)                                                        \
             {                                                                        \
-                const uint4 k = tdes_key2<kKeysShared, I>(kst, gst);                 \
+                const uint4 k = tdes_key2<kKeys, I>(kst, gst, st);                   \
                 uint32_t t = l ^ tdes_f<kMode>(r, k.x, k.y, tb, a.tables);           \
                 l = r;                                                               \
                 r = t;                                                               \
@@ -314,7 +327,7 @@ struct FirstBlockOnly {   /* makes tdes_blocks process block 0 of its args only 
 /* Two blocks per loop trip (blocks b and b + T of this thread): one round-key load serves both,
  * halving the key wavefronts, and the two rounds are independent chains.  Resident tables,
  * keys in the TB's shared memory. */
-template <class Env>
+template <int kKeys, class Env>
 __device__ __forceinline__ void tdes_blocks_pair(const Env& e, const pagoda_tdes_args& a, uint32_t tb, uint32_t kb)
 {
     const uint32_t T = (uint32_t)total_threads(e);
@@ -331,7 +344,7 @@ __device__ __forceinline__ void tdes_blocks_pair(const Env& e, const pagoda_tdes
             const uint32_t kst = kb + st * 128;
 #define PAGODA_TDES_ROUND2P(I)                                                                   \
             {                                                                                    \
-                const uint4 k = tdes_key2<true, I>(kst, nullptr);                                \
+                const uint4 k = tdes_key2<kKeys, I>(kst, nullptr, st);                           \
                 uint32_t t0 = l0 ^ tdes_f<kTdesResident>(r0, k.x, k.y, tb, nullptr);             \
                 uint32_t t1 = l1 ^ tdes_f<kTdesResident>(r1, k.x, k.y, tb, nullptr);             \
                 l0 = r0; r0 = t0; l1 = r1; r1 = t1;                                              \
@@ -355,7 +368,7 @@ __device__ __forceinline__ void tdes_blocks_pair(const Env& e, const pagoda_tdes
         rest.in += blk;
         rest.out += blk;
         rest.nblk = 1;
-        tdes_blocks<kTdesResident, true>(FirstBlockOnly{}, rest, tb, kb);
+        tdes_blocks<kTdesResident, kKeys>(FirstBlockOnly{}, rest, tb, kb);
     }
 }
 
@@ -363,6 +376,11 @@ template <class Env>
 __device__ void body_tdes(const Env& e, const pagoda_tdes_args& a)
 {
     const uint32_t res = e.getResidentTdes();
+    if (res && (unsigned long long)a.tables == c_tdes_tables) {   /* resident tables, registered keys: */
+        if (PAGODA_TDES_PAIR) tdes_blocks_pair<kKeysConst>(e, a, lane_id() << 2, 0);   /* nothing to stage */
+        else tdes_blocks<kTdesResident, kKeysConst>(e, a, lane_id() << 2, 0);
+        return;
+    }
     const uint32_t need = res ? 384u : kTdesStageBytes;
     uint32_t sb = 0;
     if (e.getSMBytes() >= need && e.canSync()) {   /* stage round keys (and SP boxes) into the TB's shmem */
@@ -371,11 +389,11 @@ __device__ void body_tdes(const Env& e, const pagoda_tdes_args& a)
         e.syncBlock();
         sb = smem_u32(s);
     }
-    if (PAGODA_TDES_PAIR && res && sb) tdes_blocks_pair(e, a, lane_id() << 2, sb);
-    else if (res && sb) tdes_blocks<kTdesResident, true>(e, a, lane_id() << 2, sb);
-    else if (res) tdes_blocks<kTdesResident, false>(e, a, lane_id() << 2, 0);
-    else if (sb) tdes_blocks<kTdesShared, true>(e, a, sb, sb + 2048);
-    else tdes_blocks<kTdesGlobal, false>(e, a, 0, 0);
+    if (PAGODA_TDES_PAIR && res && sb) tdes_blocks_pair<kKeysShared>(e, a, lane_id() << 2, sb);
+    else if (res && sb) tdes_blocks<kTdesResident, kKeysShared>(e, a, lane_id() << 2, sb);
+    else if (res) tdes_blocks<kTdesResident, kKeysGlobal>(e, a, lane_id() << 2, 0);
+    else if (sb) tdes_blocks<kTdesShared, kKeysShared>(e, a, sb, sb + 2048);
+    else tdes_blocks<kTdesGlobal, kKeysGlobal>(e, a, 0, 0);
 }
 
 /* ------------------------------------------------------------- MM

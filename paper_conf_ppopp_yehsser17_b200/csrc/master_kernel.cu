@@ -1301,6 +1301,14 @@ __global__ void __launch_bounds__(1024, kMinBlocks) master_kernel(MkParams p)
 template __global__ void master_kernel<1>(MkParams);
 template __global__ void master_kernel<2>(MkParams);
 
+/* host side (runtime.cu): the registered 3DES key schedule of this module's MasterKernel */
+cudaError_t set_tdes_const_keys(const void* keys384, uint64_t tables_ptr)
+{
+    cudaError_t e = cudaMemcpyToSymbol(c_tdes_keys, keys384, sizeof(c_tdes_keys));
+    if (e == cudaSuccess) e = cudaMemcpyToSymbol(c_tdes_tables, &tables_ptr, sizeof(tables_ptr));
+    return e;
+}
+
 /* host-side launcher (called by runtime.cu) */
 cudaError_t launch_master(int mtbs_per_sm, int n_mtb, size_t smem_bytes, cudaStream_t stream, MkParams* params,
                           int* regs_out)

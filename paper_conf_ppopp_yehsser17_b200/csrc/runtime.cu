@@ -37,6 +37,7 @@
 namespace pagoda {
 cudaError_t launch_master(int mtbs_per_sm, int n_mtb, size_t smem_bytes, cudaStream_t stream, MkParams* params,
                           int* regs_out);
+cudaError_t set_tdes_const_keys(const void* keys384, uint64_t tables_ptr);
 }
 using namespace pagoda;
 
@@ -796,6 +797,24 @@ int64_t pagoda_inflight_warps(pagoda_ctx* c)
     const int64_t spawned = c->warps_spawned.load(std::memory_order_acquire);
     const int64_t done = l ? c->warps_prefix[(l - 1) & (c->C - 1)] : 0;
     return spawned - done;
+}
+
+int pagoda_tdes_register(pagoda_ctx* c, const void* dev_tables)
+{
+    if (!c) return -EINVAL;
+    if (c->running.load()) return -EBUSY;
+    cudaSetDevice(c->device);
+    uint8_t keys[384] = {0};
+    uint64_t ptr = 0;
+    if (dev_tables) {
+        if (cudaMemcpy(keys, static_cast<const uint8_t*>(dev_tables) + 2048, sizeof keys, cudaMemcpyDeviceToHost) !=
+            cudaSuccess) {
+            cudaGetLastError();
+            return -EINVAL;
+        }
+        ptr = (uint64_t)(uintptr_t)dev_tables;
+    }
+    return set_tdes_const_keys(keys, ptr) == cudaSuccess ? 0 : -EIO;
 }
 
 int pagoda_read_counters(pagoda_ctx* c, uint64_t* out, int n)

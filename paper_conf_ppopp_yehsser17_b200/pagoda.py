@@ -75,6 +75,7 @@ def lib() -> C.CDLL:
         L.pagoda_tdes_tables.argtypes = [P, P]
         L.pagoda_naive_run.argtypes = [I, I, P, P, SZ, SZ, I, C.POINTER(I64)]
         L.pagoda_pingpong.argtypes = [I, I, P]
+        L.pagoda_tdes_register.argtypes = [P, P]
         L.pagoda_fused_run.argtypes = [I, I, P, P, SZ, SZ, I, C.POINTER(I64), C.POINTER(C.c_float)]
         L.pagoda_pool_init.argtypes = [I, P, C.POINTER(pagoda_config), C.POINTER(P)]
         L.pagoda_pool_pick.argtypes = [P, I]
@@ -210,6 +211,10 @@ class Pagoda:
         _check(lib().pagoda_latency_loop(self.h, n, threads, n_tb, shmem, int(sync), func_id, b,
                                          len(b) if b else 0, _ptr(lat)), "pagoda_latency_loop")
         return lat
+
+    def tdes_register(self, dev_tables) -> int:
+        """Resident round keys for 3DES tasks using this tables pointer (context stopped)."""
+        return _check(lib().pagoda_tdes_register(self.h, dev_tables), "pagoda_tdes_register")
 
     def info(self) -> pagoda_info:
         i = pagoda_info()

@@ -41,6 +41,7 @@ class Workload:
         self.name, self.shapes, self.args, self.host = name, shapes, args, host
         self._outs, self._keep = outs, keep
         self.in_bytes, self.out_bytes = in_bytes, out_bytes   # algorithmic HBM bytes per run
+        self.tdes_tables = None   # device pointer of the 3DES tables its tasks use (pagoda_tdes_register)
 
     @property
     def n(self):
@@ -81,8 +82,10 @@ def tdes(n_tasks=32768, device="cuda", nbytes=4096, threads=128, shmem=2560, fir
     a["out"] = out.data_ptr() + np.arange(n_tasks) * nbytes
     a["tables"], a["nblk"] = tab.data_ptr(), nbytes // 8
     host = {"packets": pk, "key": I.TDES_KEYS}
-    return Workload("tdes", _shapes(n_tasks, threads, 1, shmem, True, T.TDES), T.to_raw(a), host,
-                    {"out": (out, np.uint8, (n_tasks, nbytes))}, [inp, out, tab], pk.nbytes, pk.nbytes)
+    w = Workload("tdes", _shapes(n_tasks, threads, 1, shmem, True, T.TDES), T.to_raw(a), host,
+                 {"out": (out, np.uint8, (n_tasks, nbytes))}, [inp, out, tab], pk.nbytes, pk.nbytes)
+    w.tdes_tables = tab.data_ptr()
+    return w
 
 
 # ---------------------------------------------------------------- config 3: MM
@@ -342,7 +345,10 @@ def pooled(name, pool: InputPool, kinds, in_idx, threads, shmem, device="cuda", 
         elif k == "dct":
             a["img"], a["coef"], a["out"] = d[0][j], d[1], out_ptr[i]
         raw[i] = T.to_raw(a)
-    return PooledWorkload(name, pool, kinds, in_idx, shapes, raw, buf, base[:-1], out_len, [buf] + pool.keep)
+    w = PooledWorkload(name, pool, kinds, in_idx, shapes, raw, buf, base[:-1], out_len, [buf] + pool.keep)
+    if "tdes" in pool.dev:
+        w.tdes_tables = pool.dev["tdes"][1]
+    return w
 
 
 def mpe(n_tasks=32768, device="cuda", resident=False, fill=None):

@@ -17,7 +17,7 @@ import pytest
 import oracle
 from paper_conf_ppopp_yehsser17_b200 import inputs as I
 from paper_conf_ppopp_yehsser17_b200 import workloads as W
-from paper_conf_ppopp_yehsser17_b200.pagoda import RESIDENT_TDES, Pagoda, naive_run
+from paper_conf_ppopp_yehsser17_b200.pagoda import NO_START, RESIDENT_TDES, Pagoda, naive_run
 
 pytestmark = pytest.mark.gpu
 
@@ -210,3 +210,45 @@ def test_static_fusion_parity():
     bad[3, 1] = 2   # multi-block tasks cannot be fused one block per task
     with pytest.raises(PagodaError):
         fused_run(0, bad, w.args, 256)
+
+
+# ---------------------------------------------------------------- 3DES with registered (constant-bank) round keys
+@pytest.mark.parametrize("threads", [128, 96, 32, 256])
+def test_tdes_registered_keys(threads):
+    """Resident SP tables + the registered key schedule: tasks using the
+    registered tables take no shared memory for keys; tasks with another
+    tables buffer (same key) still stage theirs; both bit-exact."""
+    w = W.tdes(64, shmem=512, threads=threads)
+    w2 = W.tdes(16, shmem=512, threads=threads, first=64)   # its own tables buffer: not registered
+    with Pagoda(flags=RESIDENT_TDES | NO_START, arena_bytes=40 * 1024) as p:
+        p.tdes_register(w.tdes_tables)
+        assert p.start() == 0
+        p.spawn_shapes(w.shapes, w.args)
+        p.spawn_shapes(w2.shapes, w2.args)
+        assert p.waitAll() == 0 and p.info().device_error == 0
+        assert p.stop() == 0
+        p.tdes_register(None)
+    for ww in (w, w2):
+        out = ww.outputs()["out"]
+        for k in range(ww.n):
+            assert np.array_equal(out[k], _tdes_ref(ww.host["packets"][k])), k
+
+
+def test_tdes_registered_keys_full_size():
+    from cryptography.hazmat.decrepit.ciphers.algorithms import TripleDES
+    from cryptography.hazmat.primitives.ciphers import Cipher, modes
+    w = W.tdes(32768, shmem=512)
+    with Pagoda(flags=RESIDENT_TDES | NO_START, arena_bytes=40 * 1024) as p:
+        p.tdes_register(w.tdes_tables)
+        assert p.start() == 0
+        p.spawn_shapes(w.shapes, w.args)
+        assert p.waitAll() == 0 and p.info().device_error == 0
+        assert p.stop() == 0
+        p.tdes_register(None)
+    out = w.outputs()["out"]
+    pk = w.host["packets"]
+    enc = Cipher(TripleDES(I.TDES_KEYS), modes.ECB()).encryptor()
+    ref = np.frombuffer(enc.update(pk.tobytes()) + enc.finalize(), np.uint8).reshape(pk.shape)
+    assert np.array_equal(out, ref)
+    for k in (0, 1, 16383, 32767):
+        assert np.array_equal(out[k], _tdes_ref(pk[k]))
