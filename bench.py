@@ -338,13 +338,13 @@ def make_workload(name, resident=False, d=None):
 PRESETS = {
     "tdes": {"mtbs_per_sm": 2, "arena_bytes": 40 * 1024, "resident": True},
     "mb": {"mtbs_per_sm": 2, "arena_bytes": 96 * 1024, "resident": False},
-    "mm": {"mtbs_per_sm": 2, "arena_bytes": 96 * 1024, "resident": False},
+    "mm": {"mtbs_per_sm": 4, "arena_bytes": 48 * 1024, "resident": False},   # 512-thread MTBs: 2x schedulers
     "mix": {"mtbs_per_sm": 1, "arena_bytes": 200 * 1024, "resident": False},
     "nop": {"mtbs_per_sm": 2, "arena_bytes": 96 * 1024, "resident": False},
     "c5": {"mtbs_per_sm": 1, "arena_bytes": 144 * 1024, "resident": True},
     "mpe": {"mtbs_per_sm": 2, "arena_bytes": 40 * 1024, "resident": True},
     "tdes_var": {"mtbs_per_sm": 2, "arena_bytes": 40 * 1024, "resident": True},
-    "mm_tc": {"mtbs_per_sm": 2, "arena_bytes": 96 * 1024, "resident": False},
+    "mm_tc": {"mtbs_per_sm": 4, "arena_bytes": 48 * 1024, "resident": False},
 }
 
 

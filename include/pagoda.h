@@ -46,12 +46,14 @@ typedef int64_t pagoda_task_t;          /* >= 0: task id; < 0: -errno */
 
 typedef struct {
     int      device;        /* CUDA device ordinal (default 0) */
-    int      mtbs_per_sm;   /* MasterKernel thread blocks (MTBs) per SM: 1 or 2 (default 2) */
+    int      mtbs_per_sm;   /* MasterKernel thread blocks (MTBs) per SM: 1 or 2 (1024 threads each; default 2,
+                               P:453-455) or 4 (512 threads each: twice the schedulers per SM; arena <= 48 KiB) */
     int      num_sms;       /* SMs to occupy, 0 = all (148 on B200) */
     uint32_t ring_entries;  /* TaskTable ring entries, host and device, power of 2 (default 65536) */
     uint32_t comp_entries;  /* completion window, power of 2 >= ring_entries (default 1<<20) */
     uint32_t arena_bytes;   /* shared-memory arena per MTB, multiple of 512 (default 96 KiB at 2 MTB/SM) */
-    uint32_t exec_warps;    /* worker warps per MTB, 1..32 (default 32; fewer = debug config) */
+    uint32_t exec_warps;    /* worker warps per MTB, 1..32, capped at the MTB's warps (default 32 = all;
+                               fewer = debug config) */
     uint32_t flags;         /* PAGODA_TRACE */
     uint32_t trace_events;  /* ledger capacity per MTB when PAGODA_TRACE (default 8192) */
     double   watchdog_s;    /* wait/waitAll/shutdown give up with -ETIMEDOUT after this many

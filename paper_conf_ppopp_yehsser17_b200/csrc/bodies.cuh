@@ -297,10 +297,10 @@ __device__ __forceinline__ void tdes_blocks(const Env& e, const pagoda_tdes_args
 #define PAGODA_TDES_ROUND2(I)                                                        \
             {                                                                        \
                 const uint4 k = tdes_key2<kKeys, I>(kst, gst, st);                   \
-                uint32_t t = l ^ tdes_f<kMode>(r, k.x, k.y, tb, a.tables);           \
+                uint32_t t = l ^ tdes_f<kMode>(r, k.x, k.y, tb, a.tables);      \
                 l = r;                                                               \
                 r = t;                                                               \
-                t = l ^ tdes_f<kMode>(r, k.z, k.w, tb, a.tables);                    \
+                t = l ^ tdes_f<kMode>(r, k.z, k.w, tb, a.tables);               \
                 l = r;                                                               \
                 r = t;                                                               \
             }
@@ -317,7 +317,7 @@ __device__ __forceinline__ void tdes_blocks(const Env& e, const pagoda_tdes_args
 }
 
 #ifndef PAGODA_TDES_PAIR
-#define PAGODA_TDES_PAIR 0
+#define PAGODA_TDES_PAIR 1
 #endif
 struct FirstBlockOnly {   /* makes tdes_blocks process block 0 of its args only */
     __device__ __forceinline__ int getTid() const { return 0; }
@@ -345,11 +345,11 @@ __device__ __forceinline__ void tdes_blocks_pair(const Env& e, const pagoda_tdes
 #define PAGODA_TDES_ROUND2P(I)                                                                   \
             {                                                                                    \
                 const uint4 k = tdes_key2<kKeys, I>(kst, nullptr, st);                           \
-                uint32_t t0 = l0 ^ tdes_f<kTdesResident>(r0, k.x, k.y, tb, nullptr);             \
-                uint32_t t1 = l1 ^ tdes_f<kTdesResident>(r1, k.x, k.y, tb, nullptr);             \
+                uint32_t t0 = l0 ^ tdes_f<kTdesResident>(r0, k.x, k.y, tb, nullptr);        \
+                uint32_t t1 = l1 ^ tdes_f<kTdesResident>(r1, k.x, k.y, tb, nullptr);        \
                 l0 = r0; r0 = t0; l1 = r1; r1 = t1;                                              \
-                t0 = l0 ^ tdes_f<kTdesResident>(r0, k.z, k.w, tb, nullptr);                      \
-                t1 = l1 ^ tdes_f<kTdesResident>(r1, k.z, k.w, tb, nullptr);                      \
+                t0 = l0 ^ tdes_f<kTdesResident>(r0, k.z, k.w, tb, nullptr);                 \
+                t1 = l1 ^ tdes_f<kTdesResident>(r1, k.z, k.w, tb, nullptr);                 \
                 l0 = r0; r0 = t0; l1 = r1; r1 = t1;                                              \
             }
             PAGODA_TDES_ROUND2P(0) PAGODA_TDES_ROUND2P(2) PAGODA_TDES_ROUND2P(4) PAGODA_TDES_ROUND2P(6)

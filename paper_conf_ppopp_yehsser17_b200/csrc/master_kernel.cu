@@ -1169,7 +1169,7 @@ __device__ __noinline__ bool holder_phase(MtbShared& S, const MkParams& p, int m
     }
 }
 
-/* Every worker warp runs this loop (warps 0..exec_warps-1; MTB 0's warp 31 ingests). */
+/* Every worker warp runs this loop (warps 0..exec_warps-1; MTB 0's last warp ingests). */
 __device__ void worker(MtbShared& S, char* smem_base, const MkParams& p, int mtb, int w, uint32_t resident,
                        uint32_t exec_mask, bool holder)
 {
@@ -1193,9 +1193,10 @@ __device__ void worker(MtbShared& S, char* smem_base, const MkParams& p, int mtb
 }
 
 /* ------------------------------------------------------------------ the kernel */
-template <int kMinBlocks>
-__global__ void __launch_bounds__(1024, kMinBlocks) master_kernel(MkParams p)
+template <int kMinBlocks, int kThreads>
+__global__ void __launch_bounds__(kThreads, kMinBlocks) master_kernel(MkParams p)
 {
+    constexpr int nw = kThreads / 32;   /* warps per MTB */
     extern __shared__ __align__(1024) unsigned char pagoda_mk_smem[];
     MtbShared& S = *reinterpret_cast<MtbShared*>(pagoda_mk_smem);
     char* smem_base = reinterpret_cast<char*>(pagoda_mk_smem);
@@ -1244,12 +1245,13 @@ __global__ void __launch_bounds__(1024, kMinBlocks) master_kernel(MkParams p)
         }
     }
     /* worker warps 0..exec_warps-1 (MTB 0: minus the ingest warp) */
-    uint32_t exec_mask = p.exec_warps >= 32 ? 0xffffffffu : ((1u << p.exec_warps) - 1u);
-    if (mtb == 0) exec_mask &= ~(1u << kIngestWarp);
+    const int ew = min(p.exec_warps, nw);
+    uint32_t exec_mask = ew >= 32 ? 0xffffffffu : ((1u << ew) - 1u);
+    if (mtb == 0) exec_mask &= ~(1u << ingest_loader_warp(nw));
     if (io)   /* the I/O roles: loader (31), host poster (30), forwarder (28), publishers (29, 27, ...) */
     {
-        exec_mask &= ~((1u << kHostPosterWarp) | (1u << kForwarderWarp));
-        for (uint32_t i = 0; i < kIngestPublishers; i++) exec_mask &= ~(1u << ingest_publisher_warp(i));
+        exec_mask &= ~((1u << host_poster_warp(nw)) | (1u << forwarder_warp(nw)));
+        for (uint32_t i = 0; i < kIngestPublishers; i++) exec_mask &= ~(1u << ingest_publisher_warp(i, nw));
     }
     const int first = __ffs(exec_mask) - 1;
     if (warp == 0) {
@@ -1289,17 +1291,18 @@ __global__ void __launch_bounds__(1024, kMinBlocks) master_kernel(MkParams p)
         }
     }
     __syncthreads();
-    if (mtb == 0 && p.n_mtb == 1 && warp == kIngestWarp) ingest(S, p, ingest_stage, S.ingest_bar);
-    else if (mtb == 0 && warp == kIngestWarp) ingest_loader(S, p, ingest_stage);
-    else if (io && ingest_publisher_index(warp) < kIngestPublishers)
-        ingest_publisher(S, p, ingest_stage, ingest_publisher_index(warp));
-    else if (mtb == 0 && warp == kHostPosterWarp) host_poster(S, p);
-    else if (mtb == 0 && warp == kForwarderWarp) comp_forwarder(S, p);
+    if (mtb == 0 && p.n_mtb == 1 && warp == ingest_loader_warp(nw)) ingest(S, p, ingest_stage, S.ingest_bar);
+    else if (mtb == 0 && warp == ingest_loader_warp(nw)) ingest_loader(S, p, ingest_stage);
+    else if (io && ingest_publisher_index(warp, nw) < kIngestPublishers)
+        ingest_publisher(S, p, ingest_stage, ingest_publisher_index(warp, nw));
+    else if (mtb == 0 && warp == host_poster_warp(nw)) host_poster(S, p);
+    else if (mtb == 0 && warp == forwarder_warp(nw)) comp_forwarder(S, p);
     else if ((exec_mask >> warp) & 1u) worker(S, smem_base, p, mtb, warp, resident, exec_mask, warp == first);
 }
 
-template __global__ void master_kernel<1>(MkParams);
-template __global__ void master_kernel<2>(MkParams);
+template __global__ void master_kernel<1, 1024>(MkParams);
+template __global__ void master_kernel<2, 1024>(MkParams);
+template __global__ void master_kernel<4, 512>(MkParams);   /* twice the MTBs (schedulers) per SM */
 
 /* host side (runtime.cu): the registered 3DES key schedule of this module's MasterKernel */
 cudaError_t set_tdes_const_keys(const void* keys384, uint64_t tables_ptr)
@@ -1313,18 +1316,20 @@ cudaError_t set_tdes_const_keys(const void* keys384, uint64_t tables_ptr)
 cudaError_t launch_master(int mtbs_per_sm, int n_mtb, size_t smem_bytes, cudaStream_t stream, MkParams* params,
                           int* regs_out)
 {
-    const void* fn = mtbs_per_sm == 2 ? reinterpret_cast<const void*>(&master_kernel<2>)
-                                      : reinterpret_cast<const void*>(&master_kernel<1>);
+    const void* fn = mtbs_per_sm == 4   ? reinterpret_cast<const void*>(&master_kernel<4, 512>)
+                     : mtbs_per_sm == 2 ? reinterpret_cast<const void*>(&master_kernel<2, 1024>)
+                                        : reinterpret_cast<const void*>(&master_kernel<1, 1024>);
+    const int threads = mtbs_per_sm == 4 ? 512 : 1024;
     cudaError_t err = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_bytes);
     if (err != cudaSuccess) return err;
     cudaFuncAttributes attr;
     if (cudaFuncGetAttributes(&attr, fn) == cudaSuccess && regs_out) *regs_out = attr.numRegs;
     int per_sm = 0;
-    err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, 1024, smem_bytes);
+    err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, threads, smem_bytes);
     if (err != cudaSuccess) return err;
     if (per_sm < mtbs_per_sm) return cudaErrorCooperativeLaunchTooLarge;
     void* args[] = {params};
-    return cudaLaunchCooperativeKernel(fn, dim3(n_mtb), dim3(1024), args, smem_bytes, stream);
+    return cudaLaunchCooperativeKernel(fn, dim3(n_mtb), dim3(threads), args, smem_bytes, stream);
 }
 
 } // namespace pagoda

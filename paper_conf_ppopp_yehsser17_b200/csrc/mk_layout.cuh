@@ -113,23 +113,27 @@ struct MkParams {
     uint32_t*    exec_count;  /* [n_mtb][32] */
 };
 
-constexpr int kIngestWarp = 31;          /* warp 31 of MTB 0 feeds the device ring */
-constexpr int kHostPosterWarp = 30;      /* warp 30 of MTB 0 (when n_mtb > 1): host-visible ingest stores */
-constexpr int kForwarderWarp = 28;       /* warp 28 of MTB 0 (when n_mtb > 1): completion records -> host */
-/* n_mtb > 1: kIngestPublishers publisher warps (29, 27, 26, ...) publish the loader's stages
- * round-robin, each double-buffered (kIngestStages = 2 x publishers), so their per-batch
- * latencies (cell checks, the bulk store, the release fence) overlap */
+/* MTB 0's I/O roles (n_mtb > 1), by position from its last warp (nw = warps per MTB: 32, or 16
+ * at 4 MTBs per SM): the loader (nw-1) feeds the device ring (alone it is the whole ingest when
+ * n_mtb == 1), the host poster (nw-2) makes the ingest's host-visible stores, the forwarder
+ * (nw-4) moves completion records to the host, and kIngestPublishers publisher warps (nw-3,
+ * nw-5, nw-6, ...) publish the loader's stages round-robin, each double-buffered
+ * (kIngestStages = 2 x publishers), so their per-batch latencies (cell checks, the bulk store,
+ * the release fence) overlap */
+__host__ __device__ constexpr int ingest_loader_warp(int nw) { return nw - 1; }
+__host__ __device__ constexpr int host_poster_warp(int nw) { return nw - 2; }
+__host__ __device__ constexpr int forwarder_warp(int nw) { return nw - 4; }
 #ifndef PAGODA_INGEST_PUBLISHERS
 #define PAGODA_INGEST_PUBLISHERS 2
 #endif
 constexpr uint32_t kIngestPublishers = PAGODA_INGEST_PUBLISHERS;
 constexpr uint32_t kIngestStages = 2u * kIngestPublishers;
 constexpr uint32_t kIngestFinSlots = 64;   /* >= kIngestStages: per-stage completion records */
-static_assert(kIngestPublishers >= 1 && kIngestPublishers <= 4, "publisher warps 29, 27, 26, 25");
-__host__ __device__ constexpr int ingest_publisher_warp(uint32_t i) { return i == 0 ? 29 : 28 - (int)i; }
-__host__ __device__ constexpr uint32_t ingest_publisher_index(int warp)   /* kIngestPublishers+ if none */
+static_assert(kIngestPublishers >= 1 && kIngestPublishers <= 4, "publisher warps nw-3, nw-5, nw-6, nw-7");
+__host__ __device__ constexpr int ingest_publisher_warp(uint32_t i, int nw) { return i == 0 ? nw - 3 : nw - 4 - (int)i; }
+__host__ __device__ constexpr uint32_t ingest_publisher_index(int warp, int nw)   /* kIngestPublishers+ if none */
 {
-    return warp == 29 ? 0u : (warp >= 25 && warp <= 27) ? (uint32_t)(28 - warp) : 99u;
+    return warp == nw - 3 ? 0u : (warp >= nw - 7 && warp <= nw - 5) ? (uint32_t)(nw - 4 - warp) : 99u;
 }
 constexpr uint32_t kDqEntries = 1u << 16;  /* device completion queue */
 /* ingest staging: 2 stages of MkParams::ingest_stage_entries entries (64 B each).  One MTB: lent

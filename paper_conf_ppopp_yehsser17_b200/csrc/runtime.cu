@@ -336,11 +336,13 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
     pagoda_config cfg;
     if (cfg_in) cfg = *cfg_in;
     else pagoda_config_default(&cfg);
-    if (cfg.mtbs_per_sm != 1 && cfg.mtbs_per_sm != 2) return -EINVAL;
+    if (cfg.mtbs_per_sm != 1 && cfg.mtbs_per_sm != 2 && cfg.mtbs_per_sm != 4) return -EINVAL;
+    const uint32_t block_warps = cfg.mtbs_per_sm == 4 ? 16u : 32u;   /* 4 MTBs/SM: 512-thread MTBs */
     if (!pow2(cfg.ring_entries) || !pow2(cfg.comp_entries) || cfg.comp_entries < cfg.ring_entries ||
         cfg.ring_entries < 2 * kSpawnChunk)
         return -EINVAL;
     if (cfg.exec_warps < 1 || cfg.exec_warps > 32) return -EINVAL;
+    cfg.exec_warps = std::min(cfg.exec_warps, block_warps);
     if (cfg.arena_bytes % PAGODA_GRANULE || cfg.arena_bytes / PAGODA_GRANULE > (uint32_t)kMaxGranules ||
         cfg.arena_bytes < 2u * 128u * 64u + 8u * PAGODA_GRANULE)   /* ingest staging + room for tasks */
         return -EINVAL;
@@ -371,7 +373,7 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
     c->C = cfg.comp_entries;
     const uint32_t arena_g = cfg.arena_bytes / PAGODA_GRANULE;
     if (c->n_mtb == 1) {   /* MTB 0 alone: it also hosts the ingest warp and its staging */
-        c->max_task_warps = cfg.exec_warps == 32 ? 31 : (int)cfg.exec_warps;
+        c->max_task_warps = cfg.exec_warps == block_warps ? (int)block_warps - 1 : (int)cfg.exec_warps;
         c->max_task_granules = arena_g - 2u * ingest_stage_entries(cfg.arena_bytes, 1) * 64u / PAGODA_GRANULE;
     } else {
         c->max_task_warps = (int)cfg.exec_warps;

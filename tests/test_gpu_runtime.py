@@ -362,3 +362,24 @@ def test_spread_task_parity_and_sync():
     for k in range(6):
         assert np.array_equal(out[k], O.tdes_ecb(td.host["packets"][k], I.TDES_KEYS))
     assert Dev.get(err, np.uint32)[0] == 0
+
+
+def test_four_mtbs_per_sm():
+    """512-thread MTBs, 4 per SM (twice the schedulers): 592 MTBs, 16 worker
+    warps each; a 1024-thread TB no longer fits one MTB (-EINVAL); 16-warp TBs
+    and tasks spread over MTBs still run exactly once; MM parity."""
+    import oracle
+    from paper_conf_ppopp_yehsser17_b200 import workloads as W
+    w = W.matmul(2000)
+    with Pagoda(mtbs_per_sm=4, arena_bytes=48 * 1024) as p:
+        i = p.info()
+        assert i.n_mtb == 592 and i.exec_warps == 16
+        assert p.taskSpawn(1024, 1, 0, 0, T.NOP) == -errno.EINVAL
+        ids = p.spawn_many(3000, 512, 1, 0, True, T.NOP, None, ids=True)
+        big = p.taskSpawn(128, 40, 0, 1, T.NOP)
+        p.spawn_shapes(w.shapes, w.args)
+        assert p.waitAll() == 0 and p.info().device_error == 0
+        assert all(p.check(int(x)) == 1 for x in ids[::101]) and p.check(big) == 1
+    out = w.outputs()["C"]
+    for k in range(0, 2000, 37):
+        assert np.array_equal(out[k], oracle.mm32(w.host["A"][k], w.host["B"][k])), k
