@@ -81,6 +81,8 @@ def parse():
     ap.add_argument("--arena-kb", type=int, default=0, help="task arena per MTB in KiB (default: preset)")
     ap.add_argument("--no-resident", action="store_true", help="3DES: stage SP tables per task instead")
     ap.add_argument("--no-const-keys", action="store_true", help="3DES: stage round keys per task instead")
+    ap.add_argument("--pool", action="store_true",
+                    help="one process drives every visible GPU through the least-loaded pool (no torchrun)")
     ap.add_argument("--prespawn", action="store_true",
                     help="spawn a step's tasks before launching a self-draining session (ncu-compatible)")
     return ap.parse_args()
@@ -312,25 +314,25 @@ CPU_SAMPLE = {"tdes": 16384, "mb": 1024, "mm": 65536, "mix": 4096, "nop": 16384,
               "tdes_var": 4096, "mm_tc": 65536}  # cpu_baseline sample
 
 
-def make_workload(name, resident=False, d=None):
+def make_workload(name, resident=False, d=None, device="cuda"):
     from paper_conf_ppopp_yehsser17_b200 import workloads as W
     if name == "c5":
-        return W.c5(1_000_000, resident=resident, shard=(d.rank, d.world) if d else (0, 1))
+        return W.c5(1_000_000, resident=resident, shard=(d.rank, d.world) if d else (0, 1), device=device)
     if name == "mpe":
-        return W.mpe(32768, resident=resident)
+        return W.mpe(32768, resident=resident, device=device)
     if name == "tdes_var":
-        return W.tdes_var(32768, resident=resident)
+        return W.tdes_var(32768, resident=resident, device=device)
     if name == "mm_tc":
         from paper_conf_ppopp_yehsser17_b200 import tasks as T
-        return W.matmul(65536, func=T.MM_TC)
+        return W.matmul(65536, func=T.MM_TC, device=device)
     if name == "tdes":   # with resident SP tables a task only stages its 384 B of round keys
-        return W.tdes(32768, shmem=512 if resident else 2560)
+        return W.tdes(32768, shmem=512 if resident else 2560, device=device)
     if name == "mb":
-        return W.mandelbrot(1024)
+        return W.mandelbrot(1024, device=device)
     if name == "mm":
-        return W.matmul(65536)
+        return W.matmul(65536, device=device)
     if name == "mix":
-        return W.mix(32768)
+        return W.mix(32768, device=device)
     return W.nop(200000)
 
 
@@ -361,11 +363,51 @@ def ctx_config(a, PG):
 
 
 # ----------------------------------------------------------------- main GPU leg
+def run_pool(a):
+    """--pool: SURVEY §8(e)'s in-process form — one context per GPU, the host spawner sends runs of
+    64 tasks to the GPU with the fewest in-flight warps (pagoda_pool_spawn_shapes).  Every device
+    holds the whole workload's inputs and outputs (a task may land anywhere).  A step = spawn the
+    whole workload + waitAll on every GPU, timed on the host (spawn-to-done, the metric's
+    definition; the MasterKernels stay resident across steps)."""
+    import torch
+    from paper_conf_ppopp_yehsser17_b200 import pagoda as PG
+    n_dev = a.gpus if a.gpus > 1 else torch.cuda.device_count()
+    ws = []
+    for i in range(n_dev):
+        torch.cuda.set_device(i)
+        ws.append(make_workload(a.workload, use_resident(a), device=f"cuda:{i}"))
+    cfg = ctx_config(a, PG)
+    cfg["flags"] &= ~PG.NO_START
+    pool = PG.Pool(range(n_dev), **cfg)
+    w0 = ws[0]
+    times, per_dev = [], np.zeros(n_dev, np.int64)
+    for it in range(a.warmup + a.steps):
+        t0 = time.perf_counter_ns()
+        _, dev = pool.spawn_shapes(w0.shapes, [w.args for w in ws])
+        assert pool.waitAll() == 0
+        if it >= a.warmup:
+            times.append((time.perf_counter_ns() - t0) * 1e-9)
+            per_dev += np.bincount(dev, minlength=n_dev)
+    assert pool.shutdown() == 0
+    tot = sum(times)
+    line = {"metric": BASE["metric"], "value": w0.n * a.steps / tot, "unit": "tasks/s", "n_gpus": n_dev,
+            "steps": a.steps, "warmup": a.warmup, "ms_per_step": 1e3 * tot / a.steps, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": DTYPE[a.workload], "data": "synthetic",
+            "config": workload_config(a.workload) | {
+                "parallelism": f"{n_dev} GPU(s), one process, least-loaded pool (runs of 64 tasks)"},
+            "tasks_per_gpu": per_dev.tolist(), "gpu_launches": n_dev,
+            "timing": "host CLOCK_MONOTONIC, spawn of the first task -> waitAll on every GPU"}
+    print(json.dumps(line), flush=True)
+
+
 def main():
     a = parse()
     d = Dist()
     if a.impl == "reference":
         run_reference(a, d)
+        return
+    if a.pool:
+        run_pool(a)
         return
     import torch
     from paper_conf_ppopp_yehsser17_b200 import pagoda as PG

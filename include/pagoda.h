@@ -260,6 +260,15 @@ int pagoda_pool_size(pagoda_pool* pool);
 pagoda_task_t pagoda_pool_spawn(pagoda_pool* pool, int threads, int n_threadblocks, int shmem_bytes,
                                 int sync_flag, int func_id, const void* const* args_per_dev,
                                 size_t args_bytes, int* index_out);
+/* Batched form: runs of up to `chunk` consecutive tasks (shapes as in
+ * pagoda_taskSpawnShapes) each go to the least-loaded context at the time of
+ * the pick; args_base_per_dev[i] + k * args_stride are task k's args if it
+ * lands on device i (device pointers of that device).  ids_out / dev_out
+ * (nullable) receive each task's id and device index.  Returns n or the first
+ * error. */
+int64_t pagoda_pool_spawn_shapes(pagoda_pool* pool, int n, const int32_t* shapes, const void* const* args_base_per_dev,
+                                 size_t args_stride, size_t args_bytes, int chunk, pagoda_task_t* ids_out,
+                                 int32_t* dev_out);
 int pagoda_pool_waitAll(pagoda_pool* pool);
 int pagoda_pool_shutdown(pagoda_pool* pool);
 

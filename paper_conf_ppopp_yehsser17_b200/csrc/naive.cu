@@ -19,6 +19,7 @@
 #include <time.h>
 
 #include <algorithm>
+#include <climits>
 #include <mutex>
 #include <vector>
 
@@ -218,6 +219,38 @@ extern "C" pagoda_task_t pagoda_pool_spawn(pagoda_pool* p, int threads, int n_tb
     }
     if (index_out) *index_out = i;
     return id;
+}
+
+/* Batched least-loaded spawning: runs of up to `chunk` tasks go
+ * to the context with the fewest in-flight warps at the time of the pick (each
+ * run one pagoda_taskSpawnShapes on that context, with that device's args). */
+extern "C" int64_t pagoda_pool_spawn_shapes(pagoda_pool* p, int n, const int32_t* shapes,
+                                            const void* const* args_base_per_dev, size_t args_stride,
+                                            size_t args_bytes, int chunk, pagoda_task_t* ids_out, int32_t* dev_out)
+{
+    if (!p || n < 0 || (n > 0 && !shapes) || chunk < 1) return -EINVAL;
+    for (int base = 0; base < n; base += chunk) {
+        const int m = std::min(chunk, n - base);
+        int64_t w = 0;
+        for (int i = 0; i < m; i++) {
+            const int32_t* s = shapes + 5 * (size_t)(base + i);
+            w += (int64_t)((s[0] + 31) / 32) * s[1];
+        }
+        const int d = pagoda_pool_pick(p, (int)std::min<int64_t>(w, INT32_MAX));
+        if (d < 0) return d;
+        const char* a = args_base_per_dev ? static_cast<const char*>(args_base_per_dev[d]) : nullptr;
+        const int64_t rc = pagoda_taskSpawnShapes(p->ctx[d], m, shapes + 5 * (size_t)base,
+                                                  a ? a + (size_t)base * args_stride : nullptr, args_stride, args_bytes,
+                                                  ids_out ? ids_out + base : nullptr);
+        {
+            std::lock_guard<std::mutex> lk(p->m);
+            p->pending[d] -= (int64_t)std::min<int64_t>(w, INT32_MAX);
+        }
+        if (rc < 0) return rc;
+        if (dev_out)
+            for (int i = 0; i < m; i++) dev_out[base + i] = d;
+    }
+    return n;
 }
 
 extern "C" int pagoda_pool_waitAll(pagoda_pool* p)

@@ -85,6 +85,8 @@ def lib() -> C.CDLL:
         L.pagoda_pool_spawn.argtypes = [P, I, I, I, I, I, P, SZ, C.POINTER(I)]
         L.pagoda_pool_spawn.restype = I64
         L.pagoda_pool_waitAll.argtypes = [P]
+        L.pagoda_pool_spawn_shapes.argtypes = [P, I, P, P, SZ, SZ, I, P, P]
+        L.pagoda_pool_spawn_shapes.restype = I64
         L.pagoda_pool_shutdown.argtypes = [P]
         L.pagoda_inflight_warps.argtypes = [P]
         L.pagoda_inflight_warps.restype = I64
@@ -329,6 +331,20 @@ class Pool:
         tid = lib().pagoda_pool_spawn(self.h, threads, n_tb, shmem, int(sync), func_id, arr, nbytes,
                                       C.byref(idx))
         return tid, idx.value
+
+    def spawn_shapes(self, shapes: np.ndarray, args_per_dev, chunk: int = 64):
+        """args_per_dev[i]: uint8 [n, 40] args valid on device i.  Returns (ids, dev) per task."""
+        shapes = np.ascontiguousarray(shapes, np.int32)
+        args_per_dev = [np.ascontiguousarray(a, np.uint8) for a in args_per_dev]
+        n = len(shapes)
+        ids, dev = np.empty(n, np.int64), np.empty(n, np.int32)
+        arr = (C.c_void_p * len(args_per_dev))(*[a.ctypes.data for a in args_per_dev])
+        _check(lib().pagoda_pool_spawn_shapes(self.h, n, _ptr(shapes), arr, 40, 40, chunk, _ptr(ids), _ptr(dev)),
+               "pagoda_pool_spawn_shapes")
+        return ids, dev
+
+    def ctx(self, i: int):
+        return lib().pagoda_pool_ctx(self.h, i)
 
     def waitAll(self) -> int:
         return lib().pagoda_pool_waitAll(self.h)

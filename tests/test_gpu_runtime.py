@@ -383,3 +383,32 @@ def test_four_mtbs_per_sm():
     out = w.outputs()["C"]
     for k in range(0, 2000, 37):
         assert np.array_equal(out[k], oracle.mm32(w.host["A"][k], w.host["B"][k])), k
+
+
+def test_pool_least_loaded_spawner():
+    """The in-process multi-GPU pool on the device(s) present:
+    single spawns and batched least-loaded spawns land, complete and compute
+    what the oracle does (config 5 tasks)."""
+    import oracle
+    import torch
+    from paper_conf_ppopp_yehsser17_b200 import workloads as W
+    from paper_conf_ppopp_yehsser17_b200.pagoda import Pool
+    n_dev = torch.cuda.device_count()
+    ws = [W.c5(3000, pool_size=32, device=f"cuda:{i}", fill=0xAB) for i in range(n_dev)]
+    pool = Pool(range(n_dev))
+    assert pool.pick(4) in range(n_dev)
+    tid, idx = pool.spawn(128, 1, 0, False, T.NOP, [b""] * n_dev)
+    assert tid >= 0 and idx in range(n_dev)
+    ids, dev = pool.spawn_shapes(ws[0].shapes, [w.args for w in ws])
+    assert pool.waitAll() == 0
+    assert (ids >= 0).all() and set(np.unique(dev)) <= set(range(n_dev))
+    assert pool.shutdown() == 0
+    for k in range(0, 3000, 97):
+        w = ws[int(dev[k])]
+        kind = w.kind(k)
+        args = w.pool.oracle_inputs(kind, int(w.in_idx[k]))
+        ref = {"mb": lambda *a: oracle.mandelbrot_tile(*a), "mm": oracle.mm32, "fb": oracle.filterbank,
+               "bf": oracle.beamformer, "conv": oracle.conv, "dct": oracle.dct,
+               "tdes": lambda pk: oracle.tdes_ecb(pk, __import__("paper_conf_ppopp_yehsser17_b200.inputs",
+                                                                  fromlist=["x"]).TDES_KEYS)}[kind](*args)
+        assert np.array_equal(w.task_output(k), ref), (kind, k)
