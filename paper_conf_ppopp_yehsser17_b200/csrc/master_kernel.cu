@@ -21,6 +21,9 @@
 #include "bodies.cuh"
 #include "mk_layout.cuh"
 /* A/B switches (scripts/build_variants.sh) */
+#ifndef PAGODA_IDLE_NS
+#define PAGODA_IDLE_NS 1024   /* longest back-off of an idle scheduler / I/O warp between polls */
+#endif
 #ifndef PAGODA_CTA_FENCE
 #define PAGODA_CTA_FENCE 0    /* executors release with a CTA-scope fence (the poster's GPU fence covers them) */
 #endif
@@ -328,7 +331,7 @@ __device__ void comp_forwarder(MtbShared& S, const MkParams& p)
             if (lane == 0) done = *(volatile uint32_t*)&p.dctl->exited >= (uint32_t)p.n_mtb &&
                                   *(volatile uint64_t*)&p.dctl->dq_tail == c;
             if (__shfl_sync(0xffffffffu, done, 0)) break;
-            __nanosleep(idle < 16 ? 64 : 512);
+            __nanosleep(idle < 16 ? 64 : min(512, PAGODA_IDLE_NS));
             idle++;
             continue;
         }
@@ -523,14 +526,15 @@ __device__ __forceinline__ bool ingest_publish(const MkParams& p, const char* sr
 
 /* doorbell: lane 0 reads the host's published count and terminate word */
 __device__ __forceinline__ void ingest_doorbell(const MkParams& p, uint64_t& pub, uint32_t& term, uint32_t& last_err,
-                                                bool post_err, IngestCtr& c)
+                                                bool post_err, IngestCtr& c, uint64_t fetched)
 {
     const uint32_t lane = threadIdx.x & 31u;
     const uint64_t t0 = globaltimer_ns();
     uint32_t err = 0;
     if (lane == 0) {
         pub = ld_acquire_sys(&p.hctl->published);
-        term = ld_relaxed_sys32(&p.hctl->terminate);
+        /* terminate matters only when nothing new was published: one PCIe round trip per poll otherwise */
+        term = pub > fetched ? 0u : ld_relaxed_sys32(&p.hctl->terminate);
         if (term) {   /* the host publishes every entry of the session before it sets terminate: */
             term = ld_acquire_sys32(&p.hctl->terminate);   /* re-read the count after an acquire of it */
             pub = ld_acquire_sys(&p.hctl->published);       /* (so this count is final) */
@@ -587,7 +591,7 @@ __device__ void ingest(MtbShared& S, const MkParams& p, char* stage_buf, uint64_
     IngestCtr c;
     for (;;) {
         if (fetched >= pub) {
-            ingest_doorbell(p, pub, term, last_err, true, c);
+            ingest_doorbell(p, pub, term, last_err, true, c, fetched);
             if (term == kStopAbort) {   /* host watchdog: abandon the queue, let idle MTBs exit */
                 if (lane == 0) st_release_gpu32(&p.dctl->stop, kStopAbort);
                 break;
@@ -619,7 +623,7 @@ __device__ void ingest(MtbShared& S, const MkParams& p, char* stage_buf, uint64_
             if (lane == 0) st_release_gpu32(&p.dctl->stop, 1u);
             break;
         } else if (++idle > 64) {
-            __nanosleep(256);
+            __nanosleep(min(256, PAGODA_IDLE_NS));
         }
     }
     if (lane == 0) {
@@ -652,7 +656,7 @@ __device__ void ingest_loader(MtbShared& S, const MkParams& p, char* stage_buf)
     IngestCtr c;
     for (;;) {
         if (fetched >= pub) {
-            ingest_doorbell(p, pub, term, last_err, false, c);
+            ingest_doorbell(p, pub, term, last_err, false, c, fetched);
             if (term == kStopAbort) {   /* host watchdog: the publishers see stop and leave too */
                 if (lane == 0) st_release_gpu32(&p.dctl->stop, kStopAbort);
                 break;
@@ -680,7 +684,7 @@ __device__ void ingest_loader(MtbShared& S, const MkParams& p, char* stage_buf)
             fetched += n;
             idle = 0;
         } else if (++idle > 64) {
-            __nanosleep(256);
+            __nanosleep(min(256, PAGODA_IDLE_NS));
         }
     }
     ingest_flush(p, c);
@@ -1157,7 +1161,7 @@ __device__ __noinline__ bool holder_phase(MtbShared& S, const MkParams& p, int m
             else {
                 /* with work queued only shared-memory mailboxes are polled: stay responsive;
                  * otherwise the ring is polled in L2: back off */
-                backoff = (st.ph != st.pt) ? 32u : (backoff ? min(backoff * 2u, 1024u) : 32u);
+                backoff = (st.ph != st.pt) ? 32u : (backoff ? min(backoff * 2u, (uint32_t)PAGODA_IDLE_NS) : 32u);
                 const uint64_t t0 = pf_now();
                 __nanosleep(backoff);
                 pf_add(S, kPfSleep, t0, true);
