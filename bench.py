@@ -79,6 +79,8 @@ def parse():
     ap.add_argument("--quick", action="store_true", help="skip everything but the timed steps (for ncu)")
     ap.add_argument("--mtbs", type=int, default=0, help="MTBs per SM (default: the workload preset)")
     ap.add_argument("--arena-kb", type=int, default=0, help="task arena per MTB in KiB (default: preset)")
+    ap.add_argument("--producers", type=int, default=0,
+                    help="host spawner threads per step (pagoda_taskSpawnShapesMT; default: preset)")
     ap.add_argument("--no-resident", action="store_true", help="3DES: stage SP tables per task instead")
     ap.add_argument("--no-const-keys", action="store_true", help="3DES: stage round keys per task instead")
     ap.add_argument("--pool", action="store_true",
@@ -342,7 +344,7 @@ PRESETS = {
     "mb": {"mtbs_per_sm": 2, "arena_bytes": 96 * 1024, "resident": False},
     "mm": {"mtbs_per_sm": 4, "arena_bytes": 48 * 1024, "resident": False},   # 512-thread MTBs: 2x schedulers
     "mix": {"mtbs_per_sm": 1, "arena_bytes": 200 * 1024, "resident": False},
-    "nop": {"mtbs_per_sm": 2, "arena_bytes": 96 * 1024, "resident": False},
+    "nop": {"mtbs_per_sm": 2, "arena_bytes": 96 * 1024, "resident": False, "producers": 2},
     "c5": {"mtbs_per_sm": 1, "arena_bytes": 144 * 1024, "resident": True},
     "mpe": {"mtbs_per_sm": 2, "arena_bytes": 40 * 1024, "resident": True},
     "tdes_var": {"mtbs_per_sm": 2, "arena_bytes": 40 * 1024, "resident": True},
@@ -450,13 +452,15 @@ def main():
     if use_resident(a) and w.tdes_tables and not a.no_const_keys:
         p.tdes_register(w.tdes_tables)   # resident round keys (constant bank) for the resident SP tables
 
+    producers = a.producers or PRESETS[a.workload].get("producers", 1)
+
     def step():
         if a.prespawn:
-            p.spawn_shapes(w.shapes, w.args)
+            p.spawn_shapes(w.shapes, w.args, producers=producers)
             assert p.start_drain() == 0
         else:
             assert p.start() == 0
-            p.spawn_shapes(w.shapes, w.args)
+            p.spawn_shapes(w.shapes, w.args, producers=producers)
         rc = p.stop()
         assert rc == 0, rc
 
@@ -546,7 +550,7 @@ def main():
             "dtype": DTYPE[a.workload],
             "data": "synthetic (seeded splitmix64 inputs, SURVEY §8(c) recipe)",
             "config": workload_config(a.workload) | {"parallelism": f"{d.world} GPU(s), one MasterKernel each",
-                                                      "mtbs": info.n_mtb, "regs_per_thread": info.regs_per_thread,
+                                                      "mtbs": info.n_mtb, "producers": producers, "regs_per_thread": info.regs_per_thread,
                                                       "context": {k: v for k, v in ctx_config(a, PG).items()
                                                                   if k != "flags"} | {
                                                           "resident_tdes_tables": use_resident(a),

@@ -128,6 +128,19 @@ int64_t pagoda_taskSpawnMany(pagoda_ctx* ctx, int n, int threads, int n_threadbl
 int64_t pagoda_taskSpawnShapes(pagoda_ctx* ctx, int n, const int32_t* shapes, const void* args_base,
                                size_t args_stride, size_t args_bytes, pagoda_task_t* ids_out);
 
+/* The same from n_producers host threads (Fig. 1a: several CPU
+ * threads spawn into one TaskTable): the calling thread and n_producers - 1
+ * helper threads the context starts on first use (kept until shutdown) each
+ * spawn every n_producers-th block of 256 consecutive tasks.  Every task is
+ * validated before any is spawned (-EINVAL spawns nothing).  ids_out[i] is task
+ * i's id; ids are not in workload order across blocks.  One multi-producer call
+ * runs at a time per context (others wait); plain taskSpawn calls may run
+ * concurrently.  1 <= n_producers <= PAGODA_MAX_PRODUCERS.  Returns n or the
+ * first error (tasks of other blocks may have been spawned by then). */
+#define PAGODA_MAX_PRODUCERS 8
+int64_t pagoda_taskSpawnShapesMT(pagoda_ctx* ctx, int n, const int32_t* shapes, const void* args_base,
+                                 size_t args_stride, size_t args_bytes, pagoda_task_t* ids_out, int n_producers);
+
 /* ---- MasterKernel sessions ------------------------------------------------
  * pagoda_init starts a session.  pagoda_stop waits for every issued task,
  * asks the MasterKernel to drain and exit, and waits for it (the ring, the

@@ -30,6 +30,15 @@
 #ifndef PAGODA_CLAIM_FIRST
 #define PAGODA_CLAIM_FIRST 0  /* a scheduling round claims before it loads: fresh tickets load in the same round */
 #endif
+#ifndef PAGODA_CELL_ACQ
+#define PAGODA_CELL_ACQ 1     /* ring cells are read with acquire loads and handed back with relaxed stores */
+#endif
+#ifndef PAGODA_LOOKAHEAD
+#define PAGODA_LOOKAHEAD 1    /* tickets claimed beyond what the free warps fit now */
+#endif
+#ifndef PAGODA_CLAIM_MIN
+#define PAGODA_CLAIM_MIN 1    /* with tickets queued, claim only when at least this many are wanted */
+#endif
 #ifndef PAGODA_CLAIM_SMALL
 #define PAGODA_CLAIM_SMALL 1  /* tickets per claim while the backlog is below what all MTBs could take */
 #endif
@@ -875,8 +884,10 @@ __device__ int sched_claim(MtbShared& S, Sched& st, const MkParams& p)
     uint32_t want;
     if (st.est_w == 0) want = queued == 0 ? 1u : 0u;
     else {   /* what fits now, plus one task of lookahead so the next is loaded when warps free */
-        want = (uint32_t)__popc(st.free_w) / st.est_w + 1u;
+        want = (uint32_t)__popc(st.free_w) / st.est_w + (uint32_t)PAGODA_LOOKAHEAD;
         want = want > queued ? want - queued : 0u;
+        /* hysteresis: refill the queue in batches (one fetch-add and one load round per batch) */
+        if (queued && want < (uint32_t)PAGODA_CLAIM_MIN) want = 0;
     }
     want = min(want, cap);
     if (want == 0) return 0;
@@ -923,7 +934,29 @@ __device__ int sched_load(MtbShared& S, Sched& st, const MkParams& p)
         sc_add(S, kScLoadNotReady, 1);
         return 0;
     }
-    for (uint32_t c = lane; c < r * 4u; c += 32u) {
+#if PAGODA_CELL_ACQ
+    /* lane i copies cell i whole with acquire loads (LDG.STRONG.GPU + L1 invalidate, no MEMBAR),
+     * so its own hand-back store below is ordered after every read of the cell in program order.
+     * (A st.release would be a MEMBAR.GPU, which waits for every memory operation in flight on
+     * the SM: the holder's largest single cost per scheduling round.) */
+    uint32_t used = 0;
+    if (lane < r) {
+        const uint32_t slot = nth_set_bit(st.free_task, lane);
+        const int4* src = reinterpret_cast<const int4*>(p.dring + (t & p.ring_mask));
+        int4* dst = reinterpret_cast<int4*>(&S.tasks[slot]);
+#pragma unroll
+        for (int q = 0; q < 4; q++) {
+            int4 v;
+            asm volatile("ld.acquire.gpu.global.v4.s32 {%0,%1,%2,%3}, [%4];"
+                         : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(src + q) : "memory");
+            dst[q] = v;
+        }
+        S.pend[(st.pl + lane) & 31u] = (uint8_t)slot;
+        st_relaxed_gpu32(&p.dseq[t & p.ring_mask], (uint32_t)(t + (uint64_t)p.ring_mask + 1));
+        used = 1u << slot;
+    }
+#else
+    for (uint32_t c = lane; c < r * 4u; c += 32u) {   /* 4 lanes per cell, coalesced */
         const uint32_t i = c >> 2;
         const uint64_t ti = S.pend_ticket[(st.pl + i) & 31u];
         const int4 v = __ldcg(reinterpret_cast<const int4*>(p.dring + (ti & p.ring_mask)) + (c & 3u));
@@ -937,6 +970,7 @@ __device__ int sched_load(MtbShared& S, Sched& st, const MkParams& p)
         st_release_gpu32(&p.dseq[t & p.ring_mask], (uint32_t)(t + (uint64_t)p.ring_mask + 1));
         used = 1u << slot;
     }
+#endif
     used = __reduce_or_sync(0xffffffffu, used);
     st.free_task &= ~used;
     st.pl += r;

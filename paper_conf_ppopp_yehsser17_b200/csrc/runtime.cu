@@ -75,6 +75,21 @@ struct pagoda_ctx {
     std::atomic<int> faulted{0};
     std::vector<int64_t> warps_prefix;      /* warps_prefix[id mod C] = sum of warps of tasks <= id */
     std::atomic<int64_t> warps_spawned{0};
+    /* helper producer threads of pagoda_taskSpawnShapesMT (Fig. 1a: several CPU threads
+     * spawn into the TaskTable), started on first use and kept until shutdown */
+    struct SpawnJob {
+        const int32_t* shapes;
+        const char* args;
+        size_t stride, bytes;
+        pagoda_task_t* ids;
+        int n, P;
+    } job{};
+    std::vector<std::thread> helpers;
+    std::mutex mt_mtx;                      /* one multi-producer spawn at a time */
+    std::atomic<uint64_t> job_gen{0};
+    std::atomic<int> job_left{0};
+    std::atomic<int64_t> job_rc{0};
+    std::atomic<int> helpers_quit{0};
     /* MasterKernel session */
     MkParams params;
     size_t smem = 0;
@@ -312,6 +327,8 @@ static int stop_kernel(pagoda_ctx* c, bool abort_now = false)
 static void free_ctx(pagoda_ctx* c)
 {
     if (!c) return;
+    c->helpers_quit.store(1, std::memory_order_release);
+    for (auto& t : c->helpers) t.join();
     if (c->hctl) cudaFreeHost(c->hctl);
     if (c->hring) cudaFreeHost(c->hring);
     if (c->comp) cudaFreeHost((void*)c->comp);
@@ -603,7 +620,83 @@ static int64_t spawn_batch(pagoda_ctx* c, int n, ShapeOf shape_of, const void* a
     return n;
 }
 
+/* Multi-producer spawn: the workload is cut into blocks of kMtBlock tasks and
+ * block b is spawned by producer b mod P (the caller is producer 0), each
+ * through spawn_batch.  Entries are written in parallel; publication stays in
+ * id order (a chunk is published once every lower id is), so the GPU sees one
+ * contiguous TaskTable exactly as with one producer. */
+static const int kMtBlock = 4 * kSpawnChunk;
+
+static int64_t spawn_part(pagoda_ctx* c, const pagoda_ctx::SpawnJob& j, int t)
+{
+    for (int b0 = t * kMtBlock; b0 < j.n; b0 += j.P * kMtBlock) {
+        const int m = std::min(kMtBlock, j.n - b0);
+        const int32_t* sh = j.shapes + 5 * (size_t)b0;
+        const int64_t rc = spawn_batch(c, m, [&](int i) { return sh + 5 * (size_t)i; },
+                                       j.bytes ? j.args + (size_t)b0 * j.stride : nullptr, j.stride, j.bytes,
+                                       j.ids ? j.ids + b0 : nullptr);
+        if (rc < 0) return rc;
+    }
+    return 0;
+}
+
+static void helper_main(pagoda_ctx* c, int t)
+{
+    uint64_t seen = 0;
+    uint64_t idle = 0;
+    for (;;) {
+        const uint64_t g = c->job_gen.load(std::memory_order_acquire);
+        if (g != seen) {
+            seen = g;
+            idle = 0;
+            const pagoda_ctx::SpawnJob j = c->job;
+            if (t < j.P) {
+                const int64_t rc = spawn_part(c, j, t);
+                if (rc < 0) {
+                    int64_t z = 0;
+                    c->job_rc.compare_exchange_strong(z, rc);
+                }
+                c->job_left.fetch_sub(1, std::memory_order_acq_rel);
+            }
+            continue;
+        }
+        if (c->helpers_quit.load(std::memory_order_acquire)) return;
+        /* spin while jobs are likely to follow (back-to-back steps), then sleep */
+        if (++idle < (1u << 16)) _mm_pause();
+        else std::this_thread::sleep_for(std::chrono::microseconds(idle < (1u << 20) ? 2 : 50));
+    }
+}
+
 extern "C" {
+
+int64_t pagoda_taskSpawnShapesMT(pagoda_ctx* c, int n, const int32_t* shapes, const void* args_base,
+                                 size_t args_stride, size_t args_bytes, pagoda_task_t* ids_out, int n_producers)
+{
+    if (!c || n < 0 || (!shapes && n > 0) || n_producers < 1 || n_producers > PAGODA_MAX_PRODUCERS) return -EINVAL;
+    if (args_bytes > PAGODA_ARGS_MAX || (args_bytes > 0 && !args_base)) return -EINVAL;
+    const int P = std::min(n_producers, std::max(1, (n + kMtBlock - 1) / kMtBlock));
+    if (P == 1)
+        return spawn_batch(c, n, [&](int i) { return shapes + 5 * (size_t)i; }, args_base, args_stride, args_bytes,
+                           ids_out);
+    std::lock_guard<std::mutex> lk(c->mt_mtx);
+    ShapeMemo memo;   /* validate everything first: a rejected workload spawns nothing */
+    for (int i = 0; i < n; i++) {
+        Split sp;
+        if (int rc = memo.check(c, shapes + 5 * (size_t)i, sp)) return rc;
+    }
+    while ((int)c->helpers.size() < P - 1) {
+        const int t = (int)c->helpers.size() + 1;
+        c->helpers.emplace_back(helper_main, c, t);
+    }
+    c->job = pagoda_ctx::SpawnJob{shapes, static_cast<const char*>(args_base), args_stride, args_bytes, ids_out, n, P};
+    c->job_rc.store(0);
+    c->job_left.store(P - 1, std::memory_order_release);
+    c->job_gen.fetch_add(1, std::memory_order_acq_rel);
+    const int64_t rc0 = spawn_part(c, c->job, 0);
+    while (c->job_left.load(std::memory_order_acquire) > 0) _mm_pause();
+    const int64_t rc = rc0 < 0 ? rc0 : c->job_rc.load();
+    return rc < 0 ? rc : n;
+}
 
 int64_t pagoda_taskSpawnMany(pagoda_ctx* c, int n, int threads, int n_tb, int shmem_bytes, int sync_flag, int func_id,
                              const void* args_base, size_t args_stride, size_t args_bytes, pagoda_task_t* ids_out)

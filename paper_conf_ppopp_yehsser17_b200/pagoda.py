@@ -67,6 +67,8 @@ def lib() -> C.CDLL:
         L.pagoda_taskSpawnMany.restype = I64
         L.pagoda_taskSpawnShapes.argtypes = [P, I, P, P, SZ, SZ, P]
         L.pagoda_taskSpawnShapes.restype = I64
+        L.pagoda_taskSpawnShapesMT.argtypes = [P, I, P, P, SZ, SZ, P, I]
+        L.pagoda_taskSpawnShapesMT.restype = I64
         L.pagoda_get_info.argtypes = [P, C.POINTER(pagoda_info)]
         L.pagoda_trace_read.argtypes = [P, I, P, SZ]
         L.pagoda_trace_read.restype = I64
@@ -170,15 +172,21 @@ class Pagoda:
         _check(rc, "pagoda_taskSpawnMany")
         return out
 
-    def spawn_shapes(self, shapes: np.ndarray, args: np.ndarray, ids=False):
-        """shapes: int32 [n,5] = threads, n_tb, shmem, sync, func_id; args: uint8 [n,40]."""
+    def spawn_shapes(self, shapes: np.ndarray, args: np.ndarray, ids=False, producers: int = 1):
+        """shapes: int32 [n,5] = threads, n_tb, shmem, sync, func_id; args: uint8 [n,40].
+        producers > 1: pagoda_taskSpawnShapesMT (that many host threads)."""
         shapes = np.ascontiguousarray(shapes, np.int32)
         args = np.ascontiguousarray(args, np.uint8)
         n = len(shapes)
         out = np.empty(n, np.int64) if ids else None
-        rc = lib().pagoda_taskSpawnShapes(self.h, n, _ptr(shapes), _ptr(args), args.shape[1], args.shape[1],
-                                          _ptr(out))
-        _check(rc, "pagoda_taskSpawnShapes")
+        if producers > 1:
+            rc = lib().pagoda_taskSpawnShapesMT(self.h, n, _ptr(shapes), _ptr(args), args.shape[1], args.shape[1],
+                                                _ptr(out), producers)
+            _check(rc, "pagoda_taskSpawnShapesMT")
+        else:
+            rc = lib().pagoda_taskSpawnShapes(self.h, n, _ptr(shapes), _ptr(args), args.shape[1], args.shape[1],
+                                              _ptr(out))
+            _check(rc, "pagoda_taskSpawnShapes")
         return out
 
     # --- sessions ------------------------------------------------------------

@@ -41,19 +41,25 @@ def run(w, **cfg):
 
 
 # ---------------------------------------------------------------- MB (config 1)
-def test_mandelbrot_config1_bit_exact():
+# 2 MTBs/SM: the one-pixel body (32 registers); 1 MTB/SM: the two-pixel body (64 registers, bench preset)
+MB_CFGS = [{}, {"mtbs_per_sm": 1, "arena_bytes": 96 * 1024}]
+
+
+@pytest.mark.parametrize("cfg", MB_CFGS)
+def test_mandelbrot_config1_bit_exact(cfg):
     w = W.mandelbrot(1024)
-    out = run(w)["out"]
+    out = run(w, **cfg)["out"]
     for k in range(1024):
         ref = oracle.mandelbrot_tile(int(w.host["tx"][k]), int(w.host["ty"][k]))
         assert np.array_equal(out[k], ref), k
     assert int(out.astype(np.int64).sum()) == 199370695
 
 
+@pytest.mark.parametrize("cfg", MB_CFGS)
 @pytest.mark.parametrize("threads", [32, 100, 992])
-def test_mandelbrot_other_thread_counts(threads):
+def test_mandelbrot_other_thread_counts(threads, cfg):
     w = W.mandelbrot(96, threads=threads)
-    out = run(w)["out"]
+    out = run(w, **cfg)["out"]
     for k in range(0, 96, 7):
         assert np.array_equal(out[k], oracle.mandelbrot_tile(int(w.host["tx"][k]), int(w.host["ty"][k])))
 
@@ -203,6 +209,11 @@ def test_static_fusion_parity():
     out = w.outputs()["out"]
     for k in range(40):
         assert np.array_equal(out[k], _tdes_ref(w.host["packets"][k]))
+    w = W.mandelbrot(64)
+    fused_run(0, w.shapes, w.args, 256)
+    out = w.outputs()["out"]
+    for k in range(64):
+        assert np.array_equal(out[k], oracle.mandelbrot_tile(int(w.host["tx"][k]), int(w.host["ty"][k])))
     w = W.matmul(50)
     fused_run(0, w.shapes, w.args, 256)
     _mm_check(w, w.outputs()["C"], range(50))

@@ -171,6 +171,37 @@ def test_multi_producer_ids_unique():
         assert allids == list(range(n_thr * per))              # unique across producers
 
 
+@pytest.mark.parametrize("producers", [2, 3, 8])
+def test_spawn_shapes_multi_producer_exactly_once(producers):
+    """pagoda_taskSpawnShapesMT: several host threads spawn one workload (blocks of 256
+    tasks, block b by producer b mod P) across a ring wrap: every task runs exactly once
+    with its own args, the ids are a permutation of the range, and a bad shape anywhere
+    rejects the whole call before anything is spawned."""
+    n = 70000 + 123                                   # > ring entries (2^16): producers wait for slots
+    dev = Dev()
+    cnt = dev.zeros(n * 4)
+    shapes = np.zeros((n, 5), np.int32)
+    shapes[:, 0] = np.where(np.arange(n) % 3 == 0, 64, 32)
+    shapes[:, 1] = 1
+    shapes[:, 4] = T.MARK
+    a = T.records(T.MARK, n)
+    out = dev.zeros(64 * 4)
+    a["out"], a["base"], a["tag"] = ptr(out), 0, 1
+    a["cnt"] = ptr(cnt) + 4 * np.arange(n)
+    with Pagoda() as p:
+        bad = shapes.copy()
+        bad[n - 1, 4] = 999
+        with pytest.raises(OSError):
+            p.spawn_shapes(bad, T.to_raw(a), producers=producers)
+        assert p.info().completed_low == 0 and p.waitAll() == 0
+        ids = p.spawn_shapes(shapes, T.to_raw(a), ids=True, producers=producers)
+        assert p.waitAll() == 0
+        assert np.array_equal(np.sort(ids), np.arange(n))
+        assert all(p.check(int(i)) == 1 for i in ids[::1001])
+    c = Dev.get(cnt, np.uint32)
+    assert np.array_equal(c, shapes[:, 0].astype(np.uint32))   # each task's threads ran once
+
+
 def test_ring_wraparound_and_completion_window():
     """More tasks than ring entries and completion slots: slots are reused only
     after their previous occupant is consumed / done."""
