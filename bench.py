@@ -341,7 +341,7 @@ def make_workload(name, resident=False, d=None, device="cuda"):
 # per-workload context presets
 PRESETS = {
     "tdes": {"mtbs_per_sm": 2, "arena_bytes": 40 * 1024, "resident": True},
-    "mb": {"mtbs_per_sm": 2, "arena_bytes": 96 * 1024, "resident": False},
+    "mb": {"mtbs_per_sm": 2, "arena_bytes": 96 * 1024, "resident": False, "spread": True},
     "mm": {"mtbs_per_sm": 4, "arena_bytes": 48 * 1024, "resident": False},   # 512-thread MTBs: 2x schedulers
     "mix": {"mtbs_per_sm": 1, "arena_bytes": 200 * 1024, "resident": False},
     "nop": {"mtbs_per_sm": 2, "arena_bytes": 96 * 1024, "resident": False, "producers": 2},
@@ -358,7 +358,7 @@ def use_resident(a):
 
 def ctx_config(a, PG):
     pr = PRESETS[a.workload]
-    cfg = {"flags": PG.NO_START | (PG.RESIDENT_TDES if use_resident(a) else 0),
+    cfg = {"flags": PG.NO_START | (PG.RESIDENT_TDES if use_resident(a) else 0) | (PG.SPREAD if pr.get("spread") else 0),
            "mtbs_per_sm": a.mtbs or pr["mtbs_per_sm"],
            "arena_bytes": (a.arena_kb * 1024) if a.arena_kb else pr["arena_bytes"]}
     return cfg
@@ -554,6 +554,7 @@ def main():
                                                       "context": {k: v for k, v in ctx_config(a, PG).items()
                                                                   if k != "flags"} | {
                                                           "resident_tdes_tables": use_resident(a),
+                                                          "spread_first_claims": bool(PRESETS[a.workload].get("spread")),
                                                           "resident_tdes_keys": bool(use_resident(a) and w.tdes_tables
                                                                                      and not a.no_const_keys)},
                                                       "task_shmem_bytes": int(w.shapes[0][2])},

@@ -43,6 +43,11 @@ typedef int64_t pagoda_task_t;          /* >= 0: task id; < 0: -errno */
 #define PAGODA_NO_START      0x2u /* pagoda_init allocates but does not launch; call pagoda_start(_drain) */
 #define PAGODA_RESIDENT_TDES 0x4u /* keep 64 KiB of lane-replicated 3DES S-box tables resident in every MTB
                                      (conflict-free lookups; the arena starts after them) */
+#define PAGODA_SPREAD        0x10u /* spread-first claims: while the ring backlog is small, an MTB running
+                                      tasks claims the next one later the more warps it has busy (6 us per
+                                      4 warps), so few, uneven tasks (config 1) go to the idlest MTBs */
+#define PAGODA_LIFECYCLE     0x8u /* stamp every task's life cycle on the GPU clock (profiling; 64 B per
+                                     completion slot): see pagoda_lifecycle_read */
 
 typedef struct {
     int      device;        /* CUDA device ordinal (default 0) */
@@ -220,6 +225,17 @@ int64_t pagoda_trace_read(pagoda_ctx* ctx, int mtb, void* dst, size_t cap);
  * {u64 task_id; u16 tb; u16 smid; u16 mtb; u16 warp; u64 t_start_ns; u64 t_end_ns} (32 B).
  * Copies up to cap records of (mtb, warp) into dst; returns the count. */
 int64_t pagoda_trace_read_exec(pagoda_ctx* ctx, int mtb, int warp, void* dst, size_t cap);
+
+/* Task life cycle (PAGODA_LIFECYCLE): for task ids [first, first + n) copy 8 u64
+ * %globaltimer stamps each (ns; 0 = not seen) into dst (host memory), in order:
+ * [0] published into the device ring (ingest), [1] loaded into an MTB's task
+ * slot (claim + load done), [2] placed (warps/granules/barrier assigned,
+ * executors released), [3] first warp starts the body, [4] last warp ends the
+ * body, [5] last warp's completion fence done, [6] completion record queued
+ * (device queue, or the host window with one MTB), [7] record forwarded to
+ * the host window.  Slots are indexed id mod comp_entries and zeroed at each
+ * pagoda_start.  Returns n, -EINVAL or -ENODATA (flag not set). */
+int64_t pagoda_lifecycle_read(pagoda_ctx* ctx, uint64_t first, size_t n, uint64_t* dst);
 
 /* Host-side preparation of the 3DES task's device tables:
  * writes PAGODA_TDES_TABLE_BYTES bytes to dst (HOST memory) for the EDE3 key

@@ -39,6 +39,15 @@
 #ifndef PAGODA_CLAIM_MIN
 #define PAGODA_CLAIM_MIN 1    /* with tickets queued, claim only when at least this many are wanted */
 #endif
+#ifndef PAGODA_FUSED_CLAIM
+#define PAGODA_FUSED_CLAIM 0  /* claim, tail/head reads and publication checks in one round trip */
+#endif
+#ifndef PAGODA_CLAIM_FAIR
+#define PAGODA_CLAIM_FAIR 0   /* claims take at most max(CLAIM_SMALL, backlog / n_mtb) tickets */
+#endif
+#ifndef PAGODA_SMALL_MULT
+#define PAGODA_SMALL_MULT 8   /* (not FAIR) backlog below n_mtb x this: CLAIM_SMALL tickets per claim */
+#endif
 #ifndef PAGODA_CLAIM_SMALL
 #define PAGODA_CLAIM_SMALL 1  /* tickets per claim while the backlog is below what all MTBs could take */
 #endif
@@ -216,6 +225,16 @@ __device__ __forceinline__ void pf_add(MtbShared& S, int i, uint64_t t0, bool sh
     else S.sprof[i] += d;
 }
 
+/* ------------------------------------------------------------------ life cycle stamps (PAGODA_LIFECYCLE) */
+__device__ __forceinline__ uint64_t* life_slot(const MkParams& p, uint64_t id, int ev)
+{
+    return p.life + ((id & p.comp_mask) * 8u + (uint32_t)ev);
+}
+__device__ __forceinline__ void life_stamp(const MkParams& p, uint64_t id, int ev)
+{
+    if (p.life) *life_slot(p, id, ev) = globaltimer_ns();
+}
+
 /* ------------------------------------------------------------------ trace */
 __device__ __forceinline__ void trace_ev(const MkParams& p, int mtb, uint32_t& seq, uint8_t kind, uint64_t task_id,
                                          uint16_t tb, uint32_t mask, uint16_t goff, uint16_t glen, uint8_t bar)
@@ -276,18 +295,30 @@ __device__ __forceinline__ void post_completions(MtbShared& S, const MkParams& p
             if (p.n_mtb == 1) {
                 asm volatile("fence.acq_rel.sys;" ::: "memory");
                 if (mine) st_relaxed_sys(reinterpret_cast<volatile uint64_t*>(&p.comp[id & p.comp_mask]), id);
+                if (mine) life_stamp(p, id, kLifeQueued);
             } else {
+                /* queue positions below dq_safe were cleared by the forwarders (their cursors, read
+                 * by an acquire below when a position reaches the horizon) */
+                const uint64_t safe = *(volatile unsigned long long*)&S.dq_safe;
                 fence_acq_rel_gpu();   /* release: the tasks' writes (fenced by each of their warps) */
                 const uint32_t pm = __ballot_sync(0xffffffffu, mine);
                 unsigned long long base = 0;
                 if (lane == 0 && pm) base = atomicAdd(reinterpret_cast<unsigned long long*>(&p.dctl->dq_tail),
                                                       (unsigned long long)__popc(pm));
                 base = __shfl_sync(0xffffffffu, base, 0);
+                const uint64_t slot = base + (uint64_t)__popc(pm & ((1u << lane) - 1u));
+                if (__any_sync(0xffffffffu, mine && slot >= safe)) {   /* refresh the horizon */
+                    uint64_t m = 0;
+                    m = lane < p.n_fwd ? ld_acquire_gpu(&p.dctl->fwd_cur[lane]) : ~0ull;
+                    for (uint32_t o = 1; o < kForwarders; o <<= 1) m = min(m, __shfl_xor_sync(0xffffffffu, m, o));
+                    if (lane == 0) atomicMax(&S.dq_safe, (unsigned long long)(m + kDqEntries));
+                }
                 if (mine) {
-                    const uint64_t slot = base + (uint64_t)__popc(pm & ((1u << lane) - 1u));
                     uint64_t* q = &p.dq[slot & p.dq_mask];
-                    while (*(volatile uint64_t*)q != 0) __nanosleep(64);   /* previous lap not forwarded yet */
+                    if (slot >= safe)
+                        while (*(volatile uint64_t*)q != 0) __nanosleep(64);   /* previous lap not forwarded yet */
                     st_relaxed_gpu(q, id + 1);
+                    life_stamp(p, id, kLifeQueued);
                 }
             }
             __syncwarp();
@@ -306,39 +337,53 @@ __device__ __forceinline__ void post_completions(MtbShared& S, const MkParams& p
     }
 }
 
-/* MTB 0's forwarder (n_mtb > 1): the completion queue in order -> the host's
- * completion window.  Per sweep: find the run of filled records (up to 1024),
+/* MTB 0's forwarders (n_mtb > 1): completion queue -> the host's completion
+ * window.  Forwarder f owns the queue chunks (kFwdChunk records) whose index
+ * is f mod kForwarders and walks them in order.  Per sweep: the run of filled
+ * records at its cursor (up to the chunk's end, 8 loads per lane in flight),
  * one system-scope fence (cumulative: orders the task writes the posters
- * released), then post the records and clear their queue slots.  Exits once
- * every MTB exited and the queue is drained. */
-__device__ void comp_forwarder(MtbShared& S, const MkParams& p)
+ * released), then post the records and clear their queue slots.  The fence of
+ * the NEXT sweep also orders those clears before the cursor's publication
+ * (fwd_cur, the posters' wrap check).  Each exits once every MTB exited and
+ * no record is left at or past its cursor; the last one out records where the
+ * next session resumes. */
+__device__ void comp_forwarder(MtbShared& S, const MkParams& p, uint32_t f)
 {
     const uint32_t lane = threadIdx.x & 31u;
+    const uint64_t K = p.n_fwd, CH = kFwdChunk;
     uint64_t c = *(volatile uint64_t*)&p.dctl->dq_head;
+    {   /* first position >= c in a chunk of mine */
+        const uint64_t ch = c / CH, o = (f + K - ch % K) % K;
+        if (o) c = (ch + o) * CH;
+    }
+    uint64_t published = ~0ull;
     uint32_t idle = 0;
     for (;;) {
-        uint32_t n = 0;   /* the run of filled records at c, c+1, ... (8 loads per lane in flight) */
+        const uint32_t span = (uint32_t)((c / CH + 1) * CH - c);   /* records left in this chunk */
+        uint64_t v[8];
+#pragma unroll
+        for (int i = 0; i < 8; i++) {
+            const uint32_t k = (uint32_t)i * 32u + lane;
+            v[i] = k < span ? *(volatile uint64_t*)&p.dq[(c + k) & p.dq_mask] : 0;
+        }
+        uint32_t n = 0;
         bool gap = false;
-        for (int trip = 0; trip < 4 && !gap; trip++) {
-            uint64_t v[8];
 #pragma unroll
-            for (int i = 0; i < 8; i++) v[i] = *(volatile uint64_t*)&p.dq[(c + n + (uint32_t)i * 32u + lane) & p.dq_mask];
-#pragma unroll
-            for (int i = 0; i < 8; i++) {
-                const uint32_t full = __ballot_sync(0xffffffffu, v[i] != 0);
-                if (!gap) {
-                    if (full == 0xffffffffu) n += 32u;
-                    else {
-                        n += (uint32_t)__ffs(~full) - 1u;
-                        gap = true;
-                    }
+        for (int i = 0; i < 8; i++) {
+            const uint32_t full = __ballot_sync(0xffffffffu, v[i] != 0);
+            if (!gap) {
+                if (full == 0xffffffffu) n += 32u;
+                else {
+                    n += (uint32_t)__ffs(~full) - 1u;
+                    gap = true;
                 }
             }
         }
+        n = min(n, span);
         if (n == 0) {
             uint32_t done = 0;
             if (lane == 0) done = *(volatile uint32_t*)&p.dctl->exited >= (uint32_t)p.n_mtb &&
-                                  *(volatile uint64_t*)&p.dctl->dq_tail == c;
+                                  *(volatile uint64_t*)&p.dctl->dq_tail <= c;
             if (__shfl_sync(0xffffffffu, done, 0)) break;
             __nanosleep(idle < 16 ? 64 : min(512, PAGODA_IDLE_NS));
             idle++;
@@ -346,16 +391,30 @@ __device__ void comp_forwarder(MtbShared& S, const MkParams& p)
         }
         idle = 0;
         asm volatile("fence.acq_rel.sys;" ::: "memory");
-        for (uint32_t i = lane; i < n; i += 32u) {
-            uint64_t* q = &p.dq[(c + i) & p.dq_mask];
-            const uint64_t id = *(volatile uint64_t*)q - 1;
-            st_relaxed_sys(reinterpret_cast<volatile uint64_t*>(&p.comp[id & p.comp_mask]), id);
-            st_relaxed_gpu(q, 0);
+        if (lane == 0 && published != c) {   /* the previous sweeps' clears are ordered before this */
+            st_relaxed_gpu(&p.dctl->fwd_cur[f], c);
+            published = c;
+        }
+#pragma unroll
+        for (int i = 0; i < 8; i++) {
+            const uint32_t k = (uint32_t)i * 32u + lane;
+            if (k < n) {
+                const uint64_t id = v[i] - 1;
+                st_relaxed_sys(reinterpret_cast<volatile uint64_t*>(&p.comp[id & p.comp_mask]), id);
+                life_stamp(p, id, kLifeFwd);
+                st_relaxed_gpu(&p.dq[(c + k) & p.dq_mask], 0);
+            }
         }
         __syncwarp();
         c += n;
+        if (n == span) c += (K - 1) * CH;   /* chunk done: my next one */
     }
-    if (lane == 0) *(volatile uint64_t*)&p.dctl->dq_head = c;
+    if (lane == 0 && atomicAdd(&S.fwd_done, 1u) + 1u == (uint32_t)K) {
+        /* every record below the final tail was forwarded: the next session resumes there */
+        const uint64_t t = *(volatile uint64_t*)&p.dctl->dq_tail;
+        *(volatile uint64_t*)&p.dctl->dq_head = t;
+        for (uint32_t i = 0; i < 4; i++) *(volatile uint64_t*)&p.dctl->fwd_cur[i] = t;
+    }
 }
 
 /* ------------------------------------------------------------------ task execution
@@ -372,10 +431,16 @@ __device__ __forceinline__ void run_task(MtbShared& S, char* smem_base, const Mk
     uint64_t t0 = 0;
     if (p.trace_cap) t0 = globaltimer_ns();
     TaskEnv env{&p.dctl->error, resident};
+    if (p.life && lane == 0)   /* the first warp to start stamps the body start */
+        atomicCAS(reinterpret_cast<unsigned long long*>(life_slot(p, s.task_id, kLifeStart)), 0ull,
+                  (unsigned long long)globaltimer_ns());
     uint64_t tp = pf_now();
     if (!run_body(t.func_id, env, t.args) && lane == 0) atomicOr(&p.dctl->error, PAGODA_DEVERR_BAD_FUNC);
     __syncwarp();
     pf_add(S, kPfBody, tp, true);
+    if (p.life && lane == 0)
+        atomicMax(reinterpret_cast<unsigned long long*>(life_slot(p, s.task_id, kLifeEnd)),
+                  (unsigned long long)globaltimer_ns());
     tp = pf_now();
     uint32_t last = 0;
     if (lane == 0) {
@@ -402,6 +467,7 @@ __device__ __forceinline__ void run_task(MtbShared& S, char* smem_base, const Mk
         if (atomicSub(&S.tb_warps_left[s.tbslot], 1u) == 1u) atomicOr(&S.mb_tbs, 1u << s.tbslot);
         if (atomicSub(&S.task_warps_left[s.task], 1u) == 1u) {
             /* last warp of the task (Alg. 1 L41-42): its completion record is pending */
+            life_stamp(p, s.task_id, kLifeDone);
             atomicOr(&S.comp_pending, 1u << s.task);
             __threadfence_block();   /* pending bit before the poster-flag attempt */
             last = 1;
@@ -524,6 +590,7 @@ __device__ __forceinline__ bool ingest_publish(const MkParams& p, const char* sr
     for (uint32_t i = lane; i < n; i += 32u) {
         const uint64_t t = s + i;
         st_relaxed_gpu32(&p.dseq[t & p.ring_mask], (uint32_t)(t + 1));
+        if (p.life) life_stamp(p, reinterpret_cast<const TaskEntry*>(src)[i].id, kLifePub);
     }
     __syncwarp();
     /* hint for schedulers that work exists (publishers finish out of order: the max) */
@@ -867,6 +934,7 @@ __device__ bool sched_place(MtbShared& S, Sched& st, const MkParams& p, int mtb,
         }
         all |= m;
     }
+    if (lane == 0 && !group) life_stamp(p, id, kLifePlace);
     __syncwarp();   /* counters written by lane 0 happen-before every lane's release-arrive */
     if ((all >> lane) & 1u) mbar_arrive(&S.exec_bar[lane]);   /* Alg. 2 L14: exec <- 1 */
     return true;
@@ -903,7 +971,21 @@ __device__ int sched_claim(MtbShared& S, Sched& st, const MkParams& p)
         return 0;
     }
     const uint64_t backlog = tail - head;
-    if (backlog < (uint64_t)p.n_mtb * 8u) want = min(want, (uint32_t)PAGODA_CLAIM_SMALL);
+    if (p.spread_ns && backlog < (uint64_t)p.n_mtb * PAGODA_SMALL_MULT) {
+        /* PAGODA_SPREAD, small backlog: a busier MTB claims later (its busy warps / 4 + 1 times
+         * spread_ns after its last claim), so tasks go to the least-loaded MTBs first */
+        const uint32_t busy = (uint32_t)__popc(st.exec_mask & ~st.free_w);
+        const uint64_t now = globaltimer_ns();
+        if (busy && now < S.claim_after) return 0;
+        if (lane == 0) S.claim_after = now + (uint64_t)(busy + 4u) * p.spread_ns / 4u;
+    }
+#if PAGODA_CLAIM_FAIR
+    /* at most a fair share of the backlog per claim: spreads consecutive tasks over MTBs when
+     * the backlog is small, takes batches (one fetch-add and one load round) when it is not */
+    want = min(want, max((uint32_t)PAGODA_CLAIM_SMALL, (uint32_t)min(backlog / (uint64_t)p.n_mtb, (uint64_t)32)));
+#else
+    if (backlog < (uint64_t)p.n_mtb * PAGODA_SMALL_MULT) want = min(want, (uint32_t)PAGODA_CLAIM_SMALL);
+#endif
     const uint32_t k = (uint32_t)min((uint64_t)want, backlog);
     unsigned long long t0 = 0;
     if (lane == 0) t0 = atomicAdd(reinterpret_cast<unsigned long long*>(&p.dctl->head), (unsigned long long)k);
@@ -915,6 +997,8 @@ __device__ int sched_claim(MtbShared& S, Sched& st, const MkParams& p)
     return (int)k;
 }
 
+__device__ int sched_copy(MtbShared& S, Sched& st, const MkParams& p, uint32_t r);
+
 /* Load the published tickets at the front of the FIFO into free task slots,
  * then hand their cells back to the producer (seq = t + R). */
 __device__ int sched_load(MtbShared& S, Sched& st, const MkParams& p)
@@ -922,10 +1006,9 @@ __device__ int sched_load(MtbShared& S, Sched& st, const MkParams& p)
     const uint32_t lane = threadIdx.x & 31u;
     const uint32_t n = min(st.pt - st.pl, (uint32_t)__popc(st.free_task));
     if (n == 0) return 0;
-    uint64_t t = 0;
     bool ready = false;
     if (lane < n) {
-        t = S.pend_ticket[(st.pl + lane) & 31u];
+        const uint64_t t = S.pend_ticket[(st.pl + lane) & 31u];
         ready = ld_acquire_gpu32(&p.dseq[t & p.ring_mask]) == (uint32_t)(t + 1);
     }
     const uint32_t nr = __ballot_sync(0xffffffffu, !ready);
@@ -934,6 +1017,15 @@ __device__ int sched_load(MtbShared& S, Sched& st, const MkParams& p)
         sc_add(S, kScLoadNotReady, 1);
         return 0;
     }
+    return sched_copy(S, st, p, r);
+}
+
+/* Copy the first r tickets of the FIFO (published: their cells' sequence words
+ * were acquired) into free task slots and hand the cells back. */
+__device__ int sched_copy(MtbShared& S, Sched& st, const MkParams& p, uint32_t r)
+{
+    const uint32_t lane = threadIdx.x & 31u;
+    const uint64_t t = lane < r ? S.pend_ticket[(st.pl + lane) & 31u] : 0;
 #if PAGODA_CELL_ACQ
     /* lane i copies cell i whole with acquire loads (LDG.STRONG.GPU + L1 invalidate, no MEMBAR),
      * so its own hand-back store below is ordered after every read of the cell in program order.
@@ -953,6 +1045,7 @@ __device__ int sched_load(MtbShared& S, Sched& st, const MkParams& p)
         }
         S.pend[(st.pl + lane) & 31u] = (uint8_t)slot;
         st_relaxed_gpu32(&p.dseq[t & p.ring_mask], (uint32_t)(t + (uint64_t)p.ring_mask + 1));
+        if (p.life && !(S.tasks[slot].flags & kEntryGroup)) life_stamp(p, S.tasks[slot].id, kLifeLoad);
         used = 1u << slot;
     }
 #else
@@ -979,6 +1072,63 @@ __device__ int sched_load(MtbShared& S, Sched& st, const MkParams& p)
     st.est_w = (uint32_t)last.warps_tb * last.n_tb;
     return (int)r;
 }
+
+#if PAGODA_FUSED_CLAIM
+/* One L2 round trip for all of a round's questions to the device ring: lane 0
+ * takes new tickets (fetch-add on the head), lanes 1-2 read the tail and the
+ * head, lanes 3.. acquire the sequence words of up to 29 tickets claimed in
+ * earlier rounds.  The claim size comes from the backlog seen last time (a
+ * fair share of it per MTB), and an MTB that holds no tickets keeps ONE
+ * standing reservation even when the ring is empty: the next task published
+ * at that position is its own (consecutive tasks land on different MTBs).
+ * Reserved positions past the final tail are void at stop (head = tail).
+ * Returns how many tickets at the FIFO front are published (sched_copy). */
+__device__ int sched_claim_check(MtbShared& S, Sched& st, const MkParams& p)
+{
+    const uint32_t lane = threadIdx.x & 31u;
+    const uint32_t queued = st.pt - st.ph;
+    uint32_t want = 0;
+    if (!S.no_tickets) {
+        if (st.est_w == 0) want = queued == 0 ? 1u : 0u;
+        else {
+            want = (uint32_t)__popc(st.free_w) / st.est_w + (uint32_t)PAGODA_LOOKAHEAD;
+            want = want > queued ? want - queued : 0u;
+            if (queued && want < (uint32_t)PAGODA_CLAIM_MIN) want = 0;
+        }
+        const uint32_t est = S.backlog_est;
+        if (est == 0) want = min(want, st.pt == st.pl ? 1u : 0u);   /* a standing reservation */
+        else want = min(want, max((uint32_t)PAGODA_CLAIM_SMALL, min(est / (uint32_t)p.n_mtb, 32u)));
+        want = min(want, 32u - queued);
+    }
+    const uint32_t n = min(st.pt - st.pl, min((uint32_t)__popc(st.free_task), 29u));
+    uint64_t v = 0;
+    bool ready = false;
+    if (lane == 0) {
+        if (want) v = atomicAdd(reinterpret_cast<unsigned long long*>(&p.dctl->head), (unsigned long long)want);
+    } else if (lane == 1) {
+        v = ld_acquire_gpu(&p.dctl->tail);
+    } else if (lane == 2) {
+        v = ld_relaxed_gpu(&p.dctl->head);
+    } else if (lane - 3u < n) {
+        const uint64_t t = S.pend_ticket[(st.pl + lane - 3u) & 31u];
+        ready = ld_acquire_gpu32(&p.dseq[t & p.ring_mask]) == (uint32_t)(t + 1);
+    }
+    const uint64_t old = __shfl_sync(0xffffffffu, v, 0);
+    const uint64_t tail = __shfl_sync(0xffffffffu, v, 1);
+    uint64_t head = __shfl_sync(0xffffffffu, v, 2);
+    const uint32_t rb = __ballot_sync(0xffffffffu, ready) >> 3;
+    const uint32_t r = min((uint32_t)__ffs(~rb) - 1u, n);   /* leading published tickets */
+    if (want) head = max(head, old + want);
+    if (lane < want) S.pend_ticket[(st.pt + lane) & 31u] = old + lane;
+    if (lane == 0) S.backlog_est = (uint32_t)min(tail > head ? tail - head : 0ull, 0xffffffffull);
+    sc_add(S, kScTickets, want);
+    if (want && old >= tail) sc_add(S, kScClaimEmpty, 1);
+    if (n && r == 0) sc_add(S, kScLoadNotReady, 1);
+    st.pt += want;
+    __syncwarp();
+    return (int)r;
+}
+#endif
 
 /* ------------------------------------------------------------------ self-scheduling
  * The paper dedicates warp 0 of every MTB to scheduling.  Here the
@@ -1088,6 +1238,18 @@ __device__ bool sched_round(MtbShared& S, Sched& st, const MkParams& p, int mtb,
     uint64_t t0 = pf_now();
     bool progress = sched_fold(S, st, p, mtb);
     pf_add(S, kPfFold, t0, true);
+#if PAGODA_FUSED_CLAIM
+    t0 = pf_now();
+    {
+        const uint32_t pt0 = st.pt;
+        const int r = sched_claim_check(S, st, p);
+        if (st.pt != pt0) progress = true;
+        pf_add(S, kPfClaim, t0, true);
+        t0 = pf_now();
+        if (r > 0 && sched_copy(S, st, p, (uint32_t)r) > 0) progress = true;
+        pf_add(S, kPfLoad, t0, true);
+    }
+#else
     if (PAGODA_CLAIM_FIRST) {
         t0 = pf_now();
         if (!S.no_tickets && sched_claim(S, st, p) > 0) progress = true;
@@ -1096,6 +1258,7 @@ __device__ bool sched_round(MtbShared& S, Sched& st, const MkParams& p, int mtb,
     t0 = pf_now();
     if (st.pl != st.pt && sched_load(S, st, p) > 0) progress = true;
     pf_add(S, kPfLoad, t0, true);
+#endif
     t0 = pf_now();
     while (st.ph != st.pl) {
         if (!sched_place(S, st, p, mtb, S.pend[st.ph & 31u])) {
@@ -1109,7 +1272,7 @@ __device__ bool sched_round(MtbShared& S, Sched& st, const MkParams& p, int mtb,
     pf_add(S, kPfPlace, t0, true);
     /* MTB 0 (the I/O MTB: ingest, host stores) and the MTB sharing its SM take no tickets
      * unless MTB 0 is the only MTB (validation then caps every task to its capacity) */
-    if (!PAGODA_CLAIM_FIRST) {
+    if (!PAGODA_CLAIM_FIRST && !PAGODA_FUSED_CLAIM) {
         t0 = pf_now();
         if (!S.no_tickets && sched_claim(S, st, p) > 0) progress = true;
         pf_add(S, kPfClaim, t0, true);
@@ -1288,7 +1451,8 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) master_kernel(MkParams p
     if (mtb == 0) exec_mask &= ~(1u << ingest_loader_warp(nw));
     if (io)   /* the I/O roles: loader (31), host poster (30), forwarder (28), publishers (29, 27, ...) */
     {
-        exec_mask &= ~((1u << host_poster_warp(nw)) | (1u << forwarder_warp(nw)));
+        exec_mask &= ~(1u << host_poster_warp(nw));
+        for (uint32_t i = 0; i < p.n_fwd; i++) exec_mask &= ~(1u << forwarder_warp_i(i, nw));
         for (uint32_t i = 0; i < kIngestPublishers; i++) exec_mask &= ~(1u << ingest_publisher_warp(i, nw));
     }
     const int first = __ffs(exec_mask) - 1;
@@ -1311,6 +1475,10 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) master_kernel(MkParams p
             S.sst_free_bar = 0xfffeu;   /* named barriers 1..15; 0 belongs to the MTB */
             S.sst_ph = S.sst_pl = S.sst_pt = 0;
             S.sst_est_w = 0;
+            S.backlog_est = 0;
+            S.fwd_done = 0;
+            S.claim_after = 0;
+            S.dq_safe = *(volatile uint64_t*)&p.dctl->dq_head + kDqEntries;
             S.sst_seq = 0;
             S.token = 1;
             S.comp_pending = 0;
@@ -1333,8 +1501,8 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) master_kernel(MkParams p
     else if (mtb == 0 && warp == ingest_loader_warp(nw)) ingest_loader(S, p, ingest_stage);
     else if (io && ingest_publisher_index(warp, nw) < kIngestPublishers)
         ingest_publisher(S, p, ingest_stage, ingest_publisher_index(warp, nw));
-    else if (mtb == 0 && warp == host_poster_warp(nw)) host_poster(S, p);
-    else if (mtb == 0 && warp == forwarder_warp(nw)) comp_forwarder(S, p);
+    else if (io && warp == host_poster_warp(nw)) host_poster(S, p);
+    else if (io && forwarder_index(warp, nw) < p.n_fwd) comp_forwarder(S, p, forwarder_index(warp, nw));
     else if ((exec_mask >> warp) & 1u) worker(S, smem_base, p, mtb, warp, resident, exec_mask, warp == first);
 }
 

@@ -53,7 +53,8 @@ struct DevCtl {
     alignas(128) uint32_t exited;  /* MTBs that exited */
     alignas(128) unsigned long long ctr[kNumCounters];   /* runtime counters (pagoda_read_counters) */
     alignas(128) uint64_t dq_tail; /* completion queue: records reserved by task posters (fetch-add) */
-    alignas(128) uint64_t dq_head; /* completion queue: records forwarded to the host (forwarder; resumes) */
+    alignas(128) uint64_t dq_head; /* completion queue: records forwarded to the host (forwarders; resumes) */
+    alignas(128) uint64_t fwd_cur[4]; /* each forwarder's cursor: its records below it are forwarded and cleared */
     alignas(128) uint32_t io_smid; /* the SM of MTB 0 (kIoSmidNone until MTB 0 starts) */
 };
 constexpr uint32_t kIoSmidNone = 0xFFFFFFFFu;
@@ -111,18 +112,21 @@ struct MkParams {
     uint32_t*    trace_count; /* [n_mtb] */
     ExecRecord*  exec_trace;  /* [n_mtb][32][trace_cap] */
     uint32_t*    exec_count;  /* [n_mtb][32] */
+    uint64_t*    life;        /* PAGODA_LIFECYCLE: [comp_mask + 1][8] stamps (pagoda_lifecycle_read), or null */
+    uint32_t     n_fwd;       /* completion forwarders in MTB 0 (1..kForwarders) */
+    uint32_t     spread_ns;   /* PAGODA_SPREAD: spread-first claim delay per 4 busy warps (0 = off) */
 };
+enum { kLifePub = 0, kLifeLoad, kLifePlace, kLifeStart, kLifeEnd, kLifeDone, kLifeQueued, kLifeFwd };
 
 /* MTB 0's I/O roles (n_mtb > 1), by position from its last warp (nw = warps per MTB: 32, or 16
  * at 4 MTBs per SM): the loader (nw-1) feeds the device ring (alone it is the whole ingest when
- * n_mtb == 1), the host poster (nw-2) makes the ingest's host-visible stores, the forwarder
- * (nw-4) moves completion records to the host, and kIngestPublishers publisher warps (nw-3,
+ * n_mtb == 1), the host poster (nw-2) makes the ingest's host-visible stores, the completion
+ * forwarders (nw-4, nw-8, ...) move completion records to the host, and kIngestPublishers publisher warps (nw-3,
  * nw-5, nw-6, ...) publish the loader's stages round-robin, each double-buffered
  * (kIngestStages = 2 x publishers), so their per-batch latencies (cell checks, the bulk store,
  * the release fence) overlap */
 __host__ __device__ constexpr int ingest_loader_warp(int nw) { return nw - 1; }
 __host__ __device__ constexpr int host_poster_warp(int nw) { return nw - 2; }
-__host__ __device__ constexpr int forwarder_warp(int nw) { return nw - 4; }
 #ifndef PAGODA_INGEST_PUBLISHERS
 #define PAGODA_INGEST_PUBLISHERS 2
 #endif
@@ -136,6 +140,19 @@ __host__ __device__ constexpr uint32_t ingest_publisher_index(int warp, int nw) 
     return warp == nw - 3 ? 0u : (warp >= nw - 7 && warp <= nw - 5) ? (uint32_t)(nw - 4 - warp) : 99u;
 }
 constexpr uint32_t kDqEntries = 1u << 16;  /* device completion queue */
+/* completion forwarders (MTB 0, n_mtb > 1): forwarder f of MkParams::n_fwd (<= kForwarders) owns
+ * the queue's chunks of kFwdChunk records whose index is f mod n_fwd (warps nw-4, nw-8, nw-9, nw-10) */
+#ifndef PAGODA_FORWARDERS
+#define PAGODA_FORWARDERS 4
+#endif
+constexpr uint32_t kForwarders = PAGODA_FORWARDERS;
+constexpr uint32_t kFwdChunk = 256;
+static_assert(kForwarders >= 1 && kForwarders <= 4, "forwarder warps nw-4, nw-8, nw-9, nw-10");
+__host__ __device__ constexpr int forwarder_warp_i(uint32_t f, int nw) { return f == 0 ? nw - 4 : nw - 7 - (int)f; }
+__host__ __device__ constexpr uint32_t forwarder_index(int warp, int nw)   /* kForwarders+ if none */
+{
+    return warp == nw - 4 ? 0u : (warp >= nw - 10 && warp <= nw - 8) ? (uint32_t)(nw - 7 - warp) : 99u;
+}
 /* ingest staging: 2 stages of MkParams::ingest_stage_entries entries (64 B each).  One MTB: lent
  * from the top of MTB 0's arena (128 entries).  Several: MTB 0 runs no tasks and gives its whole
  * shared memory after the control block (stage_offset) to them. */
@@ -166,7 +183,7 @@ struct MtbShared {
     uint32_t  mb_warps;              /* 4032: mailbox: warps that finished (atomicOr by executors) */
     uint32_t  mb_tbs;                /*       mailbox: TB records whose last warp finished */
     uint32_t  mb_tasks;              /*       mailbox: task slots whose last warp finished */
-    uint32_t  pad_;
+    uint32_t  backlog_est;           /*       ring backlog (tail - head) at the holder's last look (fused claims) */
     uint64_t  tb_task[32];           /* 4048: task id of each TB record (ledger) */
     uint16_t  tb_idx[32];            /* 4304: TB index j of each TB record (ledger) */
     uint64_t  pend_ticket[32];       /* 4368: claimed ring positions, FIFO (pend[] holds their slots once loaded) */
@@ -193,6 +210,9 @@ struct MtbShared {
     uint32_t  comp_pending;          /* task slots finished, completion record not yet posted */
     uint32_t  no_tickets;            /* this MTB runs no tasks (MTB 0 and the MTB sharing its SM) */
     unsigned long long sprof[8];     /* PAGODA_PROFILE: ns per phase (PAGODA_CTR_SCHED_NS_FOLD + i) */
+    unsigned long long dq_safe;      /* completion-queue positions below this are known free (posters' cache) */
+    uint32_t  fwd_done;              /* MTB 0: forwarders that exited */
+    unsigned long long claim_after;  /* PAGODA_SPREAD_NS: no claim before this %globaltimer value */
 };
 static_assert(offsetof(MtbShared, wt) == kWarpTableOffset, "WarpTable offset");
 static_assert(offsetof(MtbShared, stage_bar) == kStageBarOffset, "staging mbarriers offset");

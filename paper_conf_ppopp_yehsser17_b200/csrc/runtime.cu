@@ -64,6 +64,7 @@ struct pagoda_ctx {
     LedgerEvent* trace = nullptr;
     uint32_t* trace_count = nullptr;
     ExecRecord* exec_trace = nullptr;
+    uint64_t* life = nullptr;               /* PAGODA_LIFECYCLE stamps */
     uint32_t* exec_count = nullptr;
     /* host state */
     std::atomic<uint64_t> next_id{0};
@@ -258,6 +259,7 @@ static bool pow2(uint32_t x) { return x && !(x & (x - 1)); }
 static int start_kernel(pagoda_ctx* c)
 {
     cudaSetDevice(c->device);
+    if (c->life) cudaMemsetAsync(c->life, 0, (size_t)c->C * 8 * sizeof(uint64_t), c->stream);
     if (c->trace_count) {
         cudaMemsetAsync(c->trace_count, 0, (size_t)c->n_mtb * sizeof(uint32_t), c->stream);
         cudaMemsetAsync(c->exec_count, 0, (size_t)c->n_mtb * 32 * sizeof(uint32_t), c->stream);
@@ -341,6 +343,7 @@ static void free_ctx(pagoda_ctx* c)
     if (c->trace) cudaFree(c->trace);
     if (c->trace_count) cudaFree(c->trace_count);
     if (c->exec_trace) cudaFree(c->exec_trace);
+    if (c->life) cudaFree(c->life);
     if (c->exec_count) cudaFree(c->exec_count);
     if (c->stream) cudaStreamDestroy(c->stream);
     delete c;
@@ -435,6 +438,10 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
         cudaMemset(c->trace_count, 0, (size_t)c->n_mtb * sizeof(uint32_t));
         cudaMemset(c->exec_count, 0, (size_t)c->n_mtb * 32 * sizeof(uint32_t));
     }
+    if (cfg.flags & PAGODA_LIFECYCLE) {
+        if (cudaMalloc(&c->life, (size_t)c->C * 8 * sizeof(uint64_t)) != cudaSuccess) goto fail;
+        if (cudaMemset(c->life, 0, (size_t)c->C * 8 * sizeof(uint64_t)) != cudaSuccess) goto fail;
+    }
     if (cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking) != cudaSuccess) goto fail;
     if (cudaEventCreate(&c->ev_start) != cudaSuccess || cudaEventCreate(&c->ev_stop) != cudaSuccess) goto fail;
     if (cudaDeviceSynchronize() != cudaSuccess) goto fail;
@@ -477,6 +484,11 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
             p.exec_trace = c->exec_trace;
             p.exec_count = c->exec_count;
         }
+        p.life = c->life;
+        /* completion forwarders: 4 when MTB 0 has 32 warps; 1 at 4 MTBs/SM (512 threads), where more
+         * cost MM ~7 % (45 -> 42 M tasks/s) while NOP's forwarding is not the limit there */
+        p.n_fwd = cfg.mtbs_per_sm == 4 ? 1u : (uint32_t)kForwarders;
+        p.spread_ns = (cfg.flags & PAGODA_SPREAD) ? 6000u : 0u;
         c->smem = smem;
         rc = (cfg.flags & PAGODA_NO_START) ? 0 : start_kernel(c);
         if (rc) goto fail;
@@ -865,6 +877,18 @@ int64_t pagoda_trace_read(pagoda_ctx* c, int mtb, void* dst, size_t cap)
             cudaSuccess)
         return -EIO;
     return n;
+}
+
+int64_t pagoda_lifecycle_read(pagoda_ctx* c, uint64_t first, size_t n, uint64_t* dst)
+{
+    if (!c || (!dst && n) || n > c->C) return -EINVAL;
+    if (!c->life) return -ENODATA;
+    cudaSetDevice(c->device);
+    const uint64_t f = first & (c->C - 1);
+    const size_t n1 = std::min<size_t>(n, c->C - f);
+    if (cudaMemcpy(dst, c->life + f * 8, n1 * 64, cudaMemcpyDeviceToHost) != cudaSuccess) return -EIO;
+    if (n1 < n && cudaMemcpy(dst + n1 * 8, c->life, (n - n1) * 64, cudaMemcpyDeviceToHost) != cudaSuccess) return -EIO;
+    return (int64_t)n;
 }
 
 int64_t pagoda_trace_read_exec(pagoda_ctx* c, int mtb, int warp, void* dst, size_t cap)

@@ -20,6 +20,9 @@ LIB_PATH = os.environ.get("PAGODA_LIB") or os.path.join(PKG, "libpagoda.so")
 TRACE = 0x1
 NO_START = 0x2
 RESIDENT_TDES = 0x4
+LIFECYCLE = 0x8
+SPREAD = 0x10
+LIFE_EVENTS = ("pub", "load", "place", "start", "end", "done", "queued", "fwd")
 
 
 class pagoda_config(C.Structure):
@@ -74,6 +77,8 @@ def lib() -> C.CDLL:
         L.pagoda_trace_read.restype = I64
         L.pagoda_trace_read_exec.argtypes = [P, I, I, P, SZ]
         L.pagoda_trace_read_exec.restype = I64
+        L.pagoda_lifecycle_read.argtypes = [P, C.c_uint64, SZ, P]
+        L.pagoda_lifecycle_read.restype = I64
         L.pagoda_tdes_tables.argtypes = [P, P]
         L.pagoda_naive_run.argtypes = [I, I, P, P, SZ, SZ, I, C.POINTER(I64)]
         L.pagoda_pingpong.argtypes = [I, I, P]
@@ -257,6 +262,12 @@ class Pagoda:
         n = _check(lib().pagoda_trace_read_exec(self.h, mtb, warp, None, 0), "pagoda_trace_read_exec")
         buf = np.zeros(min(n, self.cfg.trace_events), EXEC_DTYPE)
         _check(lib().pagoda_trace_read_exec(self.h, mtb, warp, _ptr(buf), len(buf)), "pagoda_trace_read_exec")
+        return buf
+
+    def lifecycle(self, first: int, n: int) -> np.ndarray:
+        """PAGODA_LIFECYCLE stamps of tasks [first, first+n): uint64 [n, 8] (LIFE_EVENTS order, GPU ns)."""
+        buf = np.zeros((n, 8), np.uint64)
+        _check(lib().pagoda_lifecycle_read(self.h, first, n, _ptr(buf)), "pagoda_lifecycle_read")
         return buf
 
     def shutdown(self) -> int:

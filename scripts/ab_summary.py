@@ -7,8 +7,8 @@ import sys
 
 d = sys.argv[1] if len(sys.argv) > 1 else "gpurun_out"
 rows = {}
-for f in sorted(glob.glob(os.path.join(d, "ab_*_*_*.json"))):
-    m = re.match(r"ab_(\w+?)_(\w+)_(\d+)\.json", os.path.basename(f))
+for f in sorted(glob.glob(os.path.join(d, "*_*_*.json"))):
+    m = re.match(r"(?:ab_)?(\w+?)_(\w+)_(\d+)\.json", os.path.basename(f))
     if not m:
         continue
     try:
@@ -18,7 +18,7 @@ for f in sorted(glob.glob(os.path.join(d, "ab_*_*_*.json"))):
     rows.setdefault(m.group(1), {}).setdefault(m.group(2), []).append(v)
 for w, vs in rows.items():
     print(w, {k: [round(x / 1e6, 2) if x else x for x in xs] for k, xs in vs.items()})
-for f in sorted(glob.glob(os.path.join(d, "ab_t*.txt"))):
+for f in sorted(glob.glob(os.path.join(d, "*t*.txt"))):
     print(os.path.basename(f), open(f).read().strip())
 for f in sorted(glob.glob(os.path.join(d, "ab_probe_*.json"))):
     try:

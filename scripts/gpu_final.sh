@@ -7,6 +7,7 @@ timeout 900 python bench.py > $F/bench_tdes.json 2> $F/bench_tdes.err
 for w in ${WORKLOADS:-mb mm mm_tc mix c5 mpe tdes_var nop}; do
   timeout 900 python bench.py --workload $w > $F/bench_$w.json 2> $F/bench_$w.err
 done
+timeout 600 python scripts/probe_life.py nop mm tdes mix mb c5 mpe > $F/life.jsonl 2> $F/life.err
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $F/launches_tdes.csv \
   python bench.py --prespawn --steps 3 --warmup 3 --no-naive --no-cpu --quick > $F/ncu_launch.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:master -s 3 -c 1 -o $F/tdes_full \
@@ -18,5 +19,5 @@ python scripts/ncu_summary.py $F/mm_full.ncu-rep > $F/ncu_mm_full.txt 2>&1
 rm -f $F/*.ncu-rep
 timeout 600 python scripts/probe_busy.py mm tdes nop mb > $F/busy.jsonl 2>&1
 timeout 300 python scripts/probe_session_overhead.py > $F/session_overhead.json 2>&1
-timeout 1200 python scripts/sweeps.py > $F/sweeps.jsonl 2> $F/sweeps.err
+timeout 600 python scripts/probe_runtime.py > $F/runtime.json 2>&1
 ls -la $F

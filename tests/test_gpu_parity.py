@@ -41,8 +41,8 @@ def run(w, **cfg):
 
 
 # ---------------------------------------------------------------- MB (config 1)
-# 2 MTBs/SM: the one-pixel body (32 registers); 1 MTB/SM: the two-pixel body (64 registers, bench preset)
-MB_CFGS = [{}, {"mtbs_per_sm": 1, "arena_bytes": 96 * 1024}]
+# 2 and 1 MTBs per SM (32 / 64 registers per thread), and spread-first claims (the bench preset)
+MB_CFGS = [{}, {"mtbs_per_sm": 1, "arena_bytes": 96 * 1024}, {"flags": 0x10}]   # 0x10: PAGODA_SPREAD (bench preset)
 
 
 @pytest.mark.parametrize("cfg", MB_CFGS)

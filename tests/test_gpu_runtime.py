@@ -202,6 +202,33 @@ def test_spawn_shapes_multi_producer_exactly_once(producers):
     assert np.array_equal(c, shapes[:, 0].astype(np.uint32))   # each task's threads ran once
 
 
+def test_lifecycle_stamps_ordered():
+    """PAGODA_LIFECYCLE: every stage of every task is stamped once, in causal order
+    (published -> loaded -> placed -> body start -> body end -> fenced -> queued ->
+    forwarded; %globaltimer is one clock for all SMs, 1 us slack for its granularity)."""
+    from paper_conf_ppopp_yehsser17_b200.pagoda import LIFECYCLE, NO_START
+    n = 5000
+    with Pagoda(flags=LIFECYCLE | NO_START) as p:
+        assert p.start() == 0
+        ids = p.spawn_many(n, 128, 1, 1024, True, T.NOP, None, ids=True)
+        assert p.stop() == 0
+        L = p.lifecycle(int(ids[0]), n).astype(np.int64)
+    assert (L > 0).all()
+    assert (np.diff(L, axis=1) >= -1000).all()
+
+
+def test_single_mtb_context():
+    """One MTB on one SM: MTB 0 runs tasks itself (single-warp ingest, completion records
+    straight to the host window, no forwarders): spawn across a ring wrap and check."""
+    with Pagoda(num_sms=1, mtbs_per_sm=1, arena_bytes=64 * 1024, ring_entries=1024) as p:
+        assert p.info().n_mtb == 1
+        ids = p.spawn_many(5000, 128, 1, 2048, True, T.NOP, None, ids=True)
+        assert p.waitAll() == 0
+        assert all(p.check(int(i)) == 1 for i in ids[::101])
+        ids = [p.taskSpawn(992, 1, 0, True, T.NOP) for _ in range(50)]
+        assert p.waitAll() == 0 and all(p.check(i) == 1 for i in ids)
+
+
 def test_ring_wraparound_and_completion_window():
     """More tasks than ring entries and completion slots: slots are reused only
     after their previous occupant is consumed / done."""
