@@ -488,7 +488,11 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
         /* completion forwarders: 4 when MTB 0 has 32 warps; 1 at 4 MTBs/SM (512 threads), where more
          * cost MM ~7 % (45 -> 42 M tasks/s) while NOP's forwarding is not the limit there */
         p.n_fwd = cfg.mtbs_per_sm == 4 ? 1u : (uint32_t)kForwarders;
-        p.spread_ns = (cfg.flags & PAGODA_SPREAD) ? 6000u : 0u;
+        p.spread_ns = 0;
+        if (cfg.flags & PAGODA_SPREAD) {   /* PAGODA_SPREAD_NS (environment) overrides the 6 us default */
+            const char* e = getenv("PAGODA_SPREAD_NS");
+            p.spread_ns = e ? (uint32_t)strtoul(e, nullptr, 10) : 6000u;
+        }
         c->smem = smem;
         rc = (cfg.flags & PAGODA_NO_START) ? 0 : start_kernel(c);
         if (rc) goto fail;
