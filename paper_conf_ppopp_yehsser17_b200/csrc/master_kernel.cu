@@ -39,8 +39,8 @@
 #ifndef PAGODA_CLAIM_MIN
 #define PAGODA_CLAIM_MIN 1    /* with tickets queued, claim only when at least this many are wanted */
 #endif
-#ifndef PAGODA_FREE_EARLY
-#define PAGODA_FREE_EARLY 0   /* a task's last warp frees itself before posting the completion record */
+#ifndef PAGODA_WAKE_HINT_NS
+#define PAGODA_WAKE_HINT_NS 1000000   /* suspend-time hint of an idle executor's mbarrier try_wait */
 #endif
 #ifndef PAGODA_FUSED_CLAIM
 #define PAGODA_FUSED_CLAIM 0  /* claim, tail/head reads and publication checks in one round trip */
@@ -72,9 +72,9 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity)
     const uint32_t a = smem_u32(bar);
     while (!done) {
         asm volatile(
-            "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, 1000000; selp.u32 %0, 1, 0, p; }"
+            "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3; selp.u32 %0, 1, 0, p; }"
             : "=r"(done)
-            : "r"(a), "r"(parity)
+            : "r"(a), "r"(parity), "n"(PAGODA_WAKE_HINT_NS)
             : "memory");
     }
 }
@@ -478,19 +478,6 @@ __device__ __forceinline__ void run_task(MtbShared& S, char* smem_base, const Mk
     }
     pf_add(S, kPfFence, tp, true);
     tp = pf_now();
-#if PAGODA_FREE_EARLY
-    /* free the warp first, then post: the scheduler can place the next task on this warp (and
-     * its TB partners) while the completion record is still on its way; the holder does not
-     * exit while a completion is pending or being posted (sched_round) */
-    if (lane == 0) {
-        __threadfence_block();   /* TB / task frees are visible before the warp frees itself */
-        atomicOr(&S.mb_warps, 1u << w);
-        __threadfence_block();
-    }
-    __syncwarp();
-    if (__shfl_sync(0xffffffffu, last, 0)) post_completions(S, p);
-    pf_add(S, kPfPost, tp, true);
-#else
     if (__shfl_sync(0xffffffffu, last, 0)) post_completions(S, p);
     pf_add(S, kPfPost, tp, true);
     if (lane == 0) {
@@ -499,7 +486,6 @@ __device__ __forceinline__ void run_task(MtbShared& S, char* smem_base, const Mk
         __threadfence_block();   /* ... and the warp's free bit before its attempt at the token */
     }
     __syncwarp();
-#endif
 }
 
 /* MTB 0's host poster (n_mtb > 1): the ingest warp's host-visible stores
@@ -1300,10 +1286,6 @@ __device__ bool sched_round(MtbShared& S, Sched& st, const MkParams& p, int mtb,
     if (!progress && st.free_w == st.exec_mask && st.ph == st.pl) {
         uint32_t stop = 0;
         if (lane == 0) stop = ld_acquire_gpu32(&p.dctl->stop);
-        /* PAGODA_FREE_EARLY: a free warp may still be posting a completion: not yet */
-        if (PAGODA_FREE_EARLY && lane == 0 && stop != kStopAbort &&
-            (*(volatile uint32_t*)&S.comp_pending | *(volatile uint32_t*)&S.poster))
-            stop = 0;
         stop = __shfl_sync(0xffffffffu, stop, 0);
         if (stop == kStopAbort) exit = true;   /* host watchdog gave up */
         else if (stop) {

@@ -42,7 +42,8 @@ def run(w, **cfg):
 
 # ---------------------------------------------------------------- MB (config 1)
 # 2 and 1 MTBs per SM (32 / 64 registers per thread), and spread-first claims (the bench preset)
-MB_CFGS = [{}, {"mtbs_per_sm": 1, "arena_bytes": 96 * 1024}, {"flags": 0x10}]   # 0x10: PAGODA_SPREAD (bench preset)
+MB_CFGS = [{}, {"mtbs_per_sm": 1, "arena_bytes": 96 * 1024}, {"flags": 0x10},   # 0x10: PAGODA_SPREAD
+           {"mtbs_per_sm": 1, "arena_bytes": 96 * 1024, "flags": 0x10}]          # the bench preset
 
 
 @pytest.mark.parametrize("cfg", MB_CFGS)
