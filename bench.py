@@ -338,18 +338,8 @@ def make_workload(name, resident=False, d=None, device="cuda"):
     return W.nop(200000)
 
 
-# per-workload context presets
-PRESETS = {
-    "tdes": {"mtbs_per_sm": 2, "arena_bytes": 40 * 1024, "resident": True},
-    "mb": {"mtbs_per_sm": 1, "arena_bytes": 96 * 1024, "resident": False, "spread": True},   # 4.2 vs 3.8 M at 2
-    "mm": {"mtbs_per_sm": 4, "arena_bytes": 48 * 1024, "resident": False},   # 512-thread MTBs: 2x schedulers
-    "mix": {"mtbs_per_sm": 1, "arena_bytes": 200 * 1024, "resident": False},
-    "nop": {"mtbs_per_sm": 2, "arena_bytes": 96 * 1024, "resident": False, "producers": 2},
-    "c5": {"mtbs_per_sm": 1, "arena_bytes": 144 * 1024, "resident": True},
-    "mpe": {"mtbs_per_sm": 2, "arena_bytes": 40 * 1024, "resident": True},
-    "tdes_var": {"mtbs_per_sm": 2, "arena_bytes": 40 * 1024, "resident": True},
-    "mm_tc": {"mtbs_per_sm": 4, "arena_bytes": 48 * 1024, "resident": False},
-}
+# per-workload context presets: paper_conf_ppopp_yehsser17_b200/presets.py
+from paper_conf_ppopp_yehsser17_b200.presets import PRESETS  # noqa: E402
 
 
 def use_resident(a):

@@ -1,0 +1,27 @@
+"""Per-workload MasterKernel context presets: the launch configuration bench.py
+times for each BASELINE.json workload, shared with the
+full-size parity tests so that they run in exactly that configuration."""
+
+# mtbs_per_sm / arena_bytes: pagoda_config; resident: PAGODA_RESIDENT_TDES (+ registered round
+# keys in bench.py); spread: PAGODA_SPREAD; producers: host spawner threads per step
+PRESETS = {
+    "tdes": {"mtbs_per_sm": 2, "arena_bytes": 40 * 1024, "resident": True},
+    "mb": {"mtbs_per_sm": 1, "arena_bytes": 96 * 1024, "resident": False, "spread": True},   # 4.2 vs 3.8 M at 2
+    "mm": {"mtbs_per_sm": 4, "arena_bytes": 48 * 1024, "resident": False},   # 512-thread MTBs: 2x schedulers
+    "mix": {"mtbs_per_sm": 1, "arena_bytes": 200 * 1024, "resident": False},
+    "nop": {"mtbs_per_sm": 2, "arena_bytes": 96 * 1024, "resident": False, "producers": 2},
+    "c5": {"mtbs_per_sm": 1, "arena_bytes": 144 * 1024, "resident": True},
+    "mpe": {"mtbs_per_sm": 2, "arena_bytes": 40 * 1024, "resident": True},
+    "tdes_var": {"mtbs_per_sm": 2, "arena_bytes": 40 * 1024, "resident": True},
+    "mm_tc": {"mtbs_per_sm": 4, "arena_bytes": 48 * 1024, "resident": False},
+}
+
+RESIDENT_TDES = 0x4   # include/pagoda.h
+SPREAD = 0x10
+
+
+def ctx_kwargs(workload: str, flags: int = 0) -> dict:
+    """pagoda_config keyword arguments (Pagoda(**...)) of the workload's preset."""
+    pr = PRESETS[workload]
+    f = flags | (RESIDENT_TDES if pr["resident"] else 0) | (SPREAD if pr.get("spread") else 0)
+    return {"flags": f, "mtbs_per_sm": pr["mtbs_per_sm"], "arena_bytes": pr["arena_bytes"]}

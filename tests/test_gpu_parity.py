@@ -18,6 +18,7 @@ import oracle
 from paper_conf_ppopp_yehsser17_b200 import inputs as I
 from paper_conf_ppopp_yehsser17_b200 import workloads as W
 from paper_conf_ppopp_yehsser17_b200.pagoda import NO_START, RESIDENT_TDES, Pagoda, naive_run
+from paper_conf_ppopp_yehsser17_b200.presets import ctx_kwargs
 
 pytestmark = pytest.mark.gpu
 
@@ -113,7 +114,7 @@ def test_mm_small(shmem, threads):
 
 def test_mm_config3_full_size():
     w = W.matmul(65536)
-    out = run(w)["C"]
+    out = run(w, **ctx_kwargs("mm"))["C"]   # the bench's launch configuration
     rng = np.random.default_rng(3)
     _mm_check(w, out, list(rng.choice(65536, 256, replace=False)) + [0, 65535])
 
@@ -141,7 +142,7 @@ def test_mm_tc_integer_exact_and_full_size():
     for k in range(64):
         assert np.array_equal(out[k], oracle.mm32_exact(w.host["A"][k], w.host["B"][k])), k
     w = W.matmul(65536, func=T.MM_TC)
-    out = run(w)["C"]
+    out = run(w, **ctx_kwargs("mm_tc"))["C"]   # the bench's launch configuration
     rng = np.random.default_rng(5)
     _mm_tc_check(w, out, list(rng.choice(65536, 256, replace=False)) + [0, 65535])
 
@@ -178,7 +179,7 @@ def test_mix_small_all_shapes():
 
 def test_mix_config4_full_size_sampled():
     w = W.mix(32768)
-    _mix_check(w, run(w), frac=0.004, seed=4)
+    _mix_check(w, run(w, **ctx_kwargs("mix")), frac=0.004, seed=4)   # the bench's launch configuration
 
 
 # ---------------------------------------------------------------- the naive baseline runs the same bodies
