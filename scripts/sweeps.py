@@ -5,6 +5,10 @@
             and 8192 MB tiles (MB repeats config 1's 1024 tiles)
   large   : 4096 CONV tasks (128x128) of 128 .. 16384 threads; above 1024 the task is
             several 1024-thread TBs spread over MTBs (Fig. 8's large tasks)
+  size    : input size x threads (Fig. 8): 3DES packets of 1 .. 64 KiB with
+            64 .. 512 threads per task, 64 MiB of packets per point (65536 .. 1024 tasks)
+
+    python scripts/sweeps.py [tasks threads large size]   # default: all
 
 Each point: Pagoda (one session: start -> spawn all -> stop; CUDA-event
 device time and host time), the naive one-launch-per-task baseline and the
@@ -67,18 +71,29 @@ def point(sweep, label, w, **cfg):
 
 def main():
     torch.cuda.set_device(0)
+    which = set(sys.argv[1:]) or {"tasks", "threads", "large", "size"}
     res = {"flags": PG.RESIDENT_TDES, "arena_bytes": 40 * 1024}
-    for n in (32, 128, 512, 2048, 8192, 32768):   # Fig. 6: the number of tasks
-        w = W.tdes(n, shmem=512)
-        point("tasks", {"body": "tdes", "threads": 128}, w, **res)
-    for th in (32, 64, 128, 256, 512, 1024):       # Fig. 7: threads per task
-        w = W.tdes(32768, shmem=512, threads=th)
-        point("threads", {"body": "tdes", "threads": th}, w, **res)
-        w = W.mandelbrot(8192, threads=th)
-        point("threads", {"body": "mb", "threads": th}, w)
-    for th in (128, 512, 1024, 4096, 16384):       # Fig. 8: large tasks, spread over MTBs above 1024
-        w = W.conv_only(4096, threads=min(th, 1024), n_tb=max(1, th // 1024))
-        point("large", {"body": "conv", "threads": th, "tbs": max(1, th // 1024)}, w)
+    if "tasks" in which:
+        for n in (32, 128, 512, 2048, 8192, 32768):   # Fig. 6: the number of tasks
+            w = W.tdes(n, shmem=512)
+            point("tasks", {"body": "tdes", "threads": 128}, w, **res)
+    if "threads" in which:
+        for th in (32, 64, 128, 256, 512, 1024):       # Fig. 7: threads per task
+            w = W.tdes(32768, shmem=512, threads=th)
+            point("threads", {"body": "tdes", "threads": th}, w, **res)
+            w = W.mandelbrot(8192, threads=th)
+            point("threads", {"body": "mb", "threads": th}, w)
+    if "large" in which:
+        for th in (128, 512, 1024, 4096, 16384):       # Fig. 8: large tasks, spread over MTBs above 1024
+            w = W.conv_only(4096, threads=min(th, 1024), n_tb=max(1, th // 1024))
+            point("large", {"body": "conv", "threads": th, "tbs": max(1, th // 1024)}, w)
+    if "size" in which:
+        for kib in (1, 4, 16, 64):                     # Fig. 8: input size x threads, 64 MiB per point
+            for th in (64, 128, 256, 512):
+                w = W.tdes((64 << 20) // (kib << 10), nbytes=kib << 10, threads=th, shmem=512)
+                point("size", {"body": "tdes", "packet_kib": kib, "threads": th}, w, **res)
+                del w
+                torch.cuda.empty_cache()
 
 
 if __name__ == "__main__":
