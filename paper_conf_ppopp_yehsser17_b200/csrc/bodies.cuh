@@ -419,13 +419,33 @@ __device__ void body_mm(const Env& e, const pagoda_mm_args& a)
         A = s;
         B = s + 1024;
     }
+    /* A thread's outputs idx, idx + T, ... (same column j when 32 | T) advance together, four
+     * independent fma chains at a time (each still k ascending from 0): one B load serves all */
     const int T = total_threads(e);
-    for (int idx = e.getTid(); idx < 1024; idx += T) {
-        const int i = idx >> 5, j = idx & 31;
-        float acc = 0.0f;
+    for (int base = e.getTid(); base < 1024; base += 4 * T) {
+        float acc[4] = {0.0f, 0.0f, 0.0f, 0.0f};
+        int row[4];
+#pragma unroll
+        for (int q = 0; q < 4; q++) row[q] = min(base + q * T, 1023) >> 5;   /* past the end: a dummy row */
+        const int j = base & 31;
+        if ((T & 31) == 0) {
 #pragma unroll 8
-        for (int k = 0; k < 32; k++) acc = __fmaf_rn(A[i * 32 + k], B[k * 32 + j], acc);
-        a.C[idx] = acc;
+            for (int k = 0; k < 32; k++) {
+                const float b = B[k * 32 + j];
+#pragma unroll
+                for (int q = 0; q < 4; q++) acc[q] = __fmaf_rn(A[row[q] * 32 + k], b, acc[q]);
+            }
+        } else {   /* T not a multiple of 32: each item has its own column */
+#pragma unroll 4
+            for (int k = 0; k < 32; k++) {
+#pragma unroll
+                for (int q = 0; q < 4; q++)
+                    acc[q] = __fmaf_rn(A[row[q] * 32 + k], B[k * 32 + (min(base + q * T, 1023) & 31)], acc[q]);
+            }
+        }
+#pragma unroll
+        for (int q = 0; q < 4; q++)
+            if (base + q * T < 1024) a.C[base + q * T] = acc[q];
     }
 }
 
