@@ -57,6 +57,7 @@ def lib():
             L.orc_tdes_ecb.argtypes = [P, P, SZ, P, I]
             L.orc_mm32.argtypes = [P, P, P]
             L.orc_mm32_f64.argtypes = [P, P, P]
+            L.orc_mm64.argtypes = [P, P, P]
             L.orc_filterbank.argtypes = [P, P, P, P]
             L.orc_beamformer.argtypes = [P, P, P, P]
             L.orc_conv.argtypes = [P, P, P, P]
@@ -112,6 +113,14 @@ def mm32(A, B) -> np.ndarray:
     A = np.ascontiguousarray(A, np.float32); B = np.ascontiguousarray(B, np.float32)
     Cm = np.zeros((32, 32), np.float32)
     lib().orc_mm32(_p(A), _p(B), _p(Cm))
+    return Cm
+
+
+def mm64(A, B) -> np.ndarray:
+    """Table 4's 64x64x64 MatrixMul: fma chain over k ascending, as mm32."""
+    A = np.ascontiguousarray(A, np.float32); B = np.ascontiguousarray(B, np.float32)
+    Cm = np.zeros((64, 64), np.float32)
+    lib().orc_mm64(_p(A), _p(B), _p(Cm))
     return Cm
 
 

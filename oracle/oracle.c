@@ -191,6 +191,18 @@ void orc_mm32(const float* A, const float* B, float* C)
         }
 }
 
+/* MM 64x64x64 fp32: Table 4's "MatrixMul ... 64 x 64 matrix" (SURVEY §8(f)
+ * NEXT-4): the same definition at n = 64, C[i][j] = fma-chain over k ascending. */
+void orc_mm64(const float* A, const float* B, float* C)
+{
+    for (int i = 0; i < 64; i++)
+        for (int j = 0; j < 64; j++) {
+            float acc = 0.0f;
+            for (int k = 0; k < 64; k++) acc = fmaf(A[i * 64 + k], B[k * 64 + j], acc);
+            C[i * 64 + j] = acc;
+        }
+}
+
 /* MM on the tensor cores: the same product C = A B,
  * whose summation order the hardware picks; the definition is the exact
  * product, here accumulated in fp64 (each fp32 x fp32 product is exact in

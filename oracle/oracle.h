@@ -49,6 +49,7 @@ void orc_des_key_schedule(const uint8_t key8[8], uint64_t subkeys[16]);
 uint64_t orc_des_block(uint64_t block, const uint64_t subkeys[16], int decrypt);
 void orc_tdes_ecb(const uint8_t* in, uint8_t* out, size_t nbytes, const uint8_t key24[24], int decrypt);
 void orc_mm32(const float* A, const float* B, float* C);
+void orc_mm64(const float* A, const float* B, float* C);       /* Table 4's 64x64 size (NEXT-4) */
 void orc_mm32_f64(const float* A, const float* B, float* C);   /* exact product, one rounding (NEXT-4) */
 void orc_filterbank(const float* r, const float* H, const float* F, float* y);
 void orc_beamformer(const float* x, const float* h, const float* w, float* out);

@@ -30,7 +30,7 @@ _TASK_MUL = np.uint64(0xD1B54A32D192ED03)
 # different numbers for the same task index
 TAG = {
     "mb": 0x0, "tdes": 0x3DE5, "mm": 0x3232, "fb": 0xFB00, "bf": 0xBF00,
-    "conv": 0xC0DE, "dct": 0xDC70, "mix": 0x4D1C, "misc": 0x7E57,
+    "conv": 0xC0DE, "dct": 0xDC70, "mix": 0x4D1C, "misc": 0x7E57, "mm64": 0x6464,
 }
 
 
@@ -97,6 +97,17 @@ def mm_inputs(n_tasks: int, first: int = 0, integer: bool = False):
         v = to_f32(z)
     return (np.ascontiguousarray(v[:, :1024].reshape(-1, 32, 32)),
             np.ascontiguousarray(v[:, 1024:].reshape(-1, 32, 32)))
+
+
+def mm64_inputs(n_tasks: int, first: int = 0, integer: bool = False):
+    """A, B: [n_tasks, 64, 64] fp32 uniform in [-1,1) (or integers in [-8,8]); Table 4's MM size."""
+    z = splitmix64(np.arange(first, first + n_tasks), 8192, SEED ^ TAG["mm64"])
+    if integer:
+        v = (((z >> np.uint64(40)) % np.uint64(17)).astype(np.int64) - 8).astype(np.float32)
+    else:
+        v = to_f32(z)
+    return (np.ascontiguousarray(v[:, :4096].reshape(-1, 64, 64)),
+            np.ascontiguousarray(v[:, 4096:].reshape(-1, 64, 64)))
 
 
 FB_NSIM, FB_NCOL, FB_NSAMP = 2048, 32, 8

@@ -147,6 +147,26 @@ def test_mm_within_error_bound(orc):
     assert not np.allclose(orc.mm32(A[0], B[0]), (A[0].astype(np.float64) @ B[0].T), atol=1e-3)
 
 
+def test_mm64_pins(orc):
+    """Table 4's 64x64 size: identity both sides, integer inputs exact (every partial sum
+    is an integer below 2^24), random inputs within the fma chain's bound gamma_64 |A||B|,
+    a transposed operand and a dropped last k term are caught."""
+    A, B = inputs.mm64_inputs(2)
+    I64 = np.eye(64, dtype=np.float32)
+    assert np.array_equal(orc.mm64(A[0], I64), A[0])
+    assert np.array_equal(orc.mm64(I64, B[1]), B[1])
+    Ai, Bi = inputs.mm64_inputs(3, integer=True)
+    for i in range(3):
+        assert np.array_equal(orc.mm64(Ai[i], Bi[i]).astype(np.int64), Ai[i].astype(np.int64) @ Bi[i].astype(np.int64))
+    for i in range(2):
+        a, b = A[i].astype(np.float64), B[i].astype(np.float64)
+        got = orc.mm64(A[i], B[i]).astype(np.float64)
+        assert (np.abs(got - a @ b) <= gamma(64) * (np.abs(a) @ np.abs(b))).all()
+    assert not np.allclose(orc.mm64(A[0], B[0]), A[0].astype(np.float64) @ B[0].T, atol=1e-3)
+    got = orc.mm64(Ai[0], Bi[0]).astype(np.int64)
+    assert not np.array_equal(got, Ai[0][:, :63].astype(np.int64) @ Bi[0][:63].astype(np.int64))
+
+
 def test_mm_exact_variant(orc):
     """mm32_exact (NEXT-4's definition): integer inputs exact; random inputs
     equal the exactly rounded product (exact rational sum via fractions,
