@@ -2,7 +2,7 @@
 """bench.py — narrow tasks/s and p50 spawn-to-done latency of the B200 Pagoda
 hot path (BASELINE.json "metric"), one JSON line on rank 0.
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload tdes|mb|mm|mix|nop|c5|mpe|tdes_var]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload tdes|mb|mm|mix|nop|c5|mpe|tdes_var|mm_tc|dct|dct_noshm|mm_noshm|mm64]
     python bench.py --impl reference ...     # the oracle on the host cores (base contract's reference arm)
     torchrun --nproc-per-node N bench.py --gpus N   # one process per GPU
 
@@ -45,8 +45,10 @@ BASE = json.load(open(os.path.join(ROOT, "BASELINE.json")))
 TDES_LOOKUPS_PER_TASK = 512 * 48 * 8          # S-box table lookups (LDS) per 4 KiB packet
 LDS_LANES_PER_SM_CLK = 32                     # one 128 B shared-memory wavefront per SM per clock
 DTYPE = {"tdes": "u32", "mb": "f32", "mm": "f32", "mix": "f32", "nop": "none", "c5": "f32+u32", "mpe": "f32+u32",
-         "tdes_var": "u32", "mm_tc": "tf32x3"}   # arithmetic type of the path
-WORKLOADS = ("tdes", "mb", "mm", "mix", "nop", "c5", "mpe", "tdes_var", "mm_tc")
+         "tdes_var": "u32", "mm_tc": "tf32x3", "dct": "f32", "dct_noshm": "f32",
+         "mm_noshm": "f32", "mm64": "f32"}   # arithmetic type of the path
+WORKLOADS = ("tdes", "mb", "mm", "mix", "nop", "c5", "mpe", "tdes_var", "mm_tc", "dct", "dct_noshm", "mm_noshm",
+             "mm64")
 STRONG = ("c5",)   # total work fixed as N grows; the others: each rank runs the whole config
 
 # Algorithmic work per task by body:
@@ -58,6 +60,7 @@ DEMAND = {
     "mb": {"fma": 8 * 199370695 / 1024, "hbm": 8192},
     "mm": {"fma": 32768, "hbm": 12288},
     "mm_tc": {"hbm": 12288},
+    "mm64": {"fma": 262144, "hbm": 49152},
     "fb": {"fma": 130080, "hbm": 16640},
     "bf": {"fma": 166912, "hbm": 25216},
     "conv": {"fma": 557056, "hbm": 131208},
@@ -81,6 +84,8 @@ def parse():
     ap.add_argument("--arena-kb", type=int, default=0, help="task arena per MTB in KiB (default: preset)")
     ap.add_argument("--producers", type=int, default=0,
                     help="host spawner threads per step (pagoda_taskSpawnShapesMT; default: preset)")
+    ap.add_argument("--task-shmem", type=int, default=-1,
+                    help="override every task's shared-memory request in bytes (Table 5 sweeps)")
     ap.add_argument("--no-resident", action="store_true", help="3DES: stage SP tables per task instead")
     ap.add_argument("--no-const-keys", action="store_true", help="3DES: stage round keys per task instead")
     ap.add_argument("--pool", action="store_true",
@@ -217,16 +222,22 @@ def oracle_tasks(workload: str, n_sample: int):
             return I.conv_inputs(size)
         return I.dct_inputs(size), I.dct_coef()
 
+    if workload == "mm64":
+        A, B = I.mm64_inputs(n_sample)
+        return [(lambda k=k: oracle.mm64(A[k], B[k])) for k in range(n_sample)], \
+            f"{n_sample} 64x64x64 fp32 MM tasks"
     if workload == "mm_tc":
         A, B = I.mm_inputs(n_sample)
         return [(lambda k=k: oracle.mm32_exact(A[k], B[k])) for k in range(n_sample)], \
             f"{n_sample} 32x32x32 MM tasks (fp64-accumulated definition)"
-    if workload in ("tdes", "mb", "mm", "tdes_var"):
-        kind = "tdes" if workload == "tdes_var" else workload
+    if workload in ("tdes", "mb", "mm", "tdes_var", "dct", "dct_noshm", "mm_noshm"):
+        kind = {"tdes_var": "tdes", "dct_noshm": "dct", "mm_noshm": "mm"}.get(workload, workload)
         ph = pool(kind, n_sample, var=workload == "tdes_var")
         what = {"tdes": f"{n_sample} of the 32768 3DES packets (4 KiB, EDE3 ECB)",
                 "mb": f"{n_sample} Mandelbrot tiles of config 1", "mm": f"{n_sample} 32x32x32 fp32 MM tasks",
-                "tdes_var": f"{n_sample} of the irregular (2-64 KiB) 3DES packets"}[workload]
+                "tdes_var": f"{n_sample} of the irregular (2-64 KiB) 3DES packets",
+                "dct": f"{n_sample} DCT8x8 tasks (128x128 images)", "dct_noshm": f"{n_sample} DCT8x8 tasks (128x128 images)",
+                "mm_noshm": f"{n_sample} 32x32x32 fp32 MM tasks"}[workload]
         return [body(kind, ph, k) for k in range(n_sample)], what
     if workload == "mix":
         kinds = I.mix_schedule(n_sample)[0]
@@ -305,15 +316,28 @@ def workload_config(name):
                 "n_tasks": 32768},
         "mm_tc": {"workload": "NEXT-4: configs[2] on the tensor cores (3xTF32 mma.sync), 65536 tasks x 256 threads",
                   "n_tasks": 65536, "threads": 256, "l2": "inputs+outputs 768 MiB > L2"},
+        "dct": {"workload": "Table 5 (NEXT-4): DCT8x8 over 128x128 images, 32768 tasks x 64 threads, 16 KiB shmem "
+                            "(TMA-staged bands of block rows)", "n_tasks": 32768, "threads": 64, "shmem_bytes": 16384,
+                "l2": "inputs+outputs 4 GiB > L2"},
+        "dct_noshm": {"workload": "Table 5 (NEXT-4): DCT8x8 over 128x128 images, 32768 tasks x 64 threads, no shmem "
+                                  "(blocks read from global memory)", "n_tasks": 32768, "threads": 64, "shmem_bytes": 0,
+                      "l2": "inputs+outputs 4 GiB > L2"},
+        "mm_noshm": {"workload": "Table 5 (NEXT-4): configs[2] MM without shmem (A, B read from global memory), "
+                                 "65536 tasks x 256 threads", "n_tasks": 65536, "threads": 256, "shmem_bytes": 0,
+                     "l2": "inputs+outputs 768 MiB > L2"},
+        "mm64": {"workload": "NEXT-4 Table 4's MatrixMul: fp32 64x64x64, 32768 tasks x 256 threads, 32 KiB shmem",
+                 "n_tasks": 32768, "threads": 256, "shmem_bytes": 32768, "l2": "inputs+outputs 1.5 GiB > L2"},
         "tdes_var": {"workload": "NEXT-1 irregular 3DES: 32768 packets log-uniform 2-64 KiB, 128 threads each",
                      "n_tasks": 32768, "l2": "inputs+outputs 1.2 GB > L2"},
     }[name]
 
 
 REF_SAMPLE = {"tdes": 2048, "mb": 512, "mm": 20000, "mix": 2048, "nop": 2048, "c5": 2048, "mpe": 1024,
-              "tdes_var": 512, "mm_tc": 20000}   # --impl reference: tasks per step
+              "tdes_var": 512, "mm_tc": 20000,
+              "dct": 1024, "dct_noshm": 1024, "mm_noshm": 20000, "mm64": 4096}   # --impl reference: tasks per step
 CPU_SAMPLE = {"tdes": 16384, "mb": 1024, "mm": 65536, "mix": 4096, "nop": 16384, "c5": 4096, "mpe": 4096,
-              "tdes_var": 4096, "mm_tc": 65536}  # cpu_baseline sample
+              "tdes_var": 4096, "mm_tc": 65536,
+              "dct": 4096, "dct_noshm": 4096, "mm_noshm": 65536, "mm64": 16384}  # cpu_baseline sample
 
 
 def make_workload(name, resident=False, d=None, device="cuda"):
@@ -327,6 +351,14 @@ def make_workload(name, resident=False, d=None, device="cuda"):
     if name == "mm_tc":
         from paper_conf_ppopp_yehsser17_b200 import tasks as T
         return W.matmul(65536, func=T.MM_TC, device=device)
+    if name == "mm64":
+        return W.matmul64(32768, device=device)
+    if name == "dct":
+        return W.dct(32768, device=device)
+    if name == "dct_noshm":
+        return W.dct(32768, shmem=0, sync=False, device=device)
+    if name == "mm_noshm":
+        return W.matmul(65536, shmem=0, device=device)
     if name == "tdes":   # with resident SP tables a task only stages its 384 B of round keys
         return W.tdes(32768, shmem=512 if resident else 2560, device=device)
     if name == "mb":
@@ -410,6 +442,8 @@ def main():
     dev = d.local
     peaks = measured_peaks()
     w = make_workload(a.workload, use_resident(a), d)
+    if a.task_shmem >= 0:
+        w.shapes[:, 2] = a.task_shmem
     n = w.n
     out = {}
 

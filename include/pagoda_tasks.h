@@ -32,7 +32,9 @@ enum pagoda_func_id {
     PAGODA_CONV = 21,  /* separable 17-tap convolution, 128x128 */
     PAGODA_DCT  = 22,  /* 8x8 DCT-II over 128x128 */
     /* variants */
-    PAGODA_MM_TC = 23  /* the MM task on the tensor cores: 3xTF32 mma.sync (args: pagoda_mm_args) */
+    PAGODA_MM_TC = 23, /* the MM task on the tensor cores: 3xTF32 mma.sync (args: pagoda_mm_args) */
+    PAGODA_MM64 = 24   /* Table 4's MatrixMul size: row-major 64x64x64 fp32 (args: pagoda_mm_args);
+                          stages A and B (32 KiB) when granted >= 32768 bytes and sync */
 };
 
 typedef struct { uint32_t* out; uint32_t* cnt; uint32_t base; uint32_t tag; } pagoda_mark_args;

@@ -449,6 +449,61 @@ __device__ void body_mm(const Env& e, const pagoda_mm_args& a)
     }
 }
 
+/* ------------------------------------------------------------- MM 64x64
+ * Table 4's MatrixMul size ("64 x 64 matrix", shared memory and
+ * barrier used), NEXT-4: C = A B, 64x64x64 fp32, each C[i][j] the fma chain
+ * over k ascending from 0 (oracle orc_mm64).  A and B (16 KiB each) are staged
+ * by TMA when 32 KiB were granted and the TB can synchronise; four independent
+ * chains per thread share each B load, as in body_mm. */
+template <class Env>
+__device__ void body_mm64(const Env& e, const pagoda_mm_args& a)
+{
+    const float* A = a.A;
+    const float* B = a.B;
+    if (e.getSMBytes() >= 32768 && e.canSync()) {
+        float* s = reinterpret_cast<float*>(e.getSMPtr());
+        const int w = e.getBlockTid() >> 5;
+        if (e.getBlockWarps() >= 2) {
+            if (w == 0) e.stage(s, A, 16384);
+            else if (w == 1) e.stage(s + 4096, B, 16384);
+        } else {
+            e.stage(s, A, 16384);
+            e.stage(s + 4096, B, 16384);
+        }
+        e.syncBlock();
+        A = s;
+        B = s + 4096;
+    }
+    const int T = total_threads(e);
+    for (int base = e.getTid(); base < 4096; base += 4 * T) {
+        float acc[4] = {0.0f, 0.0f, 0.0f, 0.0f};
+        int row[4], col[4];
+#pragma unroll
+        for (int q = 0; q < 4; q++) {
+            const int o = min(base + q * T, 4095);   /* past the end: a dummy item */
+            row[q] = o >> 6;
+            col[q] = o & 63;
+        }
+        if ((T & 63) == 0) {   /* the four items share column col[0] */
+#pragma unroll 8
+            for (int k = 0; k < 64; k++) {
+                const float b = B[k * 64 + col[0]];
+#pragma unroll
+                for (int q = 0; q < 4; q++) acc[q] = __fmaf_rn(A[row[q] * 64 + k], b, acc[q]);
+            }
+        } else {
+#pragma unroll 4
+            for (int k = 0; k < 64; k++) {
+#pragma unroll
+                for (int q = 0; q < 4; q++) acc[q] = __fmaf_rn(A[row[q] * 64 + k], B[k * 64 + col[q]], acc[q]);
+            }
+        }
+#pragma unroll
+        for (int q = 0; q < 4; q++)
+            if (base + q * T < 4096) a.C[base + q * T] = acc[q];
+    }
+}
+
 /* ------------------------------------------------------------- MM, tensor cores
  * NEXT-4: the same C = A B (32x32x32 fp32) on the tensor cores
  * as 3xTF32: x = hi + lo with hi = tf32(x) and lo = tf32(x - hi), and
@@ -668,51 +723,76 @@ __device__ void body_conv(const Env& e, const pagoda_conv_args& a)
 /* ------------------------------------------------------------- DCT
  * CUDA SDK DCT8x8 [21]: per 8x8 block
  * T[u][y] = sum_x C[u][x] X[x][y], Y[u][v] = sum_y T[u][y] C[v][y].
- * Work item (block, u): one thread computes T[u][*] and Y[u][*]. */
+ * Work item (block, u): one thread computes T[u][*] and Y[u][*] of the block
+ * whose top-left sample is X (row stride 128) into Y (row u of the output block). */
+__device__ __forceinline__ void dct_item(const pagoda_dct_args& a, const float* X, int u, float* Y)
+{
+    /* row x of the block arrives as two float4; the 8 chains T[u][*] advance together
+     * (each still accumulates over x ascending) */
+    float Tu[8] = {0.0f, 0.0f, 0.0f, 0.0f, 0.0f, 0.0f, 0.0f, 0.0f};
+#pragma unroll
+    for (int x = 0; x < 8; x++) {
+        const float cu = a.coef[u * 8 + x];
+        const float4 lo = *reinterpret_cast<const float4*>(X + x * 128);
+        const float4 hi = *reinterpret_cast<const float4*>(X + x * 128 + 4);
+        Tu[0] = __fmaf_rn(cu, lo.x, Tu[0]);
+        Tu[1] = __fmaf_rn(cu, lo.y, Tu[1]);
+        Tu[2] = __fmaf_rn(cu, lo.z, Tu[2]);
+        Tu[3] = __fmaf_rn(cu, lo.w, Tu[3]);
+        Tu[4] = __fmaf_rn(cu, hi.x, Tu[4]);
+        Tu[5] = __fmaf_rn(cu, hi.y, Tu[5]);
+        Tu[6] = __fmaf_rn(cu, hi.z, Tu[6]);
+        Tu[7] = __fmaf_rn(cu, hi.w, Tu[7]);
+    }
+    float Yv[8];
+#pragma unroll
+    for (int v = 0; v < 8; v++) {
+        const float4 clo = *reinterpret_cast<const float4*>(a.coef + v * 8);
+        const float4 chi = *reinterpret_cast<const float4*>(a.coef + v * 8 + 4);
+        float acc = 0.0f;
+        acc = __fmaf_rn(Tu[0], clo.x, acc);
+        acc = __fmaf_rn(Tu[1], clo.y, acc);
+        acc = __fmaf_rn(Tu[2], clo.z, acc);
+        acc = __fmaf_rn(Tu[3], clo.w, acc);
+        acc = __fmaf_rn(Tu[4], chi.x, acc);
+        acc = __fmaf_rn(Tu[5], chi.y, acc);
+        acc = __fmaf_rn(Tu[6], chi.z, acc);
+        acc = __fmaf_rn(Tu[7], chi.w, acc);
+        Yv[v] = acc;
+    }
+    *reinterpret_cast<float4*>(Y) = make_float4(Yv[0], Yv[1], Yv[2], Yv[3]);
+    *reinterpret_cast<float4*>(Y + 4) = make_float4(Yv[4], Yv[5], Yv[6], Yv[7]);
+}
+
+/* Table 5: with >= 4 KiB of shared memory granted and a barrier, a TB
+ * stages bands of whole 8-row block rows (4 KiB each, as many as the grant holds) with
+ * TMA bulk copies and transforms them from shared memory; TB j takes bands j, j + nb, ...
+ * Otherwise every item reads its block from global memory.  Same arithmetic either way. */
 template <class Env>
 __device__ void body_dct(const Env& e, const pagoda_dct_args& a)
 {
+    if (e.getSMBytes() >= 4096 && e.canSync()) {
+        float* s = reinterpret_cast<float*>(e.getSMPtr());
+        const int R = min(16, (int)(e.getSMBytes() >> 12));      /* block rows per band */
+        const int nbands = (16 + R - 1) / R, nb = e.getNumBlocks();
+        const int n = tb_threads(e), bt = e.getBlockTid(), w = bt >> 5, W = e.getBlockWarps();
+        for (int band = e.getBlockIdx(); band < nbands; band += nb) {
+            const int r0 = band * R, rows = min(R, 16 - r0);
+            for (int r = w; r < rows; r += W) e.stage(s + r * 1024, a.img + (r0 + r) * 1024, 4096);
+            e.syncBlock();
+            for (int item = bt; item < rows * 128; item += n) {
+                const int rb = item >> 7, bx = (item >> 3) & 15, u = item & 7;
+                dct_item(a, s + rb * 1024 + bx * 8, u, a.out + ((r0 + rb) * 8 + u) * 128 + bx * 8);
+            }
+            e.syncBlock();   /* before the next band overwrites the stage */
+        }
+        return;
+    }
     const int T = total_threads(e);
     for (int item = e.getTid(); item < 256 * 8; item += T) {
         const int blk = item >> 3, u = item & 7;
         const int by = blk >> 4, bx = blk & 15;
-        const float* X = a.img + (by * 8) * 128 + bx * 8;
-        /* row x of the block arrives as two float4; the 8 chains T[u][*] advance together
-         * (each still accumulates over x ascending) */
-        float Tu[8] = {0.0f, 0.0f, 0.0f, 0.0f, 0.0f, 0.0f, 0.0f, 0.0f};
-#pragma unroll
-        for (int x = 0; x < 8; x++) {
-            const float cu = a.coef[u * 8 + x];
-            const float4 lo = *reinterpret_cast<const float4*>(X + x * 128);
-            const float4 hi = *reinterpret_cast<const float4*>(X + x * 128 + 4);
-            Tu[0] = __fmaf_rn(cu, lo.x, Tu[0]);
-            Tu[1] = __fmaf_rn(cu, lo.y, Tu[1]);
-            Tu[2] = __fmaf_rn(cu, lo.z, Tu[2]);
-            Tu[3] = __fmaf_rn(cu, lo.w, Tu[3]);
-            Tu[4] = __fmaf_rn(cu, hi.x, Tu[4]);
-            Tu[5] = __fmaf_rn(cu, hi.y, Tu[5]);
-            Tu[6] = __fmaf_rn(cu, hi.z, Tu[6]);
-            Tu[7] = __fmaf_rn(cu, hi.w, Tu[7]);
-        }
-        float Yv[8];
-#pragma unroll
-        for (int v = 0; v < 8; v++) {
-            const float4 clo = *reinterpret_cast<const float4*>(a.coef + v * 8);
-            const float4 chi = *reinterpret_cast<const float4*>(a.coef + v * 8 + 4);
-            float acc = 0.0f;
-            acc = __fmaf_rn(Tu[0], clo.x, acc);
-            acc = __fmaf_rn(Tu[1], clo.y, acc);
-            acc = __fmaf_rn(Tu[2], clo.z, acc);
-            acc = __fmaf_rn(Tu[3], clo.w, acc);
-            acc = __fmaf_rn(Tu[4], chi.x, acc);
-            acc = __fmaf_rn(Tu[5], chi.y, acc);
-            acc = __fmaf_rn(Tu[6], chi.z, acc);
-            acc = __fmaf_rn(Tu[7], chi.w, acc);
-            Yv[v] = acc;
-        }
-        float* Y = a.out + (by * 8 + u) * 128 + bx * 8;
-        *reinterpret_cast<float4*>(Y) = make_float4(Yv[0], Yv[1], Yv[2], Yv[3]);
-        *reinterpret_cast<float4*>(Y + 4) = make_float4(Yv[4], Yv[5], Yv[6], Yv[7]);
+        dct_item(a, a.img + (by * 8) * 128 + bx * 8, u, a.out + (by * 8 + u) * 128 + bx * 8);
     }
 }
 
@@ -736,13 +816,14 @@ __device__ __forceinline__ bool run_body(int func_id, const Env& e, const void* 
     case PAGODA_CONV: body_conv(e, *static_cast<const pagoda_conv_args*>(args)); return true;
     case PAGODA_DCT: body_dct(e, *static_cast<const pagoda_dct_args*>(args)); return true;
     case PAGODA_MM_TC: body_mm_tc(e, *static_cast<const pagoda_mm_args*>(args)); return true;
+    case PAGODA_MM64: body_mm64(e, *static_cast<const pagoda_mm_args*>(args)); return true;
     default: return false;
     }
 }
 
 __host__ __device__ inline bool known_func(int f)
 {
-    return (f >= PAGODA_NOP && f <= PAGODA_GATE) || (f >= PAGODA_MB && f <= PAGODA_MM_TC);
+    return (f >= PAGODA_NOP && f <= PAGODA_GATE) || (f >= PAGODA_MB && f <= PAGODA_MM64);
 }
 
 } // namespace pagoda

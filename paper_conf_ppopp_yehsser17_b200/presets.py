@@ -14,6 +14,10 @@ PRESETS = {
     "mpe": {"mtbs_per_sm": 2, "arena_bytes": 40 * 1024, "resident": True},
     "tdes_var": {"mtbs_per_sm": 2, "arena_bytes": 40 * 1024, "resident": True},
     "mm_tc": {"mtbs_per_sm": 4, "arena_bytes": 48 * 1024, "resident": False},
+    "mm64": {"mtbs_per_sm": 2, "arena_bytes": 96 * 1024, "resident": False},        # 3 tasks x 32 KiB per MTB
+    "mm_noshm": {"mtbs_per_sm": 4, "arena_bytes": 48 * 1024, "resident": False},    # Table 5 ablation
+    "dct": {"mtbs_per_sm": 2, "arena_bytes": 96 * 1024, "resident": False},         # 6 tasks x 16 KiB per MTB
+    "dct_noshm": {"mtbs_per_sm": 2, "arena_bytes": 96 * 1024, "resident": False},
 }
 
 RESIDENT_TDES = 0x4   # include/pagoda.h

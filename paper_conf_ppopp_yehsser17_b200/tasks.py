@@ -8,9 +8,10 @@ import numpy as np
 NOP, MARK, TID, BAR, SMEM, SPIN, GATE = 0, 1, 2, 3, 4, 5, 6
 MB, TDES, MM, FB, BF, CONV, DCT = 16, 17, 18, 19, 20, 21, 22
 MM_TC = 23
+MM64 = 24   # Table 4's 64x64 MatrixMul (NEXT-4)
 
 NAMES = {NOP: "nop", MARK: "mark", TID: "tid", BAR: "bar", SMEM: "smem", SPIN: "spin", GATE: "gate",
-         MB: "mb", TDES: "tdes", MM: "mm", FB: "fb", BF: "bf", CONV: "conv", DCT: "dct", MM_TC: "mm_tc"}
+         MB: "mb", TDES: "tdes", MM: "mm", FB: "fb", BF: "bf", CONV: "conv", DCT: "dct", MM_TC: "mm_tc", MM64: "mm64"}
 
 _p = "<u8"
 ARGS = {
@@ -25,6 +26,7 @@ ARGS = {
     TDES: np.dtype([("inp", _p), ("out", _p), ("tables", _p), ("nblk", "<u4"), ("pad", "<u4")]),
     MM: np.dtype([("A", _p), ("B", _p), ("C", _p)]),
     MM_TC: np.dtype([("A", _p), ("B", _p), ("C", _p)]),
+    MM64: np.dtype([("A", _p), ("B", _p), ("C", _p)]),
     FB: np.dtype([("r", _p), ("H", _p), ("F", _p), ("y", _p), ("scratch", _p)]),
     BF: np.dtype([("x", _p), ("h", _p), ("w", _p), ("out", _p)]),
     CONV: np.dtype([("img", _p), ("krow", _p), ("kcol", _p), ("out", _p), ("scratch", _p)]),

@@ -102,6 +102,19 @@ def matmul(n_tasks=65536, device="cuda", threads=256, shmem=8192, first=0, func=
                     {"C": (dC, np.float32, (n_tasks, 32, 32))}, [dA, dB, dC], 2 * A.nbytes, A.nbytes)
 
 
+# ---------------------------------------------------------------- Table 4's 64x64 MM (NEXT-4)
+def matmul64(n_tasks=32768, device="cuda", threads=256, shmem=32768, first=0, integer=False):
+    """32K MatrixMul tasks of 64x64x64 fp32 (Table 4); A, B staged in 32 KiB of shmem."""
+    A, B = I.mm64_inputs(n_tasks, first, integer=integer)
+    dA, dB = _dev(A, device), _dev(B, device)
+    dC = _zeros(A.nbytes, device)
+    a = T.records(T.MM64, n_tasks)
+    off = np.arange(n_tasks) * 16384
+    a["A"], a["B"], a["C"] = dA.data_ptr() + off, dB.data_ptr() + off, dC.data_ptr() + off
+    return Workload("mm64", _shapes(n_tasks, threads, 1, shmem, True, T.MM64), T.to_raw(a), {"A": A, "B": B},
+                    {"C": (dC, np.float32, (n_tasks, 64, 64))}, [dA, dB, dC], 2 * A.nbytes, A.nbytes)
+
+
 # ---------------------------------------------------------------- config 4: mix
 def mix(n_tasks=32768, device="cuda", first=0):
     """FB / BF / CONV / DCT in a seeded random order; threads uniform in
@@ -163,6 +176,21 @@ def mix(n_tasks=32768, device="cuda", first=0):
     host["dct"] = (im, coef); outs["dct"] = (dout2, np.float32, (n, 128, 128)); keep += [dim_, dco, dout2]
     in_b += im.nbytes; out_b += im.nbytes
     return Workload("mix", shapes, raw, host, outs, keep, in_b, out_b)
+
+
+# ---------------------------------------------------------------- Table 5: DCT with / without shmem
+def dct(n_tasks=32768, device="cuda", threads=64, n_tb=1, shmem=16384, sync=True, first=0):
+    """Table 5: 32K DCT8x8 tasks of 64 threads over 128x128 images.  With
+    shmem >= 4096 and sync the body stages bands of block rows by TMA; shmem=0 reads global."""
+    im = I.dct_inputs(n_tasks, first)
+    coef = I.dct_coef()
+    dim_, dco = _dev(im, device), _dev(coef, device)
+    dout = _zeros(im.nbytes, device)
+    a = T.records(T.DCT, n_tasks)
+    a["img"], a["coef"], a["out"] = dim_.data_ptr() + np.arange(n_tasks) * 65536, dco.data_ptr(), \
+        dout.data_ptr() + np.arange(n_tasks) * 65536
+    return Workload("dct", _shapes(n_tasks, threads, n_tb, shmem, sync, T.DCT), T.to_raw(a), {"img": im, "coef": coef},
+                    {"out": (dout, np.float32, (n_tasks, 128, 128))}, [dim_, dco, dout], im.nbytes, im.nbytes)
 
 
 def nop(n_tasks, threads=128, n_tb=1, shmem=0, sync=False):

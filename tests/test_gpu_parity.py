@@ -147,6 +147,77 @@ def test_mm_tc_integer_exact_and_full_size():
     _mm_tc_check(w, out, list(rng.choice(65536, 256, replace=False)) + [0, 65535])
 
 
+# ---------------------------------------------------------------- DCT with / without shmem (Table 5, NEXT-4)
+def _dct_check(w, out, ks):
+    for k in ks:
+        ref = oracle.dct(w.host["img"][k], w.host["coef"])
+        assert fp32_close(out[k], ref) <= TOL and np.array_equal(out[k], ref), k
+
+
+# (threads, n_tb, shmem, sync): one band of 16 block rows; bands of 4, 3 (ragged last band: 16 = 5*3 + 1)
+# and 1 block row; several TBs sharing the bands (more TBs than bands too); 1-warp TBs without a
+# barrier (canSync by construction); no shmem; a grant below one block row (global path)
+DCT_SHAPES = [(64, 1, 16384, True), (64, 1, 65536, True), (128, 1, 12288, True), (32, 1, 4096, False),
+              (96, 3, 8192, True), (64, 20, 4096, True), (64, 1, 0, False), (256, 1, 2048, True)]
+
+
+@pytest.mark.parametrize("threads,n_tb,shmem,sync", DCT_SHAPES)
+def test_dct_table5_small(threads, n_tb, shmem, sync):
+    w = W.dct(200, threads=threads, n_tb=n_tb, shmem=shmem, sync=sync)
+    _dct_check(w, run(w, arena_bytes=96 * 1024)["out"], range(200))
+
+
+@pytest.mark.parametrize("name", ["dct", "dct_noshm"])
+def test_dct_table5_full_size(name):
+    w = W.dct(32768, shmem=16384 if name == "dct" else 0, sync=name == "dct")
+    out = run(w, **ctx_kwargs(name))["out"]   # the bench's launch configuration
+    rng = np.random.default_rng(11)
+    _dct_check(w, out, list(rng.choice(32768, 96, replace=False)) + [0, 32767])
+
+
+def test_dct_table5_naive_baseline():
+    w = W.dct(300, threads=64, shmem=16384)
+    naive_run(0, w.shapes, w.args, 32)
+    _dct_check(w, w.outputs()["out"], range(300))
+
+
+def _mm64_check(w, out, ks):
+    for k in ks:
+        ref = oracle.mm64(w.host["A"][k], w.host["B"][k])
+        assert fp32_close(out[k], ref) <= TOL and np.array_equal(out[k], ref), k
+
+
+# staged (32 KiB, sync), global (no shmem), threads not a multiple of 64 (own column per item),
+# 1-warp TBs (stage both operands), a grant below 32 KiB (global path), 1024 threads
+@pytest.mark.parametrize("shmem,threads,sync", [(32768, 256, True), (0, 256, False), (32768, 96, True),
+                                                (32768, 32, False), (16384, 128, True), (32768, 1024, True)])
+def test_mm64_small(shmem, threads, sync):
+    w = W.matmul64(150, shmem=shmem, threads=threads)
+    w.shapes[:, 3] = int(sync)
+    _mm64_check(w, run(w, arena_bytes=96 * 1024)["C"], range(150))
+
+
+def test_mm64_integer_exact_naive_and_full_size():
+    w = W.matmul64(40, integer=True)    # integer inputs: every partial sum exact in fp32
+    out = run(w, arena_bytes=96 * 1024)["C"]
+    for k in range(40):
+        assert np.array_equal(out[k].astype(np.int64), w.host["A"][k].astype(np.int64) @ w.host["B"][k].astype(np.int64))
+    w = W.matmul64(200)
+    naive_run(0, w.shapes, w.args, 32)
+    _mm64_check(w, w.outputs()["C"], range(200))
+    w = W.matmul64(32768)
+    out = run(w, **ctx_kwargs("mm64"))["C"]   # the bench's launch configuration
+    rng = np.random.default_rng(17)
+    _mm64_check(w, out, list(rng.choice(32768, 96, replace=False)) + [0, 32767])
+
+
+def test_mm_noshm_full_size():
+    w = W.matmul(65536, shmem=0)
+    out = run(w, **ctx_kwargs("mm_noshm"))["C"]
+    rng = np.random.default_rng(13)
+    _mm_check(w, out, list(rng.choice(65536, 128, replace=False)) + [0, 65535])
+
+
 # ---------------------------------------------------------------- mix (config 4)
 def _mix_check(w, out, frac=1.0, seed=0):
     rng = np.random.default_rng(seed)
