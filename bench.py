@@ -316,8 +316,8 @@ def workload_config(name):
                 "n_tasks": 32768},
         "mm_tc": {"workload": "NEXT-4: configs[2] on the tensor cores (3xTF32 mma.sync), 65536 tasks x 256 threads",
                   "n_tasks": 65536, "threads": 256, "l2": "inputs+outputs 768 MiB > L2"},
-        "dct": {"workload": "Table 5 (NEXT-4): DCT8x8 over 128x128 images, 32768 tasks x 64 threads, 16 KiB shmem "
-                            "(TMA-staged bands of block rows)", "n_tasks": 32768, "threads": 64, "shmem_bytes": 16384,
+        "dct": {"workload": "Table 5 (NEXT-4): DCT8x8 over 128x128 images, 32768 tasks x 64 threads, 8 KiB shmem "
+                            "(TMA-staged bands of block rows)", "n_tasks": 32768, "threads": 64, "shmem_bytes": 8192,
                 "l2": "inputs+outputs 4 GiB > L2"},
         "dct_noshm": {"workload": "Table 5 (NEXT-4): DCT8x8 over 128x128 images, 32768 tasks x 64 threads, no shmem "
                                   "(blocks read from global memory)", "n_tasks": 32768, "threads": 64, "shmem_bytes": 0,

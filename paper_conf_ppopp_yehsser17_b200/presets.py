@@ -16,7 +16,7 @@ PRESETS = {
     "mm_tc": {"mtbs_per_sm": 4, "arena_bytes": 48 * 1024, "resident": False},
     "mm64": {"mtbs_per_sm": 2, "arena_bytes": 96 * 1024, "resident": False},        # 3 tasks x 32 KiB per MTB
     "mm_noshm": {"mtbs_per_sm": 4, "arena_bytes": 48 * 1024, "resident": False},    # Table 5 ablation
-    "dct": {"mtbs_per_sm": 2, "arena_bytes": 96 * 1024, "resident": False},         # 6 tasks x 16 KiB per MTB
+    "dct": {"mtbs_per_sm": 2, "arena_bytes": 96 * 1024, "resident": False},         # 8 KiB grants (sweep: 4/8/16/32 KiB)
     "dct_noshm": {"mtbs_per_sm": 2, "arena_bytes": 96 * 1024, "resident": False},
 }
 

@@ -179,7 +179,7 @@ def mix(n_tasks=32768, device="cuda", first=0):
 
 
 # ---------------------------------------------------------------- Table 5: DCT with / without shmem
-def dct(n_tasks=32768, device="cuda", threads=64, n_tb=1, shmem=16384, sync=True, first=0):
+def dct(n_tasks=32768, device="cuda", threads=64, n_tb=1, shmem=8192, sync=True, first=0):
     """Table 5: 32K DCT8x8 tasks of 64 threads over 128x128 images.  With
     shmem >= 4096 and sync the body stages bands of block rows by TMA; shmem=0 reads global."""
     im = I.dct_inputs(n_tasks, first)

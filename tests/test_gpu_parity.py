@@ -169,7 +169,7 @@ def test_dct_table5_small(threads, n_tb, shmem, sync):
 
 @pytest.mark.parametrize("name", ["dct", "dct_noshm"])
 def test_dct_table5_full_size(name):
-    w = W.dct(32768, shmem=16384 if name == "dct" else 0, sync=name == "dct")
+    w = W.dct(32768, shmem=8192 if name == "dct" else 0, sync=name == "dct")
     out = run(w, **ctx_kwargs(name))["out"]   # the bench's launch configuration
     rng = np.random.default_rng(11)
     _dct_check(w, out, list(rng.choice(32768, 96, replace=False)) + [0, 32767])
