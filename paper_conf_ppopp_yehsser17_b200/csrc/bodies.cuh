@@ -730,9 +730,11 @@ __device__ __forceinline__ void dct_item(const pagoda_dct_args& a, const float* 
     /* row x of the block arrives as two float4; the 8 chains T[u][*] advance together
      * (each still accumulates over x ascending) */
     float Tu[8] = {0.0f, 0.0f, 0.0f, 0.0f, 0.0f, 0.0f, 0.0f, 0.0f};
+    float4 cq;   /* C[u][x..x+3], one vector load per four x (the load pipe is the limit) */
 #pragma unroll
     for (int x = 0; x < 8; x++) {
-        const float cu = a.coef[u * 8 + x];
+        if ((x & 3) == 0) cq = *reinterpret_cast<const float4*>(a.coef + u * 8 + x);
+        const float cu = (x & 3) == 0 ? cq.x : (x & 3) == 1 ? cq.y : (x & 3) == 2 ? cq.z : cq.w;
         const float4 lo = *reinterpret_cast<const float4*>(X + x * 128);
         const float4 hi = *reinterpret_cast<const float4*>(X + x * 128 + 4);
         Tu[0] = __fmaf_rn(cu, lo.x, Tu[0]);

@@ -16,7 +16,7 @@ python scripts/ncu_summary.py $F/tdes_full.ncu-rep > $F/ncu_tdes_full.txt 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:master -s 3 -c 1 -o $F/mm_full \
   python bench.py --workload mm --prespawn --steps 1 --warmup 3 --no-naive --no-cpu --quick > $F/mm_full.log 2>&1
 python scripts/ncu_summary.py $F/mm_full.ncu-rep > $F/ncu_mm_full.txt 2>&1
-rm -f $F/*.ncu-rep
+find gpurun_out/final -name "*.ncu-rep" -delete
 timeout 600 python scripts/probe_busy.py mm tdes nop mb > $F/busy.jsonl 2>&1
 timeout 300 python scripts/probe_session_overhead.py > $F/session_overhead.json 2>&1
 timeout 600 python scripts/probe_runtime.py > $F/runtime.json 2>&1
