@@ -88,6 +88,7 @@ def parse():
                     help="override every task's shared-memory request in bytes (Table 5 sweeps)")
     ap.add_argument("--no-resident", action="store_true", help="3DES: stage SP tables per task instead")
     ap.add_argument("--no-const-keys", action="store_true", help="3DES: stage round keys per task instead")
+    ap.add_argument("--no-const-coef", action="store_true", help="DCT: coefficients from global memory, not registered")
     ap.add_argument("--pool", action="store_true",
                     help="one process drives every visible GPU through the least-loaded pool (no torchrun)")
     ap.add_argument("--prespawn", action="store_true",
@@ -475,6 +476,8 @@ def main():
     p = PG.Pagoda(device=dev, **ctx_config(a, PG))
     if use_resident(a) and w.tdes_tables and not a.no_const_keys:
         p.tdes_register(w.tdes_tables)   # resident round keys (constant bank) for the resident SP tables
+    if w.dct_coef and not a.no_const_coef:
+        p.dct_register(w.dct_coef)       # Table 5 workloads: second-pass coefficients from the constant bank
 
     producers = a.producers or PRESETS[a.workload].get("producers", 1)
 
@@ -580,7 +583,8 @@ def main():
                                                           "resident_tdes_tables": use_resident(a),
                                                           "spread_first_claims": bool(PRESETS[a.workload].get("spread")),
                                                           "resident_tdes_keys": bool(use_resident(a) and w.tdes_tables
-                                                                                     and not a.no_const_keys)},
+                                                                                     and not a.no_const_keys),
+                                                          "registered_dct_coef": bool(w.dct_coef and not a.no_const_coef)},
                                                       "task_shmem_bytes": int(w.shapes[0][2])},
             "gpu_launches": a.steps, "host_ms_per_step": 1e3 * host_total / a.steps,
             "host_tasks_per_s": all_tasks / host_total, "clocks": clk}

@@ -253,6 +253,15 @@ int pagoda_tdes_tables(const uint8_t key24[24], void* dst);
  * Returns 0, -EINVAL (unreadable pointer), -EBUSY, -EIO. */
 int pagoda_tdes_register(pagoda_ctx* ctx, const void* dev_tables);
 
+/* Register a DCT coefficient matrix (pagoda_dct_args.coef: 64 fp32 C[u][x], device memory) as
+ * resident task-class data: DCT tasks whose coef pointer equals dev_coef read the second
+ * pass's coefficients from the MasterKernel's constant bank (same values, same arithmetic:
+ * outputs are bit-identical).  The matrix is copied at registration; later writes to dev_coef
+ * are not seen.  One matrix per device and process; NULL unregisters.  Call while the context
+ * is stopped: -EBUSY otherwise.  Returns 0, -EINVAL (unreadable pointer), -EBUSY, -EIO.
+ * Table 5 / DESIGN.md "DCT". */
+int pagoda_dct_register(pagoda_ctx* ctx, const float* dev_coef);
+
 /* Naive baseline (the paper's CUDA-HyperQ): launch
  * each task as its own kernel <<<n_tb, threads, shmem>>> of the same body on
  * streams[i % n_streams] (n_streams <= 32), from the calling thread, then

@@ -725,6 +725,14 @@ __device__ void body_conv(const Env& e, const pagoda_conv_args& a)
  * T[u][y] = sum_x C[u][x] X[x][y], Y[u][v] = sum_y T[u][y] C[v][y].
  * Work item (block, u): one thread computes T[u][*] and Y[u][*] of the block
  * whose top-left sample is X (row stride 128) into Y (row u of the output block). */
+/* A registered coefficient matrix (pagoda_dct_register): C in this module's constant bank,
+ * used by DCT tasks whose coef pointer equals the registered one.  The second pass then reads
+ * C[v][y] as an FFMA constant operand (v, y unrolled) instead of 16 uniform vector loads per
+ * item; 0 = none registered (and always 0 in the baselines' translation unit). */
+static __constant__ float c_dct_coef[64];
+static __constant__ unsigned long long c_dct_coef_ptr;
+
+template <bool kConstCoef>
 __device__ __forceinline__ void dct_item(const pagoda_dct_args& a, const float* X, int u, float* Y)
 {
     /* row x of the block arrives as two float4; the 8 chains T[u][*] advance together
@@ -749,8 +757,14 @@ __device__ __forceinline__ void dct_item(const pagoda_dct_args& a, const float* 
     float Yv[8];
 #pragma unroll
     for (int v = 0; v < 8; v++) {
-        const float4 clo = *reinterpret_cast<const float4*>(a.coef + v * 8);
-        const float4 chi = *reinterpret_cast<const float4*>(a.coef + v * 8 + 4);
+        float4 clo, chi;
+        if (kConstCoef) {
+            clo = make_float4(c_dct_coef[v * 8 + 0], c_dct_coef[v * 8 + 1], c_dct_coef[v * 8 + 2], c_dct_coef[v * 8 + 3]);
+            chi = make_float4(c_dct_coef[v * 8 + 4], c_dct_coef[v * 8 + 5], c_dct_coef[v * 8 + 6], c_dct_coef[v * 8 + 7]);
+        } else {
+            clo = *reinterpret_cast<const float4*>(a.coef + v * 8);
+            chi = *reinterpret_cast<const float4*>(a.coef + v * 8 + 4);
+        }
         float acc = 0.0f;
         acc = __fmaf_rn(Tu[0], clo.x, acc);
         acc = __fmaf_rn(Tu[1], clo.y, acc);
@@ -770,8 +784,8 @@ __device__ __forceinline__ void dct_item(const pagoda_dct_args& a, const float* 
  * stages bands of whole 8-row block rows (4 KiB each, as many as the grant holds) with
  * TMA bulk copies and transforms them from shared memory; TB j takes bands j, j + nb, ...
  * Otherwise every item reads its block from global memory.  Same arithmetic either way. */
-template <class Env>
-__device__ void body_dct(const Env& e, const pagoda_dct_args& a)
+template <bool kConstCoef, class Env>
+__device__ void body_dct_t(const Env& e, const pagoda_dct_args& a)
 {
     if (e.getSMBytes() >= 4096 && e.canSync()) {
         float* s = reinterpret_cast<float*>(e.getSMPtr());
@@ -784,7 +798,7 @@ __device__ void body_dct(const Env& e, const pagoda_dct_args& a)
             e.syncBlock();
             for (int item = bt; item < rows * 128; item += n) {
                 const int rb = item >> 7, bx = (item >> 3) & 15, u = item & 7;
-                dct_item(a, s + rb * 1024 + bx * 8, u, a.out + ((r0 + rb) * 8 + u) * 128 + bx * 8);
+                dct_item<kConstCoef>(a, s + rb * 1024 + bx * 8, u, a.out + ((r0 + rb) * 8 + u) * 128 + bx * 8);
             }
             e.syncBlock();   /* before the next band overwrites the stage */
         }
@@ -794,8 +808,15 @@ __device__ void body_dct(const Env& e, const pagoda_dct_args& a)
     for (int item = e.getTid(); item < 256 * 8; item += T) {
         const int blk = item >> 3, u = item & 7;
         const int by = blk >> 4, bx = blk & 15;
-        dct_item(a, a.img + (by * 8) * 128 + bx * 8, u, a.out + (by * 8 + u) * 128 + bx * 8);
+        dct_item<kConstCoef>(a, a.img + (by * 8) * 128 + bx * 8, u, a.out + (by * 8 + u) * 128 + bx * 8);
     }
+}
+
+template <class Env>
+__device__ void body_dct(const Env& e, const pagoda_dct_args& a)
+{
+    if (c_dct_coef_ptr != 0 && (unsigned long long)a.coef == c_dct_coef_ptr) body_dct_t<true>(e, a);
+    else body_dct_t<false>(e, a);
 }
 
 /* ------------------------------------------------------------- dispatch */

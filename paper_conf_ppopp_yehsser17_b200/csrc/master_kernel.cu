@@ -1522,6 +1522,14 @@ cudaError_t set_tdes_const_keys(const void* keys384, uint64_t tables_ptr)
     return e;
 }
 
+/* host side (runtime.cu): the registered DCT coefficient matrix of this module's MasterKernel */
+cudaError_t set_dct_const_coef(const void* coef256, uint64_t coef_ptr)
+{
+    cudaError_t e = cudaMemcpyToSymbol(c_dct_coef, coef256, sizeof(c_dct_coef));
+    if (e == cudaSuccess) e = cudaMemcpyToSymbol(c_dct_coef_ptr, &coef_ptr, sizeof(coef_ptr));
+    return e;
+}
+
 /* host-side launcher (called by runtime.cu) */
 cudaError_t launch_master(int mtbs_per_sm, int n_mtb, size_t smem_bytes, cudaStream_t stream, MkParams* params,
                           int* regs_out)

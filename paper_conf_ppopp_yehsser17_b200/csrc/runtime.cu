@@ -38,6 +38,7 @@ namespace pagoda {
 cudaError_t launch_master(int mtbs_per_sm, int n_mtb, size_t smem_bytes, cudaStream_t stream, MkParams* params,
                           int* regs_out);
 cudaError_t set_tdes_const_keys(const void* keys384, uint64_t tables_ptr);
+cudaError_t set_dct_const_coef(const void* coef256, uint64_t coef_ptr);
 }
 using namespace pagoda;
 
@@ -938,6 +939,23 @@ int pagoda_tdes_register(pagoda_ctx* c, const void* dev_tables)
         ptr = (uint64_t)(uintptr_t)dev_tables;
     }
     return set_tdes_const_keys(keys, ptr) == cudaSuccess ? 0 : -EIO;
+}
+
+int pagoda_dct_register(pagoda_ctx* c, const float* dev_coef)
+{
+    if (!c) return -EINVAL;
+    if (c->running.load()) return -EBUSY;
+    cudaSetDevice(c->device);
+    float coef[64] = {0};
+    uint64_t ptr = 0;
+    if (dev_coef) {
+        if (cudaMemcpy(coef, dev_coef, sizeof coef, cudaMemcpyDeviceToHost) != cudaSuccess) {
+            cudaGetLastError();
+            return -EINVAL;
+        }
+        ptr = (uint64_t)(uintptr_t)dev_coef;
+    }
+    return set_dct_const_coef(coef, ptr) == cudaSuccess ? 0 : -EIO;
 }
 
 int pagoda_read_counters(pagoda_ctx* c, uint64_t* out, int n)

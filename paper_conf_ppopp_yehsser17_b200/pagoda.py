@@ -83,6 +83,7 @@ def lib() -> C.CDLL:
         L.pagoda_naive_run.argtypes = [I, I, P, P, SZ, SZ, I, C.POINTER(I64)]
         L.pagoda_pingpong.argtypes = [I, I, P]
         L.pagoda_tdes_register.argtypes = [P, P]
+        L.pagoda_dct_register.argtypes = [P, P]
         L.pagoda_fused_run.argtypes = [I, I, P, P, SZ, SZ, I, C.POINTER(I64), C.POINTER(C.c_float)]
         L.pagoda_pool_init.argtypes = [I, P, C.POINTER(pagoda_config), C.POINTER(P)]
         L.pagoda_pool_pick.argtypes = [P, I]
@@ -230,6 +231,10 @@ class Pagoda:
     def tdes_register(self, dev_tables) -> int:
         """Resident round keys for 3DES tasks using this tables pointer (context stopped)."""
         return _check(lib().pagoda_tdes_register(self.h, dev_tables), "pagoda_tdes_register")
+
+    def dct_register(self, dev_coef) -> int:
+        """Constant-bank DCT coefficients for DCT tasks using this coef pointer (context stopped)."""
+        return _check(lib().pagoda_dct_register(self.h, dev_coef), "pagoda_dct_register")
 
     def info(self) -> pagoda_info:
         i = pagoda_info()

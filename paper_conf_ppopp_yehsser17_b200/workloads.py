@@ -42,6 +42,7 @@ class Workload:
         self._outs, self._keep = outs, keep
         self.in_bytes, self.out_bytes = in_bytes, out_bytes   # algorithmic HBM bytes per run
         self.tdes_tables = None   # device pointer of the 3DES tables its tasks use (pagoda_tdes_register)
+        self.dct_coef = None      # device pointer of the DCT coefficients its tasks use (pagoda_dct_register)
 
     @property
     def n(self):
@@ -189,8 +190,10 @@ def dct(n_tasks=32768, device="cuda", threads=64, n_tb=1, shmem=8192, sync=True,
     a = T.records(T.DCT, n_tasks)
     a["img"], a["coef"], a["out"] = dim_.data_ptr() + np.arange(n_tasks) * 65536, dco.data_ptr(), \
         dout.data_ptr() + np.arange(n_tasks) * 65536
-    return Workload("dct", _shapes(n_tasks, threads, n_tb, shmem, sync, T.DCT), T.to_raw(a), {"img": im, "coef": coef},
-                    {"out": (dout, np.float32, (n_tasks, 128, 128))}, [dim_, dco, dout], im.nbytes, im.nbytes)
+    w = Workload("dct", _shapes(n_tasks, threads, n_tb, shmem, sync, T.DCT), T.to_raw(a), {"img": im, "coef": coef},
+                 {"out": (dout, np.float32, (n_tasks, 128, 128))}, [dim_, dco, dout], im.nbytes, im.nbytes)
+    w.dct_coef = dco.data_ptr()   # for pagoda_dct_register
+    return w
 
 
 def nop(n_tasks, threads=128, n_tb=1, shmem=0, sync=False):

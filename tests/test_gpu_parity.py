@@ -170,9 +170,35 @@ def test_dct_table5_small(threads, n_tb, shmem, sync):
 @pytest.mark.parametrize("name", ["dct", "dct_noshm"])
 def test_dct_table5_full_size(name):
     w = W.dct(32768, shmem=8192 if name == "dct" else 0, sync=name == "dct")
-    out = run(w, **ctx_kwargs(name))["out"]   # the bench's launch configuration
+    kw = ctx_kwargs(name, NO_START)           # the bench's launch configuration, registered coefficients
+    with Pagoda(**kw) as p:
+        p.dct_register(w.dct_coef)
+        assert p.start() == 0
+        p.spawn_shapes(w.shapes, w.args)
+        assert p.waitAll() == 0 and p.info().device_error == 0
+        assert p.stop() == 0
+        p.dct_register(None)
+    out = w.outputs()["out"]
     rng = np.random.default_rng(11)
     _dct_check(w, out, list(rng.choice(32768, 96, replace=False)) + [0, 32767])
+
+
+@pytest.mark.parametrize("shmem,sync", [(8192, True), (0, False)])
+def test_dct_registered_coefficients(shmem, sync):
+    """pagoda_dct_register: tasks with the registered coef pointer read the constant-bank copy
+    (bit-identical outputs); another coef buffer with the same values takes the load path."""
+    w = W.dct(300, shmem=shmem, sync=sync)
+    w2 = W.dct(100, shmem=shmem, sync=sync, first=300)   # its own coef buffer (a different pointer)
+    with Pagoda(flags=NO_START, arena_bytes=96 * 1024) as p:
+        p.dct_register(w.dct_coef)
+        assert p.start() == 0
+        p.spawn_shapes(w.shapes, w.args)
+        p.spawn_shapes(w2.shapes, w2.args)
+        assert p.waitAll() == 0
+        assert p.stop() == 0
+        p.dct_register(None)
+    _dct_check(w, w.outputs()["out"], range(300))
+    _dct_check(w2, w2.outputs()["out"], range(100))
 
 
 def test_dct_table5_naive_baseline():
