@@ -456,7 +456,7 @@ __device__ void body_mm(const Env& e, const pagoda_mm_args& a)
  * by TMA when 32 KiB were granted and the TB can synchronise; four independent
  * chains per thread share each B load, as in body_mm. */
 template <class Env>
-__device__ void body_mm64(const Env& e, const pagoda_mm_args& a)
+__device__ __noinline__ void body_mm64(const Env& e, const pagoda_mm_args& a)
 {
     const float* A = a.A;
     const float* B = a.B;
@@ -785,7 +785,7 @@ __device__ __forceinline__ void dct_item(const pagoda_dct_args& a, const float* 
  * TMA bulk copies and transforms them from shared memory; TB j takes bands j, j + nb, ...
  * Otherwise every item reads its block from global memory.  Same arithmetic either way. */
 template <bool kConstCoef, class Env>
-__device__ void body_dct_t(const Env& e, const pagoda_dct_args& a)
+__device__ __noinline__ void body_dct_t(const Env& e, const pagoda_dct_args& a)
 {
     if (e.getSMBytes() >= 4096 && e.canSync()) {
         float* s = reinterpret_cast<float*>(e.getSMPtr());
