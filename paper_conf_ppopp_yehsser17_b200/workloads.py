@@ -176,7 +176,9 @@ def mix(n_tasks=32768, device="cuda", first=0):
     raw[i] = T.to_raw(a); shapes[i, 3], shapes[i, 4] = 0, T.DCT
     host["dct"] = (im, coef); outs["dct"] = (dout2, np.float32, (n, 128, 128)); keep += [dim_, dco, dout2]
     in_b += im.nbytes; out_b += im.nbytes
-    return Workload("mix", shapes, raw, host, outs, keep, in_b, out_b)
+    w = Workload("mix", shapes, raw, host, outs, keep, in_b, out_b)
+    w.dct_coef = dco.data_ptr()   # every DCT task shares one coefficient matrix (pagoda_dct_register)
+    return w
 
 
 # ---------------------------------------------------------------- Table 5: DCT with / without shmem
@@ -379,6 +381,8 @@ def pooled(name, pool: InputPool, kinds, in_idx, threads, shmem, device="cuda", 
     w = PooledWorkload(name, pool, kinds, in_idx, shapes, raw, buf, base[:-1], out_len, [buf] + pool.keep)
     if "tdes" in pool.dev:
         w.tdes_tables = pool.dev["tdes"][1]
+    if "dct" in pool.dev:
+        w.dct_coef = pool.dev["dct"][1]
     return w
 
 

@@ -276,7 +276,20 @@ def test_mix_small_all_shapes():
 
 def test_mix_config4_full_size_sampled():
     w = W.mix(32768)
-    _mix_check(w, run(w, **ctx_kwargs("mix")), frac=0.004, seed=4)   # the bench's launch configuration
+    _mix_check(w, run(w, **ctx_kwargs("mix")), frac=0.004, seed=4)
+
+
+def test_mix_config4_registered_coefficients():
+    """The bench's launch configuration: config 4 with its DCT coefficients registered."""
+    w = W.mix(32768)
+    with Pagoda(**ctx_kwargs("mix", NO_START)) as p:
+        p.dct_register(w.dct_coef)
+        assert p.start() == 0
+        p.spawn_shapes(w.shapes, w.args)
+        assert p.waitAll() == 0 and p.info().device_error == 0
+        assert p.stop() == 0
+        p.dct_register(None)
+    _mix_check(w, w.outputs(), frac=0.004, seed=6)
 
 
 # ---------------------------------------------------------------- the naive baseline runs the same bodies

@@ -12,7 +12,7 @@ import pytest
 import oracle
 from paper_conf_ppopp_yehsser17_b200 import inputs as I
 from paper_conf_ppopp_yehsser17_b200 import workloads as W
-from paper_conf_ppopp_yehsser17_b200.pagoda import RESIDENT_TDES, Pagoda
+from paper_conf_ppopp_yehsser17_b200.pagoda import NO_START, RESIDENT_TDES, Pagoda
 
 pytestmark = pytest.mark.gpu
 
@@ -105,7 +105,9 @@ def test_c5_small_all_tasks(cfg):
 def test_c5_full_size_sampled():
     """The bench's N=1 launch configuration: 1M tasks on one GPU."""
     w = W.c5(1_000_000, resident=True, fill=0xAB)
-    with Pagoda(flags=RESIDENT_TDES, mtbs_per_sm=1, arena_bytes=144 * 1024) as p:
+    with Pagoda(flags=RESIDENT_TDES | NO_START, mtbs_per_sm=1, arena_bytes=144 * 1024) as p:
+        p.dct_register(w.dct_coef)       # as bench.py: the pool's DCT coefficients registered
+        assert p.start() == 0
         ids = p.spawn_shapes(w.shapes, w.args, ids=True)
         assert p.waitAll() == 0 and p.info().device_error == 0
         assert np.array_equal(ids, np.arange(1_000_000))
