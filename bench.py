@@ -260,6 +260,21 @@ def oracle_tasks(workload: str, n_sample: int):
     return [body(names[kinds[k]], pools[names[kinds[k]]], int(idx[k])) for k in range(n_sample)], what
 
 
+def host_info():
+    """SURVEY §8(d) result record: the host the CPU oracle ran on (nproc, CPU model, NUMA nodes)."""
+    model = None
+    try:
+        with open("/proc/cpuinfo") as f:
+            model = next((l.split(":", 1)[1].strip() for l in f if l.startswith("model name")), None)
+    except OSError:
+        pass
+    try:
+        numa = len([n for n in os.listdir("/sys/devices/system/node") if n.startswith("node") and n[4:].isdigit()])
+    except OSError:
+        numa = None
+    return {"nproc": os.cpu_count(), "cpu_model": model, "numa_nodes": numa}
+
+
 def oracle_rate(workload: str, n_sample: int, threads: int):
     """The oracle as it stands, on `threads` host threads over n_sample tasks of
     the workload: returns (tasks/s, seconds, sample description)."""
@@ -294,7 +309,7 @@ def run_reference(a, d: Dist):
             "impl": "reference",
             "config": workload_config(wl) | {"step_sample_tasks": n_sample},
             "cpu_baseline": {"value": v, "unit": "tasks/s", "cores": threads, "kind": "oracle",
-                             "sample": f"each step: {what}"},
+                             "sample": f"each step: {what}", "host": host_info()},
             "e2e": {"value": v, "unit": "tasks/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -566,7 +581,7 @@ def main():
         threads = os.cpu_count() or 1
         rate, dt, what = oracle_rate(a.workload if a.workload != "nop" else "tdes", CPU_SAMPLE[a.workload], threads)
         cpu = {"value": rate, "unit": "tasks/s", "cores": threads, "kind": "oracle",
-               "sample": f"{what}, {dt:.1f} s wall on {threads} threads"}
+               "sample": f"{what}, {dt:.1f} s wall on {threads} threads", "host": host_info()}
 
     if d.rank != 0:
         return
