@@ -73,6 +73,7 @@ def lib():
             L.orc_occupancy_pct.argtypes = [I, I]
             L.orc_occupancy_pct.restype = C.c_double
             L.orc_ledger_check.argtypes = [P, SZ, I, I, I, I, P, SZ, C.c_char_p, SZ]
+            L.orc_exec_check.argtypes = [P, SZ, P, SZ, P, SZ, P, SZ, C.c_char_p, SZ]
             _lib = L
     return _lib
 
@@ -209,4 +210,26 @@ def ledger_check(events: np.ndarray, n_mtb: int, exec_warps: int, arena_granules
     rc = lib().orc_ledger_check(_p(events) if len(events) else None, len(events), n_mtb, exec_warps,
                                 arena_granules, n_bar_ids, _p(tasks) if len(tasks) else None,
                                 len(tasks), err, 512)
+    return rc == 0, err.value.decode()
+
+
+EXEC_DTYPE = np.dtype([("task_id", "<u8"), ("tb", "<u2"), ("smid", "<u2"), ("mtb", "<u2"), ("warp", "<u2"),
+                       ("t_start", "<u8"), ("t_end", "<u8")])
+COMP_DTYPE = np.dtype([("task_id", "<u8"), ("t_done", "<u8")])
+assert EXEC_DTYPE.itemsize == 32 and COMP_DTYPE.itemsize == 16
+
+
+def exec_check(events: np.ndarray, execs: np.ndarray, comps: np.ndarray, tasks: np.ndarray):
+    """Executor intervals + completion records against the ledger (oracle.h orc_exec_check).
+    Return (ok, message)."""
+    events = np.ascontiguousarray(events, LEDGER_DTYPE)
+    execs = np.ascontiguousarray(execs, EXEC_DTYPE)
+    comps = np.ascontiguousarray(comps, COMP_DTYPE)
+    tasks = np.ascontiguousarray(tasks, TASK_DTYPE)
+    err = C.create_string_buffer(512)
+
+    def q(a):
+        return _p(a) if len(a) else None
+    rc = lib().orc_exec_check(q(events), len(events), q(execs), len(execs), q(comps), len(comps),
+                              q(tasks), len(tasks), err, 512)
     return rc == 0, err.value.decode()

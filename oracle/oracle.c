@@ -623,3 +623,134 @@ done:
     free(ev); free(recs); free(live_w); free(live_b); free(live_g);
     return rc;
 }
+
+/* ======================================================================
+ * Executor intervals + completion records (oracle.h orc_exec_check).
+ * Sorted copies and binary searches: the brute-force schedules replay
+ * ~10^5 records per session.
+ * ==================================================================== */
+typedef struct { uint64_t task_id; uint16_t tb, mtb; uint32_t mask, seen; } alloc_key;
+
+static int ak_cmp(const void* a, const void* b)
+{
+    const alloc_key* x = (const alloc_key*)a;
+    const alloc_key* y = (const alloc_key*)b;
+    if (x->task_id != y->task_id) return x->task_id < y->task_id ? -1 : 1;
+    return (int)x->tb - (int)y->tb;
+}
+static int ex_task_cmp(const void* a, const void* b)   /* (task, tb, warp) */
+{
+    const orc_exec_record* x = (const orc_exec_record*)a;
+    const orc_exec_record* y = (const orc_exec_record*)b;
+    if (x->task_id != y->task_id) return x->task_id < y->task_id ? -1 : 1;
+    if (x->tb != y->tb) return (int)x->tb - (int)y->tb;
+    return (int)x->warp - (int)y->warp;
+}
+static int ex_warp_cmp(const void* a, const void* b)   /* (mtb, warp, t_start) */
+{
+    const orc_exec_record* x = (const orc_exec_record*)a;
+    const orc_exec_record* y = (const orc_exec_record*)b;
+    if (x->mtb != y->mtb) return (int)x->mtb - (int)y->mtb;
+    if (x->warp != y->warp) return (int)x->warp - (int)y->warp;
+    if (x->t_start != y->t_start) return x->t_start < y->t_start ? -1 : 1;
+    return 0;
+}
+static int comp_cmp(const void* a, const void* b)
+{
+    const orc_completion* x = (const orc_completion*)a;
+    const orc_completion* y = (const orc_completion*)b;
+    return x->task_id < y->task_id ? -1 : x->task_id > y->task_id ? 1 : 0;
+}
+
+int orc_exec_check(const orc_ledger_event* ev, size_t n_ev, const orc_exec_record* ex_in, size_t n_ex,
+                   const orc_completion* comp_in, size_t n_comp, const orc_ledger_task* tasks,
+                   size_t n_tasks, char* err, size_t err_len)
+{
+    int rc = 0;
+    size_t n_al = 0;
+    alloc_key* al = (alloc_key*)malloc((n_ev ? n_ev : 1) * sizeof *al);
+    orc_exec_record* ex = (orc_exec_record*)malloc((n_ex ? n_ex : 1) * sizeof *ex);
+    orc_exec_record* exw = (orc_exec_record*)malloc((n_ex ? n_ex : 1) * sizeof *exw);
+    orc_completion* cp = (orc_completion*)malloc((n_comp ? n_comp : 1) * sizeof *cp);
+    orc_completion* tid = NULL;   /* sorted task ids */
+    if (!al || !ex || !exw || !cp) FAIL("out of memory");
+    for (size_t i = 0; i < n_ev; i++)
+        if (ev[i].kind == 1) {
+            alloc_key k = {ev[i].task_id, ev[i].tb, ev[i].mtb, ev[i].warp_mask, 0};
+            al[n_al++] = k;
+        }
+    qsort(al, n_al, sizeof *al, ak_cmp);
+    for (size_t i = 1; i < n_al; i++)
+        if (ak_cmp(&al[i - 1], &al[i]) == 0)
+            FAIL("task %llu tb %u allocated twice", (unsigned long long)al[i].task_id, al[i].tb);
+    memcpy(ex, ex_in, n_ex * sizeof *ex);
+    memcpy(exw, ex_in, n_ex * sizeof *exw);
+    qsort(ex, n_ex, sizeof *ex, ex_task_cmp);
+    qsort(exw, n_ex, sizeof *exw, ex_warp_cmp);
+    memcpy(cp, comp_in, n_comp * sizeof *cp);
+    qsort(cp, n_comp, sizeof *cp, comp_cmp);
+
+    /* 1. every execution interval is well formed and lies in its TB's allocation */
+    for (size_t i = 0; i < n_ex; i++) {
+        const orc_exec_record* r = &ex[i];
+        if (r->t_end < r->t_start)
+            FAIL("task %llu tb %u warp %u: interval ends before it starts", (unsigned long long)r->task_id, r->tb, r->warp);
+        if (i > 0 && ex_task_cmp(&ex[i - 1], r) == 0)
+            FAIL("task %llu tb %u warp %u ran twice", (unsigned long long)r->task_id, r->tb, r->warp);
+        alloc_key k = {r->task_id, r->tb, 0, 0, 0};
+        alloc_key* a = (alloc_key*)bsearch(&k, al, n_al, sizeof *al, ak_cmp);
+        if (!a) FAIL("task %llu tb %u ran without an ALLOC", (unsigned long long)r->task_id, r->tb);
+        if (a->mtb != r->mtb)
+            FAIL("task %llu tb %u ran on MTB %u, allocated on MTB %u", (unsigned long long)r->task_id, r->tb, r->mtb, a->mtb);
+        if (r->warp >= 32 || !((a->mask >> r->warp) & 1u))
+            FAIL("task %llu tb %u ran on warp %u outside its ALLOC mask %08x", (unsigned long long)r->task_id, r->tb, r->warp, a->mask);
+        a->seen |= 1u << r->warp;
+    }
+    for (size_t i = 0; i < n_al; i++)
+        if (al[i].seen != al[i].mask)
+            FAIL("task %llu tb %u: warps %08x allocated, %08x ran", (unsigned long long)al[i].task_id, al[i].tb, al[i].mask, al[i].seen);
+    /* 2. a warp never runs two tasks at once */
+    for (size_t i = 1; i < n_ex; i++) {
+        const orc_exec_record *p = &exw[i - 1], *q = &exw[i];
+        if (p->mtb == q->mtb && p->warp == q->warp && q->t_start < p->t_end)
+            FAIL("mtb %u warp %u: task %llu starts at %llu before task %llu ends at %llu", q->mtb, q->warp,
+                 (unsigned long long)q->task_id, (unsigned long long)q->t_start, (unsigned long long)p->task_id,
+                 (unsigned long long)p->t_end);
+    }
+    /* 3. exactly one completion per task, after the last warp of the task ended */
+    for (size_t i = 1; i < n_comp; i++)
+        if (cp[i - 1].task_id == cp[i].task_id) FAIL("task %llu completed twice", (unsigned long long)cp[i].task_id);
+    for (size_t t = 0; t < n_tasks; t++) {
+        orc_completion k = {tasks[t].task_id, 0};
+        const orc_completion* c = (const orc_completion*)bsearch(&k, cp, n_comp, sizeof *cp, comp_cmp);
+        if (!c) FAIL("task %llu has no completion record", (unsigned long long)tasks[t].task_id);
+        /* the task's execution records are contiguous in ex (sorted by task first) */
+        size_t lo = 0, hi = n_ex;
+        while (lo < hi) {
+            const size_t mid = (lo + hi) / 2;
+            if (ex[mid].task_id < tasks[t].task_id) lo = mid + 1;
+            else hi = mid;
+        }
+        uint64_t last_end = 0;
+        uint32_t warps = 0;
+        for (size_t i = lo; i < n_ex && ex[i].task_id == tasks[t].task_id; i++) {
+            if (ex[i].t_end > last_end) last_end = ex[i].t_end;
+            warps++;
+        }
+        if (warps != tasks[t].warps_total)
+            FAIL("task %llu: %u warps ran, expected %u", (unsigned long long)tasks[t].task_id, warps, tasks[t].warps_total);
+        if (c->t_done < last_end)
+            FAIL("task %llu completed at %llu before its last warp ended at %llu", (unsigned long long)tasks[t].task_id,
+                 (unsigned long long)c->t_done, (unsigned long long)last_end);
+    }
+    tid = (orc_completion*)malloc((n_tasks ? n_tasks : 1) * sizeof *tid);
+    if (!tid) FAIL("out of memory");
+    for (size_t t = 0; t < n_tasks; t++) tid[t].task_id = tasks[t].task_id, tid[t].t_done = 0;
+    qsort(tid, n_tasks, sizeof *tid, comp_cmp);
+    for (size_t i = 0; i < n_comp; i++)
+        if (!bsearch(&cp[i], tid, n_tasks, sizeof *tid, comp_cmp))
+            FAIL("completion record of unlisted task %llu", (unsigned long long)cp[i].task_id);
+done:
+    free(al); free(ex); free(exw); free(cp); free(tid);
+    return rc;
+}

@@ -15,7 +15,13 @@
  * DESIGN.md "Readings") fix the fp32 operation order (fmaf where the definition
  * says fma, no contraction elsewhere: build with -ffp-contract=off).  Every
  * fp32 body is pinned in tests/ against fp64 library routines / closed forms
- * within the textbook error bound, so the fp32 op order is checked, not trusted.
+ * within the textbook error bound; error bounds alone cannot tell fmaf from
+ * mul+add or one summation order from another, so each fp32 body also has a
+ * hand-derived closed-form pin whose exact value exists only under the defined
+ * order (tests/test_oracle_bodies.py "fma / order pins": one cancelling step
+ * gives 2^-24 fused and in order, 0 unfused or reordered).  MB, defined
+ * without fma, is pinned by the whole-config checksum of an independent numpy
+ * emulation (scripts/gen_mandelbrot_pins.py), which a contracted build misses.
  */
 #ifndef PAGODA_ORACLE_H
 #define PAGODA_ORACLE_H
@@ -93,6 +99,30 @@ typedef struct { uint64_t task_id; uint32_t warps_total; uint32_t n_tb; } orc_le
 int orc_ledger_check(const orc_ledger_event* ev, size_t n_ev, int n_mtb, int exec_warps,
                      int arena_granules, int n_bar_ids, const orc_ledger_task* tasks,
                      size_t n_tasks, char* err, size_t err_len);
+
+/* ---- executor-interval and completion checker (SURVEY §8(c) invariants 2-4:
+ * "a warp never runs two tasks at once", "exactly one completion record, and it
+ * comes after the last t_end of its warps").  One record per (task, TB, warp)
+ * that ran, with %globaltimer start/end; one completion record per task with
+ * the time it was posted to the host.  Cross-checked against the ledger: every
+ * executed warp must lie in its TB's ALLOC mask on the same MTB (Alg. 2 L9-12,
+ * P:846-851), every allocated warp must have run once (Alg. 1 L29-33,
+ * P:781-785), and a task completes only after all its warps ended (Alg. 1
+ * L41-43).  Returns 0 or a negative code with a message in err. */
+typedef struct {
+    uint64_t task_id;
+    uint16_t tb;
+    uint16_t smid;       /* informational */
+    uint16_t mtb;
+    uint16_t warp;
+    uint64_t t_start, t_end;
+} orc_exec_record;       /* 32 bytes */
+
+typedef struct { uint64_t task_id; uint64_t t_done; } orc_completion;   /* 16 bytes */
+
+int orc_exec_check(const orc_ledger_event* ev, size_t n_ev, const orc_exec_record* ex, size_t n_ex,
+                   const orc_completion* comp, size_t n_comp, const orc_ledger_task* tasks,
+                   size_t n_tasks, char* err, size_t err_len);
 
 #ifdef __cplusplus
 }

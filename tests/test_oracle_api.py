@@ -127,3 +127,46 @@ def test_ledger_rejects(orc, bad, needle):
     n_tb = 2 if needle == "TBs on MTBs" else 1
     ok, msg = check(bad, tasks((1, 1 * n_tb, n_tb), (2, 2, 1)))
     assert not ok and needle in msg, msg
+
+
+# ------------------------------------------------------------------ executor-interval / completion checker
+# Two tasks on MTB 0: task 1 (1 TB, warps 1-2), task 2 (1 TB, warp 1 after task 1 freed it).
+def _valid_exec_case():
+    evs = [ev(0, 0, 1, 1, 0, 0b110), ev(1, 0, 2, 1, 0, 0b110), ev(2, 0, 3, 1, 0, 0),
+           ev(3, 0, 1, 2, 0, 0b10), ev(4, 0, 2, 2, 0, 0b10), ev(5, 0, 3, 2, 0, 0)]
+    ex = [(1, 0, 0, 0, 1, 100, 200), (1, 0, 0, 0, 2, 110, 210), (2, 0, 0, 0, 1, 220, 300)]
+    comps = [(1, 215), (2, 305)]
+    return evs, ex, comps, tasks((1, 2, 1), (2, 1, 1))
+
+
+def xcheck(evs, ex, comps, ts):
+    return O.exec_check(np.array(evs, O.LEDGER_DTYPE), np.array(ex, O.EXEC_DTYPE),
+                        np.array(comps, O.COMP_DTYPE), ts)
+
+
+def test_exec_check_accepts_valid(orc):
+    evs, ex, comps, ts = _valid_exec_case()
+    ok, msg = xcheck(evs, ex, comps, ts)
+    assert ok, msg
+    ok, msg = check(evs, ts, n_mtb=1)        # the same trace passes the allocator replay too
+    assert ok, msg
+
+
+@pytest.mark.parametrize("mutate,needle", [
+    (lambda e, x, c: x.__setitem__(2, (2, 0, 0, 0, 1, 190, 300)), "before task"),          # warp 1 overlap
+    (lambda e, x, c: c.__setitem__(0, (1, 205)), "before its last warp ended"),          # early completion
+    (lambda e, x, c: c.pop(), "no completion"),
+    (lambda e, x, c: c.append((1, 400)), "completed twice"),
+    (lambda e, x, c: x.__setitem__(2, (2, 0, 0, 0, 3, 220, 300)), "outside its ALLOC"),  # wrong warp
+    (lambda e, x, c: x.__setitem__(2, (2, 0, 0, 1, 1, 220, 300)), "allocated on MTB"),   # wrong MTB
+    (lambda e, x, c: x.pop(1), "allocated"),                                              # a warp never ran
+    (lambda e, x, c: x.append((1, 0, 0, 0, 1, 500, 600)), "ran twice"),
+    (lambda e, x, c: x.__setitem__(0, (1, 0, 0, 0, 1, 200, 100)), "ends before"),
+    (lambda e, x, c: x.append((3, 0, 0, 0, 5, 500, 600)), "without an ALLOC"),
+    (lambda e, x, c: c.append((9, 1)), "unlisted"),
+])
+def test_exec_check_rejects(orc, mutate, needle):
+    evs, ex, comps, ts = _valid_exec_case()
+    mutate(evs, ex, comps)
+    ok, msg = xcheck(evs, ex, comps, ts)
+    assert not ok and needle in msg, msg

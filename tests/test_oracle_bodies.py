@@ -374,3 +374,97 @@ def test_schedules_mpe_and_c5():
     assert set(np.unique(shm // 1024)) == set(I.MIX_SHMEM_KB)
     k2 = I.c5_schedule(1000)[0]
     assert np.array_equal(k2, kinds[:1000])                     # prefix-stable: shards agree with the whole
+
+
+# ------------------------------------------------------------------ fma / order pins
+# Error bounds cannot tell fmaf from mul+add, nor one summation order from another.
+# These closed forms can: with P = 1 + 2^-12 and Q = 1 + 2^-11 (both fp32),
+# P*P = 1 + 2^-11 + 2^-24 exactly, whose fp32 rounding is Q (a tie, to even).
+# So the step "acc = -Q; acc = fmaf(P, P, acc)" gives exactly 2^-24 when it is
+# fused and taken in the defined (ascending) order; rounding the product first
+# (mul+add) or taking the P*P term first (descending order) gives 0.  Each body
+# gets one such step at a place its definition fixes.
+P32 = 1.0 + 2.0 ** -12
+Q32 = 1.0 + 2.0 ** -11
+
+
+def test_fma_order_pin_mm(orc):
+    """C[i][j] = fma chain over k ascending (DESIGN.md MM): A[:,0] = 1, B[0,:] = -Q,
+    A[:,1] = B[1,:] = P -> every C[i][j] = 2^-24 exactly."""
+    for n, f in ((32, orc.mm32), (64, orc.mm64)):
+        A = np.zeros((n, n), np.float32)
+        B = np.zeros((n, n), np.float32)
+        A[:, 0], B[0, :] = 1.0, -Q32
+        A[:, 1], B[1, :] = P32, P32
+        C = f(A, B)
+        assert (C == np.float32(2.0 ** -24)).all(), (n, np.unique(C))
+
+
+def test_fma_order_pin_filterbank(orc):
+    """VH[8] = fma chain k = 0..8 of H[k] r[8-k] with H[0] r[8] = -Q, H[8] r[0] = P*P -> 2^-24;
+    with F = delta, y[8] = VU[8] = VD[1] = VH[8] and y[0] = VH[0] = P."""
+    r = np.zeros(2048, np.float32)
+    H = np.zeros(32, np.float32)
+    F = np.zeros(32, np.float32)
+    r[0], r[8] = P32, -Q32
+    H[0], H[8] = 1.0, P32
+    F[0] = 1.0
+    y = orc.filterbank(r, H, F)
+    assert y[8] == np.float32(2.0 ** -24) and y[0] == np.float32(P32)
+
+
+def test_fma_order_pin_beamformer(orc):
+    """out = fmaf(y.re, y.re, y.im*y.im) with y = (P, 2^-12): fused = RN(1 + 2^-11 + 2^-23)
+    = 1 + 2^-11 + 2^-23; mul+add (or the other operand fused) = Q."""
+    x = np.zeros((4, 512, 2), np.float32)
+    h = np.zeros((4, 16, 2), np.float32)
+    w = np.zeros((4, 4, 2), np.float32)
+    x[0, 0] = (P32, 2.0 ** -12)
+    h[0, 0] = (1.0, 0.0)
+    w[0, 0] = (1.0, 0.0)
+    out = orc.beamformer(x, h, w)
+    assert out[0, 0] == np.float32(1.0 + 2.0 ** -11 + 2.0 ** -23)
+    assert (out[1:] == 0).all()
+
+
+def test_fma_order_pin_conv(orc):
+    """Row pass d ascending: img[64][64] krow[8] = -Q, then img[64][65] krow[7] = P*P ->
+    tmp[64][64] = 2^-24; kcol = delta -> out[64][64] = 2^-24."""
+    img = np.zeros((128, 128), np.float32)
+    krow = np.zeros(17, np.float32)
+    kcol = np.zeros(17, np.float32)
+    img[64, 64], img[64, 65] = 1.0, P32
+    krow[8], krow[7] = -Q32, P32
+    kcol[8] = 1.0
+    out = orc.conv(img, krow, kcol)
+    assert out[64, 64] == np.float32(2.0 ** -24)
+
+
+def test_fma_order_pin_dct(orc):
+    """T[0][0] = fma chain over x ascending: C[0][0] X[0][0] = -Q, then C[0][1] X[1][0] = P*P ->
+    2^-24; Y[0][0] = T[0][0] C[0][0] = -(2^-24 + 2^-35) (exact)."""
+    img = np.zeros((128, 128), np.float32)
+    coef = np.zeros((8, 8), np.float32)
+    img[0, 0], img[1, 0] = 1.0, P32
+    coef[0, 0], coef[0, 1] = -Q32, P32
+    out = orc.dct(img, coef)
+    assert out[0, 0] == np.float32(-(2.0 ** -24 + 2.0 ** -35))
+    assert (out[8:, :] == 0).all() and (out[:, 8:] == 0).all()
+
+
+# ------------------------------------------------------------------ Mandelbrot pin provenance
+def test_mb_golden_file_regenerates():
+    """tests/golden/mandelbrot_pins.txt is exactly what scripts/gen_mandelbrot_pins.py (an
+    independent numpy float32 emulation, no oracle code) writes; and a contracted (fma)
+    evaluation of the same iteration changes the whole-config sum, so that pin catches it."""
+    import importlib.util
+    import os
+    spec = importlib.util.spec_from_file_location(
+        "gen_mb", os.path.join(os.path.dirname(__file__), "..", "scripts", "gen_mandelbrot_pins.py"))
+    gen = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(gen)
+    counts = gen.iteration_counts()
+    with open(gen.GOLDEN) as f:
+        assert f.read() == gen.render(counts)
+    fused = gen.iteration_counts(fused=True)
+    assert int(fused.sum(dtype=np.int64)) != int(counts.sum(dtype=np.int64))
