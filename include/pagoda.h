@@ -48,6 +48,9 @@ typedef int64_t pagoda_task_t;          /* >= 0: task id; < 0: -errno */
                                       4 warps), so few, uneven tasks (config 1) go to the idlest MTBs */
 #define PAGODA_LIFECYCLE     0x8u /* stamp every task's life cycle on the GPU clock (profiling; 64 B per
                                      completion slot): see pagoda_lifecycle_read */
+#define PAGODA_NONBLOCKING_SPAWN 0x20u /* taskSpawn returns -EAGAIN instead of waiting when the TaskTable
+                                     ring slot or completion slot a new task needs is still taken
+                                     (the paper's CPU waits for a free entry) */
 
 typedef struct {
     int      device;        /* CUDA device ordinal (default 0) */
@@ -57,8 +60,10 @@ typedef struct {
     uint32_t ring_entries;  /* TaskTable ring entries, host and device, power of 2 (default 65536) */
     uint32_t comp_entries;  /* completion window, power of 2 >= ring_entries (default 1<<20) */
     uint32_t arena_bytes;   /* shared-memory arena per MTB, multiple of 512 (default 96 KiB at 2 MTB/SM) */
-    uint32_t exec_warps;    /* worker warps per MTB, 1..32, capped at the MTB's warps (default 32 = all;
-                               fewer = debug config) */
+    uint32_t exec_warps;    /* worker warps per MTB, 1..32, capped at the MTB's warps (32 at 1-2 MTBs/SM,
+                               16 at 4 MTBs/SM; default 32 = all; fewer = debug config).  One thread
+                               block may use at most this many warps (pagoda_info.exec_warps); a
+                               single-MTB context keeps one warp for its ingest */
     uint32_t flags;         /* PAGODA_TRACE */
     uint32_t trace_events;  /* ledger capacity per MTB when PAGODA_TRACE (default 8192) */
     double   watchdog_s;    /* wait/waitAll/shutdown give up with -ETIMEDOUT after this many
@@ -88,7 +93,9 @@ int pagoda_shutdown(pagoda_ctx* ctx);
  * (pagoda_tasks.h); args/args_bytes (<= 40) are copied into the entry.
  * Non-blocking: returns once the entry is published (it blocks, with back-off,
  * only while the TaskTable ring or completion window is full, as the paper's
- * CPU does when no entry is free).
+ * CPU does when no entry is free; with PAGODA_NONBLOCKING_SPAWN it
+ * returns -EAGAIN instead).  Ids never skip a number because of an error: a
+ * spawn that cannot get its slots without waiting in vain reserves no id.
  * A task whose thread blocks all fit one MTB (warps, shared memory, 15
  * barrier IDs) runs inside one MTB.  A larger task (e.g. the
  * "64K threads" of Fig. 8) is spread TB by TB over k MTB-sized
@@ -96,19 +103,29 @@ int pagoda_shutdown(pagoda_ctx* ctx);
  * stay strictly increasing but skip k - 1) and completes when its last TB does.
  * Returns the task id (>= 0, strictly increasing per context) or
  *   -EINVAL  threads < 1 or > 1024, n_threadblocks < 1 or (spread) > 65535,
- *            ceil(threads/32) > worker warps per MTB (32), round_up(shmem, 512)
- *            > arena (one TB must fit an MTB), k > ring_entries / 4,
- *            unknown func_id, args_bytes > 40 or args NULL with args_bytes > 0;
- *   -ESHUTDOWN after pagoda_shutdown began;  -EIO after a device fault. */
+ *            ceil(threads/32) > exec_warps (the worker warps of one MTB: 32 by
+ *            default, 16 at 4 MTBs per SM, 31 in a single-MTB context; see
+ *            pagoda_info.exec_warps), round_up(shmem, 512) > arena (one TB
+ *            must fit an MTB), k > ring_entries / 4, unknown func_id,
+ *            args_bytes > 40 or args NULL with args_bytes > 0;
+ *   -EAGAIN  the ring / completion slot is taken and the spawn may not wait:
+ *            PAGODA_NONBLOCKING_SPAWN, or the session is stopped (nothing
+ *            drains the ring until pagoda_start); nothing was spawned;
+ *   -ETIMEDOUT  the watchdog expired while waiting for a slot (the context is
+ *            then faulted: later calls return -EIO);
+ *   -ESHUTDOWN after pagoda_shutdown began;  -EIO after a device fault
+ *            (PAGODA_DEVERR_SYNC_WITHOUT_FLAG / _BAD_FUNC) or a failed spawn. */
 pagoda_task_t pagoda_taskSpawn(pagoda_ctx* ctx, int threads, int n_threadblocks, int shmem_bytes,
                                int sync_flag, int func_id, const void* args, size_t args_bytes);
 
 /* wait (Table 1): block until task `id` is done.  After it returns 0
  * the task's device writes are visible to later host copies and to every task
- * spawned afterwards.  Returns 0, -EINVAL (id never issued), -EIO, -ETIMEDOUT. */
+ * spawned afterwards.  Returns 0, -EINVAL (id never issued), -EIO (a device
+ * fault was seen: every call from then on returns it), -ETIMEDOUT. */
 int pagoda_wait(pagoda_ctx* ctx, pagoda_task_t id);
 
-/* check (Table 1): non-blocking; 1 if done, 0 if pending, < 0 error. */
+/* check (Table 1): non-blocking; 1 if done, 0 if pending, -EINVAL
+ * (id never issued), -EIO (device fault seen). */
 int pagoda_check(pagoda_ctx* ctx, pagoda_task_t id);
 
 /* waitAll (Table 1): block until every task whose id was issued before
@@ -129,7 +146,10 @@ int64_t pagoda_taskSpawnMany(pagoda_ctx* ctx, int n, int threads, int n_threadbl
                              size_t args_bytes, pagoda_task_t* ids_out);
 
 /* Same with a per-task shape: shapes[i] = {threads, n_threadblocks, shmem_bytes,
- * sync_flag, func_id} (5 int32 per task). */
+ * sync_flag, func_id} (5 int32 per task).  Both batched forms return n, or,
+ * when the ring fills and the call may not wait (PAGODA_NONBLOCKING_SPAWN or
+ * a stopped session), the number of leading tasks spawned (0 < count < n; with
+ * none spawned -EAGAIN), or the first error. */
 int64_t pagoda_taskSpawnShapes(pagoda_ctx* ctx, int n, const int32_t* shapes, const void* args_base,
                                size_t args_stride, size_t args_bytes, pagoda_task_t* ids_out);
 
@@ -211,7 +231,12 @@ typedef struct {
 } pagoda_info;
 int pagoda_get_info(pagoda_ctx* ctx, pagoda_info* out);
 
-#define PAGODA_DEVERR_SYNC_WITHOUT_FLAG 1u  /* syncBlock() in a multi-warp TB spawned with sync=0 */
+/* Device errors (SURVEY §8(b) "Device errors"): the MasterKernel ORs a code into the device
+ * error word, which reaches the host within microseconds; from then on every host call on
+ * the context (spawn, wait, check, waitAll, stop, shutdown) returns -EIO.  LAYOUT is a notice
+ * only (the tasks still run correctly). */
+#define PAGODA_DEVERR_SYNC_WITHOUT_FLAG 1u  /* syncBlock() in a multi-warp TB spawned with sync=0 (P:976-983:
+                                               only sync tasks get a barrier ID) */
 #define PAGODA_DEVERR_BAD_FUNC          2u  /* entry with unknown func_id reached an executor */
 #define PAGODA_DEVERR_LAYOUT            4u  /* resident tables did not fit the shared-memory layout (fell back) */
 
@@ -248,17 +273,18 @@ int pagoda_tdes_tables(const uint8_t key24[24], void* dst);
  * PAGODA_RESIDENT_TDES): 3DES tasks whose `tables` pointer equals dev_tables
  * (device memory written by pagoda_tdes_tables) take their 48 round keys from
  * the MasterKernel's constant bank instead of staging them through shared
- * memory.  One schedule per device and process; NULL unregisters.  Call while
- * the context is stopped (NO_START or after pagoda_stop): -EBUSY otherwise.
- * Returns 0, -EINVAL (unreadable pointer), -EBUSY, -EIO. */
+ * memory.  One schedule per device and process (the MasterKernel's constant
+ * bank is shared by every context on the device); NULL unregisters.  Call while
+ * NO context on the device is running (NO_START or after pagoda_stop):
+ * -EBUSY otherwise.  Returns 0, -EINVAL (unreadable pointer), -EBUSY, -EIO. */
 int pagoda_tdes_register(pagoda_ctx* ctx, const void* dev_tables);
 
 /* Register a DCT coefficient matrix (pagoda_dct_args.coef: 64 fp32 C[u][x], device memory) as
  * resident task-class data: DCT tasks whose coef pointer equals dev_coef read the second
  * pass's coefficients from the MasterKernel's constant bank (same values, same arithmetic:
  * outputs are bit-identical).  The matrix is copied at registration; later writes to dev_coef
- * are not seen.  One matrix per device and process; NULL unregisters.  Call while the context
- * is stopped: -EBUSY otherwise.  Returns 0, -EINVAL (unreadable pointer), -EBUSY, -EIO.
+ * are not seen.  One matrix per device and process; NULL unregisters.  Call while no context on
+ * the device is running: -EBUSY otherwise.  Returns 0, -EINVAL (unreadable pointer), -EBUSY, -EIO.
  * Table 5 / DESIGN.md "DCT". */
 int pagoda_dct_register(pagoda_ctx* ctx, const float* dev_coef);
 

@@ -53,6 +53,9 @@ constexpr uint32_t kResidentOffset = 8192;          /* room reserved for the con
 constexpr uint32_t kResidentTdesBytes = 8 * 64 * 32 * 4;   /* 3DES SP tables, one copy per lane */
 constexpr uint32_t kResidentTdesAddr = 8192;        /* shared-WINDOW address of the resident tables: a
                                                        constant, so lookups carry it as an immediate */
+constexpr uint32_t kDevErrorPtrOffset = 5960;       /* MtbShared.dev_error: the device error word's address, for
+                                                       the paper-named free syncBlock() (which has no TaskEnv) */
+constexpr uint32_t kDevErrSyncWithoutFlag = 1u;     /* == PAGODA_DEVERR_SYNC_WITHOUT_FLAG (pagoda.h) */
 
 __device__ __forceinline__ uint32_t lane_id() { return threadIdx.x & 31u; }
 
@@ -117,7 +120,7 @@ struct TaskEnv {
             named_bar_sync(bar, 32u * wtb);
         } else {
             /* spawned with sync=0: contract violation */
-            atomicOr(dev_error, 1u);
+            atomicOr(dev_error, kDevErrSyncWithoutFlag);
             __syncwarp();
         }
     }
@@ -227,10 +230,19 @@ __device__ __forceinline__ int getTid()
     return ((int)s.tb * (int)s.warps_tb + (int)s.warp_in_tb) * 32 + (int)pagoda::lane_id();
 }
 __device__ __forceinline__ void syncBlock()
-{
+{   /* same semantics as TaskEnv::syncBlock: a multi-warp TB spawned with sync=0 has no barrier ID,
+     * which is a contract violation: flag it, later host calls return -EIO */
+    extern __shared__ __align__(1024) unsigned char pagoda_mk_smem[];
     const pagoda::WarpSlot& s = pagoda_my_slot();
-    if (s.warps_tb == 1 || s.bar_id == 0) __syncwarp();
-    else pagoda::named_bar_sync(s.bar_id, 32u * s.warps_tb);
+    if (s.warps_tb == 1) {
+        __syncwarp();
+    } else if (s.bar_id != 0) {
+        pagoda::named_bar_sync(s.bar_id, 32u * s.warps_tb);
+    } else {
+        uint32_t* err = *reinterpret_cast<uint32_t* const*>(pagoda_mk_smem + pagoda::kDevErrorPtrOffset);
+        atomicOr(err, pagoda::kDevErrSyncWithoutFlag);
+        __syncwarp();
+    }
 }
 __device__ __forceinline__ char* getSMPtr()
 {

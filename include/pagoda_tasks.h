@@ -23,6 +23,11 @@ enum pagoda_func_id {
     PAGODA_SMEM = 4,   /* fill getSMPtr()[0:bytes], spin, syncBlock, verify; errors -> err[0] */
     PAGODA_SPIN = 5,   /* busy-wait ns (%globaltimer) */
     PAGODA_GATE = 6,   /* spin until *flag != 0 (flag in pinned host memory) */
+    PAGODA_HOLD = 7,   /* brute-force schedules: count the warp in *started, fill getSMPtr()[0:grant] with a
+                          pattern, hold until *flag != 0, verify the pattern after syncBlock; errors -> err[0] */
+    PAGODA_PAPER = 8,  /* written against the paper's free functions only (Table 1: getTid,
+                          syncBlock, getSMPtr; no Env): out[base + getTid()] = getTid() + 1 for live threads,
+                          syncBlock(), then each thread checks its warp-mate 32 lanes on; errors -> err[0] */
     /* paper benchmarks (Table 3) */
     PAGODA_MB   = 16,  /* Mandelbrot 64x64 tile */
     PAGODA_TDES = 17,  /* 3DES EDE3 ECB over a packet */
@@ -43,6 +48,10 @@ typedef struct { uint32_t* err; uint32_t* scratch; uint32_t phases; uint32_t pad
 typedef struct { uint32_t* err; uint32_t bytes; uint32_t spin_ns; uint32_t seed; uint32_t pad; } pagoda_smem_args;
 typedef struct { uint64_t ns; } pagoda_spin_args;
 typedef struct { const volatile uint32_t* flag; } pagoda_gate_args;
+/* flag / started may be pinned host memory (mapped): the host releases and watches the task */
+typedef struct { const volatile uint32_t* flag; uint32_t* err; uint32_t* started; uint32_t seed; uint32_t pad; }
+    pagoda_hold_args;
+typedef struct { uint32_t* out; uint32_t* err; uint32_t base; uint32_t pad; } pagoda_paper_args;
 
 /* MB: pixel (px,py) of tile (tx,ty): c = (x0 + (64tx+px)*dx, y0 + (64ty+py)*dx) */
 typedef struct { uint16_t* out; float x0, y0, dx; int32_t tx, ty, maxit; } pagoda_mb_args;

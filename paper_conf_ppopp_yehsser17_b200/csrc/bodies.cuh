@@ -82,6 +82,7 @@ __device__ void body_smem(const Env& e, const pagoda_smem_args& a)
     const int n = tb_threads(e);
     uint32_t errs = 0;
     if (e.getBlockTid() == 0 && ((uintptr_t)p & 31u) != 0) errs++;   /* getSMPtr is 32-byte aligned */
+    if (e.getBlockTid() == 0 && e.getSMBytes() < a.bytes) errs++;      /* the grant covers the request */
     for (uint32_t i = e.getBlockTid(); i < words; i += n) p[i] = key ^ (i * 0x9E3779B9u);
     if (a.spin_ns) {
         uint64_t t0 = globaltimer_ns();
@@ -107,6 +108,50 @@ __device__ void body_gate(const Env&, const pagoda_gate_args& a)
     }
     __syncwarp();
 }
+
+/* Brute-force schedule body (SURVEY §4 layer 4): announce the start, fill the whole grant with a
+ * per-TB pattern, hold until the host opens the gate, then verify that no other task wrote into
+ * the grant meanwhile (granules never overlap).  `started` and `flag` may live in pinned
+ * host memory: plain stores / loads, one per warp (no system-scope atomics over PCIe). */
+template <class Env>
+__device__ __noinline__ void body_hold(const Env& e, const pagoda_hold_args& a)
+{
+    uint32_t* p = reinterpret_cast<uint32_t*>(e.getSMPtr());
+    const uint32_t words = e.getSMBytes() / 4u;
+    const uint32_t key = a.seed * 2654435761u + (uint32_t)e.getBlockIdx() * 40503u;
+    const int n = tb_threads(e);
+    uint32_t errs = 0;
+    if (lane_id() == 0) *reinterpret_cast<volatile uint32_t*>(a.started) = 1u;
+    for (uint32_t i = e.getBlockTid(); i < words; i += n) p[i] = key ^ (i * 0x9E3779B9u);
+    if (lane_id() == 0)
+        while (*a.flag == 0) __nanosleep(500);
+    __syncwarp();
+    if (e.canSync()) e.syncBlock();
+    for (uint32_t i = e.getBlockTid(); i < words; i += n) errs += (p[i] != (key ^ (i * 0x9E3779B9u)));
+    if (errs) atomicAdd(a.err, errs);
+}
+
+/* A body written the way the paper's users write one (Table 1, Fig. 1c): only the free
+ * functions getTid() / syncBlock() / getSMPtr(), no Env.  They read the MasterKernel's WarpTable, so
+ * this body exists only inside the MasterKernel (run_body refuses it elsewhere). */
+static __device__ __noinline__ void body_paper(const pagoda_paper_args& a)
+{
+    const pagoda::WarpSlot& s = pagoda_my_slot();
+    const int tid = getTid();
+    const int bt = (int)s.warp_in_tb * 32 + (int)lane_id(), n = 32 * (int)s.warps_tb;
+    const bool live = bt < (int)s.threads_tb;
+    uint32_t errs = 0;
+    if (live) a.out[a.base + (uint32_t)tid] = (uint32_t)tid + 1u;
+    syncBlock();
+    const int nb = (bt + 32) % n;   /* the thread one warp on, in this TB */
+    const int ntid = ((int)s.tb * (int)s.warps_tb) * 32 + nb;
+    if (live && nb < (int)s.threads_tb && a.out[a.base + (uint32_t)ntid] != (uint32_t)ntid + 1u) errs++;
+    if (bt == 0 && (reinterpret_cast<uintptr_t>(getSMPtr()) & 31u) != 0) errs++;   /* 32-byte aligned */
+    if (errs) atomicAdd(a.err, errs);
+}
+
+template <class Env> struct IsTaskEnv { static constexpr bool value = false; };
+template <> struct IsTaskEnv<TaskEnv> { static constexpr bool value = true; };
 
 /* ------------------------------------------------------------- MB
  * Table 3; strict '>' escape test, count includes
@@ -831,6 +876,14 @@ __device__ __forceinline__ bool run_body(int func_id, const Env& e, const void* 
     case PAGODA_SMEM: body_smem(e, *static_cast<const pagoda_smem_args*>(args)); return true;
     case PAGODA_SPIN: body_spin(e, *static_cast<const pagoda_spin_args*>(args)); return true;
     case PAGODA_GATE: body_gate(e, *static_cast<const pagoda_gate_args*>(args)); return true;
+    case PAGODA_HOLD: body_hold(e, *static_cast<const pagoda_hold_args*>(args)); return true;
+    case PAGODA_PAPER:
+        if constexpr (IsTaskEnv<Env>::value) {
+            body_paper(*static_cast<const pagoda_paper_args*>(args));
+            return true;
+        } else {
+            return false;
+        }
     case PAGODA_MB: body_mb(e, *static_cast<const pagoda_mb_args*>(args)); return true;
     case PAGODA_TDES: body_tdes(e, *static_cast<const pagoda_tdes_args*>(args)); return true;
     case PAGODA_MM: body_mm(e, *static_cast<const pagoda_mm_args*>(args)); return true;
@@ -846,7 +899,7 @@ __device__ __forceinline__ bool run_body(int func_id, const Env& e, const void* 
 
 __host__ __device__ inline bool known_func(int f)
 {
-    return (f >= PAGODA_NOP && f <= PAGODA_GATE) || (f >= PAGODA_MB && f <= PAGODA_MM64);
+    return (f >= PAGODA_NOP && f <= PAGODA_PAPER) || (f >= PAGODA_MB && f <= PAGODA_MM64);
 }
 
 } // namespace pagoda

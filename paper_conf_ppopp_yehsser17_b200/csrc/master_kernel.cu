@@ -385,8 +385,10 @@ __device__ void comp_forwarder(MtbShared& S, const MkParams& p, uint32_t f)
         n = min(n, span);
         if (n == 0) {
             uint32_t done = 0;
-            if (lane == 0) done = *(volatile uint32_t*)&p.dctl->exited >= (uint32_t)p.n_mtb &&
-                                  *(volatile uint64_t*)&p.dctl->dq_tail <= c;
+            /* acquire of the exit count orders the tail read after it: every MTB's reservations
+             * (made before its release-ordered exit increment) are then in the tail we read */
+            if (lane == 0) done = ld_acquire_gpu32(&p.dctl->exited) >= (uint32_t)p.n_mtb &&
+                                  ld_relaxed_gpu(&p.dctl->dq_tail) <= c;
             if (__shfl_sync(0xffffffffu, done, 0)) break;
             __nanosleep(idle < 16 ? 64 : min(512, PAGODA_IDLE_NS));
             idle++;
@@ -869,7 +871,9 @@ __device__ bool sched_place(MtbShared& S, Sched& st, const MkParams& p, int mtb,
 {
     const uint32_t lane = threadIdx.x & 31u;
     const TaskEntry& e = S.tasks[slot];
-    const uint32_t wtb = e.warps_tb, ntb = e.n_tb, gtb = e.gran_tb;
+    /* granules from the request itself (the entry's u8 gran_tb field saturates above 255 granules,
+     * while an MTB's arena can hold up to kMaxGranules) */
+    const uint32_t wtb = e.warps_tb, ntb = e.n_tb, gtb = (e.shmem_bytes + PAGODA_GRANULE - 1u) / PAGODA_GRANULE;
     const bool need_bar = (e.flags & 1u) && wtb > 1;
     if ((uint32_t)__popc(st.free_w) < wtb * ntb || (uint32_t)__popc(st.free_tbs) < ntb ||
         (need_bar && (uint32_t)__popc(st.free_bar) < ntb))
@@ -1482,6 +1486,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) master_kernel(MkParams p
             S.backlog_est = 0;
             S.fwd_done = 0;
             S.claim_after = 0;
+            S.dev_error = &p.dctl->error;
             S.dq_safe = *(volatile uint64_t*)&p.dctl->dq_head + kDqEntries;
             S.sst_seq = 0;
             S.token = 1;

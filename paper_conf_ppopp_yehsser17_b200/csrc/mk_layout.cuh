@@ -22,7 +22,7 @@ struct __align__(64) TaskEntry {
     uint16_t threads_tb;   /* requested threads per TB */
     uint8_t  warps_tb;     /* ceil(threads/32) */
     uint8_t  n_tb;
-    uint8_t  gran_tb;      /* ceil(shmem/512) granules per TB */
+    uint8_t  gran_tb;      /* min(255, ceil(shmem/512)): informational; the MasterKernel derives granules from shmem_bytes */
     uint8_t  flags;        /* bit0 = sync, bit1 = one entry of a task spread over several MTBs (kEntryGroup) */
     uint32_t shmem_bytes;  /* requested bytes per TB */
     uint32_t reserved;     /* group entries: first TB (bits 0-15) | the task's TB count (bits 16-31) */
@@ -213,10 +213,13 @@ struct MtbShared {
     unsigned long long dq_safe;      /* completion-queue positions below this are known free (posters' cache) */
     uint32_t  fwd_done;              /* MTB 0: forwarders that exited */
     unsigned long long claim_after;  /* PAGODA_SPREAD_NS: no claim before this %globaltimer value */
+    uint32_t* dev_error;             /* &DevCtl.error, for the paper-named free syncBlock() (kDevErrorPtrOffset) */
 };
 static_assert(offsetof(MtbShared, wt) == kWarpTableOffset, "WarpTable offset");
 static_assert(offsetof(MtbShared, stage_bar) == kStageBarOffset, "staging mbarriers offset");
 static_assert(offsetof(MtbShared, stage_ph) == kStagePhaseOffset, "staging parities offset");
+static_assert(offsetof(MtbShared, dev_error) == kDevErrorPtrOffset, "device error pointer offset");
+static_assert(kDevErrSyncWithoutFlag == PAGODA_DEVERR_SYNC_WITHOUT_FLAG, "error code");
 static_assert(sizeof(MtbShared) <= kControlBytes && kControlBytes <= kResidentOffset, "control block fits");
 
 } // namespace pagoda

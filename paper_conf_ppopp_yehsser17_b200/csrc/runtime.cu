@@ -101,6 +101,12 @@ struct pagoda_ctx {
     int sessions = 0;
 };
 
+/* Every live context, by device: the MasterKernel's constant bank (registered 3DES keys, DCT
+ * coefficients) is one per device and process, so registration must not race a running
+ * MasterKernel of ANY context on that device (start_kernel takes the same lock). */
+static std::mutex g_ctx_mtx;
+static std::vector<pagoda_ctx*> g_ctxs;
+
 /* ------------------------------------------------------------------ helpers */
 static inline uint64_t now_ns()
 {
@@ -109,11 +115,20 @@ static inline uint64_t now_ns()
     return (uint64_t)ts.tv_sec * 1000000000ull + (uint64_t)ts.tv_nsec;
 }
 
+/* Device error bits that are contract violations (the context is unusable after
+ * them: every later call returns -EIO); PAGODA_DEVERR_LAYOUT is only a notice. */
+static const uint32_t kFatalDevErr = PAGODA_DEVERR_SYNC_WITHOUT_FLAG | PAGODA_DEVERR_BAD_FUNC;
+static inline bool dev_fault(const pagoda_ctx* c)
+{
+    return (c->hctl->error & kFatalDevErr) != 0 || c->faulted.load(std::memory_order_relaxed);
+}
+
 /* Spin with pause / yield back-off; every ~1 ms check device faults and the
  * watchdog.  pred() returns true when done. */
 template <class Pred>
 static int spin_until(pagoda_ctx* c, Pred pred)
 {
+    if (dev_fault(c)) return -EIO;
     if (pred()) return 0;
     const uint64_t t0 = now_ns();
     uint64_t last_check = t0;
@@ -129,7 +144,7 @@ static int spin_until(pagoda_ctx* c, Pred pred)
         const uint64_t t = now_ns();
         if (t - last_check > 1000000ull) {
             last_check = t;
-            if (c->hctl->error) return -EIO;
+            if (dev_fault(c)) return -EIO;
             if (!c->running.load(std::memory_order_acquire)) return pred() ? 0 : -EAGAIN;   /* stopped */
             cudaError_t q = cudaStreamQuery(c->stream);
             if (q != cudaErrorNotReady) {   /* MasterKernel gone while it should run: fault */
@@ -216,7 +231,7 @@ static inline void write_entry(pagoda_ctx* c, uint64_t id0, int j, const int32_t
     e.threads_tb = (uint16_t)s[0];
     e.warps_tb = (uint8_t)sp.wtb;
     e.n_tb = (uint8_t)std::min(sp.cap, s[1] - tb0);
-    e.gran_tb = (uint8_t)sp.gtb;
+    e.gran_tb = (uint8_t)std::min<uint32_t>(sp.gtb, 255u);
     e.flags = (s[3] ? 1 : 0) | (sp.k > 1 ? kEntryGroup : 0);
     e.shmem_bytes = (uint32_t)s[2];
     e.reserved = sp.k > 1 ? ((uint32_t)tb0 | ((uint32_t)s[1] << 16)) : 0u;
@@ -234,6 +249,52 @@ static inline void write_entry(pagoda_ctx* c, uint64_t id0, int j, const int32_t
 template <class ShapeOf>
 static int64_t spawn_batch(pagoda_ctx* c, int n, ShapeOf shape_of, const void* args_base, size_t args_stride,
                            size_t args_bytes, pagoda_task_t* ids_out);
+
+/* Ring slot `last` (and every one before it) is free: the ingest warp has copied entry last - R. */
+static bool ring_room(pagoda_ctx* c, uint64_t last)
+{
+    if (last < c->R) return true;
+    uint64_t cur = c->consumed_cache.load(std::memory_order_acquire);
+    if (cur > last - c->R) return true;
+    const uint64_t v = c->hctl->consumed;
+    while (v > cur && !c->consumed_cache.compare_exchange_weak(cur, v)) { }
+    return v > last - c->R;
+}
+/* Completion slot `last` is free: task last - C is done. */
+static bool comp_room(pagoda_ctx* c, uint64_t last)
+{
+    if (last < c->C || c->low.load(std::memory_order_acquire) > last - c->C) return true;
+    advance_low(c, last - c->C + 1);
+    return c->low.load(std::memory_order_acquire) > last - c->C;
+}
+
+/* Reserve K consecutive ids.  The id sequence never gets a hole: when the ring
+ * or completion slots those ids need are taken and waiting could not free them
+ * (PAGODA_NONBLOCKING_SPAWN, or a stopped session, where nothing drains the
+ * ring), nothing is reserved and -EAGAIN returned.  Otherwise the caller waits
+ * for the slots after reserving; if that wait then fails (device fault,
+ * watchdog) the ids stay unpublished, so the context is marked faulted
+ * (reserve_failed) and every later call returns -EIO instead of waiting for
+ * them. */
+static int reserve_ids(pagoda_ctx* c, uint64_t K, uint64_t* id0)
+{
+    const bool nonblock = (c->cfg.flags & PAGODA_NONBLOCKING_SPAWN) != 0;
+    uint64_t cur = c->next_id.load(std::memory_order_acquire);
+    for (;;) {
+        const uint64_t last = cur + K - 1;
+        const bool room = ring_room(c, last) && comp_room(c, last);
+        if (!room && (nonblock || !c->running.load(std::memory_order_acquire))) return -EAGAIN;
+        if (c->next_id.compare_exchange_weak(cur, cur + K, std::memory_order_acq_rel)) {
+            *id0 = cur;
+            return 0;
+        }
+    }
+}
+static int reserve_failed(pagoda_ctx* c, int rc)
+{
+    c->faulted.store(1, std::memory_order_release);
+    return rc;
+}
 
 extern "C" {
 
@@ -265,6 +326,7 @@ static int start_kernel(pagoda_ctx* c)
         cudaMemsetAsync(c->trace_count, 0, (size_t)c->n_mtb * sizeof(uint32_t), c->stream);
         cudaMemsetAsync(c->exec_count, 0, (size_t)c->n_mtb * 32 * sizeof(uint32_t), c->stream);
     }
+    std::lock_guard<std::mutex> reg(g_ctx_mtx);   /* no constant-bank registration during the launch */
     cudaEventRecord(c->ev_start, c->stream);
     cudaError_t e = launch_master(c->cfg.mtbs_per_sm, c->n_mtb, c->smem, c->stream, &c->params, &c->regs);
     if (e != cudaSuccess) {
@@ -324,12 +386,16 @@ static int stop_kernel(pagoda_ctx* c, bool abort_now = false)
     const uint32_t none = kIoSmidNone;   /* MTB 0 announces its SM again next session */
     cudaMemcpy(&c->dctl->io_smid, &none, 4, cudaMemcpyHostToDevice);
     if (cudaStreamSynchronize(c->stream) != cudaSuccess) return -EIO;
-    return c->hctl->error ? -EIO : 0;
+    return (c->hctl->error & kFatalDevErr) ? -EIO : 0;
 }
 
 static void free_ctx(pagoda_ctx* c)
 {
     if (!c) return;
+    {
+        std::lock_guard<std::mutex> reg(g_ctx_mtx);
+        g_ctxs.erase(std::remove(g_ctxs.begin(), g_ctxs.end(), c), g_ctxs.end());
+    }
     c->helpers_quit.store(1, std::memory_order_release);
     for (auto& t : c->helpers) t.join();
     if (c->hctl) cudaFreeHost(c->hctl);
@@ -495,6 +561,10 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
             p.spread_ns = e ? (uint32_t)strtoul(e, nullptr, 10) : 6000u;
         }
         c->smem = smem;
+        {
+            std::lock_guard<std::mutex> reg(g_ctx_mtx);
+            g_ctxs.push_back(c);
+        }
         rc = (cfg.flags & PAGODA_NO_START) ? 0 : start_kernel(c);
         if (rc) goto fail;
     }
@@ -511,7 +581,7 @@ pagoda_task_t pagoda_taskSpawn(pagoda_ctx* c, int threads, int n_tb, int shmem_b
 {
     if (!c) return -EINVAL;
     if (c->shutting.load(std::memory_order_acquire)) return -ESHUTDOWN;
-    if (c->faulted.load(std::memory_order_relaxed)) return -EIO;
+    if (dev_fault(c)) return -EIO;
     const int32_t shape[5] = {threads, n_tb, shmem_bytes, sync_flag, func_id};
     Split sp;
     if (int rc = shape_check(c, shape, sp)) return rc;
@@ -524,24 +594,17 @@ pagoda_task_t pagoda_taskSpawn(pagoda_ctx* c, int threads, int n_tb, int shmem_b
     const int wtb = sp.wtb;
     const uint32_t gtb = sp.gtb;
 
-    const uint64_t id = c->next_id.fetch_add(1, std::memory_order_acq_rel);
+    uint64_t id = 0;
+    if (int rc = reserve_ids(c, 1, &id)) return rc;
     /* 1. ring slot free: the ingest warp has copied entry id - R */
-    if (id >= c->R && c->consumed_cache.load(std::memory_order_acquire) <= id - c->R) {
-        int rc = spin_until(c, [&] {
-            const uint64_t v = c->hctl->consumed;
-            uint64_t cur = c->consumed_cache.load(std::memory_order_relaxed);
-            while (v > cur && !c->consumed_cache.compare_exchange_weak(cur, v)) { }
-            return v > id - c->R;
-        });
-        if (rc) return rc;
+    if (!ring_room(c, id)) {
+        int rc = spin_until(c, [&] { return ring_room(c, id); });
+        if (rc) return reserve_failed(c, rc);
     }
     /* 2. completion slot free: task id - C is done */
-    if (id >= c->C && c->low.load(std::memory_order_acquire) <= id - c->C) {
-        int rc = spin_until(c, [&] {
-            advance_low(c, id - c->C + 1);
-            return c->low.load(std::memory_order_acquire) > id - c->C;
-        });
-        if (rc) return rc;
+    if (!comp_room(c, id)) {
+        int rc = spin_until(c, [&] { return comp_room(c, id); });
+        if (rc) return reserve_failed(c, rc);
     }
     /* 3. the entry */
     write_entry(c, id, 0, shape, sp, args, args_bytes);
@@ -550,7 +613,7 @@ pagoda_task_t pagoda_taskSpawn(pagoda_ctx* c, int threads, int n_tb, int shmem_b
     /* 4. in-order commit of the doorbell (x86 stores are ordered; the fence is for the compiler) */
     if (c->published.load(std::memory_order_acquire) != id) {
         int rc = spin_until(c, [&] { return c->published.load(std::memory_order_acquire) == id; });
-        if (rc) return rc;
+        if (rc) return reserve_failed(c, rc);
     }
     c->warps_prefix[id & (c->C - 1)] = c->warps_spawned.fetch_add(w, std::memory_order_relaxed) + w;
     std::atomic_thread_fence(std::memory_order_release);
@@ -571,7 +634,7 @@ static int64_t spawn_batch(pagoda_ctx* c, int n, ShapeOf shape_of, const void* a
 {
     if (!c || n < 0) return -EINVAL;
     if (c->shutting.load(std::memory_order_acquire)) return -ESHUTDOWN;
-    if (c->faulted.load(std::memory_order_relaxed)) return -EIO;
+    if (dev_fault(c)) return -EIO;
     if (args_bytes > PAGODA_ARGS_MAX || (args_bytes > 0 && !args_base)) return -EINVAL;
     ShapeMemo memo;
     for (int i = 0; i < n; i++) {
@@ -590,23 +653,16 @@ static int64_t spawn_batch(pagoda_ctx* c, int n, ShapeOf shape_of, const void* a
             K += (uint64_t)sps[m].k;
             m++;
         }
-        const uint64_t id0 = c->next_id.fetch_add(K, std::memory_order_acq_rel);
+        uint64_t id0 = 0;
+        if (int rc = reserve_ids(c, K, &id0)) return base ? (int64_t)base : (int64_t)rc;   /* tasks before stay */
         const uint64_t last = id0 + K - 1;
-        if (last >= c->R && c->consumed_cache.load(std::memory_order_acquire) <= last - c->R) {
-            int rc = spin_until(c, [&] {
-                const uint64_t v = c->hctl->consumed;
-                uint64_t cur = c->consumed_cache.load(std::memory_order_relaxed);
-                while (v > cur && !c->consumed_cache.compare_exchange_weak(cur, v)) { }
-                return v > last - c->R;
-            });
-            if (rc) return rc;
+        if (!ring_room(c, last)) {
+            int rc = spin_until(c, [&] { return ring_room(c, last); });
+            if (rc) return reserve_failed(c, rc);
         }
-        if (last >= c->C && c->low.load(std::memory_order_acquire) <= last - c->C) {
-            int rc = spin_until(c, [&] {
-                advance_low(c, last - c->C + 1);
-                return c->low.load(std::memory_order_acquire) > last - c->C;
-            });
-            if (rc) return rc;
+        if (!comp_room(c, last)) {
+            int rc = spin_until(c, [&] { return comp_room(c, last); });
+            if (rc) return reserve_failed(c, rc);
         }
         uint64_t id = id0;
         for (int i = 0; i < m; i++) {
@@ -619,7 +675,7 @@ static int64_t spawn_batch(pagoda_ctx* c, int n, ShapeOf shape_of, const void* a
         }
         if (c->published.load(std::memory_order_acquire) != id0) {
             int rc = spin_until(c, [&] { return c->published.load(std::memory_order_acquire) == id0; });
-            if (rc) return rc;
+            if (rc) return reserve_failed(c, rc);
         }
         int64_t ws = c->warps_spawned.load(std::memory_order_relaxed);
         id = id0;
@@ -653,6 +709,7 @@ static int64_t spawn_part(pagoda_ctx* c, const pagoda_ctx::SpawnJob& j, int t)
                                        j.bytes ? j.args + (size_t)b0 * j.stride : nullptr, j.stride, j.bytes,
                                        j.ids ? j.ids + b0 : nullptr);
         if (rc < 0) return rc;
+        if (rc < m) return -EAGAIN;   /* ring full (non-blocking spawn / stopped): the block is cut short */
     }
     return 0;
 }
@@ -734,9 +791,9 @@ int pagoda_check(pagoda_ctx* c, pagoda_task_t id)
 {
     if (!c) return -EINVAL;
     if (id < 0 || (uint64_t)id >= c->next_id.load(std::memory_order_acquire)) return -EINVAL;
+    if (dev_fault(c)) return -EIO;
     if ((uint64_t)id < c->low.load(std::memory_order_acquire)) return 1;
     if (c->comp[(uint64_t)id & (c->C - 1)] >= id) return 1;
-    if (c->hctl->error) return -EIO;
     return 0;
 }
 
@@ -744,6 +801,7 @@ int pagoda_wait(pagoda_ctx* c, pagoda_task_t id)
 {
     if (!c) return -EINVAL;
     if (id < 0 || (uint64_t)id >= c->next_id.load(std::memory_order_acquire)) return -EINVAL;
+    if (dev_fault(c)) return -EIO;
     if ((uint64_t)id < c->low.load(std::memory_order_acquire)) return 0;
     volatile int64_t* slot = &c->comp[(uint64_t)id & (c->C - 1)];
     int rc = spin_until(c, [&] { return *slot >= id; });
@@ -842,7 +900,7 @@ int pagoda_shutdown(pagoda_ctx* c)
         }
         c->shutting.store(1, std::memory_order_release);
     }
-    if (c->hctl->error && rc == 0) rc = -EIO;
+    if ((c->hctl->error & kFatalDevErr) && rc == 0) rc = -EIO;
     cudaSetDevice(c->device);
     if (c->ev_start) cudaEventDestroy(c->ev_start);
     if (c->ev_stop) cudaEventDestroy(c->ev_stop);
@@ -923,10 +981,19 @@ int64_t pagoda_inflight_warps(pagoda_ctx* c)
     return spawned - done;
 }
 
+/* a MasterKernel of some context on c's device is running (caller holds g_ctx_mtx) */
+static bool device_busy(const pagoda_ctx* c)
+{
+    for (const pagoda_ctx* o : g_ctxs)
+        if (o->device == c->device && o->running.load(std::memory_order_acquire)) return true;
+    return false;
+}
+
 int pagoda_tdes_register(pagoda_ctx* c, const void* dev_tables)
 {
     if (!c) return -EINVAL;
-    if (c->running.load()) return -EBUSY;
+    std::lock_guard<std::mutex> reg(g_ctx_mtx);
+    if (device_busy(c)) return -EBUSY;
     cudaSetDevice(c->device);
     uint8_t keys[384] = {0};
     uint64_t ptr = 0;
@@ -944,7 +1011,8 @@ int pagoda_tdes_register(pagoda_ctx* c, const void* dev_tables)
 int pagoda_dct_register(pagoda_ctx* c, const float* dev_coef)
 {
     if (!c) return -EINVAL;
-    if (c->running.load()) return -EBUSY;
+    std::lock_guard<std::mutex> reg(g_ctx_mtx);
+    if (device_busy(c)) return -EBUSY;
     cudaSetDevice(c->device);
     float coef[64] = {0};
     uint64_t ptr = 0;

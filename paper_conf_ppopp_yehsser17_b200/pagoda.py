@@ -22,6 +22,7 @@ NO_START = 0x2
 RESIDENT_TDES = 0x4
 LIFECYCLE = 0x8
 SPREAD = 0x10
+NONBLOCKING_SPAWN = 0x20
 LIFE_EVENTS = ("pub", "load", "place", "start", "end", "done", "queued", "fwd")
 
 
@@ -122,6 +123,18 @@ def _check(rc: int, what: str) -> int:
     return rc
 
 
+def _check_count(rc: int, n: int, what: str) -> None:
+    """A batched spawn cut short by a full ring (PAGODA_NONBLOCKING_SPAWN or a stopped
+    session) returns how many it spawned; `spawned` carries that count."""
+    if rc == n:
+        return
+    if rc == -errno.EAGAIN or 0 <= rc < n:
+        e = PagodaError(errno.EAGAIN, f"{what}: ring full after {max(rc, 0)} of {n} tasks")
+        e.spawned = max(rc, 0)
+        raise e
+    _check(rc, what)
+
+
 def _ptr(a):
     if a is None:
         return None
@@ -175,7 +188,7 @@ class Pagoda:
         stride = args.dtype.itemsize if args is not None else 0
         rc = lib().pagoda_taskSpawnMany(self.h, n, threads, n_tb, shmem, int(sync), func_id, _ptr(args),
                                         stride, stride, _ptr(out))
-        _check(rc, "pagoda_taskSpawnMany")
+        _check_count(rc, n, "pagoda_taskSpawnMany")
         return out
 
     def spawn_shapes(self, shapes: np.ndarray, args: np.ndarray, ids=False, producers: int = 1):
@@ -192,7 +205,7 @@ class Pagoda:
         else:
             rc = lib().pagoda_taskSpawnShapes(self.h, n, _ptr(shapes), _ptr(args), args.shape[1], args.shape[1],
                                               _ptr(out))
-            _check(rc, "pagoda_taskSpawnShapes")
+            _check_count(rc, n, "pagoda_taskSpawnShapes")
         return out
 
     # --- sessions ------------------------------------------------------------

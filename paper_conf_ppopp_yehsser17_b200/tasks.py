@@ -5,12 +5,13 @@ Marshalling only: these are the byte layouts the C structs have.
 """
 import numpy as np
 
-NOP, MARK, TID, BAR, SMEM, SPIN, GATE = 0, 1, 2, 3, 4, 5, 6
+NOP, MARK, TID, BAR, SMEM, SPIN, GATE, HOLD, PAPER = 0, 1, 2, 3, 4, 5, 6, 7, 8
 MB, TDES, MM, FB, BF, CONV, DCT = 16, 17, 18, 19, 20, 21, 22
 MM_TC = 23
 MM64 = 24   # Table 4's 64x64 MatrixMul (NEXT-4)
 
 NAMES = {NOP: "nop", MARK: "mark", TID: "tid", BAR: "bar", SMEM: "smem", SPIN: "spin", GATE: "gate",
+         HOLD: "hold", PAPER: "paper",
          MB: "mb", TDES: "tdes", MM: "mm", FB: "fb", BF: "bf", CONV: "conv", DCT: "dct", MM_TC: "mm_tc", MM64: "mm64"}
 
 _p = "<u8"
@@ -21,6 +22,8 @@ ARGS = {
     SMEM: np.dtype([("err", _p), ("bytes", "<u4"), ("spin_ns", "<u4"), ("seed", "<u4"), ("pad", "<u4")]),
     SPIN: np.dtype([("ns", "<u8")]),
     GATE: np.dtype([("flag", _p)]),
+    HOLD: np.dtype([("flag", _p), ("err", _p), ("started", _p), ("seed", "<u4"), ("pad", "<u4")]),
+    PAPER: np.dtype([("out", _p), ("err", _p), ("base", "<u4"), ("pad", "<u4")]),
     MB: np.dtype([("out", _p), ("x0", "<f4"), ("y0", "<f4"), ("dx", "<f4"), ("tx", "<i4"), ("ty", "<i4"),
                   ("maxit", "<i4")]),
     TDES: np.dtype([("inp", _p), ("out", _p), ("tables", _p), ("nblk", "<u4"), ("pad", "<u4")]),

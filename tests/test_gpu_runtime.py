@@ -470,3 +470,100 @@ def test_pool_least_loaded_spawner():
                "tdes": lambda pk: oracle.tdes_ecb(pk, __import__("paper_conf_ppopp_yehsser17_b200.inputs",
                                                                   fromlist=["x"]).TDES_KEYS)}[kind](*args)
         assert np.array_equal(w.task_output(k), ref), (kind, k)
+
+
+# ---------------------------------------------------------------- device errors and the paper-named device API
+def test_paper_free_functions_body():
+    """A body written only against the paper's free functions getTid() / syncBlock() /
+    getSMPtr() (Table 1, PAGODA_PAPER): multi-warp TBs of sync tasks exchange
+    values across warps through syncBlock, getTid covers [0, 32 w n_tb) once, no errors."""
+    dev = Dev()
+    shapes = [(64, 1, 1), (100, 3, 1), (256, 2, 1), (32, 4, 0), (1024, 1, 1)]   # threads, n_tb, sync
+    span = [((th + 31) // 32) * 32 * nb for th, nb, _ in shapes]
+    out = dev.zeros(4 * sum(span))
+    err = dev.zeros(8)
+    with Pagoda() as p:
+        base = 0
+        for (th, nb, sy), sp in zip(shapes, span):
+            a = np.array([(ptr(out), ptr(err), base, 0)], T.ARGS[T.PAPER])
+            assert p.taskSpawn(th, nb, 512, sy, T.PAPER, a) >= 0
+            base += sp
+        assert p.waitAll() == 0 and p.info().device_error == 0
+    o = Dev.get(out, np.uint32)
+    assert Dev.get(err, np.uint32)[0] == 0
+    base = 0
+    for (th, nb, _), sp in zip(shapes, span):
+        w = (th + 31) // 32
+        seg = o[base: base + sp].reshape(nb, 32 * w)
+        tids = np.arange(sp).reshape(nb, 32 * w)
+        assert (seg[:, :th] == tids[:, :th] + 1).all() and (seg[:, th:] == 0).all()
+        base += sp
+
+
+@pytest.mark.parametrize("body", ["paper", "env"])
+def test_sync_without_flag_is_a_device_error(body):
+    """syncBlock() in a multi-warp TB spawned with sync=0 (it has no barrier ID)
+    sets PAGODA_DEVERR_SYNC_WITHOUT_FLAG — from the free function (PAPER body) and from the
+    Env form (BAR body) alike — and every later host call on the context returns -EIO."""
+    dev = Dev()
+    out = dev.zeros(4 * 4096)
+    err = dev.zeros(8)
+    scratch = dev.zeros(4 * 4096)
+    p = Pagoda()
+    if body == "paper":
+        good = np.array([(ptr(out), ptr(err), 0, 0)], T.ARGS[T.PAPER])
+        bad = np.array([(ptr(out), ptr(err), 1024, 0)], T.ARGS[T.PAPER])
+        func = T.PAPER
+    else:
+        good = bad = np.array([(ptr(err), ptr(scratch), 2, 0)], T.ARGS[T.BAR])
+        func = T.BAR
+    ok = p.taskSpawn(128, 2, 0, 1, func, good)
+    one_warp = p.taskSpawn(32, 2, 0, 0, func, good)      # 1-warp TBs may syncBlock without the flag
+    assert p.wait(ok) == 0 and p.wait(one_warp) == 0 and p.info().device_error == 0
+    tid = p.taskSpawn(64, 1, 0, 0, func, bad)           # 2 warps, sync = 0: violation
+    assert tid >= 0
+    t0 = time.time()
+    while p.info().device_error == 0 and time.time() - t0 < 5:
+        time.sleep(0.001)
+    assert p.info().device_error & 1
+    E = -errno.EIO
+    assert p.wait(tid) == E and p.check(tid) == E and p.check(ok) == E
+    assert p.waitAll() == E
+    assert p.taskSpawn(32, 1, 0, 0, T.NOP) == E
+    assert p.shutdown() == E
+
+
+def test_nonblocking_spawn_eagain_without_id_holes():
+    """PAGODA_NONBLOCKING_SPAWN: while the ring is full, taskSpawn returns
+    -EAGAIN at once and reserves no id; a stopped session with a full ring does the same
+    even without the flag; the ids that were issued stay contiguous and all complete."""
+    from paper_conf_ppopp_yehsser17_b200.pagoda import NO_START, NONBLOCKING_SPAWN, PagodaError
+    R = 256
+    for flags in (NO_START | NONBLOCKING_SPAWN, NO_START):
+        with Pagoda(ring_entries=R, comp_entries=1024, flags=flags, watchdog_s=20.0) as p:
+            ids = p.spawn_many(R, 64, 1, 0, False, T.NOP, None, ids=True)   # stopped: fills the ring
+            assert np.array_equal(ids, np.arange(R))
+            assert p.taskSpawn(64, 1, 0, False, T.NOP) == -errno.EAGAIN
+            with pytest.raises(PagodaError) as ei:
+                p.spawn_many(10, 64, 1, 0, False, T.NOP, None)
+            assert ei.value.errno == errno.EAGAIN and ei.value.spawned == 0
+            assert p.info().spawned == R                                   # no id was taken
+            assert p.start() == 0
+            assert p.waitAll() == 0
+            tid = p.taskSpawn(64, 1, 0, False, T.NOP)
+            assert tid == R and p.wait(tid) == 0
+
+
+def test_shmem_grant_above_255_granules():
+    """A request of more than 255 granules (here 140000 B = 274 granules, 1 MTB/SM with a
+    200 KiB arena) gets its whole grant: the SMEM body fails if getSMBytes() < the request
+    and verifies every word it filled."""
+    dev = Dev()
+    err = dev.zeros(8)
+    with Pagoda(mtbs_per_sm=1, arena_bytes=200 * 1024) as p:
+        for k, nbytes in enumerate((130560, 131072, 140000, 200 * 1024)):
+            a = T.records(T.SMEM, 1)
+            a["err"], a["bytes"], a["spin_ns"], a["seed"] = ptr(err), nbytes, 1000, k
+            assert p.taskSpawn(256, 1, nbytes, True, T.SMEM, a) >= 0
+        assert p.waitAll() == 0 and p.info().device_error == 0
+    assert Dev.get(err, np.uint32)[0] == 0
