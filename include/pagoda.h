@@ -203,6 +203,15 @@ int pagoda_latency_loop(pagoda_ctx* ctx, int n, int threads, int n_threadblocks,
  * -ENOMEM, -EIO, -ETIMEDOUT. */
 int pagoda_pingpong(int device, int n, int64_t* rtt_ns);
 
+/* Roofline denominators the paper's hardware never had to name ("the LDS and
+ * INT32 peaks are not published: microbenchmark them on the box").  which = 0: shared-memory
+ * lookups of the 3DES pattern (lane-replicated table, one bank per lane); which = 1: INT32
+ * lop3.b32.  Two 1024-thread blocks per SM, 8 independent chains per thread; each block times
+ * itself in SM cycles.  *per_sm_clk = lanes (ops) per SM per clock; *ops_per_s (nullable) =
+ * whole-kernel ops/s by CUDA events at the clock it ran at.  Run while no MasterKernel holds
+ * the device.  Returns 0, -EINVAL, -ENODEV, -ENOMEM, -EIO. */
+int pagoda_measure_pipe_peak(int device, int which, double* per_sm_clk, double* ops_per_s);
+
 /* Runtime counters accumulated on the device since the context was created
  * (read while stopped or running; ns are %globaltimer nanoseconds). */
 enum {
@@ -309,9 +318,14 @@ int pagoda_naive_run(int device, int n, const int32_t* shapes, const void* args_
 int pagoda_fused_run(int device, int n, const int32_t* shapes, const void* args_base, size_t args_stride,
                      size_t args_bytes, int threads_per_task, int64_t* elapsed_ns, float* kernel_ms);
 
-/* ---- multi-GPU pool: one context per GPU, least-loaded picker */
+/* ---- multi-GPU pool: one context (MasterKernel) per GPU, tasks least-loaded-first.
+ * Tasks are independent: no collective, host-side only.  Each member has its own
+ * spawner thread, bound to the CPUs of its GPU's NUMA node; that thread creates the member's
+ * context, so the pinned rings are allocated on that node. */
 typedef struct pagoda_pool pagoda_pool;
-/* Start one context per device in devices[0..n_dev) with cfg (device field ignored). */
+/* One member per entry of devices[0..n_dev) with cfg (device field ignored; several entries may
+ * name the same device, each then running a MasterKernel of cfg->num_sms SMs, e.g. 2 x 74 on
+ * one B200).  cfg may carry PAGODA_NO_START (start members with pagoda_start(pagoda_pool_ctx)). */
 int pagoda_pool_init(int n_dev, const int* devices, const pagoda_config* cfg, pagoda_pool** out);
 /* Index of the device with the fewest in-flight warps (spawned, not yet seen
  * completed); ties go to the lowest index.  warps_hint is added to the chosen
@@ -324,17 +338,26 @@ int pagoda_pool_size(pagoda_pool* pool);
 pagoda_task_t pagoda_pool_spawn(pagoda_pool* pool, int threads, int n_threadblocks, int shmem_bytes,
                                 int sync_flag, int func_id, const void* const* args_per_dev,
                                 size_t args_bytes, int* index_out);
-/* Batched form: runs of up to `chunk` consecutive tasks (shapes as in
- * pagoda_taskSpawnShapes) each go to the least-loaded context at the time of
- * the pick; args_base_per_dev[i] + k * args_stride are task k's args if it
- * lands on device i (device pointers of that device).  ids_out / dev_out
- * (nullable) receive each task's id and device index.  Returns n or the first
- * error. */
+/* Batched form: the n tasks (shapes as in pagoda_taskSpawnShapes) are cut into
+ * runs of `chunk` consecutive tasks; every member's spawner thread claims the
+ * next run only while its GPU is among the least loaded (in-flight warps within
+ * two runs' warps of the smallest member's: pagoda_pool_may_claim), and spawns
+ * it on its own context; so runs go least-loaded-first and the members' rings
+ * are written in parallel.  args_base_per_dev[i] + k * args_stride are task k's
+ * args if it lands on member i (device pointers of that device).  ids_out /
+ * dev_out (nullable) receive each task's id and member index.  Returns n once
+ * every task is spawned, or the first error. */
 int64_t pagoda_pool_spawn_shapes(pagoda_pool* pool, int n, const int32_t* shapes, const void* const* args_base_per_dev,
                                  size_t args_stride, size_t args_bytes, int chunk, pagoda_task_t* ids_out,
                                  int32_t* dev_out);
 int pagoda_pool_waitAll(pagoda_pool* pool);
 int pagoda_pool_shutdown(pagoda_pool* pool);
+/* NUMA node member i's spawner thread is bound to (-1: unknown / not bound). */
+int pagoda_pool_numa_node(pagoda_pool* pool, int index);
+/* Member i's share of the last batched spawn: tasks it spawned, ns inside its spawn calls
+ * (the host cost: tasks / spawn_ns is that thread's spawn rate), ns it held back because
+ * another member was less loaded.  Returns 0 or -EINVAL. */
+int pagoda_pool_stats(pagoda_pool* pool, int index, int64_t* tasks, int64_t* spawn_ns, int64_t* hold_ns);
 
 /* In-flight warps of one context: warps of spawned tasks minus those of the
  * tasks below its completion watermark (the pool's load measure). */
@@ -342,6 +365,9 @@ int64_t pagoda_inflight_warps(pagoda_ctx* ctx);
 /* The picker rule alone (host-only, testable without a GPU): index of the
  * smallest of loads[0..n), ties to the lowest index; -EINVAL if n < 1. */
 int pagoda_pick_least_loaded(const int64_t* loads, int n);
+/* The spawner's claim rule alone (host-only): 1 if loads[me] <= min(loads) + slack, else 0;
+ * -EINVAL on bad arguments. */
+int pagoda_pool_may_claim(const int64_t* loads, int n, int me, int64_t slack);
 
 /* Library version string. */
 const char* pagoda_version(void);

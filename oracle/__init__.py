@@ -22,33 +22,39 @@ import numpy as np
 HERE = os.path.dirname(os.path.abspath(__file__))
 SRC = os.path.join(HERE, "oracle.c")
 LIB = os.path.join(HERE, "liboracle.so")
+LIB_FAST = os.path.join(HERE, "liboracle_fast.so")
 
 CFLAGS = ["-O2", "-std=c11", "-Wall", "-ffp-contract=off", "-fno-fast-math", "-fPIC", "-shared"]
+# the TIMED build (SURVEY §8(d) "CPU oracle"): same source, -O3 -march=native, still no contraction
+# (so its outputs equal the parity build's; bench.py checks a sample)
+CFLAGS_FAST = ["-O3", "-march=native", "-std=c11", "-Wall", "-ffp-contract=off", "-fno-fast-math", "-fPIC",
+               "-shared"]
 
 # func ids — the oracle's own numbering (oracle.h)
 NOP, MARK, TID, MB, TDES, MM, FB, BF, CONV, DCT, MM_TC = 0, 1, 2, 16, 17, 18, 19, 20, 21, 22, 23
 
 _lock = threading.Lock()
-_lib = None
+_libs = {}
 
 
-def build(force: bool = False) -> str:
-    """Compile oracle.c -> liboracle.so with gcc (no CUDA)."""
-    stale = (not os.path.exists(LIB)) or any(
-        os.path.getmtime(os.path.join(HERE, f)) > os.path.getmtime(LIB)
-        for f in ("oracle.c", "oracle.h"))
+def build(force: bool = False, fast: bool = False) -> str:
+    """Compile oracle.c -> liboracle.so (parity build) or liboracle_fast.so (timed build) with gcc (no CUDA)."""
+    out, flags = (LIB_FAST, CFLAGS_FAST) if fast else (LIB, CFLAGS)
+    stale = (not os.path.exists(out)) or any(
+        os.path.getmtime(os.path.join(HERE, f)) > os.path.getmtime(out)
+        for f in ("oracle.c", "oracle.h", "__init__.py"))
     if force or stale:
-        tmp = LIB + f".tmp{os.getpid()}"
-        subprocess.check_call(["gcc", *CFLAGS, "-o", tmp, SRC, "-lm"])
-        os.replace(tmp, LIB)
-    return LIB
+        tmp = out + f".tmp{os.getpid()}"
+        subprocess.check_call(["gcc", *flags, "-o", tmp, SRC, "-lm"])
+        os.replace(tmp, out)
+    return out
 
 
-def lib():
-    global _lib
+def lib(fast: bool = False):
+    """The parity build (default) or the -O3 -march=native timed build."""
     with _lock:
-        if _lib is None:
-            L = C.CDLL(build())
+        if fast not in _libs:
+            L = C.CDLL(build(fast=fast))
             P, I, I64, F, SZ = C.c_void_p, C.c_int, C.c_int64, C.c_float, C.c_size_t
             L.orc_mandelbrot_tile.argtypes = [P, F, F, F, I, I, I]
             L.orc_des_key_schedule.argtypes = [P, P]
@@ -74,8 +80,8 @@ def lib():
             L.orc_occupancy_pct.restype = C.c_double
             L.orc_ledger_check.argtypes = [P, SZ, I, I, I, I, P, SZ, C.c_char_p, SZ]
             L.orc_exec_check.argtypes = [P, SZ, P, SZ, P, SZ, P, SZ, C.c_char_p, SZ]
-            _lib = L
-    return _lib
+            _libs[fast] = L
+    return _libs[fast]
 
 
 def _p(a: np.ndarray):
@@ -84,9 +90,9 @@ def _p(a: np.ndarray):
 
 
 # ----------------------------------------------------------------- bodies
-def mandelbrot_tile(tx: int, ty: int, x0=-2.0, y0=-1.5, dx=3.0 / 2048, maxit=256) -> np.ndarray:
+def mandelbrot_tile(tx: int, ty: int, x0=-2.0, y0=-1.5, dx=3.0 / 2048, maxit=256, L=None) -> np.ndarray:
     out = np.zeros((64, 64), np.uint16)
-    lib().orc_mandelbrot_tile(_p(out), x0, y0, dx, tx, ty, maxit)
+    (L or lib()).orc_mandelbrot_tile(_p(out), x0, y0, dx, tx, ty, maxit)
     return out
 
 
@@ -102,62 +108,62 @@ def des_block(block: int, key8: bytes, decrypt=False) -> int:
     return int(lib().orc_des_block(C.c_uint64(block), _p(sk), int(decrypt)))
 
 
-def tdes_ecb(data, key24: bytes, decrypt=False) -> np.ndarray:
+def tdes_ecb(data, key24: bytes, decrypt=False, L=None) -> np.ndarray:
     inp = np.ascontiguousarray(np.frombuffer(bytes(data), np.uint8) if not isinstance(data, np.ndarray) else data, dtype=np.uint8)
     out = np.zeros_like(inp)
     k = np.frombuffer(key24, np.uint8).copy()
-    lib().orc_tdes_ecb(_p(inp), _p(out), inp.size, _p(k), int(decrypt))
+    (L or lib()).orc_tdes_ecb(_p(inp), _p(out), inp.size, _p(k), int(decrypt))
     return out
 
 
-def mm32(A, B) -> np.ndarray:
+def mm32(A, B, L=None) -> np.ndarray:
     A = np.ascontiguousarray(A, np.float32); B = np.ascontiguousarray(B, np.float32)
     Cm = np.zeros((32, 32), np.float32)
-    lib().orc_mm32(_p(A), _p(B), _p(Cm))
+    (L or lib()).orc_mm32(_p(A), _p(B), _p(Cm))
     return Cm
 
 
-def mm64(A, B) -> np.ndarray:
+def mm64(A, B, L=None) -> np.ndarray:
     """Table 4's 64x64x64 MatrixMul: fma chain over k ascending, as mm32."""
     A = np.ascontiguousarray(A, np.float32); B = np.ascontiguousarray(B, np.float32)
     Cm = np.zeros((64, 64), np.float32)
-    lib().orc_mm64(_p(A), _p(B), _p(Cm))
+    (L or lib()).orc_mm64(_p(A), _p(B), _p(Cm))
     return Cm
 
 
-def mm32_exact(A, B) -> np.ndarray:
+def mm32_exact(A, B, L=None) -> np.ndarray:
     """C = A B accumulated in fp64, rounded once (the tensor-core MM variant's definition)."""
     A = np.ascontiguousarray(A, np.float32); B = np.ascontiguousarray(B, np.float32)
     Cm = np.zeros((32, 32), np.float32)
-    lib().orc_mm32_f64(_p(A), _p(B), _p(Cm))
+    (L or lib()).orc_mm32_f64(_p(A), _p(B), _p(Cm))
     return Cm
 
 
-def filterbank(r, H, F) -> np.ndarray:
+def filterbank(r, H, F, L=None) -> np.ndarray:
     r, H, F = (np.ascontiguousarray(v, np.float32) for v in (r, H, F))
     y = np.zeros(2048, np.float32)
-    lib().orc_filterbank(_p(r), _p(H), _p(F), _p(y))
+    (L or lib()).orc_filterbank(_p(r), _p(H), _p(F), _p(y))
     return y
 
 
-def beamformer(x, h, w) -> np.ndarray:
+def beamformer(x, h, w, L=None) -> np.ndarray:
     x, h, w = (np.ascontiguousarray(v, np.float32) for v in (x, h, w))
     out = np.zeros((4, 512), np.float32)
-    lib().orc_beamformer(_p(x), _p(h), _p(w), _p(out))
+    (L or lib()).orc_beamformer(_p(x), _p(h), _p(w), _p(out))
     return out
 
 
-def conv(img, krow, kcol) -> np.ndarray:
+def conv(img, krow, kcol, L=None) -> np.ndarray:
     img, krow, kcol = (np.ascontiguousarray(v, np.float32) for v in (img, krow, kcol))
     out = np.zeros((128, 128), np.float32)
-    lib().orc_conv(_p(img), _p(krow), _p(kcol), _p(out))
+    (L or lib()).orc_conv(_p(img), _p(krow), _p(kcol), _p(out))
     return out
 
 
-def dct(img, coef) -> np.ndarray:
+def dct(img, coef, L=None) -> np.ndarray:
     img, coef = (np.ascontiguousarray(v, np.float32) for v in (img, coef))
     out = np.zeros((128, 128), np.float32)
-    lib().orc_dct(_p(img), _p(coef), _p(out))
+    (L or lib()).orc_dct(_p(img), _p(coef), _p(out))
     return out
 
 

@@ -135,3 +135,110 @@ extern "C" int pagoda_pingpong(int device, int n, int64_t* rtt_ns)
     cudaFreeHost(h);
     return rc;
 }
+
+/* ------------------------------------------------------------------ pipe peaks (roofline denominators)
+ * the LDS and INT32 peaks are not published for B200; measure them.
+ * Each block times itself in SM cycles (clock64), so the result is per SM per
+ * clock, independent of the clock the GPU ran at; lookups/s follow at any clock.
+ *
+ * LDS: 8 independent chains per thread of v = load(table + v) over a
+ * lane-replicated table (word row * 32 + lane: every lane its own bank, one
+ * wavefront per warp instruction, the 3DES S-box pattern with resident tables);
+ * each entry holds the byte offset of the next lookup, so no ALU op sits
+ * between two lookups and only the shared-memory pipe is measured.
+ * INT32: 8 independent chains of lop3.b32 (the 3DES round's logic op). */
+constexpr int kPeakChains = 8;
+
+__global__ void __launch_bounds__(1024, 2) lds_peak_kernel(uint32_t iters, unsigned long long* cycles, uint32_t* sink)
+{
+    __shared__ uint32_t tab[64 * 32];
+    for (uint32_t i = threadIdx.x; i < 64 * 32; i += blockDim.x)
+        tab[i] = (((((i >> 5) * 37u + 11u) & 63u) << 7) | ((i & 31u) << 2));   /* next row's offset, same lane */
+    __syncthreads();
+    const uint32_t lane = threadIdx.x & 31u;
+    const char* t = reinterpret_cast<const char*>(tab);
+    uint32_t v[kPeakChains];
+#pragma unroll
+    for (int k = 0; k < kPeakChains; k++) v[k] = ((((threadIdx.x >> 5) + (uint32_t)k * 5u) & 63u) << 7) | (lane << 2);
+    __syncthreads();
+    const unsigned long long c0 = clock64();
+    for (uint32_t it = 0; it < iters; it++) {
+#pragma unroll
+        for (int k = 0; k < kPeakChains; k++) v[k] = *reinterpret_cast<const uint32_t*>(t + v[k]);
+    }
+    __syncthreads();
+    const unsigned long long c1 = clock64();
+    uint32_t s = 0;
+#pragma unroll
+    for (int k = 0; k < kPeakChains; k++) s ^= v[k];
+    if (s == 0x9E3779B9u) sink[0] = s;   /* keeps the chains alive */
+    if (threadIdx.x == 0) cycles[blockIdx.x] = c1 - c0;
+}
+
+__global__ void __launch_bounds__(1024, 2) int32_peak_kernel(uint32_t iters, uint32_t a, uint32_t b,
+                                                             unsigned long long* cycles, uint32_t* sink)
+{
+    uint32_t v[kPeakChains];
+#pragma unroll
+    for (int k = 0; k < kPeakChains; k++) v[k] = threadIdx.x * 7u + (uint32_t)k;
+    __syncthreads();
+    const unsigned long long c0 = clock64();
+    for (uint32_t it = 0; it < iters; it++) {
+#pragma unroll
+        for (int k = 0; k < kPeakChains; k++)
+            asm volatile("lop3.b32 %0, %0, %1, %2, 0x96;" : "+r"(v[k]) : "r"(a), "r"(b));
+    }
+    __syncthreads();
+    const unsigned long long c1 = clock64();
+    uint32_t s = 0;
+#pragma unroll
+    for (int k = 0; k < kPeakChains; k++) s ^= v[k];
+    if (s == 0x9E3779B9u) sink[0] = s;
+    if (threadIdx.x == 0) cycles[blockIdx.x] = c1 - c0;
+}
+
+/* which: 0 = LDS lookups, 1 = INT32 lop3.  Outputs: lanes (ops) per SM per clock, and
+ * ops/s over the whole kernel (CUDA events) at the clock it ran at. */
+extern "C" int pagoda_measure_pipe_peak(int device, int which, double* per_sm_clk, double* ops_per_s)
+{
+    if ((which != 0 && which != 1) || !per_sm_clk) return -EINVAL;
+    if (cudaSetDevice(device) != cudaSuccess) return -ENODEV;
+    cudaDeviceProp prop;
+    if (cudaGetDeviceProperties(&prop, device) != cudaSuccess) return -ENODEV;
+    const int blocks = prop.multiProcessorCount * 2, threads = 1024;
+    const uint32_t iters = which == 0 ? 2048u : 8192u;
+    unsigned long long* cyc = nullptr;
+    uint32_t* sink = nullptr;
+    if (cudaMalloc(&cyc, sizeof(unsigned long long) * blocks) != cudaSuccess) return -ENOMEM;
+    if (cudaMalloc(&sink, 64) != cudaSuccess) {
+        cudaFree(cyc);
+        return -ENOMEM;
+    }
+    cudaEvent_t e0, e1;
+    cudaEventCreate(&e0);
+    cudaEventCreate(&e1);
+    float ms = 0;
+    for (int rep = 0; rep < 2; rep++) {   /* the first launch warms up */
+        cudaEventRecord(e0);
+        if (which == 0) lds_peak_kernel<<<blocks, threads>>>(iters, cyc, sink);
+        else int32_peak_kernel<<<blocks, threads>>>(iters, 0x5A5A5A5Au, 0x3C3C3C3Cu, cyc, sink);
+        cudaEventRecord(e1);
+    }
+    int rc = cudaEventSynchronize(e1) == cudaSuccess ? 0 : -EIO;
+    cudaEventElapsedTime(&ms, e0, e1);
+    std::vector<unsigned long long> c((size_t)blocks);
+    if (!rc && cudaMemcpy(c.data(), cyc, sizeof(unsigned long long) * blocks, cudaMemcpyDeviceToHost) != cudaSuccess)
+        rc = -EIO;
+    if (!rc) {
+        const double per_block = (double)threads * iters * kPeakChains;   /* ops per block */
+        double rate = 0;   /* sum over blocks of ops per cycle; 2 co-resident blocks per SM */
+        for (int b = 0; b < blocks; b++) rate += per_block / (double)c[(size_t)b];
+        *per_sm_clk = rate / prop.multiProcessorCount;
+        if (ops_per_s) *ops_per_s = per_block * blocks / (ms * 1e-3);
+    }
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    cudaFree(cyc);
+    cudaFree(sink);
+    return rc;
+}

@@ -1,5 +1,5 @@
 /*
- * naive.cu — two host-side pieces that sit beside the MasterKernel:
+ * naive.cu — the two baselines that sit beside the MasterKernel:
  *
  * 1. The naive baseline: every task is its own kernel launch
  *    <<<n_tb, warps*32, shmem>>> of the SAME body (NativeEnv), issued
@@ -9,8 +9,7 @@
  * 2. The static-fusion baseline (NEXT-2): every task fused into
  *    ONE kernel launch, one thread block of a fixed thread count per task
  *    (the paper uses 256), the task's shape and args read from a device table.
- * 3. The multi-GPU pool: one context per GPU and a
- *    least-loaded picker (fewest in-flight warps, ties to the lowest index).
+ * (The multi-GPU pool lives in pool.cu.)
  */
 #include <cuda_runtime.h>
 #include <errno.h>
@@ -141,137 +140,4 @@ extern "C" int pagoda_fused_run(int device, int n, const int32_t* shapes, const 
     cudaStreamDestroy(st);
     if (d) cudaFree(d);
     return err == cudaSuccess ? 0 : -EIO;
-}
-
-/* ------------------------------------------------------------------ pool */
-extern "C" int64_t pagoda_inflight_warps(pagoda_ctx* c);
-
-/* pure picker: index of the smallest load, ties to the lowest index */
-extern "C" int pagoda_pick_least_loaded(const int64_t* loads, int n)
-{
-    if (!loads || n < 1) return -EINVAL;
-    int best = 0;
-    for (int i = 1; i < n; i++)
-        if (loads[i] < loads[best]) best = i;
-    return best;
-}
-
-struct pagoda_pool {
-    std::vector<pagoda_ctx*> ctx;
-    std::vector<int64_t> pending;   /* warps picked but not yet counted by the context */
-    std::mutex m;
-};
-
-extern "C" int pagoda_pool_init(int n_dev, const int* devices, const pagoda_config* cfg, pagoda_pool** out)
-{
-    if (!out || n_dev < 1 || !devices) return -EINVAL;
-    pagoda_pool* p = new pagoda_pool;
-    pagoda_config c;
-    if (cfg) c = *cfg;
-    else pagoda_config_default(&c);
-    for (int i = 0; i < n_dev; i++) {
-        c.device = devices[i];
-        pagoda_ctx* x = nullptr;
-        int rc = pagoda_init(&c, &x);
-        if (rc) {
-            for (auto* y : p->ctx) pagoda_shutdown(y);
-            delete p;
-            return rc;
-        }
-        p->ctx.push_back(x);
-    }
-    p->pending.assign(n_dev, 0);
-    *out = p;
-    return 0;
-}
-
-extern "C" int pagoda_pool_size(pagoda_pool* p) { return p ? (int)p->ctx.size() : -EINVAL; }
-
-extern "C" pagoda_ctx* pagoda_pool_ctx(pagoda_pool* p, int i)
-{
-    return (p && i >= 0 && i < (int)p->ctx.size()) ? p->ctx[i] : nullptr;
-}
-
-extern "C" int pagoda_pool_pick(pagoda_pool* p, int warps_hint)
-{
-    if (!p) return -EINVAL;
-    std::lock_guard<std::mutex> lk(p->m);
-    std::vector<int64_t> load(p->ctx.size());
-    for (size_t i = 0; i < p->ctx.size(); i++) load[i] = pagoda_inflight_warps(p->ctx[i]) + p->pending[i];
-    const int best = pagoda_pick_least_loaded(load.data(), (int)load.size());
-    p->pending[best] += warps_hint;
-    return best;
-}
-
-extern "C" pagoda_task_t pagoda_pool_spawn(pagoda_pool* p, int threads, int n_tb, int shmem_bytes, int sync_flag,
-                                           int func_id, const void* const* args_per_dev, size_t args_bytes,
-                                           int* index_out)
-{
-    if (!p) return -EINVAL;
-    const int w = ((threads + 31) / 32) * n_tb;
-    const int i = pagoda_pool_pick(p, w);
-    if (i < 0) return i;
-    pagoda_task_t id = pagoda_taskSpawn(p->ctx[i], threads, n_tb, shmem_bytes, sync_flag, func_id,
-                                        args_per_dev ? args_per_dev[i] : nullptr, args_bytes);
-    {
-        std::lock_guard<std::mutex> lk(p->m);
-        p->pending[i] -= w;   /* now counted by the context itself (or failed) */
-    }
-    if (index_out) *index_out = i;
-    return id;
-}
-
-/* Batched least-loaded spawning: runs of up to `chunk` tasks go
- * to the context with the fewest in-flight warps at the time of the pick (each
- * run one pagoda_taskSpawnShapes on that context, with that device's args). */
-extern "C" int64_t pagoda_pool_spawn_shapes(pagoda_pool* p, int n, const int32_t* shapes,
-                                            const void* const* args_base_per_dev, size_t args_stride,
-                                            size_t args_bytes, int chunk, pagoda_task_t* ids_out, int32_t* dev_out)
-{
-    if (!p || n < 0 || (n > 0 && !shapes) || chunk < 1) return -EINVAL;
-    for (int base = 0; base < n; base += chunk) {
-        const int m = std::min(chunk, n - base);
-        int64_t w = 0;
-        for (int i = 0; i < m; i++) {
-            const int32_t* s = shapes + 5 * (size_t)(base + i);
-            w += (int64_t)((s[0] + 31) / 32) * s[1];
-        }
-        const int d = pagoda_pool_pick(p, (int)std::min<int64_t>(w, INT32_MAX));
-        if (d < 0) return d;
-        const char* a = args_base_per_dev ? static_cast<const char*>(args_base_per_dev[d]) : nullptr;
-        const int64_t rc = pagoda_taskSpawnShapes(p->ctx[d], m, shapes + 5 * (size_t)base,
-                                                  a ? a + (size_t)base * args_stride : nullptr, args_stride, args_bytes,
-                                                  ids_out ? ids_out + base : nullptr);
-        {
-            std::lock_guard<std::mutex> lk(p->m);
-            p->pending[d] -= (int64_t)std::min<int64_t>(w, INT32_MAX);
-        }
-        if (rc < 0) return rc;
-        if (dev_out)
-            for (int i = 0; i < m; i++) dev_out[base + i] = d;
-    }
-    return n;
-}
-
-extern "C" int pagoda_pool_waitAll(pagoda_pool* p)
-{
-    if (!p) return -EINVAL;
-    int rc = 0;
-    for (auto* c : p->ctx) {
-        int r = pagoda_waitAll(c);
-        if (r && !rc) rc = r;
-    }
-    return rc;
-}
-
-extern "C" int pagoda_pool_shutdown(pagoda_pool* p)
-{
-    if (!p) return -EINVAL;
-    int rc = 0;
-    for (auto* c : p->ctx) {
-        int r = pagoda_shutdown(c);
-        if (r && !rc) rc = r;
-    }
-    delete p;
-    return rc;
 }

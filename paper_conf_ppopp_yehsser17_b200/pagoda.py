@@ -83,6 +83,7 @@ def lib() -> C.CDLL:
         L.pagoda_tdes_tables.argtypes = [P, P]
         L.pagoda_naive_run.argtypes = [I, I, P, P, SZ, SZ, I, C.POINTER(I64)]
         L.pagoda_pingpong.argtypes = [I, I, P]
+        L.pagoda_measure_pipe_peak.argtypes = [I, I, C.POINTER(C.c_double), C.POINTER(C.c_double)]
         L.pagoda_tdes_register.argtypes = [P, P]
         L.pagoda_dct_register.argtypes = [P, P]
         L.pagoda_fused_run.argtypes = [I, I, P, P, SZ, SZ, I, C.POINTER(I64), C.POINTER(C.c_float)]
@@ -97,6 +98,9 @@ def lib() -> C.CDLL:
         L.pagoda_pool_spawn_shapes.argtypes = [P, I, P, P, SZ, SZ, I, P, P]
         L.pagoda_pool_spawn_shapes.restype = I64
         L.pagoda_pool_shutdown.argtypes = [P]
+        L.pagoda_pool_numa_node.argtypes = [P, I]
+        L.pagoda_pool_stats.argtypes = [P, I, P, P, P]
+        L.pagoda_pool_may_claim.argtypes = [P, I, I, I64]
         L.pagoda_inflight_warps.argtypes = [P]
         L.pagoda_inflight_warps.restype = I64
         L.pagoda_pick_least_loaded.argtypes = [P, I]
@@ -142,6 +146,12 @@ def _ptr(a):
         assert a.flags["C_CONTIGUOUS"]
         return a.ctypes.data_as(C.c_void_p)
     return a
+
+
+def pool_may_claim(loads, me: int, slack: int) -> int:
+    """The pool spawners' claim rule (host-only): 1 if loads[me] <= min(loads) + slack."""
+    a = np.ascontiguousarray(loads, np.int64)
+    return lib().pagoda_pool_may_claim(_ptr(a), len(a), me, slack)
 
 
 def default_config(**kw) -> pagoda_config:
@@ -338,6 +348,15 @@ def pingpong(device: int, n: int = 2000) -> np.ndarray:
     return out
 
 
+def pipe_peak(device: int, which: str):
+    """Measured pipe peak: which = 'lds' (3DES-pattern lookups) or 'int32' (lop3).
+    Returns (ops per SM per clock, ops/s at the clock the kernel ran at)."""
+    per, rate = C.c_double(), C.c_double()
+    _check(lib().pagoda_measure_pipe_peak(device, {"lds": 0, "int32": 1}[which], C.byref(per), C.byref(rate)),
+           "pagoda_measure_pipe_peak")
+    return per.value, rate.value
+
+
 def pick_least_loaded(loads) -> int:
     a = np.ascontiguousarray(loads, np.int64)
     return lib().pagoda_pick_least_loaded(_ptr(a), len(a))
@@ -369,8 +388,9 @@ class Pool:
                                       C.byref(idx))
         return tid, idx.value
 
-    def spawn_shapes(self, shapes: np.ndarray, args_per_dev, chunk: int = 64):
-        """args_per_dev[i]: uint8 [n, 40] args valid on device i.  Returns (ids, dev) per task."""
+    def spawn_shapes(self, shapes: np.ndarray, args_per_dev, chunk: int = 256):
+        """args_per_dev[i]: uint8 [n, 40] args valid on member i's device.  Every member's own
+        spawner thread claims runs of `chunk` tasks least-loaded-first.  Returns (ids, member) per task."""
         shapes = np.ascontiguousarray(shapes, np.int32)
         args_per_dev = [np.ascontiguousarray(a, np.uint8) for a in args_per_dev]
         n = len(shapes)
@@ -382,6 +402,48 @@ class Pool:
 
     def ctx(self, i: int):
         return lib().pagoda_pool_ctx(self.h, i)
+
+    def size(self) -> int:
+        return lib().pagoda_pool_size(self.h)
+
+    def numa_node(self, i: int) -> int:
+        return lib().pagoda_pool_numa_node(self.h, i)
+
+    def stats(self, i: int):
+        """(tasks, spawn_ns, hold_ns) of member i in the last batched spawn."""
+        t, s, h = C.c_int64(), C.c_int64(), C.c_int64()
+        _check(lib().pagoda_pool_stats(self.h, i, C.byref(t), C.byref(s), C.byref(h)), "pagoda_pool_stats")
+        return t.value, s.value, h.value
+
+    def start(self) -> int:
+        """pagoda_start on every member (a pool made with NO_START)."""
+        for i in range(self.size()):
+            rc = lib().pagoda_start(self.ctx(i))
+            if rc:
+                return rc
+        return 0
+
+    def stop(self) -> int:
+        rc = 0
+        for i in range(self.size()):
+            r = lib().pagoda_stop(self.ctx(i))
+            rc = rc or r
+        return rc
+
+    def session_ms(self, i: int) -> float:
+        ms = C.c_float()
+        _check(lib().pagoda_session_ms(self.ctx(i), C.byref(ms)), "pagoda_session_ms")
+        return ms.value
+
+    def dct_register(self, dev_coef_per_member):
+        """dev_coef_per_member[i]: device pointer (int) of member i's coefficient matrix."""
+        for i, t in enumerate(dev_coef_per_member):
+            _check(lib().pagoda_dct_register(self.ctx(i), C.c_void_p(int(t))), "pagoda_dct_register")
+
+    def tdes_register(self, dev_tables_per_member):
+        """dev_tables_per_member[i]: device pointer (int) of member i's 3DES tables."""
+        for i, t in enumerate(dev_tables_per_member):
+            _check(lib().pagoda_tdes_register(self.ctx(i), C.c_void_p(int(t))), "pagoda_tdes_register")
 
     def waitAll(self) -> int:
         return lib().pagoda_pool_waitAll(self.h)

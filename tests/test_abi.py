@@ -69,6 +69,18 @@ def test_picker_rule(L):
     assert L.pagoda_pick_least_loaded(None, 0) == -errno.EINVAL
 
 
+def test_pool_claim_rule(L):
+    """A pool member claims the next run of tasks only while it is within `slack` warps of
+    the least-loaded member (SURVEY §8(e) least-loaded-first)."""
+    assert PG.pool_may_claim([10, 3, 7], 1, 0) == 1           # the least loaded always may
+    assert PG.pool_may_claim([10, 3, 7], 2, 0) == 0
+    assert PG.pool_may_claim([10, 3, 7], 2, 4) == 1           # within slack
+    assert PG.pool_may_claim([5, 5], 0, 0) == 1 and PG.pool_may_claim([5, 5], 1, 0) == 1   # ties: both
+    assert PG.pool_may_claim([5], 0, 0) == 1
+    assert L.pagoda_pool_may_claim(None, 0, 0, 0) == -errno.EINVAL
+    assert PG.pool_may_claim([1, 2], 2, 0) == -errno.EINVAL
+
+
 def test_args_layouts_fit_the_entry():
     for f, d in T.ARGS.items():
         assert d.itemsize <= 40

@@ -94,3 +94,53 @@ def test_c5_strong_scaling_shards_two_ranks():
     from paper_conf_ppopp_yehsser17_b200 import workloads as W
     kinds = I.c5_schedule(10000)[0]
     assert res[1][4] == W.KIND_FUNC[I.C5_KINDS[kinds[5000]]]          # rank 1 starts at global task 5000
+
+
+def _claims_worker(rank, world, port, q):
+    """bench.SharedClaims: two ranks claim runs of one step's tasks from the shared counter
+    under the least-loaded rule (loads published by each rank); two steps back to back."""
+    os.environ.update({"RANK": str(rank), "LOCAL_RANK": str(rank), "WORLD_SIZE": str(world),
+                       "MASTER_ADDR": "127.0.0.1", "MASTER_PORT": str(port)})
+    sys.path.insert(0, ROOT)
+    import bench
+    from paper_conf_ppopp_yehsser17_b200 import pagoda as PG
+    d = bench.Dist()
+    cl = bench.SharedClaims(d, f"test{port}")
+    got = []
+    n, chunk = 10000, 128
+    for step in range(2):
+        d.barrier()
+        cl.reset(step)
+        mine, load = [], 0
+        while True:
+            cl.publish(load)
+            if PG.pool_may_claim(cl.loads(), rank, 4 * chunk) != 1:
+                load = max(0, load - chunk)   # "completions" drain this rank's load
+                continue
+            c = cl.claim(step, chunk, n)
+            if c is None:
+                break
+            mine.append(c)
+            load += chunk if rank == 0 else chunk // 2   # rank 1 drains twice as fast: it should claim more
+            load = max(0, load - chunk // 2)
+        got.append(mine)
+    d.barrier()
+    cl.close()
+    q.put((rank, got))
+    import torch.distributed as dist
+    dist.destroy_process_group()
+
+
+def test_shared_claims_two_ranks_cover_each_step_once():
+    world, port = 2, _free_port()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_claims_worker, args=(r, world, port, q)) for r in range(world)]
+    [p.start() for p in procs]
+    [p.join(timeout=300) for p in procs]
+    assert all(p.exitcode == 0 for p in procs)
+    res = dict(q.get(timeout=5) for _ in range(world))
+    for step in range(2):
+        runs = sorted(res[0][step] + res[1][step])
+        assert runs == list(range(0, 10000, 128))          # every run of the step claimed exactly once
+        assert res[0][step] and res[1][step]               # both ranks took work

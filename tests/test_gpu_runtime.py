@@ -443,23 +443,34 @@ def test_four_mtbs_per_sm():
         assert np.array_equal(out[k], oracle.mm32(w.host["A"][k], w.host["B"][k])), k
 
 
-def test_pool_least_loaded_spawner():
-    """The in-process multi-GPU pool on the device(s) present:
-    single spawns and batched least-loaded spawns land, complete and compute
-    what the oracle does (config 5 tasks)."""
-    import oracle
+def _pool_members():
+    """Pool members: every GPU present; on a one-GPU machine two half-GPU members (2 x 74 SMs:
+    two co-resident MasterKernels, SURVEY §4 layer 6)."""
     import torch
+    n = torch.cuda.device_count()
+    return (list(range(n)), {}) if n > 1 else ([0, 0], {"num_sms": 74})
+
+
+def test_pool_least_loaded_spawner():
+    """The in-process multi-GPU pool: one spawner thread per member (NUMA-bound),
+    runs of tasks claimed least-loaded-first.  Single spawns and batched spawns land on every
+    member, complete, and compute what the oracle does (config 5 tasks)."""
+    import oracle
     from paper_conf_ppopp_yehsser17_b200 import workloads as W
     from paper_conf_ppopp_yehsser17_b200.pagoda import Pool
-    n_dev = torch.cuda.device_count()
-    ws = [W.c5(3000, pool_size=32, device=f"cuda:{i}", fill=0xAB) for i in range(n_dev)]
-    pool = Pool(range(n_dev))
+    devs, cfg = _pool_members()
+    n_dev = len(devs)
+    ws = [W.c5(3000, pool_size=32, device=f"cuda:{d}", fill=0xAB) for d in devs]
+    pool = Pool(devs, **cfg)
+    assert pool.size() == n_dev
     assert pool.pick(4) in range(n_dev)
     tid, idx = pool.spawn(128, 1, 0, False, T.NOP, [b""] * n_dev)
     assert tid >= 0 and idx in range(n_dev)
-    ids, dev = pool.spawn_shapes(ws[0].shapes, [w.args for w in ws])
+    ids, dev = pool.spawn_shapes(ws[0].shapes, [w.args for w in ws], chunk=64)
     assert pool.waitAll() == 0
-    assert (ids >= 0).all() and set(np.unique(dev)) <= set(range(n_dev))
+    assert (ids >= 0).all() and set(np.unique(dev)) == set(range(n_dev))   # every member took runs
+    st = [pool.stats(i) for i in range(n_dev)]
+    assert sum(s[0] for s in st) == 3000 and all(s[1] > 0 for s in st)
     assert pool.shutdown() == 0
     for k in range(0, 3000, 97):
         w = ws[int(dev[k])]
@@ -470,6 +481,39 @@ def test_pool_least_loaded_spawner():
                "tdes": lambda pk: oracle.tdes_ecb(pk, __import__("paper_conf_ppopp_yehsser17_b200.inputs",
                                                                   fromlist=["x"]).TDES_KEYS)}[kind](*args)
         assert np.array_equal(w.task_output(k), ref), (kind, k)
+
+
+def test_pool_two_members_c5_parity_every_task():
+    """Config 5's mix through the pool's least-loaded spawners on two members (two GPUs, or
+    two 74-SM MasterKernels on one): every task runs once, on exactly one member, with that
+    member's inputs, and matches the oracle (all 4000 tasks checked)."""
+    import oracle
+    from paper_conf_ppopp_yehsser17_b200 import inputs as I
+    from paper_conf_ppopp_yehsser17_b200 import workloads as W
+    from paper_conf_ppopp_yehsser17_b200.pagoda import NO_START, Pool
+    devs, cfg = _pool_members()
+    devs = devs[:2]
+    n = 4000
+    ws = [W.c5(n, pool_size=64, device=f"cuda:{d}", fill=0xCD) for d in devs]
+    pool = Pool(devs, flags=NO_START, **cfg)
+    pool.dct_register([w.dct_coef for w in ws])     # registered before any member starts
+    assert pool.start() == 0
+    ids, dev = pool.spawn_shapes(ws[0].shapes, [w.args for w in ws], chunk=32)
+    assert pool.waitAll() == 0 and pool.stop() == 0
+    assert pool.shutdown() == 0
+    assert np.bincount(dev, minlength=2).min() > 0
+    ref = {"mm": oracle.mm32, "fb": oracle.filterbank, "bf": oracle.beamformer, "conv": oracle.conv,
+           "dct": oracle.dct, "mb": lambda *a: oracle.mandelbrot_tile(*a),
+           "tdes": lambda pk: oracle.tdes_ecb(pk, I.TDES_KEYS)}
+    cache = {}
+    for k in range(n):
+        mine, other = ws[int(dev[k])], ws[1 - int(dev[k])]
+        kind = mine.kind(k)
+        key = (kind, int(mine.in_idx[k]))
+        if key not in cache:
+            cache[key] = ref[kind](*mine.pool.oracle_inputs(kind, int(mine.in_idx[k])))
+        assert np.array_equal(mine.task_output(k), cache[key]), (kind, k)
+        assert not np.array_equal(other.task_output(k), cache[key]), (kind, k)   # ran on one member only
 
 
 # ---------------------------------------------------------------- device errors and the paper-named device API

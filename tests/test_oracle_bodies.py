@@ -468,3 +468,27 @@ def test_mb_golden_file_regenerates():
         assert f.read() == gen.render(counts)
     fused = gen.iteration_counts(fused=True)
     assert int(fused.sum(dtype=np.int64)) != int(counts.sum(dtype=np.int64))
+
+
+# ------------------------------------------------------------------ the timed oracle build
+def test_fast_build_outputs_equal_parity_build():
+    """bench.py times the oracle built -O3 -march=native -ffp-contract=off; with
+    contraction still off its outputs must equal the parity build's, body by body."""
+    import oracle as O
+    from paper_conf_ppopp_yehsser17_b200 import inputs as I
+    F = O.lib(fast=True)
+    assert np.array_equal(O.mandelbrot_tile(24, 16), O.mandelbrot_tile(24, 16, L=F))
+    pk = I.tdes_packets(2, 4096, 0)
+    assert np.array_equal(O.tdes_ecb(pk[1], I.TDES_KEYS), O.tdes_ecb(pk[1], I.TDES_KEYS, L=F))
+    A, B = I.mm_inputs(2)
+    assert np.array_equal(O.mm32(A[1], B[1]), O.mm32(A[1], B[1], L=F))
+    A, B = I.mm64_inputs(1)
+    assert np.array_equal(O.mm64(A[0], B[0]), O.mm64(A[0], B[0], L=F))
+    r, H, Fi = I.fb_inputs(1)
+    assert np.array_equal(O.filterbank(r[0], H[0], Fi[0]), O.filterbank(r[0], H[0], Fi[0], L=F))
+    x, h, w = I.bf_inputs(1)
+    assert np.array_equal(O.beamformer(x[0], h[0], w[0]), O.beamformer(x[0], h[0], w[0], L=F))
+    img, kr, kc = I.conv_inputs(1)
+    assert np.array_equal(O.conv(img[0], kr[0], kc[0]), O.conv(img[0], kr[0], kc[0], L=F))
+    im = I.dct_inputs(1)
+    assert np.array_equal(O.dct(im[0], I.dct_coef()), O.dct(im[0], I.dct_coef(), L=F))
