@@ -19,7 +19,7 @@ def test_ctx_kwargs_match_bench_context():
             no_resident = False
             mtbs = 0
             arena_kb = 0
-        cfg = bench.ctx_config(A, PG)
+        cfg = bench.ctx_config(A, PG, w)
         kw = presets.ctx_kwargs(w, PG.NO_START)
         assert cfg == kw, w
 
