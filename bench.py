@@ -977,6 +977,24 @@ def e2e_run(p, w, steps, torch, a):
             tl["d2h"].append((time.perf_counter_ns() - t0) / 1e3)
         done.set()
 
+    # the PCIe bound of one step: every input H2D alone, every output D2H alone (CUDA events on
+    # the copy streams, no MasterKernel resident); both directions overlap in the e2e run
+    def copy_ms(stream, pairs):
+        if not pairs:
+            return 0.0
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        with torch.cuda.stream(stream):
+            e0.record(stream)
+            for dst, src in pairs:
+                dst.copy_(src, non_blocking=True)
+            e1.record(stream)
+        e1.synchronize()
+        return e0.elapsed_time(e1)
+    in_pairs = [(dt[:w.n * per], hi_t) for (dt, _, per), hi_t in zip(ins, host_in)]
+    out_pairs = [(ho, dt[:w.n * per]) for (dt, per), ho in zip(outs, host_out)]
+    copy_ms(s_in, in_pairs)   # warm-up
+    h2d_ms, d2h_ms = copy_ms(s_in, in_pairs), copy_ms(s_out, out_pairs)
+    bound = w.n / (max(h2d_ms, d2h_ms) * 1e-3)
     times = []
     assert p.start() == 0
     for it in range(steps + 1):
@@ -1031,6 +1049,10 @@ def e2e_run(p, w, steps, torch, a):
             "d2h_bytes_per_step": int(d2h), "ms_per_step": 1e3 * tot / steps,
             "pcie_gbs_h2d": h2d / (tot / steps) / 1e9, "pcie_gbs_d2h": d2h / (tot / steps) / 1e9,
             "chunks": chunks, "ahead": ahead,
+            "pcie_bound": {"h2d_alone_ms": h2d_ms, "d2h_alone_ms": d2h_ms, "tasks_per_s": bound,
+                           "e2e_frac": (w.n * steps / tot) / bound,
+                           "how": "all of a step's inputs H2D alone / outputs D2H alone (CUDA events); the e2e "
+                                  "run overlaps both directions, so the slower one bounds it"},
             "how": f"pinned host inputs -> H2D ({chunks} chunks, copy stream, {ahead} ahead) -> taskSpawn per task; a "
                    "drain thread waitBelow()s each chunk and queues its D2H on a second copy stream (both directions "
                    "overlap); outputs of the first tasks checked against the oracle in the cpu_baseline leg",

@@ -261,6 +261,24 @@ __device__ __forceinline__ uint32_t lds_at(uint32_t addr)
 
 enum { kTdesResident = 0, kTdesShared = 1, kTdesGlobal = 2 };
 
+/* The 8 table words of a round have disjoint bits (P maps each S-box's 4 output bits to its own 4
+ * positions), so their XOR equals their SUM.  A sum can run on the FMA pipe as IMAD d = a * one + b
+ * (one = 1 from the constant bank, opaque to ptxas, so it is not folded into an IADD3 on the ALU
+ * pipe).  A resident round had 16 ALU instructions (2 SHF, 2 LOP3, 8 PRMT, 4 LOP3 for the XORs with
+ * l) per 8 shared-memory lookups: ALU and LDS both at 8 SM-clocks per warp-round.  Summing the words
+ * in pairs on the FMA pipe (4 IMAD) leaves 2 XOR LOP3s: 14 ALU (7 clocks), 26 issued (6.5 clocks),
+ * so the lookups alone bound the round. */
+#ifndef PAGODA_TDES_FMA_SUM
+#define PAGODA_TDES_FMA_SUM 1
+#endif
+static __constant__ uint32_t c_one = 1u;
+__device__ __forceinline__ uint32_t sum_fma_pipe(uint32_t a, uint32_t b)
+{
+    uint32_t d;
+    asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(c_one), "r"(b));
+    return d;
+}
+
 /* f(R) for table placement kMode.
  * resident: the MTB-resident table at window address kResidentTdesAddr holds
  * SP[j][v] for lane l at word 4096 p + 64 v + 32 h + l, where byte p of x
@@ -276,10 +294,17 @@ __device__ __forceinline__ uint32_t tdes_f(uint32_t r, uint32_t kx, uint32_t ky,
         const uint32_t y = (__funnelshift_l(r, r, 1) ^ ky) & 0x3F3F3F3Fu;
         const uint32_t t1 = tb | 128u;
         constexpr uint32_t A = kResidentTdesAddr;
-        return lds_at<A + 0 * 16384>(__byte_perm(x, tb, 0x7604)) ^ lds_at<A + 1 * 16384>(__byte_perm(x, tb, 0x7614)) ^
-               lds_at<A + 2 * 16384>(__byte_perm(x, tb, 0x7624)) ^ lds_at<A + 3 * 16384>(__byte_perm(x, tb, 0x7634)) ^
-               lds_at<A + 0 * 16384>(__byte_perm(y, t1, 0x7604)) ^ lds_at<A + 1 * 16384>(__byte_perm(y, t1, 0x7614)) ^
-               lds_at<A + 2 * 16384>(__byte_perm(y, t1, 0x7624)) ^ lds_at<A + 3 * 16384>(__byte_perm(y, t1, 0x7634));
+        const uint32_t s0 = lds_at<A + 0 * 16384>(__byte_perm(x, tb, 0x7604));
+        const uint32_t s1 = lds_at<A + 1 * 16384>(__byte_perm(x, tb, 0x7614));
+        const uint32_t s2 = lds_at<A + 2 * 16384>(__byte_perm(x, tb, 0x7624));
+        const uint32_t s3 = lds_at<A + 3 * 16384>(__byte_perm(x, tb, 0x7634));
+        const uint32_t s4 = lds_at<A + 0 * 16384>(__byte_perm(y, t1, 0x7604));
+        const uint32_t s5 = lds_at<A + 1 * 16384>(__byte_perm(y, t1, 0x7614));
+        const uint32_t s6 = lds_at<A + 2 * 16384>(__byte_perm(y, t1, 0x7624));
+        const uint32_t s7 = lds_at<A + 3 * 16384>(__byte_perm(y, t1, 0x7634));
+        if (PAGODA_TDES_FMA_SUM)   /* 4 IMAD pair sums + the caller's 3-input XORs (with l): 2 LOP3 */
+            return sum_fma_pipe(s0, s1) ^ sum_fma_pipe(s2, s3) ^ sum_fma_pipe(s4, s5) ^ sum_fma_pipe(s6, s7);
+        return s0 ^ s1 ^ s2 ^ s3 ^ s4 ^ s5 ^ s6 ^ s7;
     }
     const uint32_t x = __funnelshift_l(r, r, 5) ^ kx;
     const uint32_t y = __funnelshift_l(r, r, 1) ^ ky;

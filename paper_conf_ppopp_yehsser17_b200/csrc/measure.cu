@@ -12,6 +12,7 @@
 #include <time.h>
 #include <immintrin.h>
 
+#include <algorithm>
 #include <atomic>
 #include <thread>
 #include <vector>
@@ -138,8 +139,10 @@ extern "C" int pagoda_pingpong(int device, int n, int64_t* rtt_ns)
 
 /* ------------------------------------------------------------------ pipe peaks (roofline denominators)
  * the LDS and INT32 peaks are not published for B200; measure them.
- * Each block times itself in SM cycles (clock64), so the result is per SM per
- * clock, independent of the clock the GPU ran at; lookups/s follow at any clock.
+ * Each block stamps its start and end in SM cycles (clock64, one counter per SM)
+ * with its %smid; per SM the window runs from the first start to the last end
+ * of its co-resident blocks, so the result is ops per SM per clock whatever
+ * clock the GPU ran at (lookups/s then follow at any clock).
  *
  * LDS: 8 independent chains per thread of v = load(table + v) over a
  * lane-replicated table (word row * 32 + lane: every lane its own bank, one
@@ -148,6 +151,15 @@ extern "C" int pagoda_pingpong(int device, int n, int64_t* rtt_ns)
  * between two lookups and only the shared-memory pipe is measured.
  * INT32: 8 independent chains of lop3.b32 (the 3DES round's logic op). */
 constexpr int kPeakChains = 8;
+
+__device__ __forceinline__ void peak_stamp(unsigned long long* rec, unsigned long long c0, unsigned long long c1)
+{   /* rec[3 b .. 3 b + 2] = smid, start, end */
+    uint32_t smid;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+    rec[3 * blockIdx.x] = smid;
+    rec[3 * blockIdx.x + 1] = c0;
+    rec[3 * blockIdx.x + 2] = c1;
+}
 
 __global__ void __launch_bounds__(1024, 2) lds_peak_kernel(uint32_t iters, unsigned long long* cycles, uint32_t* sink)
 {
@@ -172,7 +184,7 @@ __global__ void __launch_bounds__(1024, 2) lds_peak_kernel(uint32_t iters, unsig
 #pragma unroll
     for (int k = 0; k < kPeakChains; k++) s ^= v[k];
     if (s == 0x9E3779B9u) sink[0] = s;   /* keeps the chains alive */
-    if (threadIdx.x == 0) cycles[blockIdx.x] = c1 - c0;
+    if (threadIdx.x == 0) peak_stamp(cycles, c0, c1);
 }
 
 __global__ void __launch_bounds__(1024, 2) int32_peak_kernel(uint32_t iters, uint32_t a, uint32_t b,
@@ -194,7 +206,7 @@ __global__ void __launch_bounds__(1024, 2) int32_peak_kernel(uint32_t iters, uin
 #pragma unroll
     for (int k = 0; k < kPeakChains; k++) s ^= v[k];
     if (s == 0x9E3779B9u) sink[0] = s;
-    if (threadIdx.x == 0) cycles[blockIdx.x] = c1 - c0;
+    if (threadIdx.x == 0) peak_stamp(cycles, c0, c1);
 }
 
 /* which: 0 = LDS lookups, 1 = INT32 lop3.  Outputs: lanes (ops) per SM per clock, and
@@ -209,7 +221,7 @@ extern "C" int pagoda_measure_pipe_peak(int device, int which, double* per_sm_cl
     const uint32_t iters = which == 0 ? 2048u : 8192u;
     unsigned long long* cyc = nullptr;
     uint32_t* sink = nullptr;
-    if (cudaMalloc(&cyc, sizeof(unsigned long long) * blocks) != cudaSuccess) return -ENOMEM;
+    if (cudaMalloc(&cyc, sizeof(unsigned long long) * 3 * blocks) != cudaSuccess) return -ENOMEM;
     if (cudaMalloc(&sink, 64) != cudaSuccess) {
         cudaFree(cyc);
         return -ENOMEM;
@@ -226,14 +238,29 @@ extern "C" int pagoda_measure_pipe_peak(int device, int which, double* per_sm_cl
     }
     int rc = cudaEventSynchronize(e1) == cudaSuccess ? 0 : -EIO;
     cudaEventElapsedTime(&ms, e0, e1);
-    std::vector<unsigned long long> c((size_t)blocks);
-    if (!rc && cudaMemcpy(c.data(), cyc, sizeof(unsigned long long) * blocks, cudaMemcpyDeviceToHost) != cudaSuccess)
+    std::vector<unsigned long long> c((size_t)3 * blocks);
+    if (!rc && cudaMemcpy(c.data(), cyc, sizeof(unsigned long long) * 3 * blocks, cudaMemcpyDeviceToHost) != cudaSuccess)
         rc = -EIO;
     if (!rc) {
         const double per_block = (double)threads * iters * kPeakChains;   /* ops per block */
-        double rate = 0;   /* sum over blocks of ops per cycle; 2 co-resident blocks per SM */
-        for (int b = 0; b < blocks; b++) rate += per_block / (double)c[(size_t)b];
-        *per_sm_clk = rate / prop.multiProcessorCount;
+        const int nsm = prop.multiProcessorCount;
+        std::vector<unsigned long long> lo((size_t)nsm, ~0ull), hi((size_t)nsm, 0);
+        std::vector<int> cnt((size_t)nsm, 0);
+        for (int b = 0; b < blocks; b++) {
+            const unsigned long long sm = c[3 * (size_t)b];
+            if (sm >= (unsigned long long)nsm) continue;
+            lo[sm] = std::min(lo[sm], c[3 * (size_t)b + 1]);
+            hi[sm] = std::max(hi[sm], c[3 * (size_t)b + 2]);
+            cnt[sm]++;
+        }
+        double rate = 0;   /* per SM: its blocks' ops over its busy window; the mean over SMs */
+        int used = 0;
+        for (int sm = 0; sm < nsm; sm++)
+            if (cnt[sm] && hi[sm] > lo[sm]) {
+                rate += per_block * cnt[sm] / (double)(hi[sm] - lo[sm]);
+                used++;
+            }
+        *per_sm_clk = used ? rate / used : 0.0;
         if (ops_per_s) *ops_per_s = per_block * blocks / (ms * 1e-3);
     }
     cudaEventDestroy(e0);

@@ -5,6 +5,9 @@ context; per stage the median / p90 duration (us) and the mean number of tasks i
 that stage (Little's law: stage time x throughput).  One JSON line per workload.
 
     python scripts/probe_life.py [nop mm tdes mix mb]
+    PRODUCERS=2 python scripts/probe_life.py mm     # host spawner threads (default: the preset's)
+    DRAIN=1 python scripts/probe_life.py mm         # spawn while stopped, then one self-draining session
+                                                    # (the device alone: no host spawn in the timed span)
 """
 import json
 import os
@@ -29,23 +32,30 @@ def main():
             no_resident = False
             mtbs = 0
             arena_kb = 0
-        cfg = bench.ctx_config(A, PG)
+        cfg = bench.ctx_config(A, PG, name)
         cfg["flags"] |= PG.LIFECYCLE
-        w = bench.make_workload(name, bench.use_resident(A), bench.Dist())
+        w = bench.make_workload(name, bench.use_resident(A, name), bench.Dist())
         with PG.Pagoda(**cfg) as p:
             n_mtb = p.info().n_mtb
-            if bench.use_resident(A) and w.tdes_tables:
+            if bench.use_resident(A, name) and w.tdes_tables:
                 p.tdes_register(w.tdes_tables)
+            producers = int(os.environ.get("PRODUCERS", "0")) or bench.PRESETS[name].get("producers", 1)
+            drain = os.environ.get("DRAIN") == "1"
             for stamped in (False, True):
-                assert p.start() == 0
-                ids = p.spawn_shapes(w.shapes, w.args, ids=True)
+                if drain:
+                    ids = p.spawn_shapes(w.shapes[:65536], w.args[:65536], ids=True, producers=producers)
+                    assert p.start_drain() == 0
+                else:
+                    assert p.start() == 0
+                    ids = p.spawn_shapes(w.shapes, w.args, ids=True, producers=producers)
                 assert p.stop() == 0
             ms = p.session_ms()
-            L = p.lifecycle(int(ids[0]), w.n).astype(np.int64)
+            L = p.lifecycle(int(ids.min()), len(ids)).astype(np.int64)
         ok = (L > 0).all(axis=1)
         L = L[ok]
-        out = {"workload": name, "tasks": w.n, "stamped": int(ok.sum()), "session_ms": ms,
-               "tasks_per_s": w.n / ms * 1e3, "mtbs": n_mtb}
+        n = len(ids)
+        out = {"workload": name, "tasks": n, "stamped": int(ok.sum()), "session_ms": ms,
+               "tasks_per_s": n / ms * 1e3, "mtbs": n_mtb, "producers": producers, "drain": drain}
         span = (L[:, 7].max() - L[:, 0].min()) * 1e-9
         rate = len(L) / span
         st = {}
