@@ -732,6 +732,11 @@ __device__ void body_bf(const Env& e, const pagoda_bf_args& a)
  * tmp[y+d][x] kcol[8-d], zero outside, d ascending.  TB j produces output rows
  * [r0, r1) and first computes the tmp rows [r0-8, r1+8) they need into
  * scratch + 16384*j (same row indexing as the full image). */
+__device__ __forceinline__ void discard_l2(const void* line128)
+{
+    asm volatile("discard.global.L2 [%0], 128;" ::"l"(line128) : "memory");
+}
+
 template <class Env>
 __device__ void body_conv(const Env& e, const pagoda_conv_args& a)
 {
@@ -788,6 +793,12 @@ __device__ void body_conv(const Env& e, const pagoda_conv_args& a)
         if (y0 + 2 < r1) o[256] = c2;
         if (y0 + 3 < r1) o[384] = c3;
     }
+    /* The row-pass rows are dead now.  Written moments ago, they sit dirty in L2; without this
+     * they would be written back to HBM on eviction (64 KiB per task, half again the task's
+     * algorithmic traffic).  discard.global.L2 drops the lines without a write-back, once every
+     * thread of the TB has finished reading them (the barrier). */
+    e.syncBlock();
+    for (int i = bt; i < (t1 - t0) * 4; i += n) discard_l2(tmp + t0 * 128 + i * 32);
 }
 
 /* ------------------------------------------------------------- DCT

@@ -54,6 +54,10 @@
 #ifndef PAGODA_CLAIM_SMALL
 #define PAGODA_CLAIM_SMALL 1  /* tickets per claim while the backlog is below what all MTBs could take */
 #endif
+#ifndef PAGODA_HOLDER_POSTS
+#define PAGODA_HOLDER_POSTS 0 /* the scheduler token holder posts completion records (batched per round);
+                                 the last warp of a task only marks it pending and frees itself */
+#endif
 
 namespace pagoda {
 
@@ -480,7 +484,7 @@ __device__ __forceinline__ void run_task(MtbShared& S, char* smem_base, const Mk
     }
     pf_add(S, kPfFence, tp, true);
     tp = pf_now();
-    if (__shfl_sync(0xffffffffu, last, 0)) post_completions(S, p);
+    if (!PAGODA_HOLDER_POSTS && __shfl_sync(0xffffffffu, last, 0)) post_completions(S, p);
     pf_add(S, kPfPost, tp, true);
     if (lane == 0) {
         __threadfence_block();   /* TB / task frees are visible before the warp frees itself */
@@ -1245,6 +1249,15 @@ __device__ bool sched_round(MtbShared& S, Sched& st, const MkParams& p, int mtb,
     uint64_t t0 = pf_now();
     bool progress = sched_fold(S, st, p, mtb);
     pf_add(S, kPfFold, t0, true);
+    /* completion records of the tasks whose last warp finished (a warp marks comp_pending before
+     * it frees itself, so every task of a folded warp is in it): one fence and one queue
+     * reservation for the whole batch, off the executors' path */
+    if (PAGODA_HOLDER_POSTS && *(volatile uint32_t*)&S.comp_pending) {
+        t0 = pf_now();
+        post_completions(S, p);
+        pf_add(S, kPfPost, t0, true);
+        progress = true;
+    }
 #if PAGODA_FUSED_CLAIM
     t0 = pf_now();
     {
@@ -1287,7 +1300,7 @@ __device__ bool sched_round(MtbShared& S, Sched& st, const MkParams& p, int mtb,
     exit = false;
     sc_add(S, kScRounds, 1);
     if (progress) sc_add(S, kScProgress, 1);
-    if (!progress && st.free_w == st.exec_mask && st.ph == st.pl) {
+    if (!progress && st.free_w == st.exec_mask && st.ph == st.pl && *(volatile uint32_t*)&S.comp_pending == 0u) {
         uint32_t stop = 0;
         if (lane == 0) stop = ld_acquire_gpu32(&p.dctl->stop);
         stop = __shfl_sync(0xffffffffu, stop, 0);
