@@ -89,6 +89,8 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--quick", action="store_true", help="skip everything but the timed steps (for ncu)")
     ap.add_argument("--mtbs", type=int, default=0, help="MTBs per SM (default: the workload preset)")
+    ap.add_argument("--exec-warps", type=int, default=0, help="worker warps per MTB (default: the preset's, else all)")
+    ap.add_argument("--spread", type=int, default=-1, help="spread-first claims on (1) / off (0) (default: preset)")
     ap.add_argument("--arena-kb", type=int, default=0, help="task arena per MTB in KiB (default: preset)")
     ap.add_argument("--producers", type=int, default=0,
                     help="host spawner threads per step (pagoda_taskSpawnShapesMT; default: preset)")
@@ -416,10 +418,14 @@ def ctx_config(a, PG, name):
     """The workload's preset context; --mtbs / --arena-kb override the headline workload only."""
     pr = PRESETS[name]
     mine = name == a.workload
+    spread = (a.spread == 1) if mine and getattr(a, "spread", -1) >= 0 else bool(pr.get("spread"))
     cfg = {"flags": PG.NO_START | (PG.RESIDENT_TDES if use_resident(a, name) else 0) |
-           (PG.SPREAD if pr.get("spread") else 0),
+           (PG.SPREAD if spread else 0),
            "mtbs_per_sm": (a.mtbs if mine and a.mtbs else pr["mtbs_per_sm"]),
            "arena_bytes": (a.arena_kb * 1024) if mine and a.arena_kb else pr["arena_bytes"]}
+    ew = a.exec_warps if mine and getattr(a, "exec_warps", 0) else pr.get("exec_warps", 0)
+    if ew:
+        cfg["exec_warps"] = ew
     return cfg
 
 

@@ -251,7 +251,8 @@ __device__ __forceinline__ void trace_ev(const MkParams& p, int mtb, uint32_t& s
         if (seq < p.trace_cap) {
             LedgerEvent e;
             e.seq = seq; e.mtb = (uint16_t)mtb; e.kind = kind; e.bar_id = bar; e.task_id = task_id;
-            e.warp_mask = mask; e.tb = tb; e.gran_off = goff; e.gran_len = glen; e.pad = 0; e.pad2 = 0;
+            e.warp_mask = mask; e.tb = tb; e.gran_off = goff; e.gran_len = glen; e.pad = 0;
+            e.pad2 = (uint32_t)globaltimer_ns();   /* low 32 bits of the event's %globaltimer (profiling) */
             p.trace[(size_t)mtb * p.trace_cap + seq] = e;
         }
         p.trace_count[mtb] = seq + 1;

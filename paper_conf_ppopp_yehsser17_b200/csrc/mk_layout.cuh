@@ -70,7 +70,7 @@ struct LedgerEvent {   /* 32 B; identical field order to the oracle's checker in
     uint16_t gran_off;
     uint16_t gran_len;
     uint16_t pad;
-    uint32_t pad2;
+    uint32_t pad2;     /* low 32 bits of %globaltimer when the scheduler logged it (not checked) */
 };
 static_assert(sizeof(LedgerEvent) == 32, "LedgerEvent is 32 bytes");
 

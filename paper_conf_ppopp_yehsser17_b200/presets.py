@@ -28,4 +28,7 @@ def ctx_kwargs(workload: str, flags: int = 0) -> dict:
     """pagoda_config keyword arguments (Pagoda(**...)) of the workload's preset."""
     pr = PRESETS[workload]
     f = flags | (RESIDENT_TDES if pr["resident"] else 0) | (SPREAD if pr.get("spread") else 0)
-    return {"flags": f, "mtbs_per_sm": pr["mtbs_per_sm"], "arena_bytes": pr["arena_bytes"]}
+    kw = {"flags": f, "mtbs_per_sm": pr["mtbs_per_sm"], "arena_bytes": pr["arena_bytes"]}
+    if pr.get("exec_warps"):
+        kw["exec_warps"] = pr["exec_warps"]
+    return kw

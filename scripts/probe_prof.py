@@ -39,4 +39,5 @@ if __name__ == "__main__":
     run("nop4", W.nop(65536, threads=128))
     run("nop8", W.nop(65536, threads=256))
     run("mm", W.matmul(65536))
+    run("mm_4mtb", W.matmul(65536), mtbs_per_sm=4, arena_bytes=48 * 1024)
     run("tdes", W.tdes(32768, shmem=512), flags=PG.RESIDENT_TDES, arena_bytes=40 * 1024)

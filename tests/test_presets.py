@@ -19,6 +19,8 @@ def test_ctx_kwargs_match_bench_context():
             no_resident = False
             mtbs = 0
             arena_kb = 0
+            exec_warps = 0
+            spread = -1
         cfg = bench.ctx_config(A, PG, w)
         kw = presets.ctx_kwargs(w, PG.NO_START)
         assert cfg == kw, w
