@@ -54,6 +54,15 @@
 #ifndef PAGODA_CLAIM_SMALL
 #define PAGODA_CLAIM_SMALL 1  /* tickets per claim while the backlog is below what all MTBs could take */
 #endif
+#ifndef PAGODA_FAST_LOAD
+#define PAGODA_FAST_LOAD 1    /* ring cells are copied 4 lanes per cell with relaxed 16-byte loads all in
+                                 flight together (one L2 round trip; the cells' sequence words were already
+                                 acquired), not 4 serial acquire loads per cell */
+#endif
+#ifndef PAGODA_FAST_PUB
+#define PAGODA_FAST_PUB 1     /* a publisher checks 256 cells with relaxed loads all in flight, then one
+                                 acquire fence (not 8 serial acquire loads per lane) */
+#endif
 #ifndef PAGODA_HOLDER_POSTS
 #define PAGODA_HOLDER_POSTS 0 /* the scheduler token holder posts completion records (batched per round);
                                  the last warp of a task only marks it pending and frees itself */
@@ -75,6 +84,27 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity)
     uint32_t done = 0;
     const uint32_t a = smem_u32(bar);
     while (!done) {
+        asm volatile(
+            "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3; selp.u32 %0, 1, 0, p; }"
+            : "=r"(done)
+            : "r"(a), "r"(parity), "n"(PAGODA_WAKE_HINT_NS)
+            : "memory");
+    }
+}
+/* An idle executor's wait for its dispatch mbarrier (exec_bar[warp], at the start of the MTB's
+ * control block).  A warp suspended in try_wait is woken by mbarrier traffic anywhere in the CTA,
+ * so idle warps run this loop millions of times per session; the loop therefore recomputes its
+ * barrier address from %tid (two ALU ops) every trip instead of keeping it live across the task
+ * body, where the 32-register build spilled it: a local-memory load per trip put idle warps on
+ * the load/store pipe the busy warps' bodies need (ncu source counters). */
+__device__ __forceinline__ void exec_wait(uint32_t parity)
+{
+    extern __shared__ __align__(1024) unsigned char pagoda_mk_smem[];
+    uint32_t done = 0;
+    while (!done) {
+        uint32_t tid;
+        asm volatile("mov.u32 %0, %%tid.x;" : "=r"(tid));
+        const uint32_t a = smem_u32(pagoda_mk_smem) + ((tid >> 5) << 3);   /* &S.exec_bar[warp] */
         asm volatile(
             "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3; selp.u32 %0, 1, 0, p; }"
             : "=r"(done)
@@ -564,8 +594,11 @@ __device__ __forceinline__ bool ingest_publish(const MkParams& p, const char* sr
 #pragma unroll
         for (int i = 0; i < 8; i++) {
             const uint32_t k = base + (uint32_t)i * 32u + lane;
-            /* acquire (LDG.STRONG + L1 invalidate, no MEMBAR): the cell's previous reader is done */
-            sv[i] = k < n ? ld_acquire_gpu32(&p.dseq[(s + k) & p.ring_mask]) : (uint32_t)(s + k);
+            /* the cell's previous reader is done: acquire (LDG.STRONG + L1 invalidate, no MEMBAR) per load,
+             * or (FAST_PUB) relaxed loads all in flight at once, made an acquire by the fence below */
+            sv[i] = k < n ? (PAGODA_FAST_PUB ? ld_relaxed_gpu32(&p.dseq[(s + k) & p.ring_mask])
+                                             : ld_acquire_gpu32(&p.dseq[(s + k) & p.ring_mask]))
+                          : (uint32_t)(s + k);
         }
         uint32_t bad = 0;
 #pragma unroll
@@ -578,6 +611,7 @@ __device__ __forceinline__ bool ingest_publish(const MkParams& p, const char* sr
         }
         base += 256u;
     }
+    if (PAGODA_FAST_PUB) fence_acq_rel_gpu();   /* acquire pattern: relaxed reads of the cells, then this fence */
     const uint64_t t3 = globaltimer_ns();
     __syncwarp();          /* every lane's acquire precedes lane 0's bulk store */
     const uint64_t t4 = globaltimer_ns();
@@ -1038,11 +1072,36 @@ __device__ int sched_copy(MtbShared& S, Sched& st, const MkParams& p, uint32_t r
 {
     const uint32_t lane = threadIdx.x & 31u;
     const uint64_t t = lane < r ? S.pend_ticket[(st.pl + lane) & 31u] : 0;
-#if PAGODA_CELL_ACQ
+#if PAGODA_FAST_LOAD
+    /* 4 lanes per cell, one 16-byte relaxed load each: up to 8 cells per warp instruction, all in
+     * flight together (one L2 round trip; the sequence words' acquires in sched_load ordered these
+     * loads after them and invalidated L1).  The hand-back store of a cell must not be performed
+     * before the cell's loads: the warp issues in order, and the shared-memory stores of the loaded
+     * words (STS, which wait for the data) precede the hand-back in program order. */
+    for (uint32_t c = lane; c < r * 4u; c += 32u) {
+        const uint32_t i = c >> 2, q = c & 3u;
+        const uint64_t ti = S.pend_ticket[(st.pl + i) & 31u];
+        int4 v;
+        asm volatile("ld.relaxed.gpu.global.v4.s32 {%0,%1,%2,%3}, [%4];"
+                     : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
+                     : "l"(reinterpret_cast<const int4*>(p.dring + (ti & p.ring_mask)) + q)
+                     : "memory");
+        reinterpret_cast<int4*>(&S.tasks[nth_set_bit(st.free_task, i)])[q] = v;
+    }
+    __syncwarp();
+    uint32_t used = 0;
+    if (lane < r) {
+        const uint32_t slot = nth_set_bit(st.free_task, lane);
+        S.pend[(st.pl + lane) & 31u] = (uint8_t)slot;
+        st_relaxed_gpu32(&p.dseq[t & p.ring_mask], (uint32_t)(t + (uint64_t)p.ring_mask + 1));
+        if (p.life && !(S.tasks[slot].flags & kEntryGroup)) life_stamp(p, S.tasks[slot].id, kLifeLoad);
+        used = 1u << slot;
+    }
+#elif PAGODA_CELL_ACQ
     /* lane i copies cell i whole with acquire loads (LDG.STRONG.GPU + L1 invalidate, no MEMBAR),
      * so its own hand-back store below is ordered after every read of the cell in program order.
-     * (A st.release would be a MEMBAR.GPU, which waits for every memory operation in flight on
-     * the SM: the holder's largest single cost per scheduling round.) */
+     * (A st.release would be a MEMBAR.GPU, which waits for every memory operation in flight on the
+     * SM.)  The four acquires are serial: four round trips. */
     uint32_t used = 0;
     if (lane < r) {
         const uint32_t slot = nth_set_bit(st.free_task, lane);
@@ -1402,7 +1461,7 @@ __device__ void worker(MtbShared& S, char* smem_base, const MkParams& p, int mtb
             if (holder_phase(S, p, mtb, w, exec_mask)) return;
             holder = false;
         }
-        mbar_wait(&S.exec_bar[w], phase);
+        exec_wait(phase);   /* mbar_wait(&S.exec_bar[w], phase) without a live address register */
         phase ^= 1u;
         const uint8_t task = *(volatile uint8_t*)&S.wt[w].task;
         if (task == SLOT_TERMINATE) return;
