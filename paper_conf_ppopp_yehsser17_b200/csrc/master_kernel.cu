@@ -55,7 +55,7 @@
 #define PAGODA_CLAIM_SMALL 1  /* tickets per claim while the backlog is below what all MTBs could take */
 #endif
 #ifndef PAGODA_FAST_LOAD
-#define PAGODA_FAST_LOAD 1    /* ring cells are copied 4 lanes per cell with relaxed 16-byte loads all in
+#define PAGODA_FAST_LOAD 0    /* ring cells are copied 4 lanes per cell with relaxed 16-byte loads all in
                                  flight together (one L2 round trip; the cells' sequence words were already
                                  acquired), not 4 serial acquire loads per cell */
 #endif
@@ -986,6 +986,118 @@ __device__ bool sched_place(MtbShared& S, Sched& st, const MkParams& p, int mtb,
     return true;
 }
 
+/* Batched placement ("__match_any_sync on (w, shmem, sync) groups identical tasks so
+ * one pass places them"): the run of loaded tasks at the FIFO head that share the head's shape
+ * (one thread block, same warps, granules and barrier need; a task spread over MTBs goes through
+ * sched_place) is placed in ONE pass, as many as the MTB holds now: one free-mask update, lane i
+ * keeps task i's bookkeeping, lane l writes warp l's WarpTable slot, one arrive per warp.  The
+ * cost of placing k tasks is then about that of one (the holder's place step was the largest share
+ * of its time: it runs among the body warps' shared-memory traffic).  Returns the number placed;
+ * -1 if the head is not batchable (the caller uses sched_place). */
+#ifndef PAGODA_BATCH_PLACE
+#define PAGODA_BATCH_PLACE 1
+#endif
+__device__ int sched_place_run(MtbShared& S, Sched& st, const MkParams& p, int mtb)
+{
+    const uint32_t lane = threadIdx.x & 31u;
+    const uint32_t navail = min(st.pl - st.ph, 32u);
+    uint32_t key = 0xFFFFFFFFu, slot = 0;
+    if (lane < navail) {
+        slot = S.pend[(st.ph + lane) & 31u];
+        const TaskEntry& e = S.tasks[slot];
+        const uint32_t g = (e.shmem_bytes + PAGODA_GRANULE - 1u) / PAGODA_GRANULE;
+        if (e.n_tb == 1 && !(e.flags & kEntryGroup))
+            key = (uint32_t)e.warps_tb | (g << 6) | ((((e.flags & kEntrySync) != 0) && e.warps_tb > 1) ? (1u << 17) : 0u);
+    }
+    const uint32_t k0 = __shfl_sync(0xffffffffu, key, 0);
+    if (k0 == 0xFFFFFFFFu) return -1;
+    const uint32_t same = __ballot_sync(0xffffffffu, key == k0);
+    uint32_t fit = same == 0xffffffffu ? 32u : (uint32_t)__ffs(~same) - 1u;   /* the run at the head */
+    const uint32_t wtb = k0 & 63u, gtb = (k0 >> 6) & 2047u;
+    const bool need_bar = (k0 >> 17) & 1u;
+    fit = min(fit, (uint32_t)__popc(st.free_w) / wtb);
+    fit = min(fit, (uint32_t)__popc(st.free_tbs));
+    if (need_bar) fit = min(fit, (uint32_t)__popc(st.free_bar));
+    /* granules: first fit task by task (register and shuffle work only); lane i keeps task i's offset */
+    uint32_t off = 0;
+    if (gtb) {
+        for (uint32_t i = 0; i < fit; i++) {
+            const int o = bm_first_fit(st.fg, gtb, lane);
+            if (o < 0) {
+                fit = i;
+                break;
+            }
+            st.fg &= ~bm_range_bits((uint32_t)o, gtb, lane);
+            if (lane == i) off = (uint32_t)o;
+        }
+    }
+    if (fit == 0) return 0;
+    /* warps: the lowest fit * wtb free ones, the token holder last (it keeps scheduling unless needed) */
+    const uint32_t nw = fit * wtb;
+    uint32_t sel = 0, fw = st.free_w & ~st.holder_bit;
+    for (uint32_t i = 0; i < nw; i++) {
+        if (!fw) fw = st.free_w & st.holder_bit;
+        sel |= fw & (0u - fw);
+        fw &= fw - 1u;
+    }
+    st.free_w &= ~sel;
+    /* lane i < fit: task i's TB record, barrier, id */
+    uint32_t tbs = 0, bar = 0;
+    uint64_t id = 0;
+    uint16_t threads = 0;
+    if (lane < fit) {
+        tbs = nth_set_bit(st.free_tbs, lane);
+        if (need_bar) bar = nth_set_bit(st.free_bar, lane);
+        const TaskEntry& e = S.tasks[slot];
+        id = e.id;
+        threads = e.threads_tb;
+        S.task_warps_left[slot] = wtb;
+        S.tb_warps_left[tbs] = wtb;
+        S.tb_goff[tbs] = (uint16_t)off;
+        S.tb_glen[tbs] = (uint16_t)gtb;
+        S.tb_bar[tbs] = (uint8_t)bar;
+        S.tb_task[tbs] = id;
+        S.tb_idx[tbs] = 0;
+        if (p.life) life_stamp(p, id, kLifePlace);
+    }
+    st.free_tbs &= ~__reduce_or_sync(0xffffffffu, lane < fit ? (1u << tbs) : 0u);
+    if (need_bar) st.free_bar &= ~__reduce_or_sync(0xffffffffu, lane < fit ? (1u << bar) : 0u);
+    /* lane l of the selected warps: task i = rank / wtb, warp wtb-rank within it */
+    const uint32_t r = (uint32_t)__popc(sel & ((1u << lane) - 1u));
+    const uint32_t ti = ((sel >> lane) & 1u) ? r / wtb : 0u;
+    const uint32_t t_slot = __shfl_sync(0xffffffffu, slot, ti), t_tbs = __shfl_sync(0xffffffffu, tbs, ti);
+    const uint32_t t_off = __shfl_sync(0xffffffffu, off, ti), t_bar = __shfl_sync(0xffffffffu, bar, ti);
+    const uint32_t t_thr = __shfl_sync(0xffffffffu, (uint32_t)threads, ti);
+    const uint64_t t_id = __shfl_sync(0xffffffffu, id, ti);
+    if (p.trace_cap) {   /* the ledger: one ALLOC per task, in FIFO order */
+        for (uint32_t i = 0; i < fit; i++) {
+            const uint32_t mi = __ballot_sync(0xffffffffu, ((sel >> lane) & 1u) && ti == i);
+            trace_ev(p, mtb, st.seq, 1, __shfl_sync(0xffffffffu, id, i), 0, mi,
+                     (uint16_t)__shfl_sync(0xffffffffu, off, i), (uint16_t)gtb,
+                     (uint8_t)__shfl_sync(0xffffffffu, bar, i));
+        }
+    }
+    if ((sel >> lane) & 1u) {
+        WarpSlot ws;
+        ws.smem_off = p.arena_offset + t_off * PAGODA_GRANULE;
+        ws.smem_bytes = gtb * PAGODA_GRANULE;
+        ws.tb = 0;
+        ws.threads_tb = (uint16_t)t_thr;
+        ws.task = (uint8_t)t_slot;
+        ws.warp_in_tb = (uint8_t)(r - ti * wtb);
+        ws.warps_tb = (uint8_t)wtb;
+        ws.n_tb = 1;
+        ws.bar_id = (uint8_t)t_bar;
+        ws.tbslot = (uint8_t)t_tbs;
+        ws.n_tb_all = 1;
+        ws.task_id = t_id;
+        S.wt[lane] = ws;
+    }
+    __syncwarp();   /* every lane's bookkeeping happens-before the release-arrives */
+    if ((sel >> lane) & 1u) mbar_arrive(&S.exec_bar[lane]);
+    return (int)fit;
+}
+
 /* Take tickets: as many tasks as the free warps fit at the last task size
  * (one ticket when the size is unknown), never more than the ring holds; one
  * at a time while the backlog is smaller than what all MTBs could take, so
@@ -1341,7 +1453,14 @@ __device__ bool sched_round(MtbShared& S, Sched& st, const MkParams& p, int mtb,
 #endif
     t0 = pf_now();
     while (st.ph != st.pl) {
-        if (!sched_place(S, st, p, mtb, S.pend[st.ph & 31u])) {
+        const int k = PAGODA_BATCH_PLACE ? sched_place_run(S, st, p, mtb) : -1;
+        if (k > 0) {   /* a run of identical single-TB tasks placed in one pass */
+            sc_add(S, kScPlaced, (uint32_t)k);
+            st.ph += (uint32_t)k;
+            progress = true;
+            continue;
+        }
+        if (k == 0 || !sched_place(S, st, p, mtb, S.pend[st.ph & 31u])) {
             sc_add(S, kScNoFit, 1);
             break;
         }

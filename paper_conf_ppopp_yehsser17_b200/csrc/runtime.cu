@@ -511,7 +511,10 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
     }
     if (cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking) != cudaSuccess) goto fail;
     if (cudaEventCreate(&c->ev_start) != cudaSuccess || cudaEventCreate(&c->ev_stop) != cudaSuccess) goto fail;
-    if (cudaDeviceSynchronize() != cudaSuccess) goto fail;
+    /* the set-up copies and memsets above ran on the legacy stream: wait for that stream only.  A
+     * device-wide synchronize would also wait for another context's persistent MasterKernel on the
+     * same device (pool members sharing a GPU) and never return. */
+    if (cudaStreamSynchronize(cudaStreamLegacy) != cudaSuccess) goto fail;
     {
         MkParams& p = c->params;
         memset(&p, 0, sizeof p);
