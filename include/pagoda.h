@@ -83,7 +83,10 @@ void pagoda_config_default(pagoda_config* cfg);
 int pagoda_init(const pagoda_config* cfg, pagoda_ctx** out);
 
 /* waitAll, then stop the MasterKernel, free everything and *out is invalid.
- * Returns 0, -EIO (device fault seen), -ETIMEDOUT (watchdog; resources leaked). */
+ * Freeing device memory synchronizes the whole device, so another context's
+ * MasterKernel still running on the same GPU must be stopped first (the pool
+ * does this for its members).  Returns 0, -EIO (device fault seen),
+ * -ETIMEDOUT (watchdog; resources leaked). */
 int pagoda_shutdown(pagoda_ctx* ctx);
 
 /* taskSpawn (Table 1, §3): spawn one task of n_threadblocks

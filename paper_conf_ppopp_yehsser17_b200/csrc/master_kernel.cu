@@ -995,7 +995,7 @@ __device__ bool sched_place(MtbShared& S, Sched& st, const MkParams& p, int mtb,
  * of its time: it runs among the body warps' shared-memory traffic).  Returns the number placed;
  * -1 if the head is not batchable (the caller uses sched_place). */
 #ifndef PAGODA_BATCH_PLACE
-#define PAGODA_BATCH_PLACE 1
+#define PAGODA_BATCH_PLACE 0   /* measured: slower (most rounds place one task; the run logic costs more than it saves) */
 #endif
 __device__ int sched_place_run(MtbShared& S, Sched& st, const MkParams& p, int mtb)
 {

@@ -371,6 +371,17 @@ extern "C" int pagoda_pool_shutdown(pagoda_pool* p)
     if (!p) return -EINVAL;
     stop_spawners(p);
     int rc = 0;
+    /* every member's MasterKernel exits BEFORE any member frees memory: cudaFree synchronizes the
+     * whole device, so freeing one member while another (sharing the GPU) still runs would never
+     * return */
+    for (auto* m : p->m) {
+        int r = pagoda_waitAll(m->ctx);
+        if (r && !rc) rc = r;
+    }
+    for (auto* m : p->m) {
+        int r = pagoda_stop(m->ctx);
+        if (r && r != -EALREADY && !rc) rc = r;
+    }
     for (auto* m : p->m) {
         int r = pagoda_shutdown(m->ctx);
         if (r && !rc) rc = r;
