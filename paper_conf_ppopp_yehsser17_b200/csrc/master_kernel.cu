@@ -233,6 +233,35 @@ __device__ __forceinline__ int bm_first_fit(uint32_t fg, uint32_t g, uint32_t la
     const uint32_t w = __shfl_sync(0xffffffffu, R, L);
     return (int)(L * 32u + __ffs(w) - 1);
 }
+/* The same for g <= 32 without shuffles: the lowest run of g free granules that lies inside one
+ * lane's 32-granule word (runs across two words are left to bm_first_fit).  Shuffles travel the
+ * shared-memory crossbar the task bodies keep busy; the holder's place step was the largest share
+ * of its time under load (scripts/probe_prof.py). */
+__device__ __forceinline__ int bm_first_fit_local(uint32_t fg, uint32_t g)
+{
+    uint32_t R = fg, len = 1;
+    while (len * 2u <= g) {
+        R &= R >> len;
+        len *= 2u;
+    }
+    if (g > len) R &= R >> (g - len);
+    const uint32_t b = __ballot_sync(0xffffffffu, R != 0);
+    if (!b) return -1;
+    const uint32_t L = __ffs(b) - 1;
+    const uint32_t w = __shfl_sync(0xffffffffu, R, L);
+    return (int)(L * 32u + __ffs(w) - 1);
+}
+#ifndef PAGODA_LOCAL_FIT
+#define PAGODA_LOCAL_FIT 1
+#endif
+__device__ __forceinline__ int bm_fit(uint32_t fg, uint32_t g, uint32_t lane)
+{
+    if (PAGODA_LOCAL_FIT && g <= 32u) {
+        const int o = bm_first_fit_local(fg, g);
+        if (o >= 0) return o;
+    }
+    return bm_first_fit(fg, g, lane);
+}
 __device__ __forceinline__ uint32_t bm_range_bits(uint32_t off, uint32_t g, uint32_t lane)
 {
     const uint32_t lo = max(off, lane * 32u), hi = min(off + g, lane * 32u + 32u);
@@ -917,12 +946,18 @@ __device__ bool sched_place(MtbShared& S, Sched& st, const MkParams& p, int mtb,
     if ((uint32_t)__popc(st.free_w) < wtb * ntb || (uint32_t)__popc(st.free_tbs) < ntb ||
         (need_bar && (uint32_t)__popc(st.free_bar) < ntb))
         return false;
+    int off0 = 0;   /* one TB: its first fit, found once (the feasibility check IS the allocation) */
     if (gtb) {   /* feasibility of all TBs' shared memory first (all-or-nothing per task) */
-        uint32_t fg2 = st.fg;
-        for (uint32_t j = 0; j < ntb; j++) {
-            const int off = bm_first_fit(fg2, gtb, lane);
-            if (off < 0) return false;
-            fg2 &= ~bm_range_bits((uint32_t)off, gtb, lane);
+        if (ntb == 1) {
+            off0 = bm_fit(st.fg, gtb, lane);
+            if (off0 < 0) return false;
+        } else {
+            uint32_t fg2 = st.fg;
+            for (uint32_t j = 0; j < ntb; j++) {
+                const int off = bm_fit(fg2, gtb, lane);
+                if (off < 0) return false;
+                fg2 &= ~bm_range_bits((uint32_t)off, gtb, lane);
+            }
         }
     }
     const uint64_t id = e.id;
@@ -950,7 +985,7 @@ __device__ bool sched_place(MtbShared& S, Sched& st, const MkParams& p, int mtb,
         }
         uint32_t off = 0;
         if (gtb) {
-            off = (uint32_t)bm_first_fit(st.fg, gtb, lane);
+            off = ntb == 1 ? (uint32_t)off0 : (uint32_t)bm_fit(st.fg, gtb, lane);
             st.fg &= ~bm_range_bits(off, gtb, lane);
         }
         if (lane == 0) {
