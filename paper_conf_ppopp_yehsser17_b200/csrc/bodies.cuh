@@ -161,32 +161,29 @@ __device__ void body_mb(const Env& e, const pagoda_mb_args& a)
 {
     const int T = total_threads(e);
     const int maxit = a.maxit;
-    /* Each lane walks its own pixels p = tid, tid + T, ... independently: one trip of the loop is
-     * one step of the lane's current pixel, and a lane whose pixel finished writes it and starts
-     * its next at once.  A warp then runs until its lanes' TOTAL work is done, not the sum over
-     * pixel rounds of the slowest lane's pixel (lockstep rounds idle most lanes of a warp on
-     * tiles where the set's boundary passes: the irregularity the paper's MB is about).  Every
-     * pixel's own sequence of operations is unchanged (outputs are bit-identical).
-     * A step is four iterations: each tests |z|^2 > 4 on its own z and updates z unconditionally;
-     * the count advances to the first escaping iteration (later ones only touch discarded
-     * values); within 4 of maxit, single iterations. */
-    int p = e.getTid();
-    bool live = p < 4096;
-    float cr = 0.0f, ci = 0.0f, zr = 0.0f, zi = 0.0f;
-    int n = 0;
-    auto start = [&](int q) {
-        const int gx = 64 * a.tx + (q & 63), gy = 64 * a.ty + (q >> 6);
-        cr = __fadd_rn(a.x0, __fmul_rn((float)gx, a.dx));
-        ci = __fadd_rn(a.y0, __fmul_rn((float)gy, a.dx));
-        zr = 0.0f;
-        zi = 0.0f;
-        n = 0;
-    };
-    if (live) start(p);
-    while (__any_sync(0xffffffffu, live)) {
-        if (!live) continue;
-        bool fin;
-        if (n + 4 <= maxit) {
+    for (int p = e.getTid(); p < 4096; p += T) {
+        const int gx = 64 * a.tx + (p & 63), gy = 64 * a.ty + (p >> 6);
+        const float cr = __fadd_rn(a.x0, __fmul_rn((float)gx, a.dx));
+        const float ci = __fadd_rn(a.y0, __fmul_rn((float)gy, a.dx));
+        float zr = 0.0f, zi = 0.0f;
+        int n = 0;
+        /* Four iterations per branch: each step tests |z|^2 > 4 on its own z and
+         * updates z unconditionally; the count advances to the first escaping step
+         * (steps after it only touch values that are discarded).  A branch per
+         * iteration costs more than the iteration itself on the critical path. */
+        for (;;) {
+            if (n + 4 > maxit) {   /* remainder: one iteration at a time */
+                while (n < maxit) {
+                    const float zr2 = __fmul_rn(zr, zr);
+                    const float zi2 = __fmul_rn(zi, zi);
+                    if (__fadd_rn(zr2, zi2) > 4.0f) break;
+                    const float t = __fadd_rn(zr, zr);
+                    zi = __fadd_rn(__fmul_rn(t, zi), ci);
+                    zr = __fadd_rn(__fsub_rn(zr2, zi2), cr);
+                    n++;
+                }
+                break;
+            }
             bool esc[4];
 #pragma unroll
             for (int s = 0; s < 4; s++) {
@@ -197,27 +194,13 @@ __device__ void body_mb(const Env& e, const pagoda_mb_args& a)
                 zi = __fadd_rn(__fmul_rn(t, zi), ci);
                 zr = __fadd_rn(__fsub_rn(zr2, zi2), cr);
             }
-            fin = esc[0] | esc[1] | esc[2] | esc[3];
-            n += esc[0] ? 0 : esc[1] ? 1 : esc[2] ? 2 : esc[3] ? 3 : 4;
-        } else if (n < maxit) {   /* remainder: one iteration */
-            const float zr2 = __fmul_rn(zr, zr);
-            const float zi2 = __fmul_rn(zi, zi);
-            fin = __fadd_rn(zr2, zi2) > 4.0f;
-            if (!fin) {
-                const float t = __fadd_rn(zr, zr);
-                zi = __fadd_rn(__fmul_rn(t, zi), ci);
-                zr = __fadd_rn(__fsub_rn(zr2, zi2), cr);
-                n++;
+            if (esc[0] | esc[1] | esc[2] | esc[3]) {
+                n += esc[0] ? 0 : esc[1] ? 1 : esc[2] ? 2 : 3;
+                break;
             }
-        } else {
-            fin = true;
+            n += 4;
         }
-        if (fin || n >= maxit) {
-            a.out[p] = (uint16_t)n;
-            p += T;
-            live = p < 4096;
-            if (live) start(p);
-        }
+        a.out[p] = (uint16_t)n;
     }
 }
 
