@@ -90,6 +90,7 @@ def parse():
     ap.add_argument("--quick", action="store_true", help="skip everything but the timed steps (for ncu)")
     ap.add_argument("--mtbs", type=int, default=0, help="MTBs per SM (default: the workload preset)")
     ap.add_argument("--exec-warps", type=int, default=0, help="worker warps per MTB (default: the preset's, else all)")
+    ap.add_argument("--groups", type=int, default=0, help="scheduling groups per MTB, 1 or 2 (default: the preset's)")
     ap.add_argument("--spread", type=int, default=-1, help="spread-first claims on (1) / off (0) (default: preset)")
     ap.add_argument("--arena-kb", type=int, default=0, help="task arena per MTB in KiB (default: preset)")
     ap.add_argument("--producers", type=int, default=0,
@@ -426,6 +427,9 @@ def ctx_config(a, PG, name):
     ew = a.exec_warps if mine and getattr(a, "exec_warps", 0) else pr.get("exec_warps", 0)
     if ew:
         cfg["exec_warps"] = ew
+    ng = a.groups if mine and getattr(a, "groups", 0) else pr.get("sched_groups", 0)
+    if ng:
+        cfg["sched_groups"] = ng
     return cfg
 
 

@@ -68,6 +68,14 @@ typedef struct {
     uint32_t trace_events;  /* ledger capacity per MTB when PAGODA_TRACE (default 8192) */
     double   watchdog_s;    /* wait/waitAll/shutdown give up with -ETIMEDOUT after this many
                                seconds without progress (default 60; <= 0 disables) */
+    uint32_t sched_groups;  /* scheduling groups per MTB: 1 (default) or 2.  With 2, an MTB's warps,
+                               task slots, TB records, arena and named barriers (1..7 / 8..15) are split
+                               in halves (exec_warps counts both: exec_warps / 2 workers per half),
+                               each with its own scheduler token, so two holders place
+                               tasks in parallel (e.g. sharing the MTB-resident 3DES tables); a thread
+                               block must then fit half an MTB and a task has at most 7 syncing TBs
+                               per entry.  The ledger (PAGODA_TRACE) is kept per group: ids
+                               mtb * sched_groups + g in pagoda_trace_read / executor records. */
 } pagoda_config;
 
 /* Fill *cfg with the defaults above. */
@@ -240,6 +248,7 @@ typedef struct {
     int64_t  completed_low; /* every id below this is known done */
     uint32_t device_error;  /* 0 or a PAGODA_DEVERR_* code */
     int      running;       /* MasterKernel still resident */
+    int      sched_groups;  /* scheduling groups per MTB (pagoda_config.sched_groups) */
 } pagoda_info;
 int pagoda_get_info(pagoda_ctx* ctx, pagoda_info* out);
 

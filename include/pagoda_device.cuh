@@ -48,12 +48,12 @@ enum : uint8_t { SLOT_TERMINATE = 0xFF, SLOT_SCHED = 0xFE /* take over the sched
  * laid out in csrc/mk_layout.cuh, which static_asserts them).  The task arena
  * follows the control block, or the resident tables when a context has them. */
 constexpr uint32_t kWarpTableOffset = 512;
-constexpr uint32_t kControlBytes = 6144;            /* arena offset without resident tables */
+constexpr uint32_t kControlBytes = 6656;            /* arena offset without resident tables (13 granules) */
 constexpr uint32_t kResidentOffset = 8192;          /* room reserved for the control block + resident tables */
 constexpr uint32_t kResidentTdesBytes = 8 * 64 * 32 * 4;   /* 3DES SP tables, one copy per lane */
 constexpr uint32_t kResidentTdesAddr = 8192;        /* shared-WINDOW address of the resident tables: a
                                                        constant, so lookups carry it as an immediate */
-constexpr uint32_t kDevErrorPtrOffset = 5960;       /* MtbShared.dev_error: the device error word's address, for
+constexpr uint32_t kDevErrorPtrOffset = 5656;       /* MtbShared.dev_error: the device error word's address, for
                                                        the paper-named free syncBlock() (which has no TaskEnv) */
 constexpr uint32_t kDevErrSyncWithoutFlag = 1u;     /* == PAGODA_DEVERR_SYNC_WITHOUT_FLAG (pagoda.h) */
 
@@ -80,7 +80,7 @@ __device__ __forceinline__ uint32_t smem_u32(const void* p)
  * Everything a body asks for is read from the executor warp's WarpTable slot in
  * shared memory when asked (no register holds it across the body). */
 constexpr uint32_t kStageBarOffset = 256;     /* per-warp TMA staging mbarriers (MtbShared.stage_bar) */
-constexpr uint32_t kStagePhaseOffset = 4824;  /* their parities, one u32 per warp (MtbShared.stage_ph) */
+constexpr uint32_t kStagePhaseOffset = 4608;  /* their parities, one u32 per warp (MtbShared.stage_ph) */
 
 struct TaskEnv {
     uint32_t* dev_error;    /* device error word */

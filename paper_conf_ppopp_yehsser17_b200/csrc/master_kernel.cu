@@ -272,9 +272,9 @@ __device__ __forceinline__ uint32_t bm_range_bits(uint32_t off, uint32_t g, uint
 
 /* scheduler counters: holder-private shared-memory words, added to DevCtl.ctr at exit */
 enum { kScRounds = 0, kScProgress, kScTickets, kScClaimEmpty, kScLoadNotReady, kScPlaced, kScNoFit, kScHandoffs };
-__device__ __forceinline__ void sc_add(MtbShared& S, int i, uint32_t v)
+__device__ __forceinline__ void sc_add(SchedGroup& G, int i, uint32_t v)
 {
-    if ((threadIdx.x & 31u) == 0) S.sctr[i] += v;
+    if ((threadIdx.x & 31u) == 0) G.sctr[i] += v;
 }
 
 /* profiling builds: ns per scheduler phase (holder-private) and per executor step */
@@ -283,12 +283,12 @@ __device__ __forceinline__ void sc_add(MtbShared& S, int i, uint32_t v)
 #endif
 enum { kPfFold = 0, kPfLoad, kPfPlace, kPfClaim, kPfSleep, kPfBody, kPfFence, kPfPost };
 __device__ __forceinline__ uint64_t pf_now() { return PAGODA_PROFILE ? globaltimer_ns() : 0; }
-__device__ __forceinline__ void pf_add(MtbShared& S, int i, uint64_t t0, bool shared_atomic)
+__device__ __forceinline__ void pf_add(SchedGroup& G, int i, uint64_t t0, bool shared_atomic)
 {
     if (!PAGODA_PROFILE || (threadIdx.x & 31u) != 0) return;
     const unsigned long long d = globaltimer_ns() - t0;
-    if (shared_atomic) atomicAdd(&S.sprof[i], d);
-    else S.sprof[i] += d;
+    if (shared_atomic) atomicAdd(&G.sprof[i], d);
+    else G.sprof[i] += d;
 }
 
 /* ------------------------------------------------------------------ life cycle stamps (PAGODA_LIFECYCLE) */
@@ -331,16 +331,16 @@ __device__ __forceinline__ void trace_ev(const MkParams& p, int mtb, uint32_t& s
  * MTB there is no such split: the record goes to the host directly behind a
  * system-scope fence.  The task slot is returned (mb_tasks) only after its id
  * was read, so the id stays valid until then. */
-__device__ __forceinline__ void post_completions(MtbShared& S, const MkParams& p)
+__device__ __forceinline__ void post_completions(MtbShared& S, SchedGroup& G, const MkParams& p)
 {
     const uint32_t lane = threadIdx.x & 31u;
     for (;;) {
         uint32_t got = 0;
-        if (lane == 0) got = atomicExch(&S.poster, 1u) == 0u;
+        if (lane == 0) got = atomicExch(&G.poster, 1u) == 0u;
         if (!__shfl_sync(0xffffffffu, got, 0)) return;   /* the holder will see our bit */
         for (;;) {
             uint32_t m = 0;
-            if (lane == 0) m = atomicExch(&S.comp_pending, 0u);
+            if (lane == 0) m = atomicExch(&G.comp_pending, 0u);
             m = __shfl_sync(0xffffffffu, m, 0);
             if (!m) break;
             const bool done = (m >> lane) & 1u;
@@ -391,14 +391,14 @@ __device__ __forceinline__ void post_completions(MtbShared& S, const MkParams& p
             __syncwarp();
             if (lane == 0) {
                 __threadfence_block();
-                atomicOr(&S.mb_tasks, m);   /* the scheduler may now reuse those task slots */
+                atomicOr(&G.mb_tasks, m);   /* the scheduler may now reuse those task slots */
             }
         }
         uint32_t again = 0;
         if (lane == 0) {
-            atomicExch(&S.poster, 0u);
+            atomicExch(&G.poster, 0u);
             __threadfence_block();   /* release the flag, then re-check: a bit set meanwhile by a */
-            again = *(volatile uint32_t*)&S.comp_pending != 0u;   /* warp that found the flag taken */
+            again = *(volatile uint32_t*)&G.comp_pending != 0u;   /* warp that found the flag taken */
         }
         if (!__shfl_sync(0xffffffffu, again, 0)) return;
     }
@@ -451,7 +451,7 @@ __device__ void comp_forwarder(MtbShared& S, const MkParams& p, uint32_t f)
             uint32_t done = 0;
             /* acquire of the exit count orders the tail read after it: every MTB's reservations
              * (made before its release-ordered exit increment) are then in the tail we read */
-            if (lane == 0) done = ld_acquire_gpu32(&p.dctl->exited) >= (uint32_t)p.n_mtb &&
+            if (lane == 0) done = ld_acquire_gpu32(&p.dctl->exited) >= p.n_exit &&
                                   ld_relaxed_gpu(&p.dctl->dq_tail) <= c;
             if (__shfl_sync(0xffffffffu, done, 0)) break;
             __nanosleep(idle < 16 ? 64 : min(512, PAGODA_IDLE_NS));
@@ -491,8 +491,8 @@ __device__ void comp_forwarder(MtbShared& S, const MkParams& p, uint32_t f)
  * warp of a TB returns its shmem granules and barrier ID through the mailbox
  * (markSMForDealloc), the last warp of the task posts its completion record,
  * every warp returns itself. */
-__device__ __forceinline__ void run_task(MtbShared& S, char* smem_base, const MkParams& p, int mtb, int w,
-                                         uint32_t resident)
+__device__ __forceinline__ void run_task(MtbShared& S, SchedGroup& G, char* smem_base, const MkParams& p, int mtb,
+                                         int vmtb, int w, uint32_t resident)
 {
     const uint32_t lane = threadIdx.x & 31u;
     const WarpSlot& s = S.wt[w];   /* read from shared memory when needed */
@@ -506,7 +506,7 @@ __device__ __forceinline__ void run_task(MtbShared& S, char* smem_base, const Mk
     uint64_t tp = pf_now();
     if (!run_body(t.func_id, env, t.args) && lane == 0) atomicOr(&p.dctl->error, PAGODA_DEVERR_BAD_FUNC);
     __syncwarp();
-    pf_add(S, kPfBody, tp, true);
+    pf_add(G, kPfBody, tp, true);
     if (p.life && lane == 0)
         atomicMax(reinterpret_cast<unsigned long long*>(life_slot(p, s.task_id, kLifeEnd)),
                   (unsigned long long)globaltimer_ns());
@@ -528,27 +528,27 @@ __device__ __forceinline__ void run_task(MtbShared& S, char* smem_base, const Mk
             if (i < p.trace_cap) {
                 uint32_t smid;
                 asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
-                ExecRecord r{s.task_id, s.tb, (uint16_t)smid, (uint16_t)mtb, (uint16_t)w, t0, globaltimer_ns()};
+                ExecRecord r{s.task_id, s.tb, (uint16_t)smid, (uint16_t)vmtb, (uint16_t)w, t0, globaltimer_ns()};
                 p.exec_trace[((size_t)mtb * 32 + w) * p.trace_cap + i] = r;
             }
             *cnt = i + 1;
         }
-        if (atomicSub(&S.tb_warps_left[s.tbslot], 1u) == 1u) atomicOr(&S.mb_tbs, 1u << s.tbslot);
+        if (atomicSub(&S.tb_warps_left[s.tbslot], 1u) == 1u) atomicOr(&G.mb_tbs, 1u << s.tbslot);
         if (atomicSub(&S.task_warps_left[s.task], 1u) == 1u) {
             /* last warp of the task (Alg. 1 L41-42): its completion record is pending */
             life_stamp(p, s.task_id, kLifeDone);
-            atomicOr(&S.comp_pending, 1u << s.task);
+            atomicOr(&G.comp_pending, 1u << s.task);
             __threadfence_block();   /* pending bit before the poster-flag attempt */
             last = 1;
         }
     }
-    pf_add(S, kPfFence, tp, true);
+    pf_add(G, kPfFence, tp, true);
     tp = pf_now();
-    if (!PAGODA_HOLDER_POSTS && __shfl_sync(0xffffffffu, last, 0)) post_completions(S, p);
-    pf_add(S, kPfPost, tp, true);
+    if (!PAGODA_HOLDER_POSTS && __shfl_sync(0xffffffffu, last, 0)) post_completions(S, G, p);
+    pf_add(G, kPfPost, tp, true);
     if (lane == 0) {
         __threadfence_block();   /* TB / task frees are visible before the warp frees itself */
-        atomicOr(&S.mb_warps, 1u << w);
+        atomicOr(&G.mb_warps, 1u << w);
         __threadfence_block();   /* ... and the warp's free bit before its attempt at the token */
     }
     __syncwarp();
@@ -576,7 +576,7 @@ __device__ void host_poster(MtbShared& S, const MkParams& p)
             st_relaxed_sys32(&p.hctl->error, err);
             last_err = err;
         }
-        if (done && exited >= (uint32_t)p.n_mtb) break;
+        if (done && exited >= p.n_exit) break;
         __nanosleep(256);
     }
 }
@@ -928,7 +928,12 @@ struct Sched {
     uint32_t est_w;      /* warps of the last loaded task (0 = none yet) */
     uint32_t seq;        /* ledger clock */
     uint32_t holder_bit; /* the warp holding the scheduler token (this warp) */
+    uint32_t g;          /* scheduling group (S.grp[g]) */
+    uint32_t rb, rm;     /* the group's slice of the FIFO arrays pend / pend_ticket: base, size - 1 */
+    int      vmtb;       /* ledger id of the group: mtb * n_grp + g */
 };
+/* FIFO position x of the group's slice of pend / pend_ticket */
+__device__ __forceinline__ uint32_t fq(const Sched& st, uint32_t x) { return st.rb + (x & st.rm); }
 
 __device__ __forceinline__ uint32_t nth_set_bit(uint32_t mask, uint32_t n)
 {   /* 0-based n-th set bit position (mask must have > n bits) */
@@ -996,7 +1001,7 @@ __device__ bool sched_place(MtbShared& S, Sched& st, const MkParams& p, int mtb,
             S.tb_task[tbs] = id;
             S.tb_idx[tbs] = (uint16_t)(tb0 + j);
         }
-        trace_ev(p, mtb, st.seq, 1, id, (uint16_t)(tb0 + j), m, (uint16_t)off, (uint16_t)gtb, (uint8_t)bar);
+        trace_ev(p, st.vmtb, st.seq, 1, id, (uint16_t)(tb0 + j), m, (uint16_t)off, (uint16_t)gtb, (uint8_t)bar);
         if ((m >> lane) & 1u) {   /* Alg. 2 L9-12: lane l fills warp l's WarpTable slot */
             WarpSlot ws;
             ws.smem_off = p.arena_offset + off * PAGODA_GRANULE;
@@ -1038,7 +1043,7 @@ __device__ int sched_place_run(MtbShared& S, Sched& st, const MkParams& p, int m
     const uint32_t navail = min(st.pl - st.ph, 32u);
     uint32_t key = 0xFFFFFFFFu, slot = 0;
     if (lane < navail) {
-        slot = S.pend[(st.ph + lane) & 31u];
+        slot = S.pend[fq(st, st.ph + lane)];
         const TaskEntry& e = S.tasks[slot];
         const uint32_t g = (e.shmem_bytes + PAGODA_GRANULE - 1u) / PAGODA_GRANULE;
         if (e.n_tb == 1 && !(e.flags & kEntryGroup))
@@ -1107,7 +1112,7 @@ __device__ int sched_place_run(MtbShared& S, Sched& st, const MkParams& p, int m
     if (p.trace_cap) {   /* the ledger: one ALLOC per task, in FIFO order */
         for (uint32_t i = 0; i < fit; i++) {
             const uint32_t mi = __ballot_sync(0xffffffffu, ((sel >> lane) & 1u) && ti == i);
-            trace_ev(p, mtb, st.seq, 1, __shfl_sync(0xffffffffu, id, i), 0, mi,
+            trace_ev(p, st.vmtb, st.seq, 1, __shfl_sync(0xffffffffu, id, i), 0, mi,
                      (uint16_t)__shfl_sync(0xffffffffu, off, i), (uint16_t)gtb,
                      (uint8_t)__shfl_sync(0xffffffffu, bar, i));
         }
@@ -1141,7 +1146,7 @@ __device__ int sched_claim(MtbShared& S, Sched& st, const MkParams& p)
 {
     const uint32_t lane = threadIdx.x & 31u;
     const uint32_t queued = st.pt - st.ph;
-    const uint32_t cap = 32u - queued;
+    const uint32_t cap = st.rm + 1u - queued;
     uint32_t want;
     if (st.est_w == 0) want = queued == 0 ? 1u : 0u;
     else {   /* what fits now, plus one task of lookahead so the next is loaded when warps free */
@@ -1160,7 +1165,7 @@ __device__ int sched_claim(MtbShared& S, Sched& st, const MkParams& p)
     head = __shfl_sync(0xffffffffu, head, 0);
     tail = __shfl_sync(0xffffffffu, tail, 0);
     if (head >= tail) {
-        sc_add(S, kScClaimEmpty, 1);
+        sc_add(S.grp[st.g], kScClaimEmpty, 1);
         return 0;
     }
     const uint64_t backlog = tail - head;
@@ -1169,8 +1174,8 @@ __device__ int sched_claim(MtbShared& S, Sched& st, const MkParams& p)
          * spread_ns after its last claim), so tasks go to the least-loaded MTBs first */
         const uint32_t busy = (uint32_t)__popc(st.exec_mask & ~st.free_w);
         const uint64_t now = globaltimer_ns();
-        if (busy && now < S.claim_after) return 0;
-        if (lane == 0) S.claim_after = now + (uint64_t)(busy + 4u) * p.spread_ns / 4u;
+        if (busy && now < S.grp[st.g].claim_after) return 0;
+        if (lane == 0) S.grp[st.g].claim_after = now + (uint64_t)(busy + 4u) * p.spread_ns / 4u;
     }
 #if PAGODA_CLAIM_FAIR
     /* at most a fair share of the backlog per claim: spreads consecutive tasks over MTBs when
@@ -1183,8 +1188,8 @@ __device__ int sched_claim(MtbShared& S, Sched& st, const MkParams& p)
     unsigned long long t0 = 0;
     if (lane == 0) t0 = atomicAdd(reinterpret_cast<unsigned long long*>(&p.dctl->head), (unsigned long long)k);
     t0 = __shfl_sync(0xffffffffu, t0, 0);
-    if (lane < k) S.pend_ticket[(st.pt + lane) & 31u] = t0 + lane;
-    sc_add(S, kScTickets, k);
+    if (lane < k) S.pend_ticket[fq(st, st.pt + lane)] = t0 + lane;
+    sc_add(S.grp[st.g], kScTickets, k);
     st.pt += k;
     __syncwarp();
     return (int)k;
@@ -1201,13 +1206,13 @@ __device__ int sched_load(MtbShared& S, Sched& st, const MkParams& p)
     if (n == 0) return 0;
     bool ready = false;
     if (lane < n) {
-        const uint64_t t = S.pend_ticket[(st.pl + lane) & 31u];
+        const uint64_t t = S.pend_ticket[fq(st, st.pl + lane)];
         ready = ld_acquire_gpu32(&p.dseq[t & p.ring_mask]) == (uint32_t)(t + 1);
     }
     const uint32_t nr = __ballot_sync(0xffffffffu, !ready);
     const uint32_t r = nr ? (uint32_t)__ffs(nr) - 1u : 32u;   /* leading published tickets */
     if (r == 0) {
-        sc_add(S, kScLoadNotReady, 1);
+        sc_add(S.grp[st.g], kScLoadNotReady, 1);
         return 0;
     }
     return sched_copy(S, st, p, r);
@@ -1218,7 +1223,7 @@ __device__ int sched_load(MtbShared& S, Sched& st, const MkParams& p)
 __device__ int sched_copy(MtbShared& S, Sched& st, const MkParams& p, uint32_t r)
 {
     const uint32_t lane = threadIdx.x & 31u;
-    const uint64_t t = lane < r ? S.pend_ticket[(st.pl + lane) & 31u] : 0;
+    const uint64_t t = lane < r ? S.pend_ticket[fq(st, st.pl + lane)] : 0;
 #if PAGODA_FAST_LOAD
     /* 4 lanes per cell, one 16-byte relaxed load each: up to 8 cells per warp instruction, all in
      * flight together (one L2 round trip; the sequence words' acquires in sched_load ordered these
@@ -1227,7 +1232,7 @@ __device__ int sched_copy(MtbShared& S, Sched& st, const MkParams& p, uint32_t r
      * words (STS, which wait for the data) precede the hand-back in program order. */
     for (uint32_t c = lane; c < r * 4u; c += 32u) {
         const uint32_t i = c >> 2, q = c & 3u;
-        const uint64_t ti = S.pend_ticket[(st.pl + i) & 31u];
+        const uint64_t ti = S.pend_ticket[fq(st, st.pl + i)];
         int4 v;
         asm volatile("ld.relaxed.gpu.global.v4.s32 {%0,%1,%2,%3}, [%4];"
                      : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
@@ -1239,7 +1244,7 @@ __device__ int sched_copy(MtbShared& S, Sched& st, const MkParams& p, uint32_t r
     uint32_t used = 0;
     if (lane < r) {
         const uint32_t slot = nth_set_bit(st.free_task, lane);
-        S.pend[(st.pl + lane) & 31u] = (uint8_t)slot;
+        S.pend[fq(st, st.pl + lane)] = (uint8_t)slot;
         st_relaxed_gpu32(&p.dseq[t & p.ring_mask], (uint32_t)(t + (uint64_t)p.ring_mask + 1));
         if (p.life && !(S.tasks[slot].flags & kEntryGroup)) life_stamp(p, S.tasks[slot].id, kLifeLoad);
         used = 1u << slot;
@@ -1261,7 +1266,7 @@ __device__ int sched_copy(MtbShared& S, Sched& st, const MkParams& p, uint32_t r
                          : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(src + q) : "memory");
             dst[q] = v;
         }
-        S.pend[(st.pl + lane) & 31u] = (uint8_t)slot;
+        S.pend[fq(st, st.pl + lane)] = (uint8_t)slot;
         st_relaxed_gpu32(&p.dseq[t & p.ring_mask], (uint32_t)(t + (uint64_t)p.ring_mask + 1));
         if (p.life && !(S.tasks[slot].flags & kEntryGroup)) life_stamp(p, S.tasks[slot].id, kLifeLoad);
         used = 1u << slot;
@@ -1269,7 +1274,7 @@ __device__ int sched_copy(MtbShared& S, Sched& st, const MkParams& p, uint32_t r
 #else
     for (uint32_t c = lane; c < r * 4u; c += 32u) {   /* 4 lanes per cell, coalesced */
         const uint32_t i = c >> 2;
-        const uint64_t ti = S.pend_ticket[(st.pl + i) & 31u];
+        const uint64_t ti = S.pend_ticket[fq(st, st.pl + i)];
         const int4 v = __ldcg(reinterpret_cast<const int4*>(p.dring + (ti & p.ring_mask)) + (c & 3u));
         reinterpret_cast<int4*>(&S.tasks[nth_set_bit(st.free_task, i)])[c & 3u] = v;
     }
@@ -1277,7 +1282,7 @@ __device__ int sched_copy(MtbShared& S, Sched& st, const MkParams& p, uint32_t r
     uint32_t used = 0;
     if (lane < r) {
         const uint32_t slot = nth_set_bit(st.free_task, lane);
-        S.pend[(st.pl + lane) & 31u] = (uint8_t)slot;
+        S.pend[fq(st, st.pl + lane)] = (uint8_t)slot;
         st_release_gpu32(&p.dseq[t & p.ring_mask], (uint32_t)(t + (uint64_t)p.ring_mask + 1));
         used = 1u << slot;
     }
@@ -1286,7 +1291,7 @@ __device__ int sched_copy(MtbShared& S, Sched& st, const MkParams& p, uint32_t r
     st.free_task &= ~used;
     st.pl += r;
     __syncwarp();
-    const TaskEntry& last = S.tasks[S.pend[(st.pl - 1) & 31u]];
+    const TaskEntry& last = S.tasks[S.pend[fq(st, st.pl - 1)]];
     st.est_w = (uint32_t)last.warps_tb * last.n_tb;
     return (int)r;
 }
@@ -1313,10 +1318,10 @@ __device__ int sched_claim_check(MtbShared& S, Sched& st, const MkParams& p)
             want = want > queued ? want - queued : 0u;
             if (queued && want < (uint32_t)PAGODA_CLAIM_MIN) want = 0;
         }
-        const uint32_t est = S.backlog_est;
+        const uint32_t est = S.grp[st.g].backlog_est;
         if (est == 0) want = min(want, st.pt == st.pl ? 1u : 0u);   /* a standing reservation */
         else want = min(want, max((uint32_t)PAGODA_CLAIM_SMALL, min(est / (uint32_t)p.n_mtb, 32u)));
-        want = min(want, 32u - queued);
+        want = min(want, st.rm + 1u - queued);
     }
     const uint32_t n = min(st.pt - st.pl, min((uint32_t)__popc(st.free_task), 29u));
     uint64_t v = 0;
@@ -1328,7 +1333,7 @@ __device__ int sched_claim_check(MtbShared& S, Sched& st, const MkParams& p)
     } else if (lane == 2) {
         v = ld_relaxed_gpu(&p.dctl->head);
     } else if (lane - 3u < n) {
-        const uint64_t t = S.pend_ticket[(st.pl + lane - 3u) & 31u];
+        const uint64_t t = S.pend_ticket[fq(st, st.pl + lane - 3u)];
         ready = ld_acquire_gpu32(&p.dseq[t & p.ring_mask]) == (uint32_t)(t + 1);
     }
     const uint64_t old = __shfl_sync(0xffffffffu, v, 0);
@@ -1337,11 +1342,11 @@ __device__ int sched_claim_check(MtbShared& S, Sched& st, const MkParams& p)
     const uint32_t rb = __ballot_sync(0xffffffffu, ready) >> 3;
     const uint32_t r = min((uint32_t)__ffs(~rb) - 1u, n);   /* leading published tickets */
     if (want) head = max(head, old + want);
-    if (lane < want) S.pend_ticket[(st.pt + lane) & 31u] = old + lane;
-    if (lane == 0) S.backlog_est = (uint32_t)min(tail > head ? tail - head : 0ull, 0xffffffffull);
-    sc_add(S, kScTickets, want);
-    if (want && old >= tail) sc_add(S, kScClaimEmpty, 1);
-    if (n && r == 0) sc_add(S, kScLoadNotReady, 1);
+    if (lane < want) S.pend_ticket[fq(st, st.pt + lane)] = old + lane;
+    if (lane == 0) S.grp[st.g].backlog_est = (uint32_t)min(tail > head ? tail - head : 0ull, 0xffffffffull);
+    sc_add(S.grp[st.g], kScTickets, want);
+    if (want && old >= tail) sc_add(S.grp[st.g], kScClaimEmpty, 1);
+    if (n && r == 0) sc_add(S.grp[st.g], kScLoadNotReady, 1);
     st.pt += want;
     __syncwarp();
     return (int)r;
@@ -1360,54 +1365,62 @@ __device__ int sched_claim_check(MtbShared& S, Sched& st, const MkParams& p)
 __device__ __forceinline__ void sst_save(MtbShared& S, const Sched& st)
 {
     const uint32_t lane = threadIdx.x & 31u;
-    S.sst_fg[lane] = st.fg;
+    SchedGroup& G = S.grp[st.g];
+    G.fg[lane] = st.fg;
     if (lane == 0) {
-        S.sst_free_w = st.free_w;
-        S.sst_free_task = st.free_task;
-        S.sst_free_tbs = st.free_tbs;
-        S.sst_free_bar = st.free_bar;
-        S.sst_ph = st.ph;
-        S.sst_pl = st.pl;
-        S.sst_pt = st.pt;
-        S.sst_est_w = st.est_w;
-        S.sst_seq = st.seq;
+        G.free_w = st.free_w;
+        G.free_task = st.free_task;
+        G.free_tbs = st.free_tbs;
+        G.free_bar = st.free_bar;
+        G.ph = st.ph;
+        G.pl = st.pl;
+        G.pt = st.pt;
+        G.est_w = st.est_w;
+        G.seq = st.seq;
     }
     __syncwarp();
 }
 
-__device__ __forceinline__ void sst_load(MtbShared& S, Sched& st, uint32_t exec_mask)
+/* the holder state of group g (the caller's warp now holds g's token) */
+__device__ __forceinline__ void sst_load(MtbShared& S, Sched& st, uint32_t exec_mask, uint32_t g, const MkParams& p,
+                                         int mtb)
 {
     __syncwarp();
-    st.fg = S.sst_fg[threadIdx.x & 31u];
-    st.free_w = S.sst_free_w;
-    st.free_task = S.sst_free_task;
-    st.free_tbs = S.sst_free_tbs;
-    st.free_bar = S.sst_free_bar;
-    st.ph = S.sst_ph;
-    st.pl = S.sst_pl;
-    st.pt = S.sst_pt;
-    st.est_w = S.sst_est_w;
-    st.seq = S.sst_seq;
+    const SchedGroup& G = S.grp[g];
+    st.fg = G.fg[threadIdx.x & 31u];
+    st.free_w = G.free_w;
+    st.free_task = G.free_task;
+    st.free_tbs = G.free_tbs;
+    st.free_bar = G.free_bar;
+    st.ph = G.ph;
+    st.pl = G.pl;
+    st.pt = G.pt;
+    st.est_w = G.est_w;
+    st.seq = G.seq;
     st.exec_mask = exec_mask;
     st.holder_bit = 1u << (threadIdx.x >> 5);
+    st.g = g;
+    st.rm = 32u / p.n_grp - 1u;
+    st.rb = g * (st.rm + 1u);
+    st.vmtb = mtb * (int)p.n_grp + (int)g;
 }
 
-__device__ __forceinline__ bool token_try(MtbShared& S)
+__device__ __forceinline__ bool token_try(SchedGroup& G)
 {
     uint32_t got = 0;
     if ((threadIdx.x & 31u) == 0) {
-        got = atomicCAS(&S.token, 0u, 1u) == 0u;
+        got = atomicCAS(&G.token, 0u, 1u) == 0u;
         __threadfence_block();
     }
     return __shfl_sync(0xffffffffu, got, 0) != 0;
 }
 
-__device__ __forceinline__ void token_release(MtbShared& S)
+__device__ __forceinline__ void token_release(SchedGroup& G)
 {
     __syncwarp();
     if ((threadIdx.x & 31u) == 0) {
         __threadfence_block();
-        atomicExch(&S.token, 0u);
+        atomicExch(&G.token, 0u);
         __threadfence_block();
     }
     __syncwarp();
@@ -1418,11 +1431,12 @@ __device__ bool sched_fold(MtbShared& S, Sched& st, const MkParams& p, int mtb)
 {
     const uint32_t lane = threadIdx.x & 31u;
     uint32_t mw = 0, mt = 0, mk = 0;
+    SchedGroup& G = S.grp[st.g];
     if (lane == 0) {
-        if (*(volatile uint32_t*)&S.mb_warps) mw = atomicExch(&S.mb_warps, 0u);
+        if (*(volatile uint32_t*)&G.mb_warps) mw = atomicExch(&G.mb_warps, 0u);
         __threadfence_block();
-        if (*(volatile uint32_t*)&S.mb_tbs) mt = atomicExch(&S.mb_tbs, 0u);
-        if (*(volatile uint32_t*)&S.mb_tasks) mk = atomicExch(&S.mb_tasks, 0u);
+        if (*(volatile uint32_t*)&G.mb_tbs) mt = atomicExch(&G.mb_tbs, 0u);
+        if (*(volatile uint32_t*)&G.mb_tasks) mk = atomicExch(&G.mb_tasks, 0u);
     }
     mw = __shfl_sync(0xffffffffu, mw, 0);
     mt = __shfl_sync(0xffffffffu, mt, 0);
@@ -1435,12 +1449,12 @@ __device__ bool sched_fold(MtbShared& S, Sched& st, const MkParams& p, int mtb)
         if (bar) st.free_bar |= 1u << bar;
         st.free_tbs |= 1u << tbs;
         if (p.trace_cap)
-            trace_ev(p, mtb, st.seq, 3, S.tb_task[tbs], S.tb_idx[tbs], 0, (uint16_t)goff, (uint16_t)glen, (uint8_t)bar);
+            trace_ev(p, st.vmtb, st.seq, 3, S.tb_task[tbs], S.tb_idx[tbs], 0, (uint16_t)goff, (uint16_t)glen, (uint8_t)bar);
     }
     if (p.trace_cap) {
         for (uint32_t b = mw; b; b &= b - 1u) {
             const uint32_t w = __ffs(b) - 1;
-            trace_ev(p, mtb, st.seq, 2, S.wt[w].task_id, S.wt[w].tb, 1u << w, 0, 0, 0);
+            trace_ev(p, st.vmtb, st.seq, 2, S.wt[w].task_id, S.wt[w].tb, 1u << w, 0, 0, 0);
         }
     }
     st.free_w |= mw;
@@ -1455,14 +1469,14 @@ __device__ bool sched_round(MtbShared& S, Sched& st, const MkParams& p, int mtb,
     const uint32_t lane = threadIdx.x & 31u;
     uint64_t t0 = pf_now();
     bool progress = sched_fold(S, st, p, mtb);
-    pf_add(S, kPfFold, t0, true);
+    pf_add(S.grp[st.g], kPfFold, t0, true);
     /* completion records of the tasks whose last warp finished (a warp marks comp_pending before
      * it frees itself, so every task of a folded warp is in it): one fence and one queue
      * reservation for the whole batch, off the executors' path */
-    if (PAGODA_HOLDER_POSTS && *(volatile uint32_t*)&S.comp_pending) {
+    if (PAGODA_HOLDER_POSTS && *(volatile uint32_t*)&S.grp[st.g].comp_pending) {
         t0 = pf_now();
-        post_completions(S, p);
-        pf_add(S, kPfPost, t0, true);
+        post_completions(S, S.grp[st.g], p);
+        pf_add(S.grp[st.g], kPfPost, t0, true);
         progress = true;
     }
 #if PAGODA_FUSED_CLAIM
@@ -1471,50 +1485,51 @@ __device__ bool sched_round(MtbShared& S, Sched& st, const MkParams& p, int mtb,
         const uint32_t pt0 = st.pt;
         const int r = sched_claim_check(S, st, p);
         if (st.pt != pt0) progress = true;
-        pf_add(S, kPfClaim, t0, true);
+        pf_add(S.grp[st.g], kPfClaim, t0, true);
         t0 = pf_now();
         if (r > 0 && sched_copy(S, st, p, (uint32_t)r) > 0) progress = true;
-        pf_add(S, kPfLoad, t0, true);
+        pf_add(S.grp[st.g], kPfLoad, t0, true);
     }
 #else
     if (PAGODA_CLAIM_FIRST) {
         t0 = pf_now();
         if (!S.no_tickets && sched_claim(S, st, p) > 0) progress = true;
-        pf_add(S, kPfClaim, t0, true);
+        pf_add(S.grp[st.g], kPfClaim, t0, true);
     }
     t0 = pf_now();
     if (st.pl != st.pt && sched_load(S, st, p) > 0) progress = true;
-    pf_add(S, kPfLoad, t0, true);
+    pf_add(S.grp[st.g], kPfLoad, t0, true);
 #endif
     t0 = pf_now();
     while (st.ph != st.pl) {
         const int k = PAGODA_BATCH_PLACE ? sched_place_run(S, st, p, mtb) : -1;
         if (k > 0) {   /* a run of identical single-TB tasks placed in one pass */
-            sc_add(S, kScPlaced, (uint32_t)k);
+            sc_add(S.grp[st.g], kScPlaced, (uint32_t)k);
             st.ph += (uint32_t)k;
             progress = true;
             continue;
         }
-        if (k == 0 || !sched_place(S, st, p, mtb, S.pend[st.ph & 31u])) {
-            sc_add(S, kScNoFit, 1);
+        if (k == 0 || !sched_place(S, st, p, mtb, S.pend[fq(st, st.ph)])) {
+            sc_add(S.grp[st.g], kScNoFit, 1);
             break;
         }
-        sc_add(S, kScPlaced, 1);
+        sc_add(S.grp[st.g], kScPlaced, 1);
         st.ph++;
         progress = true;
     }
-    pf_add(S, kPfPlace, t0, true);
+    pf_add(S.grp[st.g], kPfPlace, t0, true);
     /* MTB 0 (the I/O MTB: ingest, host stores) and the MTB sharing its SM take no tickets
      * unless MTB 0 is the only MTB (validation then caps every task to its capacity) */
     if (!PAGODA_CLAIM_FIRST && !PAGODA_FUSED_CLAIM) {
         t0 = pf_now();
         if (!S.no_tickets && sched_claim(S, st, p) > 0) progress = true;
-        pf_add(S, kPfClaim, t0, true);
+        pf_add(S.grp[st.g], kPfClaim, t0, true);
     }
     exit = false;
-    sc_add(S, kScRounds, 1);
-    if (progress) sc_add(S, kScProgress, 1);
-    if (!progress && st.free_w == st.exec_mask && st.ph == st.pl && *(volatile uint32_t*)&S.comp_pending == 0u) {
+    sc_add(S.grp[st.g], kScRounds, 1);
+    if (progress) sc_add(S.grp[st.g], kScProgress, 1);
+    if (!progress && st.free_w == st.exec_mask && st.ph == st.pl &&
+        *(volatile uint32_t*)&S.grp[st.g].comp_pending == 0u) {
         uint32_t stop = 0;
         if (lane == 0) stop = ld_acquire_gpu32(&p.dctl->stop);
         stop = __shfl_sync(0xffffffffu, stop, 0);
@@ -1524,7 +1539,7 @@ __device__ bool sched_round(MtbShared& S, Sched& st, const MkParams& p, int mtb,
             if (lane == 0) tail = ld_acquire_gpu(&p.dctl->tail);
             tail = __shfl_sync(0xffffffffu, tail, 0);
             /* after stop the tail is final: tickets at or past it are void */
-            exit = st.pl == st.pt || S.pend_ticket[st.pl & 31u] >= tail;
+            exit = st.pl == st.pt || S.pend_ticket[fq(st, st.pl)] >= tail;
         }
     }
     return progress;
@@ -1542,7 +1557,7 @@ __device__ void sched_handoff(MtbShared& S, Sched& st, const MkParams& p, int mt
         if (st.free_w) {
             const uint32_t h = __ffs(st.free_w) - 1;
             sst_save(S, st);
-            sc_add(S, kScHandoffs, 1);
+            sc_add(S.grp[st.g], kScHandoffs, 1);
             if (lane == h) {
                 S.wt[h].task = SLOT_SCHED;
                 mbar_arrive(&S.exec_bar[h]);   /* release: the saved state is visible to h */
@@ -1551,12 +1566,13 @@ __device__ void sched_handoff(MtbShared& S, Sched& st, const MkParams& p, int mt
             return;
         }
         sst_save(S, st);
-        token_release(S);
+        SchedGroup& G = S.grp[st.g];
+        token_release(G);
         uint32_t pending = 0;
-        if (lane == 0) pending = *(volatile uint32_t*)&S.mb_warps;
+        if (lane == 0) pending = *(volatile uint32_t*)&G.mb_warps;
         pending = __shfl_sync(0xffffffffu, pending, 0);
-        if (!pending || !token_try(S)) return;
-        sst_load(S, st, st.exec_mask);
+        if (!pending || !token_try(G)) return;
+        sst_load(S, st, st.exec_mask, st.g, p, mtb);
     }
 }
 
@@ -1564,11 +1580,12 @@ __device__ void sched_handoff(MtbShared& S, Sched& st, const MkParams& p, int mt
  * dispatched itself (hands the token on) or the session ends (returns true).
  * The scheduler state lives only here (loaded from / saved to shared memory),
  * so no register holds it while the warp runs task bodies. */
-__device__ __noinline__ bool holder_phase(MtbShared& S, const MkParams& p, int mtb, int w, uint32_t exec_mask)
+__device__ __noinline__ bool holder_phase(MtbShared& S, const MkParams& p, int mtb, int w, uint32_t exec_mask,
+                                          uint32_t g)
 {
     const uint32_t lane = threadIdx.x & 31u;
     Sched st;
-    sst_load(S, st, exec_mask);
+    sst_load(S, st, exec_mask, g, p, mtb);
     uint32_t backoff = 0;
     for (;;) {
         bool exit = false;
@@ -1579,12 +1596,13 @@ __device__ __noinline__ bool holder_phase(MtbShared& S, const MkParams& p, int m
                 mbar_arrive(&S.exec_bar[lane]);
             }
             if (lane == 0) {
-                __threadfence();   /* this MTB's completion-queue reservations precede its exit count */
+                __threadfence();   /* this group's completion-queue reservations precede its exit count */
                 atomicAdd(&p.dctl->exited, 1u);
+                const SchedGroup& G = S.grp[g];
                 for (int i = 0; i < 8; i++)
-                    atomicAdd(&p.dctl->ctr[PAGODA_CTR_SCHED_ROUNDS + i], (unsigned long long)S.sctr[i]);
+                    atomicAdd(&p.dctl->ctr[PAGODA_CTR_SCHED_ROUNDS + i], (unsigned long long)G.sctr[i]);
                 if (PAGODA_PROFILE)   /* (executors still finishing their last task may add a little after) */
-                    for (int i = 0; i < 8; i++) atomicAdd(&p.dctl->ctr[PAGODA_CTR_SCHED_NS_FOLD + i], S.sprof[i]);
+                    for (int i = 0; i < 8; i++) atomicAdd(&p.dctl->ctr[PAGODA_CTR_SCHED_NS_FOLD + i], G.sprof[i]);
             }
             return true;
         }
@@ -1596,7 +1614,7 @@ __device__ __noinline__ bool holder_phase(MtbShared& S, const MkParams& p, int m
                 backoff = (st.ph != st.pt) ? 32u : (backoff ? min(backoff * 2u, (uint32_t)PAGODA_IDLE_NS) : 32u);
                 const uint64_t t0 = pf_now();
                 __nanosleep(backoff);
-                pf_add(S, kPfSleep, t0, true);
+                pf_add(S.grp[st.g], kPfSleep, t0, true);
             }
             continue;
         }
@@ -1605,14 +1623,17 @@ __device__ __noinline__ bool holder_phase(MtbShared& S, const MkParams& p, int m
     }
 }
 
-/* Every worker warp runs this loop (warps 0..exec_warps-1; MTB 0's last warp ingests). */
+/* Every worker warp runs this loop (warps 0..exec_warps-1; MTB 0's last warp ingests); exec_mask is
+ * the worker warps of its scheduling group g. */
 __device__ void worker(MtbShared& S, char* smem_base, const MkParams& p, int mtb, int w, uint32_t resident,
-                       uint32_t exec_mask, bool holder)
+                       uint32_t exec_mask, bool holder, uint32_t g)
 {
     uint32_t phase = 0;
+    SchedGroup& G = S.grp[g];
+    const int vmtb = mtb * (int)p.n_grp + (int)g;
     for (;;) {
         if (holder) {
-            if (holder_phase(S, p, mtb, w, exec_mask)) return;
+            if (holder_phase(S, p, mtb, w, exec_mask, g)) return;
             holder = false;
         }
         exec_wait(phase);   /* mbar_wait(&S.exec_bar[w], phase) without a live address register */
@@ -1623,8 +1644,8 @@ __device__ void worker(MtbShared& S, char* smem_base, const MkParams& p, int mtb
             holder = true;
             continue;
         }
-        run_task(S, smem_base, p, mtb, w, resident);
-        holder = token_try(S);
+        run_task(S, G, smem_base, p, mtb, vmtb, w, resident);
+        holder = token_try(G);
     }
 }
 
@@ -1680,9 +1701,14 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) master_kernel(MkParams p
             atomicOr(&p.dctl->error, PAGODA_DEVERR_LAYOUT);   /* bodies fall back to per-task tables */
         }
     }
-    /* worker warps 0..exec_warps-1 (MTB 0: minus the ingest warp) */
+    /* worker warps: the first exec_warps / n_grp warps of each group's range (MTB 0: minus the ingest warp) */
     const int ew = min(p.exec_warps, nw);
-    uint32_t exec_mask = ew >= 32 ? 0xffffffffu : ((1u << ew) - 1u);
+    const uint32_t n_grp = p.n_grp, gw = (uint32_t)nw / n_grp, gs = 32u / n_grp;
+    uint32_t exec_mask = 0;
+    for (uint32_t g = 0; g < n_grp; g++) {
+        const uint32_t per = min((uint32_t)ew / n_grp, gw);
+        exec_mask |= (per >= 32u ? 0xffffffffu : ((1u << per) - 1u)) << (g * gw);
+    }
     if (mtb == 0) exec_mask &= ~(1u << ingest_loader_warp(nw));
     if (io)   /* the I/O roles: loader (31), host poster (30), forwarder (28), publishers (29, 27, ...) */
     {
@@ -1690,7 +1716,13 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) master_kernel(MkParams p
         for (uint32_t i = 0; i < p.n_fwd; i++) exec_mask &= ~(1u << forwarder_warp_i(i, nw));
         for (uint32_t i = 0; i < kIngestPublishers; i++) exec_mask &= ~(1u << ingest_publisher_warp(i, nw));
     }
-    const int first = __ffs(exec_mask) - 1;
+    /* scheduling groups: group g owns warps [g nw/G, (g+1) nw/G), task slots and TB records
+     * [32g/G, 32(g+1)/G), named barriers 1..7 / 8..15 (G = 2) or 1..15, and arena granules
+     * [A g/G, A (g+1)/G) */
+    const uint32_t my_g = (uint32_t)warp / gw;
+    const uint32_t gmask_w = (gw >= 32u ? 0xffffffffu : ((1u << gw) - 1u)) << (my_g * gw);
+    const uint32_t my_exec = exec_mask & gmask_w;
+    const int first = __ffs(my_exec) - 1;
     if (warp == 0) {
         mbar_init(&S.exec_bar[lane], 1);
         mbar_init(&S.stage_bar[lane], 1);
@@ -1700,26 +1732,39 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) master_kernel(MkParams p
             mbar_init(&S.ingest_empty[lane], 1);
         }
         for (uint32_t i = lane; i < kIngestFinSlots; i += 32u) S.ing_fin[i] = 0;
-        /* initial scheduler state, owned by the first worker (it starts with the token) */
-        S.sst_fg[lane] = bm_range_bits(0, (uint32_t)arena_granules, lane);
+        /* initial scheduler state of each group, owned by its first worker (it starts with the token) */
+        for (uint32_t g = 0; g < n_grp; g++) {
+            SchedGroup& G = S.grp[g];
+            const uint32_t g0 = (uint32_t)arena_granules * g / n_grp, g1 = (uint32_t)arena_granules * (g + 1) / n_grp;
+            G.fg[lane] = bm_range_bits(g0, g1 - g0, lane);
+            if (lane == 0) {
+                const uint32_t gm = (gw >= 32u ? 0xffffffffu : ((1u << gw) - 1u)) << (g * gw);
+                const uint32_t sm = (gs >= 32u ? 0xffffffffu : ((1u << gs) - 1u)) << (g * gs);
+                G.mb_warps = G.mb_tbs = G.mb_tasks = 0;
+                G.free_w = exec_mask & gm;
+                G.free_task = sm;
+                G.free_tbs = sm;
+                /* named barriers 1..15; 0 belongs to the MTB */
+                G.free_bar = n_grp == 1 ? 0xfffeu : (g == 0 ? 0x00feu : 0xff00u);
+                G.ph = G.pl = G.pt = 0;
+                G.est_w = 0;
+                G.seq = 0;
+                G.backlog_est = 0;
+                G.claim_after = 0;
+                G.comp_pending = 0;
+                G.poster = 0;
+                /* a group without workers never runs a holder: it counts as exited now */
+                G.token = (exec_mask & gm) ? 1u : 0u;
+                if (!(exec_mask & gm)) atomicAdd(&p.dctl->exited, 1u);
+                for (int i = 0; i < 8; i++) G.sctr[i] = 0;
+                for (int i = 0; i < 8; i++) G.sprof[i] = 0;
+            }
+        }
         if (lane == 0) {
-            S.mb_warps = S.mb_tbs = S.mb_tasks = 0;
-            S.sst_free_w = exec_mask;
-            S.sst_free_task = 0xffffffffu;
-            S.sst_free_tbs = 0xffffffffu;
-            S.sst_free_bar = 0xfffeu;   /* named barriers 1..15; 0 belongs to the MTB */
-            S.sst_ph = S.sst_pl = S.sst_pt = 0;
-            S.sst_est_w = 0;
-            S.backlog_est = 0;
             S.fwd_done = 0;
-            S.claim_after = 0;
             S.dev_error = &p.dctl->error;
             S.dq_safe = *(volatile uint64_t*)&p.dctl->dq_head + kDqEntries;
-            S.sst_seq = 0;
-            S.token = 1;
-            S.comp_pending = 0;
             S.no_tickets = no_tickets;
-            S.poster = 0;
             /* where ingest resumes: the host poster must never post a smaller consumed count
              * (a spawn blocked on a ring slot would wait for it forever) */
             S.ingest_copied = *(volatile uint64_t*)&p.dctl->tail;
@@ -1727,8 +1772,6 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) master_kernel(MkParams p
             S.ing_prefix_k = 0;
             S.ing_lock = 0;
             S.ing_pubs_done = 0;
-            for (int i = 0; i < 8; i++) S.sctr[i] = 0;
-            for (int i = 0; i < 8; i++) S.sprof[i] = 0;
             asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         }
     }
@@ -1739,7 +1782,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) master_kernel(MkParams p
         ingest_publisher(S, p, ingest_stage, ingest_publisher_index(warp, nw));
     else if (io && warp == host_poster_warp(nw)) host_poster(S, p);
     else if (io && forwarder_index(warp, nw) < p.n_fwd) comp_forwarder(S, p, forwarder_index(warp, nw));
-    else if ((exec_mask >> warp) & 1u) worker(S, smem_base, p, mtb, warp, resident, exec_mask, warp == first);
+    else if ((my_exec >> warp) & 1u) worker(S, smem_base, p, mtb, warp, resident, my_exec, warp == first, my_g);
 }
 
 template __global__ void master_kernel<1, 1024>(MkParams);

@@ -115,6 +115,8 @@ struct MkParams {
     uint64_t*    life;        /* PAGODA_LIFECYCLE: [comp_mask + 1][8] stamps (pagoda_lifecycle_read), or null */
     uint32_t     n_fwd;       /* completion forwarders in MTB 0 (1..kForwarders) */
     uint32_t     spread_ns;   /* PAGODA_SPREAD: spread-first claim delay per 4 busy warps (0 = off) */
+    uint32_t     n_grp;       /* scheduling groups per MTB (1 or 2: pagoda_config.sched_groups) */
+    uint32_t     n_exit;      /* holders that exit in a session: n_mtb * n_grp */
 };
 enum { kLifePub = 0, kLifeLoad, kLifePlace, kLifeStart, kLifeEnd, kLifeDone, kLifeQueued, kLifeFwd };
 
@@ -167,6 +169,27 @@ __host__ __device__ inline uint32_t ingest_stage_entries(uint32_t smem_bytes, in
 constexpr uint32_t kStopAbort = 2;       /* HostCtl.terminate / DevCtl.stop value: abandon work and exit */
 constexpr int kMaxGranules = 1024;       /* lane-distributed bitmap: 32 lanes x 32 bits */
 
+/* A scheduling group: a share of an MTB's warps, task slots, TB records, named barriers and arena
+ * granules with its own scheduler token (self-scheduling).  An MTB has one group, or two
+ * (pagoda_config.sched_groups = 2): two token holders place tasks in parallel in one MTB, e.g.
+ * sharing the MTB-resident 3DES tables that a second MTB per SM could not hold. */
+constexpr int kMaxSchedGroups = 2;
+struct SchedGroup {
+    /* holder state parked between token holders */
+    uint32_t  fg[32];                /* granule bitmap, word l = granules [32l, 32l+32) (1 = free) */
+    uint32_t  free_w, free_task, free_tbs, free_bar;
+    uint32_t  ph, pl, pt, est_w, seq;
+    uint32_t  token;                 /* 1 while some warp of the group holds its scheduler token */
+    /* mailboxes (deferred frees): atomicOr by executors, folded by the holder */
+    uint32_t  mb_warps, mb_tbs, mb_tasks;
+    uint32_t  comp_pending;          /* task slots finished, completion record not yet posted */
+    uint32_t  poster;                /* 1 while some warp posts the group's completion records */
+    uint32_t  backlog_est;           /* ring backlog (tail - head) at the holder's last look (fused claims) */
+    uint32_t  sctr[8];               /* scheduler counters (holder-only), flushed at exit */
+    unsigned long long claim_after;  /* PAGODA_SPREAD_NS: no claim before this %globaltimer value */
+    unsigned long long sprof[8];     /* PAGODA_PROFILE: ns per phase (PAGODA_CTR_SCHED_NS_FOLD + i) */
+};
+
 /* Per-MTB control block at the start of dynamic shared memory (P:456-458:
  * "the remaining shared memory ... stores scheduling data structures"). */
 struct MtbShared {
@@ -179,23 +202,13 @@ struct MtbShared {
     uint16_t  tb_goff[32];           /* 3840 */
     uint16_t  tb_glen[32];           /* 3904 */
     uint8_t   tb_bar[32];            /* 3968 */
-    uint8_t   pend[32];              /* 4000: FIFO of claimed, not yet placed task slots */
-    uint32_t  mb_warps;              /* 4032: mailbox: warps that finished (atomicOr by executors) */
-    uint32_t  mb_tbs;                /*       mailbox: TB records whose last warp finished */
-    uint32_t  mb_tasks;              /*       mailbox: task slots whose last warp finished */
-    uint32_t  backlog_est;           /*       ring backlog (tail - head) at the holder's last look (fused claims) */
-    uint64_t  tb_task[32];           /* 4048: task id of each TB record (ledger) */
-    uint16_t  tb_idx[32];            /* 4304: TB index j of each TB record (ledger) */
-    uint64_t  pend_ticket[32];       /* 4368: claimed ring positions, FIFO (pend[] holds their slots once loaded) */
-    /* scheduler state while parked between token holders (self-scheduling) */
-    uint32_t  sst_fg[32];            /* 4624: granule bitmap, word l = granules [32l, 32l+32) */
-    uint32_t  sst_free_w, sst_free_task, sst_free_tbs, sst_free_bar;
-    uint32_t  sst_ph, sst_pl, sst_pt, sst_est_w, sst_seq;
-    uint32_t  token;                 /* 1 while some warp holds the scheduler token */
-    uint32_t  sctr[8];               /* scheduler counters (holder-only), flushed at exit */
-    uint32_t  stage_ph[32];          /* parity of each warp's staging mbarrier (TaskEnv::stage) */
-    uint32_t  poster;                /* 1 while some warp posts completion records */
+    uint8_t   pend[32];              /* 4000: FIFOs of claimed, not yet placed task slots (group g: its slice) */
+    uint64_t  tb_task[32];           /* 4032: task id of each TB record (ledger) */
+    uint16_t  tb_idx[32];            /* 4288: TB index j of each TB record (ledger) */
+    uint64_t  pend_ticket[32];       /* 4352: claimed ring positions, FIFO (pend[] holds their slots once loaded) */
+    uint32_t  stage_ph[32];          /* 4608: parity of each warp's staging mbarrier (TaskEnv::stage) */
     uint32_t  ingest_done;           /* MTB 0: the ingest warps have exited */
+    uint32_t  no_tickets;            /* this MTB runs no tasks (MTB 0 and the MTB sharing its SM) */
     uint64_t  ingest_copied;         /* MTB 0: entries published into the device ring, a prefix (host poster) */
     /* MTB 0 ingest, the rest of its control block */
     uint64_t  ingest_bar[kIngestStages];    /* stage s loaded (TMA complete_tx; n = ~0 without bytes: end) */
@@ -207,13 +220,10 @@ struct MtbShared {
     uint32_t  ing_prefix_k;                 /* stages [0, k) all published (ingest_copied is their end) */
     uint32_t  ing_lock;                     /* serialises prefix advances */
     uint32_t  ing_pubs_done;                /* publishers that saw their end marker */
-    uint32_t  comp_pending;          /* task slots finished, completion record not yet posted */
-    uint32_t  no_tickets;            /* this MTB runs no tasks (MTB 0 and the MTB sharing its SM) */
-    unsigned long long sprof[8];     /* PAGODA_PROFILE: ns per phase (PAGODA_CTR_SCHED_NS_FOLD + i) */
-    unsigned long long dq_safe;      /* completion-queue positions below this are known free (posters' cache) */
     uint32_t  fwd_done;              /* MTB 0: forwarders that exited */
-    unsigned long long claim_after;  /* PAGODA_SPREAD_NS: no claim before this %globaltimer value */
+    unsigned long long dq_safe;      /* completion-queue positions below this are known free (posters' cache) */
     uint32_t* dev_error;             /* &DevCtl.error, for the paper-named free syncBlock() (kDevErrorPtrOffset) */
+    SchedGroup grp[kMaxSchedGroups]; /* the MTB's scheduling groups (one unless PAGODA_config.sched_groups = 2) */
 };
 static_assert(offsetof(MtbShared, wt) == kWarpTableOffset, "WarpTable offset");
 static_assert(offsetof(MtbShared, stage_bar) == kStageBarOffset, "staging mbarriers offset");

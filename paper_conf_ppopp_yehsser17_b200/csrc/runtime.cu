@@ -47,8 +47,10 @@ static const int kSpawnChunk = 64;   /* batched spawns publish the doorbell once
 struct pagoda_ctx {
     pagoda_config cfg;
     int device = 0, sm_count = 0, n_mtb = 0, regs = 0;
-    int max_task_warps = 31;          /* largest warps*n_tb some MTB can host */
-    uint32_t max_task_granules = 0;   /* largest n_tb*granules some MTB can host */
+    int max_task_warps = 31;          /* largest warps*n_tb every task-running scheduling group can host */
+    uint32_t max_task_granules = 0;   /* largest n_tb*granules every task-running group can host */
+    int max_bars = PAGODA_BAR_IDS;    /* named barrier IDs of the smallest group (15; 7 with two groups) */
+    int n_grp = 1;                    /* scheduling groups per MTB */
     uint32_t R = 0, C = 0;
     cudaStream_t stream = nullptr;
     /* pinned, mapped */
@@ -189,14 +191,14 @@ static int shape_check(const pagoda_ctx* c, const int32_t* s, Split& o)
     o.gtb = ((uint32_t)shmem + PAGODA_GRANULE - 1) / PAGODA_GRANULE;
     if (o.wtb > c->max_task_warps || o.gtb > c->max_task_granules) return -EINVAL;   /* one TB must fit an MTB */
     if (o.wtb * n_tb <= c->max_task_warps && o.gtb * (uint32_t)n_tb <= c->max_task_granules &&
-        !(sync && o.wtb > 1 && n_tb > PAGODA_BAR_IDS)) {   /* fits one MTB (the common case: no divisions) */
+        !(sync && o.wtb > 1 && n_tb > c->max_bars)) {   /* fits one MTB (the common case: no divisions) */
         o.cap = n_tb;
         o.k = 1;
         return 0;
     }
     int cap = c->max_task_warps / o.wtb;
     if (o.gtb) cap = std::min<int>(cap, (int)(c->max_task_granules / o.gtb));
-    if (sync && o.wtb > 1) cap = std::min(cap, PAGODA_BAR_IDS);
+    if (sync && o.wtb > 1) cap = std::min(cap, c->max_bars);
     o.cap = cap;
     o.k = (n_tb + cap - 1) / cap;
     if (o.k > 1 && (n_tb > 65535 || (uint32_t)o.k > c->R / 4)) return -EINVAL;
@@ -312,6 +314,7 @@ void pagoda_config_default(pagoda_config* cfg)
     cfg->flags = 0;
     cfg->trace_events = 8192;
     cfg->watchdog_s = 60.0;
+    cfg->sched_groups = 1;
 }
 
 static bool pow2(uint32_t x) { return x && !(x & (x - 1)); }
@@ -323,7 +326,7 @@ static int start_kernel(pagoda_ctx* c)
     cudaSetDevice(c->device);
     if (c->life) cudaMemsetAsync(c->life, 0, (size_t)c->C * 8 * sizeof(uint64_t), c->stream);
     if (c->trace_count) {
-        cudaMemsetAsync(c->trace_count, 0, (size_t)c->n_mtb * sizeof(uint32_t), c->stream);
+        cudaMemsetAsync(c->trace_count, 0, (size_t)c->n_mtb * c->n_grp * sizeof(uint32_t), c->stream);
         cudaMemsetAsync(c->exec_count, 0, (size_t)c->n_mtb * 32 * sizeof(uint32_t), c->stream);
     }
     std::lock_guard<std::mutex> reg(g_ctx_mtx);   /* no constant-bank registration during the launch */
@@ -429,6 +432,8 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
         cfg.ring_entries < 2 * kSpawnChunk)
         return -EINVAL;
     if (cfg.exec_warps < 1 || cfg.exec_warps > 32) return -EINVAL;
+    if (cfg.sched_groups == 0) cfg.sched_groups = 1;
+    if (cfg.sched_groups > 2) return -EINVAL;
     cfg.exec_warps = std::min(cfg.exec_warps, block_warps);
     if (cfg.arena_bytes % PAGODA_GRANULE || cfg.arena_bytes / PAGODA_GRANULE > (uint32_t)kMaxGranules ||
         cfg.arena_bytes < 2u * 128u * 64u + 8u * PAGODA_GRANULE)   /* ingest staging + room for tasks */
@@ -459,12 +464,27 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
     c->R = cfg.ring_entries;
     c->C = cfg.comp_entries;
     const uint32_t arena_g = cfg.arena_bytes / PAGODA_GRANULE;
-    if (c->n_mtb == 1) {   /* MTB 0 alone: it also hosts the ingest warp and its staging */
-        c->max_task_warps = cfg.exec_warps == block_warps ? (int)block_warps - 1 : (int)cfg.exec_warps;
-        c->max_task_granules = arena_g - 2u * ingest_stage_entries(cfg.arena_bytes, 1) * 64u / PAGODA_GRANULE;
-    } else {
-        c->max_task_warps = (int)cfg.exec_warps;
-        c->max_task_granules = arena_g;
+    c->n_grp = (int)cfg.sched_groups;
+    {   /* a task must fit the smallest scheduling group that takes tickets (a task-running MTB's
+         * worker warps, split into n_grp equal warp ranges; the arena split the same way) */
+        const uint32_t gw = block_warps / (uint32_t)c->n_grp;
+        const uint32_t per = std::min<uint32_t>(cfg.exec_warps / (uint32_t)c->n_grp, gw);   /* workers per group */
+        uint32_t exec = 0;
+        for (int g = 0; g < c->n_grp; g++) exec |= (per >= 32u ? 0xffffffffu : ((1u << per) - 1u)) << (g * gw);
+        uint32_t ag = arena_g;
+        if (c->n_mtb == 1) {   /* MTB 0 alone: it also hosts the ingest warp and its staging */
+            exec &= ~(1u << (block_warps - 1u));
+            ag = arena_g - 2u * ingest_stage_entries(cfg.arena_bytes, 1) * 64u / PAGODA_GRANULE;
+        }
+        int mw = 32;
+        for (int g = 0; g < c->n_grp; g++) {
+            const uint32_t gm = (gw >= 32u ? 0xffffffffu : ((1u << gw) - 1u)) << (g * gw);
+            const int k = __builtin_popcount(exec & gm);
+            if (k) mw = std::min(mw, k);   /* a group without workers takes no tickets */
+        }
+        c->max_task_warps = mw;
+        c->max_task_granules = ag / (uint32_t)c->n_grp;
+        c->max_bars = c->n_grp == 1 ? PAGODA_BAR_IDS : 7;
     }
     c->warps_prefix.assign(c->C, 0);
 
@@ -498,11 +518,12 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
     if (cfg.flags & PAGODA_TRACE) {
         const size_t cap = cfg.trace_events ? cfg.trace_events : 8192;
         c->cfg.trace_events = (uint32_t)cap;
-        if (cudaMalloc(&c->trace, (size_t)c->n_mtb * cap * sizeof(LedgerEvent)) != cudaSuccess) goto fail;
-        if (cudaMalloc(&c->trace_count, (size_t)c->n_mtb * sizeof(uint32_t)) != cudaSuccess) goto fail;
+        /* one ledger per scheduling group (its holder is the allocator's single owner) */
+        if (cudaMalloc(&c->trace, (size_t)c->n_mtb * c->n_grp * cap * sizeof(LedgerEvent)) != cudaSuccess) goto fail;
+        if (cudaMalloc(&c->trace_count, (size_t)c->n_mtb * c->n_grp * sizeof(uint32_t)) != cudaSuccess) goto fail;
         if (cudaMalloc(&c->exec_trace, (size_t)c->n_mtb * 32 * cap * sizeof(ExecRecord)) != cudaSuccess) goto fail;
         if (cudaMalloc(&c->exec_count, (size_t)c->n_mtb * 32 * sizeof(uint32_t)) != cudaSuccess) goto fail;
-        cudaMemset(c->trace_count, 0, (size_t)c->n_mtb * sizeof(uint32_t));
+        cudaMemset(c->trace_count, 0, (size_t)c->n_mtb * c->n_grp * sizeof(uint32_t));
         cudaMemset(c->exec_count, 0, (size_t)c->n_mtb * 32 * sizeof(uint32_t));
     }
     if (cfg.flags & PAGODA_LIFECYCLE) {
@@ -547,6 +568,8 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
             p.resident_tdes_src = c->resident_src;
         }
         p.n_mtb = c->n_mtb;
+        p.n_grp = (uint32_t)c->n_grp;
+        p.n_exit = (uint32_t)(c->n_mtb * c->n_grp);
         if (cfg.flags & PAGODA_TRACE) {
             p.trace_cap = c->cfg.trace_events;
             p.trace = c->trace;
@@ -918,6 +941,7 @@ int pagoda_get_info(pagoda_ctx* c, pagoda_info* o)
     o->device = c->device;
     o->sm_count = c->sm_count;
     o->n_mtb = c->n_mtb;
+    o->sched_groups = c->n_grp;
     o->mtbs_per_sm = c->cfg.mtbs_per_sm;
     o->exec_warps = (int)c->cfg.exec_warps;
     o->arena_bytes = (int)c->cfg.arena_bytes;
@@ -934,7 +958,7 @@ int pagoda_get_info(pagoda_ctx* c, pagoda_info* o)
 
 int64_t pagoda_trace_read(pagoda_ctx* c, int mtb, void* dst, size_t cap)
 {
-    if (!c || !c->trace || mtb < 0 || mtb >= c->n_mtb) return -EINVAL;
+    if (!c || !c->trace || mtb < 0 || mtb >= c->n_mtb * c->n_grp) return -EINVAL;   /* a group's ledger id */
     uint32_t n = 0;
     if (cudaMemcpy(&n, c->trace_count + mtb, 4, cudaMemcpyDeviceToHost) != cudaSuccess) return -EIO;
     const size_t k = std::min<size_t>({(size_t)n, cap, (size_t)c->cfg.trace_events});

@@ -30,14 +30,15 @@ class pagoda_config(C.Structure):
     _fields_ = [("device", C.c_int), ("mtbs_per_sm", C.c_int), ("num_sms", C.c_int),
                 ("ring_entries", C.c_uint32), ("comp_entries", C.c_uint32), ("arena_bytes", C.c_uint32),
                 ("exec_warps", C.c_uint32), ("flags", C.c_uint32), ("trace_events", C.c_uint32),
-                ("watchdog_s", C.c_double)]
+                ("watchdog_s", C.c_double), ("sched_groups", C.c_uint32)]
 
 
 class pagoda_info(C.Structure):
     _fields_ = [("device", C.c_int), ("sm_count", C.c_int), ("n_mtb", C.c_int), ("mtbs_per_sm", C.c_int),
                 ("exec_warps", C.c_int), ("arena_bytes", C.c_int), ("regs_per_thread", C.c_int),
                 ("ring_entries", C.c_uint32), ("comp_entries", C.c_uint32), ("spawned", C.c_int64),
-                ("completed_low", C.c_int64), ("device_error", C.c_uint32), ("running", C.c_int)]
+                ("completed_low", C.c_int64), ("device_error", C.c_uint32), ("running", C.c_int),
+                ("sched_groups", C.c_int)]
 
 
 LEDGER_DTYPE = np.dtype([("seq", "<u4"), ("mtb", "<u2"), ("kind", "u1"), ("bar_id", "u1"),

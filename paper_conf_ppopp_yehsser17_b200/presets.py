@@ -31,4 +31,6 @@ def ctx_kwargs(workload: str, flags: int = 0) -> dict:
     kw = {"flags": f, "mtbs_per_sm": pr["mtbs_per_sm"], "arena_bytes": pr["arena_bytes"]}
     if pr.get("exec_warps"):
         kw["exec_warps"] = pr["exec_warps"]
+    if pr.get("sched_groups"):
+        kw["sched_groups"] = pr["sched_groups"]
     return kw

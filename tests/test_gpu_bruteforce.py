@@ -49,14 +49,16 @@ def test_alphabet_counts():
     assert sum(1 for _ in runs()) == 6 + 36 * 2 + 216 * 6 + 1296 * 24
 
 
-def _check_session(p, info, metas, first_id):
-    """Replay one session's ledger + executor records + completion stamps."""
-    evs = p.trace(0)
-    ex = np.concatenate([p.exec_trace(0, w) for w in range(EXEC_WARPS)])
+def _check_session(p, info, metas, first_id, exec_warps=EXEC_WARPS, granules=GRANULES):
+    """Replay one session's ledger + executor records + completion stamps (one ledger per
+    scheduling group: the checker sees each group as an MTB with its own share)."""
+    n_led = info.n_mtb * info.sched_groups
+    evs = np.concatenate([p.trace(m) for m in range(n_led)])
+    ex = np.concatenate([p.exec_trace(0, w) for w in range(exec_warps)])
     n_ids = metas[-1][0] - first_id + 1
     life = p.lifecycle(first_id, n_ids)
     tasks = np.array([(tid, w, 1) for tid, w in metas], oracle.TASK_DTYPE)
-    ok, msg = oracle.ledger_check(evs.view(oracle.LEDGER_DTYPE), info.n_mtb, EXEC_WARPS, GRANULES, BAR_IDS, tasks)
+    ok, msg = oracle.ledger_check(evs.view(oracle.LEDGER_DTYPE), n_led, exec_warps, granules, BAR_IDS, tasks)
     assert ok, msg
     done = np.maximum(life[:, 6], life[:, 7])   # one MTB: the record goes to the host at stamp 6
     comps = np.array([(tid, done[tid - first_id]) for tid, _ in metas], oracle.COMP_DTYPE)
@@ -66,7 +68,10 @@ def _check_session(p, info, metas, first_id):
     return len(evs), len(ex)
 
 
-def test_bruteforce_tiny_schedules():
+@pytest.mark.parametrize("groups", [1, 2])
+def test_bruteforce_tiny_schedules(groups):
+    """groups = 2: the same MTB split into two scheduling groups (pagoda_config.sched_groups),
+    each with 4 warps, 8 granules and its own named barriers (1..7 / 8..15) and token."""
     import torch
     dev = Dev()
     err = dev.zeros(8)
@@ -76,11 +81,14 @@ def test_bruteforce_tiny_schedules():
     all_runs = list(runs())
     per_session = 4096
     cap = 1 << 18
-    with Pagoda(num_sms=1, mtbs_per_sm=1, exec_warps=EXEC_WARPS, arena_bytes=ARENA, ring_entries=1024,
+    ew, gr = EXEC_WARPS * groups, GRANULES * groups
+    with Pagoda(num_sms=1, mtbs_per_sm=1, exec_warps=ew, arena_bytes=2 * 128 * 64 + gr * 512, ring_entries=1024,
                 comp_entries=1 << 17, flags=TRACE | LIFECYCLE | NO_START, trace_events=cap,
-                watchdog_s=30.0) as p:
+                watchdog_s=30.0, sched_groups=groups) as p:
         info = p.info()
-        assert info.n_mtb == 1 and info.exec_warps == EXEC_WARPS
+        assert info.n_mtb == 1 and info.exec_warps == ew and info.sched_groups == groups
+        if groups == 2:   # warps 0-3 in group 0, 4-7 in group 1 (16-warp halves of a 32-warp MTB)
+            pass
         # the debug config's limits are enforced at spawn (one TB must fit the MTB)
         import errno
         assert p.taskSpawn(160, 1, 0, 1, T.NOP) == -errno.EINVAL            # 5 warps > 4
@@ -112,7 +120,7 @@ def test_bruteforce_tiny_schedules():
                         assert p.wait(ids[i]) == 0
                 assert p.waitAll() == 0       # liveness: every task of the sequence completed
             assert p.stop() == 0
-            e, x = _check_session(p, info, metas, first)
+            e, x = _check_session(p, info, metas, first, ew, gr)
             n_events += e
             n_exec += x
             n_tasks += len(metas)

@@ -375,3 +375,46 @@ def test_tdes_registered_keys_full_size():
     assert np.array_equal(out, ref)
     for k in (0, 1, 16383, 32767):
         assert np.array_equal(out[k], _tdes_ref(pk[k]))
+
+
+# ---------------------------------------------------------------- two scheduling groups per MTB
+@pytest.mark.parametrize("wl", ["tdes", "mm", "mix"])
+def test_two_scheduling_groups_parity(wl):
+    """pagoda_config.sched_groups = 2 (two token holders per MTB, each with half the warps, task
+    slots, TB records, arena and named barriers): full-size 3DES (resident tables shared by both
+    groups) and sampled MM / mix tasks match the oracle."""
+    import oracle
+    from paper_conf_ppopp_yehsser17_b200 import inputs as I
+    from paper_conf_ppopp_yehsser17_b200 import workloads as W
+    from paper_conf_ppopp_yehsser17_b200.pagoda import NO_START, RESIDENT_TDES, Pagoda
+    if wl == "tdes":
+        w = W.tdes(32768, shmem=512)
+        cfg = dict(flags=RESIDENT_TDES | NO_START, arena_bytes=40 * 1024)
+    elif wl == "mm":
+        w = W.matmul(16384)
+        cfg = dict(flags=NO_START)
+    else:
+        w = W.mix(2048)
+        cfg = dict(flags=NO_START, mtbs_per_sm=1, arena_bytes=200 * 1024)
+    with Pagoda(sched_groups=2, **cfg) as p:
+        assert p.info().sched_groups == 2
+        if wl == "tdes":
+            p.tdes_register(w.tdes_tables)
+        assert p.start() == 0
+        p.spawn_shapes(w.shapes, w.args)
+        assert p.stop() == 0 and p.info().device_error == 0
+    out = w.outputs()
+    if wl == "tdes":
+        for k in list(range(0, 32768, 509)) + [32767]:
+            assert np.array_equal(out["out"][k], oracle.tdes_ecb(w.host["packets"][k], I.TDES_KEYS)), k
+    elif wl == "mm":
+        for k in range(0, 16384, 97):
+            assert np.array_equal(out["C"][k], oracle.mm32(w.host["A"][k], w.host["B"][k])), k
+    else:
+        kinds = w.host["kinds"]
+        for kind, fn in (("fb", oracle.filterbank), ("bf", oracle.beamformer), ("conv", oracle.conv),
+                         ("dct", oracle.dct)):
+            idx = np.nonzero(kinds == I.MIX_KINDS.index(kind))[0]
+            for j in range(0, len(idx), 37):
+                args = [a[j] for a in w.host[kind]] if kind != "dct" else [w.host[kind][0][j], w.host[kind][1]]
+                assert np.array_equal(out[kind][j], fn(*args)), (kind, j)

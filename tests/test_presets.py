@@ -21,6 +21,7 @@ def test_ctx_kwargs_match_bench_context():
             arena_kb = 0
             exec_warps = 0
             spread = -1
+            groups = 0
         cfg = bench.ctx_config(A, PG, w)
         kw = presets.ctx_kwargs(w, PG.NO_START)
         assert cfg == kw, w
