@@ -63,6 +63,10 @@
 #define PAGODA_FAST_PUB 1     /* a publisher checks 256 cells with relaxed loads all in flight, then one
                                  acquire fence (not 8 serial acquire loads per lane) */
 #endif
+#ifndef PAGODA_DIRECT_POST
+#define PAGODA_DIRECT_POST 0  /* task MTBs write completion records straight to the host window (one
+                                 system-scope fence per batch) instead of the device queue + forwarders */
+#endif
 #ifndef PAGODA_HOLDER_POSTS
 #define PAGODA_HOLDER_POSTS 0 /* the scheduler token holder posts completion records (batched per round);
                                  the last warp of a task only marks it pending and frees itself */
@@ -359,7 +363,7 @@ __device__ __forceinline__ void post_completions(MtbShared& S, SchedGroup& G, co
                 }
                 fence_acq_rel_gpu();
             }
-            if (p.n_mtb == 1) {
+            if (p.n_mtb == 1 || PAGODA_DIRECT_POST) {
                 asm volatile("fence.acq_rel.sys;" ::: "memory");
                 if (mine) st_relaxed_sys(reinterpret_cast<volatile uint64_t*>(&p.comp[id & p.comp_mask]), id);
                 if (mine) life_stamp(p, id, kLifeQueued);

@@ -54,11 +54,23 @@ def _check_session(p, info, metas, first_id, exec_warps=EXEC_WARPS, granules=GRA
     scheduling group: the checker sees each group as an MTB with its own share)."""
     n_led = info.n_mtb * info.sched_groups
     evs = np.concatenate([p.trace(m) for m in range(n_led)])
-    ex = np.concatenate([p.exec_trace(0, w) for w in range(exec_warps)])
+    ex = np.concatenate([p.exec_trace(0, w) for w in range(32)])
     n_ids = metas[-1][0] - first_id + 1
     life = p.lifecycle(first_id, n_ids)
     tasks = np.array([(tid, w, 1) for tid, w in metas], oracle.TASK_DTYPE)
-    ok, msg = oracle.ledger_check(evs.view(oracle.LEDGER_DTYPE), n_led, exec_warps, granules, BAR_IDS, tasks)
+    if info.sched_groups == 1:
+        ok, msg = oracle.ledger_check(evs.view(oracle.LEDGER_DTYPE), n_led, exec_warps, granules, BAR_IDS, tasks)
+    else:
+        # group g's workers are warps [16 g, 16 g + exec_warps / 2) and its granules / barrier IDs its own
+        # halves: every ALLOC must lie in its group's share (the checker then replays all 32 warp bits)
+        per = exec_warps // 2
+        for g in range(2):
+            e = evs[(evs["mtb"] == g) & (evs["kind"] == 1)]
+            assert not (e["warp_mask"] & ~np.uint32(((1 << per) - 1) << (16 * g))).any(), g
+            assert ((e["gran_off"] >= granules // 2 * g) & (e["gran_off"] + e["gran_len"] <= granules // 2 * (g + 1))).all()
+            b = e["bar_id"][e["bar_id"] > 0]
+            assert ((b >= 1) & (b <= 7)).all() if g == 0 else ((b >= 8) & (b <= 15)).all()
+        ok, msg = oracle.ledger_check(evs.view(oracle.LEDGER_DTYPE), n_led, 32, granules, BAR_IDS, tasks)
     assert ok, msg
     done = np.maximum(life[:, 6], life[:, 7])   # one MTB: the record goes to the host at stamp 6
     comps = np.array([(tid, done[tid - first_id]) for tid, _ in metas], oracle.COMP_DTYPE)
@@ -87,8 +99,6 @@ def test_bruteforce_tiny_schedules(groups):
                 watchdog_s=30.0, sched_groups=groups) as p:
         info = p.info()
         assert info.n_mtb == 1 and info.exec_warps == ew and info.sched_groups == groups
-        if groups == 2:   # warps 0-3 in group 0, 4-7 in group 1 (16-warp halves of a 32-warp MTB)
-            pass
         # the debug config's limits are enforced at spawn (one TB must fit the MTB)
         import errno
         assert p.taskSpawn(160, 1, 0, 1, T.NOP) == -errno.EINVAL            # 5 warps > 4
