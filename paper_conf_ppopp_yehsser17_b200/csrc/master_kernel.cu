@@ -64,8 +64,11 @@
                                  acquire fence (not 8 serial acquire loads per lane) */
 #endif
 #ifndef PAGODA_DIRECT_POST
-#define PAGODA_DIRECT_POST 0  /* task MTBs write completion records straight to the host window (one
+#define PAGODA_DIRECT_POST 0  /* task MTBs always write completion records straight to the host window (one
                                  system-scope fence per batch) instead of the device queue + forwarders */
+#endif
+#ifndef PAGODA_DIRECT_IDLE_NS
+#define PAGODA_DIRECT_IDLE_NS 50000   /* ... or when the group posted nothing for this long (lone tasks) */
 #endif
 #ifndef PAGODA_HOLDER_POSTS
 #define PAGODA_HOLDER_POSTS 0 /* the scheduler token holder posts completion records (batched per round);
@@ -101,10 +104,34 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity)
  * barrier address from %tid (two ALU ops) every trip instead of keeping it live across the task
  * body, where the 32-register build spilled it: a local-memory load per trip put idle warps on
  * the load/store pipe the busy warps' bodies need (ncu source counters). */
+#ifndef PAGODA_WAIT_SLEEP_MAX
+#define PAGODA_WAIT_SLEEP_MAX 1024   /* 0: wait in mbarrier.try_wait (suspend); else test + nanosleep back-off (ns cap) */
+#endif
 __device__ __forceinline__ void exec_wait(uint32_t parity)
 {
     extern __shared__ __align__(1024) unsigned char pagoda_mk_smem[];
     uint32_t done = 0;
+#if PAGODA_WAIT_SLEEP_MAX
+    /* A warp suspended in try_wait is woken by ANY mbarrier traffic of the CTA (every dispatch of
+     * every task), so idle warps re-checked their barrier every few tens of ns: the check and the
+     * re-suspend were two thirds of all instructions a 3DES session issued, and they occupy the
+     * load/store pipe the S-box lookups need (ncu source counters).  Instead: a
+     * non-blocking test, then a plain nanosleep that only time ends, doubling from 64 ns up to the
+     * cap (a dispatch is seen at most one sleep late). */
+    uint32_t ns = 64;
+    for (;;) {
+        uint32_t tid;
+        asm volatile("mov.u32 %0, %%tid.x;" : "=r"(tid));
+        const uint32_t a = smem_u32(pagoda_mk_smem) + ((tid >> 5) << 3);   /* &S.exec_bar[warp] */
+        asm volatile("{ .reg .pred p; mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+                     : "=r"(done)
+                     : "r"(a), "r"(parity)
+                     : "memory");
+        if (done) return;
+        __nanosleep(ns);
+        ns = min(ns * 2u, (uint32_t)PAGODA_WAIT_SLEEP_MAX);
+    }
+#else
     while (!done) {
         uint32_t tid;
         asm volatile("mov.u32 %0, %%tid.x;" : "=r"(tid));
@@ -115,6 +142,7 @@ __device__ __forceinline__ void exec_wait(uint32_t parity)
             : "r"(a), "r"(parity), "n"(PAGODA_WAKE_HINT_NS)
             : "memory");
     }
+#endif
 }
 __device__ __forceinline__ void fence_acq_rel_gpu()
 {
@@ -363,7 +391,19 @@ __device__ __forceinline__ void post_completions(MtbShared& S, SchedGroup& G, co
                 }
                 fence_acq_rel_gpu();
             }
-            if (p.n_mtb == 1 || PAGODA_DIRECT_POST) {
+            /* A lone task skips the forwarder hop: the group's last post is long ago, so its SM is quiet
+             * and a system-scope fence is cheap.  Under load the queue path stays (a system fence on an
+             * SM full of memory traffic waits for all of it: MM -12 % if every post went direct). */
+            uint32_t direct = (p.n_mtb == 1 || PAGODA_DIRECT_POST) ? 1u : 0u;
+            if (!direct && PAGODA_DIRECT_IDLE_NS) {
+                if (lane == 0) {
+                    const unsigned long long now = globaltimer_ns();
+                    direct = now - G.last_post > (unsigned long long)PAGODA_DIRECT_IDLE_NS;
+                    G.last_post = now;
+                }
+                direct = __shfl_sync(0xffffffffu, direct, 0);
+            }
+            if (direct) {
                 asm volatile("fence.acq_rel.sys;" ::: "memory");
                 if (mine) st_relaxed_sys(reinterpret_cast<volatile uint64_t*>(&p.comp[id & p.comp_mask]), id);
                 if (mine) life_stamp(p, id, kLifeQueued);
@@ -1757,6 +1797,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) master_kernel(MkParams p
                 G.claim_after = 0;
                 G.comp_pending = 0;
                 G.poster = 0;
+                G.last_post = 0;
                 /* a group without workers never runs a holder: it counts as exited now */
                 G.token = (exec_mask & gm) ? 1u : 0u;
                 if (!(exec_mask & gm)) atomicAdd(&p.dctl->exited, 1u);

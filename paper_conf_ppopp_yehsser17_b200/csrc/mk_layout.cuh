@@ -188,6 +188,7 @@ struct SchedGroup {
     uint32_t  sctr[8];               /* scheduler counters (holder-only), flushed at exit */
     unsigned long long claim_after;  /* PAGODA_SPREAD_NS: no claim before this %globaltimer value */
     unsigned long long sprof[8];     /* PAGODA_PROFILE: ns per phase (PAGODA_CTR_SCHED_NS_FOLD + i) */
+    unsigned long long last_post;    /* %globaltimer of the group's last completion post */
 };
 
 /* Per-MTB control block at the start of dynamic shared memory (P:456-458:
