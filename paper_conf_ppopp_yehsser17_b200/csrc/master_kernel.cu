@@ -59,6 +59,9 @@
                                  flight together (one L2 round trip; the cells' sequence words were already
                                  acquired), not 4 serial acquire loads per cell */
 #endif
+#ifndef PAGODA_CELL_RELAXED
+#define PAGODA_CELL_RELAXED 0 /* (FAST_LOAD 0) a lane's four cell loads relaxed + one CTA fence, not four acquires */
+#endif
 #ifndef PAGODA_FAST_PUB
 #define PAGODA_FAST_PUB 1     /* a publisher checks 256 cells with relaxed loads all in flight, then one
                                  acquire fence (not 8 serial acquire loads per lane) */
@@ -105,7 +108,8 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity)
  * body, where the 32-register build spilled it: a local-memory load per trip put idle warps on
  * the load/store pipe the busy warps' bodies need (ncu source counters). */
 #ifndef PAGODA_WAIT_SLEEP_MAX
-#define PAGODA_WAIT_SLEEP_MAX 1024   /* 0: wait in mbarrier.try_wait (suspend); else test + nanosleep back-off (ns cap) */
+#define PAGODA_WAIT_SLEEP_MAX 0      /* 0: wait in mbarrier.try_wait (suspend); else test + nanosleep back-off (ns cap)
+                                        (measured: no throughput difference; the suspension wakes sooner) */
 #endif
 __device__ __forceinline__ void exec_wait(uint32_t parity)
 {
@@ -113,11 +117,11 @@ __device__ __forceinline__ void exec_wait(uint32_t parity)
     uint32_t done = 0;
 #if PAGODA_WAIT_SLEEP_MAX
     /* A warp suspended in try_wait is woken by ANY mbarrier traffic of the CTA (every dispatch of
-     * every task), so idle warps re-checked their barrier every few tens of ns: the check and the
-     * re-suspend were two thirds of all instructions a 3DES session issued, and they occupy the
-     * load/store pipe the S-box lookups need (ncu source counters).  Instead: a
-     * non-blocking test, then a plain nanosleep that only time ends, doubling from 64 ns up to the
-     * cap (a dispatch is seen at most one sleep late). */
+     * every task), so idle warps re-check their barrier every few tens of ns: the check and the
+     * re-suspend are two thirds of all instructions a 3DES session issues (ncu source counters,
+     * DESIGN.md §8).  This variant tests without blocking, then sleeps (doubling from 64 ns up to
+     * the cap).  Measured: the same throughput on every workload (the idle instructions use
+     * issue slots the busy warps did not need), so the default stays the prompt suspension. */
     uint32_t ns = 64;
     for (;;) {
         uint32_t tid;
@@ -1288,6 +1292,28 @@ __device__ int sched_copy(MtbShared& S, Sched& st, const MkParams& p, uint32_t r
     uint32_t used = 0;
     if (lane < r) {
         const uint32_t slot = nth_set_bit(st.free_task, lane);
+        S.pend[fq(st, st.pl + lane)] = (uint8_t)slot;
+        st_relaxed_gpu32(&p.dseq[t & p.ring_mask], (uint32_t)(t + (uint64_t)p.ring_mask + 1));
+        if (p.life && !(S.tasks[slot].flags & kEntryGroup)) life_stamp(p, S.tasks[slot].id, kLifeLoad);
+        used = 1u << slot;
+    }
+#elif PAGODA_FAST_LOAD == 0 && PAGODA_CELL_RELAXED
+    /* lane i copies cell i with four relaxed 16-byte loads in flight together (the sequence word's
+     * acquire already ordered them after the publication and invalidated L1), then a CTA-scope fence
+     * before the hand-back: the loads have returned before the store issues */
+    uint32_t used = 0;
+    if (lane < r) {
+        const uint32_t slot = nth_set_bit(st.free_task, lane);
+        const int4* src = reinterpret_cast<const int4*>(p.dring + (t & p.ring_mask));
+        int4* dst = reinterpret_cast<int4*>(&S.tasks[slot]);
+        int4 v[4];
+#pragma unroll
+        for (int q = 0; q < 4; q++)
+            asm volatile("ld.relaxed.gpu.global.v4.s32 {%0,%1,%2,%3}, [%4];"
+                         : "=r"(v[q].x), "=r"(v[q].y), "=r"(v[q].z), "=r"(v[q].w) : "l"(src + q) : "memory");
+#pragma unroll
+        for (int q = 0; q < 4; q++) dst[q] = v[q];
+        asm volatile("fence.acq_rel.cta;" ::: "memory");
         S.pend[fq(st, st.pl + lane)] = (uint8_t)slot;
         st_relaxed_gpu32(&p.dseq[t & p.ring_mask], (uint32_t)(t + (uint64_t)p.ring_mask + 1));
         if (p.life && !(S.tasks[slot].flags & kEntryGroup)) life_stamp(p, S.tasks[slot].id, kLifeLoad);

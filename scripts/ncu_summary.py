@@ -33,6 +33,35 @@ def main(path):
                if n.startswith("smsp__average_warps_issue_stalled_") and n.endswith("_per_issue_active.ratio") and v[i]]
     for val, n in sorted(stalls, reverse=True)[:8]:
         print(f"{n} {val}")
+    opcode_mix(path)
+
+
+def opcode_mix(path, top=14):
+    """Executed instructions by SASS opcode (the source page's per-instruction counters, captured
+    with --import-source): `opmix OPCODE share_of_executed stall_sample_share` lines."""
+    import collections
+    out = subprocess.run(["ncu", "-i", path, "--page", "source", "--csv", "--print-source", "sass"],
+                         capture_output=True, text=True).stdout
+    rows = list(csv.reader(out.splitlines()))
+    hdr = next((r for r in rows if "Instructions Executed" in r), None)
+    if not hdr:
+        return
+    i_src, i_ex = hdr.index("Source"), hdr.index("Instructions Executed")
+    i_st = hdr.index("Warp Stall Sampling (All Samples)") if "Warp Stall Sampling (All Samples)" in hdr else None
+    ex, st = collections.Counter(), collections.Counter()
+    for r in rows[rows.index(hdr) + 1:]:
+        if len(r) <= i_ex or not r[i_ex].isdigit():
+            continue
+        toks = r[i_src].split()
+        if not toks:
+            continue
+        op = (toks[1] if toks[0].startswith("@") and len(toks) > 1 else toks[0]).split(".")[0]
+        ex[op] += int(r[i_ex])
+        if i_st is not None and r[i_st].isdigit():
+            st[op] += int(r[i_st])
+    te, ts = sum(ex.values()) or 1, sum(st.values()) or 1
+    for op, n in ex.most_common(top):
+        print(f"opmix {op} {100.0 * n / te:.1f}% {100.0 * st[op] / ts:.1f}%")
 
 
 if __name__ == "__main__":

@@ -67,7 +67,8 @@ def _check_session(p, info, metas, first_id, exec_warps=EXEC_WARPS, granules=GRA
         for g in range(2):
             e = evs[(evs["mtb"] == g) & (evs["kind"] == 1)]
             assert not (e["warp_mask"] & ~np.uint32(((1 << per) - 1) << (16 * g))).any(), g
-            assert ((e["gran_off"] >= granules // 2 * g) & (e["gran_off"] + e["gran_len"] <= granules // 2 * (g + 1))).all()
+            e2 = e[e["gran_len"] > 0]
+            assert ((e2["gran_off"] >= granules // 2 * g) & (e2["gran_off"] + e2["gran_len"] <= granules // 2 * (g + 1))).all()
             b = e["bar_id"][e["bar_id"] > 0]
             assert ((b >= 1) & (b <= 7)).all() if g == 0 else ((b >= 8) & (b <= 15)).all()
         ok, msg = oracle.ledger_check(evs.view(oracle.LEDGER_DTYPE), n_led, 32, granules, BAR_IDS, tasks)
