@@ -60,7 +60,8 @@
                                  acquired), not 4 serial acquire loads per cell */
 #endif
 #ifndef PAGODA_CELL_RELAXED
-#define PAGODA_CELL_RELAXED 0 /* (FAST_LOAD 0) a lane's four cell loads relaxed + one CTA fence, not four acquires */
+#define PAGODA_CELL_RELAXED 1 /* (FAST_LOAD 0) a lane's four cell loads relaxed + one CTA fence, not four serial
+                                 acquires (measured +1-2 % on 3DES / MM / NOP) */
 #endif
 #ifndef PAGODA_FAST_PUB
 #define PAGODA_FAST_PUB 1     /* a publisher checks 256 cells with relaxed loads all in flight, then one
