@@ -74,6 +74,13 @@
 #ifndef PAGODA_DIRECT_IDLE_NS
 #define PAGODA_DIRECT_IDLE_NS 50000   /* ... or when the group posted nothing for this long (lone tasks) */
 #endif
+#ifndef PAGODA_FIXED_GROUPS
+#define PAGODA_FIXED_GROUPS 0 /* > 0: compile for exactly this many scheduling groups (A/B of the group indexing) */
+#endif
+__device__ __forceinline__ uint32_t n_groups(const MkParams& p)
+{
+    return PAGODA_FIXED_GROUPS ? (uint32_t)PAGODA_FIXED_GROUPS : p.n_grp;
+}
 #ifndef PAGODA_HOLDER_POSTS
 #define PAGODA_HOLDER_POSTS 0 /* the scheduler token holder posts completion records (batched per round);
                                  the last warp of a task only marks it pending and frees itself */
@@ -412,6 +419,7 @@ __device__ __forceinline__ void post_completions(MtbShared& S, SchedGroup& G, co
                 asm volatile("fence.acq_rel.sys;" ::: "memory");
                 if (mine) st_relaxed_sys(reinterpret_cast<volatile uint64_t*>(&p.comp[id & p.comp_mask]), id);
                 if (mine) life_stamp(p, id, kLifeQueued);
+                if (mine && p.n_mtb > 1) life_stamp(p, id, kLifeFwd);   /* in the host window already: no hop */
             } else {
                 /* queue positions below dq_safe were cleared by the forwarders (their cursors, read
                  * by an acquire below when a position reaches the horizon) */
@@ -1471,9 +1479,9 @@ __device__ __forceinline__ void sst_load(MtbShared& S, Sched& st, uint32_t exec_
     st.exec_mask = exec_mask;
     st.holder_bit = 1u << (threadIdx.x >> 5);
     st.g = g;
-    st.rm = 32u / p.n_grp - 1u;
+    st.rm = 32u / n_groups(p) - 1u;
     st.rb = g * (st.rm + 1u);
-    st.vmtb = mtb * (int)p.n_grp + (int)g;
+    st.vmtb = mtb * (int)n_groups(p) + (int)g;
 }
 
 __device__ __forceinline__ bool token_try(SchedGroup& G)
@@ -1701,7 +1709,7 @@ __device__ void worker(MtbShared& S, char* smem_base, const MkParams& p, int mtb
 {
     uint32_t phase = 0;
     SchedGroup& G = S.grp[g];
-    const int vmtb = mtb * (int)p.n_grp + (int)g;
+    const int vmtb = mtb * (int)n_groups(p) + (int)g;
     for (;;) {
         if (holder) {
             if (holder_phase(S, p, mtb, w, exec_mask, g)) return;
@@ -1774,7 +1782,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) master_kernel(MkParams p
     }
     /* worker warps: the first exec_warps / n_grp warps of each group's range (MTB 0: minus the ingest warp) */
     const int ew = min(p.exec_warps, nw);
-    const uint32_t n_grp = p.n_grp, gw = (uint32_t)nw / n_grp, gs = 32u / n_grp;
+    const uint32_t n_grp = n_groups(p), gw = (uint32_t)nw / n_grp, gs = 32u / n_grp;
     uint32_t exec_mask = 0;
     for (uint32_t g = 0; g < n_grp; g++) {
         const uint32_t per = min((uint32_t)ew / n_grp, gw);
