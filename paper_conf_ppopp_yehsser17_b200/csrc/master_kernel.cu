@@ -77,16 +77,17 @@
 #ifndef PAGODA_FIXED_GROUPS
 #define PAGODA_FIXED_GROUPS 0 /* > 0: compile for exactly this many scheduling groups (A/B of the group indexing) */
 #endif
-__device__ __forceinline__ uint32_t n_groups(const MkParams& p)
-{
-    return PAGODA_FIXED_GROUPS ? (uint32_t)PAGODA_FIXED_GROUPS : p.n_grp;
-}
 #ifndef PAGODA_HOLDER_POSTS
 #define PAGODA_HOLDER_POSTS 0 /* the scheduler token holder posts completion records (batched per round);
                                  the last warp of a task only marks it pending and frees itself */
 #endif
 
 namespace pagoda {
+
+__device__ __forceinline__ uint32_t n_groups(const MkParams& p)
+{
+    return PAGODA_FIXED_GROUPS ? (uint32_t)PAGODA_FIXED_GROUPS : p.n_grp;
+}
 
 /* ------------------------------------------------------------------ PTX helpers */
 __device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count)

@@ -15,7 +15,10 @@ def parse(path):
     for line in open(path):
         parts = line.split()
         if len(parts) >= 2:
-            vals[parts[0]] = (float(parts[1].replace(",", "")), parts[2] if len(parts) > 2 else "")
+            try:
+                vals[parts[0]] = (float(parts[1].replace(",", "")), parts[2] if len(parts) > 2 else "")
+            except ValueError:   # opmix lines
+                pass
     b = sum(v * UNIT.get(u, 1) for k, (v, u) in vals.items() if k in ("dram__bytes_read.sum", "dram__bytes_write.sum"))
     return b, vals.get("gpu__time_duration.sum")
 
