@@ -74,9 +74,6 @@
 #ifndef PAGODA_DIRECT_IDLE_NS
 #define PAGODA_DIRECT_IDLE_NS 50000   /* ... or when the group posted nothing for this long (lone tasks) */
 #endif
-#ifndef PAGODA_FIXED_GROUPS
-#define PAGODA_FIXED_GROUPS 0 /* > 0: compile for exactly this many scheduling groups (A/B of the group indexing) */
-#endif
 #ifndef PAGODA_HOLDER_POSTS
 #define PAGODA_HOLDER_POSTS 0 /* the scheduler token holder posts completion records (batched per round);
                                  the last warp of a task only marks it pending and frees itself */
@@ -84,10 +81,6 @@
 
 namespace pagoda {
 
-__device__ __forceinline__ uint32_t n_groups(const MkParams& p)
-{
-    return PAGODA_FIXED_GROUPS ? (uint32_t)PAGODA_FIXED_GROUPS : p.n_grp;
-}
 
 /* ------------------------------------------------------------------ PTX helpers */
 __device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count)
@@ -979,7 +972,9 @@ __device__ __noinline__ void ingest_publisher(MtbShared& S, const MkParams& p, c
  * fit at the last task size seen, so no claim ever fails or retries; a ticket
  * is loaded into a task slot once its cell is published, and placed in FIFO
  * order as soon as the MTB has the resources. */
+template <int kG>   /* kG: scheduling groups per MTB, a compile-time constant (the kernel is instantiated per count) */
 struct Sched {
+    static constexpr uint32_t rm = 32u / (uint32_t)kG - 1u;   /* the group's FIFO slice size - 1 */
     uint32_t free_w, free_task, free_tbs, free_bar, exec_mask;
     uint32_t fg;         /* this lane's 32 granule bits */
     uint32_t ph, pl, pt; /* FIFO: [ph,pl) loaded task slots, [pl,pt) tickets not yet loaded */
@@ -987,18 +982,22 @@ struct Sched {
     uint32_t seq;        /* ledger clock */
     uint32_t holder_bit; /* the warp holding the scheduler token (this warp) */
     uint32_t g;          /* scheduling group (S.grp[g]) */
-    uint32_t rb, rm;     /* the group's slice of the FIFO arrays pend / pend_ticket: base, size - 1 */
-    int      vmtb;       /* ledger id of the group: mtb * n_grp + g */
+    int      vmtb;       /* ledger id of the group: mtb * kG + g */
 };
 /* FIFO position x of the group's slice of pend / pend_ticket */
-__device__ __forceinline__ uint32_t fq(const Sched& st, uint32_t x) { return st.rb + (x & st.rm); }
+template <int kG>
+__device__ __forceinline__ uint32_t fq(const Sched<kG>& st, uint32_t x)
+{
+    return kG == 1 ? (x & 31u) : st.g * (Sched<kG>::rm + 1u) + (x & Sched<kG>::rm);
+}
 
 __device__ __forceinline__ uint32_t nth_set_bit(uint32_t mask, uint32_t n)
 {   /* 0-based n-th set bit position (mask must have > n bits) */
     return __fns(mask, 0, (int)n + 1);
 }
 
-__device__ bool sched_place(MtbShared& S, Sched& st, const MkParams& p, int mtb, uint32_t slot)
+template <int kG>
+__device__ bool sched_place(MtbShared& S, Sched<kG>& st, const MkParams& p, int mtb, uint32_t slot)
 {
     const uint32_t lane = threadIdx.x & 31u;
     const TaskEntry& e = S.tasks[slot];
@@ -1095,7 +1094,8 @@ __device__ bool sched_place(MtbShared& S, Sched& st, const MkParams& p, int mtb,
 #ifndef PAGODA_BATCH_PLACE
 #define PAGODA_BATCH_PLACE 0   /* measured: slower (most rounds place one task; the run logic costs more than it saves) */
 #endif
-__device__ int sched_place_run(MtbShared& S, Sched& st, const MkParams& p, int mtb)
+template <int kG>
+__device__ int sched_place_run(MtbShared& S, Sched<kG>& st, const MkParams& p, int mtb)
 {
     const uint32_t lane = threadIdx.x & 31u;
     const uint32_t navail = min(st.pl - st.ph, 32u);
@@ -1200,7 +1200,8 @@ __device__ int sched_place_run(MtbShared& S, Sched& st, const MkParams& p, int m
  * (one ticket when the size is unknown), never more than the ring holds; one
  * at a time while the backlog is smaller than what all MTBs could take, so
  * consecutive (often similar-cost) tasks spread over MTBs. */
-__device__ int sched_claim(MtbShared& S, Sched& st, const MkParams& p)
+template <int kG>
+__device__ int sched_claim(MtbShared& S, Sched<kG>& st, const MkParams& p)
 {
     const uint32_t lane = threadIdx.x & 31u;
     const uint32_t queued = st.pt - st.ph;
@@ -1253,11 +1254,13 @@ __device__ int sched_claim(MtbShared& S, Sched& st, const MkParams& p)
     return (int)k;
 }
 
-__device__ int sched_copy(MtbShared& S, Sched& st, const MkParams& p, uint32_t r);
+template <int kG>
+__device__ int sched_copy(MtbShared& S, Sched<kG>& st, const MkParams& p, uint32_t r);
 
 /* Load the published tickets at the front of the FIFO into free task slots,
  * then hand their cells back to the producer (seq = t + R). */
-__device__ int sched_load(MtbShared& S, Sched& st, const MkParams& p)
+template <int kG>
+__device__ int sched_load(MtbShared& S, Sched<kG>& st, const MkParams& p)
 {
     const uint32_t lane = threadIdx.x & 31u;
     const uint32_t n = min(st.pt - st.pl, (uint32_t)__popc(st.free_task));
@@ -1278,7 +1281,8 @@ __device__ int sched_load(MtbShared& S, Sched& st, const MkParams& p)
 
 /* Copy the first r tickets of the FIFO (published: their cells' sequence words
  * were acquired) into free task slots and hand the cells back. */
-__device__ int sched_copy(MtbShared& S, Sched& st, const MkParams& p, uint32_t r)
+template <int kG>
+__device__ int sched_copy(MtbShared& S, Sched<kG>& st, const MkParams& p, uint32_t r)
 {
     const uint32_t lane = threadIdx.x & 31u;
     const uint64_t t = lane < r ? S.pend_ticket[fq(st, st.pl + lane)] : 0;
@@ -1386,7 +1390,8 @@ __device__ int sched_copy(MtbShared& S, Sched& st, const MkParams& p, uint32_t r
  * at that position is its own (consecutive tasks land on different MTBs).
  * Reserved positions past the final tail are void at stop (head = tail).
  * Returns how many tickets at the FIFO front are published (sched_copy). */
-__device__ int sched_claim_check(MtbShared& S, Sched& st, const MkParams& p)
+template <int kG>
+__device__ int sched_claim_check(MtbShared& S, Sched<kG>& st, const MkParams& p)
 {
     const uint32_t lane = threadIdx.x & 31u;
     const uint32_t queued = st.pt - st.ph;
@@ -1442,7 +1447,8 @@ __device__ int sched_claim_check(MtbShared& S, Sched& st, const MkParams& p)
  * warp holds the token, or every worker is running a task (and the next one to
  * finish takes it).  So every warp of the MTB executes tasks: eight 4-warp tasks
  * per MTB instead of seven (SURVEY App. A "v2: self-scheduling"). */
-__device__ __forceinline__ void sst_save(MtbShared& S, const Sched& st)
+template <int kG>
+__device__ __forceinline__ void sst_save(MtbShared& S, const Sched<kG>& st)
 {
     const uint32_t lane = threadIdx.x & 31u;
     SchedGroup& G = S.grp[st.g];
@@ -1462,7 +1468,8 @@ __device__ __forceinline__ void sst_save(MtbShared& S, const Sched& st)
 }
 
 /* the holder state of group g (the caller's warp now holds g's token) */
-__device__ __forceinline__ void sst_load(MtbShared& S, Sched& st, uint32_t exec_mask, uint32_t g, const MkParams& p,
+template <int kG>
+__device__ __forceinline__ void sst_load(MtbShared& S, Sched<kG>& st, uint32_t exec_mask, uint32_t g, const MkParams& p,
                                          int mtb)
 {
     __syncwarp();
@@ -1480,9 +1487,8 @@ __device__ __forceinline__ void sst_load(MtbShared& S, Sched& st, uint32_t exec_
     st.exec_mask = exec_mask;
     st.holder_bit = 1u << (threadIdx.x >> 5);
     st.g = g;
-    st.rm = 32u / n_groups(p) - 1u;
-    st.rb = g * (st.rm + 1u);
-    st.vmtb = mtb * (int)n_groups(p) + (int)g;
+    st.vmtb = mtb * kG + (int)g;
+    (void)p;
 }
 
 __device__ __forceinline__ bool token_try(SchedGroup& G)
@@ -1507,7 +1513,8 @@ __device__ __forceinline__ void token_release(SchedGroup& G)
 }
 
 /* fold the mailboxes into the holder's state (deallocMarkedSM, Alg. 1 L22) */
-__device__ bool sched_fold(MtbShared& S, Sched& st, const MkParams& p, int mtb)
+template <int kG>
+__device__ bool sched_fold(MtbShared& S, Sched<kG>& st, const MkParams& p, int mtb)
 {
     const uint32_t lane = threadIdx.x & 31u;
     uint32_t mw = 0, mt = 0, mk = 0;
@@ -1544,7 +1551,8 @@ __device__ bool sched_fold(MtbShared& S, Sched& st, const MkParams& p, int mtb)
 
 /* One scheduling round: fold, load published tickets, place in FIFO order
  * (Alg. 1 L14-28), take more tickets.  Sets exit when the session is over. */
-__device__ bool sched_round(MtbShared& S, Sched& st, const MkParams& p, int mtb, bool& exit)
+template <int kG>
+__device__ bool sched_round(MtbShared& S, Sched<kG>& st, const MkParams& p, int mtb, bool& exit)
 {
     const uint32_t lane = threadIdx.x & 31u;
     uint64_t t0 = pf_now();
@@ -1629,7 +1637,8 @@ __device__ bool sched_round(MtbShared& S, Sched& st, const MkParams& p, int mtb,
  * warp (it wakes with a SCHED slot), else release it — re-checking the mailbox
  * afterwards so a warp that freed itself meanwhile, and failed to take the
  * token, is not left without a scheduler. */
-__device__ void sched_handoff(MtbShared& S, Sched& st, const MkParams& p, int mtb)
+template <int kG>
+__device__ void sched_handoff(MtbShared& S, Sched<kG>& st, const MkParams& p, int mtb)
 {
     const uint32_t lane = threadIdx.x & 31u;
     for (;;) {
@@ -1660,11 +1669,12 @@ __device__ void sched_handoff(MtbShared& S, Sched& st, const MkParams& p, int mt
  * dispatched itself (hands the token on) or the session ends (returns true).
  * The scheduler state lives only here (loaded from / saved to shared memory),
  * so no register holds it while the warp runs task bodies. */
+template <int kG>
 __device__ __noinline__ bool holder_phase(MtbShared& S, const MkParams& p, int mtb, int w, uint32_t exec_mask,
                                           uint32_t g)
 {
     const uint32_t lane = threadIdx.x & 31u;
-    Sched st;
+    Sched<kG> st;
     sst_load(S, st, exec_mask, g, p, mtb);
     uint32_t backoff = 0;
     for (;;) {
@@ -1705,15 +1715,16 @@ __device__ __noinline__ bool holder_phase(MtbShared& S, const MkParams& p, int m
 
 /* Every worker warp runs this loop (warps 0..exec_warps-1; MTB 0's last warp ingests); exec_mask is
  * the worker warps of its scheduling group g. */
+template <int kG>
 __device__ void worker(MtbShared& S, char* smem_base, const MkParams& p, int mtb, int w, uint32_t resident,
                        uint32_t exec_mask, bool holder, uint32_t g)
 {
     uint32_t phase = 0;
     SchedGroup& G = S.grp[g];
-    const int vmtb = mtb * (int)n_groups(p) + (int)g;
+    const int vmtb = mtb * kG + (int)g;
     for (;;) {
         if (holder) {
-            if (holder_phase(S, p, mtb, w, exec_mask, g)) return;
+            if (holder_phase<kG>(S, p, mtb, w, exec_mask, g)) return;
             holder = false;
         }
         exec_wait(phase);   /* mbar_wait(&S.exec_bar[w], phase) without a live address register */
@@ -1730,7 +1741,7 @@ __device__ void worker(MtbShared& S, char* smem_base, const MkParams& p, int mtb
 }
 
 /* ------------------------------------------------------------------ the kernel */
-template <int kMinBlocks, int kThreads>
+template <int kMinBlocks, int kThreads, int kG>
 __global__ void __launch_bounds__(kThreads, kMinBlocks) master_kernel(MkParams p)
 {
     constexpr int nw = kThreads / 32;   /* warps per MTB */
@@ -1783,7 +1794,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) master_kernel(MkParams p
     }
     /* worker warps: the first exec_warps / n_grp warps of each group's range (MTB 0: minus the ingest warp) */
     const int ew = min(p.exec_warps, nw);
-    const uint32_t n_grp = n_groups(p), gw = (uint32_t)nw / n_grp, gs = 32u / n_grp;
+    const uint32_t n_grp = (uint32_t)kG, gw = (uint32_t)nw / n_grp, gs = 32u / n_grp;
     uint32_t exec_mask = 0;
     for (uint32_t g = 0; g < n_grp; g++) {
         const uint32_t per = min((uint32_t)ew / n_grp, gw);
@@ -1863,12 +1874,15 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) master_kernel(MkParams p
         ingest_publisher(S, p, ingest_stage, ingest_publisher_index(warp, nw));
     else if (io && warp == host_poster_warp(nw)) host_poster(S, p);
     else if (io && forwarder_index(warp, nw) < p.n_fwd) comp_forwarder(S, p, forwarder_index(warp, nw));
-    else if ((my_exec >> warp) & 1u) worker(S, smem_base, p, mtb, warp, resident, my_exec, warp == first, my_g);
+    else if ((my_exec >> warp) & 1u) worker<kG>(S, smem_base, p, mtb, warp, resident, my_exec, warp == first, my_g);
 }
 
-template __global__ void master_kernel<1, 1024>(MkParams);
-template __global__ void master_kernel<2, 1024>(MkParams);
-template __global__ void master_kernel<4, 512>(MkParams);   /* twice the MTBs (schedulers) per SM */
+template __global__ void master_kernel<1, 1024, 1>(MkParams);
+template __global__ void master_kernel<2, 1024, 1>(MkParams);
+template __global__ void master_kernel<4, 512, 1>(MkParams);   /* twice the MTBs (schedulers) per SM */
+template __global__ void master_kernel<1, 1024, 2>(MkParams);   /* two scheduling groups per MTB */
+template __global__ void master_kernel<2, 1024, 2>(MkParams);
+template __global__ void master_kernel<4, 512, 2>(MkParams);
 
 /* host side (runtime.cu): the registered 3DES key schedule of this module's MasterKernel */
 cudaError_t set_tdes_const_keys(const void* keys384, uint64_t tables_ptr)
@@ -1890,9 +1904,13 @@ cudaError_t set_dct_const_coef(const void* coef256, uint64_t coef_ptr)
 cudaError_t launch_master(int mtbs_per_sm, int n_mtb, size_t smem_bytes, cudaStream_t stream, MkParams* params,
                           int* regs_out)
 {
-    const void* fn = mtbs_per_sm == 4   ? reinterpret_cast<const void*>(&master_kernel<4, 512>)
-                     : mtbs_per_sm == 2 ? reinterpret_cast<const void*>(&master_kernel<2, 1024>)
-                                        : reinterpret_cast<const void*>(&master_kernel<1, 1024>);
+    const bool g2 = params->n_grp == 2;
+    const void* fn = mtbs_per_sm == 4   ? (g2 ? reinterpret_cast<const void*>(&master_kernel<4, 512, 2>)
+                                              : reinterpret_cast<const void*>(&master_kernel<4, 512, 1>))
+                     : mtbs_per_sm == 2 ? (g2 ? reinterpret_cast<const void*>(&master_kernel<2, 1024, 2>)
+                                              : reinterpret_cast<const void*>(&master_kernel<2, 1024, 1>))
+                                        : (g2 ? reinterpret_cast<const void*>(&master_kernel<1, 1024, 2>)
+                                              : reinterpret_cast<const void*>(&master_kernel<1, 1024, 1>));
     const int threads = mtbs_per_sm == 4 ? 512 : 1024;
     cudaError_t err = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_bytes);
     if (err != cudaSuccess) return err;
