@@ -93,6 +93,8 @@ def parse():
     ap.add_argument("--groups", type=int, default=0, help="scheduling groups per MTB, 1 or 2 (default: the preset's)")
     ap.add_argument("--spread", type=int, default=-1, help="spread-first claims on (1) / off (0) (default: preset)")
     ap.add_argument("--arena-kb", type=int, default=0, help="task arena per MTB in KiB (default: preset)")
+    ap.add_argument("--max-tasks", type=int, default=-1,
+                    help="pagoda_config.max_tasks for the headline workload (-1: its preset)")
     ap.add_argument("--producers", type=int, default=0,
                     help="host spawner threads per step (pagoda_taskSpawnShapesMT; default: preset)")
     ap.add_argument("--task-shmem", type=int, default=-1,
@@ -430,6 +432,9 @@ def ctx_config(a, PG, name):
     ng = a.groups if mine and getattr(a, "groups", 0) else pr.get("sched_groups", 0)
     if ng:
         cfg["sched_groups"] = ng
+    mt = a.max_tasks if mine and getattr(a, "max_tasks", -1) >= 0 else pr.get("max_tasks", 0)
+    if mt:
+        cfg["max_tasks"] = mt
     return cfg
 
 

@@ -76,6 +76,11 @@ typedef struct {
                                block must then fit half an MTB and a task has at most 7 syncing TBs
                                per entry.  The ledger (PAGODA_TRACE) is kept per group: ids
                                mtb * sched_groups + g in pagoda_trace_read / executor records. */
+    uint32_t max_tasks;     /* tasks one scheduling group holds at once (claimed, loaded, running or
+                               posting), 0..32; 0 (default) = as many as its free warps fit plus one
+                               of lookahead.  A small cap leaves the rest in the shared ring for
+                               whichever MTB frees first: uneven task costs (config 1) then spread
+                               over MTBs by completion instead of by claim order */
 } pagoda_config;
 
 /* Fill *cfg with the defaults above. */

@@ -1215,6 +1215,11 @@ __device__ int sched_claim(MtbShared& S, Sched<kG>& st, const MkParams& p)
         if (queued && want < (uint32_t)PAGODA_CLAIM_MIN) want = 0;
     }
     want = min(want, cap);
+    if (p.max_tasks) {   /* pagoda_config.max_tasks: tasks held (task slots taken + tickets not yet loaded) */
+        const uint32_t gslots = kG == 1 ? 0xffffffffu : (0xffffu << (16u * st.g));
+        const uint32_t held = (uint32_t)__popc(gslots & ~st.free_task) + (st.pt - st.pl);
+        want = min(want, p.max_tasks > held ? p.max_tasks - held : 0u);
+    }
     if (want == 0) return 0;
     uint64_t head = 0, tail = 0;
     if (lane == 0) {

@@ -117,6 +117,7 @@ struct MkParams {
     uint32_t     spread_ns;   /* PAGODA_SPREAD: spread-first claim delay per 4 busy warps (0 = off) */
     uint32_t     n_grp;       /* scheduling groups per MTB (1 or 2: pagoda_config.sched_groups) */
     uint32_t     n_exit;      /* holders that exit in a session: n_mtb * n_grp */
+    uint32_t     max_tasks;   /* pagoda_config.max_tasks: cap on the tasks a group holds (0 = none) */
 };
 enum { kLifePub = 0, kLifeLoad, kLifePlace, kLifeStart, kLifeEnd, kLifeDone, kLifeQueued, kLifeFwd };
 

@@ -434,6 +434,7 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
     if (cfg.exec_warps < 1 || cfg.exec_warps > 32) return -EINVAL;
     if (cfg.sched_groups == 0) cfg.sched_groups = 1;
     if (cfg.sched_groups > 2) return -EINVAL;
+    if (cfg.max_tasks > 32) return -EINVAL;
     cfg.exec_warps = std::min(cfg.exec_warps, block_warps);
     if (cfg.arena_bytes % PAGODA_GRANULE || cfg.arena_bytes / PAGODA_GRANULE > (uint32_t)kMaxGranules ||
         cfg.arena_bytes < 2u * 128u * 64u + 8u * PAGODA_GRANULE)   /* ingest staging + room for tasks */
@@ -570,6 +571,7 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
         p.n_mtb = c->n_mtb;
         p.n_grp = (uint32_t)c->n_grp;
         p.n_exit = (uint32_t)(c->n_mtb * c->n_grp);
+        p.max_tasks = cfg.max_tasks;
         if (cfg.flags & PAGODA_TRACE) {
             p.trace_cap = c->cfg.trace_events;
             p.trace = c->trace;

@@ -30,7 +30,7 @@ class pagoda_config(C.Structure):
     _fields_ = [("device", C.c_int), ("mtbs_per_sm", C.c_int), ("num_sms", C.c_int),
                 ("ring_entries", C.c_uint32), ("comp_entries", C.c_uint32), ("arena_bytes", C.c_uint32),
                 ("exec_warps", C.c_uint32), ("flags", C.c_uint32), ("trace_events", C.c_uint32),
-                ("watchdog_s", C.c_double), ("sched_groups", C.c_uint32)]
+                ("watchdog_s", C.c_double), ("sched_groups", C.c_uint32), ("max_tasks", C.c_uint32)]
 
 
 class pagoda_info(C.Structure):

@@ -33,4 +33,6 @@ def ctx_kwargs(workload: str, flags: int = 0) -> dict:
         kw["exec_warps"] = pr["exec_warps"]
     if pr.get("sched_groups"):
         kw["sched_groups"] = pr["sched_groups"]
+    if pr.get("max_tasks"):
+        kw["max_tasks"] = pr["max_tasks"]
     return kw

@@ -73,7 +73,31 @@ def main():
                     gaps["alloc_to_start"].append(ts[i + 1] - a.min())
                     gaps["gap"].append(ts[i + 1] - te[i])
                     gaps["body"].append(te[i] - ts[i])
-        out = {"workload": name, "tasks": n, "session_ms": ms, "tasks_per_s": n / ms * 1e3, "mtbs": info.n_mtb}
+        # concurrency per MTB: time-average number of warps in a body, and the share of the MTB's
+        # active span with 0 / 1 / 2 / 3+ tasks in a body (a task is in its body from its first warp's
+        # start to its last warp's end)
+        warps_busy, occ, span_tot = 0.0, np.zeros(4), 0.0
+        for m in range(info.n_mtb):
+            recs = [r for wp in range(32) for r in ex[m][wp]]
+            if not recs:
+                continue
+            tid = np.array([r["task_id"] for r in recs], np.int64)
+            ts = np.array([int(r["t_start"]) for r in recs], np.int64)
+            te = np.array([int(r["t_end"]) for r in recs], np.int64)
+            warps_busy += float((te - ts).sum())
+            ut = np.unique(tid)
+            st = np.array([ts[tid == u].min() for u in ut]); en = np.array([te[tid == u].max() for u in ut])
+            t0, t1 = st.min(), en.max()
+            span_tot += t1 - t0
+            evs = sorted([(x, 1) for x in st] + [(x, -1) for x in en])
+            cur, last = 0, t0
+            for x, dv in evs:
+                occ[min(cur, 3)] += x - last
+                cur += dv
+                last = x
+        out = {"workload": name, "tasks": n, "session_ms": ms, "tasks_per_s": n / ms * 1e3, "mtbs": info.n_mtb,
+               "exec_warps_busy_share": warps_busy / (info.n_mtb * info.exec_warps * ms * 1e6),
+               "tasks_in_body_share_0_1_2_3plus": [round(float(v / occ.sum()), 3) for v in occ]}
         for k, v in gaps.items():
             v = np.array(v) / 1e3
             out[k] = {"p50_us": float(np.median(v)), "mean_us": float(v.mean()), "n": int(len(v))} if len(v) else None

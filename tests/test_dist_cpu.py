@@ -4,6 +4,7 @@ region, and the reference arm under a 2-rank launch (rank 0 prints one line,
 rank 1 exits without work)."""
 import json
 import os
+import time
 import socket
 import subprocess
 import sys
@@ -112,10 +113,13 @@ def _claims_worker(rank, world, port, q):
         d.barrier()
         cl.reset(step)
         mine, load = [], 0
+        cl.publish(load)
+        d.barrier()   # both ranks start claiming together (a late starter would otherwise find nothing left)
         while True:
             cl.publish(load)
             if PG.pool_may_claim(cl.loads(), rank, 4 * chunk) != 1:
-                load = max(0, load - chunk)   # "completions" drain this rank's load
+                time.sleep(0.002)             # "completions" take time ...
+                load = max(0, load - chunk)   # ... and drain this rank's load
                 continue
             c = cl.claim(step, chunk, n)
             if c is None:
