@@ -589,6 +589,7 @@ def measure(a, d, name, dev, peaks, PG, torch, *, steps, warmup, headline):
     d.barrier()
     torch.cuda.synchronize()
     host_s, dev_ms, mine = [], [], 0
+    ctr0 = p.counters()
     for _ in range(steps):
         t0 = time.perf_counter_ns()
         step()
@@ -611,6 +612,11 @@ def measure(a, d, name, dev, peaks, PG, torch, *, steps, warmup, headline):
                "resident_tdes_keys": bool(use_resident(a, name) and w.tdes_tables and not a.no_const_keys),
                "registered_dct_coef": bool(w.dct_coef and not a.no_const_coef)},
            "task_shmem_bytes": shmem_summary(w)}
+    ctr1 = p.counters()
+    rec["runtime_counters_per_task"] = {   # MasterKernel counters over the timed steps, per task
+        k: (ctr1[k] - ctr0[k]) / max(1, n * steps)
+        for k in ("tickets", "claim_empty", "load_not_ready", "sched_rounds", "handoffs", "place_nofit",
+                  "ingest_batches", "ingest_ring_full")}
     if claims_mode:
         rec["tasks_this_rank_per_step"] = mine / steps
         rec["sharding"] = "runs of 1024 tasks claimed least-loaded-first by each rank's spawner (SharedClaims)"
@@ -831,7 +837,7 @@ def main():
             "host_tasks_per_s": rec["host_tasks_per_s"], "clocks": rec["clocks"]}
     for k in ("p50_spawn_to_done_us", "latency", "naive", "static_fusion", "speedup_vs_naive",
               "speedup_vs_naive_basis", "vs_static_fusion", "nop128_tasks_per_s", "persistent_tasks_per_s",
-              "batching", "roofline", "e2e", "tasks_this_rank_per_step", "sharding"):
+              "batching", "roofline", "e2e", "tasks_this_rank_per_step", "sharding", "runtime_counters_per_task"):
         if k in rec:
             line[k] = rec[k]
     line["cpu_baseline"] = cpu

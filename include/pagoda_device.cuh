@@ -53,7 +53,7 @@ constexpr uint32_t kResidentOffset = 8192;          /* room reserved for the con
 constexpr uint32_t kResidentTdesBytes = 8 * 64 * 32 * 4;   /* 3DES SP tables, one copy per lane */
 constexpr uint32_t kResidentTdesAddr = 8192;        /* shared-WINDOW address of the resident tables: a
                                                        constant, so lookups carry it as an immediate */
-constexpr uint32_t kDevErrorPtrOffset = 5656;       /* MtbShared.dev_error: the device error word's address, for
+constexpr uint32_t kDevErrorPtrOffset = 4736;       /* MtbShared.dev_error: the device error word's address, for
                                                        the paper-named free syncBlock() (which has no TaskEnv) */
 constexpr uint32_t kDevErrSyncWithoutFlag = 1u;     /* == PAGODA_DEVERR_SYNC_WITHOUT_FLAG (pagoda.h) */
 

@@ -34,7 +34,7 @@ enum pagoda_func_id {
     PAGODA_MM   = 18,  /* 32x32x32 fp32 matrix multiply */
     PAGODA_FB   = 19,  /* FilterBank, one channel of 2048 */
     PAGODA_BF   = 20,  /* BeamFormer, 4 ch x 512 complex */
-    PAGODA_CONV = 21,  /* separable 17-tap convolution, 128x128 */
+    PAGODA_CONV = 21,  /* separable 17-tap convolution, 128x128 (row pass through args.scratch, 64 KiB per TB) */
     PAGODA_DCT  = 22,  /* 8x8 DCT-II over 128x128 */
     /* variants */
     PAGODA_MM_TC = 23, /* the MM task on the tensor cores: 3xTF32 mma.sync (args: pagoda_mm_args) */

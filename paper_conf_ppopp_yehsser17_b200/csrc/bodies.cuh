@@ -271,12 +271,43 @@ enum { kTdesResident = 0, kTdesShared = 1, kTdesGlobal = 2 };
 #ifndef PAGODA_TDES_FMA_SUM
 #define PAGODA_TDES_FMA_SUM 1
 #endif
+/* Resident tables hold SP words rotated left by one bit, and the resident rounds keep L and R
+ * rotated the same way (set after IP, undone before FP; rotation commutes with XOR): the S-box
+ * inputs of boxes 7,5,3,1 are then R itself and those of boxes 0,6,4,2 R rotated by 4 (one funnel
+ * shift per round instead of two). */
+#ifndef PAGODA_TDES_ROT
+#define PAGODA_TDES_ROT 1
+#endif
+/* The eight SP words of a round have disjoint bits (P permutes the 32 S-box output bits), so
+ * their XOR is their sum: seven IMADs on the FMA pipe and one XOR with L on the ALU pipe.
+ * Measured slower than four pair sums + two 3-input XORs (33.1 vs 33.7 M tasks/s: the longer
+ * IMAD chain), so off. */
+#ifndef PAGODA_TDES_FULL_SUM
+#define PAGODA_TDES_FULL_SUM 0
+#endif
 static __constant__ uint32_t c_one = 1u;
 __device__ __forceinline__ uint32_t sum_fma_pipe(uint32_t a, uint32_t b)
 {
     uint32_t d;
     asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(c_one), "r"(b));
     return d;
+}
+/* into / out of the resident rounds' rotated domain (PAGODA_TDES_ROT) */
+template <int kMode>
+__device__ __forceinline__ void tdes_rot_in(uint32_t& l, uint32_t& r)
+{
+    if (kMode == kTdesResident && PAGODA_TDES_ROT) {
+        l = __funnelshift_l(l, l, 1);
+        r = __funnelshift_l(r, r, 1);
+    }
+}
+template <int kMode>
+__device__ __forceinline__ void tdes_rot_out(uint32_t& l, uint32_t& r)
+{
+    if (kMode == kTdesResident && PAGODA_TDES_ROT) {
+        l = __funnelshift_r(l, l, 1);
+        r = __funnelshift_r(r, r, 1);
+    }
 }
 
 /* f(R) for table placement kMode.
@@ -290,8 +321,8 @@ template <int kMode>
 __device__ __forceinline__ uint32_t tdes_f(uint32_t r, uint32_t kx, uint32_t ky, uint32_t tb, const uint32_t* sp)
 {
     if (kMode == kTdesResident) {
-        const uint32_t x = (__funnelshift_l(r, r, 5) ^ kx) & 0x3F3F3F3Fu;
-        const uint32_t y = (__funnelshift_l(r, r, 1) ^ ky) & 0x3F3F3F3Fu;
+        const uint32_t x = (__funnelshift_l(r, r, PAGODA_TDES_ROT ? 4 : 5) ^ kx) & 0x3F3F3F3Fu;
+        const uint32_t y = ((PAGODA_TDES_ROT ? r : __funnelshift_l(r, r, 1)) ^ ky) & 0x3F3F3F3Fu;
         const uint32_t t1 = tb | 128u;
         constexpr uint32_t A = kResidentTdesAddr;
         const uint32_t s0 = lds_at<A + 0 * 16384>(__byte_perm(x, tb, 0x7604));
@@ -302,6 +333,12 @@ __device__ __forceinline__ uint32_t tdes_f(uint32_t r, uint32_t kx, uint32_t ky,
         const uint32_t s5 = lds_at<A + 1 * 16384>(__byte_perm(y, t1, 0x7614));
         const uint32_t s6 = lds_at<A + 2 * 16384>(__byte_perm(y, t1, 0x7624));
         const uint32_t s7 = lds_at<A + 3 * 16384>(__byte_perm(y, t1, 0x7634));
+        if (PAGODA_TDES_FULL_SUM == 1)
+            return sum_fma_pipe(sum_fma_pipe(sum_fma_pipe(s0, s1), sum_fma_pipe(s2, s3)),
+                                sum_fma_pipe(sum_fma_pipe(s4, s5), sum_fma_pipe(s6, s7)));
+        if (PAGODA_TDES_FULL_SUM == 2)   /* two quad sums (6 IMAD) + the caller's XOR with l: one LOP3 */
+            return sum_fma_pipe(sum_fma_pipe(s0, s1), sum_fma_pipe(s2, s3)) ^
+                   sum_fma_pipe(sum_fma_pipe(s4, s5), sum_fma_pipe(s6, s7));
         if (PAGODA_TDES_FMA_SUM)   /* 4 IMAD pair sums + the caller's 3-input XORs (with l): 2 LOP3 */
             return sum_fma_pipe(s0, s1) ^ sum_fma_pipe(s2, s3) ^ sum_fma_pipe(s4, s5) ^ sum_fma_pipe(s6, s7);
         return s0 ^ s1 ^ s2 ^ s3 ^ s4 ^ s5 ^ s6 ^ s7;
@@ -359,6 +396,7 @@ __device__ __forceinline__ void tdes_blocks(const Env& e, const pagoda_tdes_args
         /* bytes are the block in FIPS (big-endian) order: L = bytes 0..3, R = bytes 4..7 */
         uint32_t l = __byte_perm(in.x, 0, 0x0123), r = __byte_perm(in.y, 0, 0x0123);
         tdes_ip(l, r);
+        tdes_rot_in<kMode>(l, r);
 #pragma unroll 1
         for (int st = 0; st < 3; st++) {
             const uint32_t kst = kb + st * 128;    /* 16 rounds x 8 bytes per stage */
@@ -381,6 +419,7 @@ __device__ __forceinline__ void tdes_blocks(const Env& e, const pagoda_tdes_args
             l = r;
             r = t;
         }
+        tdes_rot_out<kMode>(l, r);
         tdes_fp(l, r);
         reinterpret_cast<uint2*>(a.out)[blk] = make_uint2(__byte_perm(l, 0, 0x0123), __byte_perm(r, 0, 0x0123));
     }
@@ -409,6 +448,8 @@ __device__ __forceinline__ void tdes_blocks_pair(const Env& e, const pagoda_tdes
         uint32_t l1 = __byte_perm(in1.x, 0, 0x0123), r1 = __byte_perm(in1.y, 0, 0x0123);
         tdes_ip(l0, r0);
         tdes_ip(l1, r1);
+        tdes_rot_in<kTdesResident>(l0, r0);
+        tdes_rot_in<kTdesResident>(l1, r1);
 #pragma unroll 1
         for (int st = 0; st < 3; st++) {
             const uint32_t kst = kb + st * 128;
@@ -428,6 +469,8 @@ __device__ __forceinline__ void tdes_blocks_pair(const Env& e, const pagoda_tdes
             uint32_t t = l0; l0 = r0; r0 = t;
             t = l1; l1 = r1; r1 = t;
         }
+        tdes_rot_out<kTdesResident>(l0, r0);
+        tdes_rot_out<kTdesResident>(l1, r1);
         tdes_fp(l0, r0);
         tdes_fp(l1, r1);
         reinterpret_cast<uint2*>(a.out)[blk] = make_uint2(__byte_perm(l0, 0, 0x0123), __byte_perm(r0, 0, 0x0123));
@@ -737,18 +780,15 @@ __device__ __forceinline__ void discard_l2(const void* line128)
     asm volatile("discard.global.L2 [%0], 128;" ::"l"(line128) : "memory");
 }
 
+/* Row pass over image rows [t0, t1): tmp row y at tmp + (y - base) * 128.  Each thread produces 4
+ * neighbouring outputs with a sliding register window: per tap one new input load, one kernel
+ * load and 4 independent fma chains.  Samples outside the image read as 0, which is exact (an
+ * fma with a zero factor leaves the accumulator unchanged). */
 template <class Env>
-__device__ void body_conv(const Env& e, const pagoda_conv_args& a)
+__device__ __forceinline__ void conv_rows(const Env& e, const pagoda_conv_args& a, float* tmp, int base, int t0, int t1)
 {
-    const int nb = e.getNumBlocks(), j = e.getBlockIdx();
-    const int r0 = (128 * j) / nb, r1 = (128 * (j + 1)) / nb;
-    const int t0 = max(0, r0 - 8), t1 = min(128, r1 + 8);
-    float* tmp = a.scratch + 16384 * j;
     const int n = tb_threads(e), bt = e.getBlockTid();
-    /* Each thread produces 4 neighbouring outputs with a sliding register window: per tap one
-     * new input load, one kernel load and 4 independent fma chains.  Samples outside the image
-     * read as 0, which is exact (an fma with a zero factor leaves the accumulator unchanged). */
-    for (int item = bt; item < (t1 - t0) * 32; item += n) {           /* row pass */
+    for (int item = bt; item < (t1 - t0) * 32; item += n) {
         const int y = t0 + (item >> 5), x0 = (item & 31) * 4;
         const float* row = a.img + y * 128;
         auto in = [&](int xx) { return (xx >= 0 && xx < 128) ? row[xx] : 0.0f; };
@@ -766,13 +806,22 @@ __device__ void body_conv(const Env& e, const pagoda_conv_args& a)
             w2 = w3;
             if (d < 8) w3 = in(x0 + 4 + d);
         }
-        *reinterpret_cast<float4*>(tmp + y * 128 + x0) = make_float4(c0, c1, c2, c3);
+        *reinterpret_cast<float4*>(tmp + (y - base) * 128 + x0) = make_float4(c0, c1, c2, c3);
     }
-    e.syncBlock();
-    const int groups = (r1 - r0 + 3) / 4;
-    for (int item = bt; item < groups * 128; item += n) {             /* column pass */
-        const int x = item & 127, y0 = r0 + (item >> 7) * 4;
-        auto tv = [&](int yy) { return (yy >= 0 && yy < 128) ? tmp[yy * 128 + x] : 0.0f; };
+}
+/* Column pass for output rows [b0, b1) from tmp rows [lo, hi) (at tmp + (y - base) * 128): rows
+ * outside [lo, hi) read as 0.  For an output row in [b0, b1) that is exactly the image's zero
+ * padding ([lo, hi) holds every in-image row within 8 of the band); the rows of a ragged last
+ * group of 4 past b1 are computed from those zeros and dropped. */
+template <class Env>
+__device__ __forceinline__ void conv_cols(const Env& e, const pagoda_conv_args& a, const float* tmp, int base, int lo,
+                                          int hi, int b0, int b1)
+{
+    const int n = tb_threads(e), bt = e.getBlockTid();
+    const int groups = (b1 - b0 + 3) / 4;
+    for (int item = bt; item < groups * 128; item += n) {
+        const int x = item & 127, y0 = b0 + (item >> 7) * 4;
+        auto tv = [&](int yy) { return (yy >= lo && yy < hi) ? tmp[(yy - base) * 128 + x] : 0.0f; };
         float w0 = tv(y0 - 8), w1 = tv(y0 - 7), w2 = tv(y0 - 6), w3 = tv(y0 - 5);
         float c0 = 0.0f, c1 = 0.0f, c2 = 0.0f, c3 = 0.0f;
 #pragma unroll
@@ -788,16 +837,34 @@ __device__ void body_conv(const Env& e, const pagoda_conv_args& a)
             if (d < 8) w3 = tv(y0 + 4 + d);
         }
         float* o = a.out + y0 * 128 + x;
-        if (y0 + 0 < r1) o[0] = c0;       /* rows of another TB's band (or past the image) are */
-        if (y0 + 1 < r1) o[128] = c1;     /* computed from values this TB never wrote: dropped */
-        if (y0 + 2 < r1) o[256] = c2;
-        if (y0 + 3 < r1) o[384] = c3;
+        if (y0 + 0 < b1) o[0] = c0;
+        if (y0 + 1 < b1) o[128] = c1;
+        if (y0 + 2 < b1) o[256] = c2;
+        if (y0 + 3 < b1) o[384] = c3;
     }
+}
+
+/* The row-pass intermediate goes through the TB's global scratch, even when the TB is granted shared
+ * memory: keeping it in the grant band by band (B output rows need B + 16 tmp rows, 512 B each;
+ * the halo rows recomputed per band) was measured slower on config 4 at every threshold tried
+ * (bands of >= 32 rows: 11.5 -> 10.3 M tasks/s; >= 64 rows: 12.7 -> 12.4 M): CONV is bound by
+ * its load latency, not by the scratch round trip through L2. */
+template <class Env>
+__device__ __forceinline__ void body_conv(const Env& e, const pagoda_conv_args& a)
+{
+    const int nb = e.getNumBlocks(), j = e.getBlockIdx();
+    const int r0 = (128 * j) / nb, r1 = (128 * (j + 1)) / nb;
+    const int t0 = max(0, r0 - 8), t1 = min(128, r1 + 8);
+    float* tmp = a.scratch + 16384 * j;
+    conv_rows(e, a, tmp, 0, t0, t1);
+    e.syncBlock();
+    conv_cols(e, a, tmp, 0, 0, 128, r0, r1);   /* rows of [0,128) outside [t0,t1) feed dropped outputs only */
     /* The row-pass rows are dead now.  Written moments ago, they sit dirty in L2; without this
      * they would be written back to HBM on eviction (64 KiB per task, half again the task's
      * algorithmic traffic).  discard.global.L2 drops the lines without a write-back, once every
      * thread of the TB has finished reading them (the barrier). */
     e.syncBlock();
+    const int n = tb_threads(e), bt = e.getBlockTid();
     for (int i = bt; i < (t1 - t0) * 4; i += n) discard_l2(tmp + t0 * 128 + i * 32);
 }
 

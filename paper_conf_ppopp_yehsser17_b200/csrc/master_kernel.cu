@@ -664,12 +664,45 @@ struct IngestCtr {
 /* Publish one staged batch [s, s+n) into the device ring: wait until its cells
  * are free (seq == position: previous occupants loaded), acquire, bulk-store
  * the entries, order them before the cells' release (seq = position + 1). */
+#ifndef PAGODA_EARLY_CHECK
+#define PAGODA_EARLY_CHECK 1  /* publishers check a stage's ring cells from its header, while its bytes cross PCIe */
+#endif
+#ifndef PAGODA_EARLY_EMPTY
+#define PAGODA_EARLY_EMPTY 0  /* a stage is handed back to the loader once the bulk store has READ it, before the
+                                 store completes and the cells are released (the stage's next fill overlaps them) */
+#endif
+/* Wait until the cells of positions [s, s+n) are free (seq == position: previous occupants loaded),
+ * with relaxed loads (the caller's acquire fence completes the pattern).  False on abort. */
+__device__ __forceinline__ bool ingest_check_cells(const MkParams& p, uint64_t s, uint32_t n, IngestCtr& c)
+{
+    const uint32_t lane = threadIdx.x & 31u;
+    for (uint32_t base = 0; base < n;) {   /* 256 cells per round trip (8 loads per lane) */
+        uint32_t sv[8];
+#pragma unroll
+        for (int i = 0; i < 8; i++) {
+            const uint32_t k = base + (uint32_t)i * 32u + lane;
+            sv[i] = k < n ? ld_relaxed_gpu32(&p.dseq[(s + k) & p.ring_mask]) : (uint32_t)(s + k);
+        }
+        uint32_t bad = 0;
+#pragma unroll
+        for (int i = 0; i < 8; i++) bad |= __ballot_sync(0xffffffffu, sv[i] != (uint32_t)(s + base + (uint32_t)i * 32u + lane));
+        if (bad) {
+            c.full++;
+            if (*(volatile uint32_t*)&p.dctl->stop == kStopAbort) return false;
+            __nanosleep(128);
+            continue;
+        }
+        base += 256u;
+    }
+    return true;
+}
+
 __device__ __forceinline__ bool ingest_publish(const MkParams& p, const char* src, uint64_t s, uint32_t n,
-                                               IngestCtr& c)
+                                               IngestCtr& c, uint64_t* empty_bar = nullptr, bool checked = false)
 {
     const uint32_t lane = threadIdx.x & 31u;
     const uint64_t R = (uint64_t)p.ring_mask + 1;
-    for (uint32_t base = 0; base < n;) {   /* 256 cells per round trip (8 loads per lane) */
+    for (uint32_t base = checked ? n : 0u; base < n;) {   /* 256 cells per round trip (8 loads per lane) */
         uint32_t sv[8];
 #pragma unroll
         for (int i = 0; i < 8; i++) {
@@ -691,7 +724,7 @@ __device__ __forceinline__ bool ingest_publish(const MkParams& p, const char* sr
         }
         base += 256u;
     }
-    if (PAGODA_FAST_PUB) fence_acq_rel_gpu();   /* acquire pattern: relaxed reads of the cells, then this fence */
+    if (PAGODA_FAST_PUB || checked) fence_acq_rel_gpu();   /* acquire pattern: relaxed reads of the cells, then this fence */
     const uint64_t t3 = globaltimer_ns();
     __syncwarp();          /* every lane's acquire precedes lane 0's bulk store */
     const uint64_t t4 = globaltimer_ns();
@@ -702,7 +735,12 @@ __device__ __forceinline__ bool ingest_publish(const MkParams& p, const char* sr
         const uint32_t n1 = min(n, (uint32_t)(R - e0));
         tma_store_1d(p.dring + e0, src, n1 * 64u);
         if (n1 < n) tma_store_1d(p.dring, src + n1 * 64u, (n - n1) * 64u);
-        asm volatile("cp.async.bulk.commit_group;\n\tcp.async.bulk.wait_group 0;" ::: "memory");
+        asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+        if (empty_bar) {   /* the stage's bytes have been read: the loader may refill it now */
+            asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+            mbar_arrive(empty_bar);
+        }
+        asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
         asm volatile("fence.proxy.async.global;" ::: "memory");
     }
     __syncwarp();
@@ -870,6 +908,8 @@ __device__ void ingest_loader(MtbShared& S, const MkParams& p, char* stage_buf)
             if (end) {   /* one end marker per publisher, in its next stage */
                 if (lane == 0) {
                     S.ing_n[b] = ~0u;
+                    __threadfence_block();
+                    *(volatile uint32_t*)&S.ing_hdr[b] = k;   /* k was incremented above: stage k - 1 */
                     mbar_arrive(&S.ingest_bar[b]);
                 }
                 if (++ends == kIngestPublishers) break;
@@ -879,6 +919,8 @@ __device__ void ingest_loader(MtbShared& S, const MkParams& p, char* stage_buf)
             if (lane == 0) {
                 S.ing_start[b] = fetched;
                 S.ing_n[b] = n;
+                __threadfence_block();
+                *(volatile uint32_t*)&S.ing_hdr[b] = k;   /* stage k - 1's header: its publisher checks the cells */
             }
             ingest_load(p, stage_buf + b * (SE * 64u), fetched, n, &S.ingest_bar[b]);
             fetched += n;
@@ -932,6 +974,29 @@ __device__ __noinline__ void ingest_publisher(MtbShared& S, const MkParams& p, c
     for (uint32_t k = me;; k += kIngestPublishers) {   /* my stages: me, me + P, ... */
         const uint32_t b = k % kIngestStages;
         const uint64_t t1 = globaltimer_ns();
+        bool checked = false;
+        if (PAGODA_EARLY_CHECK) {
+            /* the stage's header arrives before its bytes: check its cells while the host read is in
+             * flight (the round trip leaves the publish chain); the acquire fence follows the load */
+            while (*(volatile uint32_t*)&S.ing_hdr[b] != k + 1u) {
+                if (*(volatile uint32_t*)&p.dctl->stop == kStopAbort) {
+                    aborted = true;
+                    break;
+                }
+                __nanosleep(32);
+            }
+            if (aborted) break;
+            __syncwarp();
+            __threadfence_block();   /* the header's fields after the header */
+            const uint32_t n0 = *(volatile uint32_t*)&S.ing_n[b];
+            if (n0 != ~0u) {
+                if (!ingest_check_cells(p, *(volatile uint64_t*)&S.ing_start[b], n0, c)) {
+                    aborted = true;
+                    break;
+                }
+                checked = true;
+            }
+        }
         while (!mbar_try_wait(&S.ingest_bar[b], (k / kIngestStages) & 1u, 20000u)) {
             if (*(volatile uint32_t*)&p.dctl->stop == kStopAbort) {
                 aborted = true;
@@ -944,12 +1009,13 @@ __device__ __noinline__ void ingest_publisher(MtbShared& S, const MkParams& p, c
         if (n == ~0u) break;
         c.ns_copy += t2 - t1;
         const uint64_t s = *(volatile uint64_t*)&S.ing_start[b];
-        if (!ingest_publish(p, stage_buf + b * (SE * 64u), s, n, c)) {
+        if (!ingest_publish(p, stage_buf + b * (SE * 64u), s, n, c, PAGODA_EARLY_EMPTY ? &S.ingest_empty[b] : nullptr,
+                            checked)) {
             aborted = true;
             break;
         }
         ingest_finish(S, k, s + n);
-        if (lane == 0) mbar_arrive(&S.ingest_empty[b]);
+        if (!PAGODA_EARLY_EMPTY && lane == 0) mbar_arrive(&S.ingest_empty[b]);
         c.ns_pub += globaltimer_ns() - t2;
     }
     if (lane == 0) {
@@ -1791,7 +1857,8 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) master_kernel(MkParams p
             for (uint32_t i = threadIdx.x; i < kResidentTdesBytes / 4; i += blockDim.x) {
                 const uint32_t pr = i >> 12, v = (i >> 6) & 63u, h = (i >> 5) & 1u;
                 const uint32_t j = h ? 7u - 2u * pr : (8u - 2u * pr) & 7u;
-                dst[i] = __ldg(p.resident_tdes_src + j * 64u + v);
+                const uint32_t w = __ldg(p.resident_tdes_src + j * 64u + v);
+                dst[i] = PAGODA_TDES_ROT ? __funnelshift_l(w, w, 1) : w;   /* the rounds' rotated domain */
             }
         } else if (threadIdx.x == 0) {
             atomicOr(&p.dctl->error, PAGODA_DEVERR_LAYOUT);   /* bodies fall back to per-task tables */
@@ -1826,6 +1893,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) master_kernel(MkParams p
         if (lane < kIngestStages) {
             mbar_init(&S.ingest_bar[lane], 1);
             mbar_init(&S.ingest_empty[lane], 1);
+            S.ing_hdr[lane] = 0;
         }
         for (uint32_t i = lane; i < kIngestFinSlots; i += 32u) S.ing_fin[i] = 0;
         /* initial scheduler state of each group, owned by its first worker (it starts with the token) */

@@ -209,6 +209,7 @@ struct MtbShared {
     uint16_t  tb_idx[32];            /* 4288: TB index j of each TB record (ledger) */
     uint64_t  pend_ticket[32];       /* 4352: claimed ring positions, FIFO (pend[] holds their slots once loaded) */
     uint32_t  stage_ph[32];          /* 4608: parity of each warp's staging mbarrier (TaskEnv::stage) */
+    uint32_t* dev_error;             /* 4736: &DevCtl.error, for the paper-named free syncBlock() (kDevErrorPtrOffset) */
     uint32_t  ingest_done;           /* MTB 0: the ingest warps have exited */
     uint32_t  no_tickets;            /* this MTB runs no tasks (MTB 0 and the MTB sharing its SM) */
     uint64_t  ingest_copied;         /* MTB 0: entries published into the device ring, a prefix (host poster) */
@@ -217,6 +218,7 @@ struct MtbShared {
     uint64_t  ingest_empty[kIngestStages];  /* stage s free again (publisher -> loader) */
     uint64_t  ing_start[kIngestStages];     /* first ring position of the batch in stage s */
     uint32_t  ing_n[kIngestStages];         /* entries in stage s (~0: end of stream) */
+    uint32_t  ing_hdr[kIngestStages];       /* k + 1 once stage k's start / n are written (before its load lands) */
     uint64_t  ing_fin_end[kIngestFinSlots]; /* stage k published: its end position ... */
     uint32_t  ing_fin[kIngestFinSlots];     /* ... and k + 1, in slot k mod kIngestFinSlots */
     uint32_t  ing_prefix_k;                 /* stages [0, k) all published (ingest_copied is their end) */
@@ -224,7 +226,6 @@ struct MtbShared {
     uint32_t  ing_pubs_done;                /* publishers that saw their end marker */
     uint32_t  fwd_done;              /* MTB 0: forwarders that exited */
     unsigned long long dq_safe;      /* completion-queue positions below this are known free (posters' cache) */
-    uint32_t* dev_error;             /* &DevCtl.error, for the paper-named free syncBlock() (kDevErrorPtrOffset) */
     SchedGroup grp[kMaxSchedGroups]; /* the MTB's scheduling groups (one unless PAGODA_config.sched_groups = 2) */
 };
 static_assert(offsetof(MtbShared, wt) == kWarpTableOffset, "WarpTable offset");

@@ -6,7 +6,9 @@ full-size parity tests so that they run in exactly that configuration."""
 # keys in bench.py); spread: PAGODA_SPREAD; producers: host spawner threads per step
 PRESETS = {
     "tdes": {"mtbs_per_sm": 2, "arena_bytes": 40 * 1024, "resident": True},
-    "mb": {"mtbs_per_sm": 1, "arena_bytes": 96 * 1024, "resident": False, "spread": True},   # 4.2 vs 3.8 M at 2
+    # MB: 1 MTB/SM (64 registers), at most 2 tasks held per MTB: the rest wait in the ring for whichever MTB
+    # frees first, so the saturated tiles spread by completion (4.75 M vs 4.27 M with spread-first claims)
+    "mb": {"mtbs_per_sm": 1, "arena_bytes": 96 * 1024, "resident": False, "max_tasks": 2},
     "mm": {"mtbs_per_sm": 4, "arena_bytes": 48 * 1024, "resident": False},   # 512-thread MTBs: 2x schedulers
     "mix": {"mtbs_per_sm": 1, "arena_bytes": 200 * 1024, "resident": False},
     "nop": {"mtbs_per_sm": 2, "arena_bytes": 96 * 1024, "resident": False, "producers": 2},

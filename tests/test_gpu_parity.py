@@ -42,9 +42,11 @@ def run(w, **cfg):
 
 
 # ---------------------------------------------------------------- MB (config 1)
-# 2 and 1 MTBs per SM (32 / 64 registers per thread), and spread-first claims (the bench preset)
+# 2 and 1 MTBs per SM (32 / 64 registers per thread), spread-first claims, claim caps (max_tasks: 1 per
+# MTB, and 2 per MTB at 1 MTB/SM = the bench preset)
 MB_CFGS = [{}, {"mtbs_per_sm": 1, "arena_bytes": 96 * 1024}, {"flags": 0x10},   # 0x10: PAGODA_SPREAD
-           {"mtbs_per_sm": 1, "arena_bytes": 96 * 1024, "flags": 0x10}]          # the bench preset
+           {"mtbs_per_sm": 1, "arena_bytes": 96 * 1024, "flags": 0x10}, {"max_tasks": 1},
+           ctx_kwargs("mb")]
 
 
 @pytest.mark.parametrize("cfg", MB_CFGS)

@@ -256,11 +256,13 @@ def test_chain_visibility():
     assert np.array_equal(Dev.get(mats[30], np.float32, (32, 32)), A0)
 
 
-def test_ledger_invariants_debug_config():
+@pytest.mark.parametrize("max_tasks", [0, 2])
+def test_ledger_invariants_debug_config(max_tasks):
     """Trace mode on a small grid with few executor warps and a small arena:
     the oracle-side checker replays every MTB's allocator events (no double
     assignment of warps / granules / barrier IDs, frees match allocs, every
-    TB allocated once on one MTB, everything freed)."""
+    TB allocated once on one MTB, everything freed).  With a claim cap
+    (pagoda_config.max_tasks) no MTB ever runs more than that many tasks at once."""
     import oracle
     rng = np.random.default_rng(5)
     alphabet = [(32, 1, 0, 0), (64, 1, 0, 1), (128, 1, 0, 1), (32, 1, 512, 0), (64, 1, 2048, 1), (128, 1, 4096, 1),
@@ -269,7 +271,7 @@ def test_ledger_invariants_debug_config():
     err = dev.zeros(8)
     n = 1500
     with Pagoda(num_sms=2, mtbs_per_sm=1, exec_warps=8, arena_bytes=16 * 1024 + 16384, flags=TRACE,
-                trace_events=16384) as p:
+                trace_events=16384, max_tasks=max_tasks) as p:
         info = p.info()
         meta = []
         for k in range(n):
@@ -295,6 +297,20 @@ def test_ledger_invariants_debug_config():
             s = np.sort(e, order="t_start")
             assert (s["t_start"][1:] >= s["t_end"][:-1]).all()
     assert sum(len(e) for e in ex) == sum(m[1] for m in meta)
+    if max_tasks:   # tasks in a body at once, per MTB (a task: its first warp's start to its last warp's end)
+        for m in range(info.n_mtb):
+            recs = np.concatenate(ex[m * 32:(m + 1) * 32])
+            if len(recs) == 0:
+                continue
+            ids = np.unique(recs["task_id"])
+            st = np.array([recs["t_start"][recs["task_id"] == i].min() for i in ids], np.int64)
+            en = np.array([recs["t_end"][recs["task_id"] == i].max() for i in ids], np.int64)
+            evs = sorted([(int(x), 1) for x in st] + [(int(x), -1) for x in en], key=lambda e: (e[0], e[1]))
+            cur = peak = 0
+            for _, dv in evs:
+                cur += dv
+                peak = max(peak, cur)
+            assert peak <= max_tasks, (m, peak)
 
 
 def test_sessions_stop_start_and_drain():

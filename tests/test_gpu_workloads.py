@@ -140,3 +140,4 @@ def test_conv_large_tasks(threads, n_tb, shmem):
     assert (w.shapes[:, 1] == n_tb).all()
     run(w)
     assert check_tasks(w, range(12)) == {"conv"}
+
