@@ -665,7 +665,7 @@ struct IngestCtr {
  * are free (seq == position: previous occupants loaded), acquire, bulk-store
  * the entries, order them before the cells' release (seq = position + 1). */
 #ifndef PAGODA_EARLY_CHECK
-#define PAGODA_EARLY_CHECK 1  /* publishers check a stage's ring cells from its header, while its bytes cross PCIe */
+#define PAGODA_EARLY_CHECK 0  /* (measured neutral) publishers check a stage's ring cells from its header, while its bytes cross PCIe */
 #endif
 #ifndef PAGODA_EARLY_EMPTY
 #define PAGODA_EARLY_EMPTY 0  /* a stage is handed back to the loader once the bulk store has READ it, before the
