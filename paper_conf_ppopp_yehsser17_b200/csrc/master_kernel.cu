@@ -74,6 +74,9 @@
 #ifndef PAGODA_DIRECT_IDLE_NS
 #define PAGODA_DIRECT_IDLE_NS 50000   /* ... or when the group posted nothing for this long (lone tasks) */
 #endif
+#ifndef PAGODA_FREE_BEFORE_POST
+#define PAGODA_FREE_BEFORE_POST 1  /* a task's last warp frees itself before posting the completion record */
+#endif
 #ifndef PAGODA_HOLDER_POSTS
 #define PAGODA_HOLDER_POSTS 0 /* the scheduler token holder posts completion records (batched per round);
                                  the last warp of a task only marks it pending and frees itself */
@@ -594,15 +597,29 @@ __device__ __forceinline__ void run_task(MtbShared& S, SchedGroup& G, char* smem
         }
     }
     pf_add(G, kPfFence, tp, true);
+    if (PAGODA_FREE_BEFORE_POST) {
+        /* the warp is free for the next task before it posts: the post (a GPU fence and a queue
+         * reservation, ~3 us under load) overlaps the next placement and wake-up instead of holding
+         * the slot's warps.  Its WarpTable slot may be rewritten meanwhile; the post reads task
+         * slots only (returned after it), and the holder does not exit while a post is running. */
+        if (lane == 0) {
+            __threadfence_block();
+            atomicOr(&G.mb_warps, 1u << w);
+            __threadfence_block();
+        }
+        __syncwarp();
+    }
     tp = pf_now();
     if (!PAGODA_HOLDER_POSTS && __shfl_sync(0xffffffffu, last, 0)) post_completions(S, G, p);
     pf_add(G, kPfPost, tp, true);
-    if (lane == 0) {
-        __threadfence_block();   /* TB / task frees are visible before the warp frees itself */
-        atomicOr(&G.mb_warps, 1u << w);
-        __threadfence_block();   /* ... and the warp's free bit before its attempt at the token */
+    if (!PAGODA_FREE_BEFORE_POST) {
+        if (lane == 0) {
+            __threadfence_block();   /* TB / task frees are visible before the warp frees itself */
+            atomicOr(&G.mb_warps, 1u << w);
+            __threadfence_block();   /* ... and the warp's free bit before its attempt at the token */
+        }
+        __syncwarp();
     }
-    __syncwarp();
 }
 
 /* MTB 0's host poster (n_mtb > 1): the ingest warp's host-visible stores
@@ -656,6 +673,10 @@ __device__ __forceinline__ void tma_store_1d(void* gdst, const void* smem_src, u
                  : "memory");
 }
 
+#ifndef PAGODA_INGEST_TIMERS
+#define PAGODA_INGEST_TIMERS 1   /* ingest phase timers (PAGODA_CTR_INGEST_NS_*) */
+#endif
+__device__ __forceinline__ uint64_t ing_now() { return PAGODA_INGEST_TIMERS ? globaltimer_ns() : 0; }
 struct IngestCtr {
     unsigned long long batches = 0, entries = 0, ns_db = 0, ns_copy = 0, ns_pub = 0, full = 0, ns_fence = 0,
                        ns_store = 0;
@@ -725,9 +746,9 @@ __device__ __forceinline__ bool ingest_publish(const MkParams& p, const char* sr
         base += 256u;
     }
     if (PAGODA_FAST_PUB || checked) fence_acq_rel_gpu();   /* acquire pattern: relaxed reads of the cells, then this fence */
-    const uint64_t t3 = globaltimer_ns();
+    const uint64_t t3 = ing_now();
     __syncwarp();          /* every lane's acquire precedes lane 0's bulk store */
-    const uint64_t t4 = globaltimer_ns();
+    const uint64_t t4 = ing_now();
     if (lane == 0) {
         asm volatile("fence.proxy.async.global;" ::: "memory");   /* generic acquire -> async-proxy writes */
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
@@ -744,9 +765,9 @@ __device__ __forceinline__ bool ingest_publish(const MkParams& p, const char* sr
         asm volatile("fence.proxy.async.global;" ::: "memory");
     }
     __syncwarp();
-    const uint64_t t5 = globaltimer_ns();
+    const uint64_t t5 = ing_now();
     fence_acq_rel_gpu();   /* the entry writes precede every lane's relaxed cell release */
-    const uint64_t t6 = globaltimer_ns();
+    const uint64_t t6 = ing_now();
     c.ns_fence += (t4 - t3) + (t6 - t5);
     c.ns_store += t5 - t4;
     for (uint32_t i = lane; i < n; i += 32u) {
@@ -767,7 +788,7 @@ __device__ __forceinline__ void ingest_doorbell(const MkParams& p, uint64_t& pub
                                                 bool post_err, IngestCtr& c, uint64_t fetched)
 {
     const uint32_t lane = threadIdx.x & 31u;
-    const uint64_t t0 = globaltimer_ns();
+    const uint64_t t0 = ing_now();
     uint32_t err = 0;
     if (lane == 0) {
         pub = ld_acquire_sys(&p.hctl->published);
@@ -783,7 +804,7 @@ __device__ __forceinline__ void ingest_doorbell(const MkParams& p, uint64_t& pub
     pub = __shfl_sync(0xffffffffu, pub, 0);
     term = __shfl_sync(0xffffffffu, term, 0);
     last_err = __shfl_sync(0xffffffffu, err, 0);
-    c.ns_db += globaltimer_ns() - t0;
+    c.ns_db += ing_now() - t0;
 }
 
 /* issue the bulk copy of host ring entries [f, f+n) into a stage (lane 0) */
@@ -846,15 +867,15 @@ __device__ void ingest(MtbShared& S, const MkParams& p, char* stage_buf, uint64_
             idle = 0;
         }
         if (inflight) {
-            const uint64_t t1 = globaltimer_ns();
+            const uint64_t t1 = ing_now();
             mbar_wait(&bars[os], (phase >> os) & 1u);
             phase ^= 1u << os;
-            const uint64_t t2 = globaltimer_ns();
+            const uint64_t t2 = ing_now();
             c.ns_copy += t2 - t1;
             if (!ingest_publish(p, stage_buf + os * (SE * 64u), st_start[os], st_n[os], c)) break;
             copied = st_start[os] + st_n[os];
             if (lane == 0) st_relaxed_sys(&p.hctl->consumed, copied);   /* host may reuse those ring slots */
-            c.ns_pub += globaltimer_ns() - t2;
+            c.ns_pub += ing_now() - t2;
             inflight--;
             os ^= 1u;
         } else if (term) {
@@ -973,7 +994,7 @@ __device__ __noinline__ void ingest_publisher(MtbShared& S, const MkParams& p, c
     IngestCtr c;
     for (uint32_t k = me;; k += kIngestPublishers) {   /* my stages: me, me + P, ... */
         const uint32_t b = k % kIngestStages;
-        const uint64_t t1 = globaltimer_ns();
+        const uint64_t t1 = ing_now();
         bool checked = false;
         if (PAGODA_EARLY_CHECK) {
             /* the stage's header arrives before its bytes: check its cells while the host read is in
@@ -1004,7 +1025,7 @@ __device__ __noinline__ void ingest_publisher(MtbShared& S, const MkParams& p, c
             }
         }
         if (aborted) break;
-        const uint64_t t2 = globaltimer_ns();
+        const uint64_t t2 = ing_now();
         const uint32_t n = *(volatile uint32_t*)&S.ing_n[b];
         if (n == ~0u) break;
         c.ns_copy += t2 - t1;
@@ -1016,7 +1037,7 @@ __device__ __noinline__ void ingest_publisher(MtbShared& S, const MkParams& p, c
         }
         ingest_finish(S, k, s + n);
         if (!PAGODA_EARLY_EMPTY && lane == 0) mbar_arrive(&S.ingest_empty[b]);
-        c.ns_pub += globaltimer_ns() - t2;
+        c.ns_pub += ing_now() - t2;
     }
     if (lane == 0) {
         /* the last publisher out: every stage was published (each saw its end marker after its
@@ -1687,8 +1708,18 @@ __device__ bool sched_round(MtbShared& S, Sched<kG>& st, const MkParams& p, int 
     exit = false;
     sc_add(S.grp[st.g], kScRounds, 1);
     if (progress) sc_add(S.grp[st.g], kScProgress, 1);
-    if (!progress && st.free_w == st.exec_mask && st.ph == st.pl &&
-        *(volatile uint32_t*)&S.grp[st.g].comp_pending == 0u) {
+    bool quiet = !progress && st.free_w == st.exec_mask && st.ph == st.pl;
+    if (quiet) {   /* no completion pending, and (FREE_BEFORE_POST) none being posted: pending is read first,
+                      a poster clears it only while holding the poster flag */
+        uint32_t q = 0;
+        if (lane == 0) {
+            q = *(volatile uint32_t*)&S.grp[st.g].comp_pending == 0u;
+            __threadfence_block();
+            if (PAGODA_FREE_BEFORE_POST) q = q && *(volatile uint32_t*)&S.grp[st.g].poster == 0u;
+        }
+        quiet = __shfl_sync(0xffffffffu, q, 0) != 0;
+    }
+    if (quiet) {
         uint32_t stop = 0;
         if (lane == 0) stop = ld_acquire_gpu32(&p.dctl->stop);
         stop = __shfl_sync(0xffffffffu, stop, 0);
