@@ -93,6 +93,8 @@ def parse():
     ap.add_argument("--groups", type=int, default=0, help="scheduling groups per MTB, 1 or 2 (default: the preset's)")
     ap.add_argument("--spread", type=int, default=-1, help="spread-first claims on (1) / off (0) (default: preset)")
     ap.add_argument("--arena-kb", type=int, default=0, help="task arena per MTB in KiB (default: preset)")
+    ap.add_argument("--ce", type=int, default=-1,
+                    help="copy-engine ingest (PAGODA_CE_INGEST) on (1) / off (0) for the headline workload (-1: preset)")
     ap.add_argument("--max-tasks", type=int, default=-1,
                     help="pagoda_config.max_tasks for the headline workload (-1: its preset)")
     ap.add_argument("--producers", type=int, default=0,
@@ -432,6 +434,9 @@ def ctx_config(a, PG, name):
     ng = a.groups if mine and getattr(a, "groups", 0) else pr.get("sched_groups", 0)
     if ng:
         cfg["sched_groups"] = ng
+    ce = (a.ce == 1) if mine and getattr(a, "ce", -1) >= 0 else bool(pr.get("ce"))
+    if ce:
+        cfg["flags"] |= PG.CE_INGEST
     mt = a.max_tasks if mine and getattr(a, "max_tasks", -1) >= 0 else pr.get("max_tasks", 0)
     if mt:
         cfg["max_tasks"] = mt
@@ -608,7 +613,8 @@ def measure(a, d, name, dev, peaks, PG, torch, *, steps, warmup, headline):
            "host_ms_per_step": 1e3 * host_total / steps, "host_tasks_per_s": job_tasks / host_total,
            "clocks": clk, "mtbs": info.n_mtb, "regs_per_thread": info.regs_per_thread, "producers": producers,
            "context": {k: v for k, v in cfg.items() if k != "flags"} | {
-               "resident_tdes_tables": use_resident(a, name), "spread_first_claims": bool(PRESETS[name].get("spread")),
+               "resident_tdes_tables": use_resident(a, name), "spread_first_claims": bool(cfg["flags"] & PG.SPREAD),
+               "ingest": "copy engine (PAGODA_CE_INGEST)" if cfg["flags"] & PG.CE_INGEST else "doorbell + MTB 0 warps",
                "resident_tdes_keys": bool(use_resident(a, name) and w.tdes_tables and not a.no_const_keys),
                "registered_dct_coef": bool(w.dct_coef and not a.no_const_coef)},
            "task_shmem_bytes": shmem_summary(w)}

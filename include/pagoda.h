@@ -48,6 +48,12 @@ typedef int64_t pagoda_task_t;          /* >= 0: task id; < 0: -errno */
                                       4 warps), so few, uneven tasks (config 1) go to the idlest MTBs */
 #define PAGODA_LIFECYCLE     0x8u /* stamp every task's life cycle on the GPU clock (profiling; 64 B per
                                      completion slot): see pagoda_lifecycle_read */
+#define PAGODA_CE_INGEST     0x40u /* copy-engine ingest: a host thread of the context copies newly published
+                                     TaskTable entries into the device ring with cudaMemcpyAsync and
+                                     publishes the device ring's tail with a stream memory operation
+                                     (cuStreamWriteValue64, ordered after the copy), instead of MTB 0's
+                                     warps pulling entries over PCIe; MTB 0 keeps a scanner warp that
+                                     reports which ring cells the schedulers have handed back */
 #define PAGODA_NONBLOCKING_SPAWN 0x20u /* taskSpawn returns -EAGAIN instead of waiting when the TaskTable
                                      ring slot or completion slot a new task needs is still taken
                                      (the paper's CPU waits for a free entry) */
@@ -55,7 +61,9 @@ typedef int64_t pagoda_task_t;          /* >= 0: task id; < 0: -errno */
 typedef struct {
     int      device;        /* CUDA device ordinal (default 0) */
     int      mtbs_per_sm;   /* MasterKernel thread blocks (MTBs) per SM: 1 or 2 (1024 threads each; default 2,
-                               P:453-455) or 4 (512 threads each: twice the schedulers per SM; arena <= 48 KiB) */
+                               P:453-455), 4 (512 threads each: twice the schedulers per SM; arena <= 48 KiB) or
+                               8 (256 threads each: one 8-warp task per MTB; arena <= 21 KiB; the doorbell
+                               ingest's stages are then small: use PAGODA_CE_INGEST) */
     int      num_sms;       /* SMs to occupy, 0 = all (148 on B200) */
     uint32_t ring_entries;  /* TaskTable ring entries, host and device, power of 2 (default 65536) */
     uint32_t comp_entries;  /* completion window, power of 2 >= ring_entries (default 1<<20) */

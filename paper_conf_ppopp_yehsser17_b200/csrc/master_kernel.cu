@@ -25,7 +25,7 @@
 #define PAGODA_IDLE_NS 1024   /* longest back-off of an idle scheduler / I/O warp between polls */
 #endif
 #ifndef PAGODA_CTA_FENCE
-#define PAGODA_CTA_FENCE 0    /* executors release with a CTA-scope fence (the poster's GPU fence covers them) */
+#define PAGODA_CTA_FENCE 1    /* executors release with a CTA-scope fence (the poster's GPU fence covers them) */
 #endif
 #ifndef PAGODA_CLAIM_FIRST
 #define PAGODA_CLAIM_FIRST 0  /* a scheduling round claims before it loads: fresh tickets load in the same round */
@@ -636,7 +636,7 @@ __device__ void host_poster(MtbShared& S, const MkParams& p)
         const uint32_t exited = *(volatile uint32_t*)&p.dctl->exited;
         const uint64_t c = *(volatile uint64_t*)&S.ingest_copied;
         const uint32_t err = *(volatile uint32_t*)&p.dctl->error;
-        if (c != last) {
+        if (c != last && !p.ce_ingest) {   /* (CE ingest: the copy stream writes consumed) */
             st_relaxed_sys(&p.hctl->consumed, c);
             last = c;
         }
@@ -1051,6 +1051,61 @@ __device__ __noinline__ void ingest_publisher(MtbShared& S, const MkParams& p, c
     ingest_flush(p, c);
 }
 
+/* PAGODA_CE_INGEST: MTB 0's scanner warp (in place of the ingest warps).  The host's copy stream
+ * overwrites a device ring cell only once the ticket of the previous lap handed it back
+ * (seq = position + R, stored by the scheduler after it copied the cell); this warp follows the
+ * hand-backs in ring order and posts their contiguous prefix to the host (HostCtl.handed), 256
+ * cells per L2 round trip.  With one MTB it also posts the device error word.  Exits once every
+ * scheduler exited. */
+__device__ void ce_scanner(const MkParams& p)
+{
+    const uint32_t lane = threadIdx.x & 31u;
+    const uint64_t R = (uint64_t)p.ring_mask + 1;
+    uint64_t P = p.ce_base, posted = ~0ull;
+    uint32_t idle = 0, last_err = 0;
+    for (;;) {
+        uint32_t v[8];
+#pragma unroll
+        for (int i = 0; i < 8; i++) v[i] = ld_relaxed_gpu32(&p.dseq[(P + (uint64_t)i * 32u + lane) & p.ring_mask]);
+        uint32_t n = 0;
+        bool gap = false;
+#pragma unroll
+        for (int i = 0; i < 8; i++) {
+            const uint32_t ok = __ballot_sync(0xffffffffu, v[i] == (uint32_t)(P + (uint64_t)i * 32u + lane + R));
+            if (!gap) {
+                if (ok == 0xffffffffu) n += 32u;
+                else {
+                    n += (uint32_t)__ffs(~ok) - 1u;
+                    gap = true;
+                }
+            }
+        }
+        P += n;
+        if (lane == 0) {
+            if (P != posted && (n == 0 || P - posted >= 1024u || posted == ~0ull)) {
+                st_relaxed_sys(reinterpret_cast<volatile uint64_t*>(&p.hctl->handed), P);
+                posted = P;
+            }
+            if (p.n_mtb == 1) {
+                const uint32_t err = *(volatile uint32_t*)&p.dctl->error;
+                if (err != last_err) {
+                    st_relaxed_sys32(&p.hctl->error, err);
+                    last_err = err;
+                }
+            }
+        }
+        if (n) {
+            idle = 0;
+            continue;
+        }
+        uint32_t done = 0;
+        if (lane == 0) done = ld_acquire_gpu32(&p.dctl->exited) >= p.n_exit;
+        if (__shfl_sync(0xffffffffu, done, 0)) break;
+        __nanosleep(idle < 16 ? 128 : min(1024, PAGODA_IDLE_NS));
+        idle++;
+    }
+}
+
 /* ------------------------------------------------------------------ scheduler
  * Alg. 1 L1-28 + Alg. 2, re-designed: one warp per MTB owns the
  * MTB's free masks (warps, TB records, task slots, barrier IDs: one word each;
@@ -1358,7 +1413,12 @@ __device__ int sched_load(MtbShared& S, Sched<kG>& st, const MkParams& p)
     const uint32_t n = min(st.pt - st.pl, (uint32_t)__popc(st.free_task));
     if (n == 0) return 0;
     bool ready = false;
-    if (lane < n) {
+    if (p.ce_ingest) {   /* published = below the tail the copy stream wrote after the copy (acquire) */
+        uint64_t tail = 0;
+        if (lane == 0) tail = ld_acquire_gpu(&p.dctl->tail);
+        tail = __shfl_sync(0xffffffffu, tail, 0);
+        if (lane < n) ready = S.pend_ticket[fq(st, st.pl + lane)] < tail;
+    } else if (lane < n) {
         const uint64_t t = S.pend_ticket[fq(st, st.pl + lane)];
         ready = ld_acquire_gpu32(&p.dseq[t & p.ring_mask]) == (uint32_t)(t + 1);
     }
@@ -1964,7 +2024,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) master_kernel(MkParams p
             /* where ingest resumes: the host poster must never post a smaller consumed count
              * (a spawn blocked on a ring slot would wait for it forever) */
             S.ingest_copied = *(volatile uint64_t*)&p.dctl->tail;
-            S.ingest_done = 0;
+            S.ingest_done = p.ce_ingest ? 1u : 0u;   /* (CE ingest: no ingest warps) */
             S.ing_prefix_k = 0;
             S.ing_lock = 0;
             S.ing_pubs_done = 0;
@@ -1972,10 +2032,12 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) master_kernel(MkParams p
         }
     }
     __syncthreads();
-    if (mtb == 0 && p.n_mtb == 1 && warp == ingest_loader_warp(nw)) ingest(S, p, ingest_stage, S.ingest_bar);
+    if (mtb == 0 && p.ce_ingest && warp == ingest_loader_warp(nw)) ce_scanner(p);
+    else if (mtb == 0 && p.n_mtb == 1 && warp == ingest_loader_warp(nw)) ingest(S, p, ingest_stage, S.ingest_bar);
     else if (mtb == 0 && warp == ingest_loader_warp(nw)) ingest_loader(S, p, ingest_stage);
-    else if (io && ingest_publisher_index(warp, nw) < kIngestPublishers)
-        ingest_publisher(S, p, ingest_stage, ingest_publisher_index(warp, nw));
+    else if (io && ingest_publisher_index(warp, nw) < kIngestPublishers) {
+        if (!p.ce_ingest) ingest_publisher(S, p, ingest_stage, ingest_publisher_index(warp, nw));
+    }
     else if (io && warp == host_poster_warp(nw)) host_poster(S, p);
     else if (io && forwarder_index(warp, nw) < p.n_fwd) comp_forwarder(S, p, forwarder_index(warp, nw));
     else if ((my_exec >> warp) & 1u) worker<kG>(S, smem_base, p, mtb, warp, resident, my_exec, warp == first, my_g);
@@ -1987,6 +2049,8 @@ template __global__ void master_kernel<4, 512, 1>(MkParams);   /* twice the MTBs
 template __global__ void master_kernel<1, 1024, 2>(MkParams);   /* two scheduling groups per MTB */
 template __global__ void master_kernel<2, 1024, 2>(MkParams);
 template __global__ void master_kernel<4, 512, 2>(MkParams);
+template __global__ void master_kernel<8, 256, 1>(MkParams);   /* 8-warp MTBs: one 256-thread task each */
+template __global__ void master_kernel<8, 256, 2>(MkParams);
 
 /* host side (runtime.cu): the registered 3DES key schedule of this module's MasterKernel */
 cudaError_t set_tdes_const_keys(const void* keys384, uint64_t tables_ptr)
@@ -2009,13 +2073,15 @@ cudaError_t launch_master(int mtbs_per_sm, int n_mtb, size_t smem_bytes, cudaStr
                           int* regs_out)
 {
     const bool g2 = params->n_grp == 2;
-    const void* fn = mtbs_per_sm == 4   ? (g2 ? reinterpret_cast<const void*>(&master_kernel<4, 512, 2>)
+    const void* fn = mtbs_per_sm == 8   ? (g2 ? reinterpret_cast<const void*>(&master_kernel<8, 256, 2>)
+                                              : reinterpret_cast<const void*>(&master_kernel<8, 256, 1>))
+                     : mtbs_per_sm == 4 ? (g2 ? reinterpret_cast<const void*>(&master_kernel<4, 512, 2>)
                                               : reinterpret_cast<const void*>(&master_kernel<4, 512, 1>))
                      : mtbs_per_sm == 2 ? (g2 ? reinterpret_cast<const void*>(&master_kernel<2, 1024, 2>)
                                               : reinterpret_cast<const void*>(&master_kernel<2, 1024, 1>))
                                         : (g2 ? reinterpret_cast<const void*>(&master_kernel<1, 1024, 2>)
                                               : reinterpret_cast<const void*>(&master_kernel<1, 1024, 1>));
-    const int threads = mtbs_per_sm == 4 ? 512 : 1024;
+    const int threads = mtbs_per_sm == 8 ? 256 : mtbs_per_sm == 4 ? 512 : 1024;
     cudaError_t err = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_bytes);
     if (err != cudaSuccess) return err;
     cudaFuncAttributes attr;

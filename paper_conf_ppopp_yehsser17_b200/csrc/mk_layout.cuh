@@ -36,6 +36,8 @@ struct HostCtl {
     alignas(64) volatile uint64_t published;  /* host -> GPU doorbell: entries [0, published) written */
     volatile uint32_t terminate;              /* host -> GPU: drain and exit */
     alignas(64) volatile uint64_t consumed;   /* GPU -> host: entries copied to the device ring */
+    alignas(64) volatile uint64_t handed;     /* GPU -> host (PAGODA_CE_INGEST): ring positions below this were
+                                                 loaded by schedulers and handed back (their cells are free) */
     alignas(64) volatile uint32_t error;      /* GPU -> host: device error word (PAGODA_DEVERR_*) */
     volatile uint32_t ingest_alive;
     alignas(64) volatile uint64_t pad[8];
@@ -118,6 +120,10 @@ struct MkParams {
     uint32_t     n_grp;       /* scheduling groups per MTB (1 or 2: pagoda_config.sched_groups) */
     uint32_t     n_exit;      /* holders that exit in a session: n_mtb * n_grp */
     uint32_t     max_tasks;   /* pagoda_config.max_tasks: cap on the tasks a group holds (0 = none) */
+    uint64_t     ce_base;     /* PAGODA_CE_INGEST: the ring position the session starts at (everything below was
+                                 loaded and handed back in earlier sessions) */
+    uint32_t     ce_ingest;   /* PAGODA_CE_INGEST: the host copies entries and writes DevCtl.tail (no ingest warps,
+                                 no per-cell publication words: a ticket t is published once tail > t) */
 };
 enum { kLifePub = 0, kLifeLoad, kLifePlace, kLifeStart, kLifeEnd, kLifeDone, kLifeQueued, kLifeFwd };
 

@@ -14,6 +14,7 @@
  * holds the newest finished occupant, and occupant id + C is only spawned after
  * id is done, so "comp[id mod C] >= id" <=> id done.
  */
+#include <cuda.h>   /* driver types for cuStreamWriteValue64 (resolved at run time, no link) */
 #include <cuda_runtime.h>
 #include <errno.h>
 #include <stdint.h>
@@ -26,6 +27,7 @@
 #include <algorithm>
 #include <atomic>
 #include <chrono>
+#include <condition_variable>
 #include <mutex>
 #include <thread>
 #include <vector>
@@ -101,7 +103,121 @@ struct pagoda_ctx {
     std::atomic<int> running{0};
     std::mutex session_mtx;
     int sessions = 0;
+    /* PAGODA_CE_INGEST: the copy-engine ingest thread (one per context, started at init) */
+    std::thread ce_thread;
+    std::atomic<int> ce_cmd{0};             /* 0 idle, 1 run a session, 2 flush and stop it, 3 abort it, 4 exit */
+    std::atomic<int> ce_busy{0};            /* 1 while the thread serves a session */
+    std::mutex ce_mtx;
+    std::condition_variable ce_cv;
+    cudaStream_t ce_stream = nullptr;
+    uint64_t ce_issued = 0;                 /* ring positions whose copy was issued (carries over sessions) */
+    CUdeviceptr d_consumed = 0, d_tail = 0, d_stop = 0;
 };
+
+static inline uint64_t now_ns();
+
+/* cuStreamWriteValue64 / 32 through the runtime's driver entry points (no -lcuda) */
+typedef CUresult (*WriteValue64Fn)(CUstream, CUdeviceptr, cuuint64_t, unsigned int);
+typedef CUresult (*WriteValue32Fn)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+static WriteValue64Fn g_wv64 = nullptr;
+static WriteValue32Fn g_wv32 = nullptr;
+static bool load_stream_memops()
+{
+    static std::once_flag once;
+    std::call_once(once, [] {
+        cudaDriverEntryPointQueryResult q;
+        void* f = nullptr;
+        if (cudaGetDriverEntryPoint("cuStreamWriteValue64", &f, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            g_wv64 = (WriteValue64Fn)f;
+        f = nullptr;
+        if (cudaGetDriverEntryPoint("cuStreamWriteValue32", &f, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            g_wv32 = (WriteValue32Fn)f;
+        cudaGetLastError();
+    });
+    return g_wv64 && g_wv32;
+}
+
+/* The copy-engine ingest (PAGODA_CE_INGEST), one session: copies the published, not yet issued
+ * span of the host ring into the device ring (one cudaMemcpyAsync per contiguous part), then two
+ * stream memory operations ordered after it (CU_STREAM_WRITE_VALUE_DEFAULT: a memory barrier
+ * first): DevCtl.tail = the span's end (the schedulers' publication: ticket t is published once
+ * tail > t, read with an acquire) and HostCtl.consumed (the host may reuse those ring slots).  A
+ * device ring cell is overwritten only once the ticket of the previous lap handed it back
+ * (HostCtl.handed, posted by MTB 0's scanner warp).  Command 2: flush what is published, then
+ * DevCtl.stop = 1 behind it; 3: stop = kStopAbort at once. */
+static void ce_session(pagoda_ctx* c)
+{
+    const uint64_t R = c->R;
+    uint64_t issued = c->ce_issued;
+    int idle = 0;
+    for (;;) {
+        const int cmd = c->ce_cmd.load(std::memory_order_acquire);
+        if (cmd == 3 || cmd == 4) {
+            g_wv32((CUstream)c->ce_stream, c->d_stop, kStopAbort, 0);
+            break;
+        }
+        const uint64_t pub = c->hctl->published;
+        std::atomic_thread_fence(std::memory_order_acquire);   /* entries below pub were written first */
+        const uint64_t limit = std::min<uint64_t>(pub, c->hctl->handed + R);
+        if (limit > issued) {
+            const uint64_t e0 = issued & (R - 1);
+            const uint64_t n = limit - issued, n1 = std::min<uint64_t>(n, R - e0);
+            cudaMemcpyAsync(c->dring + e0, c->hring + e0, n1 * sizeof(TaskEntry), cudaMemcpyHostToDevice, c->ce_stream);
+            if (n1 < n)
+                cudaMemcpyAsync(c->dring, c->hring, (n - n1) * sizeof(TaskEntry), cudaMemcpyHostToDevice, c->ce_stream);
+            g_wv64((CUstream)c->ce_stream, c->d_tail, limit, 0);
+            g_wv64((CUstream)c->ce_stream, c->d_consumed, limit, 0);
+            issued = limit;
+            idle = 0;
+            continue;
+        }
+        if (cmd == 2 && issued >= pub) {   /* everything published is issued: drain and exit */
+            g_wv32((CUstream)c->ce_stream, c->d_stop, 1u, 0);
+            break;
+        }
+        if (++idle > 1024) std::this_thread::yield();
+        else _mm_pause();
+    }
+    cudaStreamSynchronize(c->ce_stream);
+    c->ce_issued = issued;
+}
+
+/* The context's ingest thread: serves sessions (ce_cmd 1/2/3) and idles in between (spinning
+ * for 50 ms after a session, so back-to-back sessions start without a wake-up, then blocked). */
+static void ce_thread_main(pagoda_ctx* c)
+{
+    cudaSetDevice(c->device);
+    for (;;) {
+        int cmd = c->ce_cmd.load(std::memory_order_acquire);
+        const uint64_t t0 = now_ns();
+        while (cmd == 0 && now_ns() - t0 < 50000000ull) {
+            std::this_thread::yield();
+            cmd = c->ce_cmd.load(std::memory_order_acquire);
+        }
+        if (cmd == 0) {
+            std::unique_lock<std::mutex> lk(c->ce_mtx);
+            c->ce_cv.wait(lk, [&] { return c->ce_cmd.load(std::memory_order_acquire) != 0; });
+            cmd = c->ce_cmd.load(std::memory_order_acquire);
+        }
+        if (cmd == 4) return;
+        ce_session(c);
+        /* the session is over for this thread: back to idle unless told to exit meanwhile */
+        int expect = c->ce_cmd.load(std::memory_order_acquire);
+        while (expect != 4 && !c->ce_cmd.compare_exchange_weak(expect, 0)) { }
+        c->ce_busy.store(0, std::memory_order_release);
+        if (expect == 4) return;
+    }
+}
+static void ce_command(pagoda_ctx* c, int cmd)
+{
+    {
+        std::lock_guard<std::mutex> lk(c->ce_mtx);
+        c->ce_cmd.store(cmd, std::memory_order_release);
+    }
+    c->ce_cv.notify_all();
+}
 
 /* Every live context, by device: the MasterKernel's constant bank (registered 3DES keys, DCT
  * coefficients) is one per device and process, so registration must not race a running
@@ -330,6 +446,7 @@ static int start_kernel(pagoda_ctx* c)
         cudaMemsetAsync(c->exec_count, 0, (size_t)c->n_mtb * 32 * sizeof(uint32_t), c->stream);
     }
     std::lock_guard<std::mutex> reg(g_ctx_mtx);   /* no constant-bank registration during the launch */
+    c->params.ce_base = c->ce_issued;   /* (CE ingest) the scanner's first position */
     cudaEventRecord(c->ev_start, c->stream);
     cudaError_t e = launch_master(c->cfg.mtbs_per_sm, c->n_mtb, c->smem, c->stream, &c->params, &c->regs);
     if (e != cudaSuccess) {
@@ -338,6 +455,11 @@ static int start_kernel(pagoda_ctx* c)
         return -EIO;
     }
     cudaEventRecord(c->ev_stop, c->stream);   /* completes when the session's kernel exits */
+    if (c->cfg.flags & PAGODA_CE_INGEST) {
+        /* terminate already set (pagoda_start_drain): flush what is published, then stop */
+        c->ce_busy.store(1, std::memory_order_release);
+        ce_command(c, c->hctl->terminate ? 2 : 1);
+    }
     c->running.store(1, std::memory_order_release);
     c->sessions++;
     return 0;
@@ -347,6 +469,8 @@ static int start_kernel(pagoda_ctx* c)
 static int stop_kernel(pagoda_ctx* c, bool abort_now = false)
 {
     c->hctl->terminate = abort_now ? kStopAbort : 1;
+    const bool ce = (c->cfg.flags & PAGODA_CE_INGEST) != 0;
+    if (ce) ce_command(c, abort_now ? 3 : 2);
     const uint64_t t0 = now_ns();
     cudaError_t q;
     bool aborted = abort_now;
@@ -357,6 +481,7 @@ static int stop_kernel(pagoda_ctx* c, bool abort_now = false)
             /* abandon the queue: idle MTBs exit, tasks still running are waited for a while */
             fprintf(stderr, "pagoda: MasterKernel did not drain (watchdog): aborting the session\n");
             c->hctl->terminate = kStopAbort;
+            if (ce) ce_command(c, 3);
             aborted = true;
         }
         if (aborted && waited > c->cfg.watchdog_s + 10.0) {
@@ -364,6 +489,7 @@ static int stop_kernel(pagoda_ctx* c, bool abort_now = false)
             return -ETIMEDOUT;   /* still resident: buffers must not be freed */
         }
     }
+    while (ce && c->ce_busy.load(std::memory_order_acquire)) std::this_thread::yield();   /* its stream synced */
     c->running.store(0, std::memory_order_release);
     if (aborted) {
         c->faulted.store(1);
@@ -415,6 +541,11 @@ static void free_ctx(pagoda_ctx* c)
     if (c->exec_trace) cudaFree(c->exec_trace);
     if (c->life) cudaFree(c->life);
     if (c->exec_count) cudaFree(c->exec_count);
+    if (c->ce_thread.joinable()) {
+        ce_command(c, 4);
+        c->ce_thread.join();
+    }
+    if (c->ce_stream) cudaStreamDestroy(c->ce_stream);
     if (c->stream) cudaStreamDestroy(c->stream);
     delete c;
 }
@@ -426,8 +557,9 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
     pagoda_config cfg;
     if (cfg_in) cfg = *cfg_in;
     else pagoda_config_default(&cfg);
-    if (cfg.mtbs_per_sm != 1 && cfg.mtbs_per_sm != 2 && cfg.mtbs_per_sm != 4) return -EINVAL;
-    const uint32_t block_warps = cfg.mtbs_per_sm == 4 ? 16u : 32u;   /* 4 MTBs/SM: 512-thread MTBs */
+    if (cfg.mtbs_per_sm != 1 && cfg.mtbs_per_sm != 2 && cfg.mtbs_per_sm != 4 && cfg.mtbs_per_sm != 8) return -EINVAL;
+    /* 4 MTBs/SM: 512-thread MTBs; 8: 256-thread MTBs (their I/O MTB's stages are small: use PAGODA_CE_INGEST) */
+    const uint32_t block_warps = cfg.mtbs_per_sm == 8 ? 8u : cfg.mtbs_per_sm == 4 ? 16u : 32u;
     if (!pow2(cfg.ring_entries) || !pow2(cfg.comp_entries) || cfg.comp_entries < cfg.ring_entries ||
         cfg.ring_entries < 2 * kSpawnChunk)
         return -EINVAL;
@@ -532,6 +664,19 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
         if (cudaMemset(c->life, 0, (size_t)c->C * 8 * sizeof(uint64_t)) != cudaSuccess) goto fail;
     }
     if (cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking) != cudaSuccess) goto fail;
+    if (cfg.flags & PAGODA_CE_INGEST) {
+        if (!load_stream_memops()) {
+            rc = -ENOTSUP;
+            goto fail;
+        }
+        if (cudaStreamCreateWithFlags(&c->ce_stream, cudaStreamNonBlocking) != cudaSuccess) goto fail;
+        void* hc = nullptr;
+        cudaHostGetDevicePointer(&hc, (void*)c->hctl, 0);
+        c->d_consumed = (CUdeviceptr)((char*)hc + offsetof(HostCtl, consumed));
+        c->d_tail = (CUdeviceptr)&c->dctl->tail;
+        c->d_stop = (CUdeviceptr)&c->dctl->stop;
+        c->ce_thread = std::thread(ce_thread_main, c);
+    }
     if (cudaEventCreate(&c->ev_start) != cudaSuccess || cudaEventCreate(&c->ev_stop) != cudaSuccess) goto fail;
     /* the set-up copies and memsets above ran on the legacy stream: wait for that stream only.  A
      * device-wide synchronize would also wait for another context's persistent MasterKernel on the
@@ -572,6 +717,7 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
         p.n_grp = (uint32_t)c->n_grp;
         p.n_exit = (uint32_t)(c->n_mtb * c->n_grp);
         p.max_tasks = cfg.max_tasks;
+        p.ce_ingest = (cfg.flags & PAGODA_CE_INGEST) ? 1u : 0u;
         if (cfg.flags & PAGODA_TRACE) {
             p.trace_cap = c->cfg.trace_events;
             p.trace = c->trace;
@@ -582,7 +728,7 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
         p.life = c->life;
         /* completion forwarders: 4 when MTB 0 has 32 warps; 1 at 4 MTBs/SM (512 threads), where more
          * cost MM ~7 % (45 -> 42 M tasks/s) while NOP's forwarding is not the limit there */
-        p.n_fwd = cfg.mtbs_per_sm == 4 ? 1u : (uint32_t)kForwarders;
+        p.n_fwd = cfg.mtbs_per_sm >= 4 ? 1u : (uint32_t)kForwarders;
         p.spread_ns = 0;
         if (cfg.flags & PAGODA_SPREAD) {   /* PAGODA_SPREAD_NS (environment) overrides the 6 us default */
             const char* e = getenv("PAGODA_SPREAD_NS");

@@ -23,6 +23,7 @@ RESIDENT_TDES = 0x4
 LIFECYCLE = 0x8
 SPREAD = 0x10
 NONBLOCKING_SPAWN = 0x20
+CE_INGEST = 0x40
 LIFE_EVENTS = ("pub", "load", "place", "start", "end", "done", "queued", "fwd")
 
 

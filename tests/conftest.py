@@ -10,6 +10,20 @@ if ROOT not in sys.path:
 GOLDEN = os.path.join(ROOT, "tests", "golden")
 
 
+if os.environ.get("PAGODA_TEST_FLAGS"):
+    # run the suite with extra context flags (e.g. PAGODA_TEST_FLAGS=0x40: every context uses the
+    # copy-engine ingest): pagoda_config.flags of every context the tests create is OR-ed with them
+    from paper_conf_ppopp_yehsser17_b200 import pagoda as _pg
+    _extra = int(os.environ["PAGODA_TEST_FLAGS"], 0)
+    _default_config = _pg.default_config
+
+    def _with_flags(**kw):
+        cfg = _default_config(**kw)
+        cfg.flags |= _extra
+        return cfg
+    _pg.default_config = _with_flags
+
+
 def pytest_configure(config):
     config.addinivalue_line("markers", "gpu: needs a B200 (sm_100a) GPU; parity tests through the C-ABI")
     config.addinivalue_line("markers", "slow: long-running")
