@@ -1460,7 +1460,10 @@ __device__ int sched_copy(MtbShared& S, Sched<kG>& st, const MkParams& p, uint32
         const uint32_t slot = nth_set_bit(st.free_task, lane);
         S.pend[fq(st, st.pl + lane)] = (uint8_t)slot;
         st_relaxed_gpu32(&p.dseq[t & p.ring_mask], (uint32_t)(t + (uint64_t)p.ring_mask + 1));
-        if (p.life && !(S.tasks[slot].flags & kEntryGroup)) life_stamp(p, S.tasks[slot].id, kLifeLoad);
+        if (p.life && !(S.tasks[slot].flags & kEntryGroup)) {
+            if (p.ce_ingest) life_stamp(p, S.tasks[slot].id, kLifePub);   /* (no device-side publication step) */
+            life_stamp(p, S.tasks[slot].id, kLifeLoad);
+        }
         used = 1u << slot;
     }
 #elif PAGODA_FAST_LOAD == 0 && PAGODA_CELL_RELAXED
@@ -1482,7 +1485,10 @@ __device__ int sched_copy(MtbShared& S, Sched<kG>& st, const MkParams& p, uint32
         asm volatile("fence.acq_rel.cta;" ::: "memory");
         S.pend[fq(st, st.pl + lane)] = (uint8_t)slot;
         st_relaxed_gpu32(&p.dseq[t & p.ring_mask], (uint32_t)(t + (uint64_t)p.ring_mask + 1));
-        if (p.life && !(S.tasks[slot].flags & kEntryGroup)) life_stamp(p, S.tasks[slot].id, kLifeLoad);
+        if (p.life && !(S.tasks[slot].flags & kEntryGroup)) {
+            if (p.ce_ingest) life_stamp(p, S.tasks[slot].id, kLifePub);   /* (no device-side publication step) */
+            life_stamp(p, S.tasks[slot].id, kLifeLoad);
+        }
         used = 1u << slot;
     }
 #elif PAGODA_CELL_ACQ
@@ -1504,7 +1510,10 @@ __device__ int sched_copy(MtbShared& S, Sched<kG>& st, const MkParams& p, uint32
         }
         S.pend[fq(st, st.pl + lane)] = (uint8_t)slot;
         st_relaxed_gpu32(&p.dseq[t & p.ring_mask], (uint32_t)(t + (uint64_t)p.ring_mask + 1));
-        if (p.life && !(S.tasks[slot].flags & kEntryGroup)) life_stamp(p, S.tasks[slot].id, kLifeLoad);
+        if (p.life && !(S.tasks[slot].flags & kEntryGroup)) {
+            if (p.ce_ingest) life_stamp(p, S.tasks[slot].id, kLifePub);   /* (no device-side publication step) */
+            life_stamp(p, S.tasks[slot].id, kLifeLoad);
+        }
         used = 1u << slot;
     }
 #else

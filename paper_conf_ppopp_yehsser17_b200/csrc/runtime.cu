@@ -151,6 +151,14 @@ static void ce_session(pagoda_ctx* c)
 {
     const uint64_t R = c->R;
     uint64_t issued = c->ce_issued;
+    /* at most kInFlight copies in the stream: a small copy and its two memory operations take
+     * several microseconds on the GPU whatever their size, so the next copy waits for the
+     * oldest to land (HostCtl.consumed) and then takes everything published meanwhile */
+    constexpr int kInFlight = 2;
+    constexpr uint64_t kChunk = 2048;   /* entries per copy: a backlog (a prespawned session) streams in
+                                           128 KiB steps, the first tasks start after the first one */
+    uint64_t ends[kInFlight];
+    int nq = 0;
     int idle = 0;
     for (;;) {
         const int cmd = c->ce_cmd.load(std::memory_order_acquire);
@@ -160,15 +168,31 @@ static void ce_session(pagoda_ctx* c)
         }
         const uint64_t pub = c->hctl->published;
         std::atomic_thread_fence(std::memory_order_acquire);   /* entries below pub were written first */
-        const uint64_t limit = std::min<uint64_t>(pub, c->hctl->handed + R);
-        if (limit > issued) {
+        const uint64_t limit = std::min<uint64_t>(std::min<uint64_t>(pub, c->hctl->handed + R), issued + kChunk);
+        if (nq) {
+            const uint64_t done = c->hctl->consumed;
+            int k = 0;
+            while (k < nq && done >= ends[k]) k++;
+            if (k) {
+                for (int i = k; i < nq; i++) ends[i - k] = ends[i];
+                nq -= k;
+            }
+        }
+        if (limit > issued && nq < kInFlight) {
             const uint64_t e0 = issued & (R - 1);
             const uint64_t n = limit - issued, n1 = std::min<uint64_t>(n, R - e0);
             cudaMemcpyAsync(c->dring + e0, c->hring + e0, n1 * sizeof(TaskEntry), cudaMemcpyHostToDevice, c->ce_stream);
             if (n1 < n)
                 cudaMemcpyAsync(c->dring, c->hring, (n - n1) * sizeof(TaskEntry), cudaMemcpyHostToDevice, c->ce_stream);
-            g_wv64((CUstream)c->ce_stream, c->d_tail, limit, 0);
-            g_wv64((CUstream)c->ce_stream, c->d_consumed, limit, 0);
+            const CUresult r1 = g_wv64((CUstream)c->ce_stream, c->d_tail, limit, 0);
+            const CUresult r2 = g_wv64((CUstream)c->ce_stream, c->d_consumed, limit, 0);
+            if (r1 != CUDA_SUCCESS || r2 != CUDA_SUCCESS) {
+                fprintf(stderr, "pagoda: cuStreamWriteValue64 failed (%d, %d): copy-engine ingest stops\n", (int)r1,
+                        (int)r2);
+                c->faulted.store(1);
+                break;
+            }
+            ends[nq++] = limit;
             issued = limit;
             idle = 0;
             continue;

@@ -18,9 +18,9 @@ pytestmark = pytest.mark.gpu
 def test_ce_mark_exactly_once_and_tid():
     dev = Dev()
     n = 300
-    cnt = dev.zeros(1)
+    cnt = dev.zeros(4)
+    out = dev.zeros(n * 256 * 4)
     with Pagoda(flags=CE_INGEST) as p:
-        out = dev.zeros(n * 256)
         for k in range(n):
             a = T.records(T.MARK, 1)
             a["out"], a["cnt"], a["base"], a["tag"] = ptr(out), ptr(cnt), k * 256, k + 1
