@@ -17,6 +17,7 @@
  */
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdio.h>
 
 #include "bodies.cuh"
 #include "mk_layout.cuh"
@@ -2098,7 +2099,11 @@ cudaError_t launch_master(int mtbs_per_sm, int n_mtb, size_t smem_bytes, cudaStr
     int per_sm = 0;
     err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, threads, smem_bytes);
     if (err != cudaSuccess) return err;
-    if (per_sm < mtbs_per_sm) return cudaErrorCooperativeLaunchTooLarge;
+    if (per_sm < mtbs_per_sm) {
+        fprintf(stderr, "pagoda: %d MTBs per SM requested, %d fit (%zu B of shared memory, %d threads, %d registers)\n",
+                mtbs_per_sm, per_sm, smem_bytes, threads, regs_out ? *regs_out : -1);
+        return cudaErrorCooperativeLaunchTooLarge;
+    }
     void* args[] = {params};
     return cudaLaunchCooperativeKernel(fn, dim3(n_mtb), dim3(threads), args, smem_bytes, stream);
 }

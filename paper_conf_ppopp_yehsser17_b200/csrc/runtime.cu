@@ -593,7 +593,7 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
     if (cfg.max_tasks > 32) return -EINVAL;
     cfg.exec_warps = std::min(cfg.exec_warps, block_warps);
     if (cfg.arena_bytes % PAGODA_GRANULE || cfg.arena_bytes / PAGODA_GRANULE > (uint32_t)kMaxGranules ||
-        cfg.arena_bytes < 2u * 128u * 64u + 8u * PAGODA_GRANULE)   /* ingest staging + room for tasks */
+        cfg.arena_bytes < 8u * PAGODA_GRANULE)
         return -EINVAL;
     int ndev = 0;
     if (cudaGetDeviceCount(&ndev) != cudaSuccess || cfg.device < 0 || cfg.device >= ndev) {
@@ -617,6 +617,10 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
     c->device = cfg.device;
     c->sm_count = prop.multiProcessorCount;
     const int nsm = cfg.num_sms ? cfg.num_sms : prop.multiProcessorCount;
+    if (nsm * cfg.mtbs_per_sm == 1 && cfg.arena_bytes < 2u * 128u * 64u + 8u * PAGODA_GRANULE) {
+        delete c;   /* one MTB lends the top of its arena to its ingest warp's two stages */
+        return -EINVAL;
+    }
     c->n_mtb = nsm * cfg.mtbs_per_sm;
     c->R = cfg.ring_entries;
     c->C = cfg.comp_entries;
