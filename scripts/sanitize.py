@@ -23,7 +23,7 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 
 from paper_conf_ppopp_yehsser17_b200 import tasks as T  # noqa: E402
 from paper_conf_ppopp_yehsser17_b200 import workloads as W  # noqa: E402
-from paper_conf_ppopp_yehsser17_b200.pagoda import NO_START, Pagoda  # noqa: E402
+from paper_conf_ppopp_yehsser17_b200.pagoda import CE_INGEST, NO_START, Pagoda  # noqa: E402
 
 
 def run(cfg, label, big):
@@ -32,7 +32,8 @@ def run(cfg, label, big):
     err, out, scratch = dev(64), dev(4 * 4096), dev(4 * 4096)
     ws = [W.mandelbrot(2), W.tdes(2, shmem=2560)] + ([W.matmul(2), W.mix(8)] if big else [])
     torch.cuda.synchronize()
-    with Pagoda(flags=NO_START, **cfg) as p:
+    flags = cfg.pop("flags", 0)
+    with Pagoda(flags=NO_START | flags, **cfg) as p:
         shapes = [(32, 1, 0, 0, T.NOP, None),
                   (96, 1, 0, 0, T.MARK, np.array([(out.data_ptr(), err.data_ptr() + 32, 0, 7)], T.ARGS[T.MARK])),
                   (64, 2, 0, 0, T.TID, np.array([(out.data_ptr() + 4096, 0, 0)], T.ARGS[T.TID])),
@@ -57,6 +58,8 @@ def main():
     run({"num_sms": 1, "mtbs_per_sm": 1, "exec_warps": 4, "arena_bytes": 2 * 128 * 64 + 8 * 512}, "debug 1 MTB",
         big=False)
     run({"num_sms": 2, "mtbs_per_sm": 1, "arena_bytes": 200 * 1024}, "2 SMs (I/O MTB + task MTB)", big=True)
+    run({"num_sms": 2, "mtbs_per_sm": 1, "arena_bytes": 200 * 1024, "flags": CE_INGEST},
+        "2 SMs, copy-engine ingest (scanner warp)", big=True)
 
 
 if __name__ == "__main__":
