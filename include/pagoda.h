@@ -61,9 +61,7 @@ typedef int64_t pagoda_task_t;          /* >= 0: task id; < 0: -errno */
 typedef struct {
     int      device;        /* CUDA device ordinal (default 0) */
     int      mtbs_per_sm;   /* MasterKernel thread blocks (MTBs) per SM: 1 or 2 (1024 threads each; default 2,
-                               P:453-455), 4 (512 threads each: twice the schedulers per SM; arena <= 48 KiB) or
-                               8 (256 threads each: one 8-warp task per MTB; arena <= 21 KiB; the doorbell
-                               ingest's stages are then small: use PAGODA_CE_INGEST) */
+                               P:453-455) or 4 (512 threads each: twice the schedulers per SM; arena <= 48 KiB) */
     int      num_sms;       /* SMs to occupy, 0 = all (148 on B200) */
     uint32_t ring_entries;  /* TaskTable ring entries, host and device, power of 2 (default 65536) */
     uint32_t comp_entries;  /* completion window, power of 2 >= ring_entries (default 1<<20) */

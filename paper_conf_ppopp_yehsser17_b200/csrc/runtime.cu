@@ -581,9 +581,11 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
     pagoda_config cfg;
     if (cfg_in) cfg = *cfg_in;
     else pagoda_config_default(&cfg);
-    if (cfg.mtbs_per_sm != 1 && cfg.mtbs_per_sm != 2 && cfg.mtbs_per_sm != 4 && cfg.mtbs_per_sm != 8) return -EINVAL;
-    /* 4 MTBs/SM: 512-thread MTBs; 8: 256-thread MTBs (their I/O MTB's stages are small: use PAGODA_CE_INGEST) */
-    const uint32_t block_warps = cfg.mtbs_per_sm == 8 ? 8u : cfg.mtbs_per_sm == 4 ? 16u : 32u;
+    /* 4 MTBs/SM: 512-thread MTBs.  (8 MTBs/SM of 256 threads were tried: the cooperative launch fails with
+     * "too many blocks" although the occupancy API reports 8 per SM; each MTB uses all 16 named
+     * barriers, the likely per-SM limit.) */
+    if (cfg.mtbs_per_sm != 1 && cfg.mtbs_per_sm != 2 && cfg.mtbs_per_sm != 4) return -EINVAL;
+    const uint32_t block_warps = cfg.mtbs_per_sm == 4 ? 16u : 32u;
     if (!pow2(cfg.ring_entries) || !pow2(cfg.comp_entries) || cfg.comp_entries < cfg.ring_entries ||
         cfg.ring_entries < 2 * kSpawnChunk)
         return -EINVAL;
@@ -756,7 +758,7 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
         p.life = c->life;
         /* completion forwarders: 4 when MTB 0 has 32 warps; 1 at 4 MTBs/SM (512 threads), where more
          * cost MM ~7 % (45 -> 42 M tasks/s) while NOP's forwarding is not the limit there */
-        p.n_fwd = cfg.mtbs_per_sm >= 4 ? 1u : (uint32_t)kForwarders;
+        p.n_fwd = cfg.mtbs_per_sm == 4 ? 1u : (uint32_t)kForwarders;
         p.spread_ns = 0;
         if (cfg.flags & PAGODA_SPREAD) {   /* PAGODA_SPREAD_NS (environment) overrides the 6 us default */
             const char* e = getenv("PAGODA_SPREAD_NS");
