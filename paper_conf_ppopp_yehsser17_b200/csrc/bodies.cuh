@@ -513,8 +513,19 @@ __device__ void body_tdes(const Env& e, const pagoda_tdes_args& a)
  * CUDA SDK MatrixMul [22] (Table 3); 32x32x32 fp32; C[i][j] is the
  * fma chain over k ascending from 0.  A and B are staged into the TB's shmem
  * with TMA bulk copies when 8 KiB were granted and the TB can synchronise. */
+#ifndef PAGODA_MM_VEC
+#define PAGODA_MM_VEC 1        /* A's rows as float4 loads (64 shared loads per thread instead of 160) */
+#endif
+#ifndef PAGODA_MM_NOINLINE
+#define PAGODA_MM_NOINLINE 1   /* a call: keeps the 32-register executors' allocation (spills 508 vs 880 B) */
+#endif
+#if PAGODA_MM_NOINLINE
+#define PAGODA_MM_ATTR __noinline__
+#else
+#define PAGODA_MM_ATTR
+#endif
 template <class Env>
-__device__ void body_mm(const Env& e, const pagoda_mm_args& a)
+__device__ PAGODA_MM_ATTR void body_mm(const Env& e, const pagoda_mm_args& a)
 {
     const float* A = a.A;
     const float* B = a.B;
@@ -541,7 +552,25 @@ __device__ void body_mm(const Env& e, const pagoda_mm_args& a)
 #pragma unroll
         for (int q = 0; q < 4; q++) row[q] = min(base + q * T, 1023) >> 5;   /* past the end: a dummy row */
         const int j = base & 31;
-        if ((T & 31) == 0) {
+        if (PAGODA_MM_VEC && (T & 31) == 0 && (reinterpret_cast<uintptr_t>(A) & 15u) == 0) {
+            /* A's row segments as float4 (one broadcast load per 4 k per row: 64 loads per thread instead
+             * of 160); every chain still accumulates k ascending */
+#pragma unroll 2
+            for (int k0 = 0; k0 < 32; k0 += 4) {
+                float4 av[4];
+#pragma unroll
+                for (int q = 0; q < 4; q++) av[q] = *reinterpret_cast<const float4*>(A + row[q] * 32 + k0);
+                const float b0 = B[(k0 + 0) * 32 + j], b1 = B[(k0 + 1) * 32 + j];
+                const float b2 = B[(k0 + 2) * 32 + j], b3 = B[(k0 + 3) * 32 + j];
+#pragma unroll
+                for (int q = 0; q < 4; q++) {
+                    acc[q] = __fmaf_rn(av[q].x, b0, acc[q]);
+                    acc[q] = __fmaf_rn(av[q].y, b1, acc[q]);
+                    acc[q] = __fmaf_rn(av[q].z, b2, acc[q]);
+                    acc[q] = __fmaf_rn(av[q].w, b3, acc[q]);
+                }
+            }
+        } else if ((T & 31) == 0) {
 #pragma unroll 8
             for (int k = 0; k < 32; k++) {
                 const float b = B[k * 32 + j];

@@ -16,7 +16,11 @@ KEYS = ["gpu__time_duration.sum", "sm__cycles_elapsed.avg", "launch__registers_p
         "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum", "l1tex__data_bank_conflicts_pipe_lsu_mem_shared_op_ld.sum",
         "l1tex__lsu_writeback_active.avg.pct_of_peak_sustained_elapsed", "l1tex__throughput.avg.pct_of_peak_sustained_active",
         "sm__throughput.avg.pct_of_peak_sustained_elapsed", "gpu__compute_memory_throughput.avg.pct_of_peak_sustained_elapsed",
-        "dram__throughput.avg.pct_of_peak_sustained_elapsed", "dram__bytes.sum.per_second"]
+        "dram__throughput.avg.pct_of_peak_sustained_elapsed", "dram__bytes.sum.per_second",
+        # local memory (register spills): bytes the LSU moved, and L2 sectors of the local aperture
+        "l1tex__t_bytes_pipe_lsu_mem_local_op_ld.sum", "l1tex__t_bytes_pipe_lsu_mem_local_op_st.sum",
+        "lts__t_sectors_srcunit_tex_aperture_local_op_write.sum", "lts__t_sectors_srcunit_tex_aperture_local_op_read.sum",
+        "lts__t_sectors_srcunit_tex_aperture_device_op_write.sum", "lts__t_sectors_srcunit_tex_aperture_device_op_read.sum"]
 
 
 def main(path):
