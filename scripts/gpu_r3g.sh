@@ -12,3 +12,12 @@ for i in 1 2; do for v in 0 nv old; do
 done; done
 unset PAGODA_LIB
 python scripts/ab_summary.py $F > $F/ab.txt 2>&1; cat $F/ab.txt
+for i in 1 2; do
+  timeout 200 python bench.py --workload mix --quick --no-configs 2>/dev/null | tail -1 > $F/mix_m1_$i.json
+  timeout 200 python bench.py --workload mix --quick --no-configs --mtbs 3 --arena-kb 64 2>/dev/null | tail -1 > $F/mix_m3_$i.json
+  timeout 300 python bench.py --workload c5 --quick --no-configs --steps 2 --warmup 1 --mtbs 3 --arena-kb 64 --no-resident 2>/dev/null | tail -1 > $F/c5_m3nr_$i.json
+  timeout 300 python bench.py --workload c5 --quick --no-configs --steps 2 --warmup 1 --no-resident 2>/dev/null | tail -1 > $F/c5_m1nr_$i.json
+  timeout 200 python bench.py --workload mm --quick --no-configs --mtbs 3 --arena-kb 48 2>/dev/null | tail -1 > $F/mm_m3_$i.json
+  timeout 200 python bench.py --workload mb --quick --no-configs --mtbs 3 --arena-kb 48 2>/dev/null | tail -1 > $F/mb_m3_$i.json
+done
+python scripts/ab_summary.py $F > $F/ab.txt 2>&1; cat $F/ab.txt
