@@ -485,8 +485,16 @@ __device__ __forceinline__ void tdes_blocks_pair(const Env& e, const pagoda_tdes
     }
 }
 
+#ifndef PAGODA_TDES_NOINLINE
+#define PAGODA_TDES_NOINLINE 0   /* the 3DES body as a call (A/B: register spills around the body) */
+#endif
+#if PAGODA_TDES_NOINLINE
+#define PAGODA_TDES_ATTR __noinline__
+#else
+#define PAGODA_TDES_ATTR
+#endif
 template <class Env>
-__device__ void body_tdes(const Env& e, const pagoda_tdes_args& a)
+__device__ PAGODA_TDES_ATTR void body_tdes(const Env& e, const pagoda_tdes_args& a)
 {
     const uint32_t res = e.getResidentTdes();
     if (res && (unsigned long long)a.tables == c_tdes_tables) {   /* resident tables, registered keys: */

@@ -18,9 +18,10 @@ KEYS = ["gpu__time_duration.sum", "sm__cycles_elapsed.avg", "launch__registers_p
         "sm__throughput.avg.pct_of_peak_sustained_elapsed", "gpu__compute_memory_throughput.avg.pct_of_peak_sustained_elapsed",
         "dram__throughput.avg.pct_of_peak_sustained_elapsed", "dram__bytes.sum.per_second",
         # local memory (register spills): bytes the LSU moved, and L2 sectors of the local aperture
-        "l1tex__t_bytes_pipe_lsu_mem_local_op_ld.sum", "l1tex__t_bytes_pipe_lsu_mem_local_op_st.sum",
-        "lts__t_sectors_srcunit_tex_aperture_local_op_write.sum", "lts__t_sectors_srcunit_tex_aperture_local_op_read.sum",
-        "lts__t_sectors_srcunit_tex_aperture_device_op_write.sum", "lts__t_sectors_srcunit_tex_aperture_device_op_read.sum"]
+        "sass__inst_executed_local_loads", "sass__inst_executed_local_stores",
+        "l1tex__t_sectors_pipe_lsu_mem_local_op_ld.sum", "l1tex__t_sectors_pipe_lsu_mem_local_op_st.sum",
+        "l1tex__t_sectors_pipe_lsu_mem_local_op_st_lookup_miss.sum",
+        "l1tex__t_output_wavefronts_pipe_lsu_mem_local_op_ld.sum", "l1tex__t_output_wavefronts_pipe_lsu_mem_local_op_st.sum"]
 
 
 def main(path):
