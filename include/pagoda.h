@@ -61,8 +61,7 @@ typedef int64_t pagoda_task_t;          /* >= 0: task id; < 0: -errno */
 typedef struct {
     int      device;        /* CUDA device ordinal (default 0) */
     int      mtbs_per_sm;   /* MasterKernel thread blocks (MTBs) per SM: 1 or 2 (1024 threads each; default 2,
-                               P:453-455), 3 (512 threads each at 40 registers: 48 warps per SM; arena <= 68 KiB)
-                               or 4 (512 threads each at 32 registers: twice the schedulers per SM; arena <= 48 KiB) */
+                               P:453-455) or 4 (512 threads each: twice the schedulers per SM; arena <= 48 KiB) */
     int      num_sms;       /* SMs to occupy, 0 = all (148 on B200) */
     uint32_t ring_entries;  /* TaskTable ring entries, host and device, power of 2 (default 65536) */
     uint32_t comp_entries;  /* completion window, power of 2 >= ring_entries (default 1<<20) */

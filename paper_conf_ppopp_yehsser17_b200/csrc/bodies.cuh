@@ -522,10 +522,11 @@ __device__ PAGODA_TDES_ATTR void body_tdes(const Env& e, const pagoda_tdes_args&
  * fma chain over k ascending from 0.  A and B are staged into the TB's shmem
  * with TMA bulk copies when 8 KiB were granted and the TB can synchronise. */
 #ifndef PAGODA_MM_VEC
-#define PAGODA_MM_VEC 1        /* A's rows as float4 loads (64 shared loads per thread instead of 160) */
+#define PAGODA_MM_VEC 0        /* A's rows as float4 loads (64 shared loads per thread instead of 160): measured
+                                  slower at 32 registers (the body spills: 46.5 vs 48.3 M tasks/s) */
 #endif
 #ifndef PAGODA_MM_NOINLINE
-#define PAGODA_MM_NOINLINE 1   /* a call: keeps the 32-register executors' allocation (spills 508 vs 880 B) */
+#define PAGODA_MM_NOINLINE 1   /* a call: keeps the 32-register executors' allocation (MM 47.4 -> 48.3 M tasks/s) */
 #endif
 #if PAGODA_MM_NOINLINE
 #define PAGODA_MM_ATTR __noinline__

@@ -2059,8 +2059,6 @@ template __global__ void master_kernel<4, 512, 1>(MkParams);   /* twice the MTBs
 template __global__ void master_kernel<1, 1024, 2>(MkParams);   /* two scheduling groups per MTB */
 template __global__ void master_kernel<2, 1024, 2>(MkParams);
 template __global__ void master_kernel<4, 512, 2>(MkParams);
-template __global__ void master_kernel<3, 512, 1>(MkParams);   /* 3 MTBs of 512 threads: 48 warps/SM at 40 registers */
-template __global__ void master_kernel<3, 512, 2>(MkParams);
 
 /* host side (runtime.cu): the registered 3DES key schedule of this module's MasterKernel */
 cudaError_t set_tdes_const_keys(const void* keys384, uint64_t tables_ptr)
@@ -2083,15 +2081,13 @@ cudaError_t launch_master(int mtbs_per_sm, int n_mtb, size_t smem_bytes, cudaStr
                           int* regs_out)
 {
     const bool g2 = params->n_grp == 2;
-    const void* fn = mtbs_per_sm == 3   ? (g2 ? reinterpret_cast<const void*>(&master_kernel<3, 512, 2>)
-                                              : reinterpret_cast<const void*>(&master_kernel<3, 512, 1>))
-                     : mtbs_per_sm == 4 ? (g2 ? reinterpret_cast<const void*>(&master_kernel<4, 512, 2>)
+    const void* fn = mtbs_per_sm == 4   ? (g2 ? reinterpret_cast<const void*>(&master_kernel<4, 512, 2>)
                                               : reinterpret_cast<const void*>(&master_kernel<4, 512, 1>))
                      : mtbs_per_sm == 2 ? (g2 ? reinterpret_cast<const void*>(&master_kernel<2, 1024, 2>)
                                               : reinterpret_cast<const void*>(&master_kernel<2, 1024, 1>))
                                         : (g2 ? reinterpret_cast<const void*>(&master_kernel<1, 1024, 2>)
                                               : reinterpret_cast<const void*>(&master_kernel<1, 1024, 1>));
-    const int threads = mtbs_per_sm >= 3 ? 512 : 1024;
+    const int threads = mtbs_per_sm == 4 ? 512 : 1024;
     cudaError_t err = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_bytes);
     if (err != cudaSuccess) return err;
     cudaFuncAttributes attr;

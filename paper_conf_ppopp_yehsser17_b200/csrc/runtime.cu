@@ -584,8 +584,9 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
     /* 4 MTBs/SM: 512-thread MTBs.  (8 MTBs/SM of 256 threads were tried: the cooperative launch fails with
      * "too many blocks" although the occupancy API reports 8 per SM; each MTB uses all 16 named
      * barriers, the likely per-SM limit.) */
-    if (cfg.mtbs_per_sm < 1 || cfg.mtbs_per_sm > 4) return -EINVAL;
-    const uint32_t block_warps = cfg.mtbs_per_sm >= 3 ? 16u : 32u;   /* 3: 512 threads at 40 registers */
+    /* (3 MTBs/SM of 512 threads at 40 registers were measured too: slower on every config, e.g. mix 12.9 -> 7.8 M) */
+    if (cfg.mtbs_per_sm != 1 && cfg.mtbs_per_sm != 2 && cfg.mtbs_per_sm != 4) return -EINVAL;
+    const uint32_t block_warps = cfg.mtbs_per_sm == 4 ? 16u : 32u;
     if (!pow2(cfg.ring_entries) || !pow2(cfg.comp_entries) || cfg.comp_entries < cfg.ring_entries ||
         cfg.ring_entries < 2 * kSpawnChunk)
         return -EINVAL;
@@ -758,7 +759,7 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
         p.life = c->life;
         /* completion forwarders: 4 when MTB 0 has 32 warps; 1 at 4 MTBs/SM (512 threads), where more
          * cost MM ~7 % (45 -> 42 M tasks/s) while NOP's forwarding is not the limit there */
-        p.n_fwd = cfg.mtbs_per_sm >= 3 ? 1u : (uint32_t)kForwarders;
+        p.n_fwd = cfg.mtbs_per_sm == 4 ? 1u : (uint32_t)kForwarders;
         p.spread_ns = 0;
         if (cfg.flags & PAGODA_SPREAD) {   /* PAGODA_SPREAD_NS (environment) overrides the 6 us default */
             const char* e = getenv("PAGODA_SPREAD_NS");
