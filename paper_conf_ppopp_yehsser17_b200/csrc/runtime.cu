@@ -110,11 +110,13 @@ struct pagoda_ctx {
     std::mutex ce_mtx;
     std::condition_variable ce_cv;
     cudaStream_t ce_stream = nullptr;
+    cudaEvent_t ce_ev[4] = {};             /* kCeInFlight copies' completion */
     uint64_t ce_issued = 0;                 /* ring positions whose copy was issued (carries over sessions) */
-    CUdeviceptr d_consumed = 0, d_tail = 0, d_stop = 0;
+    CUdeviceptr d_tail = 0, d_stop = 0;
 };
 
 static inline uint64_t now_ns();
+static constexpr int kCeInFlight = 3;
 
 /* cuStreamWriteValue64 / 32 through the runtime's driver entry points (no -lcuda) */
 typedef CUresult (*WriteValue64Fn)(CUstream, CUdeviceptr, cuuint64_t, unsigned int);
@@ -140,25 +142,25 @@ static bool load_stream_memops()
 }
 
 /* The copy-engine ingest (PAGODA_CE_INGEST), one session: copies the published, not yet issued
- * span of the host ring into the device ring (one cudaMemcpyAsync per contiguous part), then two
- * stream memory operations ordered after it (CU_STREAM_WRITE_VALUE_DEFAULT: a memory barrier
- * first): DevCtl.tail = the span's end (the schedulers' publication: ticket t is published once
- * tail > t, read with an acquire) and HostCtl.consumed (the host may reuse those ring slots).  A
- * device ring cell is overwritten only once the ticket of the previous lap handed it back
- * (HostCtl.handed, posted by MTB 0's scanner warp).  Command 2: flush what is published, then
- * DevCtl.stop = 1 behind it; 3: stop = kStopAbort at once. */
+ * span of the host ring into the device ring (one cudaMemcpyAsync per contiguous part), then a
+ * stream memory operation ordered after it (cuStreamWriteValue64, CU_STREAM_WRITE_VALUE_DEFAULT:
+ * a memory barrier first) sets DevCtl.tail = the span's end: the schedulers' publication (ticket t
+ * is published once an acquire of tail sees > t).  An event behind it tells this thread when the
+ * copy has read the host ring: HostCtl.consumed (the spawners may reuse those slots).  A device
+ * ring cell is overwritten only once the ticket of the previous lap handed it back (HostCtl.handed,
+ * posted by MTB 0's scanner warp).  Command 2: flush what is published, then DevCtl.stop = 1
+ * behind it; 3: stop = kStopAbort at once. */
 static void ce_session(pagoda_ctx* c)
 {
     const uint64_t R = c->R;
     uint64_t issued = c->ce_issued;
-    /* at most kInFlight copies in the stream: a small copy and its two memory operations take
-     * several microseconds on the GPU whatever their size, so the next copy waits for the
-     * oldest to land (HostCtl.consumed) and then takes everything published meanwhile */
-    constexpr int kInFlight = 2;
+    /* at most kCeInFlight copies in the stream: a small copy and its memory operation take a few
+     * microseconds on the GPU whatever their size, so a new copy waits for the oldest to land and
+     * then takes everything published meanwhile */
     constexpr uint64_t kChunk = 2048;   /* entries per copy: a backlog (a prespawned session) streams in
                                            128 KiB steps, the first tasks start after the first one */
-    uint64_t ends[kInFlight];
-    int nq = 0;
+    uint64_t ends[kCeInFlight];
+    int nq = 0, qh = 0;
     int idle = 0;
     for (;;) {
         const int cmd = c->ce_cmd.load(std::memory_order_acquire);
@@ -166,33 +168,29 @@ static void ce_session(pagoda_ctx* c)
             g_wv32((CUstream)c->ce_stream, c->d_stop, kStopAbort, 0);
             break;
         }
+        while (nq && cudaEventQuery(c->ce_ev[qh]) == cudaSuccess) {   /* landed: its host slots are free */
+            c->hctl->consumed = ends[qh];
+            qh = (qh + 1) % kCeInFlight;
+            nq--;
+        }
         const uint64_t pub = c->hctl->published;
         std::atomic_thread_fence(std::memory_order_acquire);   /* entries below pub were written first */
         const uint64_t limit = std::min<uint64_t>(std::min<uint64_t>(pub, c->hctl->handed + R), issued + kChunk);
-        if (nq) {
-            const uint64_t done = c->hctl->consumed;
-            int k = 0;
-            while (k < nq && done >= ends[k]) k++;
-            if (k) {
-                for (int i = k; i < nq; i++) ends[i - k] = ends[i];
-                nq -= k;
-            }
-        }
-        if (limit > issued && nq < kInFlight) {
+        if (limit > issued && nq < kCeInFlight) {
             const uint64_t e0 = issued & (R - 1);
             const uint64_t n = limit - issued, n1 = std::min<uint64_t>(n, R - e0);
             cudaMemcpyAsync(c->dring + e0, c->hring + e0, n1 * sizeof(TaskEntry), cudaMemcpyHostToDevice, c->ce_stream);
             if (n1 < n)
                 cudaMemcpyAsync(c->dring, c->hring, (n - n1) * sizeof(TaskEntry), cudaMemcpyHostToDevice, c->ce_stream);
             const CUresult r1 = g_wv64((CUstream)c->ce_stream, c->d_tail, limit, 0);
-            const CUresult r2 = g_wv64((CUstream)c->ce_stream, c->d_consumed, limit, 0);
-            if (r1 != CUDA_SUCCESS || r2 != CUDA_SUCCESS) {
-                fprintf(stderr, "pagoda: cuStreamWriteValue64 failed (%d, %d): copy-engine ingest stops\n", (int)r1,
-                        (int)r2);
+            const int slot = (qh + nq) % kCeInFlight;
+            if (r1 != CUDA_SUCCESS || cudaEventRecord(c->ce_ev[slot], c->ce_stream) != cudaSuccess) {
+                fprintf(stderr, "pagoda: copy-engine ingest: stream operation failed (%d): ingest stops\n", (int)r1);
                 c->faulted.store(1);
                 break;
             }
-            ends[nq++] = limit;
+            ends[slot] = limit;
+            nq++;
             issued = limit;
             idle = 0;
             continue;
@@ -205,6 +203,7 @@ static void ce_session(pagoda_ctx* c)
         else _mm_pause();
     }
     cudaStreamSynchronize(c->ce_stream);
+    c->hctl->consumed = issued;
     c->ce_issued = issued;
 }
 
@@ -569,6 +568,8 @@ static void free_ctx(pagoda_ctx* c)
         ce_command(c, 4);
         c->ce_thread.join();
     }
+    for (cudaEvent_t e : c->ce_ev)
+        if (e) cudaEventDestroy(e);
     if (c->ce_stream) cudaStreamDestroy(c->ce_stream);
     if (c->stream) cudaStreamDestroy(c->stream);
     delete c;
@@ -701,9 +702,8 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
             goto fail;
         }
         if (cudaStreamCreateWithFlags(&c->ce_stream, cudaStreamNonBlocking) != cudaSuccess) goto fail;
-        void* hc = nullptr;
-        cudaHostGetDevicePointer(&hc, (void*)c->hctl, 0);
-        c->d_consumed = (CUdeviceptr)((char*)hc + offsetof(HostCtl, consumed));
+        for (int i = 0; i < kCeInFlight; i++)
+            if (cudaEventCreateWithFlags(&c->ce_ev[i], cudaEventDisableTiming) != cudaSuccess) goto fail;
         c->d_tail = (CUdeviceptr)&c->dctl->tail;
         c->d_stop = (CUdeviceptr)&c->dctl->stop;
         c->ce_thread = std::thread(ce_thread_main, c);
