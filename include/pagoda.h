@@ -65,7 +65,10 @@ typedef struct {
     int      num_sms;       /* SMs to occupy, 0 = all (148 on B200) */
     uint32_t ring_entries;  /* TaskTable ring entries, host and device, power of 2 (default 65536) */
     uint32_t comp_entries;  /* completion window, power of 2 >= ring_entries (default 1<<20) */
-    uint32_t arena_bytes;   /* shared-memory arena per MTB, multiple of 512 (default 96 KiB at 2 MTB/SM) */
+    uint32_t arena_bytes;   /* shared-memory arena per MTB, multiple of 512 (default 96 KiB at 2 MTB/SM); the
+                               rest of the SM's 228 KiB is L1 (the executors' register spills live there).
+                               Without PAGODA_CE_INGEST, MTB 0's shared memory must hold 4 ingest stages
+                               of >= 32 entries (-EINVAL otherwise) */
     uint32_t exec_warps;    /* worker warps per MTB, 1..32, capped at the MTB's warps (32 at 1-2 MTBs/SM,
                                16 at 4 MTBs/SM; default 32 = all; fewer = debug config).  One thread
                                block may use at most this many warps (pagoda_info.exec_warps); a

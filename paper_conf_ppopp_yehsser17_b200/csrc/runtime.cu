@@ -625,6 +625,11 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
         delete c;   /* one MTB lends the top of its arena to its ingest warp's two stages */
         return -EINVAL;
     }
+    if (nsm * cfg.mtbs_per_sm > 1 && !(cfg.flags & PAGODA_CE_INGEST) &&
+        ingest_stage_entries((uint32_t)smem, nsm * cfg.mtbs_per_sm) < 32u) {
+        delete c;   /* the I/O MTB's shared memory holds no ingest stage of 32 entries: use PAGODA_CE_INGEST */
+        return -EINVAL;
+    }
     c->n_mtb = nsm * cfg.mtbs_per_sm;
     c->R = cfg.ring_entries;
     c->C = cfg.comp_entries;

@@ -13,6 +13,7 @@ def test_bench_uses_package_presets():
 
 def test_ctx_kwargs_match_bench_context():
     assert presets.RESIDENT_TDES == PG.RESIDENT_TDES and presets.SPREAD == PG.SPREAD
+    assert presets.CE_INGEST == PG.CE_INGEST
     for w in bench.WORKLOADS:
         class A:
             workload = w
