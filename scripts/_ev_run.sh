@@ -1,1 +1,1 @@
-OUT=final_r2b bash scripts/gpu_evidence.sh
+OUT=final_r2c bash scripts/gpu_evidence.sh
