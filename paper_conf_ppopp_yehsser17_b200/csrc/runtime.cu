@@ -179,14 +179,17 @@ static void ce_session(pagoda_ctx* c)
         if (limit > issued && nq < kCeInFlight) {
             const uint64_t e0 = issued & (R - 1);
             const uint64_t n = limit - issued, n1 = std::min<uint64_t>(n, R - e0);
-            cudaMemcpyAsync(c->dring + e0, c->hring + e0, n1 * sizeof(TaskEntry), cudaMemcpyHostToDevice, c->ce_stream);
-            if (n1 < n)
-                cudaMemcpyAsync(c->dring, c->hring, (n - n1) * sizeof(TaskEntry), cudaMemcpyHostToDevice, c->ce_stream);
-            const CUresult r1 = g_wv64((CUstream)c->ce_stream, c->d_tail, limit, 0);
+            cudaError_t ce = cudaMemcpyAsync(c->dring + e0, c->hring + e0, n1 * sizeof(TaskEntry), cudaMemcpyHostToDevice,
+                                             c->ce_stream);
+            if (ce == cudaSuccess && n1 < n)
+                ce = cudaMemcpyAsync(c->dring, c->hring, (n - n1) * sizeof(TaskEntry), cudaMemcpyHostToDevice, c->ce_stream);
+            const CUresult r1 = ce == cudaSuccess ? g_wv64((CUstream)c->ce_stream, c->d_tail, limit, 0) : CUDA_ERROR_UNKNOWN;
             const int slot = (qh + nq) % kCeInFlight;
             if (r1 != CUDA_SUCCESS || cudaEventRecord(c->ce_ev[slot], c->ce_stream) != cudaSuccess) {
-                fprintf(stderr, "pagoda: copy-engine ingest: stream operation failed (%d): ingest stops\n", (int)r1);
+                fprintf(stderr, "pagoda: copy-engine ingest: stream operation failed (%s, %d): ingest stops\n",
+                        cudaGetErrorString(ce), (int)r1);
                 c->faulted.store(1);
+                g_wv32((CUstream)c->ce_stream, c->d_stop, kStopAbort, 0);   /* let the MasterKernel leave */
                 break;
             }
             ends[slot] = limit;
