@@ -635,6 +635,22 @@ def measure(a, d, name, dev, peaks, PG, torch, *, steps, warmup, headline):
         assert p.stop() == 0
         L = (dn - sp) / 1e3
         lat["loaded_us"] = {"p50": float(np.percentile(L, 50)), "p99": float(np.percentile(L, 99))}
+        if name == "mix" and not claims_mode:
+            # SURVEY §8(d) C4 latency variant: open-loop Poisson arrivals at 50 % and 90 % of the
+            # measured capacity (this line's device rate); latency from each task's scheduled arrival
+            rng = np.random.default_rng(2017)
+            cap = value / d.world
+            for load in (0.5, 0.9):
+                gaps = rng.exponential(1e9 / (load * cap), size=w.n)
+                arr = np.cumsum(gaps).astype(np.int64)
+                assert p.start() == 0
+                sp2, dn2 = p.run_open_loop(w.shapes, w.args, arr)
+                assert p.stop() == 0
+                L2 = (dn2 - sp2) / 1e3
+                lat[f"open_loop_{int(load * 100)}pct_us"] = {
+                    "p50": float(np.percentile(L2, 50)), "p99": float(np.percentile(L2, 99)),
+                    "offered_tasks_per_s": load * cap, "achieved_tasks_per_s": w.n / ((dn2.max() - sp2[0]) * 1e-9),
+                    "arrivals": "Poisson (exponential gaps, seed 2017), latency from the scheduled arrival"}
     if headline and not a.quick:
         assert p.start() == 0
         iso = p.latency_loop(2000, 128, 1, 0, False, 0) / 1e3

@@ -217,6 +217,14 @@ int pagoda_session_ms(pagoda_ctx* ctx, float* ms);
  * check() first reports it done.  Returns n or the first error. */
 int64_t pagoda_run_timed(pagoda_ctx* ctx, int n, const int32_t* shapes, const void* args_base,
                          size_t args_stride, size_t args_bytes, int64_t* spawn_ns, int64_t* done_ns);
+/* Open loop (SURVEY §8(d) C4 latency variant): task i is spawned at t0 + arrival_ns[i] (t0 = the
+ * call; arrival_ns non-decreasing, e.g. Poisson arrivals at a fraction of the measured capacity),
+ * whether or not earlier tasks completed; arrive_ns[i] = t0 + arrival_ns[i] (the scheduled arrival,
+ * CLOCK_MONOTONIC) and done_ns[i] as in pagoda_run_timed, so done - arrive includes any wait of
+ * the spawning thread.  Returns n, -EINVAL (decreasing arrivals) or the first error. */
+int64_t pagoda_run_open_loop(pagoda_ctx* ctx, int n, const int32_t* shapes, const void* args_base,
+                             size_t args_stride, size_t args_bytes, const int64_t* arrival_ns, int64_t* arrive_ns,
+                             int64_t* done_ns);
 /* Closed loop, one task in flight: lat_ns[i] = spawn -> wait() return of task i. */
 int pagoda_latency_loop(pagoda_ctx* ctx, int n, int threads, int n_threadblocks, int shmem_bytes,
                         int sync_flag, int func_id, const void* args, size_t args_bytes, int64_t* lat_ns);

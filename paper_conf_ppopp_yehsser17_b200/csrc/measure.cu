@@ -26,8 +26,8 @@ static inline int64_t mono_ns()
     return (int64_t)ts.tv_sec * 1000000000ll + (int64_t)ts.tv_nsec;
 }
 
-extern "C" int64_t pagoda_run_timed(pagoda_ctx* c, int n, const int32_t* shapes, const void* args_base,
-                                    size_t args_stride, size_t args_bytes, int64_t* spawn_ns, int64_t* done_ns)
+static int64_t run_stamped(pagoda_ctx* c, int n, const int32_t* shapes, const void* args_base, size_t args_stride,
+                           size_t args_bytes, const int64_t* arrival_ns, int64_t* spawn_ns, int64_t* done_ns)
 {
     if (!c || n < 0 || !shapes || !spawn_ns || !done_ns) return -EINVAL;
     memset(done_ns, 0, sizeof(int64_t) * (size_t)n);
@@ -51,8 +51,11 @@ extern "C" int64_t pagoda_run_timed(pagoda_ctx* c, int n, const int32_t* shapes,
         }
     });
     const char* a = static_cast<const char*>(args_base);
+    const int64_t t0 = mono_ns();
     for (int i = 0; i < n; i++) {
         const int32_t* s = shapes + 5 * (size_t)i;
+        if (arrival_ns)   /* open loop: task i arrives at t0 + arrival_ns[i], whatever happened before */
+            while (mono_ns() - t0 < arrival_ns[i]) _mm_pause();
         spawn_ns[i] = mono_ns();
         const pagoda_task_t id =
             pagoda_taskSpawn(c, s[0], s[1], s[2], s[3], s[4], a ? a + (size_t)i * args_stride : nullptr, args_bytes);
@@ -65,7 +68,25 @@ extern "C" int64_t pagoda_run_timed(pagoda_ctx* c, int n, const int32_t* shapes,
     }
     poller.join();
     if (err.load()) return err.load();
+    if (arrival_ns)
+        for (int i = 0; i < n; i++) spawn_ns[i] = t0 + arrival_ns[i];   /* latency counts from the arrival */
     return n;
+}
+
+extern "C" int64_t pagoda_run_timed(pagoda_ctx* c, int n, const int32_t* shapes, const void* args_base,
+                                    size_t args_stride, size_t args_bytes, int64_t* spawn_ns, int64_t* done_ns)
+{
+    return run_stamped(c, n, shapes, args_base, args_stride, args_bytes, nullptr, spawn_ns, done_ns);
+}
+
+extern "C" int64_t pagoda_run_open_loop(pagoda_ctx* c, int n, const int32_t* shapes, const void* args_base,
+                                        size_t args_stride, size_t args_bytes, const int64_t* arrival_ns,
+                                        int64_t* arrive_ns, int64_t* done_ns)
+{
+    if (!arrival_ns) return -EINVAL;
+    for (int i = 1; i < n; i++)
+        if (arrival_ns[i] < arrival_ns[i - 1]) return -EINVAL;
+    return run_stamped(c, n, shapes, args_base, args_stride, args_bytes, arrival_ns, arrive_ns, done_ns);
 }
 
 extern "C" int pagoda_latency_loop(pagoda_ctx* c, int n, int threads, int n_tb, int shmem_bytes, int sync_flag,

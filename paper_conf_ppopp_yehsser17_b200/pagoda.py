@@ -113,6 +113,8 @@ def lib() -> C.CDLL:
         L.pagoda_session_ms.argtypes = [P, C.POINTER(C.c_float)]
         L.pagoda_run_timed.argtypes = [P, I, P, P, SZ, SZ, P, P]
         L.pagoda_run_timed.restype = I64
+        L.pagoda_run_open_loop.argtypes = [P, I, P, P, SZ, SZ, P, P, P]
+        L.pagoda_run_open_loop.restype = I64
         L.pagoda_latency_loop.argtypes = [P, I, I, I, I, I, I, P, SZ, P]
         L.pagoda_read_counters.argtypes = [P, P, I]
         _lib = L
@@ -244,6 +246,17 @@ class Pagoda:
         sp, dn = np.zeros(n, np.int64), np.zeros(n, np.int64)
         _check(lib().pagoda_run_timed(self.h, n, _ptr(shapes), _ptr(args), args.shape[1], args.shape[1],
                                       _ptr(sp), _ptr(dn)), "pagoda_run_timed")
+        return sp, dn
+
+    def run_open_loop(self, shapes: np.ndarray, args: np.ndarray, arrival_ns: np.ndarray):
+        """Spawn task i at call time + arrival_ns[i]; returns (arrive_ns, done_ns) (CLOCK_MONOTONIC)."""
+        shapes = np.ascontiguousarray(shapes, np.int32)
+        args = np.ascontiguousarray(args, np.uint8)
+        arr = np.ascontiguousarray(arrival_ns, np.int64)
+        n = len(shapes)
+        sp, dn = np.zeros(n, np.int64), np.zeros(n, np.int64)
+        _check(lib().pagoda_run_open_loop(self.h, n, _ptr(shapes), _ptr(args), args.shape[1], args.shape[1],
+                                          _ptr(arr), _ptr(sp), _ptr(dn)), "pagoda_run_open_loop")
         return sp, dn
 
     def latency_loop(self, n, threads, n_tb, shmem, sync, func_id, args=None) -> np.ndarray:
