@@ -110,13 +110,16 @@ struct pagoda_ctx {
     std::mutex ce_mtx;
     std::condition_variable ce_cv;
     cudaStream_t ce_stream = nullptr;
-    cudaEvent_t ce_ev[4] = {};             /* kCeInFlight copies' completion */
+    cudaEvent_t ce_ev[8] = {};             /* kCeInFlight (<= 8) copies' completion */
     uint64_t ce_issued = 0;                 /* ring positions whose copy was issued (carries over sessions) */
     CUdeviceptr d_tail = 0, d_stop = 0;
 };
 
 static inline uint64_t now_ns();
-static constexpr int kCeInFlight = 3;
+#ifndef PAGODA_CE_INFLIGHT
+#define PAGODA_CE_INFLIGHT 3
+#endif
+static constexpr int kCeInFlight = PAGODA_CE_INFLIGHT;
 
 /* cuStreamWriteValue64 / 32 through the runtime's driver entry points (no -lcuda) */
 typedef CUresult (*WriteValue64Fn)(CUstream, CUdeviceptr, cuuint64_t, unsigned int);

@@ -15,7 +15,7 @@ PRESETS = {
     # arena (2 tasks x 8 KiB): shared memory per SM drops from 227 to ~130 KiB and L1 serves the 32-register
     # spills (47 % -> most hits); 3 host producers.  48.3 -> 53-54 M tasks/s (62 M self-draining)
     "mm": {"mtbs_per_sm": 4, "arena_bytes": 24 * 1024, "resident": False, "ce": True, "producers": 3},
-    "mix": {"mtbs_per_sm": 1, "arena_bytes": 200 * 1024, "resident": False},
+    "mix": {"mtbs_per_sm": 1, "arena_bytes": 200 * 1024, "resident": False, "producers": 2},
     "nop": {"mtbs_per_sm": 2, "arena_bytes": 16 * 1024, "resident": False, "producers": 2, "ce": True},   # 68 -> 92 M
     "c5": {"mtbs_per_sm": 1, "arena_bytes": 144 * 1024, "resident": True},
     "mpe": {"mtbs_per_sm": 2, "arena_bytes": 40 * 1024, "resident": True},
