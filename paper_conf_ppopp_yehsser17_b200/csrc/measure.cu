@@ -52,10 +52,31 @@ static int64_t run_stamped(pagoda_ctx* c, int n, const int32_t* shapes, const vo
     });
     const char* a = static_cast<const char*>(args_base);
     const int64_t t0 = mono_ns();
-    for (int i = 0; i < n; i++) {
+    if (arrival_ns) {
+        /* open loop: task i arrives at t0 + arrival_ns[i], whatever happened before; every task whose
+         * arrival has passed is spawned in one batched call (one doorbell), so the spawning thread
+         * keeps up with arrival rates near the GPU's capacity */
+        for (int i = 0; i < n;) {
+            const int64_t now = mono_ns() - t0;
+            int j = i;
+            while (j < n && arrival_ns[j] <= now) j++;
+            if (j == i) {
+                _mm_pause();
+                continue;
+            }
+            const int64_t r = pagoda_taskSpawnShapes(c, j - i, shapes + 5 * (size_t)i,
+                                                     a ? a + (size_t)i * args_stride : nullptr, args_stride, args_bytes,
+                                                     ids.data() + i);
+            if (r != j - i) {
+                err.store(r < 0 ? (int)r : -EAGAIN);
+                break;
+            }
+            spawned.store(j, std::memory_order_release);
+            i = j;
+        }
+    }
+    for (int i = 0; i < n && !arrival_ns; i++) {
         const int32_t* s = shapes + 5 * (size_t)i;
-        if (arrival_ns)   /* open loop: task i arrives at t0 + arrival_ns[i], whatever happened before */
-            while (mono_ns() - t0 < arrival_ns[i]) _mm_pause();
         spawn_ns[i] = mono_ns();
         const pagoda_task_t id =
             pagoda_taskSpawn(c, s[0], s[1], s[2], s[3], s[4], a ? a + (size_t)i * args_stride : nullptr, args_bytes);

@@ -114,11 +114,23 @@ def test_mm_small(shmem, threads):
     _mm_check(w, run(w)["C"], range(300))
 
 
+def _pool_map(fn, ks):
+    """The oracle over many tasks on the host's cores (its ctypes calls release the GIL)."""
+    import concurrent.futures as cf
+    import os
+    with cf.ThreadPoolExecutor(max_workers=min(16, os.cpu_count() or 1)) as ex:
+        return list(ex.map(fn, ks, chunksize=256))
+
+
 def test_mm_config3_full_size():
+    """Every one of the 65,536 tasks against the oracle, in the bench's launch configuration."""
     w = W.matmul(65536)
     out = run(w, **ctx_kwargs("mm"))["C"]   # the bench's launch configuration
-    rng = np.random.default_rng(3)
-    _mm_check(w, out, list(rng.choice(65536, 256, replace=False)) + [0, 65535])
+    A, B = w.host["A"], w.host["B"]
+    ref = np.stack(_pool_map(lambda k: oracle.mm32(A[k], B[k]), range(65536)))
+    assert fp32_close(out, ref) <= TOL
+    bad = np.nonzero((out != ref).reshape(65536, -1).any(axis=1))[0]
+    assert len(bad) == 0, bad[:10]
 
 
 # ---------------------------------------------------------------- MM on the tensor cores (NEXT-4, 3xTF32)
@@ -276,9 +288,23 @@ def test_mix_small_all_shapes():
     _mix_check(w, run(w))
 
 
-def test_mix_config4_full_size_sampled():
+def test_mix_config4_full_size_every_task():
+    """Every one of the 32,768 FB / BF / CONV / DCT tasks against the oracle, in the bench's launch
+    configuration (the oracle on the host's cores)."""
     w = W.mix(32768)
-    _mix_check(w, run(w, **ctx_kwargs("mix")), frac=0.004, seed=4)
+    out = run(w, **ctx_kwargs("mix"))
+    fns = {"fb": (oracle.filterbank, w.host["fb"]), "bf": (oracle.beamformer, w.host["bf"]),
+           "conv": (oracle.conv, w.host["conv"]), "dct": (oracle.dct, None)}
+    for kind, (fn, ins) in fns.items():
+        if kind == "dct":
+            im, coef = w.host["dct"]
+            ref = np.stack(_pool_map(lambda k: oracle.dct(im[k], coef), range(len(im))))
+        else:
+            ref = np.stack(_pool_map(lambda k: fn(*(x[k] for x in ins)), range(len(ins[0]))))
+        got = out[kind].reshape(ref.shape)
+        assert fp32_close(got, ref) <= TOL, kind
+        bad = np.nonzero((got != ref).reshape(len(ref), -1).any(axis=1))[0]
+        assert len(bad) == 0, (kind, bad[:10])
 
 
 def test_mix_config4_registered_coefficients():
