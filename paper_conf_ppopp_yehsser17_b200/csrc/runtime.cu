@@ -165,6 +165,11 @@ static void ce_session(pagoda_ctx* c)
     uint64_t ends[kCeInFlight];
     int nq = 0, qh = 0;
     int idle = 0;
+    /* PAGODA_CE_STATS (environment): per session, copies issued, entries, ns in the issuing calls,
+     * ns with the stream full (kCeInFlight copies outstanding while entries wait), ns idle */
+    static const bool stats = getenv("PAGODA_CE_STATS") != nullptr;
+    uint64_t st_copies = 0, st_entries = 0, st_issue_ns = 0, st_full_ns = 0, st_idle_ns = 0, t_prev = now_ns();
+    const uint64_t t_begin = t_prev;
     for (;;) {
         const int cmd = c->ce_cmd.load(std::memory_order_acquire);
         if (cmd == 3 || cmd == 4) {
@@ -179,7 +184,14 @@ static void ce_session(pagoda_ctx* c)
         const uint64_t pub = c->hctl->published;
         std::atomic_thread_fence(std::memory_order_acquire);   /* entries below pub were written first */
         const uint64_t limit = std::min<uint64_t>(std::min<uint64_t>(pub, c->hctl->handed + R), issued + kChunk);
+        if (stats) {   /* account the time since the last look to the state seen then */
+            const uint64_t t = now_ns();
+            if (limit > issued && nq >= kCeInFlight) st_full_ns += t - t_prev;
+            else if (limit <= issued) st_idle_ns += t - t_prev;
+            t_prev = t;
+        }
         if (limit > issued && nq < kCeInFlight) {
+            const uint64_t t_issue = stats ? now_ns() : 0;
             const uint64_t e0 = issued & (R - 1);
             const uint64_t n = limit - issued, n1 = std::min<uint64_t>(n, R - e0);
             cudaError_t ce = cudaMemcpyAsync(c->dring + e0, c->hring + e0, n1 * sizeof(TaskEntry), cudaMemcpyHostToDevice,
@@ -197,6 +209,12 @@ static void ce_session(pagoda_ctx* c)
             }
             ends[slot] = limit;
             nq++;
+            if (stats) {
+                st_copies++;
+                st_entries += limit - issued;
+                t_prev = now_ns();
+                st_issue_ns += t_prev - t_issue;
+            }
             issued = limit;
             idle = 0;
             continue;
@@ -211,6 +229,12 @@ static void ce_session(pagoda_ctx* c)
     cudaStreamSynchronize(c->ce_stream);
     c->hctl->consumed = issued;
     c->ce_issued = issued;
+    if (stats)
+        fprintf(stderr, "pagoda CE: %llu copies, %.1f entries/copy, issue %.2f us/copy, full %.1f us, idle %.1f us, "
+                        "session %.1f us\n",
+                (unsigned long long)st_copies, st_copies ? (double)st_entries / st_copies : 0.0,
+                st_copies ? st_issue_ns * 1e-3 / st_copies : 0.0, st_full_ns * 1e-3, st_idle_ns * 1e-3,
+                (now_ns() - t_begin) * 1e-3);
 }
 
 /* The context's ingest thread: serves sessions (ce_cmd 1/2/3) and idles in between (spinning
