@@ -94,6 +94,7 @@ struct pagoda_ctx {
     std::mutex mt_mtx;                      /* one multi-producer spawn at a time */
     std::atomic<uint64_t> job_gen{0};
     std::atomic<int> job_left{0};
+    std::atomic<int> job_unvalidated{0};    /* producers still validating their blocks */
     std::atomic<int64_t> job_rc{0};
     std::atomic<int> helpers_quit{0};
     /* MasterKernel session */
@@ -419,7 +420,30 @@ static inline void write_entry(pagoda_ctx* c, uint64_t id0, int j, const int32_t
 
 template <class ShapeOf>
 static int64_t spawn_batch(pagoda_ctx* c, int n, ShapeOf shape_of, const void* args_base, size_t args_stride,
-                           size_t args_bytes, pagoda_task_t* ids_out);
+                           size_t args_bytes, pagoda_task_t* ids_out, bool validated = false);
+
+/* Validate n contiguous shape rows (5 x int32 each) before any is spawned (all-or-nothing).  Runs of
+ * rows equal to their predecessor are skipped 256 rows per memcmp (rows k and k-1 equal for every k
+ * of a chunk iff the chunk equals itself shifted by one row), so a uniform workload costs one SIMD
+ * scan of the array instead of five compares per row (65,536 rows: ~150 us on the host, inside the
+ * session that waits for the first spawn).  Returns 0 or the first error. */
+static int validate_rows(const pagoda_ctx* c, const int32_t* shapes, int n)
+{
+    ShapeMemo memo;
+    for (int i = 0; i < n;) {
+        Split sp;
+        if (int rc = memo.check(c, shapes + 5 * (size_t)i, sp)) return rc;
+        int j = i + 1;
+        while (j < n) {
+            const int m = std::min(256, n - j);
+            if (memcmp(shapes + 5 * (size_t)j, shapes + 5 * (size_t)(j - 1), 20 * (size_t)m) != 0) break;
+            j += m;
+        }
+        while (j < n && memcmp(shapes + 5 * (size_t)j, shapes + 5 * (size_t)i, 20) == 0) j++;   /* the rest of the run */
+        i = j;
+    }
+    return 0;
+}
 
 /* Ring slot `last` (and every one before it) is free: the ingest warp has copied entry last - R. */
 static bool ring_room(pagoda_ctx* c, uint64_t last)
@@ -870,14 +894,14 @@ pagoda_task_t pagoda_taskSpawn(pagoda_ctx* c, int threads, int n_tb, int shmem_b
 
 template <class ShapeOf>
 static int64_t spawn_batch(pagoda_ctx* c, int n, ShapeOf shape_of, const void* args_base, size_t args_stride,
-                           size_t args_bytes, pagoda_task_t* ids_out)
+                           size_t args_bytes, pagoda_task_t* ids_out, bool validated)
 {
     if (!c || n < 0) return -EINVAL;
     if (c->shutting.load(std::memory_order_acquire)) return -ESHUTDOWN;
     if (dev_fault(c)) return -EIO;
     if (args_bytes > PAGODA_ARGS_MAX || (args_bytes > 0 && !args_base)) return -EINVAL;
     ShapeMemo memo;
-    for (int i = 0; i < n; i++) {
+    for (int i = 0; i < n && !validated; i++) {   /* every task valid before any is spawned */
         Split sp;
         if (int rc = memo.check(c, shape_of(i), sp)) return rc;
     }
@@ -940,6 +964,28 @@ static int64_t spawn_batch(pagoda_ctx* c, int n, ShapeOf shape_of, const void* a
  * contiguous TaskTable exactly as with one producer. */
 static const int kMtBlock = 4 * kSpawnChunk;
 
+/* Producer t validates its own blocks; every producer waits until all have (all-or-nothing: a
+ * rejected workload spawns nothing), then spawns them if none failed.  The validation pass runs
+ * on all producers at once: over a large workload it is a scan of the shapes array (~1.3 MB for
+ * 65,536 tasks) that would otherwise delay the first spawn of the session. */
+static int64_t validate_part(const pagoda_ctx* c, const pagoda_ctx::SpawnJob& j, int t)
+{
+    for (int b0 = t * kMtBlock; b0 < j.n; b0 += j.P * kMtBlock)
+        if (int rc = validate_rows(c, j.shapes + 5 * (size_t)b0, std::min(kMtBlock, j.n - b0))) return rc;
+    return 0;
+}
+static bool validated_all(pagoda_ctx* c, const pagoda_ctx::SpawnJob& j, int t)
+{
+    const int64_t rc = validate_part(c, j, t);
+    if (rc < 0) {
+        int64_t z = 0;
+        c->job_rc.compare_exchange_strong(z, rc);
+    }
+    c->job_unvalidated.fetch_sub(1, std::memory_order_acq_rel);
+    while (c->job_unvalidated.load(std::memory_order_acquire) > 0) _mm_pause();
+    return c->job_rc.load(std::memory_order_acquire) == 0;
+}
+
 static int64_t spawn_part(pagoda_ctx* c, const pagoda_ctx::SpawnJob& j, int t)
 {
     for (int b0 = t * kMtBlock; b0 < j.n; b0 += j.P * kMtBlock) {
@@ -947,7 +993,7 @@ static int64_t spawn_part(pagoda_ctx* c, const pagoda_ctx::SpawnJob& j, int t)
         const int32_t* sh = j.shapes + 5 * (size_t)b0;
         const int64_t rc = spawn_batch(c, m, [&](int i) { return sh + 5 * (size_t)i; },
                                        j.bytes ? j.args + (size_t)b0 * j.stride : nullptr, j.stride, j.bytes,
-                                       j.ids ? j.ids + b0 : nullptr);
+                                       j.ids ? j.ids + b0 : nullptr, true);
         if (rc < 0) return rc;
         if (rc < m) return -EAGAIN;   /* ring full (non-blocking spawn / stopped): the block is cut short */
     }
@@ -965,7 +1011,7 @@ static void helper_main(pagoda_ctx* c, int t)
             idle = 0;
             const pagoda_ctx::SpawnJob j = c->job;
             if (t < j.P) {
-                const int64_t rc = spawn_part(c, j, t);
+                const int64_t rc = validated_all(c, j, t) ? spawn_part(c, j, t) : 0;
                 if (rc < 0) {
                     int64_t z = 0;
                     c->job_rc.compare_exchange_strong(z, rc);
@@ -989,24 +1035,22 @@ int64_t pagoda_taskSpawnShapesMT(pagoda_ctx* c, int n, const int32_t* shapes, co
     if (!c || n < 0 || (!shapes && n > 0) || n_producers < 1 || n_producers > PAGODA_MAX_PRODUCERS) return -EINVAL;
     if (args_bytes > PAGODA_ARGS_MAX || (args_bytes > 0 && !args_base)) return -EINVAL;
     const int P = std::min(n_producers, std::max(1, (n + kMtBlock - 1) / kMtBlock));
-    if (P == 1)
+    if (P == 1) {
+        if (int rc = validate_rows(c, shapes, n)) return rc;
         return spawn_batch(c, n, [&](int i) { return shapes + 5 * (size_t)i; }, args_base, args_stride, args_bytes,
-                           ids_out);
-    std::lock_guard<std::mutex> lk(c->mt_mtx);
-    ShapeMemo memo;   /* validate everything first: a rejected workload spawns nothing */
-    for (int i = 0; i < n; i++) {
-        Split sp;
-        if (int rc = memo.check(c, shapes + 5 * (size_t)i, sp)) return rc;
+                           ids_out, true);
     }
+    std::lock_guard<std::mutex> lk(c->mt_mtx);
     while ((int)c->helpers.size() < P - 1) {
         const int t = (int)c->helpers.size() + 1;
         c->helpers.emplace_back(helper_main, c, t);
     }
     c->job = pagoda_ctx::SpawnJob{shapes, static_cast<const char*>(args_base), args_stride, args_bytes, ids_out, n, P};
     c->job_rc.store(0);
+    c->job_unvalidated.store(P, std::memory_order_release);
     c->job_left.store(P - 1, std::memory_order_release);
     c->job_gen.fetch_add(1, std::memory_order_acq_rel);
-    const int64_t rc0 = spawn_part(c, c->job, 0);
+    const int64_t rc0 = validated_all(c, c->job, 0) ? spawn_part(c, c->job, 0) : 0;
     while (c->job_left.load(std::memory_order_acquire) > 0) _mm_pause();
     const int64_t rc = rc0 < 0 ? rc0 : c->job_rc.load();
     return rc < 0 ? rc : n;
@@ -1023,8 +1067,10 @@ int64_t pagoda_taskSpawnShapes(pagoda_ctx* c, int n, const int32_t* shapes, cons
                                size_t args_bytes, pagoda_task_t* ids_out)
 {
     if (!shapes && n > 0) return -EINVAL;
+    if (!c || n < 0) return -EINVAL;
+    if (int rc = validate_rows(c, shapes, n)) return rc;
     return spawn_batch(c, n, [&](int i) { return shapes + 5 * (size_t)i; }, args_base, args_stride, args_bytes,
-                       ids_out);
+                       ids_out, true);
 }
 
 int pagoda_check(pagoda_ctx* c, pagoda_task_t id)
