@@ -121,6 +121,9 @@ static inline uint64_t now_ns();
 #define PAGODA_CE_INFLIGHT 3
 #endif
 static constexpr int kCeInFlight = PAGODA_CE_INFLIGHT;
+#ifndef PAGODA_FWD_4MTB
+#define PAGODA_FWD_4MTB 1   /* completion forwarders at 4 MTBs/SM (MTB 0 has 16 warps) */
+#endif
 
 /* cuStreamWriteValue64 / 32 through the runtime's driver entry points (no -lcuda) */
 typedef CUresult (*WriteValue64Fn)(CUstream, CUdeviceptr, cuuint64_t, unsigned int);
@@ -818,7 +821,7 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
         p.life = c->life;
         /* completion forwarders: 4 when MTB 0 has 32 warps; 1 at 4 MTBs/SM (512 threads), where more
          * cost MM ~7 % (45 -> 42 M tasks/s) while NOP's forwarding is not the limit there */
-        p.n_fwd = cfg.mtbs_per_sm == 4 ? 1u : (uint32_t)kForwarders;
+        p.n_fwd = cfg.mtbs_per_sm == 4 ? (uint32_t)PAGODA_FWD_4MTB : (uint32_t)kForwarders;
         p.spread_ns = 0;
         if (cfg.flags & PAGODA_SPREAD) {   /* PAGODA_SPREAD_NS (environment) overrides the 6 us default */
             const char* e = getenv("PAGODA_SPREAD_NS");
