@@ -819,9 +819,11 @@ int pagoda_init(const pagoda_config* cfg_in, pagoda_ctx** out)
             p.exec_count = c->exec_count;
         }
         p.life = c->life;
-        /* completion forwarders: 4 when MTB 0 has 32 warps; 1 at 4 MTBs/SM (512 threads), where more
-         * cost MM ~7 % (45 -> 42 M tasks/s) while NOP's forwarding is not the limit there */
-        p.n_fwd = cfg.mtbs_per_sm == 4 ? (uint32_t)PAGODA_FWD_4MTB : (uint32_t)kForwarders;
+        /* completion forwarders: 4 when MTB 0 has 32 warps; at 4 MTBs/SM (16 warps) 2 with the copy-engine
+         * ingest (MTB 0's ingest warps idle: MM 54.5 -> 57.5 M) and 1 with the doorbell ingest (more cost its
+         * publishers: MM 45 -> 42 M) */
+        p.n_fwd = cfg.mtbs_per_sm == 4 ? ((cfg.flags & PAGODA_CE_INGEST) ? 2u : (uint32_t)PAGODA_FWD_4MTB)
+                                       : (uint32_t)kForwarders;
         p.spread_ns = 0;
         if (cfg.flags & PAGODA_SPREAD) {   /* PAGODA_SPREAD_NS (environment) overrides the 6 us default */
             const char* e = getenv("PAGODA_SPREAD_NS");
