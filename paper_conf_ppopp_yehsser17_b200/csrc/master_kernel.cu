@@ -75,6 +75,9 @@
 #ifndef PAGODA_DIRECT_IDLE_NS
 #define PAGODA_DIRECT_IDLE_NS 50000   /* ... or when the group posted nothing for this long (lone tasks) */
 #endif
+#ifndef PAGODA_LOAD_AHEAD
+#define PAGODA_LOAD_AHEAD 1   /* a holder that placed itself loads its claimed tickets before handing off */
+#endif
 #ifndef PAGODA_FREE_BEFORE_POST
 #define PAGODA_FREE_BEFORE_POST 1  /* a task's last warp frees itself before posting the completion record */
 #endif
@@ -1880,7 +1883,12 @@ __device__ __noinline__ bool holder_phase(MtbShared& S, const MkParams& p, int m
             }
             continue;
         }
-        sched_handoff(S, st, p, mtb);   /* dispatched (by itself or before it took the token) */
+        /* dispatched (by itself or before it took the token).  Load-ahead: the tickets this round
+         * claimed are loaded now, before the token moves on, so the next holder (a warp freed by the
+         * next finishing task, typically) finds a loaded task and places it at once instead of paying
+         * two L2 round trips with the slot's warps idle */
+        if (PAGODA_LOAD_AHEAD && st.pl != st.pt) sched_load(S, st, p);
+        sched_handoff(S, st, p, mtb);
         return false;
     }
 }
