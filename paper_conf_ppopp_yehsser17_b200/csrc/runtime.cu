@@ -439,10 +439,14 @@ static int validate_rows(const pagoda_ctx* c, const int32_t* shapes, int n)
 {
     struct Ent {
         int32_t s[5];
-        bool used;
+        uint32_t gen;   /* valid for the call whose generation this is (no clearing per call) */
     };
     static thread_local Ent cache[4096];
-    for (Ent& e : cache) e.used = false;
+    static thread_local uint32_t gen = 0;
+    if (++gen == 0) {   /* wrapped: start over */
+        for (Ent& e : cache) e.gen = 0;
+        gen = 1;
+    }
     int run = 0;
     for (int i = 0; i < n;) {
         const int32_t* r = shapes + 5 * (size_t)i;
@@ -457,11 +461,11 @@ static int validate_rows(const pagoda_ctx* c, const int32_t* shapes, int n)
         const uint32_t h = ((uint32_t)r[0] * 2654435761u ^ (uint32_t)r[1] * 40503u ^ (uint32_t)r[2] * 2246822519u ^
                             (uint32_t)r[3] * 3266489917u ^ (uint32_t)r[4] * 668265263u) >> 20;
         Ent& e = cache[h];
-        if (!e.used || !same_row(e.s, r)) {
+        if (e.gen != gen || !same_row(e.s, r)) {
             Split sp;
             if (int rc = shape_check(c, r, sp)) return rc;
             memcpy(e.s, r, 20);
-            e.used = true;
+            e.gen = gen;
         }
         i++;
     }
