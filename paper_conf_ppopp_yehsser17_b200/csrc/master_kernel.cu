@@ -1799,11 +1799,17 @@ __device__ bool sched_round(MtbShared& S, Sched<kG>& st, const MkParams& p, int 
         stop = __shfl_sync(0xffffffffu, stop, 0);
         if (stop == kStopAbort) exit = true;   /* host watchdog gave up */
         else if (stop) {
-            uint64_t tail = 0;
-            if (lane == 0) tail = ld_acquire_gpu(&p.dctl->tail);
+            uint64_t tail = 0, head = 0;
+            if (lane == 0) {
+                tail = ld_acquire_gpu(&p.dctl->tail);
+                head = ld_relaxed_gpu(&p.dctl->head);
+            }
             tail = __shfl_sync(0xffffffffu, tail, 0);
-            /* after stop the tail is final: tickets at or past it are void */
-            exit = st.pl == st.pt || S.pend_ticket[fq(st, st.pl)] >= tail;
+            head = __shfl_sync(0xffffffffu, head, 0);
+            /* after stop the tail is final: tickets at or past it are void.  A round without progress
+             * does not prove the ring drained: a claim cap (max_tasks) holds claims back while a
+             * finished task's slot awaits its fold, so leave only once every ticket is handed out */
+            exit = (st.pl == st.pt || S.pend_ticket[fq(st, st.pl)] >= tail) && (S.no_tickets || head >= tail);
         }
     }
     return progress;

@@ -11,7 +11,7 @@ import pytest
 
 from gpu_util import Dev, ptr
 from paper_conf_ppopp_yehsser17_b200 import tasks as T
-from paper_conf_ppopp_yehsser17_b200.pagoda import Pagoda, TRACE
+from paper_conf_ppopp_yehsser17_b200.pagoda import NO_START, Pagoda, TRACE
 
 pytestmark = pytest.mark.gpu
 
@@ -627,3 +627,16 @@ def test_shmem_grant_above_255_granules():
             assert p.taskSpawn(256, 1, nbytes, True, T.SMEM, a) >= 0
         assert p.waitAll() == 0 and p.info().device_error == 0
     assert Dev.get(err, np.uint32)[0] == 0
+
+
+@pytest.mark.parametrize("max_tasks", [1, 2])
+def test_claim_cap_sessions_drain_every_task(max_tasks):
+    """A claim cap holds claims back while a finished task's slot awaits its fold (the last warp frees
+    itself before posting); a scheduler must still not leave the session while tickets remain
+    unclaimed.  Back-to-back sessions of short tasks under caps of 1 and 2 all drain."""
+    with Pagoda(max_tasks=max_tasks, flags=NO_START) as p:
+        for s in range(6):
+            assert p.start() == 0
+            p.spawn_many(4000, 128, 1, 0, False, T.NOP, None)
+            assert p.stop() == 0, s
+        assert p.info().completed_low == 24000
