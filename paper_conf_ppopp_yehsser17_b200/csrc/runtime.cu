@@ -89,7 +89,6 @@ struct pagoda_ctx {
         size_t stride, bytes;
         pagoda_task_t* ids;
         int n, P;
-        bool validate_only;   /* helpers validate their blocks, the caller spawns everything */
     } job{};
     std::vector<std::thread> helpers;
     std::mutex mt_mtx;                      /* one multi-producer spawn at a time */
@@ -993,12 +992,6 @@ static int64_t spawn_batch(pagoda_ctx* c, int n, ShapeOf shape_of, const void* a
  * id order (a chunk is published once every lower id is), so the GPU sees one
  * contiguous TaskTable exactly as with one producer. */
 static const int kMtBlock = 4 * kSpawnChunk;
-#ifndef PAGODA_PAR_VALIDATE_MIN
-#define PAGODA_PAR_VALIDATE_MIN 16384
-#endif
-static const int kParValidateMin = PAGODA_PAR_VALIDATE_MIN;   /* single-producer spawns this large validate on
-                                                                 kParValidators threads */
-static const int kParValidators = 4;
 
 /* Producer t validates its own blocks; every producer waits until all have (all-or-nothing: a
  * rejected workload spawns nothing), then spawns them if none failed.  The validation pass runs
@@ -1047,7 +1040,7 @@ static void helper_main(pagoda_ctx* c, int t)
             idle = 0;
             const pagoda_ctx::SpawnJob j = c->job;
             if (t < j.P) {
-                const int64_t rc = validated_all(c, j, t) && !j.validate_only ? spawn_part(c, j, t) : 0;
+                const int64_t rc = validated_all(c, j, t) ? spawn_part(c, j, t) : 0;
                 if (rc < 0) {
                     int64_t z = 0;
                     c->job_rc.compare_exchange_strong(z, rc);
@@ -1081,8 +1074,7 @@ int64_t pagoda_taskSpawnShapesMT(pagoda_ctx* c, int n, const int32_t* shapes, co
         const int t = (int)c->helpers.size() + 1;
         c->helpers.emplace_back(helper_main, c, t);
     }
-    c->job = pagoda_ctx::SpawnJob{shapes, static_cast<const char*>(args_base), args_stride, args_bytes, ids_out, n, P,
-                                  false};
+    c->job = pagoda_ctx::SpawnJob{shapes, static_cast<const char*>(args_base), args_stride, args_bytes, ids_out, n, P};
     c->job_rc.store(0);
     c->job_unvalidated.store(P, std::memory_order_release);
     c->job_left.store(P - 1, std::memory_order_release);
@@ -1105,27 +1097,7 @@ int64_t pagoda_taskSpawnShapes(pagoda_ctx* c, int n, const int32_t* shapes, cons
 {
     if (!shapes && n > 0) return -EINVAL;
     if (!c || n < 0) return -EINVAL;
-    if (n >= kParValidateMin) {
-        /* one producer, a large workload: the context's helper threads validate the shape rows with the
-         * caller (blocks round-robin) while the session waits for its first task, then the caller
-         * spawns them all */
-        std::lock_guard<std::mutex> lk(c->mt_mtx);
-        const int V = kParValidators;
-        while ((int)c->helpers.size() < V - 1) {
-            const int t = (int)c->helpers.size() + 1;
-            c->helpers.emplace_back(helper_main, c, t);
-        }
-        c->job = pagoda_ctx::SpawnJob{shapes, nullptr, 0, 0, nullptr, n, V, true};
-        c->job_rc.store(0);
-        c->job_unvalidated.store(V, std::memory_order_release);
-        c->job_left.store(V - 1, std::memory_order_release);
-        c->job_gen.fetch_add(1, std::memory_order_acq_rel);
-        const bool ok = validated_all(c, c->job, 0);
-        while (c->job_left.load(std::memory_order_acquire) > 0) _mm_pause();
-        if (!ok) return c->job_rc.load();
-    } else if (int rc = validate_rows(c, shapes, n)) {
-        return rc;
-    }
+    if (int rc = validate_rows(c, shapes, n)) return rc;
     return spawn_batch(c, n, [&](int i) { return shapes + 5 * (size_t)i; }, args_base, args_stride, args_bytes,
                        ids_out, true);
 }
