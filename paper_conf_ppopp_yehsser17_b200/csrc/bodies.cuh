@@ -486,7 +486,8 @@ __device__ __forceinline__ void tdes_blocks_pair(const Env& e, const pagoda_tdes
 }
 
 #ifndef PAGODA_TDES_NOINLINE
-#define PAGODA_TDES_NOINLINE 0   /* the 3DES body as a call (A/B: register spills around the body) */
+#define PAGODA_TDES_NOINLINE 1   /* the 3DES body as a call: the executor keeps its own register allocation
+                                    (35.5 -> 36.0 M tasks/s) */
 #endif
 #if PAGODA_TDES_NOINLINE
 #define PAGODA_TDES_ATTR __noinline__
