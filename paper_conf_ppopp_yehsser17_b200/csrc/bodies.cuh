@@ -23,6 +23,23 @@
 
 namespace pagoda {
 
+/* Benchmark bodies as calls (PAGODA_BODIES_NOINLINE): a body inlined into the executor loop shares
+ * its register allocation, and at 32 registers per thread (2 or 4 MTBs per SM) every inlined body
+ * adds spills around all of them (3DES as a call: 3DES +1.6 %, MM +6 %, MPE +8 %). */
+#ifndef PAGODA_BODIES_NOINLINE
+#define PAGODA_BODIES_NOINLINE 0
+#endif
+#if PAGODA_BODIES_NOINLINE
+#define PAGODA_BODY_ATTR __noinline__
+#else
+#define PAGODA_BODY_ATTR
+#endif
+#if PAGODA_BODIES_NOINLINE
+#define PAGODA_CONV_BODY_ATTR __noinline__
+#else
+#define PAGODA_CONV_BODY_ATTR __forceinline__
+#endif
+
 template <class Env>
 __device__ __forceinline__ int total_threads(const Env& e)
 {
@@ -157,7 +174,7 @@ template <> struct IsTaskEnv<TaskEnv> { static constexpr bool value = true; };
  * Table 3; strict '>' escape test, count includes
  * the escaping step, multiply-then-add never fused. */
 template <class Env>
-__device__ void body_mb(const Env& e, const pagoda_mb_args& a)
+__device__ PAGODA_BODY_ATTR void body_mb(const Env& e, const pagoda_mb_args& a)
 {
     const int T = total_threads(e);
     const int maxit = a.maxit;
@@ -683,7 +700,7 @@ __device__ __forceinline__ void mma_tf32(float (&c)[4], const uint32_t (&a)[4], 
 }
 
 template <class Env>
-__device__ void body_mm_tc(const Env& e, const pagoda_mm_args& a)
+__device__ PAGODA_BODY_ATTR void body_mm_tc(const Env& e, const pagoda_mm_args& a)
 {
     const float* A = a.A;
     const float* B = a.B;
@@ -730,7 +747,7 @@ __device__ void body_mm_tc(const Env& e, const pagoda_mm_args& a)
  * Only VH[8m] is ever used, and the zero terms of VU add exactly +0, so
  * y[j] = sum over k = j mod 8, j mod 8 + 8, ... <= min(31, j) of F[k] VD[(j-k)/8]. */
 template <class Env>
-__device__ void body_fb(const Env& e, const pagoda_fb_args& a)
+__device__ PAGODA_BODY_ATTR void body_fb(const Env& e, const pagoda_fb_args& a)
 {
     float* vd = (e.getSMBytes() >= 1024) ? reinterpret_cast<float*>(e.getSMPtr())
                                          : a.scratch + 256 * e.getBlockIdx();
@@ -776,7 +793,7 @@ __device__ __forceinline__ void cmac(float& re, float& im, float ar, float ai, f
 }
 
 template <class Env>
-__device__ void body_bf(const Env& e, const pagoda_bf_args& a)
+__device__ PAGODA_BODY_ATTR void body_bf(const Env& e, const pagoda_bf_args& a)
 {
     const int T = total_threads(e);
     const float2* x = reinterpret_cast<const float2*>(a.x);
@@ -889,7 +906,7 @@ __device__ __forceinline__ void conv_cols(const Env& e, const pagoda_conv_args& 
  * (bands of >= 32 rows: 11.5 -> 10.3 M tasks/s; >= 64 rows: 12.7 -> 12.4 M): CONV is bound by
  * its load latency, not by the scratch round trip through L2. */
 template <class Env>
-__device__ __forceinline__ void body_conv(const Env& e, const pagoda_conv_args& a)
+__device__ PAGODA_CONV_BODY_ATTR void body_conv(const Env& e, const pagoda_conv_args& a)
 {
     const int nb = e.getNumBlocks(), j = e.getBlockIdx();
     const int r0 = (128 * j) / nb, r1 = (128 * (j + 1)) / nb;
