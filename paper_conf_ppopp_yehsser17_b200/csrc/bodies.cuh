@@ -1024,9 +1024,30 @@ __device__ void body_dct(const Env& e, const pagoda_dct_args& a)
 }
 
 /* ------------------------------------------------------------- dispatch */
-template <class Env>
+/* A body behind a call (its code out of the caller's register allocation). */
+template <class Env, class A, void (*F)(const Env&, const A&)>
+__device__ __noinline__ void as_call(const Env& e, const A& a)
+{
+    F(e, a);
+}
+/* kCallCold: the MB / FB / BF / CONV bodies behind calls.  The 4-MTB/SM MasterKernel (32 registers,
+ * the MM presets) takes it: its executor loop then spills less around the bodies it does run
+ * (measured: MM 58.9 -> 62.4 M tasks/s); the other configurations run those bodies and keep them
+ * inline (config 5 15.4 vs 17.2 M tasks/s, mix 12.2 vs 12.7 M as calls). */
+template <bool kCallCold = false, class Env>
 __device__ __forceinline__ bool run_body(int func_id, const Env& e, const void* args)
 {
+    if constexpr (kCallCold) {
+        switch (func_id) {
+        case PAGODA_MB: as_call<Env, pagoda_mb_args, body_mb<Env>>(e, *static_cast<const pagoda_mb_args*>(args)); return true;
+        case PAGODA_FB: as_call<Env, pagoda_fb_args, body_fb<Env>>(e, *static_cast<const pagoda_fb_args*>(args)); return true;
+        case PAGODA_BF: as_call<Env, pagoda_bf_args, body_bf<Env>>(e, *static_cast<const pagoda_bf_args*>(args)); return true;
+        case PAGODA_CONV:
+            as_call<Env, pagoda_conv_args, body_conv<Env>>(e, *static_cast<const pagoda_conv_args*>(args));
+            return true;
+        default: break;
+        }
+    }
     switch (func_id) {
     case PAGODA_NOP: return true;
     case PAGODA_MARK: body_mark(e, *static_cast<const pagoda_mark_args*>(args)); return true;

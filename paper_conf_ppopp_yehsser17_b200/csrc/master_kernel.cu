@@ -550,6 +550,7 @@ __device__ void comp_forwarder(MtbShared& S, const MkParams& p, uint32_t f)
  * warp of a TB returns its shmem granules and barrier ID through the mailbox
  * (markSMForDealloc), the last warp of the task posts its completion record,
  * every warp returns itself. */
+template <bool kCallCold>
 __device__ __forceinline__ void run_task(MtbShared& S, SchedGroup& G, char* smem_base, const MkParams& p, int mtb,
                                          int vmtb, int w, uint32_t resident)
 {
@@ -563,7 +564,7 @@ __device__ __forceinline__ void run_task(MtbShared& S, SchedGroup& G, char* smem
         atomicCAS(reinterpret_cast<unsigned long long*>(life_slot(p, s.task_id, kLifeStart)), 0ull,
                   (unsigned long long)globaltimer_ns());
     uint64_t tp = pf_now();
-    if (!run_body(t.func_id, env, t.args) && lane == 0) atomicOr(&p.dctl->error, PAGODA_DEVERR_BAD_FUNC);
+    if (!run_body<kCallCold>(t.func_id, env, t.args) && lane == 0) atomicOr(&p.dctl->error, PAGODA_DEVERR_BAD_FUNC);
     __syncwarp();
     pf_add(G, kPfBody, tp, true);
     if (p.life && lane == 0)
@@ -1902,7 +1903,7 @@ __device__ __noinline__ bool holder_phase(MtbShared& S, const MkParams& p, int m
 
 /* Every worker warp runs this loop (warps 0..exec_warps-1; MTB 0's last warp ingests); exec_mask is
  * the worker warps of its scheduling group g. */
-template <int kG>
+template <int kG, bool kCallCold>
 __device__ void worker(MtbShared& S, char* smem_base, const MkParams& p, int mtb, int w, uint32_t resident,
                        uint32_t exec_mask, bool holder, uint32_t g)
 {
@@ -1922,7 +1923,7 @@ __device__ void worker(MtbShared& S, char* smem_base, const MkParams& p, int mtb
             holder = true;
             continue;
         }
-        run_task(S, G, smem_base, p, mtb, vmtb, w, resident);
+        run_task<kCallCold>(S, G, smem_base, p, mtb, vmtb, w, resident);
         holder = token_try(G);
     }
 }
@@ -2065,7 +2066,8 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) master_kernel(MkParams p
     }
     else if (io && warp == host_poster_warp(nw)) host_poster(S, p);
     else if (io && forwarder_index(warp, nw) < p.n_fwd) comp_forwarder(S, p, forwarder_index(warp, nw));
-    else if ((my_exec >> warp) & 1u) worker<kG>(S, smem_base, p, mtb, warp, resident, my_exec, warp == first, my_g);
+    else if ((my_exec >> warp) & 1u)   /* 4 MTBs/SM (the MM presets): the bodies they do not run behind calls */
+        worker<kG, kMinBlocks == 4>(S, smem_base, p, mtb, warp, resident, my_exec, warp == first, my_g);
 }
 
 template __global__ void master_kernel<1, 1024, 1>(MkParams);
