@@ -180,9 +180,18 @@ class Clocks:
             if len(parts) == 6:
                 self.rows.append(parts)
 
+    def wait_first(self, timeout=3.0):
+        """nvidia-smi takes a few hundred ms to its first sample: wait for it before the timed region,
+        so a short timed region (0.9 ms steps) is bracketed by samples every 100 ms."""
+        t0 = time.time()
+        while self.proc and not self.rows and time.time() - t0 < timeout:
+            time.sleep(0.01)
+
     def stop(self):
         if self.proc:
-            time.sleep(0.25)
+            n0, t0 = len(self.rows), time.time()
+            while len(self.rows) == n0 and time.time() - t0 < 1.0:   # one sample after the timed region
+                time.sleep(0.01)
             self.proc.terminate()
             try:
                 self.proc.wait(timeout=5)
@@ -591,6 +600,7 @@ def measure(a, d, name, dev, peaks, PG, torch, *, steps, warmup, headline):
     info = p.info()
     clocks = Clocks(dev)
     clocks.start()
+    clocks.wait_first()
     d.barrier()
     torch.cuda.synchronize()
     host_s, dev_ms, mine = [], [], 0
@@ -759,6 +769,7 @@ def run_pool(a, peaks):
         step()
     clocks = Clocks(members[0])
     clocks.start()
+    clocks.wait_first()
     dev_ms, host_s, per_mem = [], [], np.zeros(n_mem, np.int64)
     spawn = np.zeros((n_mem, 3), np.int64)
     for _ in range(a.steps):

@@ -1,1 +1,1 @@
-OUT=final_r2h bash scripts/gpu_evidence.sh
+OUT=final_r2i bash scripts/gpu_evidence.sh

@@ -50,7 +50,8 @@ int main()
     pagoda_gate_args g{flag};
     const pagoda_task_t gated = pagoda::taskSpawn(32, 1, 0, 0, PAGODA_GATE, g);
     REQUIRE(gated == n);
-    REQUIRE(pagoda::wait(ids[n - 1]) == 0 && pagoda::check(ids[0]) == 1);
+    // tasks complete in any order: wait for the last, then the first, and check it
+    REQUIRE(pagoda::wait(ids[n - 1]) == 0 && pagoda::wait(ids[0]) == 0 && pagoda::check(ids[0]) == 1);
     REQUIRE(pagoda::check(gated) == 0);   // still gated
     *flag = 1;
     REQUIRE(pagoda::wait(gated) == 0 && pagoda::check(gated) == 1);
